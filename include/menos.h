@@ -1,0 +1,170 @@
+/*
+ * menos.h -- C-ABI of the Menos server segment on B200 (sm_100a).
+ *
+ * Menos (Hu & Li, MIDDLEWARE '24) splits a Llama-2 model between clients and a server.  The server runs
+ * the middle segment f_s (decoder layers [cut, L)) for many clients at once over ONE shared frozen base
+ * copy (spatial sharing, §3.1), each client with its own LoRA adapters phi_s
+ * (§2.1; §5.1).  This header is the boundary the paper's problem statement
+ * implies:
+ *
+ *   server cycle (§2.2, Alg.1):
+ *     menos_forward   : x_s = f_s(x_c; theta_s, phi_s)                  (Step 2 / Alg.1 L6, L10)
+ *     menos_backward  : g_s = dL/dx_c from g_c = dL/dx_s, plus dphi_s   (Step 4 / Alg.1 L11)
+ *     menos_adapter_step : AdamW on phi_s only                          (Alg.1 L12; Eq.1)
+ *   client join / profiling (§3.3): menos_register_client, menos_client_memory.
+ *   OOM avoidance (§4.1): MENOS_ENOMEM is RETURNED, never a crash.
+ *
+ * Conventions (all functions):
+ *   - Return an int status (menos_status); 0 = OK.  Argument / shape / state errors return synchronously
+ *     and launch nothing.  Asynchronous device errors are sticky and surface from the next call or from
+ *     menos_sync().  menos_last_error() gives a thread-local message for the last failure.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - Activation buffers (x_c, x_s, g_c, g_s) are bf16, token-major row-major [T, d_model], client-major
+ *     then sequence-major packing.  They may be HOST or DEVICE pointers (detected with
+ *     cudaPointerGetAttributes): host buffers are staged through pinned memory inside the call, and the call
+ *     synchronises `stream` before returning when it wrote to a host buffer.
+ *   - No torch types, no C++ types.  The library never frees caller memory; the caller never frees
+ *     library memory except through the destroy / free calls below.
+ *   - Every kernel runs on the GPU (sm_100a); there is no CPU fallback.  If no sm_100 device is present,
+ *     menos_server_create returns MENOS_ECUDA.
+ */
+#ifndef MENOS_H_
+#define MENOS_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifndef MENOS_API
+#define MENOS_API __attribute__((visibility("default")))
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  MENOS_OK = 0,
+  MENOS_EINVAL = -1,    /* bad argument, shape or layout                                        */
+  MENOS_ENOMEM = -2,    /* arena / registry / device memory cannot hold the request */
+  MENOS_ENOCLIENT = -3, /* unknown client id                                                     */
+  MENOS_ESTATE = -4,    /* e.g. backward on a batch without a live forward, weights not loaded    */
+  MENOS_ECUDA = -5,     /* CUDA error (sticky until menos_sync)                                   */
+  MENOS_ENCCL = -6      /* reserved: tensor-parallel communicator error                           */
+} menos_status;
+
+typedef struct menos_server menos_server;
+typedef struct menos_batch menos_batch;
+
+/* Llama-2 decoder-layer dimensions (PAPER.md:292 names Llama 2 [32]; dims are Llama-2's). */
+typedef struct {
+  int d_model;     /* d                                  */
+  int n_heads;     /* H                                  */
+  int n_kv_heads;  /* H_kv (GQA when < H)                 */
+  int d_ff;        /* f (SwiGLU inner size)               */
+  float rms_eps;   /* RMSNorm epsilon (1e-5)              */
+  float rope_theta;/* RoPE base (1e4)                     */
+} menos_model_cfg;
+
+/* One decoder layer's frozen base weights, natural (HF) layouts, bf16 row-major, host or device.
+ * The library COPIES them into its single device copy (WeightStore); the caller may free them after the
+ * call returns.  hd = d_model / n_heads. */
+typedef struct {
+  const void* wq;    /* [H*hd, d]     */
+  const void* wk;    /* [H_kv*hd, d]  */
+  const void* wv;    /* [H_kv*hd, d]  */
+  const void* wo;    /* [d, H*hd]     */
+  const void* wgate; /* [f, d]        */
+  const void* wup;   /* [f, d]        */
+  const void* wdown; /* [d, f]        */
+  const void* g1;    /* [d] input RMSNorm gain          */
+  const void* g2;    /* [d] post-attention RMSNorm gain */
+} menos_layer_weights;
+
+/* LoRA target projections (bit mask).  PAPER.md:294 uses q,v. */
+enum {
+  MENOS_T_Q = 1, MENOS_T_K = 2, MENOS_T_V = 4, MENOS_T_O = 8,
+  MENOS_T_GATE = 16, MENOS_T_UP = 32, MENOS_T_DOWN = 64
+};
+/* target index (0..6) used by get/set_adapter: q, k, v, o, gate, up, down */
+
+typedef struct {
+  float lr, beta1, beta2, eps, weight_decay; /* torch.optim.AdamW semantics */
+} menos_adamw_cfg;
+
+typedef struct {
+  int max_clients;     /* registry capacity (default 64)                                     */
+  int max_rank;        /* largest LoRA rank accepted (default 64)                             */
+  int max_seq_len;     /* longest sequence (RoPE table rows; default 4096)                   */
+  size_t arena_bytes;  /* activation arena I (Eq.3); 0 = free memory - 8 GiB    */
+  int num_sms;         /* persistent-grid width; 0 = device SM count                          */
+} menos_server_opts;
+
+/* forward flags */
+enum {
+  MENOS_FWD_SAVE = 0,   /* keep the intermediates I for the backward                                   */
+  MENOS_FWD_NOGRAD = 1  /* Menos on-demand mode (Alg.1 L6): keep only x_c; backward
+                           re-forwards with SAVE, then runs backward (Alg.1 L10-11)                     */
+};
+
+/* Create a server for decoder layers [first_layer, first_layer + n_layers) on CUDA device `device`.
+ * `w` = n_layers entries (or NULL: load each layer with menos_server_load_layer before forward).
+ * opts may be NULL (defaults).  Errors: EINVAL (dims), ECUDA (no sm_100 device), ENOMEM. */
+MENOS_API int menos_server_create(const menos_model_cfg* cfg, int first_layer, int n_layers, const menos_layer_weights* w,
+                        int device, const menos_server_opts* opts, menos_server** out);
+MENOS_API int menos_server_load_layer(menos_server* s, int layer /* 0..n_layers-1 */, const menos_layer_weights* w);
+MENOS_API void menos_server_destroy(menos_server* s);
+
+/* Client join: allocates A, B (fp32 master + bf16 copy in the shared slot tables), dA,
+ * dB, AdamW m, v.  Init: A ~ U(-1/sqrt(K), 1/sqrt(K)) from init_seed, B = 0 (PEFT default).
+ * rank 1..max_rank; alpha > 0; target_mask != 0.  Returns ENOMEM when the registry is full. */
+MENOS_API int menos_register_client(menos_server* s, int rank, float alpha, uint32_t target_mask, const menos_adamw_cfg* opt,
+                          uint64_t init_seed, int32_t* client_id);
+MENOS_API int menos_unregister_client(menos_server* s, int32_t client_id);
+
+/* Closed-form memory demands (Alg.2 L2): persistent A+O bytes of the client, and the arena
+ * bytes of a SAVE forward (M_f) and of the backward (M_b) for n_tokens tokens of that client. */
+MENOS_API int menos_client_memory(menos_server* s, int32_t client_id, int n_tokens, size_t* persistent, size_t* fwd_bytes,
+                        size_t* bwd_bytes);
+
+/* Step 2: x_s = f_s(x_c).  n_seqs sequences; seq_client[i] (host) is the client of sequence i and
+ * seq_len[i] (host) its length (>= 1, <= max_seq_len).  Sequences of one client must be contiguous
+ * (client-major packing).  T = sum(seq_len).  x_c, x_s: [T, d] bf16 (host or device).
+ * On success *batch is a handle that owns the saved activations (or the x_c copy under NOGRAD) until
+ * menos_backward or menos_batch_free.  ENOMEM if the arena cannot hold them (form smaller waves). */
+MENOS_API int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_client, const int32_t* seq_len, const void* x_c,
+                  void* x_s, int flags, void* stream, menos_batch** batch);
+
+/* Step 4: g_s = dL/dx_c from g_c = dL/dx_s ([T, d] bf16, host or device).  OVERWRITES every participating
+ * client's dA, dB (summed over its tokens).  Frees the batch's arena slab; the handle is consumed. */
+MENOS_API int menos_backward(menos_server* s, menos_batch* batch, const void* g_c, void* g_s, void* stream);
+MENOS_API int menos_batch_free(menos_server* s, menos_batch* batch);
+
+/* Alg.1 L12: one fused AdamW launch over the n clients' adapters (torch.optim.AdamW semantics, per-client
+ * step count); consumes and zeroes their dA, dB and refreshes the bf16 copies used by the kernels. */
+MENOS_API int menos_adapter_step(menos_server* s, int n, const int32_t* client_ids, void* stream);
+
+/* Host copies of one adapter tensor (fp32).  which: 0 = A [r, K], 1 = B [N, r], 2 = dA, 3 = dB,
+ * 4 = m_A, 5 = m_B, 6 = v_A, 7 = v_B.  layer in 0..n_layers-1, target 0..6 (must be in the client's mask).
+ * set_adapter accepts which 0..1 (A, B) and refreshes the bf16 copy.  Both synchronise the device. */
+MENOS_API int menos_adapter_shape(menos_server* s, int32_t id, int target, int* rows, int* cols);
+MENOS_API int menos_get_adapter(menos_server* s, int32_t id, int layer, int target, int which, float* host_out);
+MENOS_API int menos_set_adapter(menos_server* s, int32_t id, int layer, int target, int which, const float* host_in);
+
+/* Statistics: bytes of the shared base copy (M), of all clients' A+O, arena capacity and in-use bytes. */
+typedef struct {
+  size_t base_bytes, adapters_bytes, arena_bytes, arena_used, arena_peak;
+  int n_clients;
+  int num_sms;
+} menos_stats;
+MENOS_API int menos_get_stats(menos_server* s, menos_stats* out);
+
+/* Number of kernels this library has launched since load (evidence for bench.py's gpu_launches). */
+MENOS_API unsigned long long menos_launch_count(void);
+
+MENOS_API int menos_sync(menos_server* s);
+MENOS_API const char* menos_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MENOS_H_ */

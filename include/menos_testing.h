@@ -1,0 +1,44 @@
+/*
+ * menos_testing.h -- kernel-level entry points of libmenos.so used ONLY by the GPU unit tests
+ * (tests/test_gpu_kernels.py).  They run exactly the kernels the server path launches, on caller-owned
+ * DEVICE buffers, and synchronise the device before returning.  Not part of the user-facing boundary
+ * (include/menos.h); same error conventions (0 = OK, menos_last_error() for the message).
+ */
+#ifndef MENOS_TESTING_H_
+#define MENOS_TESTING_H_
+#include <stdint.h>
+#ifndef MENOS_API
+#define MENOS_API __attribute__((visibility("default")))
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* tcgen05 GEMM:
+ *   out[M, N] = epi( A[M, K] . B^T  +  A2[M, window] . B2[window]^T )
+ *   b_mn = 0: B is [N, K] row-major (ldb); b_mn = 1: B is [K, N] row-major (dX form).  B2 follows B's form
+ *   with R columns / rows.  mtile_extra (host, 2 ints per 128-row tile: col_start, n16) selects each tile's
+ *   extra-K window; R = 0 disables it.  epi: 0 store, 1 +resid, 2 RoPE (head_dim, rope_cols, pos, theta),
+ *   3 SwiGLU fwd (out = gu, out2 = a), 4 SwiGLU bwd (aux = saved gu, out = dgu).  All bf16, device. */
+MENOS_API int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int lda, const void* B, int ldb, const void* A2,
+                    int lda2, const void* B2, int ldb2, int R, const int32_t* mtile_extra, int epi, void* out, int ldo,
+                    const void* resid, int ldr, void* out2, int ldo2, const void* aux, int ldaux, int head_dim,
+                    int rope_cols, const int32_t* pos, float theta, int num_sms);
+
+/* Varlen causal flash attention forward + backward (A3, A11) on a packed qkv [T, (H+2Hkv)hd] (q,k post-RoPE):
+ * O [T, H*hd], lse [H, T] fp32; if dO != NULL also dqkv [T, (H+2Hkv)hd] = gradients w.r.t. the PRE-RoPE
+ * q, k and v (RoPE backward with theta applied).  seq_len: host [n_seqs]. */
+MENOS_API int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, int Hkv, int hd, const void* qkv, void* O,
+                         float* lse, const void* dO, void* dqkv, float theta);
+
+/* RMSNorm forward (y, rstd) and backward (dx = resid + norm_bwd(dy)); g fp32 [d].  Device buffers. */
+MENOS_API int menos_test_rmsnorm(int T, int d, const void* x, const float* g, float eps, void* y, float* rstd, const void* dy,
+                       const void* resid, void* dx);
+
+MENOS_API const char* menos_testing_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

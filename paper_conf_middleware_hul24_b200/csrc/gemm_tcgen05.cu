@@ -1,0 +1,398 @@
+// tcgen05 / TMEM / TMA GEMM for the shared frozen base projections.
+//
+//   out[M, N] = A[M, K] . B^T  (+ A2[M, R] . B2^T over a per-M-tile window of R: segmented LoRA expand)
+//
+// * A is the token-major activation (K-major).  B is the ONE shared bf16 weight copy (§3.1
+//   base-model sharing): K-major [N, K] for the forward projections, MN-major [K, N] for the dX GEMMs of the
+//   backward -- the same buffer serves both, no transposed duplicate.
+// * The LoRA expand rides on the same accumulator as extra K steps: A2 = block-diagonal
+//   s*U (row t holds only its client's slot columns), B2 = all clients' B (or A for dX) stacked by slot, so
+//   zero columns contribute exactly 0 and no M tile ever mixes clients' adapters.
+// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread), warps 2-5 = epilogue
+//   (TMEM -> registers -> fused epilogue -> global).  Two TMEM accumulators (2 x 256 fp32 columns) let the
+//   epilogue of tile i overlap the MMAs of tile i+1.  Persistent grid = #SMs.
+#include <mutex>
+#include <unordered_map>
+#include <cstring>
+#include "common.cuh"
+#include "kernels.h"
+
+namespace menos {
+
+namespace {
+constexpr int BM = 128, BN = 256, BK = 64;
+constexpr int STAGES = 4;
+constexpr int A_STAGE = BM * BK * 2;   // 16 KB
+constexpr int B_STAGE = BN * BK * 2;   // 32 KB
+constexpr int STAGE_BYTES = A_STAGE + B_STAGE;
+constexpr int NTHREADS = 192;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024;
+
+struct KParams {
+  int M, N, K;
+  int kb_main;
+  int R;
+  const int2* mtile_extra;
+  const uint8_t* ntile_extra;
+  int epi;
+  bf16* out; int ldo;
+  const bf16* resid; int ldr;
+  bf16* out2; int ldo2;
+  const bf16* aux; int ldaux;
+  const float2* rope_cs;
+  const int* pos;
+  int head_dim, rope_cols;
+};
+
+__device__ __forceinline__ void store32(bf16* dst, const float (&v)[32]) {
+  uint4* d = reinterpret_cast<uint4*>(dst);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 u;
+    u.x = pack_bf16x2(v[8 * q + 0], v[8 * q + 1]);
+    u.y = pack_bf16x2(v[8 * q + 2], v[8 * q + 3]);
+    u.z = pack_bf16x2(v[8 * q + 4], v[8 * q + 5]);
+    u.w = pack_bf16x2(v[8 * q + 6], v[8 * q + 7]);
+    d[q] = u;
+  }
+}
+__device__ __forceinline__ void load32(const bf16* src, float (&v)[32]) {
+  const uint4* s = reinterpret_cast<const uint4*>(src);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 u = s[q];
+    float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
+    v[8 * q + 0] = a.x; v[8 * q + 1] = a.y; v[8 * q + 2] = b.x; v[8 * q + 3] = b.y;
+    v[8 * q + 4] = c.x; v[8 * q + 5] = c.y; v[8 * q + 6] = d.x; v[8 * q + 7] = d.y;
+  }
+}
+// RoPE inside one 32-column chunk for head_dim = 2*HALF <= 32 (pairs (j, j+HALF) of each head)
+template <int HALF>
+__device__ __forceinline__ void rope_small(const float (&v)[32], float (&o)[32], const float2* cs) {
+#pragma unroll
+  for (int j = 0; j < 32; ++j) {
+    constexpr int HD = 2 * HALF;
+    const int jj = j % HD;
+    const float2 e = cs[jj % HALF];
+    o[j] = jj < HALF ? v[j] * e.x - v[j + HALF] * e.y : v[j] * e.x + v[j - HALF] * e.y;
+  }
+}
+__device__ __forceinline__ float sigmoidf_(float x) { return 1.0f / (1.0f + __expf(-x)); }
+
+template <int B_MN>
+__global__ void __launch_bounds__(NTHREADS, 1)
+gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+               const __grid_constant__ CUtensorMap tmA2, const __grid_constant__ CUtensorMap tmB2,
+               const KParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], tfull_bar[2], tempty_bar[2];
+  __shared__ uint32_t tmem_base_sh;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int num_m = (p.M + BM - 1) / BM, num_n = (p.N + BN - 1) / BN;
+  const int total = num_m * num_n;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch(&tmA); tma_prefetch(&tmB);
+    if (p.R > 0) { tma_prefetch(&tmA2); tma_prefetch(&tmB2); }
+    for (int s = 0; s < STAGES; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
+    for (int s = 0; s < 2; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4); }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = tmem_base_sh;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ------------------------------------------------ TMA producer
+      int stage = 0; uint32_t phase = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        const int m = t % num_m, n = t / num_m;
+        int n16 = 0, col0 = 0;
+        if (p.R > 0 && (p.ntile_extra == nullptr || p.ntile_extra[n])) { int2 e = p.mtile_extra[m]; col0 = e.x; n16 = e.y; }
+        const int nkb = p.kb_main + (n16 + 3) / 4;
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&empty_bar[stage], phase ^ 1);
+          uint8_t* sa = smem + stage * STAGE_BYTES;
+          uint8_t* sb = sa + A_STAGE;
+          mbar_expect_tx(&full_bar[stage], STAGE_BYTES);
+          const bool main = kb < p.kb_main;
+          const CUtensorMap* ma = main ? &tmA : &tmA2;
+          const CUtensorMap* mb = main ? &tmB : &tmB2;
+          const int kc = main ? kb * BK : col0 + (kb - p.kb_main) * BK;
+          tma_load_2d(sa, ma, &full_bar[stage], kc, m * BM);
+          if (!B_MN) {
+            tma_load_2d(sb, mb, &full_bar[stage], kc, n * BN);
+          } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) tma_load_2d(sb + j * 8192, mb, &full_bar[stage], n * BN + j * 64, kc);
+          }
+          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ------------------------------------------------ MMA issuer (single thread)
+      constexpr uint32_t IDESC = umma_idesc_bf16(BM, BN, B_MN);
+      int stage = 0; uint32_t phase = 0;
+      int acc = 0; uint32_t acc_phase = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        const int m = t % num_m, n = t / num_m;
+        int n16 = 0;
+        if (p.R > 0 && (p.ntile_extra == nullptr || p.ntile_extra[n])) n16 = p.mtile_extra[m].y;
+        const int nkb = p.kb_main + (n16 + 3) / 4;
+        mbar_wait(&tempty_bar[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&full_bar[stage], phase);
+          tc_fence_after();
+          const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
+          const uint32_t sb = sa + A_STAGE;
+          int nsteps = 4;
+          if (kb >= p.kb_main) { nsteps = n16 - (kb - p.kb_main) * 4; if (nsteps > 4) nsteps = 4; }
+          for (int k = 0; k < nsteps; ++k) {
+            const uint64_t ad = umma_desc_sw128(sa + k * 32, 16, 1024);
+            const uint64_t bd = B_MN ? umma_desc_sw128(sb + k * 2048, 8192, 1024)
+                                     : umma_desc_sw128(sb + k * 32, 16, 1024);
+            tc_mma_bf16(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+          }
+          tc_commit(&empty_bar[stage]);
+          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+        }
+        tc_commit(&tfull_bar[acc]);
+        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    // ------------------------------------------------ epilogue warps 2..5
+    const int q = warp & 3;  // TMEM lane quadrant this warp may access
+    int acc = 0; uint32_t acc_phase = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int m = t % num_m, n = t / num_m;
+      mbar_wait(&tfull_bar[acc], acc_phase);
+      tc_fence_after();
+      const int row = m * BM + q * 32 + lane;
+      const bool rok = row < p.M;
+      const uint32_t tb = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
+      const int n0 = n * BN;
+      if (p.epi == EPI_STORE || p.epi == EPI_RESID) {
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          if (rok) {
+            if (p.epi == EPI_RESID) {
+              float r[32];
+              load32(p.resid + (size_t)row * p.ldr + col, r);
+#pragma unroll
+              for (int j = 0; j < 32; ++j) v[j] += r[j];
+            }
+            store32(p.out + (size_t)row * p.ldo + col, v);
+          }
+        }
+      } else if (p.epi == EPI_ROPE) {
+        const int hd = p.head_dim, half = hd >> 1;
+        const int ps = rok ? p.pos[row] : 0;
+        const float2* cs = p.rope_cs + (size_t)ps * half;
+        if (half >= 32) {
+          for (int c = 0; c < 8; ++c) {
+            const int col = n0 + c * 32;
+            if (col >= p.N) break;
+            if ((col % hd) >= half) continue;           // handled as a partner chunk
+            const int pc = c + half / 32;                // partner chunk (same head)
+            float x1[32], x2[32];
+            tmem_ld32(tb + c * 32, x1);
+            tmem_ld32(tb + pc * 32, x2);
+            if (col < p.rope_cols) {
+              const int i0 = col % hd;
+#pragma unroll
+              for (int j = 0; j < 32; ++j) {
+                const float2 e = cs[i0 + j];
+                const float a = x1[j], b = x2[j];
+                x1[j] = a * e.x - b * e.y;
+                x2[j] = b * e.x + a * e.y;
+              }
+            }
+            if (rok) {
+              store32(p.out + (size_t)row * p.ldo + col, x1);
+              store32(p.out + (size_t)row * p.ldo + n0 + pc * 32, x2);
+            }
+          }
+        } else {
+          for (int c = 0; c < 8; ++c) {
+            const int col = n0 + c * 32;
+            if (col >= p.N) break;
+            float v[32], o[32];
+            tmem_ld32(tb + c * 32, v);
+            if (col < p.rope_cols) {
+              if (half == 8) rope_small<8>(v, o, cs);
+              else rope_small<16>(v, o, cs);
+            } else {
+#pragma unroll
+              for (int j = 0; j < 32; ++j) o[j] = v[j];
+            }
+            if (rok) store32(p.out + (size_t)row * p.ldo + col, o);
+          }
+        }
+      } else if (p.epi == EPI_SWIGLU_FWD) {
+        // tile = [128 gate | 128 up] of f block n; a[:, n*128 + j] = silu(g_j) * u_j
+        for (int c = 0; c < 4; ++c) {
+          float g[32], u[32];
+          tmem_ld32(tb + c * 32, g);
+          tmem_ld32(tb + (c + 4) * 32, u);
+          if (rok) {
+            store32(p.out + (size_t)row * p.ldo + n0 + c * 32, g);
+            store32(p.out + (size_t)row * p.ldo + n0 + 128 + c * 32, u);
+            float a[32];
+#pragma unroll
+            for (int j = 0; j < 32; ++j) a[j] = g[j] * sigmoidf_(g[j]) * u[j];
+            store32(p.out2 + (size_t)row * p.ldo2 + n * 128 + c * 32, a);
+          }
+        }
+      } else if (p.epi == EPI_SWIGLU_BWD) {
+        // acc = da over f columns; gu saved interleaved in 128-blocks: g at fb*256+jj, u at fb*256+128+jj
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float da[32];
+          tmem_ld32(tb + c * 32, da);
+          if (rok) {
+            const int fb = col >> 7, jj = col & 127;
+            const size_t gofs = (size_t)row * p.ldaux + fb * 256 + jj;
+            float g[32], u[32], dg[32], du[32];
+            load32(p.aux + gofs, g);
+            load32(p.aux + gofs + 128, u);
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              const float sg = sigmoidf_(g[j]);
+              dg[j] = da[j] * u[j] * sg * (1.0f + g[j] * (1.0f - sg));
+              du[j] = da[j] * g[j] * sg;
+            }
+            const size_t oofs = (size_t)row * p.ldo + fb * 256 + jj;
+            store32(p.out + oofs, dg);
+            store32(p.out + oofs + 128, du);
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+      if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<512>(tmem_base);
+  }
+}
+
+// ---------------------------------------------------------------- host: tensor maps
+typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                      const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                      CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+PFN_encodeTiled_t get_encode() {
+  static PFN_encodeTiled_t fn = nullptr;
+  if (!fn) {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return nullptr;
+    fn = reinterpret_cast<PFN_encodeTiled_t>(ptr);
+  }
+  return fn;
+}
+
+struct MapKey {
+  const void* ptr; uint64_t rows, cols, ld; uint32_t bc, br;
+  bool operator==(const MapKey& o) const {
+    return ptr == o.ptr && rows == o.rows && cols == o.cols && ld == o.ld && bc == o.bc && br == o.br;
+  }
+};
+struct MapKeyHash {
+  size_t operator()(const MapKey& k) const {
+    size_t h = std::hash<const void*>()(k.ptr);
+    h ^= std::hash<uint64_t>()(k.rows * 1000003ull + k.cols * 7919ull + k.ld) + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
+    h ^= std::hash<uint64_t>()(((uint64_t)k.bc << 32) | k.br) + (h << 6);
+    return h;
+  }
+};
+std::mutex g_map_mu;
+std::unordered_map<MapKey, CUtensorMap, MapKeyHash> g_maps;
+
+// row-major [rows, cols] bf16 with leading dimension ld (elements); box = {bc cols, br rows}; SWIZZLE_128B.
+bool get_map(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc, uint32_t br) {
+  MapKey k{ptr, rows, cols, ld, bc, br};
+  std::lock_guard<std::mutex> lk(g_map_mu);
+  auto it = g_maps.find(k);
+  if (it != g_maps.end()) { *out = it->second; return true; }
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return false;
+  CUtensorMap m;
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {ld * 2};
+  cuuint32_t box[2] = {bc, br};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  if (g_maps.size() > 65536) g_maps.clear();
+  g_maps.emplace(k, m);
+  *out = m;
+  return true;
+}
+}  // namespace
+
+int gemm_run(const GemmArgs& a, cudaStream_t st) {
+  if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
+  if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;
+  if ((a.epi == EPI_SWIGLU_FWD && a.N % 256) || (a.epi == EPI_SWIGLU_BWD && a.N % 128)) return -1;
+  CUtensorMap mA, mB, mA2, mB2;
+  if (!get_map(&mA, a.A, a.M, a.K, a.lda, BK, BM)) return -2;
+  if (!a.b_mn_major) {
+    if (!get_map(&mB, a.B, a.N, a.K, a.ldb, BK, BN)) return -2;
+  } else {
+    if (!get_map(&mB, a.B, a.K, a.N, a.ldb, 64, BK)) return -2;
+  }
+  if (a.R > 0) {
+    if (!get_map(&mA2, a.A2, a.M, a.R, a.lda2, BK, BM)) return -2;
+    if (!a.b_mn_major) {
+      if (!get_map(&mB2, a.B2, a.N, a.R, a.ldb2, BK, BN)) return -2;
+    } else {
+      if (!get_map(&mB2, a.B2, a.R, a.N, a.ldb2, 64, BK)) return -2;
+    }
+  } else {
+    mA2 = mA; mB2 = mB;
+  }
+  KParams p;
+  p.M = a.M; p.N = a.N; p.K = a.K; p.kb_main = (a.K + BK - 1) / BK;
+  p.R = a.R; p.mtile_extra = a.mtile_extra; p.ntile_extra = a.ntile_extra;
+  p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr;
+  p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux;
+  p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
+  const int tiles = ((a.M + BM - 1) / BM) * ((a.N + BN - 1) / BN);
+  int grid = a.num_sms > 0 ? a.num_sms : 148;
+  if (tiles < grid) grid = tiles;
+  static bool attr_set[2] = {false, false};
+  if (a.b_mn_major) {
+    if (!attr_set[1]) { cudaFuncSetAttribute(gemm_tc_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES); attr_set[1] = true; }
+    gemm_tc_kernel<1><<<grid, NTHREADS, SMEM_BYTES, st>>>(mA, mB, mA2, mB2, p);
+  } else {
+    if (!attr_set[0]) { cudaFuncSetAttribute(gemm_tc_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES); attr_set[0] = true; }
+    gemm_tc_kernel<0><<<grid, NTHREADS, SMEM_BYTES, st>>>(mA, mB, mA2, mB2, p);
+  }
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+}  // namespace menos

@@ -1,0 +1,116 @@
+// Internal launcher interface between the Menos host runtime (server.cu) and the sm_100a kernels.
+// Not part of the C-ABI; see include/menos.h for the public boundary.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+namespace menos {
+
+typedef __nv_bfloat16 bf16;
+
+// Counts every kernel this library launches (reported as gpu_launches by bench.py).
+extern unsigned long long g_launch_count;
+
+// ---------------------------------------------------------------- tcgen05 GEMM
+enum EpiMode : int {
+  EPI_STORE = 0,       // out = bf16(acc)
+  EPI_RESID = 1,       // out = bf16(acc + resid)
+  EPI_ROPE = 2,        // columns < rope_cols rotated by RoPE at pos[row]; out = bf16
+  EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu), out2 = bf16(silu(g) u)
+  EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
+};
+
+struct GemmArgs {
+  int M, N, K;               // out[M, N] = A[M, K] . B^T  (B K-major [N, K] or MN-major [K, N])
+  int b_mn_major;            // 0: B is [N, K] row-major (weights, fwd); 1: B is [K, N] row-major (dX)
+  const bf16* A; int lda;
+  const bf16* B; int ldb;
+  // optional extra-K segment (segmented LoRA expand, block-diagonal U): A2 [M, R] K-major, B2 like B
+  const bf16* A2; int lda2;
+  const bf16* B2; int ldb2;
+  int R;                      // columns of A2 / K-extent of B2 (0 = no extra segment)
+  const int2* mtile_extra;    // device [ceil(M/128)]: (col_start, n16 = # of 16-wide K steps)
+  const uint8_t* ntile_extra; // device [ceil(N/256)] or nullptr (= all tiles)
+  // epilogue
+  int epi;
+  bf16* out; int ldo;
+  const bf16* resid; int ldr;      // EPI_RESID
+  bf16* out2; int ldo2;            // EPI_SWIGLU_FWD: a
+  const bf16* aux; int ldaux;      // EPI_SWIGLU_BWD: saved gu
+  const float2* rope_cs;           // EPI_ROPE: [max_pos][hd/2] (cos, sin)
+  const int* pos;                  // EPI_ROPE: per-row position
+  int head_dim, rope_cols;
+  int num_sms;
+};
+
+// Tensor maps are cached by (ptr, rows, cols, ld, box) on the host.
+int gemm_run(const GemmArgs& a, cudaStream_t st);
+
+// ---------------------------------------------------------------- small mma.sync GEMM (LoRA shrink/grads)
+// C[m, n] = scale * sum_k A(m, k) B(n, k)
+//   A(m,k) = a_t ? A[k*lda + map(m)] : A[m*lda + k];  B(n,k) = b_t ? B[k*ldb + n] : B[n*ldb + k]
+// Writes fp32 (c_f32) and/or bf16 (c_bf16); every problem is independent (no atomics).
+struct SmallGemmProblem {
+  const bf16* A; const bf16* B;
+  float* Cf; bf16* Cb;
+  int M, N, K, lda, ldb, ldc;
+  int a_t, b_t;
+  float scale;
+  int a_blk, a_blk_stride;    // A row-index remap (a_t only): m -> (m / a_blk) * a_blk_stride + m % a_blk
+};
+int small_gemm_run(const SmallGemmProblem* d_probs, const int4* d_tiles, int n_tiles, cudaStream_t st);
+// host helper: tiles of a problem list (problem, m0, n0, 0)
+void small_gemm_tiles(const SmallGemmProblem* probs, int n, int4* out_tiles, int* n_tiles_out);
+const int SG_BM = 64, SG_BN = 64;
+
+// ---------------------------------------------------------------- norms / elementwise
+int rmsnorm_fwd(const bf16* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st);
+// dx = resid + rstd*(gh - xh*mean(gh*xh)), gh = dy*g, xh = x*rstd
+int rmsnorm_bwd(const bf16* dy, const bf16* x, const float* g, const float* rstd, const bf16* resid, bf16* dx,
+                int T, int d, cudaStream_t st);
+int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st);
+
+// ---------------------------------------------------------------- attention (varlen causal, GQA)
+struct AttnArgs {
+  const bf16* qkv; int ld_qkv;   // q at col 0, k at H*hd, v at (H+Hkv)*hd
+  bf16* O; int ld_o;
+  float* lse;                    // [H, T]
+  const int* cu_seqlens;         // [n_seq+1]
+  const int2* qblocks;           // (seq, local q start) per 64-row q block
+  int n_qblocks;
+  const int2* kvblocks;          // (seq, local kv start) per 64-row kv block
+  int n_kvblocks;
+  int T, H, Hkv, hd;
+  float scale;
+  // backward
+  const bf16* dO; int ld_do;
+  const float* D;                // [H, T]
+  bf16* dqkv; int ld_dqkv;       // dq/dk/dv written pre-RoPE (RoPE backward applied)
+  const float2* rope_cs;         // [max_pos][hd/2]
+};
+int attn_fwd(const AttnArgs& a, cudaStream_t st);
+int attn_bwd(const AttnArgs& a, cudaStream_t st);
+
+// ---------------------------------------------------------------- AdamW + bf16 refresh
+struct AdamSeg {              // one (client, layer, target, A|B) parameter block
+  long long p_off;            // offset into the client's flat fp32 buffers
+  int rows, cols;             // source [rows, cols] row-major
+  int client;                 // index into AdamHyper array
+  bf16* dst;                  // bf16 copy destination base
+  int dst_ld;
+  int is_b;                   // B [N, r]: row n -> dst row map; col i -> dst col i
+  int row_blk, row_blk_stride, row_base;  // dst_row = row_base + (n / row_blk)*row_blk_stride + n % row_blk
+};
+struct AdamHyper {
+  float* p; float* g; float* m; float* v;
+  float lr, beta1, beta2, eps, wd, bc1, bc2_sqrt;
+  int do_update;              // 0: only refresh the bf16 copy (set_adapter / register)
+};
+int adamw_run(const AdamSeg* d_segs, const int4* d_work, int n_work, const AdamHyper* d_hyp, cudaStream_t st);
+
+int fill_rope_table(float2* cs, int max_pos, int hd, float theta, cudaStream_t st);
+int convert_bf16_to_f32(const bf16* src, float* dst, long long n, cudaStream_t st);
+
+}  // namespace menos

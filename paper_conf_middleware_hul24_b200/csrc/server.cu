@@ -1,0 +1,1298 @@
+// Menos server runtime behind include/menos.h: WeightStore (one bf16 base copy), ClientRegistry (LoRA
+// adapters + AdamW state in shared slot tables), BatchPacker (segment tables), ActivationArena (temporal
+// sharing), and the per-layer forward / backward schedules over the sm_100a kernels.
+//
+// Paper anchors: spatial sharing of theta (§3.1), on-demand allocation of I and release
+// after backward (§3.2, Eq.3), the serving process Alg.1, the 4-step
+// cycle, client profiling of M_f / M_b (Alg.2 L2).
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../include/menos.h"
+#include "kernels.h"
+
+using namespace menos;
+
+// =====================================================================================================
+// errors
+// =====================================================================================================
+static thread_local std::string tl_err;
+static void set_err(const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  tl_err = buf;
+}
+#define FAIL(code, ...) do { set_err(__VA_ARGS__); return (code); } while (0)
+#define CUDA_TRY(x)                                                                         \
+  do {                                                                                      \
+    cudaError_t e_ = (x);                                                                   \
+    if (e_ != cudaSuccess) FAIL(MENOS_ECUDA, "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+#define K_TRY(x)                                                                              \
+  do {                                                                                        \
+    int r_ = (x);                                                                             \
+    if (r_ != 0) {                                                                            \
+      cudaError_t e_ = cudaGetLastError();                                                    \
+      FAIL(MENOS_ECUDA, "%s failed (%d): %s (%s:%d)", #x, r_, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                                         \
+  } while (0)
+
+static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+static inline int ceil_div(int a, int b) { return (a + b - 1) / b; }
+
+// =====================================================================================================
+// target / group geometry
+// =====================================================================================================
+enum { TQ = 0, TK, TV, TO, TG, TU, TD, NT };
+enum { GQKV = 0, GO, GGU, GD, NG };
+static const int kTargetGroup[NT] = {GQKV, GQKV, GQKV, GO, GGU, GGU, GD};
+
+struct Dims {
+  int d, H, Hkv, hd, f, fpad, Nq, Nkv, Nqkv;
+  float eps, theta;
+  int K_t[NT], N_t[NT];            // projection input/output dims (natural)
+  int K_g[NG], N_g[NG], ldK_g[NG]; // group GEMM input dim, output dim, Acat leading dim
+  // Bcat row map per target: row = base + (n / blk) * stride + n % blk
+  int rb_base[NT], rb_blk[NT], rb_stride[NT];
+};
+
+static Dims make_dims(const menos_model_cfg& c) {
+  Dims D;
+  D.d = c.d_model; D.H = c.n_heads; D.Hkv = c.n_kv_heads; D.hd = c.d_model / c.n_heads;
+  D.f = c.d_ff; D.fpad = (int)align_up(c.d_ff, 128);
+  D.Nq = D.H * D.hd; D.Nkv = D.Hkv * D.hd; D.Nqkv = D.Nq + 2 * D.Nkv;
+  D.eps = c.rms_eps; D.theta = c.rope_theta;
+  const int K[NT] = {D.d, D.d, D.d, D.Nq, D.d, D.d, D.f};
+  const int N[NT] = {D.Nq, D.Nkv, D.Nkv, D.d, D.f, D.f, D.d};
+  for (int t = 0; t < NT; ++t) { D.K_t[t] = K[t]; D.N_t[t] = N[t]; }
+  D.K_g[GQKV] = D.d;  D.N_g[GQKV] = D.Nqkv;    D.ldK_g[GQKV] = D.d;
+  D.K_g[GO] = D.Nq;   D.N_g[GO] = D.d;         D.ldK_g[GO] = D.Nq;
+  D.K_g[GGU] = D.d;   D.N_g[GGU] = 2 * D.fpad; D.ldK_g[GGU] = D.d;
+  D.K_g[GD] = D.f;    D.N_g[GD] = D.d;         D.ldK_g[GD] = D.fpad;
+  const int big = 1 << 30;
+  int base[NT] = {0, D.Nq, D.Nq + D.Nkv, 0, 0, 128, 0};
+  int blk[NT] = {big, big, big, big, 128, 128, big};
+  int str[NT] = {0, 0, 0, 0, 256, 256, 0};
+  for (int t = 0; t < NT; ++t) { D.rb_base[t] = base[t]; D.rb_blk[t] = blk[t]; D.rb_stride[t] = str[t]; }
+  return D;
+}
+
+// =====================================================================================================
+// arena (first-fit, no cudaMalloc on the hot path)
+// =====================================================================================================
+struct Arena {
+  uint8_t* base = nullptr;
+  size_t cap = 0, used = 0, peak = 0;
+  std::map<size_t, size_t> free_;  // offset -> size
+  std::map<size_t, size_t> live_;
+  void init(uint8_t* b, size_t c) { base = b; cap = c; free_.clear(); live_.clear(); free_[0] = c; used = peak = 0; }
+  void* alloc(size_t n) {
+    n = align_up(n ? n : 256, 256);
+    for (auto it = free_.begin(); it != free_.end(); ++it) {
+      if (it->second >= n) {
+        size_t off = it->first, sz = it->second;
+        free_.erase(it);
+        if (sz > n) free_[off + n] = sz - n;
+        live_[off] = n;
+        used += n; peak = std::max(peak, used);
+        return base + off;
+      }
+    }
+    return nullptr;
+  }
+  void release(void* p) {
+    if (!p) return;
+    size_t off = (uint8_t*)p - base;
+    auto it = live_.find(off);
+    if (it == live_.end()) return;
+    size_t n = it->second;
+    live_.erase(it);
+    used -= n;
+    auto nx = free_.lower_bound(off);
+    if (nx != free_.end() && off + n == nx->first) { n += nx->second; free_.erase(nx); }
+    auto pv = free_.lower_bound(off);
+    if (pv != free_.begin()) {
+      --pv;
+      if (pv->first + pv->second == off) { off = pv->first; n += pv->second; free_.erase(pv); }
+    }
+    free_[off] = n;
+  }
+};
+
+// =====================================================================================================
+// clients
+// =====================================================================================================
+struct Client {
+  bool used = false;
+  int rank = 0, rs = 0;
+  float alpha = 0, s = 0;
+  uint32_t mask = 0;
+  menos_adamw_cfg opt{};
+  int step = 0;
+  int col_off[NG] = {0, 0, 0, 0}, width[NG] = {0, 0, 0, 0};
+  int sub[NT];                      // slot sub-offset of target t inside the group slot (j * rs), -1 if absent
+  float* buf = nullptr;             // P | G | M | V, each n_params fp32
+  size_t n_params = 0;
+  std::vector<long long> offA, offB;  // [layer * NT + t]
+  float *P() const { return buf; }
+  float *G() const { return buf + n_params; }
+  float *M() const { return buf + 2 * n_params; }
+  float *V() const { return buf + 3 * n_params; }
+};
+
+// column allocator over the slot tables of one group (16-column units)
+struct ColAlloc {
+  std::map<int, int> free_;  // off -> width
+  int cap = 0;
+  int alloc(int w) {
+    for (auto it = free_.begin(); it != free_.end(); ++it)
+      if (it->second >= w) {
+        int off = it->first, sz = it->second;
+        free_.erase(it);
+        if (sz > w) free_[off + w] = sz - w;
+        return off;
+      }
+    return -1;
+  }
+  void release(int off, int w) {
+    free_[off] = w;
+    // coalesce
+    auto it = free_.begin();
+    while (it != free_.end()) {
+      auto nx = std::next(it);
+      if (nx != free_.end() && it->first + it->second == nx->first) { it->second += nx->second; free_.erase(nx); }
+      else it = nx;
+    }
+  }
+  void grow(int newcap) {
+    if (newcap > cap) release(cap, newcap - cap);
+    cap = newcap;
+  }
+  int max_end() const {  // end of the highest allocated column
+    int end = cap;
+    auto it = free_.rbegin();
+    if (it != free_.rend() && it->first + it->second == cap) end = it->first;
+    return end;
+  }
+};
+
+// =====================================================================================================
+// batch
+// =====================================================================================================
+struct LayerSave {
+  bf16 *x, *xn, *qkv, *O, *h, *hn, *gu, *a;
+  float *rstd1, *rstd2, *lse;
+  bf16* U[NG];
+};
+struct SGList { int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0; };
+
+struct menos_batch {
+  int T = 0, n_seqs = 0;
+  bool nograd = false;
+  std::vector<int> seq_client, seq_len, cu;
+  std::vector<int> bclients, btok_off, btok_n;  // unique clients in batch order, their token ranges
+  std::vector<int> pos;
+  int R_used[NG] = {0, 0, 0, 0};
+  bool g_active[NG] = {false, false, false, false};
+  bool save_a = false;
+  int n_mt = 0, n_blocks = 0;
+  // device metadata
+  uint8_t* meta = nullptr;  // arena
+  int* d_cu = nullptr; int* d_pos = nullptr; int2* d_blocks = nullptr;
+  int2* d_mtile[NG] = {nullptr, nullptr, nullptr, nullptr};
+  uint8_t* d_ntile_qkv = nullptr;
+  SmallGemmProblem* d_probs = nullptr; int4* d_tiles = nullptr;
+  // per layer, per group: fwd shrink, bwd dU, bwd dA+dB
+  std::vector<SGList> sg_fwd, sg_du, sg_grad;  // [layer * NG + g]
+  // saved activations (SAVE) or x_c copy (NOGRAD)
+  uint8_t* slab = nullptr;
+  std::vector<LayerSave> L;
+  bf16* xout = nullptr;
+};
+
+// =====================================================================================================
+// server
+// =====================================================================================================
+struct menos_server {
+  menos_model_cfg cfg{};
+  Dims D{};
+  int first_layer = 0, n_layers = 0, device = 0, num_sms = 148;
+  menos_server_opts opts{};
+  // WeightStore: one bf16 copy of every server layer, packed for the kernels
+  uint8_t* wbuf = nullptr; size_t wbytes = 0;
+  struct LW { bf16 *wqkv, *wo, *wgu, *wd; float *g1, *g2; };
+  std::vector<LW> W;
+  std::vector<bool> loaded;
+  // LoRA slot tables per layer per group (bf16): Bcat [N_g, cap], Acat [cap, ldK_g]
+  ColAlloc cols[NG];
+  std::vector<bf16*> Bcat[NG], Acat[NG];
+  // registry
+  std::vector<Client> clients;
+  // rope table
+  float2* rope = nullptr;
+  // arena + scratch
+  Arena arena;
+  uint8_t* arena_mem = nullptr;
+  uint8_t* scratch = nullptr; size_t scratch_bytes = 0;
+  // pinned host staging for metadata uploads
+  uint8_t* pinned = nullptr; size_t pinned_bytes = 0;
+};
+
+// =====================================================================================================
+// helpers: weights
+// =====================================================================================================
+static int upload_layer(menos_server* s, int l, const menos_layer_weights* w) {
+  const Dims& D = s->D;
+  auto& L = s->W[l];
+  const size_t b2 = 2;
+  if (!w || !w->wq || !w->wk || !w->wv || !w->wo || !w->wgate || !w->wup || !w->wdown || !w->g1 || !w->g2)
+    FAIL(MENOS_EINVAL, "layer %d: null weight pointer", l);
+  cudaStream_t st = 0;
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv, w->wq, (size_t)D.Nq * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)D.Nq * D.d, w->wk, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)(D.Nq + D.Nkv) * D.d, w->wv, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wo, w->wo, (size_t)D.d * D.Nq * b2, cudaMemcpyDefault, st));
+  // gate/up interleaved in 128-row blocks: rows [fb*256, +128) gate, [fb*256+128, +128) up
+  const int nfull = D.f / 128, tail = D.f % 128;
+  const size_t rowb = (size_t)D.d * b2;
+  if (nfull > 0) {
+    CUDA_TRY(cudaMemcpy2DAsync(L.wgu, 256 * rowb, w->wgate, 128 * rowb, 128 * rowb, nfull, cudaMemcpyDefault, st));
+    CUDA_TRY(cudaMemcpy2DAsync(L.wgu + (size_t)128 * D.d, 256 * rowb, w->wup, 128 * rowb, 128 * rowb, nfull,
+                               cudaMemcpyDefault, st));
+  }
+  if (tail) {
+    CUDA_TRY(cudaMemcpyAsync(L.wgu + (size_t)nfull * 256 * D.d, (const uint8_t*)w->wgate + (size_t)nfull * 128 * rowb,
+                             tail * rowb, cudaMemcpyDefault, st));
+    CUDA_TRY(cudaMemcpyAsync(L.wgu + ((size_t)nfull * 256 + 128) * D.d,
+                             (const uint8_t*)w->wup + (size_t)nfull * 128 * rowb, tail * rowb, cudaMemcpyDefault, st));
+  }
+  CUDA_TRY(cudaMemcpy2DAsync(L.wd, (size_t)D.fpad * b2, w->wdown, (size_t)D.f * b2, (size_t)D.f * b2, D.d,
+                             cudaMemcpyDefault, st));
+  // gains -> fp32
+  bf16* tmp = nullptr;
+  CUDA_TRY(cudaMalloc(&tmp, (size_t)2 * D.d * b2));
+  CUDA_TRY(cudaMemcpyAsync(tmp, w->g1, D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(tmp + D.d, w->g2, D.d * b2, cudaMemcpyDefault, st));
+  K_TRY(convert_bf16_to_f32(tmp, L.g1, D.d, st));
+  K_TRY(convert_bf16_to_f32(tmp + D.d, L.g2, D.d, st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  CUDA_TRY(cudaFree(tmp));
+  s->loaded[l] = true;
+  return MENOS_OK;
+}
+
+// =====================================================================================================
+// helpers: slot tables
+// =====================================================================================================
+static int grow_group(menos_server* s, int g, int need_end) {
+  int cap = s->cols[g].cap;
+  if (need_end <= cap) return MENOS_OK;
+  int nc = std::max(64, cap);
+  while (nc < need_end) nc *= 2;
+  const Dims& D = s->D;
+  for (int l = 0; l < s->n_layers; ++l) {
+    bf16 *nb = nullptr, *na = nullptr;
+    if (cudaMalloc(&nb, (size_t)D.N_g[g] * nc * 2) != cudaSuccess) FAIL(MENOS_ENOMEM, "slot table growth");
+    if (cudaMalloc(&na, (size_t)nc * D.ldK_g[g] * 2) != cudaSuccess) FAIL(MENOS_ENOMEM, "slot table growth");
+    CUDA_TRY(cudaMemset(nb, 0, (size_t)D.N_g[g] * nc * 2));
+    CUDA_TRY(cudaMemset(na, 0, (size_t)nc * D.ldK_g[g] * 2));
+    if (cap > 0) {
+      CUDA_TRY(cudaMemcpy2D(nb, (size_t)nc * 2, s->Bcat[g][l], (size_t)cap * 2, (size_t)cap * 2, D.N_g[g],
+                            cudaMemcpyDeviceToDevice));
+      CUDA_TRY(cudaMemcpy(na, s->Acat[g][l], (size_t)cap * D.ldK_g[g] * 2, cudaMemcpyDeviceToDevice));
+      CUDA_TRY(cudaFree(s->Bcat[g][l]));
+      CUDA_TRY(cudaFree(s->Acat[g][l]));
+    }
+    s->Bcat[g][l] = nb;
+    s->Acat[g][l] = na;
+  }
+  s->cols[g].grow(nc);
+  return MENOS_OK;
+}
+
+// AdamW / refresh segments of one client (both A and B of every targeted (layer, target))
+static void client_segments(menos_server* s, const Client& c, int hyp_idx, std::vector<AdamSeg>& segs) {
+  const Dims& D = s->D;
+  for (int l = 0; l < s->n_layers; ++l)
+    for (int t = 0; t < NT; ++t) {
+      if (!(c.mask >> t & 1)) continue;
+      const int g = kTargetGroup[t];
+      AdamSeg a{};
+      a.p_off = c.offA[l * NT + t]; a.rows = c.rank; a.cols = D.K_t[t]; a.client = hyp_idx;
+      a.dst = s->Acat[g][l] + (size_t)(c.col_off[g] + c.sub[t]) * D.ldK_g[g];
+      a.dst_ld = D.ldK_g[g]; a.is_b = 0; a.row_blk = 1 << 30; a.row_blk_stride = 0; a.row_base = 0;
+      segs.push_back(a);
+      AdamSeg b{};
+      b.p_off = c.offB[l * NT + t]; b.rows = D.N_t[t]; b.cols = c.rank; b.client = hyp_idx;
+      b.dst = s->Bcat[g][l] + c.col_off[g] + c.sub[t];
+      b.dst_ld = s->cols[g].cap; b.is_b = 1;
+      b.row_blk = D.rb_blk[t]; b.row_blk_stride = D.rb_stride[t]; b.row_base = D.rb_base[t];
+      segs.push_back(b);
+    }
+}
+
+static int ensure_pinned(menos_server* s, size_t n) {
+  if (n <= s->pinned_bytes) return MENOS_OK;
+  if (s->pinned) cudaFreeHost(s->pinned);
+  s->pinned = nullptr;
+  size_t nb = std::max(n, (size_t)1 << 20);
+  CUDA_TRY(cudaMallocHost(&s->pinned, nb));
+  s->pinned_bytes = nb;
+  return MENOS_OK;
+}
+
+// run AdamW (do_update) or plain bf16 refresh over a set of clients; synchronous w.r.t. host staging
+static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, cudaStream_t st,
+                    const std::vector<AdamSeg>* only = nullptr) {
+  std::vector<AdamHyper> hyp;
+  std::vector<AdamSeg> segs;
+  for (size_t i = 0; i < ids.size(); ++i) {
+    Client& c = s->clients[ids[i]];
+    AdamHyper h{};
+    h.p = c.P(); h.g = c.G(); h.m = c.M(); h.v = c.V();
+    h.do_update = update ? 1 : 0;
+    if (update) {
+      c.step += 1;
+      h.lr = c.opt.lr; h.beta1 = c.opt.beta1; h.beta2 = c.opt.beta2; h.eps = c.opt.eps; h.wd = c.opt.weight_decay;
+      h.bc1 = (float)(1.0 - std::pow((double)c.opt.beta1, (double)c.step));
+      h.bc2_sqrt = (float)std::sqrt(1.0 - std::pow((double)c.opt.beta2, (double)c.step));
+    }
+    hyp.push_back(h);
+    if (!only) client_segments(s, c, (int)i, segs);
+  }
+  if (only) segs = *only;
+  std::vector<int4> work;
+  for (size_t k = 0; k < segs.size(); ++k) {
+    const long long n = (long long)segs[k].rows * segs[k].cols;
+    for (long long o = 0; o < n; o += 4096) work.push_back(make_int4((int)k, (int)o, (int)std::min<long long>(4096, n - o), 0));
+  }
+  if (work.empty()) return MENOS_OK;
+  const size_t b1 = hyp.size() * sizeof(AdamHyper), b2 = segs.size() * sizeof(AdamSeg), b3 = work.size() * sizeof(int4);
+  const size_t o2 = align_up(b1, 256), o3 = o2 + align_up(b2, 256), tot = o3 + b3;
+  uint8_t* dbuf = nullptr;
+  CUDA_TRY(cudaMallocAsync((void**)&dbuf, tot, st));
+  int rc = ensure_pinned(s, tot);
+  if (rc) return rc;
+  CUDA_TRY(cudaStreamSynchronize(st));  // pinned staging reuse
+  memcpy(s->pinned, hyp.data(), b1);
+  memcpy(s->pinned + o2, segs.data(), b2);
+  memcpy(s->pinned + o3, work.data(), b3);
+  CUDA_TRY(cudaMemcpyAsync(dbuf, s->pinned, tot, cudaMemcpyHostToDevice, st));
+  K_TRY(adamw_run((AdamSeg*)(dbuf + o2), (int4*)(dbuf + o3), (int)work.size(), (AdamHyper*)dbuf, st));
+  CUDA_TRY(cudaFreeAsync(dbuf, st));
+  return MENOS_OK;
+}
+
+// =====================================================================================================
+// C-ABI: server lifecycle
+// =====================================================================================================
+extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, int n_layers,
+                                   const menos_layer_weights* w, int device, const menos_server_opts* opts,
+                                   menos_server** out) {
+  if (!cfg || !out || n_layers <= 0 || first_layer < 0) FAIL(MENOS_EINVAL, "null cfg/out or bad layer range");
+  *out = nullptr;
+  if (cfg->d_model <= 0 || cfg->n_heads <= 0 || cfg->n_kv_heads <= 0 || cfg->d_ff <= 0 ||
+      cfg->d_model % cfg->n_heads || cfg->n_heads % cfg->n_kv_heads)
+    FAIL(MENOS_EINVAL, "bad model dims");
+  const int hd = cfg->d_model / cfg->n_heads;
+  if (hd != 16 && hd != 32 && hd != 64 && hd != 128) FAIL(MENOS_EINVAL, "head_dim %d unsupported (16/32/64/128)", hd);
+  if (cfg->d_model % 64) FAIL(MENOS_EINVAL, "d_model must be a multiple of 64");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) FAIL(MENOS_ECUDA, "no CUDA device %d", device);
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10) FAIL(MENOS_ECUDA, "device %d is sm_%d%d; this library is built for sm_100a", device, prop.major, prop.minor);
+  CUDA_TRY(cudaSetDevice(device));
+
+  std::unique_ptr<menos_server> s(new menos_server());
+  s->cfg = *cfg; s->D = make_dims(*cfg); s->first_layer = first_layer; s->n_layers = n_layers; s->device = device;
+  menos_server_opts o{};
+  if (opts) o = *opts;
+  if (o.max_clients <= 0) o.max_clients = 64;
+  if (o.max_rank <= 0) o.max_rank = 64;
+  if (o.max_seq_len <= 0) o.max_seq_len = 4096;
+  s->num_sms = o.num_sms > 0 ? o.num_sms : prop.multiProcessorCount;
+  s->opts = o;
+  const Dims& D = s->D;
+
+  // WeightStore: one allocation for all layers (a single preloaded copy)
+  const size_t per = align_up((size_t)D.Nqkv * D.d * 2, 256) + align_up((size_t)D.d * D.Nq * 2, 256) +
+                     align_up((size_t)2 * D.fpad * D.d * 2, 256) + align_up((size_t)D.d * D.fpad * 2, 256) +
+                     2 * align_up((size_t)D.d * 4, 256);
+  s->wbytes = per * n_layers;
+  if (cudaMalloc(&s->wbuf, s->wbytes) != cudaSuccess) { cudaGetLastError(); FAIL(MENOS_ENOMEM, "weight store (%zu B)", s->wbytes); }
+  CUDA_TRY(cudaMemset(s->wbuf, 0, s->wbytes));
+  s->W.resize(n_layers);
+  s->loaded.assign(n_layers, false);
+  for (int l = 0; l < n_layers; ++l) {
+    uint8_t* p = s->wbuf + per * l;
+    auto& L = s->W[l];
+    L.wqkv = (bf16*)p; p += align_up((size_t)D.Nqkv * D.d * 2, 256);
+    L.wo = (bf16*)p; p += align_up((size_t)D.d * D.Nq * 2, 256);
+    L.wgu = (bf16*)p; p += align_up((size_t)2 * D.fpad * D.d * 2, 256);
+    L.wd = (bf16*)p; p += align_up((size_t)D.d * D.fpad * 2, 256);
+    L.g1 = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.g2 = (float*)p;
+  }
+  for (int g = 0; g < NG; ++g) { s->Bcat[g].assign(n_layers, nullptr); s->Acat[g].assign(n_layers, nullptr); }
+  CUDA_TRY(cudaMalloc(&s->rope, (size_t)o.max_seq_len * (D.hd / 2) * sizeof(float2)));
+  K_TRY(fill_rope_table(s->rope, o.max_seq_len, D.hd, D.theta, 0));
+  s->clients.resize(o.max_clients);
+  if (w) {
+    for (int l = 0; l < n_layers; ++l) {
+      int rc = upload_layer(s.get(), l, &w[l]);
+      if (rc) { menos_server_destroy(s.release()); return rc; }
+    }
+  }
+  // activation arena I (Eq.3)
+  size_t fb = 0, tb = 0;
+  CUDA_TRY(cudaMemGetInfo(&fb, &tb));
+  size_t ab = o.arena_bytes;
+  if (ab == 0) ab = fb > ((size_t)8 << 30) ? fb - ((size_t)8 << 30) : fb / 2;
+  if (cudaMalloc(&s->arena_mem, ab) != cudaSuccess) { cudaGetLastError(); menos_server_destroy(s.release()); FAIL(MENOS_ENOMEM, "arena (%zu B)", ab); }
+  s->arena.init(s->arena_mem, ab);
+  CUDA_TRY(cudaDeviceSynchronize());
+  *out = s.release();
+  return MENOS_OK;
+}
+
+extern "C" int menos_server_load_layer(menos_server* s, int layer, const menos_layer_weights* w) {
+  if (!s || layer < 0 || layer >= s->n_layers) FAIL(MENOS_EINVAL, "bad server/layer");
+  CUDA_TRY(cudaSetDevice(s->device));
+  return upload_layer(s, layer, w);
+}
+
+extern "C" void menos_server_destroy(menos_server* s) {
+  if (!s) return;
+  cudaSetDevice(s->device);
+  cudaDeviceSynchronize();
+  for (auto& c : s->clients) if (c.buf) cudaFree(c.buf);
+  for (int g = 0; g < NG; ++g)
+    for (int l = 0; l < s->n_layers; ++l) { if (s->Bcat[g][l]) cudaFree(s->Bcat[g][l]); if (s->Acat[g][l]) cudaFree(s->Acat[g][l]); }
+  if (s->wbuf) cudaFree(s->wbuf);
+  if (s->rope) cudaFree(s->rope);
+  if (s->arena_mem) cudaFree(s->arena_mem);
+  if (s->pinned) cudaFreeHost(s->pinned);
+  delete s;
+}
+
+// =====================================================================================================
+// C-ABI: clients
+// =====================================================================================================
+static uint64_t splitmix(uint64_t& x) {
+  uint64_t z = (x += 0x9e3779b97f4a7c15ull);
+  z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+  z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+  return z ^ (z >> 31);
+}
+
+extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uint32_t target_mask,
+                                     const menos_adamw_cfg* opt, uint64_t init_seed, int32_t* client_id) {
+  if (!s || !client_id) FAIL(MENOS_EINVAL, "null server/id");
+  if (rank < 1 || rank > s->opts.max_rank) FAIL(MENOS_EINVAL, "rank %d outside [1, %d]", rank, s->opts.max_rank);
+  if (!(alpha > 0.f) || target_mask == 0 || (target_mask >> NT)) FAIL(MENOS_EINVAL, "bad alpha/target mask");
+  CUDA_TRY(cudaSetDevice(s->device));
+  int id = -1;
+  for (size_t i = 0; i < s->clients.size(); ++i) if (!s->clients[i].used) { id = (int)i; break; }
+  if (id < 0) FAIL(MENOS_ENOMEM, "client registry full (%d)", s->opts.max_clients);
+  const Dims& D = s->D;
+  Client c;
+  c.rank = rank; c.rs = (int)align_up(rank, 16); c.alpha = alpha; c.s = alpha / (float)rank; c.mask = target_mask;
+  c.opt = opt ? *opt : menos_adamw_cfg{1e-4f, 0.9f, 0.999f, 1e-8f, 0.01f};
+  for (int t = 0; t < NT; ++t) c.sub[t] = -1;
+  int cnt[NG] = {0, 0, 0, 0};
+  for (int t = 0; t < NT; ++t)
+    if (target_mask >> t & 1) { const int g = kTargetGroup[t]; c.sub[t] = cnt[g] * c.rs; cnt[g]++; }
+  // slot columns per group
+  for (int g = 0; g < NG; ++g) {
+    c.width[g] = cnt[g] * c.rs;
+    if (!c.width[g]) continue;
+    int off = s->cols[g].alloc(c.width[g]);
+    if (off < 0) {
+      int rc = grow_group(s, g, s->cols[g].cap + c.width[g]);
+      if (rc) return rc;
+      off = s->cols[g].alloc(c.width[g]);
+    }
+    if (off < 0) FAIL(MENOS_ENOMEM, "slot allocation");
+    c.col_off[g] = off;
+  }
+  // parameter layout
+  c.offA.assign((size_t)s->n_layers * NT, -1);
+  c.offB.assign((size_t)s->n_layers * NT, -1);
+  size_t n = 0;
+  for (int l = 0; l < s->n_layers; ++l)
+    for (int t = 0; t < NT; ++t) {
+      if (!(target_mask >> t & 1)) continue;
+      c.offA[l * NT + t] = (long long)n; n += (size_t)rank * D.K_t[t];
+      c.offB[l * NT + t] = (long long)n; n += (size_t)D.N_t[t] * rank;
+    }
+  c.n_params = n;
+  if (cudaMalloc(&c.buf, 4 * n * sizeof(float)) != cudaSuccess) { cudaGetLastError(); FAIL(MENOS_ENOMEM, "adapter state"); }
+  CUDA_TRY(cudaMemset(c.buf, 0, 4 * n * sizeof(float)));
+  // init: A ~ U(-1/sqrt(K), 1/sqrt(K)) (PEFT kaiming-uniform a=sqrt(5)), B = 0
+  std::vector<float> host(n, 0.f);
+  uint64_t st = init_seed * 0x2545F4914F6CDD1Dull + 1;
+  for (int l = 0; l < s->n_layers; ++l)
+    for (int t = 0; t < NT; ++t) {
+      if (!(target_mask >> t & 1)) continue;
+      const double bound = 1.0 / std::sqrt((double)D.K_t[t]);
+      const long long o = c.offA[l * NT + t];
+      for (long long i = 0; i < (long long)rank * D.K_t[t]; ++i) {
+        const double u = (double)(splitmix(st) >> 11) * (1.0 / 9007199254740992.0);
+        host[o + i] = (float)((2.0 * u - 1.0) * bound);
+      }
+    }
+  CUDA_TRY(cudaMemcpy(c.buf, host.data(), n * sizeof(float), cudaMemcpyHostToDevice));
+  c.used = true;
+  s->clients[id] = c;
+  int rc = run_adam(s, {id}, false, 0);
+  if (rc) return rc;
+  CUDA_TRY(cudaDeviceSynchronize());
+  *client_id = id;
+  return MENOS_OK;
+}
+
+extern "C" int menos_unregister_client(menos_server* s, int32_t id) {
+  if (!s) FAIL(MENOS_EINVAL, "null server");
+  if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+  CUDA_TRY(cudaSetDevice(s->device));
+  CUDA_TRY(cudaDeviceSynchronize());
+  Client& c = s->clients[id];
+  const Dims& D = s->D;
+  for (int g = 0; g < NG; ++g) {
+    if (!c.width[g]) continue;
+    for (int l = 0; l < s->n_layers; ++l) {
+      CUDA_TRY(cudaMemset2D(s->Bcat[g][l] + c.col_off[g], (size_t)s->cols[g].cap * 2, 0, (size_t)c.width[g] * 2, D.N_g[g]));
+      CUDA_TRY(cudaMemset(s->Acat[g][l] + (size_t)c.col_off[g] * D.ldK_g[g], 0, (size_t)c.width[g] * D.ldK_g[g] * 2));
+    }
+    s->cols[g].release(c.col_off[g], c.width[g]);
+  }
+  CUDA_TRY(cudaFree(c.buf));
+  s->clients[id] = Client();
+  CUDA_TRY(cudaDeviceSynchronize());
+  return MENOS_OK;
+}
+
+// saved bytes per token per layer in SAVE mode (excluding the LoRA U share)
+static size_t saved_bytes_per_token_layer(const Dims& D, bool save_a) {
+  size_t b = 0;
+  b += (size_t)D.d * 2 * 4;        // x, xn, h, hn
+  b += (size_t)D.Nqkv * 2;         // qkv
+  b += (size_t)D.Nq * 2;           // O
+  b += (size_t)2 * D.fpad * 2;     // gu
+  if (save_a) b += (size_t)D.fpad * 2;
+  b += 4 * 2 + (size_t)D.H * 4;    // rstd1, rstd2, lse
+  return b;
+}
+static size_t scratch_bytes_per_token(const Dims& D, int R_sum) {
+  size_t b = 0;
+  b += (size_t)D.d * 2 * 5;          // dy, dx, dhn, dh, xout
+  b += (size_t)D.Nq * 2;             // dO
+  b += (size_t)D.Nqkv * 2;           // dqkv
+  b += (size_t)2 * D.fpad * 2;       // dgu
+  b += (size_t)D.fpad * 2;           // a (when not saved)
+  b += (size_t)D.H * 4;              // D rowsums
+  b += (size_t)R_sum * 2;            // dU
+  b += 64;                           // alignment slack
+  return b;
+}
+
+extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, size_t* persistent, size_t* fwd_bytes,
+                                   size_t* bwd_bytes) {
+  if (!s) FAIL(MENOS_EINVAL, "null server");
+  if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+  if (n_tokens < 0) FAIL(MENOS_EINVAL, "n_tokens < 0");
+  const Client& c = s->clients[id];
+  const Dims& D = s->D;
+  // A + O: fp32 p, g, m, v + the bf16 slot-table copy (Acat rows + Bcat columns incl. rank padding)
+  size_t slots = 0;
+  for (int g = 0; g < NG; ++g) slots += (size_t)c.width[g] * (D.N_g[g] + D.ldK_g[g]) * 2 * s->n_layers;
+  if (persistent) *persistent = 16 * c.n_params + slots;
+  const bool save_a = (c.mask >> TD) & 1;
+  size_t ush = 0;
+  for (int g = 0; g < NG; ++g) ush += (size_t)c.width[g] * 2;
+  const size_t T = (size_t)n_tokens;
+  if (fwd_bytes) *fwd_bytes = T * ((saved_bytes_per_token_layer(D, save_a) + ush) * s->n_layers + (size_t)D.d * 2);
+  int rsum = 0;
+  for (int g = 0; g < NG; ++g) rsum += c.width[g];
+  if (bwd_bytes) *bwd_bytes = T * scratch_bytes_per_token(D, rsum);
+  return MENOS_OK;
+}
+
+extern "C" int menos_adapter_shape(menos_server* s, int32_t id, int target, int* rows, int* cols) {
+  if (!s || !rows || !cols) FAIL(MENOS_EINVAL, "null argument");
+  if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+  if (target < 0 || target >= NT) FAIL(MENOS_EINVAL, "bad target");
+  const Client& c = s->clients[id];
+  if (!(c.mask >> target & 1)) FAIL(MENOS_EINVAL, "target %d not in client mask", target);
+  rows[0] = c.rank; cols[0] = s->D.K_t[target];   // A [r, K]
+  rows[1] = s->D.N_t[target]; cols[1] = c.rank;   // B [N, r]
+  return MENOS_OK;
+}
+
+static int adapter_ptr(menos_server* s, int32_t id, int layer, int target, int which, float** p, size_t* n,
+                       Client** cp) {
+  if (!s) FAIL(MENOS_EINVAL, "null server");
+  if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+  if (layer < 0 || layer >= s->n_layers || target < 0 || target >= NT || which < 0 || which > 7)
+    FAIL(MENOS_EINVAL, "bad layer/target/which");
+  Client& c = s->clients[id];
+  if (!(c.mask >> target & 1)) FAIL(MENOS_EINVAL, "target %d not in client mask", target);
+  const bool isB = which & 1;
+  const long long off = isB ? c.offB[layer * NT + target] : c.offA[layer * NT + target];
+  *n = (size_t)c.rank * (isB ? s->D.N_t[target] : s->D.K_t[target]);
+  float* base = which < 2 ? c.P() : which < 4 ? c.G() : which < 6 ? c.M() : c.V();
+  *p = base + off;
+  *cp = &c;
+  return MENOS_OK;
+}
+
+extern "C" int menos_get_adapter(menos_server* s, int32_t id, int layer, int target, int which, float* host_out) {
+  float* p; size_t n; Client* c;
+  int rc = adapter_ptr(s, id, layer, target, which, &p, &n, &c);
+  if (rc) return rc;
+  if (!host_out) FAIL(MENOS_EINVAL, "null output");
+  CUDA_TRY(cudaSetDevice(s->device));
+  CUDA_TRY(cudaDeviceSynchronize());
+  CUDA_TRY(cudaMemcpy(host_out, p, n * sizeof(float), cudaMemcpyDeviceToHost));
+  return MENOS_OK;
+}
+
+extern "C" int menos_set_adapter(menos_server* s, int32_t id, int layer, int target, int which, const float* host_in) {
+  if (which > 1) FAIL(MENOS_EINVAL, "set_adapter: which must be 0 (A) or 1 (B)");
+  float* p; size_t n; Client* c;
+  int rc = adapter_ptr(s, id, layer, target, which, &p, &n, &c);
+  if (rc) return rc;
+  if (!host_in) FAIL(MENOS_EINVAL, "null input");
+  CUDA_TRY(cudaSetDevice(s->device));
+  CUDA_TRY(cudaDeviceSynchronize());
+  CUDA_TRY(cudaMemcpy(p, host_in, n * sizeof(float), cudaMemcpyHostToDevice));
+  std::vector<AdamSeg> all, one;
+  client_segments(s, *c, 0, all);
+  for (auto& sg : all) {
+    const long long want = which ? c->offB[layer * NT + target] : c->offA[layer * NT + target];
+    if (sg.p_off == want) one.push_back(sg);
+  }
+  rc = run_adam(s, {id}, false, 0, &one);
+  if (rc) return rc;
+  CUDA_TRY(cudaDeviceSynchronize());
+  return MENOS_OK;
+}
+
+extern "C" int menos_adapter_step(menos_server* s, int n, const int32_t* ids, void* stream) {
+  if (!s || n < 0 || (n > 0 && !ids)) FAIL(MENOS_EINVAL, "bad arguments");
+  std::vector<int> v;
+  for (int i = 0; i < n; ++i) {
+    if (ids[i] < 0 || ids[i] >= (int)s->clients.size() || !s->clients[ids[i]].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", ids[i]);
+    for (int x : v) if (x == ids[i]) FAIL(MENOS_EINVAL, "client %d listed twice", ids[i]);
+    v.push_back(ids[i]);
+  }
+  CUDA_TRY(cudaSetDevice(s->device));
+  return run_adam(s, v, true, (cudaStream_t)stream);
+}
+
+extern "C" int menos_get_stats(menos_server* s, menos_stats* o) {
+  if (!s || !o) FAIL(MENOS_EINVAL, "null argument");
+  memset(o, 0, sizeof *o);
+  o->base_bytes = s->wbytes;
+  size_t ad = 0;
+  for (auto& c : s->clients) if (c.used) { ad += 16 * c.n_params; o->n_clients++; }
+  for (int g = 0; g < NG; ++g) ad += (size_t)s->cols[g].cap * (s->D.N_g[g] + s->D.ldK_g[g]) * 2 * s->n_layers;
+  o->adapters_bytes = ad;
+  o->arena_bytes = s->arena.cap; o->arena_used = s->arena.used; o->arena_peak = s->arena.peak;
+  o->num_sms = s->num_sms;
+  return MENOS_OK;
+}
+
+extern "C" unsigned long long menos_launch_count(void) { return g_launch_count; }
+
+extern "C" int menos_sync(menos_server* s) {
+  if (!s) FAIL(MENOS_EINVAL, "null server");
+  CUDA_TRY(cudaSetDevice(s->device));
+  CUDA_TRY(cudaDeviceSynchronize());
+  CUDA_TRY(cudaGetLastError());
+  return MENOS_OK;
+}
+
+extern "C" const char* menos_last_error(void) { return tl_err.c_str(); }
+
+// =====================================================================================================
+// batch construction (BatchPacker)
+// =====================================================================================================
+struct Scratch {
+  bf16 *dy, *dx, *dhn, *dh, *dO, *dqkv, *dgu, *a, *xout;
+  float* Dsum;
+  bf16* dU[NG];
+};
+
+static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, const int32_t* seq_len, bool nograd,
+                       std::unique_ptr<menos_batch>& out) {
+  const Dims& D = s->D;
+  std::unique_ptr<menos_batch> b(new menos_batch());
+  b->n_seqs = n_seqs; b->nograd = nograd;
+  b->cu.push_back(0);
+  for (int i = 0; i < n_seqs; ++i) {
+    const int c = seq_client[i], L = seq_len[i];
+    if (c < 0 || c >= (int)s->clients.size() || !s->clients[c].used) FAIL(MENOS_ENOCLIENT, "sequence %d: unknown client %d", i, c);
+    if (L < 1 || L > s->opts.max_seq_len) FAIL(MENOS_EINVAL, "sequence %d: length %d outside [1, %d]", i, L, s->opts.max_seq_len);
+    if (i > 0 && c != seq_client[i - 1]) {
+      for (int x : b->bclients) if (x == c) FAIL(MENOS_EINVAL, "client %d's sequences are not contiguous", c);
+    }
+    if (b->bclients.empty() || b->bclients.back() != c) { b->bclients.push_back(c); b->btok_off.push_back(b->cu.back()); b->btok_n.push_back(0); }
+    b->btok_n.back() += L;
+    b->seq_client.push_back(c); b->seq_len.push_back(L);
+    b->cu.push_back(b->cu.back() + L);
+    for (int p = 0; p < L; ++p) b->pos.push_back(p);
+  }
+  b->T = b->cu.back();
+  const int T = b->T;
+  // LoRA groups active in this batch and their used slot width
+  for (int c : b->bclients) {
+    const Client& cl = s->clients[c];
+    for (int g = 0; g < NG; ++g)
+      if (cl.width[g]) { b->g_active[g] = true; b->R_used[g] = std::max(b->R_used[g], cl.col_off[g] + cl.width[g]); }
+    if (cl.mask >> TD & 1) b->save_a = true;
+  }
+  for (int g = 0; g < NG; ++g) b->R_used[g] = (int)align_up(b->R_used[g], 64);
+  b->n_mt = ceil_div(T, 128);
+  (void)D;
+  // small-GEMM problem lists are filled later (need layer buffers); reserve host vectors here
+  b->sg_fwd.resize((size_t)s->n_layers * NG);
+  b->sg_du.resize((size_t)s->n_layers * NG);
+  b->sg_grad.resize((size_t)s->n_layers * NG);
+
+  out = std::move(b);
+  return MENOS_OK;
+}
+
+// Allocate the slab (saved activations or x_c copy) and upload all metadata incl. small-GEMM problem lists.
+static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const LayerSave* ng, cudaStream_t st) {
+  const Dims& D = s->D;
+  const int T = b->T, Ls = s->n_layers;
+  // ---- sizes
+  const bool save = !b->nograd;
+  size_t ush = 0;
+  for (int g = 0; g < NG; ++g) if (b->g_active[g]) ush += (size_t)b->R_used[g] * 2;
+  size_t per_layer = 0;
+  auto A = [&](size_t n) { per_layer += align_up(n, 256); };
+  if (save) {
+    A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x, xn, rstd1
+    A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
+    A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h, hn, rstd2
+    A((size_t)T * 2 * D.fpad * 2);                                            // gu
+    if (b->save_a) A((size_t)T * D.fpad * 2);
+    for (int g = 0; g < NG; ++g) if (b->g_active[g]) A((size_t)T * b->R_used[g] * 2);
+  }
+  const size_t slab_bytes = save ? per_layer * Ls : align_up((size_t)T * D.d * 2, 256);
+  // ---- metadata blob
+  std::vector<uint8_t> blob;
+  auto put = [&](const void* p, size_t n) {
+    size_t o = align_up(blob.size(), 256); blob.resize(o + n); if (n) memcpy(blob.data() + o, p, n); return o; };
+  std::vector<int2> blocks;
+  for (int i = 0; i < b->n_seqs; ++i)
+    for (int q = 0; q < b->seq_len[i]; q += 64) blocks.push_back(make_int2(i, q));
+  std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
+  for (int g = 0; g < NG; ++g) {
+    if (!b->g_active[g]) continue;
+    for (int m = 0; m < b->n_mt; ++m) {
+      const int r0 = m * 128, r1 = std::min(T, r0 + 128);
+      int lo = 1 << 30, hi = -1;
+      for (size_t k = 0; k < b->bclients.size(); ++k) {
+        const int a0 = b->btok_off[k], a1 = a0 + b->btok_n[k];
+        if (a1 <= r0 || a0 >= r1) continue;
+        const Client& cl = s->clients[b->bclients[k]];
+        if (!cl.width[g]) continue;
+        lo = std::min(lo, cl.col_off[g]); hi = std::max(hi, cl.col_off[g] + cl.width[g]);
+      }
+      if (hi > lo) mt[(size_t)g * b->n_mt + m] = make_int2(lo, (hi - lo) / 16);
+    }
+  }
+  const int n_nt = ceil_div(D.Nqkv, 256);
+  std::vector<uint8_t> ntq(n_nt, 0);
+  for (int c : b->bclients) {
+    const Client& cl = s->clients[c];
+    const int lo[3] = {0, D.Nq, D.Nq + D.Nkv}, hi[3] = {D.Nq, D.Nq + D.Nkv, D.Nqkv};
+    for (int t = 0; t < 3; ++t)
+      if (cl.mask >> t & 1)
+        for (int n = lo[t] / 256; n <= (hi[t] - 1) / 256; ++n) ntq[n] = 1;
+  }
+  const size_t o_cu = put(b->cu.data(), b->cu.size() * 4);
+  const size_t o_pos = put(b->pos.data(), b->pos.size() * 4);
+  const size_t o_blk = put(blocks.data(), blocks.size() * sizeof(int2));
+  const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
+  const size_t o_nt = put(ntq.data(), ntq.size());
+
+  // ---- slab
+  uint8_t* slab = (uint8_t*)s->arena.alloc(slab_bytes);
+  if (!slab) FAIL(MENOS_ENOMEM, "arena: batch needs %zu B, %zu of %zu B in use", slab_bytes, s->arena.used, s->arena.cap);
+  b->slab = slab;
+  b->L.assign(Ls, LayerSave{});
+  if (save) {
+    uint8_t* p = slab;
+    auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
+    for (int l = 0; l < Ls; ++l) {
+      LayerSave& S = b->L[l];
+      S.x = (bf16*)take((size_t)T * D.d * 2); S.xn = (bf16*)take((size_t)T * D.d * 2); S.rstd1 = (float*)take((size_t)T * 4);
+      S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2); S.lse = (float*)take((size_t)D.H * T * 4);
+      S.h = (bf16*)take((size_t)T * D.d * 2); S.hn = (bf16*)take((size_t)T * D.d * 2); S.rstd2 = (float*)take((size_t)T * 4);
+      S.gu = (bf16*)take((size_t)T * 2 * D.fpad * 2);
+      S.a = b->save_a ? (bf16*)take((size_t)T * D.fpad * 2) : sc.a;
+      for (int g = 0; g < NG; ++g) S.U[g] = b->g_active[g] ? (bf16*)take((size_t)T * b->R_used[g] * 2) : nullptr;
+    }
+  } else {
+    b->L[0].x = (bf16*)slab;  // x_c copy (only the forward input is cached)
+  }
+
+  // ---- small-GEMM problem lists (need buffer pointers: built against the SAVE layout, or the scratch layer)
+  std::vector<SmallGemmProblem> probs;
+  std::vector<int4> tiles;
+  auto add_list = [&](SGList& L, const std::vector<SmallGemmProblem>& ps) {
+    L.probs_off = (int)probs.size(); L.n_probs = (int)ps.size();
+    L.tiles_off = (int)tiles.size();
+    std::vector<int4> tl(1);
+    int cnt = 0;
+    for (const auto& pp : ps) cnt += ceil_div(pp.M, SG_BM) * ceil_div(pp.N, SG_BN);
+    tl.resize(std::max(cnt, 1));
+    int nt = 0;
+    small_gemm_tiles(ps.data(), (int)ps.size(), tl.data(), &nt);
+    for (int i = 0; i < nt; ++i) tl[i].x += L.probs_off;
+    L.n_tiles = nt;
+    probs.insert(probs.end(), ps.begin(), ps.end());
+    tiles.insert(tiles.end(), tl.begin(), tl.begin() + nt);
+  };
+  for (int l = 0; l < Ls; ++l) {
+    const LayerSave& S = save ? b->L[l] : *ng;
+    bf16* dyl = ((Ls - 1 - l) % 2 == 0) ? sc.dy : sc.dx;  // layer l's incoming gradient buffer
+    for (int g = 0; g < NG; ++g) {
+      if (!b->g_active[g]) continue;
+      const int R = b->R_used[g];
+      // group input (X) and its leading dim; output-grad (dY) and its leading dim
+      const bf16* X = nullptr; int ldx = 0;
+      const bf16* dY = nullptr; int ldy = 0;
+      bf16* U = S.U[g];
+      switch (g) {
+        case GQKV: X = S.xn; ldx = D.d; dY = sc.dqkv; ldy = D.Nqkv; break;
+        case GO: X = S.O; ldx = D.Nq; dY = sc.dh; ldy = D.d; break;
+        case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = 2 * D.fpad; break;
+        case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
+      }
+      std::vector<SmallGemmProblem> f, du, gr;
+      for (size_t k = 0; k < b->bclients.size(); ++k) {
+        const Client& c = s->clients[b->bclients[k]];
+        if (!c.width[g]) continue;
+        const int t0 = b->btok_off[k], Tc = b->btok_n[k];
+        SmallGemmProblem p{};
+        p.a_blk = 1 << 30; p.a_blk_stride = 0;
+        // shrink: U[t, off..off+w) = s * X_c A^T
+        p.A = X + (size_t)t0 * ldx; p.lda = ldx;
+        p.B = s->Acat[g][l] + (size_t)c.col_off[g] * D.ldK_g[g]; p.ldb = D.ldK_g[g];
+        p.Cb = U + (size_t)t0 * R + c.col_off[g]; p.Cf = nullptr; p.ldc = R;
+        p.M = Tc; p.N = c.width[g]; p.K = D.K_g[g]; p.a_t = 0; p.b_t = 0; p.scale = c.s;
+        f.push_back(p);
+        // dU[t, off..off+w) = s * dY_c Bcat[:, off..]
+        SmallGemmProblem q{};
+        q.a_blk = 1 << 30; q.a_blk_stride = 0;
+        q.A = dY + (size_t)t0 * ldy; q.lda = ldy;
+        q.B = s->Bcat[g][l] + c.col_off[g]; q.ldb = s->cols[g].cap; q.b_t = 1; q.a_t = 0;
+        q.Cb = sc.dU[g] + (size_t)t0 * R + c.col_off[g]; q.Cf = nullptr; q.ldc = R;
+        q.M = Tc; q.N = c.width[g]; q.K = D.N_g[g]; q.scale = c.s;
+        du.push_back(q);
+        // per target: dB = dY_t^T U_t (U holds s*x A^T), dA = dU_t^T X
+        for (int t = 0; t < NT; ++t) {
+          if (kTargetGroup[t] != g || !(c.mask >> t & 1)) continue;
+          SmallGemmProblem pb{};
+          pb.A = dY + (size_t)t0 * ldy + D.rb_base[t]; pb.lda = ldy; pb.a_t = 1;
+          pb.a_blk = D.rb_blk[t]; pb.a_blk_stride = D.rb_stride[t];
+          pb.B = U + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pb.ldb = R; pb.b_t = 1;
+          pb.Cf = c.G() + c.offB[l * NT + t]; pb.Cb = nullptr; pb.ldc = c.rank;
+          pb.M = D.N_t[t]; pb.N = c.rank; pb.K = Tc; pb.scale = 1.f;
+          gr.push_back(pb);
+          SmallGemmProblem pa{};
+          pa.a_blk = 1 << 30; pa.a_blk_stride = 0;
+          pa.A = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pa.lda = R; pa.a_t = 1;
+          pa.B = X + (size_t)t0 * ldx; pa.ldb = ldx; pa.b_t = 1;
+          pa.Cf = c.G() + c.offA[l * NT + t]; pa.Cb = nullptr; pa.ldc = D.K_t[t];
+          pa.M = c.rank; pa.N = D.K_t[t]; pa.K = Tc; pa.scale = 1.f;
+          gr.push_back(pa);
+        }
+      }
+      add_list(b->sg_fwd[(size_t)l * NG + g], f);
+      add_list(b->sg_du[(size_t)l * NG + g], du);
+      add_list(b->sg_grad[(size_t)l * NG + g], gr);
+    }
+  }
+  const size_t o_pr = put(probs.data(), probs.size() * sizeof(SmallGemmProblem));
+  const size_t o_tl = put(tiles.data(), tiles.size() * sizeof(int4));
+  uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
+  if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
+  b->meta = meta;
+  int rc = ensure_pinned(s, blob.size());
+  if (rc) return rc;
+  CUDA_TRY(cudaStreamSynchronize(st));
+  memcpy(s->pinned, blob.data(), blob.size());
+  CUDA_TRY(cudaMemcpyAsync(meta, s->pinned, blob.size(), cudaMemcpyHostToDevice, st));
+  b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
+  for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
+  b->d_ntile_qkv = meta + o_nt;
+  b->d_probs = (SmallGemmProblem*)(meta + o_pr);
+  b->d_tiles = (int4*)(meta + o_tl);
+  return MENOS_OK;
+}
+
+// scratch (per server, grown to the largest batch; used only inside one call)
+static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc) {
+  const Dims& D = s->D;
+  int rsum = 0;
+  for (int g = 0; g < NG; ++g) rsum += R_used[g];
+  size_t need = 0;
+  auto A = [&](size_t n) { need += align_up(n, 256); };
+  A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.d * 2);
+  A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * 2 * D.fpad * 2); A((size_t)T * D.fpad * 2);
+  A((size_t)T * D.d * 2); A((size_t)D.H * T * 4);
+  for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
+  // NOGRAD forward layer set (x ping-pong handled by xout/dx; intermediates reuse the grad buffers)
+  A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
+  A((size_t)T * 2 * D.fpad * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
+  for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
+  if (need > s->scratch_bytes) {
+    if (s->scratch) s->arena.release(s->scratch);
+    s->scratch = (uint8_t*)s->arena.alloc(need);
+    if (!s->scratch) { s->scratch_bytes = 0; FAIL(MENOS_ENOMEM, "arena: scratch needs %zu B", need); }
+    s->scratch_bytes = need;
+  }
+  uint8_t* p = s->scratch;
+  auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
+  sc.dy = (bf16*)take((size_t)T * D.d * 2); sc.dx = (bf16*)take((size_t)T * D.d * 2);
+  sc.dhn = (bf16*)take((size_t)T * D.d * 2); sc.dh = (bf16*)take((size_t)T * D.d * 2);
+  sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
+  sc.dgu = (bf16*)take((size_t)T * 2 * D.fpad * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
+  sc.xout = (bf16*)take((size_t)T * D.d * 2); sc.Dsum = (float*)take((size_t)D.H * T * 4);
+  for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
+  return MENOS_OK;
+}
+
+// NOGRAD layer buffers carved after the regular scratch (same arena block)
+static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scratch& sc, LayerSave& S) {
+  const Dims& D = s->D;
+  uint8_t* p = (uint8_t*)(sc.dU[NG - 1]) + align_up((size_t)T * R_used[NG - 1] * 2, 256);
+  auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
+  S.xn = (bf16*)take((size_t)T * D.d * 2); S.h = (bf16*)take((size_t)T * D.d * 2);
+  S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
+  S.gu = (bf16*)take((size_t)2 * T * D.fpad * 2); S.lse = (float*)take((size_t)D.H * T * 4);
+  S.rstd1 = (float*)take((size_t)T * 8); S.rstd2 = S.rstd1 + T;
+  S.hn = sc.dhn;  // free during a forward
+  S.a = sc.a;
+  for (int g = 0; g < NG; ++g) S.U[g] = (bf16*)take((size_t)T * R_used[g] * 2);
+}
+
+// =====================================================================================================
+// per-layer schedules
+// =====================================================================================================
+static int run_sg(menos_batch* b, const SGList& L, cudaStream_t st) {
+  if (L.n_tiles == 0) return 0;
+  return small_gemm_run(b->d_probs, b->d_tiles + L.tiles_off, L.n_tiles, st);
+}
+
+static GemmArgs gemm_base(menos_server* s) {
+  GemmArgs a;
+  memset(&a, 0, sizeof a);
+  a.num_sms = s->num_sms;
+  return a;
+}
+
+// forward of layer l: x -> y; S holds the destinations of every intermediate
+static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, bf16* y, const LayerSave& S,
+                         bool use_lists, cudaStream_t st) {
+  const Dims& D = s->D;
+  const auto& W = s->W[l];
+  const int T = b->T;
+  // A1: RMSNorm1
+  K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st));
+  // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
+  if (b->g_active[GQKV]) {
+    CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
+    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GQKV], st));
+  }
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.Nqkv; a.K = D.d; a.b_mn_major = 0;
+    a.A = S.xn; a.lda = D.d; a.B = W.wqkv; a.ldb = D.d;
+    if (b->g_active[GQKV]) {
+      a.R = b->R_used[GQKV]; a.A2 = S.U[GQKV]; a.lda2 = a.R; a.B2 = s->Bcat[GQKV][l]; a.ldb2 = s->cols[GQKV].cap;
+      a.mtile_extra = b->d_mtile[GQKV]; a.ntile_extra = b->d_ntile_qkv;
+    }
+    a.epi = EPI_ROPE; a.out = S.qkv; a.ldo = D.Nqkv;
+    a.rope_cs = s->rope; a.pos = b->d_pos; a.head_dim = D.hd; a.rope_cols = D.Nq + D.Nkv;
+    K_TRY(gemm_run(a, st));
+  }
+  // A3: varlen causal flash attention
+  {
+    AttnArgs a;
+    memset(&a, 0, sizeof a);
+    a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
+    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
+    a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    K_TRY(attn_fwd(a, st));
+  }
+  // A4: O GEMM (+ LoRA o) + residual
+  if (b->g_active[GO]) {
+    CUDA_TRY(cudaMemsetAsync(S.U[GO], 0, (size_t)T * b->R_used[GO] * 2, st));
+    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GO], st));
+  }
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.d; a.K = D.Nq; a.A = S.O; a.lda = D.Nq; a.B = W.wo; a.ldb = D.Nq;
+    if (b->g_active[GO]) {
+      a.R = b->R_used[GO]; a.A2 = S.U[GO]; a.lda2 = a.R; a.B2 = s->Bcat[GO][l]; a.ldb2 = s->cols[GO].cap;
+      a.mtile_extra = b->d_mtile[GO];
+    }
+    a.epi = EPI_RESID; a.out = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
+    K_TRY(gemm_run(a, st));
+  }
+  // A5: RMSNorm2
+  K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st));
+  // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
+  if (b->g_active[GGU]) {
+    CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
+    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GGU], st));
+  }
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = 2 * D.fpad; a.K = D.d; a.A = S.hn; a.lda = D.d; a.B = W.wgu; a.ldb = D.d;
+    if (b->g_active[GGU]) {
+      a.R = b->R_used[GGU]; a.A2 = S.U[GGU]; a.lda2 = a.R; a.B2 = s->Bcat[GGU][l]; a.ldb2 = s->cols[GGU].cap;
+      a.mtile_extra = b->d_mtile[GGU];
+    }
+    a.epi = EPI_SWIGLU_FWD; a.out = S.gu; a.ldo = 2 * D.fpad; a.out2 = S.a; a.ldo2 = D.fpad;
+    K_TRY(gemm_run(a, st));
+  }
+  // A7: down GEMM (+ LoRA down) + residual
+  if (b->g_active[GD]) {
+    CUDA_TRY(cudaMemsetAsync(S.U[GD], 0, (size_t)T * b->R_used[GD] * 2, st));
+    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GD], st));
+  }
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.d; a.K = D.fpad; a.A = S.a; a.lda = D.fpad; a.B = W.wd; a.ldb = D.fpad;
+    if (b->g_active[GD]) {
+      a.R = b->R_used[GD]; a.A2 = S.U[GD]; a.lda2 = a.R; a.B2 = s->Bcat[GD][l]; a.ldb2 = s->cols[GD].cap;
+      a.mtile_extra = b->d_mtile[GD];
+    }
+    a.epi = EPI_RESID; a.out = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
+    K_TRY(gemm_run(a, st));
+  }
+  return MENOS_OK;
+}
+
+// backward of layer l: dy -> dx (LoRA grads of layer l written into each client's G)
+static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy, bf16* dx, const Scratch& sc,
+                          cudaStream_t st) {
+  const Dims& D = s->D;
+  const auto& W = s->W[l];
+  const LayerSave& S = b->L[l];
+  const int T = b->T;
+  // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
+  if (b->g_active[GD]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GD], st));
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.fpad; a.K = D.d; a.b_mn_major = 1;
+    a.A = dy; a.lda = D.d; a.B = W.wd; a.ldb = D.fpad;
+    if (b->g_active[GD]) {
+      a.R = b->R_used[GD]; a.A2 = sc.dU[GD]; a.lda2 = a.R; a.B2 = s->Acat[GD][l]; a.ldb2 = D.ldK_g[GD];
+      a.mtile_extra = b->d_mtile[GD];
+    }
+    a.epi = EPI_SWIGLU_BWD; a.out = sc.dgu; a.ldo = 2 * D.fpad; a.aux = S.gu; a.ldaux = 2 * D.fpad;
+    K_TRY(gemm_run(a, st));
+  }
+  if (b->g_active[GD]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GD], st));
+  // A9: gate/up dX (+ LoRA) -> dhn; RMSNorm2 backward + residual -> dh
+  if (b->g_active[GGU]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GGU], st));
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.d; a.K = 2 * D.fpad; a.b_mn_major = 1;
+    a.A = sc.dgu; a.lda = 2 * D.fpad; a.B = W.wgu; a.ldb = D.d;
+    if (b->g_active[GGU]) {
+      a.R = b->R_used[GGU]; a.A2 = sc.dU[GGU]; a.lda2 = a.R; a.B2 = s->Acat[GGU][l]; a.ldb2 = D.ldK_g[GGU];
+      a.mtile_extra = b->d_mtile[GGU];
+    }
+    a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
+    K_TRY(gemm_run(a, st));
+  }
+  if (b->g_active[GGU]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GGU], st));
+  K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dy, sc.dh, T, D.d, st));
+  // A10: O dX (+ LoRA o) -> dO
+  if (b->g_active[GO]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GO], st));
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
+    a.A = sc.dh; a.lda = D.d; a.B = W.wo; a.ldb = D.Nq;
+    if (b->g_active[GO]) {
+      a.R = b->R_used[GO]; a.A2 = sc.dU[GO]; a.lda2 = a.R; a.B2 = s->Acat[GO][l]; a.ldb2 = D.ldK_g[GO];
+      a.mtile_extra = b->d_mtile[GO];
+    }
+    a.epi = EPI_STORE; a.out = sc.dO; a.ldo = D.Nq;
+    K_TRY(gemm_run(a, st));
+  }
+  if (b->g_active[GO]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GO], st));
+  // A11: attention backward (+ RoPE backward) -> dqkv
+  K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st));
+  {
+    AttnArgs a;
+    memset(&a, 0, sizeof a);
+    a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
+    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
+    a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
+    K_TRY(attn_bwd(a, st));
+  }
+  // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
+  if (b->g_active[GQKV]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GQKV], st));
+  {
+    GemmArgs a = gemm_base(s);
+    a.M = T; a.N = D.d; a.K = D.Nqkv; a.b_mn_major = 1;
+    a.A = sc.dqkv; a.lda = D.Nqkv; a.B = W.wqkv; a.ldb = D.d;
+    if (b->g_active[GQKV]) {
+      a.R = b->R_used[GQKV]; a.A2 = sc.dU[GQKV]; a.lda2 = a.R; a.B2 = s->Acat[GQKV][l]; a.ldb2 = D.ldK_g[GQKV];
+      a.mtile_extra = b->d_mtile[GQKV];
+    }
+    a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
+    K_TRY(gemm_run(a, st));
+  }
+  if (b->g_active[GQKV]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GQKV], st));
+  K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dh, dx, T, D.d, st));
+  return MENOS_OK;
+}
+
+// full SAVE forward over all layers: X[0] = b->L[0].x (already filled), output -> xout
+static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, bf16* xout, cudaStream_t st) {
+  for (int l = 0; l < s->n_layers; ++l) {
+    bf16* y = (l + 1 < s->n_layers) ? b->L[l + 1].x : xout;
+    int rc = layer_forward(s, b, l, b->L[l].x, y, b->L[l], true, st);
+    if (rc) return rc;
+  }
+  return MENOS_OK;
+}
+
+// =====================================================================================================
+// C-ABI: forward / backward
+// =====================================================================================================
+extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_client, const int32_t* seq_len,
+                             const void* x_c, void* x_s, int flags, void* stream, menos_batch** batch) {
+  if (!s || !batch || n_seqs <= 0 || !seq_client || !seq_len || !x_c || !x_s) FAIL(MENOS_EINVAL, "bad arguments");
+  if (flags != MENOS_FWD_SAVE && flags != MENOS_FWD_NOGRAD) FAIL(MENOS_EINVAL, "bad flags %d", flags);
+  *batch = nullptr;
+  for (int l = 0; l < s->n_layers; ++l) if (!s->loaded[l]) FAIL(MENOS_ESTATE, "layer %d weights not loaded", l);
+  CUDA_TRY(cudaSetDevice(s->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  std::unique_ptr<menos_batch> b;
+  int rc = build_batch(s, n_seqs, seq_client, seq_len, flags == MENOS_FWD_NOGRAD, b);
+  if (rc) return rc;
+  const Dims& D = s->D;
+  const int T = b->T;
+  Scratch sc;
+  rc = get_scratch(s, T, b->R_used, sc);
+  if (rc) return rc;
+  LayerSave ng{};
+  if (b->nograd) nograd_layer(s, T, b->R_used, sc, ng);
+  rc = finalize_batch(s, b.get(), sc, &ng, st);
+  if (rc) return rc;
+  auto fail_free = [&](int code) {
+    if (b->slab) s->arena.release(b->slab);
+    if (b->meta) s->arena.release(b->meta);
+    return code;
+  };
+  if (cudaMemcpyAsync(b->L[0].x, x_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
+    set_err("copy of x_c failed");
+    return fail_free(MENOS_ECUDA);
+  }
+  if (!b->nograd) {
+    rc = forward_save(s, b.get(), sc, sc.xout, st);
+    if (rc) return fail_free(rc);
+  } else {
+    // Alg.1 L6: forward without caching activations; only x_c is kept
+    const bf16* x = b->L[0].x;
+    for (int l = 0; l < s->n_layers; ++l) {
+      bf16* y = ((s->n_layers - 1 - l) % 2 == 0) ? sc.xout : sc.dx;
+      rc = layer_forward(s, b.get(), l, x, y, ng, true, st);
+      if (rc) return fail_free(rc);
+      x = y;
+    }
+  }
+  if (cudaMemcpyAsync(x_s, sc.xout, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
+    set_err("copy of x_s failed");
+    return fail_free(MENOS_ECUDA);
+  }
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, x_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&
+      pa.type != cudaMemoryTypeManaged)
+    CUDA_TRY(cudaStreamSynchronize(st));
+  cudaGetLastError();
+  *batch = b.release();
+  return MENOS_OK;
+}
+
+extern "C" int menos_batch_free(menos_server* s, menos_batch* b) {
+  if (!s || !b) FAIL(MENOS_EINVAL, "null argument");
+  if (b->slab) s->arena.release(b->slab);
+  if (b->meta) s->arena.release(b->meta);
+  delete b;
+  return MENOS_OK;
+}
+
+extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, void* g_s, void* stream) {
+  if (!s || !b || !g_c || !g_s) FAIL(MENOS_EINVAL, "bad arguments");
+  for (int c : b->bclients) if (!s->clients[c].used) FAIL(MENOS_ESTATE, "client %d unregistered since forward", c);
+  CUDA_TRY(cudaSetDevice(s->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  const Dims& D = s->D;
+  const int T = b->T;
+  Scratch sc;
+  int rc = get_scratch(s, T, b->R_used, sc);
+  if (rc) return rc;
+  if (b->nograd) {
+    // Alg.1 L10: re-forward with gradient preparation from the cached x_c; the SAVE slab is
+    // allocated only now (on-demand allocation)
+    bf16* xc = b->L[0].x;
+    uint8_t* old_slab = b->slab;
+    uint8_t* old_meta = b->meta;
+    b->slab = nullptr; b->meta = nullptr;
+    b->nograd = false;
+    rc = finalize_batch(s, b, sc, nullptr, st);
+    if (rc) { b->nograd = true; b->slab = old_slab; b->meta = old_meta; return rc; }
+    CUDA_TRY(cudaMemcpyAsync(b->L[0].x, xc, (size_t)T * D.d * 2, cudaMemcpyDeviceToDevice, st));
+    s->arena.release(old_meta);   // stream-ordered reuse: later users run after these copies
+    s->arena.release(old_slab);
+    rc = forward_save(s, b, sc, sc.xout, st);
+    if (rc) return rc;
+  }
+  CUDA_TRY(cudaMemcpyAsync(sc.dy, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  // the block-diagonal dU scratch: zero once (a batch's slot positions are the same in every layer)
+  for (int g = 0; g < NG; ++g)
+    if (b->g_active[g]) CUDA_TRY(cudaMemsetAsync(sc.dU[g], 0, (size_t)T * b->R_used[g] * 2, st));
+  bf16* dy = sc.dy;
+  bf16* dx = sc.dx;
+  for (int l = s->n_layers - 1; l >= 0; --l) {
+    rc = layer_backward(s, b, l, dy, dx, sc, st);
+    if (rc) return rc;
+    std::swap(dy, dx);
+  }
+  CUDA_TRY(cudaMemcpyAsync(g_s, dy, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, g_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&
+      pa.type != cudaMemoryTypeManaged)
+    CUDA_TRY(cudaStreamSynchronize(st));
+  cudaGetLastError();
+  // Release I after the backward (Fig.3(b); Alg.1 L13): the slab returns to the arena; stream
+  // order guarantees later users run after this backward's kernels.
+  return menos_batch_free(s, b);
+}

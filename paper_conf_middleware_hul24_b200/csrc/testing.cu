@@ -1,0 +1,109 @@
+// Kernel-level test entry points (include/menos_testing.h): same kernels as the server path.
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/menos.h"
+#include "../../include/menos_testing.h"
+#include "kernels.h"
+
+using namespace menos;
+
+namespace {
+thread_local std::string t_err;
+int fail(const char* m) { t_err = m; return MENOS_ECUDA; }
+}  // namespace
+
+extern "C" const char* menos_testing_last_error(void) { return t_err.c_str(); }
+
+extern "C" int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int lda, const void* B, int ldb,
+                               const void* A2, int lda2, const void* B2, int ldb2, int R, const int32_t* mtile_extra,
+                               int epi, void* out, int ldo, const void* resid, int ldr, void* out2, int ldo2,
+                               const void* aux, int ldaux, int head_dim, int rope_cols, const int32_t* pos,
+                               float theta, int num_sms) {
+  GemmArgs a;
+  memset(&a, 0, sizeof a);
+  a.M = M; a.N = N; a.K = K; a.b_mn_major = b_mn;
+  a.A = (const bf16*)A; a.lda = lda; a.B = (const bf16*)B; a.ldb = ldb;
+  a.A2 = (const bf16*)A2; a.lda2 = lda2; a.B2 = (const bf16*)B2; a.ldb2 = ldb2; a.R = R;
+  a.epi = epi; a.out = (bf16*)out; a.ldo = ldo; a.resid = (const bf16*)resid; a.ldr = ldr;
+  a.out2 = (bf16*)out2; a.ldo2 = ldo2; a.aux = (const bf16*)aux; a.ldaux = ldaux;
+  a.head_dim = head_dim; a.rope_cols = rope_cols;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  a.num_sms = num_sms > 0 ? num_sms : sms;
+  const int n_mt = (M + 127) / 128;
+  int2* d_mt = nullptr; int* d_pos = nullptr; float2* d_cs = nullptr;
+  if (R > 0) {
+    if (cudaMalloc(&d_mt, n_mt * sizeof(int2)) != cudaSuccess) return fail("alloc");
+    cudaMemcpy(d_mt, mtile_extra, n_mt * sizeof(int2), cudaMemcpyHostToDevice);
+    a.mtile_extra = d_mt;
+  }
+  if (epi == EPI_ROPE) {
+    int maxp = 1;
+    for (int i = 0; i < M; ++i) maxp = std::max(maxp, pos[i] + 1);
+    cudaMalloc(&d_pos, M * sizeof(int));
+    cudaMemcpy(d_pos, pos, M * sizeof(int), cudaMemcpyHostToDevice);
+    cudaMalloc(&d_cs, (size_t)maxp * (head_dim / 2) * sizeof(float2));
+    fill_rope_table(d_cs, maxp, head_dim, theta, 0);
+    a.pos = d_pos; a.rope_cs = d_cs;
+  }
+  int rc = gemm_run(a, 0);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (d_mt) cudaFree(d_mt);
+  if (d_pos) cudaFree(d_pos);
+  if (d_cs) cudaFree(d_cs);
+  if (rc != 0) return fail("gemm_run rejected the arguments");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  return MENOS_OK;
+}
+
+extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, int Hkv, int hd, const void* qkv,
+                                    void* O, float* lse, const void* dO, void* dqkv, float theta) {
+  std::vector<int> cu(1, 0);
+  std::vector<int2> blocks;
+  int maxL = 1;
+  for (int i = 0; i < n_seqs; ++i) {
+    for (int q = 0; q < seq_len[i]; q += 64) blocks.push_back(make_int2(i, q));
+    cu.push_back(cu.back() + seq_len[i]);
+    maxL = std::max(maxL, seq_len[i]);
+  }
+  const int T = cu.back();
+  int* d_cu; int2* d_blk; float2* d_cs; float* d_D;
+  cudaMalloc(&d_cu, cu.size() * 4);
+  cudaMalloc(&d_blk, std::max<size_t>(1, blocks.size()) * sizeof(int2));
+  cudaMalloc(&d_cs, (size_t)maxL * (hd / 2) * sizeof(float2));
+  cudaMalloc(&d_D, (size_t)H * T * 4);
+  cudaMemcpy(d_cu, cu.data(), cu.size() * 4, cudaMemcpyHostToDevice);
+  cudaMemcpy(d_blk, blocks.data(), blocks.size() * sizeof(int2), cudaMemcpyHostToDevice);
+  fill_rope_table(d_cs, maxL, hd, theta, 0);
+  AttnArgs a;
+  memset(&a, 0, sizeof a);
+  const int Nqkv = (H + 2 * Hkv) * hd;
+  a.qkv = (const bf16*)qkv; a.ld_qkv = Nqkv; a.O = (bf16*)O; a.ld_o = H * hd; a.lse = lse;
+  a.cu_seqlens = d_cu; a.qblocks = d_blk; a.n_qblocks = (int)blocks.size(); a.kvblocks = d_blk;
+  a.n_kvblocks = (int)blocks.size(); a.T = T; a.H = H; a.Hkv = Hkv; a.hd = hd; a.scale = 1.f / std::sqrt((float)hd);
+  int rc = attn_fwd(a, 0);
+  if (rc == 0 && dO) {
+    attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
+    a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
+    rc = attn_bwd(a, 0);
+  }
+  cudaError_t e = cudaDeviceSynchronize();
+  cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D);
+  if (rc != 0) return fail("attention launch rejected");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  return MENOS_OK;
+}
+
+extern "C" int menos_test_rmsnorm(int T, int d, const void* x, const float* g, float eps, void* y, float* rstd,
+                                  const void* dy, const void* resid, void* dx) {
+  int rc = rmsnorm_fwd((const bf16*)x, g, (bf16*)y, rstd, T, d, eps, 0);
+  if (rc == 0 && dy) rc = rmsnorm_bwd((const bf16*)dy, (const bf16*)x, g, rstd, (const bf16*)resid, (bf16*)dx, T, d, 0);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (rc != 0) return fail("rmsnorm launch rejected");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  return MENOS_OK;
+}

@@ -1,0 +1,242 @@
+"""Thin ctypes binding of libmenos.so (include/menos.h) -- argument marshalling only.
+
+Every step of the Menos server path runs in the library's sm_100a kernels.  There is no Python or CPU
+fallback: if the shared library is missing or no sm_100 GPU is present, the calls raise.
+Buffers may be torch tensors (device or pinned host), numpy arrays (host) or raw integer addresses.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "_lib", "libmenos.so")
+
+TARGET_BITS = {"q": 1, "k": 2, "v": 4, "o": 8, "gate": 16, "up": 32, "down": 64}
+TARGET_INDEX = {"q": 0, "k": 1, "v": 2, "o": 3, "gate": 4, "up": 5, "down": 6}
+FWD_SAVE, FWD_NOGRAD = 0, 1
+WHICH = {"A": 0, "B": 1, "dA": 2, "dB": 3, "mA": 4, "mB": 5, "vA": 6, "vB": 7}
+STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ENOCLIENT", -4: "ESTATE", -5: "ECUDA", -6: "ENCCL"}
+
+
+class MenosError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"menos {STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+class ModelCfg(C.Structure):
+    _fields_ = [("d_model", C.c_int), ("n_heads", C.c_int), ("n_kv_heads", C.c_int), ("d_ff", C.c_int),
+                ("rms_eps", C.c_float), ("rope_theta", C.c_float)]
+
+
+class LayerWeights(C.Structure):
+    _fields_ = [(n, C.c_void_p) for n in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")]
+
+
+class AdamWCfg(C.Structure):
+    _fields_ = [("lr", C.c_float), ("beta1", C.c_float), ("beta2", C.c_float), ("eps", C.c_float),
+                ("weight_decay", C.c_float)]
+
+
+class ServerOpts(C.Structure):
+    _fields_ = [("max_clients", C.c_int), ("max_rank", C.c_int), ("max_seq_len", C.c_int),
+                ("arena_bytes", C.c_size_t), ("num_sms", C.c_int)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("base_bytes", C.c_size_t), ("adapters_bytes", C.c_size_t), ("arena_bytes", C.c_size_t),
+                ("arena_used", C.c_size_t), ("arena_peak", C.c_size_t), ("n_clients", C.c_int),
+                ("num_sms", C.c_int)]
+
+
+_lib = None
+
+# (name, restype, argtypes) for every symbol include/menos.h and include/menos_testing.h declare
+_P, _I, _F, _S = C.c_void_p, C.c_int, C.c_float, C.c_size_t
+_PI32 = C.POINTER(C.c_int32)
+SIGNATURES = {
+    "menos_server_create": (_I, [C.POINTER(ModelCfg), _I, _I, C.POINTER(LayerWeights), _I, C.POINTER(ServerOpts),
+                                 C.POINTER(_P)]),
+    "menos_server_load_layer": (_I, [_P, _I, C.POINTER(LayerWeights)]),
+    "menos_server_destroy": (None, [_P]),
+    "menos_register_client": (_I, [_P, _I, _F, C.c_uint32, C.POINTER(AdamWCfg), C.c_uint64, _PI32]),
+    "menos_unregister_client": (_I, [_P, C.c_int32]),
+    "menos_client_memory": (_I, [_P, C.c_int32, _I, C.POINTER(_S), C.POINTER(_S), C.POINTER(_S)]),
+    "menos_forward": (_I, [_P, _I, _PI32, _PI32, _P, _P, _I, _P, C.POINTER(_P)]),
+    "menos_backward": (_I, [_P, _P, _P, _P, _P]),
+    "menos_batch_free": (_I, [_P, _P]),
+    "menos_adapter_step": (_I, [_P, _I, _PI32, _P]),
+    "menos_adapter_shape": (_I, [_P, C.c_int32, _I, C.POINTER(_I), C.POINTER(_I)]),
+    "menos_get_adapter": (_I, [_P, C.c_int32, _I, _I, _I, C.POINTER(C.c_float)]),
+    "menos_set_adapter": (_I, [_P, C.c_int32, _I, _I, _I, C.POINTER(C.c_float)]),
+    "menos_get_stats": (_I, [_P, C.POINTER(Stats)]),
+    "menos_launch_count": (C.c_ulonglong, []),
+    "menos_sync": (_I, [_P]),
+    "menos_last_error": (C.c_char_p, []),
+    "menos_test_gemm": (_I, [_I, _I, _I, _I, _P, _I, _P, _I, _P, _I, _P, _I, _I, _PI32, _I, _P, _I, _P, _I, _P, _I,
+                             _P, _I, _I, _I, _PI32, _F, _I]),
+    "menos_test_attention": (_I, [_I, _PI32, _I, _I, _I, _P, _P, _P, _P, _P, _F]),
+    "menos_test_rmsnorm": (_I, [_I, _I, _P, _P, _F, _P, _P, _P, _P, _P]),
+    "menos_testing_last_error": (C.c_char_p, []),
+}
+
+
+def lib():
+    """Load libmenos.so (built in-tree by build.py / __graft_entry__.build()).  Raises if absent."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise FileNotFoundError(f"{LIB_PATH} not built: run __graft_entry__.build() (no CPU fallback exists)")
+        L = C.CDLL(LIB_PATH)
+        for name, (res, args) in SIGNATURES.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+def ptr(x) -> int | None:
+    """Address of a torch tensor / numpy array / int (None for None)."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if hasattr(x, "ctypes"):
+        return x.ctypes.data
+    raise TypeError(type(x))
+
+
+def check(rc: int, testing: bool = False):
+    if rc != 0:
+        msg = (lib().menos_testing_last_error() if testing else lib().menos_last_error()) or b""
+        raise MenosError(rc, msg.decode(errors="replace"))
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        return None
+    if hasattr(stream, "cuda_stream"):
+        return stream.cuda_stream
+    return int(stream)
+
+
+def _i32(seq):
+    arr = (C.c_int32 * len(seq))(*[int(v) for v in seq])
+    return arr
+
+
+class Batch:
+    def __init__(self, server: "Server", handle: int, n_tokens: int):
+        self.server, self.handle, self.n_tokens = server, handle, n_tokens
+
+
+class Server:
+    """One Menos server segment on one GPU: menos_server_create ... menos_server_destroy."""
+
+    def __init__(self, d_model, n_heads, n_kv_heads, d_ff, n_layers, first_layer=1, rms_eps=1e-5,
+                 rope_theta=1e4, weights=None, device=0, max_clients=64, max_rank=64, max_seq_len=4096,
+                 arena_bytes=0, num_sms=0):
+        self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta)
+        self.n_layers = n_layers
+        opts = ServerOpts(max_clients, max_rank, max_seq_len, arena_bytes, num_sms)
+        h = C.c_void_p()
+        warr = None
+        if weights is not None:
+            warr = (LayerWeights * n_layers)(*[self._lw(w) for w in weights])
+        check(lib().menos_server_create(C.byref(self.cfg), first_layer, n_layers, warr, device, C.byref(opts),
+                                        C.byref(h)))
+        self.h = h.value
+
+    @staticmethod
+    def _lw(w: dict) -> LayerWeights:
+        return LayerWeights(*[ptr(w[k]) for k in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")])
+
+    def load_layer(self, layer: int, w: dict):
+        lw = self._lw(w)
+        check(lib().menos_server_load_layer(self.h, layer, C.byref(lw)))
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().menos_server_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---------------------------------------------------------------- clients
+    def register_client(self, rank, alpha, targets=("q", "v"), lr=1e-4, betas=(0.9, 0.999), eps=1e-8,
+                        weight_decay=0.01, seed=0) -> int:
+        mask = 0
+        for t in targets:
+            mask |= TARGET_BITS[t]
+        opt = AdamWCfg(lr, betas[0], betas[1], eps, weight_decay)
+        cid = C.c_int32()
+        check(lib().menos_register_client(self.h, rank, alpha, mask, C.byref(opt), seed, C.byref(cid)))
+        return cid.value
+
+    def unregister_client(self, cid: int):
+        check(lib().menos_unregister_client(self.h, cid))
+
+    def client_memory(self, cid: int, n_tokens: int):
+        a, b, c = C.c_size_t(), C.c_size_t(), C.c_size_t()
+        check(lib().menos_client_memory(self.h, cid, n_tokens, C.byref(a), C.byref(b), C.byref(c)))
+        return a.value, b.value, c.value
+
+    def adapter_shape(self, cid: int, target: str):
+        r = (C.c_int * 2)()
+        c = (C.c_int * 2)()
+        check(lib().menos_adapter_shape(self.h, cid, TARGET_INDEX[target], r, c))
+        return (r[0], c[0]), (r[1], c[1])
+
+    def get_adapter(self, cid: int, layer: int, target: str, which: str):
+        import numpy as np
+        (ra, ca), (rb, cb) = self.adapter_shape(cid, target)
+        shape = (ra, ca) if WHICH[which] % 2 == 0 else (rb, cb)
+        out = np.empty(shape, np.float32)
+        check(lib().menos_get_adapter(self.h, cid, layer, TARGET_INDEX[target], WHICH[which],
+                                      out.ctypes.data_as(C.POINTER(C.c_float))))
+        return out
+
+    def set_adapter(self, cid: int, layer: int, target: str, which: str, value):
+        import numpy as np
+        v = np.ascontiguousarray(value, dtype=np.float32)
+        check(lib().menos_set_adapter(self.h, cid, layer, TARGET_INDEX[target], WHICH[which],
+                                      v.ctypes.data_as(C.POINTER(C.c_float))))
+
+    # ---------------------------------------------------------------- the hot path
+    def forward(self, seq_client, seq_len, x_c, x_s, flags=FWD_SAVE, stream=None) -> Batch:
+        b = C.c_void_p()
+        check(lib().menos_forward(self.h, len(seq_client), _i32(seq_client), _i32(seq_len), ptr(x_c), ptr(x_s),
+                                  flags, _stream(stream), C.byref(b)))
+        return Batch(self, b.value, int(sum(seq_len)))
+
+    def backward(self, batch: Batch, g_c, g_s, stream=None):
+        check(lib().menos_backward(self.h, batch.handle, ptr(g_c), ptr(g_s), _stream(stream)))
+        batch.handle = None
+
+    def batch_free(self, batch: Batch):
+        if batch.handle:
+            check(lib().menos_batch_free(self.h, batch.handle))
+            batch.handle = None
+
+    def adapter_step(self, client_ids, stream=None):
+        check(lib().menos_adapter_step(self.h, len(client_ids), _i32(client_ids), _stream(stream)))
+
+    def stats(self) -> dict:
+        s = Stats()
+        check(lib().menos_get_stats(self.h, C.byref(s)))
+        return {k: getattr(s, k) for k, _ in Stats._fields_}
+
+    def sync(self):
+        check(lib().menos_sync(self.h))
+
+
+def launch_count() -> int:
+    return int(lib().menos_launch_count())

@@ -1,0 +1,146 @@
+"""Helpers shared by the GPU parity tests, smoke() and bench.py's parity spot check.
+
+run_gpu_step  : drives libmenos.so through its C-ABI (paper_conf_middleware_hul24_b200.Server).
+run_oracle_step: the CPU oracle (oracle/menos_oracle.py) on the same seeded inputs.
+compare_step  : BASELINE.json north_star bars -- activations max|d|/max|ref| <= 2e-2, every gradient tensor
+                cosine >= 0.999 (DESIGN.md §"Tolerances").
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from workloads import TARGETS, Workload, base_layer_weights, client_adapters, client_inputs
+
+ACT_TOL = 2e-2
+COS_TOL = 0.999
+
+
+def _bf16(a, device="cpu"):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(torch.bfloat16).to(device).contiguous()
+
+
+def make_inputs(w: Workload, seed: int = 0, zero_b: bool = False, outlier: bool = False):
+    m = w.model
+    weights = [base_layer_weights(m, l, seed=seed) for l in range(m.n_layers)]
+    adapters = [client_adapters(m, c, seed=1000 + 17 * seed + i, zero_b=zero_b) for i, c in enumerate(w.clients)]
+    io = [client_inputs(m, c, seed=2000 + 17 * seed + i, outlier=outlier) for i, c in enumerate(w.clients)]
+    return weights, adapters, io
+
+
+def new_server(w: Workload, weights, arena_bytes=0, max_rank=16, device="cuda:0"):
+    import torch
+    from paper_conf_middleware_hul24_b200 import Server
+    m = w.model
+    wl = []
+    for W in weights:
+        wl.append({k: _bf16(W[k]) for k in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")})
+    names = {"wq": "wq", "wk": "wk", "wv": "wv", "wo": "wo", "wgate": "wgate", "wup": "wup", "wdown": "wdown"}
+    del names
+    max_seq = max(max(c.seq_lens) for c in w.clients)
+    srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
+                 rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=wl, max_rank=max_rank,
+                 max_seq_len=max(max_seq, 64), arena_bytes=arena_bytes)
+    return srv
+
+
+def register(srv, w: Workload, adapters, seed=0):
+    ids = []
+    for i, c in enumerate(w.clients):
+        cid = srv.register_client(c.rank, c.alpha, c.targets, seed=seed + i)
+        for l, d in enumerate(adapters[i]):
+            for t, (A, B) in d.items():
+                srv.set_adapter(cid, l, t, "A", A)
+                srv.set_adapter(cid, l, t, "B", B)
+        ids.append(cid)
+    return ids
+
+
+def run_gpu_step(w: Workload, seed: int = 0, zero_b: bool = False, flags: int = 0, inputs=None, srv=None,
+                 ids=None, keep=False, grads=True):
+    """One forward + backward of the whole batch on cuda:0.  Returns per-client x_s, g_s and adapter grads."""
+    import torch
+    m = w.model
+    weights, adapters, io = inputs if inputs is not None else make_inputs(w, seed, zero_b)
+    own = srv is None
+    if own:
+        srv = new_server(w, weights)
+        ids = register(srv, w, adapters)
+    seq_client, seq_len = [], []
+    for i, c in enumerate(w.clients):
+        seq_client += [ids[i]] * len(c.seq_lens)
+        seq_len += list(c.seq_lens)
+    x = _bf16(np.concatenate([a for a, _ in io]), "cuda")
+    g = _bf16(np.concatenate([b for _, b in io]), "cuda")
+    xs = torch.empty_like(x)
+    gs = torch.empty_like(x)
+    b = srv.forward(seq_client, seq_len, x, xs, flags=flags)
+    srv.backward(b, g, gs)
+    torch.cuda.synchronize()
+    out = {"x_s": [], "g_s": [], "grads": []}
+    off = 0
+    xs_h, gs_h = xs.float().cpu().numpy(), gs.float().cpu().numpy()
+    for i, c in enumerate(w.clients):
+        T = c.n_tokens
+        out["x_s"].append(xs_h[off:off + T])
+        out["g_s"].append(gs_h[off:off + T])
+        off += T
+        gr = []
+        if grads:
+            for l in range(m.n_layers):
+                gr.append({t: (srv.get_adapter(ids[i], l, t, "dA"), srv.get_adapter(ids[i], l, t, "dB"))
+                           for t in c.targets})
+        out["grads"].append(gr)
+    if keep:
+        out["server"], out["ids"] = srv, ids
+    elif own:
+        srv.close()
+    return out
+
+
+def run_oracle_step(w: Workload, seed: int = 0, zero_b: bool = False, inputs=None, clients=None):
+    from oracle import menos_oracle as O
+    m = w.model
+    weights, adapters, io = inputs if inputs is not None else make_inputs(w, seed, zero_b)
+    out = {"x_s": [], "g_s": [], "grads": []}
+    for i, c in enumerate(w.clients):
+        if clients is not None and i not in clients:
+            out["x_s"].append(None); out["g_s"].append(None); out["grads"].append(None)
+            continue
+        xs, gs, gr = O.client_step(io[i][0], io[i][1], c.seq_lens, weights, adapters[i], c.alpha / c.rank, m)
+        out["x_s"].append(xs)
+        out["g_s"].append(gs)
+        out["grads"].append(gr)
+    return out
+
+
+def act_err(a, ref):
+    return float(np.max(np.abs(a - ref)) / max(np.max(np.abs(ref)), 1e-30))
+
+
+def cosine(a, ref):
+    a = np.asarray(a, np.float64).ravel()
+    b = np.asarray(ref, np.float64).ravel()
+    na, nb = np.linalg.norm(a), np.linalg.norm(b)
+    if na < 1e-30 and nb < 1e-30:
+        return 1.0
+    return float(a @ b / max(na * nb, 1e-300))
+
+
+def compare_step(gpu, ora, clients=None):
+    rep = {}
+    n = len(gpu["x_s"])
+    for i in range(n):
+        if clients is not None and i not in clients:
+            continue
+        e = act_err(gpu["x_s"][i], ora["x_s"][i])
+        rep[f"c{i}.x_s"] = {"metric": e, "ok": e <= ACT_TOL, "kind": "maxrel"}
+        cg = cosine(gpu["g_s"][i], ora["g_s"][i])
+        rep[f"c{i}.g_s"] = {"metric": cg, "ok": cg >= COS_TOL, "kind": "cos"}
+        for l, d in enumerate(gpu["grads"][i]):
+            for t, (dA, dB) in d.items():
+                oA, oB = ora["grads"][i][l][t]
+                ca, cb = cosine(dA, oA), cosine(dB, oB)
+                rep[f"c{i}.L{l}.{t}.dA"] = {"metric": ca, "ok": ca >= COS_TOL, "kind": "cos"}
+                rep[f"c{i}.L{l}.{t}.dB"] = {"metric": cb, "ok": cb >= COS_TOL, "kind": "cos"}
+    return rep

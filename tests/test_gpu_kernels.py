@@ -1,0 +1,278 @@
+"""Kernel-level GPU parity (include/menos_testing.h entry points) against oracle sub-functions.
+
+Inputs are seeded and bf16-representable; the oracle computes in fp32 from the same values.  Sizes span
+several 128x256 GEMM tiles, ragged M/N/K tails, and the persistent loop (more tiles than SMs).
+"""
+import ctypes as C
+
+import numpy as np
+import pytest
+
+from oracle import menos_oracle as O
+from workloads import bf16_round
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+def lib():
+    from paper_conf_middleware_hul24_b200.menos import lib as L
+    return L()
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float32)).to(torch.bfloat16).cuda().contiguous()
+
+
+def host(t):
+    return t.float().cpu().numpy()
+
+
+def rnd(shape, seed, scale=1.0):
+    return bf16_round(np.random.default_rng(seed).standard_normal(shape).astype(np.float32) * np.float32(scale))
+
+
+def maxrel(a, b):
+    return float(np.max(np.abs(a - b)) / max(np.max(np.abs(b)), 1e-30))
+
+
+def i32(lst):
+    return (C.c_int32 * len(lst))(*lst)
+
+
+def gemm(M, N, K, b_mn, A, B, A2=None, B2=None, R=0, mt=None, epi=0, out=None, resid=None, out2=None, aux=None,
+         hd=0, rope_cols=0, pos=None, theta=1e4, num_sms=0, ldo=None, ldo2=0, ldaux=0):
+    from paper_conf_middleware_hul24_b200.menos import check
+    p = lambda t: None if t is None else t.data_ptr()
+    rc = lib().menos_test_gemm(M, N, K, b_mn, p(A), A.shape[1], p(B), B.shape[1], p(A2),
+                               A2.shape[1] if A2 is not None else 0, p(B2), B2.shape[1] if B2 is not None else 0,
+                               R, i32(mt) if mt is not None else None, epi, p(out), ldo or out.shape[1], p(resid),
+                               resid.shape[1] if resid is not None else 0, p(out2), ldo2, p(aux), ldaux, hd,
+                               rope_cols, i32(pos) if pos is not None else None, theta, num_sms)
+    check(rc, testing=True)
+
+
+@pytest.mark.parametrize("M,N,K", [(128, 256, 64), (300, 512, 320), (1000, 768, 1000), (2048, 4096, 4096)])
+def test_gemm_fwd_kmajor(M, N, K):
+    x, W = rnd((M, K), 1), rnd((N, K), 2, 0.02)
+    out = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    gemm(M, N, K, 0, dev(x), dev(W), out=out)
+    ref, _ = O.proj_fwd(x, W, None, 1.0)
+    assert maxrel(host(out), ref) < 1e-2
+
+
+@pytest.mark.parametrize("M,Nred,Kout", [(256, 384, 512), (333, 640, 320), (2048, 11008, 4096)])
+def test_gemm_dx_mnmajor(M, Nred, Kout):
+    dy, W = rnd((M, Nred), 3), rnd((Nred, Kout), 4, 0.02)
+    out = torch.empty(M, Kout, dtype=torch.bfloat16, device="cuda")
+    gemm(M, Kout, Nred, 1, dev(dy), dev(W), out=out)
+    ref = dy @ W                                              # dx = dy W (oracle proj_bwd without LoRA)
+    ref2, _ = O.proj_bwd(dy, np.zeros((M, Kout), np.float32), W, None, 1.0, None)
+    np.testing.assert_allclose(ref, ref2, rtol=1e-5, atol=1e-5)
+    assert maxrel(host(out), ref2) < 1e-2
+
+
+def test_gemm_persistent_many_tiles_small_grid():
+    M, N, K = 1024, 1024, 256
+    x, W = rnd((M, K), 5), rnd((N, K), 6, 0.05)
+    out = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    gemm(M, N, K, 0, dev(x), dev(W), out=out, num_sms=3)     # 32 tiles on 3 CTAs: TMEM double buffer wraps
+    ref, _ = O.proj_fwd(x, W, None, 1.0)
+    assert maxrel(host(out), ref) < 1e-2
+
+
+def _lora_case(seed, Ks, Ns, clients):
+    """clients: list of (T_c, r, s).  Returns x, W, per-client A/B, block-diag U_cat (s*U, bf16) and Bcat."""
+    rng = np.random.default_rng(seed)
+    T = sum(c[0] for c in clients)
+    x = rnd((T, Ks), seed)
+    W = rnd((Ns, Ks), seed + 1, 0.02)
+    As, Bs, offs = [], [], []
+    off = 0
+    for (Tc, r, s) in clients:
+        As.append(bf16_round(rng.uniform(-1 / np.sqrt(Ks), 1 / np.sqrt(Ks), (r, Ks)).astype(np.float32)))
+        Bs.append(bf16_round(rng.standard_normal((Ns, r)).astype(np.float32) * 0.02))
+        offs.append(off)
+        off += 16 * ((r + 15) // 16)
+    R = ((off + 63) // 64) * 64
+    Ucat = np.zeros((T, R), np.float32)
+    Bcat = np.zeros((Ns, R), np.float32)
+    Acat = np.zeros((R, Ks), np.float32)
+    t0 = 0
+    rows_client = []
+    for i, (Tc, r, s) in enumerate(clients):
+        Ucat[t0:t0 + Tc, offs[i]:offs[i] + r] = bf16_round(s * (x[t0:t0 + Tc] @ As[i].T))
+        Bcat[:, offs[i]:offs[i] + r] = Bs[i]
+        Acat[offs[i]:offs[i] + r] = As[i]
+        rows_client += [i] * Tc
+        t0 += Tc
+    mt = []
+    for m in range((T + 127) // 128):
+        cs = sorted(set(rows_client[m * 128:(m + 1) * 128]))
+        lo = min(offs[c] for c in cs)
+        hi = max(offs[c] + 16 * ((clients[c][1] + 15) // 16) for c in cs)
+        mt += [lo, (hi - lo) // 16]
+    return x, W, As, Bs, Ucat, Bcat, Acat, R, mt
+
+
+def test_gemm_segmented_lora_expand_fwd():
+    clients = [(100, 8, 2.0), (200, 4, 2.0), (77, 16, 2.0)]
+    x, W, As, Bs, Ucat, Bcat, Acat, R, mt = _lora_case(11, 256, 512, clients)
+    T = x.shape[0]
+    out = torch.empty(T, 512, dtype=torch.bfloat16, device="cuda")
+    gemm(T, 512, 256, 0, dev(x), dev(W), dev(Ucat), dev(Bcat), R, mt, out=out)
+    got = host(out)
+    t0 = 0
+    for i, (Tc, r, s) in enumerate(clients):
+        ref, _ = O.proj_fwd(x[t0:t0 + Tc], W, (As[i], Bs[i]), s)
+        assert maxrel(got[t0:t0 + Tc], ref) < 1.5e-2, i
+        t0 += Tc
+
+
+def test_gemm_segmented_lora_expand_dx():
+    clients = [(130, 8, 2.0), (126, 16, 2.0)]
+    x, W, As, Bs, Ucat, Bcat, Acat, R, mt = _lora_case(12, 320, 384, clients)
+    T = x.shape[0]
+    dy = rnd((T, 384), 13)
+    # dU = s dy B (block-diagonal), then dx = dy W + dU A
+    dU = np.zeros((T, R), np.float32)
+    t0 = 0
+    offs = [0, 16]
+    for i, (Tc, r, s) in enumerate(clients):
+        dU[t0:t0 + Tc, offs[i]:offs[i] + r] = bf16_round(s * (dy[t0:t0 + Tc] @ Bs[i]))
+        t0 += Tc
+    out = torch.empty(T, 320, dtype=torch.bfloat16, device="cuda")
+    gemm(T, 320, 384, 1, dev(dy), dev(W), dev(dU), dev(Acat), R, mt, out=out)
+    got = host(out)
+    t0 = 0
+    for i, (Tc, r, s) in enumerate(clients):
+        U = x[t0:t0 + Tc] @ As[i].T
+        ref, _ = O.proj_bwd(dy[t0:t0 + Tc], x[t0:t0 + Tc], W, (As[i], Bs[i]), s, U)
+        assert maxrel(got[t0:t0 + Tc], ref) < 1.5e-2, i
+        t0 += Tc
+
+
+def test_gemm_zero_b_is_bitwise_base():
+    clients = [(150, 8, 2.0), (106, 8, 2.0)]
+    x, W, As, Bs, Ucat, Bcat, Acat, R, mt = _lora_case(14, 256, 512, clients)
+    T = x.shape[0]
+    o1 = torch.empty(T, 512, dtype=torch.bfloat16, device="cuda")
+    o2 = torch.empty_like(o1)
+    gemm(T, 512, 256, 0, dev(x), dev(W), out=o1)
+    gemm(T, 512, 256, 0, dev(x), dev(W), dev(Ucat), dev(np.zeros_like(Bcat)), R, mt, out=o2)
+    assert torch.equal(o1, o2)
+
+
+def test_gemm_resid_epilogue():
+    M, N, K = 200, 256, 128
+    x, W, r = rnd((M, K), 21), rnd((N, K), 22, 0.05), rnd((M, N), 23)
+    out = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    gemm(M, N, K, 0, dev(x), dev(W), epi=1, out=out, resid=dev(r))
+    assert maxrel(host(out), r + x @ W.T) < 1e-2
+
+
+@pytest.mark.parametrize("hd,H,Hkv", [(128, 4, 2), (16, 4, 4), (64, 2, 1)])
+def test_gemm_rope_epilogue(hd, H, Hkv):
+    lens = [5, 130, 61]
+    T, K = sum(lens), 192
+    N = (H + 2 * Hkv) * hd
+    pos = [p for L in lens for p in range(L)]
+    x, W = rnd((T, K), 31), rnd((N, K), 32, 0.05)
+    out = torch.empty(T, N, dtype=torch.bfloat16, device="cuda")
+    gemm(T, N, K, 0, dev(x), dev(W), epi=2, out=out, hd=hd, rope_cols=(H + Hkv) * hd, pos=pos)
+    y = x @ W.T
+    ref = np.empty_like(y)
+    t0 = 0
+    for L in lens:
+        cos, sin = O.rope_cos_sin(L, hd, 1e4, np.float32)
+        yy = y[t0:t0 + L]
+        q = O.rope_fwd(yy[:, :H * hd].reshape(L, H, hd), cos, sin).reshape(L, -1)
+        k = O.rope_fwd(yy[:, H * hd:(H + Hkv) * hd].reshape(L, Hkv, hd), cos, sin).reshape(L, -1)
+        ref[t0:t0 + L] = np.concatenate([q, k, yy[:, (H + Hkv) * hd:]], 1)
+        t0 += L
+    assert maxrel(host(out), ref) < 1e-2
+
+
+def test_gemm_swiglu_fwd_and_bwd_epilogues():
+    T, d, f = 260, 128, 256     # f multiple of 128; interleaved gu layout [128 gate | 128 up] per block
+    x = rnd((T, d), 41)
+    Wg, Wu = rnd((f, d), 42, 0.1), rnd((f, d), 43, 0.1)
+    Wgu = np.zeros((2 * f, d), np.float32)
+    for fb in range(f // 128):
+        Wgu[fb * 256:fb * 256 + 128] = Wg[fb * 128:(fb + 1) * 128]
+        Wgu[fb * 256 + 128:fb * 256 + 256] = Wu[fb * 128:(fb + 1) * 128]
+    gu = torch.empty(T, 2 * f, dtype=torch.bfloat16, device="cuda")
+    a = torch.empty(T, f, dtype=torch.bfloat16, device="cuda")
+    gemm(T, 2 * f, d, 0, dev(x), dev(Wgu), epi=3, out=gu, out2=a, ldo2=f)
+    gt, up = x @ Wg.T, x @ Wu.T
+    assert maxrel(host(a), O.silu(gt) * up) < 1.5e-2
+    # backward: da = dy Wd  (Wd [d_out, f]); epilogue -> dgu interleaved
+    dout = 192
+    dy, Wd = rnd((T, dout), 44), rnd((dout, f), 45, 0.1)
+    dgu = torch.empty(T, 2 * f, dtype=torch.bfloat16, device="cuda")
+    gemm(T, f, dout, 1, dev(dy), dev(Wd), epi=4, out=dgu, aux=gu, ldaux=2 * f, ldo=2 * f)
+    gu_h = host(gu)
+    g_b = np.concatenate([gu_h[:, fb * 256:fb * 256 + 128] for fb in range(f // 128)], 1)
+    u_b = np.concatenate([gu_h[:, fb * 256 + 128:fb * 256 + 256] for fb in range(f // 128)], 1)
+    dg, du = O.swiglu_bwd(dy @ Wd, g_b, u_b)
+    got = host(dgu)
+    got_g = np.concatenate([got[:, fb * 256:fb * 256 + 128] for fb in range(f // 128)], 1)
+    got_u = np.concatenate([got[:, fb * 256 + 128:fb * 256 + 256] for fb in range(f // 128)], 1)
+    assert maxrel(got_g, dg) < 1.5e-2
+    assert maxrel(got_u, du) < 1.5e-2
+
+
+@pytest.mark.parametrize("hd,H,Hkv,lens", [(128, 4, 2, [1, 17, 64, 129, 300]), (16, 4, 4, [16, 16, 3]),
+                                          (64, 8, 1, [200, 65])])
+def test_attention_fwd_bwd(hd, H, Hkv, lens):
+    from paper_conf_middleware_hul24_b200.menos import check
+    T = sum(lens)
+    N = (H + 2 * Hkv) * hd
+    qkv = rnd((T, N), 51)
+    dO = rnd((T, H * hd), 52)
+    qkv_d = dev(qkv)
+    O_d = torch.empty(T, H * hd, dtype=torch.bfloat16, device="cuda")
+    lse = torch.empty(H, T, dtype=torch.float32, device="cuda")
+    dqkv = torch.zeros(T, N, dtype=torch.bfloat16, device="cuda")
+    rc = lib().menos_test_attention(len(lens), i32(lens), H, Hkv, hd, qkv_d.data_ptr(), O_d.data_ptr(),
+                                    lse.data_ptr(), dev(dO).data_ptr(), dqkv.data_ptr(), 1e4)
+    check(rc, testing=True)
+    got_O, got_lse, got_d = host(O_d), lse.cpu().numpy(), host(dqkv)
+    t0 = 0
+    for L in lens:
+        q = qkv[t0:t0 + L, :H * hd].reshape(L, H, hd)
+        k = qkv[t0:t0 + L, H * hd:(H + Hkv) * hd].reshape(L, Hkv, hd)
+        v = qkv[t0:t0 + L, (H + Hkv) * hd:].reshape(L, Hkv, hd)
+        Ob, lb = O.attention_fwd(q, k, v)
+        assert maxrel(got_O[t0:t0 + L], Ob.reshape(L, -1)) < 2e-2
+        np.testing.assert_allclose(got_lse[:, t0:t0 + L], lb, rtol=2e-3, atol=2e-3)
+        # backward uses the GPU's bf16 O (as the kernel does) only through D; compare with the oracle
+        dq, dk, dv = O.attention_bwd(dO[t0:t0 + L].reshape(L, H, hd), q, k, v)
+        cos, sin = O.rope_cos_sin(L, hd, 1e4, np.float32)
+        dq, dk = O.rope_bwd(dq, cos, sin), O.rope_bwd(dk, cos, sin)
+        ref = np.concatenate([dq.reshape(L, -1), dk.reshape(L, -1), dv.reshape(L, -1)], 1)
+        g = got_d[t0:t0 + L]
+        for lo, hi in ((0, H * hd), (H * hd, (H + Hkv) * hd), ((H + Hkv) * hd, N)):
+            num = np.sum(g[:, lo:hi].astype(np.float64) * ref[:, lo:hi])
+            den = np.linalg.norm(g[:, lo:hi]) * np.linalg.norm(ref[:, lo:hi]) + 1e-30
+            assert num / den > 0.999, (L, lo)
+            assert maxrel(g[:, lo:hi], ref[:, lo:hi]) < 3e-2, (L, lo)
+        t0 += L
+
+
+@pytest.mark.parametrize("T,d", [(7, 64), (1000, 4096)])
+def test_rmsnorm_fwd_bwd(T, d):
+    from paper_conf_middleware_hul24_b200.menos import check
+    x, dy, res = rnd((T, d), 61), rnd((T, d), 62), rnd((T, d), 63)
+    g = bf16_round((1 + 0.1 * np.random.default_rng(64).standard_normal(d)).astype(np.float32))
+    gd = torch.from_numpy(g).cuda()
+    y = torch.empty(T, d, dtype=torch.bfloat16, device="cuda")
+    rstd = torch.empty(T, dtype=torch.float32, device="cuda")
+    dx = torch.empty_like(y)
+    check(lib().menos_test_rmsnorm(T, d, dev(x).data_ptr(), gd.data_ptr(), 1e-5, y.data_ptr(), rstd.data_ptr(),
+                                   dev(dy).data_ptr(), dev(res).data_ptr(), dx.data_ptr()), testing=True)
+    ry, rr = O.rmsnorm_fwd(x, g, np.float32(1e-5))
+    assert maxrel(host(y), ry) < 1e-2
+    np.testing.assert_allclose(rstd.cpu().numpy(), rr[:, 0], rtol=1e-5)
+    assert maxrel(host(dx), res + O.rmsnorm_bwd(dy, x, g, rr)) < 1e-2

@@ -1,0 +1,179 @@
+"""End-to-end GPU parity through the C-ABI (libmenos.so) against the CPU oracle, plus the invariants the
+BASELINE.json north_star names: (b) zero-B == base, (c) batched == alone, (d) the base is never modified.
+
+Bars (BASELINE.json north_star; DESIGN.md §"Tolerances"): activations max|d|/max|ref| <= 2e-2, cosine >= 0.999
+on every gradient tensor (g_s, every dA, dB).  Invariants (b), (c), re-forward (NEXT-1) are BITWISE on the GPU.
+"""
+import dataclasses
+
+import numpy as np
+import pytest
+
+from tests.parity_util import (compare_step, make_inputs, new_server, register, run_gpu_step, run_oracle_step)
+from workloads import ClientCfg, MODELS, TARGETS, Workload, workload
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+def assert_report(rep):
+    bad = {k: v for k, v in rep.items() if not v["ok"]}
+    assert not bad, bad
+
+
+def test_cfg0_tiny_parity():
+    w = workload("cfg0_tiny")
+    rep = compare_step(run_gpu_step(w, seed=0), run_oracle_step(w, seed=0))
+    assert_report(rep)
+
+
+def test_tiny_all_targets_gqa_ragged_mixed_ranks():
+    m = dataclasses.replace(MODELS["tiny"], n_heads=4, n_kv_heads=2)
+    cl = [ClientCfg(4, 8.0, TARGETS, [1, 17, 3]), ClientCfg(16, 32.0, ("q", "v"), [129]),
+          ClientCfg(8, 16.0, ("k", "o", "gate", "up", "down"), [64, 40]), ClientCfg(5, 10.0, ("v", "down"), [200])]
+    w = Workload("tiny_mix", m, cl)
+    rep = compare_step(run_gpu_step(w, seed=3), run_oracle_step(w, seed=3))
+    assert_report(rep)
+
+
+def test_zero_b_equals_base_bitwise():
+    """Invariant (b): with B = 0 the LoRA contribution is exactly zero, whatever the targets."""
+    m = MODELS["tiny"]
+    cl = [ClientCfg(4, 8.0, ("q", "v"), [20, 12]), ClientCfg(8, 16.0, TARGETS, [20, 12])]
+    w = Workload("zb", m, cl)
+    weights, adapters, io = make_inputs(w, seed=5, zero_b=True)
+    io[1] = io[0]  # same inputs for both clients
+    out = run_gpu_step(w, inputs=(weights, adapters, io), grads=False)
+    assert np.array_equal(out["x_s"][0], out["x_s"][1])
+    ora = run_oracle_step(w, inputs=(weights, [[{} for _ in range(m.n_layers)]] * 2, io))
+    from tests.parity_util import act_err
+    assert act_err(out["x_s"][0], ora["x_s"][0]) < 2e-2
+
+
+def test_batched_equals_alone_bitwise():
+    """Invariant (c): a client's outputs and grads do not depend on who shares the batch."""
+    m = MODELS["tiny"]
+    cl = [ClientCfg(4, 8.0, ("q", "v"), [50, 30]), ClientCfg(16, 32.0, ("q", "v", "o"), [100]),
+          ClientCfg(8, 16.0, ("q", "v", "down"), [7, 70])]
+    w = Workload("bva", m, cl)
+    inputs = make_inputs(w, seed=7)
+    weights, adapters, io = inputs
+    srv = new_server(w, weights)
+    ids = register(srv, w, adapters)
+    full = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids)
+    for i in range(len(cl)):
+        wi = Workload("alone", m, [cl[i]])
+        alone = run_gpu_step(wi, inputs=(weights, [adapters[i]], [io[i]]), srv=srv, ids=[ids[i]])
+        assert np.array_equal(alone["x_s"][0], full["x_s"][i]), i
+        assert np.array_equal(alone["g_s"][0], full["g_s"][i]), i
+        for l in range(m.n_layers):
+            for t in cl[i].targets:
+                assert np.array_equal(alone["grads"][0][l][t][0], full["grads"][i][l][t][0]), (i, l, t)
+                assert np.array_equal(alone["grads"][0][l][t][1], full["grads"][i][l][t][1]), (i, l, t)
+    srv.close()
+
+
+def test_base_unchanged_and_repeatable():
+    """Invariant (d): no base gradient exists; after fwd+bwd+step the same call reproduces bit-identical
+    outputs for unchanged adapters (the shared base is read-only)."""
+    w = workload("cfg0_tiny")
+    inputs = make_inputs(w, seed=9)
+    weights, adapters, io = inputs
+    srv = new_server(w, weights)
+    ids = register(srv, w, adapters)
+    a = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids, grads=False)
+    srv.adapter_step(ids)
+    register_again = [srv.set_adapter(ids[i], l, t, wh, adapters[i][l][t][0 if wh == "A" else 1])
+                      for i in range(len(ids)) for l in range(w.model.n_layers) for t in w.clients[i].targets
+                      for wh in ("A", "B")]
+    del register_again
+    b = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids, grads=False)
+    for i in range(len(ids)):
+        assert np.array_equal(a["x_s"][i], b["x_s"][i])
+        assert np.array_equal(a["g_s"][i], b["g_s"][i])
+    st = srv.stats()
+    assert st["base_bytes"] > 0
+    srv.close()
+
+
+def test_nograd_reforward_bitwise_equals_save():
+    """NEXT-1 (Alg.1 L6/L10): NOGRAD forward + re-forward backward == SAVE mode, bitwise."""
+    m = MODELS["tiny"]
+    cl = [ClientCfg(4, 8.0, ("q", "v"), [33, 31]), ClientCfg(8, 16.0, TARGETS, [64])]
+    w = Workload("ng", m, cl)
+    inputs = make_inputs(w, seed=11)
+    weights, adapters, io = inputs
+    srv = new_server(w, weights)
+    ids = register(srv, w, adapters)
+    a = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids, flags=0)
+    b = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids, flags=1)
+    for i in range(len(cl)):
+        assert np.array_equal(a["x_s"][i], b["x_s"][i])
+        assert np.array_equal(a["g_s"][i], b["g_s"][i])
+        for l in range(m.n_layers):
+            for t in cl[i].targets:
+                assert np.array_equal(a["grads"][i][l][t][0], b["grads"][i][l][t][0])
+                assert np.array_equal(a["grads"][i][l][t][1], b["grads"][i][l][t][1])
+    srv.close()
+
+
+def test_adamw_step_matches_oracle():
+    from oracle import menos_oracle as O
+    w = workload("cfg0_tiny")
+    inputs = make_inputs(w, seed=13)
+    weights, adapters, io = inputs
+    srv = new_server(w, weights)
+    ids = register(srv, w, adapters)
+    for step in range(1, 3):
+        got = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids)
+        before = {(i, l, t, wh): srv.get_adapter(ids[i], l, t, wh)
+                  for i in range(len(ids)) for l in range(w.model.n_layers) for t in w.clients[i].targets
+                  for wh in ("A", "B", "mA", "mB", "vA", "vB")}
+        srv.adapter_step(ids)
+        torch.cuda.synchronize()
+        for i in range(len(ids)):
+            for l in range(w.model.n_layers):
+                for t in w.clients[i].targets:
+                    for wh, gi in (("A", 0), ("B", 1)):
+                        g = got["grads"][i][l][t][gi]
+                        p, m_, v_ = O.adamw_step(before[(i, l, t, wh)], g, before[(i, l, t, "m" + wh)],
+                                                 before[(i, l, t, "v" + wh)], step, 1e-4, 0.9, 0.999, 1e-8, 0.01)
+                        np.testing.assert_allclose(srv.get_adapter(ids[i], l, t, wh), p, rtol=1e-5, atol=1e-7)
+                        np.testing.assert_allclose(srv.get_adapter(ids[i], l, t, "m" + wh), m_, rtol=1e-5,
+                                                   atol=1e-9)
+                        np.testing.assert_allclose(srv.get_adapter(ids[i], l, t, "v" + wh), v_, rtol=1e-5,
+                                                   atol=1e-12)
+                        assert not np.any(srv.get_adapter(ids[i], l, t, "d" + wh))  # consumed and zeroed
+    srv.close()
+
+
+def test_enomem_returned_not_crash():
+    from paper_conf_middleware_hul24_b200 import MenosError
+    w = workload("cfg0_tiny")
+    weights, adapters, io = make_inputs(w, seed=15)
+    srv = new_server(w, weights, arena_bytes=64 * 1024)
+    ids = register(srv, w, adapters)
+    x = torch.zeros(64, 64, dtype=torch.bfloat16, device="cuda")
+    with pytest.raises(MenosError) as e:
+        srv.forward([ids[0]] * 2 + [ids[1]] * 2, [16] * 4, x, torch.empty_like(x))
+    assert e.value.code == -2
+    srv.close()
+
+
+def test_host_buffers_e2e_path():
+    """x_c / g_c given as (pinned) host buffers: same results as device buffers."""
+    w = workload("cfg0_tiny")
+    inputs = make_inputs(w, seed=17)
+    weights, adapters, io = inputs
+    srv = new_server(w, weights)
+    ids = register(srv, w, adapters)
+    dev_out = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids, grads=False)
+    x = torch.from_numpy(np.concatenate([a for a, _ in io])).to(torch.bfloat16).pin_memory()
+    g = torch.from_numpy(np.concatenate([b for _, b in io])).to(torch.bfloat16).pin_memory()
+    xs, gs = torch.empty_like(x).pin_memory(), torch.empty_like(g).pin_memory()
+    b = srv.forward([ids[0]] * 2 + [ids[1]] * 2, [16] * 4, x, xs)
+    srv.backward(b, g, gs)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(xs.float().numpy(), np.concatenate(dev_out["x_s"]))
+    np.testing.assert_array_equal(gs.float().numpy(), np.concatenate(dev_out["g_s"]))
+    srv.close()
