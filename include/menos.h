@@ -88,7 +88,7 @@ enum {
 /* target index (0..6) used by get/set_adapter: q, k, v, o, gate, up, down */
 
 typedef struct {
-  float lr, beta1, beta2, eps, weight_decay; /* torch.optim.AdamW semantics */
+  double lr, beta1, beta2, eps, weight_decay; /* torch.optim.AdamW semantics (scalars in double, as torch forms them) */
 } menos_adamw_cfg;
 
 typedef struct {

@@ -6,7 +6,9 @@
  */
 #ifndef MENOS_TESTING_H_
 #define MENOS_TESTING_H_
+#include <stddef.h>
 #include <stdint.h>
+#include "menos.h"
 #ifndef MENOS_API
 #define MENOS_API __attribute__((visibility("default")))
 #endif
@@ -35,6 +37,16 @@ MENOS_API int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, in
 /* RMSNorm forward (y, rstd) and backward (dx = resid + norm_bwd(dy)); g fp32 [d].  Device buffers. */
 MENOS_API int menos_test_rmsnorm(int T, int d, const void* x, const float* g, float eps, void* y, float* rstd, const void* dy,
                        const void* resid, void* dx);
+
+/* Copy one saved intermediate of a live SAVE batch to host (debugging / white-box tests).
+ * which: 0 x, 1 xn, 2 qkv, 3 O, 4 h, 5 hn, 6 gu, 7 a, 8 U_qkv, 9 U_o, 10 U_gu, 11 U_down (bf16), 12 lse (fp32 [H,T]).
+ * *bytes receives the size; host_out may be NULL to query it. */
+MENOS_API int menos_test_batch_tensor(menos_server* s, menos_batch* b, int layer, int which, void* host_out,
+                                      size_t* bytes);
+
+/* One segmented small GEMM problem (LoRA shrink / dU / dA / dB kernel), device buffers. */
+MENOS_API int menos_test_small_gemm(const void* A, const void* B, float* Cf, void* Cb, int M, int N, int K, int lda,
+                                    int ldb, int ldc, int a_t, int b_t, float scale, int a_blk, int a_blk_stride);
 
 MENOS_API const char* menos_testing_last_error(void);
 

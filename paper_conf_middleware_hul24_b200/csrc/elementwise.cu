@@ -120,11 +120,11 @@ __global__ void adamw_kernel(const AdamSeg* __restrict__ segs, const int4* __res
     if (hp.do_update) {
       const float g = hp.g[i];
       float m = hp.m[i], v = hp.v[i];
-      p = p * (1.f - hp.lr * hp.wd);
-      m = hp.beta1 * m + (1.f - hp.beta1) * g;
-      v = hp.beta2 * v + (1.f - hp.beta2) * g * g;
+      p = p * hp.decay;
+      m = hp.beta1 * m + hp.omb1 * g;
+      v = hp.beta2 * v + hp.omb2 * (g * g);
       const float denom = sqrtf(v) / hp.bc2_sqrt + hp.eps;
-      p = p - (hp.lr / hp.bc1) * (m / denom);
+      p = p - hp.step_size * (m / denom);
       hp.p[i] = p; hp.m[i] = m; hp.v[i] = v; hp.g[i] = 0.f;
     }
     const int rr = e / sg.cols, cc = e % sg.cols;

@@ -105,7 +105,12 @@ struct AdamSeg {              // one (client, layer, target, A|B) parameter bloc
 };
 struct AdamHyper {
   float* p; float* g; float* m; float* v;
-  float lr, beta1, beta2, eps, wd, bc1, bc2_sqrt;
+  // torch.optim.AdamW scalar conventions: every scalar below is formed in double on the host, then rounded
+  float beta1, beta2, omb1, omb2;   // beta, 1 - beta
+  float decay;                       // 1 - lr * weight_decay
+  float step_size;                   // lr / (1 - beta1^t)
+  float bc2_sqrt;                    // sqrt(1 - beta2^t)
+  float eps;
   int do_update;              // 0: only refresh the bf16 copy (set_adapter / register)
 };
 int adamw_run(const AdamSeg* d_segs, const int4* d_work, int n_work, const AdamHyper* d_hyp, cudaStream_t st);

@@ -16,6 +16,7 @@
 #include <vector>
 
 #include "../../include/menos.h"
+#include "../../include/menos_testing.h"
 #include "kernels.h"
 
 using namespace menos;
@@ -363,9 +364,12 @@ static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, c
     h.do_update = update ? 1 : 0;
     if (update) {
       c.step += 1;
-      h.lr = c.opt.lr; h.beta1 = c.opt.beta1; h.beta2 = c.opt.beta2; h.eps = c.opt.eps; h.wd = c.opt.weight_decay;
-      h.bc1 = (float)(1.0 - std::pow((double)c.opt.beta1, (double)c.step));
-      h.bc2_sqrt = (float)std::sqrt(1.0 - std::pow((double)c.opt.beta2, (double)c.step));
+      const double lr = c.opt.lr, b1 = c.opt.beta1, b2 = c.opt.beta2;
+      h.beta1 = (float)b1; h.beta2 = (float)b2; h.omb1 = (float)(1.0 - b1); h.omb2 = (float)(1.0 - b2);
+      h.decay = (float)(1.0 - lr * (double)c.opt.weight_decay);
+      h.step_size = (float)(lr / (1.0 - std::pow(b1, (double)c.step)));
+      h.bc2_sqrt = (float)std::sqrt(1.0 - std::pow(b2, (double)c.step));
+      h.eps = (float)c.opt.eps;
     }
     hyp.push_back(h);
     if (!only) client_segments(s, c, (int)i, segs);
@@ -508,7 +512,7 @@ extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uin
   const Dims& D = s->D;
   Client c;
   c.rank = rank; c.rs = (int)align_up(rank, 16); c.alpha = alpha; c.s = alpha / (float)rank; c.mask = target_mask;
-  c.opt = opt ? *opt : menos_adamw_cfg{1e-4f, 0.9f, 0.999f, 1e-8f, 0.01f};
+  c.opt = opt ? *opt : menos_adamw_cfg{1e-4, 0.9, 0.999, 1e-8, 0.01};
   for (int t = 0; t < NT; ++t) c.sub[t] = -1;
   int cnt[NG] = {0, 0, 0, 0};
   for (int t = 0; t < NT; ++t)
@@ -801,6 +805,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   std::vector<int2> blocks;
   for (int i = 0; i < b->n_seqs; ++i)
     for (int q = 0; q < b->seq_len[i]; q += 64) blocks.push_back(make_int2(i, q));
+  b->n_blocks = (int)blocks.size();
   std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
   for (int g = 0; g < NG; ++g) {
     if (!b->g_active[g]) continue;
@@ -1295,4 +1300,36 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   // Release I after the backward (Fig.3(b); Alg.1 L13): the slab returns to the arena; stream
   // order guarantees later users run after this backward's kernels.
   return menos_batch_free(s, b);
+}
+
+// =====================================================================================================
+// white-box test hooks (include/menos_testing.h)
+// =====================================================================================================
+extern "C" int menos_test_batch_tensor(menos_server* s, menos_batch* b, int layer, int which, void* host_out,
+                                       size_t* bytes) {
+  if (!s || !b || !bytes || layer < 0 || layer >= s->n_layers || b->nograd) FAIL(MENOS_EINVAL, "bad arguments");
+  const Dims& D = s->D;
+  const LayerSave& S = b->L[layer];
+  const size_t T = b->T;
+  const void* src = nullptr;
+  size_t n = 0;
+  switch (which) {
+    case 0: src = S.x; n = T * D.d * 2; break;
+    case 1: src = S.xn; n = T * D.d * 2; break;
+    case 2: src = S.qkv; n = T * D.Nqkv * 2; break;
+    case 3: src = S.O; n = T * D.Nq * 2; break;
+    case 4: src = S.h; n = T * D.d * 2; break;
+    case 5: src = S.hn; n = T * D.d * 2; break;
+    case 6: src = S.gu; n = T * 2 * D.fpad * 2; break;
+    case 7: src = S.a; n = T * D.fpad * 2; break;
+    case 8: case 9: case 10: case 11: src = S.U[which - 8]; n = src ? T * b->R_used[which - 8] * 2 : 0; break;
+    case 12: src = S.lse; n = (size_t)D.H * T * 4; break;
+    default: FAIL(MENOS_EINVAL, "bad which");
+  }
+  *bytes = n;
+  if (host_out && n) {
+    CUDA_TRY(cudaDeviceSynchronize());
+    CUDA_TRY(cudaMemcpy(host_out, src, n, cudaMemcpyDeviceToHost));
+  }
+  return MENOS_OK;
 }

@@ -107,3 +107,25 @@ extern "C" int menos_test_rmsnorm(int T, int d, const void* x, const float* g, f
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   return MENOS_OK;
 }
+
+extern "C" int menos_test_small_gemm(const void* A, const void* B, float* Cf, void* Cb, int M, int N, int K, int lda,
+                                     int ldb, int ldc, int a_t, int b_t, float scale, int a_blk, int a_blk_stride) {
+  SmallGemmProblem p{};
+  p.A = (const bf16*)A; p.B = (const bf16*)B; p.Cf = Cf; p.Cb = (bf16*)Cb;
+  p.M = M; p.N = N; p.K = K; p.lda = lda; p.ldb = ldb; p.ldc = ldc; p.a_t = a_t; p.b_t = b_t; p.scale = scale;
+  p.a_blk = a_blk > 0 ? a_blk : (1 << 30); p.a_blk_stride = a_blk_stride;
+  std::vector<int4> tiles((size_t)((M + SG_BM - 1) / SG_BM) * ((N + SG_BN - 1) / SG_BN) + 1);
+  int nt = 0;
+  small_gemm_tiles(&p, 1, tiles.data(), &nt);
+  SmallGemmProblem* dp; int4* dt;
+  cudaMalloc(&dp, sizeof p);
+  cudaMalloc(&dt, tiles.size() * sizeof(int4));
+  cudaMemcpy(dp, &p, sizeof p, cudaMemcpyHostToDevice);
+  cudaMemcpy(dt, tiles.data(), tiles.size() * sizeof(int4), cudaMemcpyHostToDevice);
+  int rc = small_gemm_run(dp, dt, nt, 0);
+  cudaError_t e = cudaDeviceSynchronize();
+  cudaFree(dp); cudaFree(dt);
+  if (rc) return fail("small gemm rejected");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  return MENOS_OK;
+}

@@ -35,8 +35,8 @@ class LayerWeights(C.Structure):
 
 
 class AdamWCfg(C.Structure):
-    _fields_ = [("lr", C.c_float), ("beta1", C.c_float), ("beta2", C.c_float), ("eps", C.c_float),
-                ("weight_decay", C.c_float)]
+    _fields_ = [("lr", C.c_double), ("beta1", C.c_double), ("beta2", C.c_double), ("eps", C.c_double),
+                ("weight_decay", C.c_double)]
 
 
 class ServerOpts(C.Structure):
@@ -78,6 +78,8 @@ SIGNATURES = {
                              _P, _I, _I, _I, _PI32, _F, _I]),
     "menos_test_attention": (_I, [_I, _PI32, _I, _I, _I, _P, _P, _P, _P, _P, _F]),
     "menos_test_rmsnorm": (_I, [_I, _I, _P, _P, _F, _P, _P, _P, _P, _P]),
+    "menos_test_batch_tensor": (_I, [_P, _P, _I, _I, _P, C.POINTER(_S)]),
+    "menos_test_small_gemm": (_I, [_P, _P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _I, _F, _I, _I]),
     "menos_testing_last_error": (C.c_char_p, []),
 }
 

@@ -235,8 +235,9 @@ def test_attention_fwd_bwd(hd, H, Hkv, lens):
     O_d = torch.empty(T, H * hd, dtype=torch.bfloat16, device="cuda")
     lse = torch.empty(H, T, dtype=torch.float32, device="cuda")
     dqkv = torch.zeros(T, N, dtype=torch.bfloat16, device="cuda")
+    dO_d = dev(dO)  # keep a reference: a temporary's memory would be recycled before the call
     rc = lib().menos_test_attention(len(lens), i32(lens), H, Hkv, hd, qkv_d.data_ptr(), O_d.data_ptr(),
-                                    lse.data_ptr(), dev(dO).data_ptr(), dqkv.data_ptr(), 1e4)
+                                    lse.data_ptr(), dO_d.data_ptr(), dqkv.data_ptr(), 1e4)
     check(rc, testing=True)
     got_O, got_lse, got_d = host(O_d), lse.cpu().numpy(), host(dqkv)
     t0 = 0
@@ -253,9 +254,15 @@ def test_attention_fwd_bwd(hd, H, Hkv, lens):
         dq, dk = O.rope_bwd(dq, cos, sin), O.rope_bwd(dk, cos, sin)
         ref = np.concatenate([dq.reshape(L, -1), dk.reshape(L, -1), dv.reshape(L, -1)], 1)
         g = got_d[t0:t0 + L]
+        scale = np.max(np.abs(ref))
         for lo, hi in ((0, H * hd), (H * hd, (H + Hkv) * hd), ((H + Hkv) * hd, N)):
+            rn = np.linalg.norm(ref[:, lo:hi])
+            if rn < 1e-6 * max(scale, 1.0):
+                # S=1: dq = dk = 0 exactly (P = 1, dS = dP - D = 0); only rounding noise allowed
+                assert np.max(np.abs(g[:, lo:hi])) < 1e-2 * max(scale, 1.0), (L, lo)
+                continue
             num = np.sum(g[:, lo:hi].astype(np.float64) * ref[:, lo:hi])
-            den = np.linalg.norm(g[:, lo:hi]) * np.linalg.norm(ref[:, lo:hi]) + 1e-30
+            den = np.linalg.norm(g[:, lo:hi]) * rn + 1e-30
             assert num / den > 0.999, (L, lo)
             assert maxrel(g[:, lo:hi], ref[:, lo:hi]) < 3e-2, (L, lo)
         t0 += L
@@ -270,8 +277,9 @@ def test_rmsnorm_fwd_bwd(T, d):
     y = torch.empty(T, d, dtype=torch.bfloat16, device="cuda")
     rstd = torch.empty(T, dtype=torch.float32, device="cuda")
     dx = torch.empty_like(y)
-    check(lib().menos_test_rmsnorm(T, d, dev(x).data_ptr(), gd.data_ptr(), 1e-5, y.data_ptr(), rstd.data_ptr(),
-                                   dev(dy).data_ptr(), dev(res).data_ptr(), dx.data_ptr()), testing=True)
+    xd, dyd, rd = dev(x), dev(dy), dev(res)
+    check(lib().menos_test_rmsnorm(T, d, xd.data_ptr(), gd.data_ptr(), 1e-5, y.data_ptr(), rstd.data_ptr(),
+                                   dyd.data_ptr(), rd.data_ptr(), dx.data_ptr()), testing=True)
     ry, rr = O.rmsnorm_fwd(x, g, np.float32(1e-5))
     assert maxrel(host(y), ry) < 1e-2
     np.testing.assert_allclose(rstd.cpu().numpy(), rr[:, 0], rtol=1e-5)
