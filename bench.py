@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""Menos server-segment benchmark (BASELINE.json metric: server fwd+bwd tokens/s at N clients, Llama-2-7B LoRA;
+HBM bytes/client).
+
+One step = menos_forward(SAVE) over every client's tokens on this GPU -> menos_backward -> menos_adapter_step
+(SURVEY.md §8(d) timing protocol; Alg.1 L10-12).  Default workload = BASELINE.json configs[1]
+(Llama-2-7B layers 2..32, 4 clients r=8 on q,v, batch 4 x 512 = 8,192 tokens) on each GPU; with --gpus N
+every rank runs its own replica with its own 4 clients (weak scaling, no collective on the path).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl menos|reference]
+
+Inputs are synthetic and resident in HBM before the timed region (value); `e2e` repeats the measurement
+through the same C-ABI with pinned HOST buffers (H2D of x_c and g_c, D2H of x_s and g_s inside the timed
+region).  The reference arm (--impl reference) is the CPU oracle (oracle/), timed on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "server fwd+bwd tokens/s at N clients (Llama-2-7B LoRA); HBM bytes/client"
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            p = json.load(fh)
+        return p, "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+# ------------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except Exception:
+            self.p.kill()
+            out = ""
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        load = [v for v in sm if smax and v > 0.5 * smax] or sm
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------------------ CPU oracle
+def oracle_sample(n_layers: int = 2, n_seqs: int = 4, seq: int = 512):
+    """Time the CPU oracle (as it stands) on a bounded sample of the cfg1 workload: one client's batch
+    (n_seqs x seq tokens) through n_layers of the 31 server layers, fwd + bwd.  Returns tokens/s scaled to
+    the full 31-layer segment."""
+    import numpy as np
+    from oracle import menos_oracle as O
+    from workloads import ClientCfg, MODELS, base_layer_weights, client_adapters, client_inputs
+    cores = len(os.sched_getaffinity(0))
+    m = MODELS["7b"].with_layers(n_layers)
+    c = ClientCfg(8, 16.0, ("q", "v"), [seq] * n_seqs)
+    W = [base_layer_weights(m, l, seed=0) for l in range(n_layers)]
+    ad = client_adapters(m, c, seed=1)
+    x, g = client_inputs(m, c, seed=2)
+    t0 = time.perf_counter()
+    O.client_step(x, g, c.seq_lens, W, ad, c.alpha / c.rank, m)
+    dt = time.perf_counter() - t0
+    full = MODELS["7b"].n_layers
+    tps = c.n_tokens / (dt * full / n_layers)
+    return {"value": tps, "unit": "tokens/s", "cores": cores, "kind": "oracle",
+            "sample": f"1 client x {n_seqs} seq x {seq} tokens through {n_layers} of {full} Llama-2-7B server "
+                      f"layers (fwd+bwd, fp32 numpy, {dt:.1f} s), scaled to the {full}-layer segment"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    for _ in range(args.warmup):
+        oracle_sample(1, 1, 512)
+    vals = []
+    for _ in range(args.steps):
+        vals.append(oracle_sample(1, 1, 512))
+    v = statistics.median([r["value"] for r in vals])
+    cb = dict(vals[-1])
+    cb["value"] = v
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 512 / v * 1000.0, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "cfg1_7b_x4", "model": "llama2-7b", "sample": cb["sample"]},
+            "cpu_baseline": cb, "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0,
+                                        "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------ GPU arm
+def build_server(torch, w, device, seed, arena_gb):
+    from paper_conf_middleware_hul24_b200 import Server
+    m = w.model
+    srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
+                 rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=None, device=device.index,
+                 max_rank=16, max_seq_len=max(max(c.seq_lens) for c in w.clients),
+                 arena_bytes=int(arena_gb * (1 << 30)))
+    gen = torch.Generator(device=device)
+    hd = m.head_dim
+    shapes = {"wq": (m.n_heads * hd, m.d_model), "wk": (m.n_kv_heads * hd, m.d_model),
+              "wv": (m.n_kv_heads * hd, m.d_model), "wo": (m.d_model, m.n_heads * hd),
+              "wgate": (m.d_ff, m.d_model), "wup": (m.d_ff, m.d_model), "wdown": (m.d_model, m.d_ff)}
+    for l in range(m.n_layers):
+        gen.manual_seed(seed * 1000 + l)
+        lw = {k: (torch.randn(s, generator=gen, device=device, dtype=torch.float32) * 0.02).to(torch.bfloat16)
+              for k, s in shapes.items()}
+        for gname in ("g1", "g2"):
+            lw[gname] = (1 + 0.1 * torch.randn(m.d_model, generator=gen, device=device)).to(torch.bfloat16)
+        srv.load_layer(l, lw)
+        del lw
+    torch.cuda.synchronize(device)
+    return srv
+
+
+def register_clients(np, srv, w, seed):
+    ids = []
+    rng = np.random.default_rng(seed)
+    for i, c in enumerate(w.clients):
+        cid = srv.register_client(c.rank, c.alpha, c.targets, seed=seed * 100 + i)
+        for l in range(w.model.n_layers):
+            for t in c.targets:
+                (_, _), (rb, cb) = srv.adapter_shape(cid, t)
+                srv.set_adapter(cid, l, t, "B", (rng.standard_normal((rb, cb)) * 0.02).astype(np.float32))
+        ids.append(cid)
+    return ids
+
+
+def run_gpu(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_hul24_b200 import menos as M
+    from workloads import workload
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    device = torch.device("cuda", local)
+    torch.cuda.set_device(device)
+    w = workload(args.workload, n_layers=args.layers)
+    T = w.n_tokens
+    d = w.model.d_model
+    srv = build_server(torch, w, device, seed=rank, arena_gb=args.arena_gb)
+    ids = register_clients(np, srv, w, seed=rank + 1)
+    seq_client, seq_len = [], []
+    for i, c in enumerate(w.clients):
+        seq_client += [ids[i]] * len(c.seq_lens)
+        seq_len += list(c.seq_lens)
+    gen = torch.Generator(device=device)
+    gen.manual_seed(7 + rank)
+    x_c = torch.randn(T, d, generator=gen, device=device).to(torch.bfloat16)
+    g_c = torch.randn(T, d, generator=gen, device=device).to(torch.bfloat16)
+    x_s, g_s = torch.empty_like(x_c), torch.empty_like(x_c)
+    stream = torch.cuda.current_stream(device)
+
+    def step(xc, xs, gc, gs):
+        b = srv.forward(seq_client, seq_len, xc, xs, stream=stream)
+        srv.backward(b, gc, gs, stream=stream)
+        srv.adapter_step(ids, stream=stream)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def timed(fn, K):
+        barrier()
+        torch.cuda.synchronize(device)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(K):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize(device)
+        barrier()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device=device)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    for _ in range(args.warmup):
+        step(x_c, x_s, g_c, g_s)
+    torch.cuda.synchronize(device)
+
+    clocks = ClockSampler(device.index)
+    clocks.start()
+    time.sleep(0.3)
+    M.profile_enable(True)
+    l0 = M.launch_count()
+    ms = timed(lambda: step(x_c, x_s, g_c, g_s), args.steps)
+    launches = M.launch_count() - l0
+    prof = M.profile_read()
+    M.profile_enable(False)
+    clk = clocks.stop()
+    ms_per_step = ms / args.steps
+    value = world * T * args.steps / (ms / 1000.0)
+
+    # e2e through the same C-ABI with pinned host buffers (copies inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        hx = x_c.cpu().pin_memory()
+        hg = g_c.cpu().pin_memory()
+        hxs, hgs = torch.empty_like(hx).pin_memory(), torch.empty_like(hg).pin_memory()
+        step(hx, hxs, hg, hgs)
+        ms_e = timed(lambda: step(hx, hxs, hg, hgs), args.steps)
+        e2e = {"value": world * T * args.steps / (ms_e / 1000.0), "unit": "tokens/s",
+               "h2d_bytes_per_step": int(hx.numel() * 2 + hg.numel() * 2),
+               "d2h_bytes_per_step": int(hxs.numel() * 2 + hgs.numel() * 2),
+               "ms_per_step": ms_e / args.steps}
+
+    # roofline of the dominant kernel (tcgen05 GEMM) from the live per-launch CUDA events
+    peaks, src = load_peaks()
+    g = prof.get("gemm_tcgen05", {})
+    total_ms = sum(v["ms"] for v in prof.values()) or 1.0
+    achieved = g["flops"] / (g["ms"] / 1000.0) / 1e12 if g.get("ms") else None
+    peak = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "gemm_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "tensor", "kernel": "gemm_tcgen05", "achieved": achieved, "peak": peak,
+                "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                "peak_source": f"{src} bf16_tflops_sustained (kernel timed inside a long step)",
+                "launches": g.get("launches"), "share_of_kernel_time": g.get("ms", 0) / total_ms,
+                "avg_launch_ms": g["ms"] / g["launches"] if g.get("launches") else None}
+    kernels = {}
+    for k, v in prof.items():
+        if not v["launches"]:
+            continue
+        e = {"launches": v["launches"], "ms_per_step": v["ms"] / args.steps, "share": v["ms"] / total_ms}
+        if v["flops"]:
+            e["tflops"] = v["flops"] / (v["ms"] / 1000.0) / 1e12
+        if v["bytes"]:
+            e["gbs"] = v["bytes"] / (v["ms"] / 1000.0) / 1e9
+            e["frac_hbm"] = e["gbs"] / peaks.get("hbm_gbs", 6650.0)
+        kernels[k] = e
+    # algorithmic FLOPs of the whole step (no recompute credit, no base dW): 4 P + attention + LoRA
+    m = w.model
+    hd = m.head_dim
+    P = m.n_layers * (m.d_model * (m.n_heads + 2 * m.n_kv_heads) * hd + m.d_model * m.n_heads * hd
+                      + 3 * m.d_model * m.d_ff)
+    pairs = sum(s * (s + 1) / 2 for c in w.clients for s in c.seq_lens)
+    attn = 12 * hd * m.n_heads * pairs * m.n_layers
+    lora = 0.0
+    from workloads import target_dims
+    for c in w.clients:
+        for t in c.targets:
+            K_, N_ = target_dims(m, t)
+            lora += 6 * c.rank * (K_ + N_) * c.n_tokens * m.n_layers
+    step_flops = 4 * P * T + attn + lora
+    step_tflops = world * step_flops * args.steps / (ms / 1000.0) / 1e12
+
+    # HBM bytes per client (persistent A+O and the SAVE-forward arena share), Eq.3 accounting
+    st = srv.stats()
+    per_client = []
+    for i, c in enumerate(w.clients):
+        pers, fwd, bwd = srv.client_memory(ids[i], c.n_tokens)
+        per_client.append({"persistent_AO": pers, "arena_I": fwd})
+    AO = statistics.mean(p["persistent_AO"] for p in per_client)
+    Mb = st["base_bytes"]
+    Nc = len(w.clients)
+    hbm = {"base_M_bytes_once_per_gpu": Mb, "per_client_persistent_AO_bytes": AO,
+           "per_client_arena_I_bytes": statistics.mean(p["arena_I"] for p in per_client),
+           "persistent_reduction_vs_vanilla": 1.0 - (Mb + Nc * AO) / (Nc * (Mb + AO)),
+           "paper_reference": "PAPER.md:352: -72.2% for 4 Llama-2-7B clients on a V100 (fp32; context only)"}
+
+    line = {"metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded random weights/activations)",
+            "config": {"workload": args.workload, "model": w.model.name, "clients_per_gpu": len(w.clients),
+                       "tokens_per_gpu_step": T, "server_layers": w.model.n_layers,
+                       "lora": sorted({f"r{c.rank} {'+'.join(c.targets)}" for c in w.clients}),
+                       "seq_lens": sorted({s for c in w.clients for s in c.seq_lens}),
+                       "parallelism": f"replica x{world} (clients partitioned, no collective)",
+                       "l2": "inputs larger than L2: 12.55 GB bf16 weights + ~28 GB saved activations streamed "
+                             "per step vs 126 MB L2"},
+            "roofline": roofline, "step_tflops": step_tflops,
+            "step_frac_of_peak": step_tflops / peak if peak else None,
+            "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            line["cpu_baseline"] = oracle_sample(args.cpu_layers, 4, 512)
+        except Exception as ex:  # never let the baseline kill the bench line
+            line["cpu_baseline"] = {"value": None, "error": repr(ex)}
+    if rank == 0:
+        print(json.dumps(line))
+    srv.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="menos", choices=["menos", "reference"])
+    ap.add_argument("--workload", default="cfg1_7b_x4")
+    ap.add_argument("--layers", type=int, default=None, help="truncate depth (debug only; not a bench value)")
+    ap.add_argument("--arena-gb", type=float, default=80.0)
+    ap.add_argument("--cpu-layers", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_gpu(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

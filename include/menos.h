@@ -158,6 +158,18 @@ typedef struct {
 } menos_stats;
 MENOS_API int menos_get_stats(menos_server* s, menos_stats* out);
 
+/* Per-kernel-class device time, measured with CUDA events recorded on the launching stream around every
+ * launch while profiling is enabled (bench.py's live roofline).  enable(1) clears the counters; read
+ * synchronises the device, fills one entry per class (max_n >= 8) and clears the counters.
+ * flops / bytes are the ALGORITHMIC work of the launches (DESIGN.md §"Roofline accounting"). */
+typedef struct {
+  char name[32];
+  int launches;
+  double ms, flops, bytes;
+} menos_kernel_stat;
+MENOS_API int menos_profile_enable(int on);
+MENOS_API int menos_profile_read(menos_kernel_stat* out, int max_n, int* n_out);
+
 /* Number of kernels this library has launched since load (evidence for bench.py's gpu_launches). */
 MENOS_API unsigned long long menos_launch_count(void);
 

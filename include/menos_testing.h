@@ -44,9 +44,14 @@ MENOS_API int menos_test_rmsnorm(int T, int d, const void* x, const float* g, fl
 MENOS_API int menos_test_batch_tensor(menos_server* s, menos_batch* b, int layer, int which, void* host_out,
                                       size_t* bytes);
 
-/* One segmented small GEMM problem (LoRA shrink / dU / dA / dB kernel), device buffers. */
-MENOS_API int menos_test_small_gemm(const void* A, const void* B, float* Cf, void* Cb, int M, int N, int K, int lda,
-                                    int ldb, int ldc, int a_t, int b_t, float scale, int a_blk, int a_blk_stride);
+/* LoRA side contractions (device buffers, one problem):
+ *   rows:   C[t, j] = scale * sum_k A[t, k] * (b_kn ? B[k, j] : B[j, k])         (bf16 out; shrink / dU)
+ *   tokred: C[m, n] = scale * sum_t P[t, map(m)] * Q[t, n]                       (fp32 out; dA / dB)
+ *           map(m) = (m / p_blk) * p_blk_stride + m % p_blk (p_blk <= 0: identity); mt = 128 (dB) or 16 (dA). */
+MENOS_API int menos_test_lora_rows(const void* A, const void* B, void* C, int M, int N, int K, int lda, int ldb,
+                                   int ldc, int b_kn, float scale);
+MENOS_API int menos_test_lora_tokred(const void* P, const void* Q, float* C, int M, int N, int T, int ldp, int ldq,
+                                     int ldc, int p_blk, int p_blk_stride, float scale, int mt);
 
 MENOS_API const char* menos_testing_last_error(void);
 

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <vector>
 
 namespace menos {
 
@@ -48,22 +49,24 @@ struct GemmArgs {
 // Tensor maps are cached by (ptr, rows, cols, ld, box) on the host.
 int gemm_run(const GemmArgs& a, cudaStream_t st);
 
-// ---------------------------------------------------------------- small mma.sync GEMM (LoRA shrink/grads)
-// C[m, n] = scale * sum_k A(m, k) B(n, k)
-//   A(m,k) = a_t ? A[k*lda + map(m)] : A[m*lda + k];  B(n,k) = b_t ? B[k*ldb + n] : B[n*ldb + k]
-// Writes fp32 (c_f32) and/or bf16 (c_bf16); every problem is independent (no atomics).
-struct SmallGemmProblem {
-  const bf16* A; const bf16* B;
-  float* Cf; bf16* Cb;
-  int M, N, K, lda, ldb, ldc;
-  int a_t, b_t;
+// ---------------------------------------------------------------- segmented LoRA side contractions
+// rows: C[t, j] = scale * sum_k A[t, k] * Bop(j, k);  Bop(j,k) = b_kn ? B[k*ldb + j] : B[j*ldb + k]  (bf16 out)
+struct LoraRowsProblem {
+  const bf16* A; const bf16* B; bf16* C;
+  int M, N, K, lda, ldb, ldc, b_kn;
   float scale;
-  int a_blk, a_blk_stride;    // A row-index remap (a_t only): m -> (m / a_blk) * a_blk_stride + m % a_blk
 };
-int small_gemm_run(const SmallGemmProblem* d_probs, const int4* d_tiles, int n_tiles, cudaStream_t st);
-// host helper: tiles of a problem list (problem, m0, n0, 0)
-void small_gemm_tiles(const SmallGemmProblem* probs, int n, int4* out_tiles, int* n_tiles_out);
-const int SG_BM = 64, SG_BN = 64;
+// token reduction: C[m, n] = scale * sum_t P[t, map(m)] * Q[t, n]   (fp32 out, overwrite)
+//   map(m) = (m / p_blk) * p_blk_stride + m % p_blk   (gate/up interleaved 128-blocks)
+struct LoraTokRedProblem {
+  const bf16* P; const bf16* Q; float* C;
+  int M, N, T, ldp, ldq, ldc, p_blk, p_blk_stride;
+  float scale;
+};
+int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st);
+int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st);
+void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out);
+void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out);
 
 // ---------------------------------------------------------------- norms / elementwise
 int rmsnorm_fwd(const bf16* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st);

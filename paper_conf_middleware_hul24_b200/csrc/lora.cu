@@ -1,118 +1,229 @@
-// Segmented multi-client LoRA side GEMMs (SURVEY.md §8(a) A2/A4/A6/A7 shrink, A8-A12 LoRA backward):
-//   shrink   U_c  = s_c * X_c A_c^T          (bf16 block-diagonal operand of the GEMM's extra-K segment)
-//   dU       dU_c = s_c * dY_c B_c            (operand of the dX GEMM's extra-K segment, and of dA)
-//   dB       dB_c = s_c * dY_c^T U_c          (fp32, reduced over the client's tokens only)
-//   dA       dA_c = dU_c^T X_c                (fp32, reduced over the client's tokens only)
-// Every problem is one client's token segment; every output tile is owned by one CTA that loops over the
-// whole reduction in a fixed order, so results are deterministic and never mix clients.
-// These are tiny contractions (rank r <= 16); they run on mma.sync tensor cores with smem staging.
+// Segmented multi-client LoRA side contractions (SURVEY.md §8(a) A2/A4/A6/A7 shrink, A8-A12 LoRA backward).
+//
+//   rows kernel (one client's 64-token block, full reduction):
+//     shrink   U_c  = s_c * X_c A_c^T      (B operand = A_cat rows   [W, K], "nk")
+//     dU       dU_c = s_c * dY_c B_c       (B operand = B_cat        [K, W], "kn")
+//   token-reduction kernel (reduce over ONE client's tokens, fixed order -> deterministic, no atomics):
+//     dB_t     = dY_t^T (s U_t)            (fp32 [N_t, r])
+//     dA_t     = dU_t^T X                  (fp32 [r, K_t])
+//
+// Paper: LoRA y += (alpha/r)(x A^T) B^T on the targeted projections (§2.1, §5.1);
+// only phi = {A, B} receives gradients (Eq.1).  These are skinny contractions (r <= 16 per
+// target): they are bound by streaming X / dY from HBM once, so the kernels stage 16-byte cp.async tiles
+// (double-buffered) and use mma.sync m16n8k16 for the little arithmetic there is.
 #include "common.cuh"
 #include "kernels.h"
 
 namespace menos {
 namespace {
 
-constexpr int BM = 64, BN = 64, BKK = 32, PAD = 8;
+// swizzled element offset inside a [rows][COLS] bf16 tile (16-byte chunk XOR row)
+template <int COLS>
+__device__ __forceinline__ int tsw(int row, int chunk) {
+  constexpr int NCH = COLS / 8;
+  constexpr int MSK = NCH - 1 < 7 ? NCH - 1 : 7;
+  return row * COLS + ((chunk ^ (row & MSK)) << 3);
+}
 
-__global__ void __launch_bounds__(128) small_gemm_kernel(const SmallGemmProblem* __restrict__ probs,
-                                                         const int4* __restrict__ tiles) {
-  __shared__ __align__(16) bf16 As[BM][BKK + PAD];
-  __shared__ __align__(16) bf16 Bs[BN][BKK + PAD];
-  const int4 tl = tiles[blockIdx.x];
-  const SmallGemmProblem P = probs[tl.x];
-  const int m0 = tl.y, n0 = tl.z;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int wm = (warp >> 1) * 32, wn = (warp & 1) * 32;
-  const int g = lane >> 2, t = lane & 3;
-  float acc[2][4][4];
-#pragma unroll
-  for (int i = 0; i < 2; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-#pragma unroll
-      for (int k = 0; k < 4; ++k) acc[i][j][k] = 0.f;
+// ============================================================================ rows kernel
+// C[t, j] = scale * sum_k A[t, k] * Bop(j, k) for t in [m0, m0+64), j in [0, NT)
+template <int NT>
+__global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* __restrict__ probs,
+                                                        const int2* __restrict__ tiles) {
+  constexpr int BM = 64, BK = 64, NNT = NT / 8;
+  __shared__ __align__(128) bf16 As[2][BM * BK];
+  __shared__ __align__(128) bf16 Bs[2][NT * BK];  // "nk": [NT][BK]; "kn": [BK][NT]
+  const int2 tl = tiles[blockIdx.x];
+  const LoraRowsProblem P = probs[tl.x];
+  const int m0 = tl.y;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
 
-  const bf16 zero = __float2bfloat16_rn(0.f);
-  for (int k0 = 0; k0 < P.K; k0 += BKK) {
-    // stage A tile [BM][BKK] and B tile [BN][BKK] (K contiguous in smem), coalesced along the source's fast dim
-    for (int idx = tid; idx < BM * BKK; idx += 128) {
-      int m, k;
-      if (!P.a_t) { m = idx / BKK; k = idx % BKK; } else { k = idx / BM; m = idx % BM; }
-      const int gm = m0 + m, gk = k0 + k;
-      bf16 v = zero;
-      if (gm < P.M && gk < P.K) {
-        if (P.a_t) {
-          const int mm = (gm / P.a_blk) * P.a_blk_stride + gm % P.a_blk;
-          v = P.A[(size_t)gk * P.lda + mm];
-        } else {
-          v = P.A[(size_t)gm * P.lda + gk];
-        }
+  auto load = [&](int buf, int k0) {
+    for (int i = tid; i < BM * (BK / 8); i += 128) {
+      const int r = i / (BK / 8), c = i % (BK / 8);
+      const int gr = m0 + r, gk = k0 + c * 8;
+      const bool ok = gr < P.M && gk < P.K;
+      cp_async16(smem_u32(&As[buf][tsw<BK>(r, c)]), P.A + (ok ? (size_t)gr * P.lda + gk : 0), ok ? 16 : 0);
+    }
+    if (!P.b_kn) {
+      for (int i = tid; i < NT * (BK / 8); i += 128) {
+        const int r = i / (BK / 8), c = i % (BK / 8);
+        const int gk = k0 + c * 8;
+        const bool ok = r < P.N && gk < P.K;
+        cp_async16(smem_u32(&Bs[buf][tsw<BK>(r, c)]), P.B + (ok ? (size_t)r * P.ldb + gk : 0), ok ? 16 : 0);
       }
-      As[m][k] = v;
+    } else {
+      for (int i = tid; i < BK * (NT / 8); i += 128) {
+        const int r = i / (NT / 8), c = i % (NT / 8);
+        const int gk = k0 + r;
+        const bool ok = gk < P.K && c * 8 < P.N;
+        cp_async16(smem_u32(&Bs[buf][tsw<NT>(r, c)]), P.B + (ok ? (size_t)gk * P.ldb + c * 8 : 0), ok ? 16 : 0);
+      }
     }
-    for (int idx = tid; idx < BN * BKK; idx += 128) {
-      int n, k;
-      if (!P.b_t) { n = idx / BKK; k = idx % BKK; } else { k = idx / BN; n = idx % BN; }
-      const int gn = n0 + n, gk = k0 + k;
-      bf16 v = zero;
-      if (gn < P.N && gk < P.K) v = P.b_t ? P.B[(size_t)gk * P.ldb + gn] : P.B[(size_t)gn * P.ldb + gk];
-      Bs[n][k] = v;
-    }
+  };
+
+  float acc[NNT][4];
+#pragma unroll
+  for (int j = 0; j < NNT; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+  const int nk = (P.K + BK - 1) / BK;
+  load(0, 0);
+  cp_async_commit();
+  for (int kb = 0; kb < nk; ++kb) {
+    if (kb + 1 < nk) { load((kb + 1) & 1, (kb + 1) * BK); cp_async_commit(); cp_async_wait<1>(); }
+    else cp_async_wait<0>();
     __syncthreads();
+    const bf16* a_s = As[kb & 1];
+    const bf16* b_s = Bs[kb & 1];
 #pragma unroll
-    for (int kk = 0; kk < BKK; kk += 16) {
-      uint32_t a[2][4];
-#pragma unroll
-      for (int i = 0; i < 2; ++i) {
-        const int r = wm + i * 16 + g;
-        a[i][0] = *reinterpret_cast<const uint32_t*>(&As[r][kk + 2 * t]);
-        a[i][1] = *reinterpret_cast<const uint32_t*>(&As[r + 8][kk + 2 * t]);
-        a[i][2] = *reinterpret_cast<const uint32_t*>(&As[r][kk + 2 * t + 8]);
-        a[i][3] = *reinterpret_cast<const uint32_t*>(&As[r + 8][kk + 2 * t + 8]);
+    for (int kk = 0; kk < BK; kk += 16) {
+      uint32_t a[4];
+      {
+        const int mat = lane >> 3, r = lane & 7;
+        const int row = warp * 16 + (mat & 1) * 8 + r, col = kk + (mat >> 1) * 8;
+        ldsm_x4(smem_u32(a_s + tsw<BK>(row, col >> 3)), a[0], a[1], a[2], a[3]);
       }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int c = wn + j * 8 + g;
-        const uint32_t b0 = *reinterpret_cast<const uint32_t*>(&Bs[c][kk + 2 * t]);
-        const uint32_t b1 = *reinterpret_cast<const uint32_t*>(&Bs[c][kk + 2 * t + 8]);
-#pragma unroll
-        for (int i = 0; i < 2; ++i) mma_bf16_16816(acc[i][j], a[i], b0, b1);
+      for (int j = 0; j < NNT; j += 2) {
+        uint32_t b0, b1, b2, b3;
+        const int mat = lane >> 3, r = lane & 7;
+        if (!P.b_kn) {
+          const int row = j * 8 + (mat >> 1) * 8 + r, col = kk + (mat & 1) * 8;
+          ldsm_x4(smem_u32(b_s + tsw<BK>(row, col >> 3)), b0, b1, b2, b3);
+        } else {
+          const int row = kk + (mat & 1) * 8 + r, col = j * 8 + (mat >> 1) * 8;
+          ldsm_x4_t(smem_u32(b_s + tsw<NT>(row, col >> 3)), b0, b1, b2, b3);
+        }
+        mma_bf16_16816(acc[j], a, b0, b1);
+        mma_bf16_16816(acc[j + 1], a, b2, b3);
       }
     }
     __syncthreads();
   }
 #pragma unroll
-  for (int i = 0; i < 2; ++i)
+  for (int j = 0; j < NNT; ++j)
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
+    for (int h = 0; h < 2; ++h) {
+      const int r = m0 + warp * 16 + g + h * 8;
+      const int c = j * 8 + 2 * t;
+      if (r >= P.M || c >= P.N) continue;
+      *reinterpret_cast<uint32_t*>(P.C + (size_t)r * P.ldc + c) =
+          pack_bf16x2(acc[j][2 * h] * P.scale, acc[j][2 * h + 1] * P.scale);
+    }
+}
+
+// ============================================================================ token-reduction kernel
+// C[m, n] = scale * sum_t P[t, map(m)] * Q[t, n]  over t in [0, T); tile (MT x NT) at (m0, n0)
+template <int MT, int NT>
+__global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProblem* __restrict__ probs,
+                                                          const int4* __restrict__ tiles) {
+  constexpr int BK = 32;                       // tokens per stage
+  constexpr int WM = MT >= 64 ? MT / 4 : MT;   // rows per warp (4 warps split M when MT is large)
+  constexpr int WN = MT >= 64 ? NT : NT / 4;   // cols per warp (else split N)
+  constexpr int NMI = WM / 16, NNJ = WN / 8;
+  __shared__ __align__(128) bf16 Ps[2][BK * MT];   // [token][m]
+  __shared__ __align__(128) bf16 Qs[2][BK * NT];   // [token][n]
+  const int4 tl = tiles[blockIdx.x];
+  const LoraTokRedProblem P = probs[tl.x];
+  const int m0 = tl.y, n0 = tl.z;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
+  const int wm0 = MT >= 64 ? warp * WM : 0, wn0 = MT >= 64 ? 0 : warp * WN;
+  // P columns of this tile are contiguous: m0 is a multiple of MT and p_blk (128) is a multiple of MT
+  const int pcol0 = (m0 / P.p_blk) * P.p_blk_stride + m0 % P.p_blk;
+
+  auto load = [&](int buf, int t0) {
+    for (int i = tid; i < BK * (MT / 8); i += 128) {
+      const int r = i / (MT / 8), c = i % (MT / 8);
+      const int tok = t0 + r;
+      const bool ok = tok < P.T && m0 + c * 8 < P.M;
+      cp_async16(smem_u32(&Ps[buf][tsw<MT>(r, c)]), P.P + (ok ? (size_t)tok * P.ldp + pcol0 + c * 8 : 0), ok ? 16 : 0);
+    }
+    for (int i = tid; i < BK * (NT / 8); i += 128) {
+      const int r = i / (NT / 8), c = i % (NT / 8);
+      const int tok = t0 + r;
+      const bool ok = tok < P.T && n0 + c * 8 < P.N;
+      cp_async16(smem_u32(&Qs[buf][tsw<NT>(r, c)]), P.Q + (ok ? (size_t)tok * P.ldq + n0 + c * 8 : 0), ok ? 16 : 0);
+    }
+  };
+
+  float acc[NMI][NNJ][4];
+#pragma unroll
+  for (int i = 0; i < NMI; ++i)
+#pragma unroll
+    for (int j = 0; j < NNJ; ++j) acc[i][j][0] = acc[i][j][1] = acc[i][j][2] = acc[i][j][3] = 0.f;
+  const int nk = (P.T + BK - 1) / BK;
+  load(0, 0);
+  cp_async_commit();
+  for (int kb = 0; kb < nk; ++kb) {
+    if (kb + 1 < nk) { load((kb + 1) & 1, (kb + 1) * BK); cp_async_commit(); cp_async_wait<1>(); }
+    else cp_async_wait<0>();
+    __syncthreads();
+    const bf16* p_s = Ps[kb & 1];
+    const bf16* q_s = Qs[kb & 1];
+#pragma unroll
+    for (int kk = 0; kk < BK; kk += 16) {
+      const int mat = lane >> 3, r = lane & 7;
+      uint32_t a[NMI][4];
+#pragma unroll
+      for (int i = 0; i < NMI; ++i) {
+        // A(m, k) = P[k][m]: transposed ldmatrix of the [token][m] tile
+        const int row = kk + (mat >> 1) * 8 + r, col = wm0 + i * 16 + (mat & 1) * 8;
+        ldsm_x4_t(smem_u32(p_s + tsw<MT>(row, col >> 3)), a[i][0], a[i][1], a[i][2], a[i][3]);
+      }
+#pragma unroll
+      for (int j = 0; j < NNJ; j += 2) {
+        uint32_t b0, b1, b2, b3;
+        const int row = kk + (mat & 1) * 8 + r, col = wn0 + j * 8 + (mat >> 1) * 8;
+        ldsm_x4_t(smem_u32(q_s + tsw<NT>(row, col >> 3)), b0, b1, b2, b3);
+#pragma unroll
+        for (int i = 0; i < NMI; ++i) {
+          mma_bf16_16816(acc[i][j], a[i], b0, b1);
+          mma_bf16_16816(acc[i][j + 1], a[i], b2, b3);
+        }
+      }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < NMI; ++i)
+#pragma unroll
+    for (int j = 0; j < NNJ; ++j)
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const int r = m0 + wm + i * 16 + g + h * 8;
-        const int c = n0 + wn + j * 8 + 2 * t;
+        const int r = m0 + wm0 + i * 16 + g + h * 8;
+        const int c = n0 + wn0 + j * 8 + 2 * t;
         if (r >= P.M) continue;
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          if (c + e >= P.N) continue;
-          const float v = acc[i][j][2 * h + e] * P.scale;
-          if (P.Cf) P.Cf[(size_t)r * P.ldc + c + e] = v;
-          if (P.Cb) P.Cb[(size_t)r * P.ldc + c + e] = __float2bfloat16_rn(v);
-        }
+        if (c < P.N) P.C[(size_t)r * P.ldc + c] = acc[i][j][2 * h] * P.scale;
+        if (c + 1 < P.N) P.C[(size_t)r * P.ldc + c + 1] = acc[i][j][2 * h + 1] * P.scale;
       }
 }
 
 }  // namespace
 
-void small_gemm_tiles(const SmallGemmProblem* probs, int n, int4* out, int* n_out) {
-  int k = 0;
+void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out) {
   for (int i = 0; i < n; ++i)
-    for (int m = 0; m < probs[i].M; m += BM)
-      for (int c = 0; c < probs[i].N; c += BN) out[k++] = make_int4(i, m, c, 0);
-  *n_out = k;
+    for (int m = 0; m < probs[i].M; m += 64) out.push_back(make_int2(i, m));
+}
+void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out) {
+  for (int i = 0; i < n; ++i)
+    for (int m = 0; m < probs[i].M; m += mt)
+      for (int c = 0; c < probs[i].N; c += nt) out.push_back(make_int4(i, m, c, 0));
 }
 
-int small_gemm_run(const SmallGemmProblem* d_probs, const int4* d_tiles, int n_tiles, cudaStream_t st) {
+int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st) {
   if (n_tiles <= 0) return 0;
-  small_gemm_kernel<<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  if (max_n <= 32) lora_rows_kernel<32><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  else if (max_n <= 64) lora_rows_kernel<64><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  else if (max_n <= 128) lora_rows_kernel<128><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  else return -1;
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st) {
+  if (n_tiles <= 0) return 0;
+  if (mt == 128) lora_tokred_kernel<128, 16><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  else if (mt == 16) lora_tokred_kernel<16, 128><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  else return -1;
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }

@@ -49,6 +49,39 @@ static void set_err(const char* fmt, ...) {
   } while (0)
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// =====================================================================================================
+// per-kernel-class CUDA-event profiler (bench.py's live roofline; off by default)
+// =====================================================================================================
+enum ProfClass { PC_GEMM = 0, PC_ATTN_FWD, PC_ATTN_BWD, PC_LORA, PC_NORM, PC_ATTN_PREP, PC_ADAMW, PC_N };
+static const char* kProfName[PC_N] = {"gemm_tcgen05", "attn_fwd", "attn_bwd", "lora_side", "rmsnorm",
+                                      "attn_bwd_prep", "adamw"};
+struct ProfRec { cudaEvent_t a, b; int cls; double flops, bytes; };
+static bool g_prof_on = false;
+static std::vector<ProfRec> g_prof;
+static std::vector<cudaEvent_t> g_ev_pool;
+static size_t g_ev_used = 0;
+static cudaEvent_t prof_event() {
+  if (g_ev_used == g_ev_pool.size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    g_ev_pool.push_back(e);
+  }
+  return g_ev_pool[g_ev_used++];
+}
+struct ProfScope {
+  bool on; ProfRec r; cudaStream_t st;
+  ProfScope(int cls, double flops, double bytes, cudaStream_t s) : on(g_prof_on), st(s) {
+    if (!on) return;
+    r.cls = cls; r.flops = flops; r.bytes = bytes; r.a = prof_event(); r.b = prof_event();
+    cudaEventRecord(r.a, st);
+  }
+  ~ProfScope() {
+    if (!on) return;
+    cudaEventRecord(r.b, st);
+    g_prof.push_back(r);
+  }
+};
 static inline int ceil_div(int a, int b) { return (a + b - 1) / b; }
 
 // =====================================================================================================
@@ -195,7 +228,7 @@ struct LayerSave {
   float *rstd1, *rstd2, *lse;
   bf16* U[NG];
 };
-struct SGList { int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0; };
+struct SGList { int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0; };
 
 struct menos_batch {
   int T = 0, n_seqs = 0;
@@ -207,14 +240,16 @@ struct menos_batch {
   bool g_active[NG] = {false, false, false, false};
   bool save_a = false;
   int n_mt = 0, n_blocks = 0;
+  double pairs = 0;   // causal (query, key) pairs summed over sequences
   // device metadata
   uint8_t* meta = nullptr;  // arena
   int* d_cu = nullptr; int* d_pos = nullptr; int2* d_blocks = nullptr;
   int2* d_mtile[NG] = {nullptr, nullptr, nullptr, nullptr};
   uint8_t* d_ntile_qkv = nullptr;
-  SmallGemmProblem* d_probs = nullptr; int4* d_tiles = nullptr;
-  // per layer, per group: fwd shrink, bwd dU, bwd dA+dB
-  std::vector<SGList> sg_fwd, sg_du, sg_grad;  // [layer * NG + g]
+  LoraRowsProblem* d_rprobs = nullptr; int2* d_rtiles = nullptr;
+  LoraTokRedProblem* d_tprobs = nullptr; int4* d_ttiles = nullptr;
+  // per layer, per group: fwd shrink, bwd dU, bwd dB, bwd dA
+  std::vector<SGList> sg_fwd, sg_du, sg_db, sg_da;  // [layer * NG + g]
   // saved activations (SAVE) or x_c copy (NOGRAD)
   uint8_t* slab = nullptr;
   std::vector<LayerSave> L;
@@ -392,7 +427,12 @@ static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, c
   memcpy(s->pinned + o2, segs.data(), b2);
   memcpy(s->pinned + o3, work.data(), b3);
   CUDA_TRY(cudaMemcpyAsync(dbuf, s->pinned, tot, cudaMemcpyHostToDevice, st));
-  K_TRY(adamw_run((AdamSeg*)(dbuf + o2), (int4*)(dbuf + o3), (int)work.size(), (AdamHyper*)dbuf, st));
+  double nparam = 0;
+  for (auto& sg : segs) nparam += (double)sg.rows * sg.cols;
+  {
+    ProfScope ps(PC_ADAMW, 0, nparam * (update ? 30.0 : 6.0), st);
+    K_TRY(adamw_run((AdamSeg*)(dbuf + o2), (int4*)(dbuf + o3), (int)work.size(), (AdamHyper*)dbuf, st));
+  }
   CUDA_TRY(cudaFreeAsync(dbuf, st));
   return MENOS_OK;
 }
@@ -720,6 +760,31 @@ extern "C" int menos_get_stats(menos_server* s, menos_stats* o) {
 
 extern "C" unsigned long long menos_launch_count(void) { return g_launch_count; }
 
+extern "C" int menos_profile_enable(int on) {
+  g_prof_on = on != 0;
+  g_prof.clear();
+  g_ev_used = 0;
+  return MENOS_OK;
+}
+
+extern "C" int menos_profile_read(menos_kernel_stat* out, int max_n, int* n_out) {
+  if (!out || !n_out || max_n < PC_N) FAIL(MENOS_EINVAL, "need room for %d classes", (int)PC_N);
+  CUDA_TRY(cudaDeviceSynchronize());
+  for (int c = 0; c < PC_N; ++c) {
+    memset(&out[c], 0, sizeof out[c]);
+    snprintf(out[c].name, sizeof out[c].name, "%s", kProfName[c]);
+  }
+  for (auto& r : g_prof) {
+    float ms = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&ms, r.a, r.b));
+    out[r.cls].launches += 1; out[r.cls].ms += ms; out[r.cls].flops += r.flops; out[r.cls].bytes += r.bytes;
+  }
+  *n_out = PC_N;
+  g_prof.clear();
+  g_ev_used = 0;
+  return MENOS_OK;
+}
+
 extern "C" int menos_sync(menos_server* s) {
   if (!s) FAIL(MENOS_EINVAL, "null server");
   CUDA_TRY(cudaSetDevice(s->device));
@@ -757,6 +822,7 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
     b->seq_client.push_back(c); b->seq_len.push_back(L);
     b->cu.push_back(b->cu.back() + L);
     for (int p = 0; p < L; ++p) b->pos.push_back(p);
+    b->pairs += 0.5 * (double)L * (L + 1);
   }
   b->T = b->cu.back();
   const int T = b->T;
@@ -773,7 +839,8 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   // small-GEMM problem lists are filled later (need layer buffers); reserve host vectors here
   b->sg_fwd.resize((size_t)s->n_layers * NG);
   b->sg_du.resize((size_t)s->n_layers * NG);
-  b->sg_grad.resize((size_t)s->n_layers * NG);
+  b->sg_db.resize((size_t)s->n_layers * NG);
+  b->sg_da.resize((size_t)s->n_layers * NG);
 
   out = std::move(b);
   return MENOS_OK;
@@ -858,22 +925,30 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->L[0].x = (bf16*)slab;  // x_c copy (only the forward input is cached)
   }
 
-  // ---- small-GEMM problem lists (need buffer pointers: built against the SAVE layout, or the scratch layer)
-  std::vector<SmallGemmProblem> probs;
-  std::vector<int4> tiles;
-  auto add_list = [&](SGList& L, const std::vector<SmallGemmProblem>& ps) {
-    L.probs_off = (int)probs.size(); L.n_probs = (int)ps.size();
-    L.tiles_off = (int)tiles.size();
-    std::vector<int4> tl(1);
-    int cnt = 0;
-    for (const auto& pp : ps) cnt += ceil_div(pp.M, SG_BM) * ceil_div(pp.N, SG_BN);
-    tl.resize(std::max(cnt, 1));
-    int nt = 0;
-    small_gemm_tiles(ps.data(), (int)ps.size(), tl.data(), &nt);
-    for (int i = 0; i < nt; ++i) tl[i].x += L.probs_off;
-    L.n_tiles = nt;
-    probs.insert(probs.end(), ps.begin(), ps.end());
-    tiles.insert(tiles.end(), tl.begin(), tl.begin() + nt);
+  // ---- LoRA side-contraction problem lists (need buffer pointers: SAVE layout, or the NOGRAD layer set)
+  std::vector<LoraRowsProblem> rprobs;
+  std::vector<int2> rtiles;
+  std::vector<LoraTokRedProblem> tprobs;
+  std::vector<int4> ttiles;
+  auto add_rows = [&](SGList& L, const std::vector<LoraRowsProblem>& ps) {
+    L.probs_off = (int)rprobs.size(); L.n_probs = (int)ps.size(); L.tiles_off = (int)rtiles.size();
+    std::vector<int2> tl;
+    lora_rows_tiles(ps.data(), (int)ps.size(), tl);
+    for (auto& x : tl) x.x += L.probs_off;
+    for (const auto& pp : ps) { L.flops += 2.0 * pp.M * pp.N * pp.K; L.max_n = std::max(L.max_n, pp.N); }
+    L.n_tiles = (int)tl.size();
+    rprobs.insert(rprobs.end(), ps.begin(), ps.end());
+    rtiles.insert(rtiles.end(), tl.begin(), tl.end());
+  };
+  auto add_tokred = [&](SGList& L, const std::vector<LoraTokRedProblem>& ps, int mt, int nt) {
+    L.probs_off = (int)tprobs.size(); L.n_probs = (int)ps.size(); L.tiles_off = (int)ttiles.size();
+    std::vector<int4> tl;
+    lora_tokred_tiles(ps.data(), (int)ps.size(), mt, nt, tl);
+    for (auto& x : tl) x.x += L.probs_off;
+    for (const auto& pp : ps) L.flops += 2.0 * pp.M * pp.N * pp.T;
+    L.n_tiles = (int)tl.size(); L.max_n = mt;
+    tprobs.insert(tprobs.end(), ps.begin(), ps.end());
+    ttiles.insert(ttiles.end(), tl.begin(), tl.end());
   };
   for (int l = 0; l < Ls; ++l) {
     const LayerSave& S = save ? b->L[l] : *ng;
@@ -891,53 +966,60 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = 2 * D.fpad; break;
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
-      std::vector<SmallGemmProblem> f, du, gr;
+      std::vector<LoraRowsProblem> f, du;
+      std::vector<LoraTokRedProblem> db, da;
       for (size_t k = 0; k < b->bclients.size(); ++k) {
         const Client& c = s->clients[b->bclients[k]];
         if (!c.width[g]) continue;
         const int t0 = b->btok_off[k], Tc = b->btok_n[k];
-        SmallGemmProblem p{};
-        p.a_blk = 1 << 30; p.a_blk_stride = 0;
-        // shrink: U[t, off..off+w) = s * X_c A^T
-        p.A = X + (size_t)t0 * ldx; p.lda = ldx;
-        p.B = s->Acat[g][l] + (size_t)c.col_off[g] * D.ldK_g[g]; p.ldb = D.ldK_g[g];
-        p.Cb = U + (size_t)t0 * R + c.col_off[g]; p.Cf = nullptr; p.ldc = R;
-        p.M = Tc; p.N = c.width[g]; p.K = D.K_g[g]; p.a_t = 0; p.b_t = 0; p.scale = c.s;
-        f.push_back(p);
-        // dU[t, off..off+w) = s * dY_c Bcat[:, off..]
-        SmallGemmProblem q{};
-        q.a_blk = 1 << 30; q.a_blk_stride = 0;
-        q.A = dY + (size_t)t0 * ldy; q.lda = ldy;
-        q.B = s->Bcat[g][l] + c.col_off[g]; q.ldb = s->cols[g].cap; q.b_t = 1; q.a_t = 0;
-        q.Cb = sc.dU[g] + (size_t)t0 * R + c.col_off[g]; q.Cf = nullptr; q.ldc = R;
-        q.M = Tc; q.N = c.width[g]; q.K = D.N_g[g]; q.scale = c.s;
-        du.push_back(q);
-        // per target: dB = dY_t^T U_t (U holds s*x A^T), dA = dU_t^T X
+        for (int j0 = 0; j0 < c.width[g]; j0 += 128) {
+          const int w = std::min(128, c.width[g] - j0);
+          const int col = c.col_off[g] + j0;
+          // shrink: U[t, col..col+w) = s * X_c Acat[col.., :]^T
+          LoraRowsProblem p{};
+          p.A = X + (size_t)t0 * ldx; p.lda = ldx;
+          p.B = s->Acat[g][l] + (size_t)col * D.ldK_g[g]; p.ldb = D.ldK_g[g]; p.b_kn = 0;
+          p.C = U + (size_t)t0 * R + col; p.ldc = R;
+          p.M = Tc; p.N = w; p.K = D.K_g[g]; p.scale = c.s;
+          f.push_back(p);
+          // dU[t, col..col+w) = s * dY_c Bcat[:, col..]   (other targets' rows of Bcat are zero in these columns)
+          LoraRowsProblem q{};
+          q.A = dY + (size_t)t0 * ldy; q.lda = ldy;
+          q.B = s->Bcat[g][l] + col; q.ldb = s->cols[g].cap; q.b_kn = 1;
+          q.C = sc.dU[g] + (size_t)t0 * R + col; q.ldc = R;
+          q.M = Tc; q.N = w; q.K = D.N_g[g]; q.scale = c.s;
+          du.push_back(q);
+        }
+        // per target: dB = dY_t^T (s U_t), dA = dU_t^T X   (fp32, overwrite; reduced over this client only)
         for (int t = 0; t < NT; ++t) {
           if (kTargetGroup[t] != g || !(c.mask >> t & 1)) continue;
-          SmallGemmProblem pb{};
-          pb.A = dY + (size_t)t0 * ldy + D.rb_base[t]; pb.lda = ldy; pb.a_t = 1;
-          pb.a_blk = D.rb_blk[t]; pb.a_blk_stride = D.rb_stride[t];
-          pb.B = U + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pb.ldb = R; pb.b_t = 1;
-          pb.Cf = c.G() + c.offB[l * NT + t]; pb.Cb = nullptr; pb.ldc = c.rank;
-          pb.M = D.N_t[t]; pb.N = c.rank; pb.K = Tc; pb.scale = 1.f;
-          gr.push_back(pb);
-          SmallGemmProblem pa{};
-          pa.a_blk = 1 << 30; pa.a_blk_stride = 0;
-          pa.A = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pa.lda = R; pa.a_t = 1;
-          pa.B = X + (size_t)t0 * ldx; pa.ldb = ldx; pa.b_t = 1;
-          pa.Cf = c.G() + c.offA[l * NT + t]; pa.Cb = nullptr; pa.ldc = D.K_t[t];
-          pa.M = c.rank; pa.N = D.K_t[t]; pa.K = Tc; pa.scale = 1.f;
-          gr.push_back(pa);
+          LoraTokRedProblem pb{};
+          pb.P = dY + (size_t)t0 * ldy + D.rb_base[t]; pb.ldp = ldy;
+          pb.p_blk = D.rb_blk[t]; pb.p_blk_stride = D.rb_stride[t];
+          pb.Q = U + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pb.ldq = R;
+          pb.C = c.G() + c.offB[l * NT + t]; pb.ldc = c.rank;
+          pb.M = D.N_t[t]; pb.N = c.rank; pb.T = Tc; pb.scale = 1.f;
+          db.push_back(pb);
+          LoraTokRedProblem pa{};
+          pa.P = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pa.ldp = R;
+          pa.p_blk = 1 << 30; pa.p_blk_stride = 0;
+          pa.Q = X + (size_t)t0 * ldx; pa.ldq = ldx;
+          pa.C = c.G() + c.offA[l * NT + t]; pa.ldc = D.K_t[t];
+          pa.M = c.rank; pa.N = D.K_t[t]; pa.T = Tc; pa.scale = 1.f;
+          da.push_back(pa);
         }
       }
-      add_list(b->sg_fwd[(size_t)l * NG + g], f);
-      add_list(b->sg_du[(size_t)l * NG + g], du);
-      add_list(b->sg_grad[(size_t)l * NG + g], gr);
+      const size_t li = (size_t)l * NG + g;
+      add_rows(b->sg_fwd[li], f);
+      add_rows(b->sg_du[li], du);
+      add_tokred(b->sg_db[li], db, 128, 16);
+      add_tokred(b->sg_da[li], da, 16, 128);
     }
   }
-  const size_t o_pr = put(probs.data(), probs.size() * sizeof(SmallGemmProblem));
-  const size_t o_tl = put(tiles.data(), tiles.size() * sizeof(int4));
+  const size_t o_rp = put(rprobs.data(), rprobs.size() * sizeof(LoraRowsProblem));
+  const size_t o_rt = put(rtiles.data(), rtiles.size() * sizeof(int2));
+  const size_t o_tp = put(tprobs.data(), tprobs.size() * sizeof(LoraTokRedProblem));
+  const size_t o_tt = put(ttiles.data(), ttiles.size() * sizeof(int4));
   uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
   if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
   b->meta = meta;
@@ -949,8 +1031,10 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
-  b->d_probs = (SmallGemmProblem*)(meta + o_pr);
-  b->d_tiles = (int4*)(meta + o_tl);
+  b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
+  b->d_rtiles = (int2*)(meta + o_rt);
+  b->d_tprobs = (LoraTokRedProblem*)(meta + o_tp);
+  b->d_ttiles = (int4*)(meta + o_tt);
   return MENOS_OK;
 }
 
@@ -1003,9 +1087,15 @@ static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scr
 // =====================================================================================================
 // per-layer schedules
 // =====================================================================================================
-static int run_sg(menos_batch* b, const SGList& L, cudaStream_t st) {
+static int run_rows(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
-  return small_gemm_run(b->d_probs, b->d_tiles + L.tiles_off, L.n_tiles, st);
+  ProfScope ps(PC_LORA, L.flops, 0, st);
+  return lora_rows_run(b->d_rprobs, b->d_rtiles + L.tiles_off, L.n_tiles, L.max_n, st);
+}
+static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
+  if (L.n_tiles == 0) return 0;
+  ProfScope ps(PC_LORA, L.flops, 0, st);
+  return lora_tokred_run(b->d_tprobs, b->d_ttiles + L.tiles_off, L.n_tiles, L.max_n, st);
 }
 
 static GemmArgs gemm_base(menos_server* s) {
@@ -1022,11 +1112,11 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
   const auto& W = s->W[l];
   const int T = b->T;
   // A1: RMSNorm1
-  K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st));
+  { ProfScope ps(PC_NORM, 0, (double)T * (4.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st)); }
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
   if (b->g_active[GQKV]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
-    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GQKV], st));
+    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GQKV], st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1038,7 +1128,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
     }
     a.epi = EPI_ROPE; a.out = S.qkv; a.ldo = D.Nqkv;
     a.rope_cs = s->rope; a.pos = b->d_pos; a.head_dim = D.hd; a.rope_cols = D.Nq + D.Nkv;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A3: varlen causal flash attention
   {
@@ -1047,12 +1137,12 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
     a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    K_TRY(attn_fwd(a, st));
+    { ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st); K_TRY(attn_fwd(a, st)); }
   }
   // A4: O GEMM (+ LoRA o) + residual
   if (b->g_active[GO]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GO], 0, (size_t)T * b->R_used[GO] * 2, st));
-    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GO], st));
+    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GO], st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1062,14 +1152,14 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
       a.mtile_extra = b->d_mtile[GO];
     }
     a.epi = EPI_RESID; a.out = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A5: RMSNorm2
-  K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st));
+  { ProfScope ps(PC_NORM, 0, (double)T * (4.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st)); }
   // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
   if (b->g_active[GGU]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
-    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GGU], st));
+    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GGU], st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1079,12 +1169,12 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
       a.mtile_extra = b->d_mtile[GGU];
     }
     a.epi = EPI_SWIGLU_FWD; a.out = S.gu; a.ldo = 2 * D.fpad; a.out2 = S.a; a.ldo2 = D.fpad;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A7: down GEMM (+ LoRA down) + residual
   if (b->g_active[GD]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GD], 0, (size_t)T * b->R_used[GD] * 2, st));
-    if (use_lists) K_TRY(run_sg(b, b->sg_fwd[(size_t)l * NG + GD], st));
+    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GD], st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1094,7 +1184,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
       a.mtile_extra = b->d_mtile[GD];
     }
     a.epi = EPI_RESID; a.out = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   return MENOS_OK;
 }
@@ -1107,7 +1197,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
   const LayerSave& S = b->L[l];
   const int T = b->T;
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
-  if (b->g_active[GD]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GD], st));
+  if (b->g_active[GD]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GD], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.fpad; a.K = D.d; a.b_mn_major = 1;
@@ -1117,11 +1207,11 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
       a.mtile_extra = b->d_mtile[GD];
     }
     a.epi = EPI_SWIGLU_BWD; a.out = sc.dgu; a.ldo = 2 * D.fpad; a.aux = S.gu; a.ldaux = 2 * D.fpad;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GD]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GD], st));
+  if (b->g_active[GD]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GD], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GD], st)); }
   // A9: gate/up dX (+ LoRA) -> dhn; RMSNorm2 backward + residual -> dh
-  if (b->g_active[GGU]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GGU], st));
+  if (b->g_active[GGU]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GGU], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = 2 * D.fpad; a.b_mn_major = 1;
@@ -1131,12 +1221,12 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
       a.mtile_extra = b->d_mtile[GGU];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GGU]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GGU], st));
-  K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dy, sc.dh, T, D.d, st));
+  if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
+  { ProfScope ps(PC_NORM, 0, (double)T * (8.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dy, sc.dh, T, D.d, st)); }
   // A10: O dX (+ LoRA o) -> dO
-  if (b->g_active[GO]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GO], st));
+  if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
@@ -1146,11 +1236,11 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
       a.mtile_extra = b->d_mtile[GO];
     }
     a.epi = EPI_STORE; a.out = sc.dO; a.ldo = D.Nq;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GO]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GO], st));
+  if (b->g_active[GO]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GO], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GO], st)); }
   // A11: attention backward (+ RoPE backward) -> dqkv
-  K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st));
+  { ProfScope ps(PC_ATTN_PREP, 0, (double)T * (4.0 * D.Nq + 4 * D.H), st); K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st)); }
   {
     AttnArgs a;
     memset(&a, 0, sizeof a);
@@ -1158,10 +1248,10 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
-    K_TRY(attn_bwd(a, st));
+    { ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * b->pairs, 0, st); K_TRY(attn_bwd(a, st)); }
   }
   // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
-  if (b->g_active[GQKV]) K_TRY(run_sg(b, b->sg_du[(size_t)l * NG + GQKV], st));
+  if (b->g_active[GQKV]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GQKV], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = D.Nqkv; a.b_mn_major = 1;
@@ -1171,10 +1261,10 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
       a.mtile_extra = b->d_mtile[GQKV];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
-    K_TRY(gemm_run(a, st));
+    { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GQKV]) K_TRY(run_sg(b, b->sg_grad[(size_t)l * NG + GQKV], st));
-  K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dh, dx, T, D.d, st));
+  if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
+  { ProfScope ps(PC_NORM, 0, (double)T * (8.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dh, dx, T, D.d, st)); }
   return MENOS_OK;
 }
 

@@ -108,24 +108,43 @@ extern "C" int menos_test_rmsnorm(int T, int d, const void* x, const float* g, f
   return MENOS_OK;
 }
 
-extern "C" int menos_test_small_gemm(const void* A, const void* B, float* Cf, void* Cb, int M, int N, int K, int lda,
-                                     int ldb, int ldc, int a_t, int b_t, float scale, int a_blk, int a_blk_stride) {
-  SmallGemmProblem p{};
-  p.A = (const bf16*)A; p.B = (const bf16*)B; p.Cf = Cf; p.Cb = (bf16*)Cb;
-  p.M = M; p.N = N; p.K = K; p.lda = lda; p.ldb = ldb; p.ldc = ldc; p.a_t = a_t; p.b_t = b_t; p.scale = scale;
-  p.a_blk = a_blk > 0 ? a_blk : (1 << 30); p.a_blk_stride = a_blk_stride;
-  std::vector<int4> tiles((size_t)((M + SG_BM - 1) / SG_BM) * ((N + SG_BN - 1) / SG_BN) + 1);
-  int nt = 0;
-  small_gemm_tiles(&p, 1, tiles.data(), &nt);
-  SmallGemmProblem* dp; int4* dt;
+extern "C" int menos_test_lora_rows(const void* A, const void* B, void* C, int M, int N, int K, int lda, int ldb,
+                                    int ldc, int b_kn, float scale) {
+  LoraRowsProblem p{};
+  p.A = (const bf16*)A; p.B = (const bf16*)B; p.C = (bf16*)C;
+  p.M = M; p.N = N; p.K = K; p.lda = lda; p.ldb = ldb; p.ldc = ldc; p.b_kn = b_kn; p.scale = scale;
+  std::vector<int2> tiles;
+  lora_rows_tiles(&p, 1, tiles);
+  LoraRowsProblem* dp; int2* dt;
   cudaMalloc(&dp, sizeof p);
-  cudaMalloc(&dt, tiles.size() * sizeof(int4));
+  cudaMalloc(&dt, tiles.size() * sizeof(int2) + 8);
   cudaMemcpy(dp, &p, sizeof p, cudaMemcpyHostToDevice);
-  cudaMemcpy(dt, tiles.data(), tiles.size() * sizeof(int4), cudaMemcpyHostToDevice);
-  int rc = small_gemm_run(dp, dt, nt, 0);
+  cudaMemcpy(dt, tiles.data(), tiles.size() * sizeof(int2), cudaMemcpyHostToDevice);
+  int rc = lora_rows_run(dp, dt, (int)tiles.size(), N, 0);
   cudaError_t e = cudaDeviceSynchronize();
   cudaFree(dp); cudaFree(dt);
-  if (rc) return fail("small gemm rejected");
+  if (rc) return fail("lora rows rejected");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  return MENOS_OK;
+}
+
+extern "C" int menos_test_lora_tokred(const void* P, const void* Q, float* C, int M, int N, int T, int ldp, int ldq,
+                                      int ldc, int p_blk, int p_blk_stride, float scale, int mt) {
+  LoraTokRedProblem p{};
+  p.P = (const bf16*)P; p.Q = (const bf16*)Q; p.C = C;
+  p.M = M; p.N = N; p.T = T; p.ldp = ldp; p.ldq = ldq; p.ldc = ldc;
+  p.p_blk = p_blk > 0 ? p_blk : (1 << 30); p.p_blk_stride = p_blk_stride; p.scale = scale;
+  std::vector<int4> tiles;
+  lora_tokred_tiles(&p, 1, mt, mt == 128 ? 16 : 128, tiles);
+  LoraTokRedProblem* dp; int4* dt;
+  cudaMalloc(&dp, sizeof p);
+  cudaMalloc(&dt, tiles.size() * sizeof(int4) + 16);
+  cudaMemcpy(dp, &p, sizeof p, cudaMemcpyHostToDevice);
+  cudaMemcpy(dt, tiles.data(), tiles.size() * sizeof(int4), cudaMemcpyHostToDevice);
+  int rc = lora_tokred_run(dp, dt, (int)tiles.size(), mt, 0);
+  cudaError_t e = cudaDeviceSynchronize();
+  cudaFree(dp); cudaFree(dt);
+  if (rc) return fail("lora tokred rejected");
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   return MENOS_OK;
 }

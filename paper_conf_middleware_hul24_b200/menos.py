@@ -50,6 +50,11 @@ class Stats(C.Structure):
                 ("num_sms", C.c_int)]
 
 
+class KernelStat(C.Structure):
+    _fields_ = [("name", C.c_char * 32), ("launches", C.c_int), ("ms", C.c_double), ("flops", C.c_double),
+                ("bytes", C.c_double)]
+
+
 _lib = None
 
 # (name, restype, argtypes) for every symbol include/menos.h and include/menos_testing.h declare
@@ -72,6 +77,8 @@ SIGNATURES = {
     "menos_set_adapter": (_I, [_P, C.c_int32, _I, _I, _I, C.POINTER(C.c_float)]),
     "menos_get_stats": (_I, [_P, C.POINTER(Stats)]),
     "menos_launch_count": (C.c_ulonglong, []),
+    "menos_profile_enable": (_I, [_I]),
+    "menos_profile_read": (_I, [C.POINTER(KernelStat), _I, C.POINTER(_I)]),
     "menos_sync": (_I, [_P]),
     "menos_last_error": (C.c_char_p, []),
     "menos_test_gemm": (_I, [_I, _I, _I, _I, _P, _I, _P, _I, _P, _I, _P, _I, _I, _PI32, _I, _P, _I, _P, _I, _P, _I,
@@ -79,7 +86,8 @@ SIGNATURES = {
     "menos_test_attention": (_I, [_I, _PI32, _I, _I, _I, _P, _P, _P, _P, _P, _F]),
     "menos_test_rmsnorm": (_I, [_I, _I, _P, _P, _F, _P, _P, _P, _P, _P]),
     "menos_test_batch_tensor": (_I, [_P, _P, _I, _I, _P, C.POINTER(_S)]),
-    "menos_test_small_gemm": (_I, [_P, _P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _I, _F, _I, _I]),
+    "menos_test_lora_rows": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _F]),
+    "menos_test_lora_tokred": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _I, _F, _I]),
     "menos_testing_last_error": (C.c_char_p, []),
 }
 
@@ -242,3 +250,15 @@ class Server:
 
 def launch_count() -> int:
     return int(lib().menos_launch_count())
+
+
+def profile_enable(on: bool = True):
+    check(lib().menos_profile_enable(1 if on else 0))
+
+
+def profile_read() -> dict:
+    arr = (KernelStat * 16)()
+    n = C.c_int()
+    check(lib().menos_profile_read(arr, 16, C.byref(n)))
+    return {arr[i].name.decode(): {"launches": arr[i].launches, "ms": arr[i].ms, "flops": arr[i].flops,
+                                   "bytes": arr[i].bytes} for i in range(n.value)}

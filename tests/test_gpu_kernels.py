@@ -284,3 +284,65 @@ def test_rmsnorm_fwd_bwd(T, d):
     assert maxrel(host(y), ry) < 1e-2
     np.testing.assert_allclose(rstd.cpu().numpy(), rr[:, 0], rtol=1e-5)
     assert maxrel(host(dx), res + O.rmsnorm_bwd(dy, x, g, rr)) < 1e-2
+
+
+def test_lora_rows_shrink_and_du():
+    from paper_conf_middleware_hul24_b200.menos import check
+    T, K, N, r, s = 300, 512, 768, 8, 2.0
+    x, dy = rnd((T, K), 71), rnd((T, N), 72)
+    A = rnd((r, K), 73, 1 / np.sqrt(K))
+    B = rnd((N, r), 74, 0.02)
+    # shrink with B-operand "nk" = A [r, K]; the slot is 16 wide (rows r..15 of the slot table are zero)
+    Aslot = np.zeros((16, K), np.float32); Aslot[:r] = A
+    Ad, xd = dev(Aslot), dev(x)
+    U = torch.zeros(T, 16, dtype=torch.bfloat16, device="cuda")
+    check(lib().menos_test_lora_rows(xd.data_ptr(), Ad.data_ptr(), U.data_ptr(), T, 16, K, K, K, 16, 0, s), testing=True)
+    _, Uref = O.proj_fwd(x, np.zeros((N, K), np.float32), (A, B), s)
+    assert maxrel(host(U)[:, :r], s * Uref) < 1e-2
+    assert not host(U)[:, r:].any()
+    # dU with B-operand "kn" = Bcat [N, 16]
+    Bslot = np.zeros((N, 16), np.float32); Bslot[:, :r] = B
+    Bd, dyd = dev(Bslot), dev(dy)
+    dU = torch.zeros(T, 16, dtype=torch.bfloat16, device="cuda")
+    check(lib().menos_test_lora_rows(dyd.data_ptr(), Bd.data_ptr(), dU.data_ptr(), T, 16, N, N, 16, 16, 1, s), testing=True)
+    assert maxrel(host(dU)[:, :r], s * (dy @ B)) < 1e-2
+
+
+@pytest.mark.parametrize("T", [1, 77, 2048])
+def test_lora_tokred_dA_dB(T):
+    from paper_conf_middleware_hul24_b200.menos import check
+    K, N, r, s = 384, 512, 8, 2.0
+    x, dy = rnd((T, K), 81), rnd((T, N), 82)
+    A, B = rnd((r, K), 83, 1 / np.sqrt(K)), rnd((N, r), 84, 0.02)
+    _, U = O.proj_fwd(x, np.zeros((N, K), np.float32), (A, B), s)
+    Us = np.zeros((T, 16), np.float32); Us[:, :r] = bf16_round(s * U)
+    dUs = np.zeros((T, 16), np.float32); dUs[:, :r] = bf16_round(s * (dy @ B))
+    _, (dA_ref, dB_ref) = O.proj_bwd(dy, x, np.zeros((N, K), np.float32), (A, B), s, U)
+    dyd, Usd, dUsd, xd = dev(dy), dev(Us), dev(dUs), dev(x)
+    dB = torch.empty(N, r, dtype=torch.float32, device="cuda")
+    check(lib().menos_test_lora_tokred(dyd.data_ptr(), Usd.data_ptr(), dB.data_ptr(), N, r, T, N, 16, r, 0, 0, 1.0, 128),
+          testing=True)
+    dA = torch.empty(r, K, dtype=torch.float32, device="cuda")
+    check(lib().menos_test_lora_tokred(dUsd.data_ptr(), xd.data_ptr(), dA.data_ptr(), r, K, T, 16, K, K, 0, 0, 1.0, 16),
+          testing=True)
+    for got, ref in ((dB.cpu().numpy(), dB_ref), (dA.cpu().numpy(), dA_ref)):
+        cos = float(np.sum(got.astype(np.float64) * ref) / (np.linalg.norm(got) * np.linalg.norm(ref) + 1e-30))
+        assert cos > 0.999
+        assert maxrel(got, ref) < 2e-2
+
+
+def test_lora_tokred_gate_up_block_remap():
+    """dB for the gate target reads dgu's interleaved layout [128 gate | 128 up] per f-block."""
+    from paper_conf_middleware_hul24_b200.menos import check
+    T, f, r = 100, 256, 4
+    dg, du = rnd((T, f), 91), rnd((T, f), 92)
+    dgu = np.zeros((T, 2 * f), np.float32)
+    for fb in range(f // 128):
+        dgu[:, fb * 256:fb * 256 + 128] = dg[:, fb * 128:(fb + 1) * 128]
+        dgu[:, fb * 256 + 128:fb * 256 + 256] = du[:, fb * 128:(fb + 1) * 128]
+    U = rnd((T, 16), 93)
+    out = torch.empty(f, r, dtype=torch.float32, device="cuda")
+    dgud, Ud = dev(dgu), dev(U)
+    check(lib().menos_test_lora_tokred(dgud.data_ptr() + 128 * 2, Ud.data_ptr(), out.data_ptr(), f, r, T, 2 * f, 16,
+                                       r, 128, 256, 1.0, 128), testing=True)   # "up" target: base column 128
+    assert maxrel(out.cpu().numpy(), du.T @ U[:, :r]) < 1e-2
