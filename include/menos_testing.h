@@ -53,6 +53,9 @@ MENOS_API int menos_test_lora_rows(const void* A, const void* B, void* C, int M,
 MENOS_API int menos_test_lora_tokred(const void* P, const void* Q, float* C, int M, int N, int T, int ldp, int ldq,
                                      int ldc, int p_blk, int p_blk_stride, float scale, int mt);
 
+/* Select the tcgen05 GEMM variant for subsequent launches: 2 = CTA pair (cta_group::2, default), 1 = single CTA. */
+MENOS_API int menos_test_set_gemm_cta_group(int cta_group);
+
 MENOS_API const char* menos_testing_last_error(void);
 
 #ifdef __cplusplus

@@ -8,9 +8,13 @@
 // * The LoRA expand rides on the same accumulator as extra K steps: A2 = block-diagonal
 //   s*U (row t holds only its client's slot columns), B2 = all clients' B (or A for dX) stacked by slot, so
 //   zero columns contribute exactly 0 and no M tile ever mixes clients' adapters.
-// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread), warps 2-5 = epilogue
+// * CG = 2 (default): a CTA pair (cluster of 2, cta_group::2) computes a 256 x 256 tile with one M=256 UMMA per
+//   K=16 step; each CTA stages its 128 rows of A and its 128-column half of B (halving the smem traffic per SM).
+//   CG = 1: one CTA computes 128 x 256.
+// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread, leader CTA), warps 2-5 = epilogue
 //   (TMEM -> registers -> fused epilogue -> global).  Two TMEM accumulators (2 x 256 fp32 columns) let the
-//   epilogue of tile i overlap the MMAs of tile i+1.  Persistent grid = #SMs.
+//   epilogue of tile i overlap the MMAs of tile i+1.  Persistent grid; tiles rasterised in groups of 16
+//   M-tiles so a wave's A rows and B panels stay L2-resident.
 #include <mutex>
 #include <unordered_map>
 #include <cstring>
@@ -21,12 +25,17 @@ namespace menos {
 
 namespace {
 constexpr int BM = 128, BN = 256, BK = 64;
-constexpr int STAGES = 4;
-constexpr int A_STAGE = BM * BK * 2;   // 16 KB
-constexpr int B_STAGE = BN * BK * 2;   // 32 KB
-constexpr int STAGE_BYTES = A_STAGE + B_STAGE;
 constexpr int NTHREADS = 192;
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024;
+constexpr int GROUP_M = 16;
+
+template <int CG> struct Cfg {
+  static constexpr int A_STAGE = BM * BK * 2;                 // 16 KB (this CTA's 128 rows)
+  static constexpr int B_STAGE = (BN / CG) * BK * 2;          // 32 KB (CG=1) or 16 KB (this CTA's half)
+  static constexpr int STAGE_BYTES = A_STAGE + B_STAGE;
+  static constexpr int STAGES = CG == 1 ? 4 : 6;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024;
+  static constexpr int TILE_M = BM * CG;
+};
 
 struct KParams {
   int M, N, K;
@@ -79,72 +88,119 @@ __device__ __forceinline__ void rope_small(const float (&v)[32], float (&o)[32],
 }
 __device__ __forceinline__ float sigmoidf_(float x) { return 1.0f / (1.0f + __expf(-x)); }
 
-template <int B_MN>
+// grouped rasterisation: groups of GROUP_M m-tiles; inside a group m runs fastest
+__device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int& m, int& n) {
+  const int per_group = GROUP_M * num_n;
+  const int g = t / per_group;
+  const int first = g * GROUP_M;
+  const int gs = min(num_m - first, GROUP_M);
+  const int tin = t - g * per_group;
+  m = first + tin % gs;
+  n = tin / gs;
+}
+
+// extra-K window (LoRA) of tile (m, n): union of the 128-row windows the tile covers
+template <int CG>
+__device__ __forceinline__ void tile_extra(const KParams& p, int m, int n, int& col0, int& n16) {
+  col0 = 0; n16 = 0;
+  if (p.R <= 0 || (p.ntile_extra != nullptr && !p.ntile_extra[n])) return;
+  const int n128 = (p.M + 127) / 128;
+  int lo = 1 << 30, hi = -1;
+#pragma unroll
+  for (int i = 0; i < CG; ++i) {
+    const int mt = m * CG + i;
+    if (mt >= n128) break;
+    const int2 e = p.mtile_extra[mt];
+    if (e.y > 0) { lo = min(lo, e.x); hi = max(hi, e.x + 16 * e.y); }
+  }
+  if (hi > lo) { col0 = lo; n16 = (hi - lo) / 16; }
+}
+
+template <int B_MN, int CG>
 __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmA2, const __grid_constant__ CUtensorMap tmB2,
                const KParams p) {
+  using C = Cfg<CG>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], tfull_bar[2], tempty_bar[2];
+  __shared__ __align__(8) uint64_t full_bar[C::STAGES], empty_bar[C::STAGES], tfull_bar[2], tempty_bar[2];
   __shared__ uint32_t tmem_base_sh;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int num_m = (p.M + BM - 1) / BM, num_n = (p.N + BN - 1) / BN;
+  const uint32_t rank = CG == 2 ? cluster_ctarank() : 0;
+  const bool leader = rank == 0;
+  const int cluster_id = blockIdx.x / CG, n_clusters = gridDim.x / CG;
+  const int num_m = (p.M + C::TILE_M - 1) / C::TILE_M, num_n = (p.N + BN - 1) / BN;
   const int total = num_m * num_n;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA); tma_prefetch(&tmB);
     if (p.R > 0) { tma_prefetch(&tmA2); tma_prefetch(&tmB2); }
-    for (int s = 0; s < STAGES; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
-    for (int s = 0; s < 2; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4); }
+    for (int s = 0; s < C::STAGES; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
+    for (int s = 0; s < 2; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4 * CG); }
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc<512>(&tmem_base_sh);
+  if (warp == 1) {
+    if (CG == 2) tmem_alloc_2sm<512>(&tmem_base_sh);
+    else tmem_alloc<512>(&tmem_base_sh);
+  }
   tc_fence_before();
-  __syncthreads();
+  if (CG == 2) cluster_sync_all(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = tmem_base_sh;
 
   if (warp == 0) {
     if (lane == 0) {
-      // ------------------------------------------------ TMA producer
+      // ------------------------------------------------ TMA producer (both CTAs of a pair)
       int stage = 0; uint32_t phase = 0;
-      for (int t = blockIdx.x; t < total; t += gridDim.x) {
-        const int m = t % num_m, n = t / num_m;
-        int n16 = 0, col0 = 0;
-        if (p.R > 0 && (p.ntile_extra == nullptr || p.ntile_extra[n])) { int2 e = p.mtile_extra[m]; col0 = e.x; n16 = e.y; }
+      for (int t = cluster_id; t < total; t += n_clusters) {
+        int m, n, col0, n16;
+        tile_coords(t, num_m, num_n, m, n);
+        tile_extra<CG>(p, m, n, col0, n16);
         const int nkb = p.kb_main + (n16 + 3) / 4;
+        const int arow = m * C::TILE_M + rank * BM;
+        const int bcol = n * BN + rank * (BN / CG);
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&empty_bar[stage], phase ^ 1);
-          uint8_t* sa = smem + stage * STAGE_BYTES;
-          uint8_t* sb = sa + A_STAGE;
-          mbar_expect_tx(&full_bar[stage], STAGE_BYTES);
+          uint8_t* sa = smem + stage * C::STAGE_BYTES;
+          uint8_t* sb = sa + C::A_STAGE;
+          if (leader) mbar_expect_tx(&full_bar[stage], C::STAGE_BYTES * CG);
           const bool main = kb < p.kb_main;
           const CUtensorMap* ma = main ? &tmA : &tmA2;
           const CUtensorMap* mb = main ? &tmB : &tmB2;
           const int kc = main ? kb * BK : col0 + (kb - p.kb_main) * BK;
-          tma_load_2d(sa, ma, &full_bar[stage], kc, m * BM);
-          if (!B_MN) {
-            tma_load_2d(sb, mb, &full_bar[stage], kc, n * BN);
-          } else {
+          if (CG == 2) {
+            tma_load_2d_2sm(sa, ma, &full_bar[stage], kc, arow);
+            if (!B_MN) {
+              tma_load_2d_2sm(sb, mb, &full_bar[stage], kc, bcol);
+            } else {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) tma_load_2d(sb + j * 8192, mb, &full_bar[stage], n * BN + j * 64, kc);
+              for (int j = 0; j < BN / CG / 64; ++j) tma_load_2d_2sm(sb + j * 8192, mb, &full_bar[stage], bcol + j * 64, kc);
+            }
+          } else {
+            tma_load_2d(sa, ma, &full_bar[stage], kc, arow);
+            if (!B_MN) {
+              tma_load_2d(sb, mb, &full_bar[stage], kc, bcol);
+            } else {
+#pragma unroll
+              for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * 8192, mb, &full_bar[stage], bcol + j * 64, kc);
+            }
           }
-          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      // ------------------------------------------------ MMA issuer (single thread)
-      constexpr uint32_t IDESC = umma_idesc_bf16(BM, BN, B_MN);
+    if (lane == 0 && leader) {
+      // ------------------------------------------------ MMA issuer (single thread of the leader CTA)
+      constexpr uint32_t IDESC = umma_idesc_bf16(BM * CG, BN, B_MN);
       int stage = 0; uint32_t phase = 0;
       int acc = 0; uint32_t acc_phase = 0;
-      for (int t = blockIdx.x; t < total; t += gridDim.x) {
-        const int m = t % num_m, n = t / num_m;
-        int n16 = 0;
-        if (p.R > 0 && (p.ntile_extra == nullptr || p.ntile_extra[n])) n16 = p.mtile_extra[m].y;
+      for (int t = cluster_id; t < total; t += n_clusters) {
+        int m, n, col0, n16;
+        tile_coords(t, num_m, num_n, m, n);
+        tile_extra<CG>(p, m, n, col0, n16);
         const int nkb = p.kb_main + (n16 + 3) / 4;
         mbar_wait(&tempty_bar[acc], acc_phase ^ 1);
         tc_fence_after();
@@ -152,32 +208,36 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&full_bar[stage], phase);
           tc_fence_after();
-          const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-          const uint32_t sb = sa + A_STAGE;
+          const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+          const uint32_t sb = sa + C::A_STAGE;
           int nsteps = 4;
           if (kb >= p.kb_main) { nsteps = n16 - (kb - p.kb_main) * 4; if (nsteps > 4) nsteps = 4; }
           for (int k = 0; k < nsteps; ++k) {
             const uint64_t ad = umma_desc_sw128(sa + k * 32, 16, 1024);
             const uint64_t bd = B_MN ? umma_desc_sw128(sb + k * 2048, 8192, 1024)
                                      : umma_desc_sw128(sb + k * 32, 16, 1024);
-            tc_mma_bf16(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+            if (CG == 2) tc_mma_bf16_2sm(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+            else tc_mma_bf16(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
           }
-          tc_commit(&empty_bar[stage]);
-          if (++stage == STAGES) { stage = 0; phase ^= 1; }
+          if (CG == 2) tc_commit_2sm_mc(&empty_bar[stage], 0x3);
+          else tc_commit(&empty_bar[stage]);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
-        tc_commit(&tfull_bar[acc]);
+        if (CG == 2) tc_commit_2sm_mc(&tfull_bar[acc], 0x3);
+        else tc_commit(&tfull_bar[acc]);
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
     }
   } else {
-    // ------------------------------------------------ epilogue warps 2..5
+    // ------------------------------------------------ epilogue warps 2..5 (both CTAs)
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     int acc = 0; uint32_t acc_phase = 0;
-    for (int t = blockIdx.x; t < total; t += gridDim.x) {
-      const int m = t % num_m, n = t / num_m;
+    for (int t = cluster_id; t < total; t += n_clusters) {
+      int m, n;
+      tile_coords(t, num_m, num_n, m, n);
       mbar_wait(&tfull_bar[acc], acc_phase);
       tc_fence_after();
-      const int row = m * BM + q * 32 + lane;
+      const int row = m * C::TILE_M + rank * BM + q * 32 + lane;
       const bool rok = row < p.M;
       const uint32_t tb = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
       const int n0 = n * BN;
@@ -283,14 +343,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+      if (lane == 0) {
+        if (CG == 2) mbar_arrive_cluster(&tempty_bar[acc], 0);   // the leader's MMA waits for both CTAs
+        else mbar_arrive(&tempty_bar[acc]);
+      }
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
   }
-  __syncthreads();
+  tc_fence_before();
+  if (CG == 2) cluster_sync_all(); else __syncthreads();
   if (warp == 1) {
     tc_fence_after();
-    tmem_dealloc<512>(tmem_base);
+    if (CG == 2) tmem_dealloc_2sm<512>(tmem_base);
+    else tmem_dealloc<512>(tmem_base);
   }
 }
 
@@ -351,23 +416,49 @@ bool get_map(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, ui
   *out = m;
   return true;
 }
+
+template <int B_MN, int CG>
+int launch(const CUtensorMap& mA, const CUtensorMap& mB, const CUtensorMap& mA2, const CUtensorMap& mB2,
+           const KParams& p, int grid, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(gemm_tc_kernel<B_MN, CG>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<CG>::SMEM_BYTES);
+    attr = true;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(NTHREADS);
+  cfg.dynamicSmemBytes = Cfg<CG>::SMEM_BYTES;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = CG; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+  cfg.attrs = at; cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_tc_kernel<B_MN, CG>, mA, mB, mA2, mB2, p);
+  ++g_launch_count;
+  return e == cudaSuccess ? 0 : -3;
+}
 }  // namespace
+
+int g_gemm_cta_group = 2;
 
 int gemm_run(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
   if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;
   if ((a.epi == EPI_SWIGLU_FWD && a.N % 256) || (a.epi == EPI_SWIGLU_BWD && a.N % 128)) return -1;
+  const int CG = g_gemm_cta_group == 1 ? 1 : 2;
+  const uint32_t bbox = BN / CG;  // B rows (K-major) staged per CTA
   CUtensorMap mA, mB, mA2, mB2;
   if (!get_map(&mA, a.A, a.M, a.K, a.lda, BK, BM)) return -2;
   if (!a.b_mn_major) {
-    if (!get_map(&mB, a.B, a.N, a.K, a.ldb, BK, BN)) return -2;
+    if (!get_map(&mB, a.B, a.N, a.K, a.ldb, BK, bbox)) return -2;
   } else {
     if (!get_map(&mB, a.B, a.K, a.N, a.ldb, 64, BK)) return -2;
   }
   if (a.R > 0) {
     if (!get_map(&mA2, a.A2, a.M, a.R, a.lda2, BK, BM)) return -2;
     if (!a.b_mn_major) {
-      if (!get_map(&mB2, a.B2, a.N, a.R, a.ldb2, BK, BN)) return -2;
+      if (!get_map(&mB2, a.B2, a.N, a.R, a.ldb2, BK, bbox)) return -2;
     } else {
       if (!get_map(&mB2, a.B2, a.R, a.N, a.ldb2, 64, BK)) return -2;
     }
@@ -380,19 +471,14 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr;
   p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux;
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
-  const int tiles = ((a.M + BM - 1) / BM) * ((a.N + BN - 1) / BN);
-  int grid = a.num_sms > 0 ? a.num_sms : 148;
-  if (tiles < grid) grid = tiles;
-  static bool attr_set[2] = {false, false};
-  if (a.b_mn_major) {
-    if (!attr_set[1]) { cudaFuncSetAttribute(gemm_tc_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES); attr_set[1] = true; }
-    gemm_tc_kernel<1><<<grid, NTHREADS, SMEM_BYTES, st>>>(mA, mB, mA2, mB2, p);
-  } else {
-    if (!attr_set[0]) { cudaFuncSetAttribute(gemm_tc_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES); attr_set[0] = true; }
-    gemm_tc_kernel<0><<<grid, NTHREADS, SMEM_BYTES, st>>>(mA, mB, mA2, mB2, p);
-  }
-  ++g_launch_count;
-  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+  const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);
+  int sms = a.num_sms > 0 ? a.num_sms : 148;
+  int clusters = sms / CG;
+  if (tiles < clusters) clusters = tiles;
+  if (clusters < 1) clusters = 1;
+  const int grid = clusters * CG;
+  if (CG == 2) return a.b_mn_major ? launch<1, 2>(mA, mB, mA2, mB2, p, grid, st) : launch<0, 2>(mA, mB, mA2, mB2, p, grid, st);
+  return a.b_mn_major ? launch<1, 1>(mA, mB, mA2, mB2, p, grid, st) : launch<0, 1>(mA, mB, mA2, mB2, p, grid, st);
 }
 
 }  // namespace menos

@@ -148,3 +148,10 @@ extern "C" int menos_test_lora_tokred(const void* P, const void* Q, float* C, in
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   return MENOS_OK;
 }
+
+namespace menos { extern int g_gemm_cta_group; }
+extern "C" int menos_test_set_gemm_cta_group(int cg) {
+  if (cg != 1 && cg != 2) return fail("cta_group must be 1 or 2");
+  menos::g_gemm_cta_group = cg;
+  return MENOS_OK;
+}

@@ -53,8 +53,16 @@ def gemm(M, N, K, b_mn, A, B, A2=None, B2=None, R=0, mt=None, epi=0, out=None, r
     check(rc, testing=True)
 
 
+@pytest.fixture(params=[2, 1], ids=["cta_pair", "single_cta"])
+def cta_group(request):
+    from paper_conf_middleware_hul24_b200.menos import check
+    check(lib().menos_test_set_gemm_cta_group(request.param), testing=True)
+    yield request.param
+    check(lib().menos_test_set_gemm_cta_group(2), testing=True)
+
+
 @pytest.mark.parametrize("M,N,K", [(128, 256, 64), (300, 512, 320), (1000, 768, 1000), (2048, 4096, 4096)])
-def test_gemm_fwd_kmajor(M, N, K):
+def test_gemm_fwd_kmajor(M, N, K, cta_group):
     x, W = rnd((M, K), 1), rnd((N, K), 2, 0.02)
     out = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
     gemm(M, N, K, 0, dev(x), dev(W), out=out)
@@ -63,7 +71,7 @@ def test_gemm_fwd_kmajor(M, N, K):
 
 
 @pytest.mark.parametrize("M,Nred,Kout", [(256, 384, 512), (333, 640, 320), (2048, 11008, 4096)])
-def test_gemm_dx_mnmajor(M, Nred, Kout):
+def test_gemm_dx_mnmajor(M, Nred, Kout, cta_group):
     dy, W = rnd((M, Nred), 3), rnd((Nred, Kout), 4, 0.02)
     out = torch.empty(M, Kout, dtype=torch.bfloat16, device="cuda")
     gemm(M, Kout, Nred, 1, dev(dy), dev(W), out=out)
@@ -73,11 +81,11 @@ def test_gemm_dx_mnmajor(M, Nred, Kout):
     assert maxrel(host(out), ref2) < 1e-2
 
 
-def test_gemm_persistent_many_tiles_small_grid():
+def test_gemm_persistent_many_tiles_small_grid(cta_group):
     M, N, K = 1024, 1024, 256
     x, W = rnd((M, K), 5), rnd((N, K), 6, 0.05)
     out = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
-    gemm(M, N, K, 0, dev(x), dev(W), out=out, num_sms=3)     # 32 tiles on 3 CTAs: TMEM double buffer wraps
+    gemm(M, N, K, 0, dev(x), dev(W), out=out, num_sms=4)     # 16-32 tiles on 2-4 CTAs: TMEM double buffer wraps
     ref, _ = O.proj_fwd(x, W, None, 1.0)
     assert maxrel(host(out), ref) < 1e-2
 
@@ -116,7 +124,7 @@ def _lora_case(seed, Ks, Ns, clients):
     return x, W, As, Bs, Ucat, Bcat, Acat, R, mt
 
 
-def test_gemm_segmented_lora_expand_fwd():
+def test_gemm_segmented_lora_expand_fwd(cta_group):
     clients = [(100, 8, 2.0), (200, 4, 2.0), (77, 16, 2.0)]
     x, W, As, Bs, Ucat, Bcat, Acat, R, mt = _lora_case(11, 256, 512, clients)
     T = x.shape[0]
@@ -130,7 +138,7 @@ def test_gemm_segmented_lora_expand_fwd():
         t0 += Tc
 
 
-def test_gemm_segmented_lora_expand_dx():
+def test_gemm_segmented_lora_expand_dx(cta_group):
     clients = [(130, 8, 2.0), (126, 16, 2.0)]
     x, W, As, Bs, Ucat, Bcat, Acat, R, mt = _lora_case(12, 320, 384, clients)
     T = x.shape[0]
