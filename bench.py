@@ -356,7 +356,7 @@ def main():
     ap.add_argument("--workload", default="cfg1_7b_x4")
     ap.add_argument("--layers", type=int, default=None, help="truncate depth (debug only; not a bench value)")
     ap.add_argument("--arena-gb", type=float, default=80.0)
-    ap.add_argument("--cpu-layers", type=int, default=2)
+    ap.add_argument("--cpu-layers", type=int, default=6)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

@@ -56,6 +56,10 @@ MENOS_API int menos_test_lora_tokred(const void* P, const void* Q, float* C, int
 /* Select the tcgen05 GEMM variant for subsequent launches: 2 = CTA pair (cta_group::2, default), 1 = single CTA. */
 MENOS_API int menos_test_set_gemm_cta_group(int cta_group);
 
+/* Time `iters` back-to-back launches of one GEMM (ld = natural) with CUDA events; *ms_out = ms per launch. */
+MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A, const void* B, void* out, int epi,
+                                   const void* aux, int iters, float* ms_out);
+
 MENOS_API const char* menos_testing_last_error(void);
 
 #ifdef __cplusplus

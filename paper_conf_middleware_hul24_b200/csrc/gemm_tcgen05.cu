@@ -32,7 +32,7 @@ template <int CG> struct Cfg {
   static constexpr int A_STAGE = BM * BK * 2;                 // 16 KB (this CTA's 128 rows)
   static constexpr int B_STAGE = (BN / CG) * BK * 2;          // 32 KB (CG=1) or 16 KB (this CTA's half)
   static constexpr int STAGE_BYTES = A_STAGE + B_STAGE;
-  static constexpr int STAGES = CG == 1 ? 4 : 6;
+  static constexpr int STAGES = CG == 1 ? 4 : 7;
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024;
   static constexpr int TILE_M = BM * CG;
 };

@@ -155,3 +155,32 @@ extern "C" int menos_test_set_gemm_cta_group(int cg) {
   menos::g_gemm_cta_group = cg;
   return MENOS_OK;
 }
+
+// Time `iters` back-to-back launches of one plain GEMM (out = A B^T or A B) with CUDA events (tuning aid).
+extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A, const void* B, void* out, int epi,
+                                    const void* aux, int iters, float* ms_out) {
+  GemmArgs a;
+  memset(&a, 0, sizeof a);
+  a.M = M; a.N = N; a.K = K; a.b_mn_major = b_mn;
+  a.A = (const bf16*)A; a.lda = K; a.B = (const bf16*)B; a.ldb = b_mn ? N : K;
+  a.epi = epi; a.out = (bf16*)out; a.ldo = epi == EPI_SWIGLU_BWD ? 2 * N : N;
+  a.out2 = (bf16*)out; a.ldo2 = N / 2; a.aux = (const bf16*)aux; a.ldaux = 2 * N;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  a.num_sms = sms;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0); cudaEventCreate(&e1);
+  int rc = gemm_run(a, 0);
+  cudaEventRecord(e0, 0);
+  for (int i = 0; i < iters && rc == 0; ++i) rc = gemm_run(a, 0);
+  cudaEventRecord(e1, 0);
+  cudaError_t e = cudaEventSynchronize(e1);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventDestroy(e0); cudaEventDestroy(e1);
+  if (rc) return fail("gemm rejected");
+  if (e != cudaSuccess) return fail(cudaGetErrorString(e));
+  *ms_out = ms / iters;
+  return MENOS_OK;
+}
