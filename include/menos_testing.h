@@ -21,8 +21,9 @@ extern "C" {
  *   out[M, N] = epi( A[M, K] . B^T  +  A2[M, window] . B2[window]^T )
  *   b_mn = 0: B is [N, K] row-major (ldb); b_mn = 1: B is [K, N] row-major (dX form).  B2 follows B's form
  *   with R columns / rows.  mtile_extra (host, 2 ints per 128-row tile: col_start, n16) selects each tile's
- *   extra-K window; R = 0 disables it.  epi: 0 store, 1 +resid, 2 RoPE (head_dim, rope_cols, pos, theta),
- *   3 SwiGLU fwd (out = gu, out2 = a), 4 SwiGLU bwd (aux = saved gu, out = dgu).  All bf16, device. */
+ *   extra-K window; R = 0 disables it.  epi: 0 store, 1 +resid (resid and out fp32: the residual stream),
+ *   2 RoPE (head_dim, rope_cols, pos, theta), 3 SwiGLU fwd (out = gu, out2 = a), 4 SwiGLU bwd (aux = saved gu,
+ *   out = dgu).  Operands bf16, device. */
 MENOS_API int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int lda, const void* B, int ldb, const void* A2,
                     int lda2, const void* B2, int ldb2, int R, const int32_t* mtile_extra, int epi, void* out, int ldo,
                     const void* resid, int ldr, void* out2, int ldo2, const void* aux, int ldaux, int head_dim,
@@ -34,9 +35,10 @@ MENOS_API int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int 
 MENOS_API int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, int Hkv, int hd, const void* qkv, void* O,
                          float* lse, const void* dO, void* dqkv, float theta);
 
-/* RMSNorm forward (y, rstd) and backward (dx = resid + norm_bwd(dy)); g fp32 [d].  Device buffers. */
-MENOS_API int menos_test_rmsnorm(int T, int d, const void* x, const float* g, float eps, void* y, float* rstd, const void* dy,
-                       const void* resid, void* dx);
+/* RMSNorm forward (y bf16, rstd) of the fp32 residual stream x, and backward dx = resid + norm_bwd(dy) with
+ * dy bf16, resid / dx fp32 and dxb = bf16(dx) (optional); g fp32 [d].  Device buffers. */
+MENOS_API int menos_test_rmsnorm(int T, int d, const float* x, const float* g, float eps, void* y, float* rstd,
+                                 const void* dy, const float* resid, float* dx, void* dxb);
 
 /* Copy one saved intermediate of a live SAVE batch to host (debugging / white-box tests).
  * which: 0 x, 1 xn, 2 qkv, 3 O, 4 h, 5 hn, 6 gu, 7 a, 8 U_qkv, 9 U_o, 10 U_gu, 11 U_down (bf16), 12 lse (fp32 [H,T]).

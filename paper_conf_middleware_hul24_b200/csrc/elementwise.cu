@@ -10,82 +10,101 @@ unsigned long long g_launch_count = 0;
 
 namespace {
 
+// 8 consecutive fp32 values / bf16 values <-> registers
+__device__ __forceinline__ void ld8f(const float* p, float (&v)[8]) {
+  const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+__device__ __forceinline__ void st8f(float* p, const float (&v)[8]) {
+  reinterpret_cast<float4*>(p)[0] = make_float4(v[0], v[1], v[2], v[3]);
+  reinterpret_cast<float4*>(p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+}
+__device__ __forceinline__ void ld8b(const bf16* p, float (&v)[8]) {
+  const uint4 u = *reinterpret_cast<const uint4*>(p);
+  float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), e = unpack_bf16x2(u.w);
+  v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y; v[4] = c.x; v[5] = c.y; v[6] = e.x; v[7] = e.y;
+}
+__device__ __forceinline__ void st8b(bf16* p, const float (&v)[8]) {
+  *reinterpret_cast<uint4*>(p) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                            pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+}
+
 // ------------------------------------------------------------------ RMSNorm forward
-// y = x * rstd * g, rstd = rsqrt(mean(x^2) + eps); x, y bf16 [T, d]; g fp32 [d]; d % 8 == 0
-__global__ void rmsnorm_fwd_kernel(const bf16* __restrict__ x, const float* __restrict__ g, bf16* __restrict__ y,
+// y = x * rstd * g, rstd = rsqrt(mean(x^2) + eps); x fp32 residual stream [T, d]; y bf16 (GEMM operand);
+// g fp32 [d]; d % 8 == 0
+__global__ void rmsnorm_fwd_kernel(const float* __restrict__ x, const float* __restrict__ g, bf16* __restrict__ y,
                                    float* __restrict__ rstd, int T, int d, float eps) {
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= T) return;
-  const uint4* xr = reinterpret_cast<const uint4*>(x + (size_t)warp * d);
-  const int nv = d >> 3;
+  const float* xr = x + (size_t)warp * d;
   float ss = 0.f;
-  for (int i = lane; i < nv; i += 32) {
-    uint4 u = xr[i];
-    uint32_t w[4] = {u.x, u.y, u.z, u.w};
+  for (int i = lane * 8; i < d; i += 256) {
+    float v[8];
+    ld8f(xr + i, v);
 #pragma unroll
-    for (int k = 0; k < 4; ++k) { float2 f = unpack_bf16x2(w[k]); ss += f.x * f.x + f.y * f.y; }
+    for (int k = 0; k < 8; ++k) ss += v[k] * v[k];
   }
   ss = warp_sum(ss);
   const float r = rsqrtf(ss / (float)d + eps);
   if (lane == 0) rstd[warp] = r;
-  uint4* yr = reinterpret_cast<uint4*>(y + (size_t)warp * d);
-  const float4* g4 = reinterpret_cast<const float4*>(g);
-  for (int i = lane; i < nv; i += 32) {
-    uint4 u = xr[i];
-    float4 ga = g4[2 * i], gb = g4[2 * i + 1];
-    float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z), f3 = unpack_bf16x2(u.w);
-    uint4 o;
-    o.x = pack_bf16x2(f0.x * r * ga.x, f0.y * r * ga.y);
-    o.y = pack_bf16x2(f1.x * r * ga.z, f1.y * r * ga.w);
-    o.z = pack_bf16x2(f2.x * r * gb.x, f2.y * r * gb.y);
-    o.w = pack_bf16x2(f3.x * r * gb.z, f3.y * r * gb.w);
-    yr[i] = o;
+  bf16* yr = y + (size_t)warp * d;
+  for (int i = lane * 8; i < d; i += 256) {
+    float v[8], gg[8];
+    ld8f(xr + i, v);
+    ld8f(g + i, gg);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = v[k] * r * gg[k];
+    st8b(yr + i, v);
   }
 }
 
 // ------------------------------------------------------------------ RMSNorm backward (+ residual)
-// dx = resid + rstd*(gh - xh*mean(gh*xh)),  gh = dy*g,  xh = x*rstd
-__global__ void rmsnorm_bwd_kernel(const bf16* __restrict__ dy, const bf16* __restrict__ x,
+// dx = resid + rstd*(gh - xh*mean(gh*xh)),  gh = dy*g,  xh = x*rstd.   dy bf16 (GEMM output), x / resid / dx
+// fp32 (residual streams); dxb = bf16 copy of dx for the next dX GEMM's A operand (optional).
+__global__ void rmsnorm_bwd_kernel(const bf16* __restrict__ dy, const float* __restrict__ x,
                                    const float* __restrict__ g, const float* __restrict__ rstd,
-                                   const bf16* __restrict__ resid, bf16* __restrict__ dx, int T, int d) {
+                                   const float* __restrict__ resid, float* __restrict__ dx, bf16* __restrict__ dxb,
+                                   int T, int d) {
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (warp >= T) return;
   const size_t ro = (size_t)warp * d;
-  const uint4* dyr = reinterpret_cast<const uint4*>(dy + ro);
-  const uint4* xr = reinterpret_cast<const uint4*>(x + ro);
-  const float4* g4 = reinterpret_cast<const float4*>(g);
-  const int nv = d >> 3;
   const float r = rstd[warp];
   float dot = 0.f;
-  for (int i = lane; i < nv; i += 32) {
-    uint4 a = dyr[i], b = xr[i];
-    float4 ga = g4[2 * i], gb = g4[2 * i + 1];
-    float gg[8] = {ga.x, ga.y, ga.z, ga.w, gb.x, gb.y, gb.z, gb.w};
-    uint32_t wa[4] = {a.x, a.y, a.z, a.w}, wb[4] = {b.x, b.y, b.z, b.w};
+  for (int i = lane * 8; i < d; i += 256) {
+    float a[8], b[8], gg[8];
+    ld8b(dy + ro + i, a);
+    ld8f(x + ro + i, b);
+    ld8f(g + i, gg);
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      float2 fa = unpack_bf16x2(wa[k]), fb = unpack_bf16x2(wb[k]);
-      dot += fa.x * gg[2 * k] * fb.x + fa.y * gg[2 * k + 1] * fb.y;
-    }
+    for (int k = 0; k < 8; ++k) dot += a[k] * gg[k] * b[k];
   }
   dot = warp_sum(dot);
   const float mean = dot * r / (float)d;  // mean(gh * xh) = r * mean(gh * x)
-  const uint4* rr = reinterpret_cast<const uint4*>(resid + ro);
-  uint4* out = reinterpret_cast<uint4*>(dx + ro);
-  for (int i = lane; i < nv; i += 32) {
-    uint4 a = dyr[i], b = xr[i], c = rr[i];
-    float4 ga = g4[2 * i], gb = g4[2 * i + 1];
-    float gg[8] = {ga.x, ga.y, ga.z, ga.w, gb.x, gb.y, gb.z, gb.w};
-    uint32_t wa[4] = {a.x, a.y, a.z, a.w}, wb[4] = {b.x, b.y, b.z, b.w}, wc[4] = {c.x, c.y, c.z, c.w};
-    uint32_t wo[4];
+  for (int i = lane * 8; i < d; i += 256) {
+    float a[8], b[8], c[8], gg[8], o[8];
+    ld8b(dy + ro + i, a);
+    ld8f(x + ro + i, b);
+    ld8f(resid + ro + i, c);
+    ld8f(g + i, gg);
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      float2 fa = unpack_bf16x2(wa[k]), fb = unpack_bf16x2(wb[k]), fc = unpack_bf16x2(wc[k]);
-      const float o0 = fc.x + r * (fa.x * gg[2 * k] - fb.x * r * mean);
-      const float o1 = fc.y + r * (fa.y * gg[2 * k + 1] - fb.y * r * mean);
-      wo[k] = pack_bf16x2(o0, o1);
-    }
-    out[i] = make_uint4(wo[0], wo[1], wo[2], wo[3]);
+    for (int k = 0; k < 8; ++k) o[k] = c[k] + r * (a[k] * gg[k] - b[k] * r * mean);
+    st8f(dx + ro + i, o);
+    if (dxb) st8b(dxb + ro + i, o);
+  }
+}
+
+__global__ void f32_to_bf16_kernel(const float* __restrict__ s, bf16* __restrict__ d, long long n8) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n8; i += (long long)gridDim.x * blockDim.x) {
+    float v[8];
+    ld8f(s + 8 * i, v);
+    st8b(d + 8 * i, v);
+  }
+}
+__global__ void bf16_to_f32_vec_kernel(const bf16* __restrict__ s, float* __restrict__ d, long long n8) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n8; i += (long long)gridDim.x * blockDim.x) {
+    float v[8];
+    ld8b(s + 8 * i, v);
+    st8f(d + 8 * i, v);
   }
 }
 
@@ -161,19 +180,31 @@ __global__ void bf16_to_f32_kernel(const bf16* __restrict__ s, float* __restrict
 
 #define LAUNCH_CHECK() (++g_launch_count, cudaPeekAtLastError() == cudaSuccess ? 0 : -3)
 
-int rmsnorm_fwd(const bf16* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st) {
+int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
   const int warps = 8;
   rmsnorm_fwd_kernel<<<(T + warps - 1) / warps, warps * 32, 0, st>>>(x, g, y, rstd, T, d, eps);
   return LAUNCH_CHECK();
 }
-int rmsnorm_bwd(const bf16* dy, const bf16* x, const float* g, const float* rstd, const bf16* resid, bf16* dx, int T,
-                int d, cudaStream_t st) {
+int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
+                bf16* dxb, int T, int d, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
   const int warps = 8;
-  rmsnorm_bwd_kernel<<<(T + warps - 1) / warps, warps * 32, 0, st>>>(dy, x, g, rstd, resid, dx, T, d);
+  rmsnorm_bwd_kernel<<<(T + warps - 1) / warps, warps * 32, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d);
+  return LAUNCH_CHECK();
+}
+int convert_f32_to_bf16(const float* src, bf16* dst, long long n, cudaStream_t st) {
+  if (n <= 0) return 0;
+  if (n % 8) return -1;
+  f32_to_bf16_kernel<<<1184, 256, 0, st>>>(src, dst, n / 8);
+  return LAUNCH_CHECK();
+}
+int convert_bf16_to_f32_vec(const bf16* src, float* dst, long long n, cudaStream_t st) {
+  if (n <= 0) return 0;
+  if (n % 8) return -1;
+  bf16_to_f32_vec_kernel<<<1184, 256, 0, st>>>(src, dst, n / 8);
   return LAUNCH_CHECK();
 }
 int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st) {

@@ -45,7 +45,8 @@ struct KParams {
   const uint8_t* ntile_extra;
   int epi;
   bf16* out; int ldo;
-  const bf16* resid; int ldr;
+  const float* resid; int ldr;
+  float* outf;
   bf16* out2; int ldo2;
   const bf16* aux; int ldaux;
   const float2* rope_cs;
@@ -241,20 +242,29 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const bool rok = row < p.M;
       const uint32_t tb = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
       const int n0 = n * BN;
-      if (p.epi == EPI_STORE || p.epi == EPI_RESID) {
+      if (p.epi == EPI_STORE) {
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
+        }
+      } else if (p.epi == EPI_RESID) {
+        // fp32 residual stream: outf = acc + resid
         for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
           float v[32];
           tmem_ld32(tb + c * 32, v);
           if (rok) {
-            if (p.epi == EPI_RESID) {
-              float r[32];
-              load32(p.resid + (size_t)row * p.ldr + col, r);
+            const float4* r4 = reinterpret_cast<const float4*>(p.resid + (size_t)row * p.ldr + col);
+            float4* o4 = reinterpret_cast<float4*>(p.outf + (size_t)row * p.ldo + col);
 #pragma unroll
-              for (int j = 0; j < 32; ++j) v[j] += r[j];
+            for (int q = 0; q < 8; ++q) {
+              const float4 r = r4[q];
+              o4[q] = make_float4(v[4 * q] + r.x, v[4 * q + 1] + r.y, v[4 * q + 2] + r.z, v[4 * q + 3] + r.w);
             }
-            store32(p.out + (size_t)row * p.ldo + col, v);
           }
         }
       } else if (p.epi == EPI_ROPE) {
@@ -468,7 +478,7 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   KParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.kb_main = (a.K + BK - 1) / BK;
   p.R = a.R; p.mtile_extra = a.mtile_extra; p.ntile_extra = a.ntile_extra;
-  p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr;
+  p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr; p.outf = a.outf;
   p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux;
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
   const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);

@@ -17,7 +17,7 @@ extern unsigned long long g_launch_count;
 // ---------------------------------------------------------------- tcgen05 GEMM
 enum EpiMode : int {
   EPI_STORE = 0,       // out = bf16(acc)
-  EPI_RESID = 1,       // out = bf16(acc + resid)
+  EPI_RESID = 1,       // outf = acc + residf   (fp32 residual stream)
   EPI_ROPE = 2,        // columns < rope_cols rotated by RoPE at pos[row]; out = bf16
   EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu), out2 = bf16(silu(g) u)
   EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
@@ -37,7 +37,8 @@ struct GemmArgs {
   // epilogue
   int epi;
   bf16* out; int ldo;
-  const bf16* resid; int ldr;      // EPI_RESID
+  const float* resid; int ldr;     // EPI_RESID: fp32 residual in, fp32 `outf` out (ld = ldo)
+  float* outf;
   bf16* out2; int ldo2;            // EPI_SWIGLU_FWD: a
   const bf16* aux; int ldaux;      // EPI_SWIGLU_BWD: saved gu
   const float2* rope_cs;           // EPI_ROPE: [max_pos][hd/2] (cos, sin)
@@ -69,10 +70,13 @@ void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out
 void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out);
 
 // ---------------------------------------------------------------- norms / elementwise
-int rmsnorm_fwd(const bf16* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st);
-// dx = resid + rstd*(gh - xh*mean(gh*xh)), gh = dy*g, xh = x*rstd
-int rmsnorm_bwd(const bf16* dy, const bf16* x, const float* g, const float* rstd, const bf16* resid, bf16* dx,
-                int T, int d, cudaStream_t st);
+// residual streams (x, h forward; dy, dh backward) are fp32; GEMM operands (xn, hn, dxn ...) are bf16
+int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st);
+// dx = resid + rstd*(gh - xh*mean(gh*xh)), gh = dy*g, xh = x*rstd; dxb (optional) = bf16(dx)
+int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
+                bf16* dxb, int T, int d, cudaStream_t st);
+int convert_f32_to_bf16(const float* src, bf16* dst, long long n, cudaStream_t st);       // n % 8 == 0
+int convert_bf16_to_f32_vec(const bf16* src, float* dst, long long n, cudaStream_t st);   // n % 8 == 0
 int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st);
 
 // ---------------------------------------------------------------- attention (varlen causal, GQA)

@@ -224,7 +224,8 @@ struct ColAlloc {
 // batch
 // =====================================================================================================
 struct LayerSave {
-  bf16 *x, *xn, *qkv, *O, *h, *hn, *gu, *a;
+  float *x, *h;                       // fp32 residual stream (layer input, post-attention residual)
+  bf16 *xn, *qkv, *O, *hn, *gu, *a;   // bf16 GEMM operands / attention inputs
   float *rstd1, *rstd2, *lse;
   bf16* U[NG];
 };
@@ -253,7 +254,6 @@ struct menos_batch {
   // saved activations (SAVE) or x_c copy (NOGRAD)
   uint8_t* slab = nullptr;
   std::vector<LayerSave> L;
-  bf16* xout = nullptr;
 };
 
 // =====================================================================================================
@@ -630,7 +630,8 @@ extern "C" int menos_unregister_client(menos_server* s, int32_t id) {
 // saved bytes per token per layer in SAVE mode (excluding the LoRA U share)
 static size_t saved_bytes_per_token_layer(const Dims& D, bool save_a) {
   size_t b = 0;
-  b += (size_t)D.d * 2 * 4;        // x, xn, h, hn
+  b += (size_t)D.d * 4 * 2;        // x, h (fp32 residual stream)
+  b += (size_t)D.d * 2 * 2;        // xn, hn
   b += (size_t)D.Nqkv * 2;         // qkv
   b += (size_t)D.Nq * 2;           // O
   b += (size_t)2 * D.fpad * 2;     // gu
@@ -640,7 +641,8 @@ static size_t saved_bytes_per_token_layer(const Dims& D, bool save_a) {
 }
 static size_t scratch_bytes_per_token(const Dims& D, int R_sum) {
   size_t b = 0;
-  b += (size_t)D.d * 2 * 5;          // dy, dx, dhn, dh, xout
+  b += (size_t)D.d * 4 * 4;          // dyf, dxf, dhf, xout (fp32)
+  b += (size_t)D.d * 2 * 5;          // dyb, dxb, dhb, dhn, io staging (bf16)
   b += (size_t)D.Nq * 2;             // dO
   b += (size_t)D.Nqkv * 2;           // dqkv
   b += (size_t)2 * D.fpad * 2;       // dgu
@@ -666,7 +668,7 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
   size_t ush = 0;
   for (int g = 0; g < NG; ++g) ush += (size_t)c.width[g] * 2;
   const size_t T = (size_t)n_tokens;
-  if (fwd_bytes) *fwd_bytes = T * ((saved_bytes_per_token_layer(D, save_a) + ush) * s->n_layers + (size_t)D.d * 2);
+  if (fwd_bytes) *fwd_bytes = T * ((saved_bytes_per_token_layer(D, save_a) + ush) * s->n_layers);
   int rsum = 0;
   for (int g = 0; g < NG; ++g) rsum += c.width[g];
   if (bwd_bytes) *bwd_bytes = T * scratch_bytes_per_token(D, rsum);
@@ -799,7 +801,9 @@ extern "C" const char* menos_last_error(void) { return tl_err.c_str(); }
 // batch construction (BatchPacker)
 // =====================================================================================================
 struct Scratch {
-  bf16 *dy, *dx, *dhn, *dh, *dO, *dqkv, *dgu, *a, *xout;
+  float *dyf, *dxf, *dhf, *xout;     // fp32 residual streams (gradient ping-pong, dh, forward output)
+  bf16 *dyb, *dxb, *dhb;             // bf16 copies (A operands of the dX GEMMs, LoRA dY)
+  bf16 *dhn, *dO, *dqkv, *dgu, *a, *io;  // io: bf16 staging of x_c / x_s / g_c / g_s
   float* Dsum;
   bf16* dU[NG];
 };
@@ -857,14 +861,14 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   size_t per_layer = 0;
   auto A = [&](size_t n) { per_layer += align_up(n, 256); };
   if (save) {
-    A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x, xn, rstd1
+    A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x (fp32), xn, rstd1
     A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
-    A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h, hn, rstd2
+    A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h (fp32), hn, rstd2
     A((size_t)T * 2 * D.fpad * 2);                                            // gu
     if (b->save_a) A((size_t)T * D.fpad * 2);
     for (int g = 0; g < NG; ++g) if (b->g_active[g]) A((size_t)T * b->R_used[g] * 2);
   }
-  const size_t slab_bytes = save ? per_layer * Ls : align_up((size_t)T * D.d * 2, 256);
+  const size_t slab_bytes = save ? per_layer * Ls : align_up((size_t)T * D.d * 4, 256);
   // ---- metadata blob
   std::vector<uint8_t> blob;
   auto put = [&](const void* p, size_t n) {
@@ -914,15 +918,15 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
     for (int l = 0; l < Ls; ++l) {
       LayerSave& S = b->L[l];
-      S.x = (bf16*)take((size_t)T * D.d * 2); S.xn = (bf16*)take((size_t)T * D.d * 2); S.rstd1 = (float*)take((size_t)T * 4);
+      S.x = (float*)take((size_t)T * D.d * 4); S.xn = (bf16*)take((size_t)T * D.d * 2); S.rstd1 = (float*)take((size_t)T * 4);
       S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2); S.lse = (float*)take((size_t)D.H * T * 4);
-      S.h = (bf16*)take((size_t)T * D.d * 2); S.hn = (bf16*)take((size_t)T * D.d * 2); S.rstd2 = (float*)take((size_t)T * 4);
+      S.h = (float*)take((size_t)T * D.d * 4); S.hn = (bf16*)take((size_t)T * D.d * 2); S.rstd2 = (float*)take((size_t)T * 4);
       S.gu = (bf16*)take((size_t)T * 2 * D.fpad * 2);
       S.a = b->save_a ? (bf16*)take((size_t)T * D.fpad * 2) : sc.a;
       for (int g = 0; g < NG; ++g) S.U[g] = b->g_active[g] ? (bf16*)take((size_t)T * b->R_used[g] * 2) : nullptr;
     }
   } else {
-    b->L[0].x = (bf16*)slab;  // x_c copy (only the forward input is cached)
+    b->L[0].x = (float*)slab;  // x_c copy (only the forward input is cached)
   }
 
   // ---- LoRA side-contraction problem lists (need buffer pointers: SAVE layout, or the NOGRAD layer set)
@@ -952,7 +956,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   };
   for (int l = 0; l < Ls; ++l) {
     const LayerSave& S = save ? b->L[l] : *ng;
-    bf16* dyl = ((Ls - 1 - l) % 2 == 0) ? sc.dy : sc.dx;  // layer l's incoming gradient buffer
+    bf16* dyl = ((Ls - 1 - l) % 2 == 0) ? sc.dyb : sc.dxb;  // bf16 copy of layer l's incoming gradient
     for (int g = 0; g < NG; ++g) {
       if (!b->g_active[g]) continue;
       const int R = b->R_used[g];
@@ -962,7 +966,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       bf16* U = S.U[g];
       switch (g) {
         case GQKV: X = S.xn; ldx = D.d; dY = sc.dqkv; ldy = D.Nqkv; break;
-        case GO: X = S.O; ldx = D.Nq; dY = sc.dh; ldy = D.d; break;
+        case GO: X = S.O; ldx = D.Nq; dY = sc.dhb; ldy = D.d; break;
         case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = 2 * D.fpad; break;
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
@@ -1045,12 +1049,14 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   for (int g = 0; g < NG; ++g) rsum += R_used[g];
   size_t need = 0;
   auto A = [&](size_t n) { need += align_up(n, 256); };
-  A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.d * 2);
+  const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
+  A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout
+  A(db); A(db); A(db); A(db); A(db);                                          // dyb, dxb, dhb, dhn, io
   A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * 2 * D.fpad * 2); A((size_t)T * D.fpad * 2);
-  A((size_t)T * D.d * 2); A((size_t)D.H * T * 4);
+  A((size_t)D.H * T * 4);
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
-  // NOGRAD forward layer set (x ping-pong handled by xout/dx; intermediates reuse the grad buffers)
-  A((size_t)T * D.d * 2); A((size_t)T * D.d * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
+  // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
+  A(db); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
   A((size_t)T * 2 * D.fpad * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   if (need > s->scratch_bytes) {
@@ -1061,11 +1067,12 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   }
   uint8_t* p = s->scratch;
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
-  sc.dy = (bf16*)take((size_t)T * D.d * 2); sc.dx = (bf16*)take((size_t)T * D.d * 2);
-  sc.dhn = (bf16*)take((size_t)T * D.d * 2); sc.dh = (bf16*)take((size_t)T * D.d * 2);
+  sc.dyf = (float*)take(df); sc.dxf = (float*)take(df); sc.dhf = (float*)take(df); sc.xout = (float*)take(df);
+  sc.dyb = (bf16*)take(db); sc.dxb = (bf16*)take(db); sc.dhb = (bf16*)take(db); sc.dhn = (bf16*)take(db);
+  sc.io = (bf16*)take(db);
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
   sc.dgu = (bf16*)take((size_t)T * 2 * D.fpad * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
-  sc.xout = (bf16*)take((size_t)T * D.d * 2); sc.Dsum = (float*)take((size_t)D.H * T * 4);
+  sc.Dsum = (float*)take((size_t)D.H * T * 4);
   for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
   return MENOS_OK;
 }
@@ -1075,7 +1082,7 @@ static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scr
   const Dims& D = s->D;
   uint8_t* p = (uint8_t*)(sc.dU[NG - 1]) + align_up((size_t)T * R_used[NG - 1] * 2, 256);
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
-  S.xn = (bf16*)take((size_t)T * D.d * 2); S.h = (bf16*)take((size_t)T * D.d * 2);
+  S.xn = (bf16*)take((size_t)T * D.d * 2); S.h = (float*)take((size_t)T * D.d * 4);
   S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
   S.gu = (bf16*)take((size_t)2 * T * D.fpad * 2); S.lse = (float*)take((size_t)D.H * T * 4);
   S.rstd1 = (float*)take((size_t)T * 8); S.rstd2 = S.rstd1 + T;
@@ -1106,13 +1113,13 @@ static GemmArgs gemm_base(menos_server* s) {
 }
 
 // forward of layer l: x -> y; S holds the destinations of every intermediate
-static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, bf16* y, const LayerSave& S,
+static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x, float* y, const LayerSave& S,
                          bool use_lists, cudaStream_t st) {
   const Dims& D = s->D;
   const auto& W = s->W[l];
   const int T = b->T;
-  // A1: RMSNorm1
-  { ProfScope ps(PC_NORM, 0, (double)T * (4.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st)); }
+  // A1: RMSNorm1 (fp32 residual in, bf16 GEMM operand out)
+  { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st)); }
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
   if (b->g_active[GQKV]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
@@ -1151,11 +1158,11 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
       a.R = b->R_used[GO]; a.A2 = S.U[GO]; a.lda2 = a.R; a.B2 = s->Bcat[GO][l]; a.ldb2 = s->cols[GO].cap;
       a.mtile_extra = b->d_mtile[GO];
     }
-    a.epi = EPI_RESID; a.out = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
+    a.epi = EPI_RESID; a.outf = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A5: RMSNorm2
-  { ProfScope ps(PC_NORM, 0, (double)T * (4.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st)); }
+  { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st)); }
   // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
   if (b->g_active[GGU]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
@@ -1183,15 +1190,16 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const bf16* x, 
       a.R = b->R_used[GD]; a.A2 = S.U[GD]; a.lda2 = a.R; a.B2 = s->Bcat[GD][l]; a.ldb2 = s->cols[GD].cap;
       a.mtile_extra = b->d_mtile[GD];
     }
-    a.epi = EPI_RESID; a.out = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
+    a.epi = EPI_RESID; a.outf = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   return MENOS_OK;
 }
 
 // backward of layer l: dy -> dx (LoRA grads of layer l written into each client's G)
-static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy, bf16* dx, const Scratch& sc,
-                          cudaStream_t st) {
+// dyf/dy: the incoming gradient (fp32 residual stream + its bf16 copy); dxf/dxb: the outgoing one
+static int layer_backward(menos_server* s, menos_batch* b, int l, const float* dyf, const bf16* dy, float* dxf,
+                          bf16* dxb, const Scratch& sc, cudaStream_t st) {
   const Dims& D = s->D;
   const auto& W = s->W[l];
   const LayerSave& S = b->L[l];
@@ -1224,13 +1232,13 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
-  { ProfScope ps(PC_NORM, 0, (double)T * (8.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dy, sc.dh, T, D.d, st)); }
+  { ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st)); }
   // A10: O dX (+ LoRA o) -> dO
   if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
-    a.A = sc.dh; a.lda = D.d; a.B = W.wo; a.ldb = D.Nq;
+    a.A = sc.dhb; a.lda = D.d; a.B = W.wo; a.ldb = D.Nq;
     if (b->g_active[GO]) {
       a.R = b->R_used[GO]; a.A2 = sc.dU[GO]; a.lda2 = a.R; a.B2 = s->Acat[GO][l]; a.ldb2 = D.ldK_g[GO];
       a.mtile_extra = b->d_mtile[GO];
@@ -1264,14 +1272,14 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const bf16* dy
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
-  { ProfScope ps(PC_NORM, 0, (double)T * (8.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dh, dx, T, D.d, st)); }
+  { ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st)); }
   return MENOS_OK;
 }
 
-// full SAVE forward over all layers: X[0] = b->L[0].x (already filled), output -> xout
-static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, bf16* xout, cudaStream_t st) {
+// full SAVE forward over all layers: X[0] = b->L[0].x (already filled), output -> xout (fp32)
+static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, float* xout, cudaStream_t st) {
   for (int l = 0; l < s->n_layers; ++l) {
-    bf16* y = (l + 1 < s->n_layers) ? b->L[l + 1].x : xout;
+    float* y = (l + 1 < s->n_layers) ? b->L[l + 1].x : xout;
     int rc = layer_forward(s, b, l, b->L[l].x, y, b->L[l], true, st);
     if (rc) return rc;
   }
@@ -1306,7 +1314,9 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     if (b->meta) s->arena.release(b->meta);
     return code;
   };
-  if (cudaMemcpyAsync(b->L[0].x, x_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
+  // x_c (bf16, host or device) -> staging -> the fp32 residual stream X[0]
+  if (cudaMemcpyAsync(sc.io, x_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess ||
+      convert_bf16_to_f32_vec(sc.io, b->L[0].x, (long long)T * D.d, st) != 0) {
     set_err("copy of x_c failed");
     return fail_free(MENOS_ECUDA);
   }
@@ -1315,15 +1325,16 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     if (rc) return fail_free(rc);
   } else {
     // Alg.1 L6: forward without caching activations; only x_c is kept
-    const bf16* x = b->L[0].x;
+    const float* x = b->L[0].x;
     for (int l = 0; l < s->n_layers; ++l) {
-      bf16* y = ((s->n_layers - 1 - l) % 2 == 0) ? sc.xout : sc.dx;
+      float* y = ((s->n_layers - 1 - l) % 2 == 0) ? sc.xout : sc.dxf;
       rc = layer_forward(s, b.get(), l, x, y, ng, true, st);
       if (rc) return fail_free(rc);
       x = y;
     }
   }
-  if (cudaMemcpyAsync(x_s, sc.xout, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
+  if (convert_f32_to_bf16(sc.xout, sc.io, (long long)T * D.d, st) != 0 ||
+      cudaMemcpyAsync(x_s, sc.io, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
     set_err("copy of x_s failed");
     return fail_free(MENOS_ECUDA);
   }
@@ -1357,31 +1368,34 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   if (b->nograd) {
     // Alg.1 L10: re-forward with gradient preparation from the cached x_c; the SAVE slab is
     // allocated only now (on-demand allocation)
-    bf16* xc = b->L[0].x;
+    float* xc = b->L[0].x;
     uint8_t* old_slab = b->slab;
     uint8_t* old_meta = b->meta;
     b->slab = nullptr; b->meta = nullptr;
     b->nograd = false;
     rc = finalize_batch(s, b, sc, nullptr, st);
     if (rc) { b->nograd = true; b->slab = old_slab; b->meta = old_meta; return rc; }
-    CUDA_TRY(cudaMemcpyAsync(b->L[0].x, xc, (size_t)T * D.d * 2, cudaMemcpyDeviceToDevice, st));
+    CUDA_TRY(cudaMemcpyAsync(b->L[0].x, xc, (size_t)T * D.d * 4, cudaMemcpyDeviceToDevice, st));
     s->arena.release(old_meta);   // stream-ordered reuse: later users run after these copies
     s->arena.release(old_slab);
     rc = forward_save(s, b, sc, sc.xout, st);
     if (rc) return rc;
   }
-  CUDA_TRY(cudaMemcpyAsync(sc.dy, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  // g_c (bf16) -> the bf16 copy of the incoming gradient and the fp32 gradient residual stream
+  CUDA_TRY(cudaMemcpyAsync(sc.dyb, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  K_TRY(convert_bf16_to_f32_vec(sc.dyb, sc.dyf, (long long)T * D.d, st));
   // the block-diagonal dU scratch: zero once (a batch's slot positions are the same in every layer)
   for (int g = 0; g < NG; ++g)
     if (b->g_active[g]) CUDA_TRY(cudaMemsetAsync(sc.dU[g], 0, (size_t)T * b->R_used[g] * 2, st));
-  bf16* dy = sc.dy;
-  bf16* dx = sc.dx;
+  float* dyf = sc.dyf; bf16* dyb = sc.dyb;
+  float* dxf = sc.dxf; bf16* dxb = sc.dxb;
   for (int l = s->n_layers - 1; l >= 0; --l) {
-    rc = layer_backward(s, b, l, dy, dx, sc, st);
+    rc = layer_backward(s, b, l, dyf, dyb, dxf, dxb, sc, st);
     if (rc) return rc;
-    std::swap(dy, dx);
+    std::swap(dyf, dxf);
+    std::swap(dyb, dxb);
   }
-  CUDA_TRY(cudaMemcpyAsync(g_s, dy, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(g_s, dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
   cudaPointerAttributes pa;
   if (cudaPointerGetAttributes(&pa, g_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&
       pa.type != cudaMemoryTypeManaged)
@@ -1404,11 +1418,11 @@ extern "C" int menos_test_batch_tensor(menos_server* s, menos_batch* b, int laye
   const void* src = nullptr;
   size_t n = 0;
   switch (which) {
-    case 0: src = S.x; n = T * D.d * 2; break;
+    case 0: src = S.x; n = T * D.d * 4; break;
     case 1: src = S.xn; n = T * D.d * 2; break;
     case 2: src = S.qkv; n = T * D.Nqkv * 2; break;
     case 3: src = S.O; n = T * D.Nq * 2; break;
-    case 4: src = S.h; n = T * D.d * 2; break;
+    case 4: src = S.h; n = T * D.d * 4; break;
     case 5: src = S.hn; n = T * D.d * 2; break;
     case 6: src = S.gu; n = T * 2 * D.fpad * 2; break;
     case 7: src = S.a; n = T * D.fpad * 2; break;

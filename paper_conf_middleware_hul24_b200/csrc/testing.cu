@@ -27,7 +27,8 @@ extern "C" int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int
   a.M = M; a.N = N; a.K = K; a.b_mn_major = b_mn;
   a.A = (const bf16*)A; a.lda = lda; a.B = (const bf16*)B; a.ldb = ldb;
   a.A2 = (const bf16*)A2; a.lda2 = lda2; a.B2 = (const bf16*)B2; a.ldb2 = ldb2; a.R = R;
-  a.epi = epi; a.out = (bf16*)out; a.ldo = ldo; a.resid = (const bf16*)resid; a.ldr = ldr;
+  a.epi = epi; a.out = (bf16*)out; a.ldo = ldo; a.resid = (const float*)resid; a.ldr = ldr;
+  a.outf = (float*)out;  // EPI_RESID: fp32 residual in, fp32 out
   a.out2 = (bf16*)out2; a.ldo2 = ldo2; a.aux = (const bf16*)aux; a.ldaux = ldaux;
   a.head_dim = head_dim; a.rope_cols = rope_cols;
   int dev = 0, sms = 148;
@@ -98,10 +99,10 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   return MENOS_OK;
 }
 
-extern "C" int menos_test_rmsnorm(int T, int d, const void* x, const float* g, float eps, void* y, float* rstd,
-                                  const void* dy, const void* resid, void* dx) {
-  int rc = rmsnorm_fwd((const bf16*)x, g, (bf16*)y, rstd, T, d, eps, 0);
-  if (rc == 0 && dy) rc = rmsnorm_bwd((const bf16*)dy, (const bf16*)x, g, rstd, (const bf16*)resid, (bf16*)dx, T, d, 0);
+extern "C" int menos_test_rmsnorm(int T, int d, const float* x, const float* g, float eps, void* y, float* rstd,
+                                  const void* dy, const float* resid, float* dx, void* dxb) {
+  int rc = rmsnorm_fwd(x, g, (bf16*)y, rstd, T, d, eps, 0);
+  if (rc == 0 && dy) rc = rmsnorm_bwd((const bf16*)dy, x, g, rstd, resid, dx, (bf16*)dxb, T, d, 0);
   cudaError_t e = cudaDeviceSynchronize();
   if (rc != 0) return fail("rmsnorm launch rejected");
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));

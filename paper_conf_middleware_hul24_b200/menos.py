@@ -84,7 +84,7 @@ SIGNATURES = {
     "menos_test_gemm": (_I, [_I, _I, _I, _I, _P, _I, _P, _I, _P, _I, _P, _I, _I, _PI32, _I, _P, _I, _P, _I, _P, _I,
                              _P, _I, _I, _I, _PI32, _F, _I]),
     "menos_test_attention": (_I, [_I, _PI32, _I, _I, _I, _P, _P, _P, _P, _P, _F]),
-    "menos_test_rmsnorm": (_I, [_I, _I, _P, _P, _F, _P, _P, _P, _P, _P]),
+    "menos_test_rmsnorm": (_I, [_I, _I, _P, _P, _F, _P, _P, _P, _P, _P, _P]),
     "menos_test_batch_tensor": (_I, [_P, _P, _I, _I, _P, C.POINTER(_S)]),
     "menos_test_lora_rows": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _F]),
     "menos_test_lora_tokred": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _I, _F, _I]),
