@@ -143,9 +143,11 @@ def build_server(torch, w, device, seed, arena_gb):
     shapes = {"wq": (m.n_heads * hd, m.d_model), "wk": (m.n_kv_heads * hd, m.d_model),
               "wv": (m.n_kv_heads * hd, m.d_model), "wo": (m.d_model, m.n_heads * hd),
               "wgate": (m.d_ff, m.d_model), "wup": (m.d_ff, m.d_model), "wdown": (m.d_model, m.d_ff)}
+    out_std = 0.02 / (2.0 * m.total_layers) ** 0.5   # same recipe as workloads.base_layer_weights (R17)
     for l in range(m.n_layers):
         gen.manual_seed(seed * 1000 + l)
-        lw = {k: (torch.randn(s, generator=gen, device=device, dtype=torch.float32) * 0.02).to(torch.bfloat16)
+        lw = {k: (torch.randn(s, generator=gen, device=device, dtype=torch.float32)
+                  * (out_std if k in ("wo", "wdown") else 0.02)).to(torch.bfloat16)
               for k, s in shapes.items()}
         for gname in ("g1", "g2"):
             lw[gname] = (1 + 0.1 * torch.randn(m.d_model, generator=gen, device=device)).to(torch.bfloat16)
@@ -183,25 +185,47 @@ def run_gpu(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     device = torch.device("cuda", local)
     torch.cuda.set_device(device)
+    from paper_conf_middleware_hul24_b200.partition import plan_waves, workload_partition
     w = workload(args.workload, n_layers=args.layers)
+    # cfg2 (32 ragged clients): LPT partition over the ranks (strong scaling); otherwise every rank serves the
+    # workload's own client set on its replica (weak scaling)
+    strong = args.workload == "cfg2_7b_x32_ragged"
+    if strong:
+        w.clients = [w.clients[i] for i in workload_partition(w, world)[rank]]
     T = w.n_tokens
     d = w.model.d_model
     srv = build_server(torch, w, device, seed=rank, arena_gb=args.arena_gb)
     ids = register_clients(np, srv, w, seed=rank + 1)
-    seq_client, seq_len = [], []
-    for i, c in enumerate(w.clients):
-        seq_client += [ids[i]] * len(c.seq_lens)
-        seq_len += list(c.seq_lens)
+    # waves: temporal sharing of the arena when the clients' saved activations do not fit at once
+    mem = [srv.client_memory(ids[i], c.n_tokens) for i, c in enumerate(w.clients)]
+    cap = srv.stats()["arena_bytes"] - (256 << 20)
+    waves = plan_waves([m[1] for m in mem], [m[2] for m in mem], cap)
+    toff = [0]
+    for c in w.clients:
+        toff.append(toff[-1] + c.n_tokens)
+    wave_args = []
+    for wv in waves:
+        sc_, sl_ = [], []
+        for i in wv:
+            sc_ += [ids[i]] * len(w.clients[i].seq_lens)
+            sl_ += list(w.clients[i].seq_lens)
+        wave_args.append((sc_, sl_, toff[wv[0]], toff[wv[-1] + 1]))
     gen = torch.Generator(device=device)
     gen.manual_seed(7 + rank)
     x_c = torch.randn(T, d, generator=gen, device=device).to(torch.bfloat16)
     g_c = torch.randn(T, d, generator=gen, device=device).to(torch.bfloat16)
     x_s, g_s = torch.empty_like(x_c), torch.empty_like(x_c)
     stream = torch.cuda.current_stream(device)
+    T_all = T
+    if world > 1:
+        tt = torch.tensor([float(T)], device=device)
+        dist.all_reduce(tt)
+        T_all = int(tt.item())
 
     def step(xc, xs, gc, gs):
-        b = srv.forward(seq_client, seq_len, xc, xs, stream=stream)
-        srv.backward(b, gc, gs, stream=stream)
+        for sc_, sl_, a, b_ in wave_args:
+            b = srv.forward(sc_, sl_, xc[a:b_], xs[a:b_], stream=stream)
+            srv.backward(b, gc[a:b_], gs[a:b_], stream=stream)
         srv.adapter_step(ids, stream=stream)
 
     def barrier():
@@ -237,7 +261,7 @@ def run_gpu(args):
     launches = M.launch_count() - l0
     clk = clocks.stop()
     ms_per_step = ms / args.steps
-    value = world * T * args.steps / (ms / 1000.0)
+    value = T_all * args.steps / (ms / 1000.0)
 
     # per-kernel CUDA events (recorded by the library on the launching stream around every launch) over a
     # second timed region of the same K steps; kept out of the headline region because an event pair around
@@ -255,7 +279,7 @@ def run_gpu(args):
         hxs, hgs = torch.empty_like(hx).pin_memory(), torch.empty_like(hg).pin_memory()
         step(hx, hxs, hg, hgs)
         ms_e = timed(lambda: step(hx, hxs, hg, hgs), args.steps)
-        e2e = {"value": world * T * args.steps / (ms_e / 1000.0), "unit": "tokens/s",
+        e2e = {"value": T_all * args.steps / (ms_e / 1000.0), "unit": "tokens/s",
                "h2d_bytes_per_step": int(hx.numel() * 2 + hg.numel() * 2),
                "d2h_bytes_per_step": int(hxs.numel() * 2 + hgs.numel() * 2),
                "ms_per_step": ms_e / args.steps}
@@ -322,10 +346,12 @@ def run_gpu(args):
            "paper_reference": "PAPER.md:352: -72.2% for 4 Llama-2-7B clients on a V100 (fp32; context only)"}
 
     line = {"metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong" if strong else "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded random weights/activations)",
             "config": {"workload": args.workload, "model": w.model.name, "clients_per_gpu": len(w.clients),
-                       "tokens_per_gpu_step": T, "server_layers": w.model.n_layers,
+                       "tokens_per_gpu_step": T, "tokens_per_step_all_gpus": T_all,
+                       "waves_per_step": len(waves), "server_layers": w.model.n_layers,
                        "lora": sorted({f"r{c.rank} {'+'.join(c.targets)}" for c in w.clients}),
                        "seq_lens": sorted({s for c in w.clients for s in c.seq_lens}),
                        "parallelism": f"replica x{world} (clients partitioned, no collective)",

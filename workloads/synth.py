@@ -32,10 +32,16 @@ class ModelCfg:
     first_layer: int = 1     # 0-indexed first server layer (layer 1 stays on the client)
     rms_eps: float = 1e-5
     rope_theta: float = 10000.0
+    model_layers: int = 0    # decoder layers of the full model (0: first_layer + n_layers)
 
     @property
     def head_dim(self) -> int:
         return self.d_model // self.n_heads
+
+    @property
+    def total_layers(self) -> int:
+        """Decoder layers of the whole model (unchanged by depth truncation)."""
+        return self.model_layers if self.model_layers > 0 else self.first_layer + self.n_layers
 
     def with_layers(self, n: int) -> "ModelCfg":
         return dataclasses.replace(self, n_layers=n)
@@ -43,11 +49,11 @@ class ModelCfg:
 
 MODELS = {
     # tiny: BASELINE.json configs[0]
-    "tiny": ModelCfg("tiny", 64, 4, 4, 172, 2),
+    "tiny": ModelCfg("tiny", 64, 4, 4, 172, 2, model_layers=3),
     # Llama-2-7B / 13B / 70B server segments (layers 2..L, 1-indexed) [ext]
-    "7b": ModelCfg("llama2-7b", 4096, 32, 32, 11008, 31),
-    "13b": ModelCfg("llama2-13b", 5120, 40, 40, 13824, 39),
-    "70b": ModelCfg("llama2-70b", 8192, 64, 8, 28672, 79),
+    "7b": ModelCfg("llama2-7b", 4096, 32, 32, 11008, 31, model_layers=32),
+    "13b": ModelCfg("llama2-13b", 5120, 40, 40, 13824, 39, model_layers=40),
+    "70b": ModelCfg("llama2-70b", 8192, 64, 8, 28672, 79, model_layers=80),
 }
 
 
@@ -118,14 +124,19 @@ def _rng(*key: int) -> np.random.Generator:
 def base_layer_weights(cfg: ModelCfg, layer: int, seed: int = 0) -> dict[str, np.ndarray]:
     """Frozen base weights of one decoder layer, natural (HF) layouts, fp32 bf16-representable.
 
-    W ~ N(0, 0.02^2) (Llama init std), gains g = 1 + 0.1 N(0,1).
+    W ~ N(0, 0.02^2) (Llama init std) for q, k, v, gate, up; the residual-branch output projections o and
+    down use the GPT-2 / Megatron scaled init std 0.02 / sqrt(2 L) (L = total decoder layers of the model),
+    so the residual stream evolves like a trained pre-norm network instead of a chaotic random one
+    (reading R17).  Gains g = 1 + 0.1 N(0,1).
     """
     out = {}
     names = ["q", "k", "v", "o", "gate", "up", "down"]
+    out_std = 0.02 / np.sqrt(2.0 * cfg.total_layers)
     for i, t in enumerate(names):
         K, N = target_dims(cfg, t)
         r = _rng(seed, layer, i)
-        out["w" + t] = bf16_round(r.standard_normal((N, K), dtype=np.float32) * np.float32(0.02))
+        std = out_std if t in ("o", "down") else 0.02
+        out["w" + t] = bf16_round(r.standard_normal((N, K), dtype=np.float32) * np.float32(std))
     for j, g in enumerate(["g1", "g2"]):
         r = _rng(seed, layer, 100 + j)
         out[g] = bf16_round(1.0 + 0.1 * r.standard_normal(cfg.d_model, dtype=np.float32))
