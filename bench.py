@@ -329,7 +329,7 @@ def run_gpu(args):
             K_, N_ = target_dims(m, t)
             lora += 6 * c.rank * (K_ + N_) * c.n_tokens * m.n_layers
     step_flops = 4 * P * T + attn + lora
-    step_tflops = world * step_flops * args.steps / (ms / 1000.0) / 1e12
+    step_tflops = step_flops * (T_all / T) * args.steps / (ms / 1000.0) / 1e12
 
     # HBM bytes per client (persistent A+O and the SAVE-forward arena share), Eq.3 accounting
     st = srv.stats()

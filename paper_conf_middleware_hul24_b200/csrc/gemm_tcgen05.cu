@@ -166,6 +166,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           mbar_wait(&empty_bar[stage], phase ^ 1);
           uint8_t* sa = smem + stage * C::STAGE_BYTES;
           uint8_t* sb = sa + C::A_STAGE;
+          if (p.epi == 98) {  // tuning aid: no operand traffic, MMAs run on stale smem (isolates MMA issue)
+            if (leader) mbar_arrive(&full_bar[stage]);
+            if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+            continue;
+          }
           if (leader) mbar_expect_tx(&full_bar[stage], C::STAGE_BYTES * CG);
           const bool main = kb < p.kb_main;
           const CUtensorMap* ma = main ? &tmA : &tmA2;
@@ -193,9 +198,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else if (warp == 1) {
-    if (lane == 0 && leader) {
-      // ------------------------------------------------ MMA issuer (single thread of the leader CTA)
+    if (leader) {
+      // ------------------------------------------------ MMA issuer: the whole warp runs the (warp-uniform) loop
+      // so descriptors stay in uniform registers; one elected lane issues the MMAs and their commits.
       constexpr uint32_t IDESC = umma_idesc_bf16(BM * CG, BN, B_MN);
+      // descriptor bases for stage 0 (16-byte units, low 14 bits = start address >> 4); stages are STAGE_BYTES apart
+      const uint64_t a_desc0 = umma_desc_sw128(smem_u32(smem), 16, 1024);
+      const uint64_t b_desc0 = B_MN ? umma_desc_sw128(smem_u32(smem) + C::A_STAGE, 8192, 1024)
+                                    : umma_desc_sw128(smem_u32(smem) + C::A_STAGE, 16, 1024);
+      constexpr uint64_t STAGE_STEP = C::STAGE_BYTES >> 4;
+      constexpr uint64_t A_KSTEP = 32 >> 4;
+      constexpr uint64_t B_KSTEP = (B_MN ? 2048 : 32) >> 4;
       int stage = 0; uint32_t phase = 0;
       int acc = 0; uint32_t acc_phase = 0;
       for (int t = cluster_id; t < total; t += n_clusters) {
@@ -209,23 +222,34 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&full_bar[stage], phase);
           tc_fence_after();
-          const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
-          const uint32_t sb = sa + C::A_STAGE;
-          int nsteps = 4;
-          if (kb >= p.kb_main) { nsteps = n16 - (kb - p.kb_main) * 4; if (nsteps > 4) nsteps = 4; }
-          for (int k = 0; k < nsteps; ++k) {
-            const uint64_t ad = umma_desc_sw128(sa + k * 32, 16, 1024);
-            const uint64_t bd = B_MN ? umma_desc_sw128(sb + k * 2048, 8192, 1024)
-                                     : umma_desc_sw128(sb + k * 32, 16, 1024);
-            if (CG == 2) tc_mma_bf16_2sm(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
-            else tc_mma_bf16(d_tmem, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+          const uint64_t ad = a_desc0 + stage * STAGE_STEP;
+          const uint64_t bd = b_desc0 + stage * STAGE_STEP;
+          if (elect_one()) {
+            if (kb < p.kb_main) {
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const uint32_t accum = (kb > 0 || k > 0) ? 1u : 0u;
+                if (CG == 2) tc_mma_bf16_2sm(d_tmem, ad + k * A_KSTEP, bd + k * B_KSTEP, IDESC, accum);
+                else tc_mma_bf16(d_tmem, ad + k * A_KSTEP, bd + k * B_KSTEP, IDESC, accum);
+              }
+            } else {
+              const int nsteps = min(4, n16 - (kb - p.kb_main) * 4);
+              for (int k = 0; k < nsteps; ++k) {
+                if (CG == 2) tc_mma_bf16_2sm(d_tmem, ad + k * A_KSTEP, bd + k * B_KSTEP, IDESC, 1u);
+                else tc_mma_bf16(d_tmem, ad + k * A_KSTEP, bd + k * B_KSTEP, IDESC, 1u);
+              }
+            }
+            if (CG == 2) tc_commit_2sm_mc(&empty_bar[stage], 0x3);
+            else tc_commit(&empty_bar[stage]);
           }
-          if (CG == 2) tc_commit_2sm_mc(&empty_bar[stage], 0x3);
-          else tc_commit(&empty_bar[stage]);
+          __syncwarp();
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
-        if (CG == 2) tc_commit_2sm_mc(&tfull_bar[acc], 0x3);
-        else tc_commit(&tfull_bar[acc]);
+        if (elect_one()) {
+          if (CG == 2) tc_commit_2sm_mc(&tfull_bar[acc], 0x3);
+          else tc_commit(&tfull_bar[acc]);
+        }
+        __syncwarp();
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
     }
@@ -250,6 +274,15 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           tmem_ld32(tb + c * 32, v);
           if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
         }
+      } else if (p.epi == 99 || p.epi == 98) {
+        // tuning aid: drain TMEM without storing (isolates the mainloop)
+        float sink = 0.f;
+        for (int c = 0; c < 8; ++c) {
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          sink += v[c];
+        }
+        if (sink == 12345.678f) p.out[0] = f2bf(sink);
       } else if (p.epi == EPI_RESID) {
         // fp32 residual stream: outf = acc + resid
         for (int c = 0; c < 8; ++c) {

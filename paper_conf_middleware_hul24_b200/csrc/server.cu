@@ -281,7 +281,10 @@ struct menos_server {
   uint8_t* arena_mem = nullptr;
   uint8_t* scratch = nullptr; size_t scratch_bytes = 0;
   // pinned host staging for metadata uploads
-  uint8_t* pinned = nullptr; size_t pinned_bytes = 0;
+  static constexpr int kRing = 4;
+  struct Slot { uint8_t* buf = nullptr; size_t bytes = 0; cudaEvent_t ev = nullptr; };
+  Slot ring[kRing];
+  int ring_next = 0;
 };
 
 // =====================================================================================================
@@ -377,13 +380,23 @@ static void client_segments(menos_server* s, const Client& c, int hyp_idx, std::
     }
 }
 
-static int ensure_pinned(menos_server* s, size_t n) {
-  if (n <= s->pinned_bytes) return MENOS_OK;
-  if (s->pinned) cudaFreeHost(s->pinned);
-  s->pinned = nullptr;
-  size_t nb = std::max(n, (size_t)1 << 20);
-  CUDA_TRY(cudaMallocHost(&s->pinned, nb));
-  s->pinned_bytes = nb;
+// Host->device upload through a ring of pinned staging slots; a slot is reused only after the copy that last
+// used it has completed (its event), so uploads never synchronise the stream with the host.
+static int upload(menos_server* s, void* dst, const void* src, size_t n, cudaStream_t st) {
+  auto& slot = s->ring[s->ring_next];
+  s->ring_next = (s->ring_next + 1) % menos_server::kRing;
+  if (slot.ev) CUDA_TRY(cudaEventSynchronize(slot.ev));
+  else CUDA_TRY(cudaEventCreateWithFlags(&slot.ev, cudaEventDisableTiming));
+  if (n > slot.bytes) {
+    if (slot.buf) CUDA_TRY(cudaFreeHost(slot.buf));
+    slot.buf = nullptr;
+    const size_t nb = std::max(n, (size_t)1 << 20);
+    CUDA_TRY(cudaMallocHost(&slot.buf, nb));
+    slot.bytes = nb;
+  }
+  memcpy(slot.buf, src, n);
+  CUDA_TRY(cudaMemcpyAsync(dst, slot.buf, n, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaEventRecord(slot.ev, st));
   return MENOS_OK;
 }
 
@@ -420,13 +433,12 @@ static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, c
   const size_t o2 = align_up(b1, 256), o3 = o2 + align_up(b2, 256), tot = o3 + b3;
   uint8_t* dbuf = nullptr;
   CUDA_TRY(cudaMallocAsync((void**)&dbuf, tot, st));
-  int rc = ensure_pinned(s, tot);
+  std::vector<uint8_t> blob(tot);
+  memcpy(blob.data(), hyp.data(), b1);
+  memcpy(blob.data() + o2, segs.data(), b2);
+  memcpy(blob.data() + o3, work.data(), b3);
+  int rc = upload(s, dbuf, blob.data(), tot, st);
   if (rc) return rc;
-  CUDA_TRY(cudaStreamSynchronize(st));  // pinned staging reuse
-  memcpy(s->pinned, hyp.data(), b1);
-  memcpy(s->pinned + o2, segs.data(), b2);
-  memcpy(s->pinned + o3, work.data(), b3);
-  CUDA_TRY(cudaMemcpyAsync(dbuf, s->pinned, tot, cudaMemcpyHostToDevice, st));
   double nparam = 0;
   for (auto& sg : segs) nparam += (double)sg.rows * sg.cols;
   {
@@ -526,7 +538,10 @@ extern "C" void menos_server_destroy(menos_server* s) {
   if (s->wbuf) cudaFree(s->wbuf);
   if (s->rope) cudaFree(s->rope);
   if (s->arena_mem) cudaFree(s->arena_mem);
-  if (s->pinned) cudaFreeHost(s->pinned);
+  for (auto& sl : s->ring) {
+    if (sl.buf) cudaFreeHost(sl.buf);
+    if (sl.ev) cudaEventDestroy(sl.ev);
+  }
   delete s;
 }
 
@@ -1027,11 +1042,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
   if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
   b->meta = meta;
-  int rc = ensure_pinned(s, blob.size());
+  int rc = upload(s, meta, blob.data(), blob.size(), st);
   if (rc) return rc;
-  CUDA_TRY(cudaStreamSynchronize(st));
-  memcpy(s->pinned, blob.data(), blob.size());
-  CUDA_TRY(cudaMemcpyAsync(meta, s->pinned, blob.size(), cudaMemcpyHostToDevice, st));
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
