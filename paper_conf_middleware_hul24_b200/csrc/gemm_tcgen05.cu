@@ -485,6 +485,12 @@ int launch(const CUtensorMap& mA, const CUtensorMap& mB, const CUtensorMap& mA2,
 
 int g_gemm_cta_group = 2;
 
+// shared with attention_tc.cu: cached 2-D SWIZZLE_128B tensor map (box = {bc cols, br rows})
+bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
+                uint32_t br) {
+  return get_map(out, ptr, rows, cols, ld, bc, br);
+}
+
 int gemm_run(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
   if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;

@@ -98,6 +98,9 @@ struct AttnArgs {
   const float2* rope_cs;         // [max_pos][hd/2]
 };
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
+// tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block
+int attn_fwd_tc(const AttnArgs& a, const int2* qblocks128, int n_qblocks128, cudaStream_t st);
+extern int g_attn_tc;  // 1: use the tcgen05 forward when head_dim == 128 (default)
 int attn_bwd(const AttnArgs& a, cudaStream_t st);
 
 // ---------------------------------------------------------------- AdamW + bf16 refresh

@@ -240,7 +240,8 @@ struct menos_batch {
   int R_used[NG] = {0, 0, 0, 0};
   bool g_active[NG] = {false, false, false, false};
   bool save_a = false;
-  int n_mt = 0, n_blocks = 0;
+  int n_mt = 0, n_blocks = 0, n_blocks128 = 0;
+  int2* d_blocks128 = nullptr;
   double pairs = 0;   // causal (query, key) pairs summed over sequences
   // device metadata
   uint8_t* meta = nullptr;  // arena
@@ -892,6 +893,10 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   for (int i = 0; i < b->n_seqs; ++i)
     for (int q = 0; q < b->seq_len[i]; q += 64) blocks.push_back(make_int2(i, q));
   b->n_blocks = (int)blocks.size();
+  std::vector<int2> blocks128;   // 128-row q blocks of the tcgen05 attention forward
+  for (int i = 0; i < b->n_seqs; ++i)
+    for (int q = 0; q < b->seq_len[i]; q += 128) blocks128.push_back(make_int2(i, q));
+  b->n_blocks128 = (int)blocks128.size();
   std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
   for (int g = 0; g < NG; ++g) {
     if (!b->g_active[g]) continue;
@@ -920,6 +925,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_cu = put(b->cu.data(), b->cu.size() * 4);
   const size_t o_pos = put(b->pos.data(), b->pos.size() * 4);
   const size_t o_blk = put(blocks.data(), blocks.size() * sizeof(int2));
+  const size_t o_blk128 = put(blocks128.data(), blocks128.size() * sizeof(int2));
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
 
@@ -1045,6 +1051,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   int rc = upload(s, meta, blob.data(), blob.size(), st);
   if (rc) return rc;
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
+  b->d_blocks128 = (int2*)(meta + o_blk128);
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
   b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
@@ -1156,7 +1163,9 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    { ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st); K_TRY(attn_fwd(a, st)); }
+    ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st);
+    if (D.hd == 128 && g_attn_tc) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+    else K_TRY(attn_fwd(a, st));
   }
   // A4: O GEMM (+ LoRA o) + residual
   if (b->g_active[GO]) {

@@ -86,7 +86,20 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   a.qkv = (const bf16*)qkv; a.ld_qkv = Nqkv; a.O = (bf16*)O; a.ld_o = H * hd; a.lse = lse;
   a.cu_seqlens = d_cu; a.qblocks = d_blk; a.n_qblocks = (int)blocks.size(); a.kvblocks = d_blk;
   a.n_kvblocks = (int)blocks.size(); a.T = T; a.H = H; a.Hkv = Hkv; a.hd = hd; a.scale = 1.f / std::sqrt((float)hd);
-  int rc = attn_fwd(a, 0);
+  int rc;
+  if (hd == 128 && g_attn_tc) {
+    std::vector<int2> b128;
+    for (int i = 0; i < n_seqs; ++i)
+      for (int q = 0; q < seq_len[i]; q += 128) b128.push_back(make_int2(i, q));
+    int2* d_b128;
+    cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
+    cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
+    rc = attn_fwd_tc(a, d_b128, (int)b128.size(), 0);
+    cudaDeviceSynchronize();
+    cudaFree(d_b128);
+  } else {
+    rc = attn_fwd(a, 0);
+  }
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
@@ -183,5 +196,11 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
   if (rc) return fail("gemm rejected");
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   *ms_out = ms / iters;
+  return MENOS_OK;
+}
+
+namespace menos { int g_attn_tc = 1; }
+extern "C" int menos_test_set_attn_tc(int on) {
+  menos::g_attn_tc = on ? 1 : 0;
   return MENOS_OK;
 }

@@ -90,6 +90,7 @@ SIGNATURES = {
     "menos_test_lora_tokred": (_I, [_P, _P, _P, _I, _I, _I, _I, _I, _I, _I, _I, _F, _I]),
     "menos_test_set_gemm_cta_group": (_I, [_I]),
     "menos_test_gemm_time": (_I, [_I, _I, _I, _I, _P, _P, _P, _I, _P, _I, C.POINTER(C.c_float)]),
+    "menos_test_set_attn_tc": (_I, [_I]),
     "menos_testing_last_error": (C.c_char_p, []),
 }
 

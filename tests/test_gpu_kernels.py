@@ -232,10 +232,12 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-@pytest.mark.parametrize("hd,H,Hkv,lens", [(128, 4, 2, [1, 17, 64, 129, 300]), (16, 4, 4, [16, 16, 3]),
-                                          (64, 8, 1, [200, 65])])
-def test_attention_fwd_bwd(hd, H, Hkv, lens):
+@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 1), (128, 4, 2, [1, 17, 64, 129, 300], 0),
+                                             (128, 2, 2, [512, 1024, 255], 1), (16, 4, 4, [16, 16, 3], 1),
+                                             (64, 8, 1, [200, 65], 1)])
+def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
     from paper_conf_middleware_hul24_b200.menos import check
+    check(lib().menos_test_set_attn_tc(tc), testing=True)
     T = sum(lens)
     N = (H + 2 * Hkv) * hd
     qkv = rnd((T, N), 51)
