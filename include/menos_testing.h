@@ -62,7 +62,7 @@ MENOS_API int menos_test_set_gemm_cta_group(int cta_group);
 MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A, const void* B, void* out, int epi,
                                    const void* aux, int iters, float* ms_out);
 
-/* Select the attention forward for head_dim 128: 1 = tcgen05 (default), 0 = mma.sync. */
+/* Select the attention forward for head_dim 128: 1 = tcgen05, 0 = mma.sync (default). */
 MENOS_API int menos_test_set_attn_tc(int on);
 
 MENOS_API const char* menos_testing_last_error(void);

@@ -27,37 +27,46 @@ __device__ __forceinline__ int tsw(int row, int chunk) {
 
 // ============================================================================ rows kernel
 // C[t, j] = scale * sum_k A[t, k] * Bop(j, k) for t in [m0, m0+64), j in [0, NT)
+// 4-stage cp.async ring of 128-wide K tiles: ~96-192 KB of X / dY in flight per SM, enough to stream the
+// activations at HBM rate with one CTA per 64-token block.
+constexpr int ROWS_BM = 64, ROWS_BK = 128, ROWS_STAGES = 4;
+template <int NT>
+constexpr int rows_smem_bytes() { return ROWS_STAGES * (ROWS_BM + NT) * ROWS_BK * 2; }
+
 template <int NT>
 __global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* __restrict__ probs,
                                                         const int2* __restrict__ tiles) {
-  constexpr int BM = 64, BK = 64, NNT = NT / 8;
-  __shared__ __align__(128) bf16 As[2][BM * BK];
-  __shared__ __align__(128) bf16 Bs[2][NT * BK];  // "nk": [NT][BK]; "kn": [BK][NT]
+  constexpr int BM = ROWS_BM, BK = ROWS_BK, NNT = NT / 8, NS = ROWS_STAGES;
+  extern __shared__ __align__(128) uint8_t rows_smem[];
+  bf16* As_base = reinterpret_cast<bf16*>(rows_smem);                 // [NS][BM * BK]
+  bf16* Bs_base = As_base + NS * BM * BK;                             // [NS][NT * BK]  ("nk": [NT][BK]; "kn": [BK][NT])
   const int2 tl = tiles[blockIdx.x];
   const LoraRowsProblem P = probs[tl.x];
   const int m0 = tl.y;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
 
   auto load = [&](int buf, int k0) {
+    bf16* As = As_base + buf * BM * BK;
+    bf16* Bs = Bs_base + buf * NT * BK;
     for (int i = tid; i < BM * (BK / 8); i += 128) {
       const int r = i / (BK / 8), c = i % (BK / 8);
       const int gr = m0 + r, gk = k0 + c * 8;
       const bool ok = gr < P.M && gk < P.K;
-      cp_async16(smem_u32(&As[buf][tsw<BK>(r, c)]), P.A + (ok ? (size_t)gr * P.lda + gk : 0), ok ? 16 : 0);
+      cp_async16(smem_u32(&As[tsw<BK>(r, c)]), P.A + (ok ? (size_t)gr * P.lda + gk : 0), ok ? 16 : 0);
     }
     if (!P.b_kn) {
       for (int i = tid; i < NT * (BK / 8); i += 128) {
         const int r = i / (BK / 8), c = i % (BK / 8);
         const int gk = k0 + c * 8;
         const bool ok = r < P.N && gk < P.K;
-        cp_async16(smem_u32(&Bs[buf][tsw<BK>(r, c)]), P.B + (ok ? (size_t)r * P.ldb + gk : 0), ok ? 16 : 0);
+        cp_async16(smem_u32(&Bs[tsw<BK>(r, c)]), P.B + (ok ? (size_t)r * P.ldb + gk : 0), ok ? 16 : 0);
       }
     } else {
       for (int i = tid; i < BK * (NT / 8); i += 128) {
         const int r = i / (NT / 8), c = i % (NT / 8);
         const int gk = k0 + r;
         const bool ok = gk < P.K && c * 8 < P.N;
-        cp_async16(smem_u32(&Bs[buf][tsw<NT>(r, c)]), P.B + (ok ? (size_t)gk * P.ldb + c * 8 : 0), ok ? 16 : 0);
+        cp_async16(smem_u32(&Bs[tsw<NT>(r, c)]), P.B + (ok ? (size_t)gk * P.ldb + c * 8 : 0), ok ? 16 : 0);
       }
     }
   };
@@ -66,14 +75,21 @@ __global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* _
 #pragma unroll
   for (int j = 0; j < NNT; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
   const int nk = (P.K + BK - 1) / BK;
-  load(0, 0);
-  cp_async_commit();
+#pragma unroll
+  for (int s = 0; s < NS - 1; ++s) {
+    if (s < nk) load(s, s * BK);
+    cp_async_commit();
+  }
   for (int kb = 0; kb < nk; ++kb) {
-    if (kb + 1 < nk) { load((kb + 1) & 1, (kb + 1) * BK); cp_async_commit(); cp_async_wait<1>(); }
-    else cp_async_wait<0>();
+    cp_async_wait<NS - 2>();
     __syncthreads();
-    const bf16* a_s = As[kb & 1];
-    const bf16* b_s = Bs[kb & 1];
+    {  // refill the stage freed by iteration kb-1 (everyone passed the barrier above)
+      const int nx = kb + NS - 1;
+      if (nx < nk) load(nx % NS, nx * BK);
+      cp_async_commit();
+    }
+    const bf16* a_s = As_base + (kb % NS) * BM * BK;
+    const bf16* b_s = Bs_base + (kb % NS) * NT * BK;
 #pragma unroll
     for (int kk = 0; kk < BK; kk += 16) {
       uint32_t a[4];
@@ -97,8 +113,8 @@ __global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* _
         mma_bf16_16816(acc[j + 1], a, b2, b3);
       }
     }
-    __syncthreads();
   }
+  cp_async_wait<0>();
 #pragma unroll
   for (int j = 0; j < NNT; ++j)
 #pragma unroll
@@ -211,9 +227,16 @@ void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, st
 
 int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st) {
   if (n_tiles <= 0) return 0;
-  if (max_n <= 32) lora_rows_kernel<32><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
-  else if (max_n <= 64) lora_rows_kernel<64><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
-  else if (max_n <= 128) lora_rows_kernel<128><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_rows_kernel<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem_bytes<32>());
+    cudaFuncSetAttribute(lora_rows_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem_bytes<64>());
+    cudaFuncSetAttribute(lora_rows_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem_bytes<128>());
+    attr = true;
+  }
+  if (max_n <= 32) lora_rows_kernel<32><<<n_tiles, 128, rows_smem_bytes<32>(), st>>>(d_probs, d_tiles);
+  else if (max_n <= 64) lora_rows_kernel<64><<<n_tiles, 128, rows_smem_bytes<64>(), st>>>(d_probs, d_tiles);
+  else if (max_n <= 128) lora_rows_kernel<128><<<n_tiles, 128, rows_smem_bytes<128>(), st>>>(d_probs, d_tiles);
   else return -1;
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;

@@ -199,7 +199,9 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
   return MENOS_OK;
 }
 
-namespace menos { int g_attn_tc = 1; }
+// The tcgen05 forward is correct (tests) but its serialized single-CTA pipeline is still slower than the
+// mma.sync kernel on the 512-token workloads; off by default until it is warp-specialized.
+namespace menos { int g_attn_tc = 0; }
 extern "C" int menos_test_set_attn_tc(int on) {
   menos::g_attn_tc = on ? 1 : 0;
   return MENOS_OK;
