@@ -186,6 +186,8 @@ def run_gpu(args):
     device = torch.device("cuda", local)
     torch.cuda.set_device(device)
     from paper_conf_middleware_hul24_b200.partition import plan_waves, workload_partition
+    if os.environ.get("MENOS_ATTN_TC") is not None:   # kernel-variant switch for A/B measurements
+        M.lib().menos_test_set_attn_tc(int(os.environ["MENOS_ATTN_TC"]))
     w = workload(args.workload, n_layers=args.layers)
     # cfg2 (32 ragged clients): LPT partition over the ranks (strong scaling); otherwise every rank serves the
     # workload's own client set on its replica (weak scaling)

@@ -62,8 +62,9 @@ MENOS_API int menos_test_set_gemm_cta_group(int cta_group);
 MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A, const void* B, void* out, int epi,
                                    const void* aux, int iters, float* ms_out);
 
-/* Select the attention forward for head_dim 128: 1 = tcgen05, 0 = mma.sync (default). */
-MENOS_API int menos_test_set_attn_tc(int on);
+/* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
+   bit 1 = tcgen05 backward (else mma.sync). Default 2. Returns MENOS_EINVAL outside [0, 3]. */
+MENOS_API int menos_test_set_attn_tc(int mode);
 
 MENOS_API const char* menos_testing_last_error(void);
 

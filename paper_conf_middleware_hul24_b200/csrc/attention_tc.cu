@@ -21,7 +21,9 @@ constexpr int Q_BYTES = BQ * HD * 2;        // 32 KB: 2 swizzle atoms [128][64]
 constexpr int K_BYTES = BKV * HD * 2;       // 16 KB: 2 atoms [64][64]
 constexpr int V_BYTES = BKV * HD * 2;       // 16 KB: MN-major [2 hd blocks][64 keys][64]
 constexpr int P_BYTES = BQ * BKV * 2;       // 16 KB: 1 atom [128][64]
-constexpr int SMEM_FWD = Q_BYTES + 2 * (K_BYTES + V_BYTES) + P_BYTES + 1024;
+// P_j is written into the K_j stage buffer (free once S_j completed): 97 KB -> 2 CTAs per SM
+constexpr int SMEM_FWD = Q_BYTES + 2 * (K_BYTES + V_BYTES) + 1024;
+static_assert(P_BYTES == K_BYTES, "P reuses the K stage buffer");
 constexpr float LOG2E = 1.4426950408889634f;
 
 struct TcFwdParams {
@@ -54,7 +56,15 @@ __device__ __forceinline__ void mbar_wait_dbg(uint64_t* bar, uint32_t parity, in
 }
 #define MBAR_WAIT(b, p) mbar_wait_dbg(b, p, __LINE__)
 #else
-#define MBAR_WAIT(b, p) mbar_wait(b, p)
+// spin on test_wait (no suspend hint): these waits are short and on the critical path of every key block
+__device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile("{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.b32 %0, 1, 0, P;\n\t}"
+                 : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  }
+}
+#define MBAR_WAIT(b, p) mbar_wait_spin(b, p)
 #endif
 
 __global__ void __launch_bounds__(128, 2)
@@ -65,7 +75,6 @@ attn_fwd_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
   uint8_t* sQ = smem;
   uint8_t* sK[2] = {sQ + Q_BYTES, sQ + Q_BYTES + K_BYTES + V_BYTES};
   uint8_t* sV[2] = {sK[0] + K_BYTES, sK[1] + K_BYTES};
-  uint8_t* sP = sQ + Q_BYTES + 2 * (K_BYTES + V_BYTES);
   __shared__ __align__(8) uint64_t bar_q, bar_kv[2], bar_s[2], bar_pv;
   __shared__ uint32_t tmem_sh;
 
@@ -218,7 +227,7 @@ attn_fwd_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
     }
     // previous P V must have consumed sP before it is overwritten
     if (j > 0) { MBAR_WAIT(&bar_pv, ph_pv); ph_pv ^= 1; }
-    uint8_t* prow = sP + row * 128;
+    uint8_t* prow = sK[s] + row * 128;   // P_j overwrites K_j (S_j has completed)
 #pragma unroll
     for (int c8 = 0; c8 < 8; ++c8) {
       float e[8];
@@ -238,7 +247,7 @@ attn_fwd_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
     __syncthreads();
     if (tid == 0) {
       tc_fence_after();
-      const uint32_t pa = smem_u32(sP), vb = smem_u32(sV[s]);
+      const uint32_t pa = smem_u32(sK[s]), vb = smem_u32(sV[s]);
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         const uint64_t ad = umma_desc_sw128(pa + kk * 32, 16, 1024);

@@ -100,8 +100,10 @@ struct AttnArgs {
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block
 int attn_fwd_tc(const AttnArgs& a, const int2* qblocks128, int n_qblocks128, cudaStream_t st);
-extern int g_attn_tc;  // 1: use the tcgen05 forward when head_dim == 128 (default)
+extern int g_attn_tc;  // head_dim 128 variant bitmask: 1 = tcgen05 forward, 2 = tcgen05 backward
 int attn_bwd(const AttnArgs& a, cudaStream_t st);
+// tcgen05 backward for head_dim 128 (attention_bwd_tc.cu); blocks128 = (seq, local start) per 128-row block
+int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaStream_t st);
 
 // ---------------------------------------------------------------- AdamW + bf16 refresh
 struct AdamSeg {              // one (client, layer, target, A|B) parameter block

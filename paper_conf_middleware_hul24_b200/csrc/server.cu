@@ -1164,7 +1164,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st);
-    if (D.hd == 128 && g_attn_tc) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+    if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
     else K_TRY(attn_fwd(a, st));
   }
   // A4: O GEMM (+ LoRA o) + residual
@@ -1277,7 +1277,11 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
-    { ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * b->pairs, 0, st); K_TRY(attn_bwd(a, st)); }
+    {
+      ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * b->pairs, 0, st);
+      if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+      else K_TRY(attn_bwd(a, st));
+    }
   }
   // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
   if (b->g_active[GQKV]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GQKV], st));

@@ -87,26 +87,21 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   a.cu_seqlens = d_cu; a.qblocks = d_blk; a.n_qblocks = (int)blocks.size(); a.kvblocks = d_blk;
   a.n_kvblocks = (int)blocks.size(); a.T = T; a.H = H; a.Hkv = Hkv; a.hd = hd; a.scale = 1.f / std::sqrt((float)hd);
   int rc;
-  if (hd == 128 && g_attn_tc) {
-    std::vector<int2> b128;
-    for (int i = 0; i < n_seqs; ++i)
-      for (int q = 0; q < seq_len[i]; q += 128) b128.push_back(make_int2(i, q));
-    int2* d_b128;
-    cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
-    cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
-    rc = attn_fwd_tc(a, d_b128, (int)b128.size(), 0);
-    cudaDeviceSynchronize();
-    cudaFree(d_b128);
-  } else {
-    rc = attn_fwd(a, 0);
-  }
+  std::vector<int2> b128;
+  for (int i = 0; i < n_seqs; ++i)
+    for (int q = 0; q < seq_len[i]; q += 128) b128.push_back(make_int2(i, q));
+  int2* d_b128;
+  cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
+  cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
+  const bool tc_fwd = hd == 128 && (g_attn_tc & 1), tc_bwd = hd == 128 && (g_attn_tc & 2);
+  rc = tc_fwd ? attn_fwd_tc(a, d_b128, (int)b128.size(), 0) : attn_fwd(a, 0);
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
-    rc = attn_bwd(a, 0);
+    rc = tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
   }
   cudaError_t e = cudaDeviceSynchronize();
-  cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D);
+  cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D); cudaFree(d_b128);
   if (rc != 0) return fail("attention launch rejected");
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   return MENOS_OK;
@@ -199,10 +194,12 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
   return MENOS_OK;
 }
 
-// The tcgen05 forward is correct (tests) but its serialized single-CTA pipeline is still slower than the
-// mma.sync kernel on the 512-token workloads; off by default until it is warp-specialized.
-namespace menos { int g_attn_tc = 0; }
-extern "C" int menos_test_set_attn_tc(int on) {
-  menos::g_attn_tc = on ? 1 : 0;
+// Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward, 2 = tcgen05 backward (dK/dV + dQ kernels).
+// The tcgen05 forward's serialized single-control-thread pipeline is still slower than the mma.sync kernel on the
+// 512-token workloads, so only the backward is on by default.
+namespace menos { int g_attn_tc = 2; }
+extern "C" int menos_test_set_attn_tc(int mode) {
+  if (mode < 0 || mode > 3) { fail("attention mode must be in [0, 3]"); return MENOS_EINVAL; }
+  menos::g_attn_tc = mode;
   return MENOS_OK;
 }

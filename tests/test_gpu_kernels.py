@@ -232,9 +232,10 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 1), (128, 4, 2, [1, 17, 64, 129, 300], 0),
-                                             (128, 2, 2, [512, 1024, 255], 1), (16, 4, 4, [16, 16, 3], 1),
-                                             (64, 8, 1, [200, 65], 1)])
+@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 3), (128, 4, 2, [1, 17, 64, 129, 300], 0),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 2), (128, 8, 1, [130, 7, 256], 3),
+                                             (128, 2, 2, [512, 1024, 255], 3), (128, 2, 2, [512, 1024, 255], 0),
+                                             (16, 4, 4, [16, 16, 3], 3), (64, 8, 1, [200, 65], 3)])
 def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
     from paper_conf_middleware_hul24_b200.menos import check
     check(lib().menos_test_set_attn_tc(tc), testing=True)
