@@ -9,7 +9,9 @@
 //       dV += P^T dO, dK += dS^T Q          (tcgen05, P^T / dS^T from swizzled smem, accumulators in TMEM)
 //   dQ     (one CTA per 128-query block x head; loop over 64-key blocks):
 //       S = Q K^T, dP = dO V^T -> dS = P (dP - D) scale -> dQ += dS K
-// Warp roles: warp 0 TMA producer, warp 1 MMA issuer (elected lane), warps 2-5 elementwise + epilogue.
+// Warp roles: warp 0 TMA producer (3-stage ring of the streamed operand), warp 1 MMA issuer (elected lane),
+// warps 2-9 elementwise (thread = TMEM lane = row; warpgroup g of them owns half the columns) + epilogue.  The epilogue stages the fp32 accumulator rows in
+// shared memory and re-reads them warp-per-row so the RoPE table reads and the bf16 row stores are coalesced.
 #include <cstdio>
 #include "common.cuh"
 #include "kernels.h"
@@ -22,6 +24,8 @@ bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols,
 namespace {
 
 constexpr int HD = 128;
+constexpr int STAGES = 3;
+constexpr int STG_LD = HD + 1;   // fp32 staging row stride (bank-conflict-free column writes)
 constexpr float LOG2E_B = 1.4426950408889634f;
 
 struct TcBwdParams {
@@ -30,7 +34,7 @@ struct TcBwdParams {
   const float* lse;        // [H, T] natural log
   const float* D;          // [H, T]
   bf16* dqkv; int ld_dqkv;
-  const float2* rope_cs;
+  const float2* rope_cs;   // [max_pos][HD/2] (cos, sin)
   int T, H, Hkv;
   float scale;
 };
@@ -40,7 +44,7 @@ __device__ __forceinline__ void bw_wait(uint64_t* bar, uint32_t parity) {
   uint64_t t0 = 0;
   for (uint32_t n = 0;; ++n) {
     uint32_t ok;
-    asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.b32 %0, 1, 0, P;\n\t}"
+    asm volatile("{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.b32 %0, 1, 0, P;\n\t}"
                  : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
     if (ok) return;
     if ((n & 255) == 255) {
@@ -52,48 +56,115 @@ __device__ __forceinline__ void bw_wait(uint64_t* bar, uint32_t parity) {
   }
 }
 
-// write 64 bf16 of one row into a [rows][64] SWIZZLE_128B K-major tile
-__device__ __forceinline__ void st_row64_sw128(uint8_t* tile, int row, const float (&v)[64]) {
+#ifdef MENOS_BWD_TRACE
+__device__ __forceinline__ unsigned long long gtime() { unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
+#define TRACED() ((blockIdx.x == 0 || blockIdx.x == 36) && (blockIdx.y == 0 || blockIdx.y == 20))
+#define TR_DECL const unsigned long long T0 = gtime(); unsigned long long tr_a[8] = {0}, tr_b[8] = {0}, tr_c[4] = {0};
+#define TR_A(i) if ((i) < 8) tr_a[i] = gtime() - T0;
+#define TR_B(i) if ((i) < 8) tr_b[i] = gtime() - T0;
+#define TR_C(i) tr_c[i] = gtime() - T0;
+#define TR_PRINT(tag) if (TRACED()) printf("%s %d,%d n %d: a %llu %llu %llu %llu %llu %llu %llu %llu | b %llu %llu %llu %llu %llu %llu %llu %llu | c %llu %llu %llu %llu\n", tag, blockIdx.x, blockIdx.y, nblk, \
+  tr_a[0], tr_a[1], tr_a[2], tr_a[3], tr_a[4], tr_a[5], tr_a[6], tr_a[7], tr_b[0], tr_b[1], tr_b[2], tr_b[3], tr_b[4], tr_b[5], tr_b[6], tr_b[7], tr_c[0], tr_c[1], tr_c[2], tr_c[3]);
+#else
+#define TR_DECL
+#define TR_A(i)
+#define TR_B(i)
+#define TR_C(i)
+#define TR_PRINT(tag)
+#endif
+
+constexpr int EW_WARPS = 8;                 // two warpgroups: each owns half of the S / dP columns
+constexpr int NTHREADS = 64 + 32 * EW_WARPS;
+
+// named barrier over the elementwise warps
+__device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
+
+// long waits of the producer / MMA warps: suspend-capable try_wait so they do not steal issue slots from the
+// elementwise warps that share their schedulers
+__device__ __forceinline__ void bw_wait_idle(uint64_t* bar, uint32_t parity) {
+  uint64_t t0 = 0;
+  for (uint32_t n = 0;; ++n) {
+    uint32_t ok;
+    asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.b32 %0, 1, 0, P;\n\t}"
+                 : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    if (ok) return;
+    if ((n & 15) == 15) {
+      uint64_t t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 2000000000ull) __trap();
+    }
+  }
+}
+
+// 32 lanes x 32 fp32 columns without the trailing wait (batch several, then tmem_wait_ld)
+__device__ __forceinline__ void tmem_ld32_nw(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// write columns [32 g, 32 g + 32) (bf16) of one row of a [rows][64] SWIZZLE_128B K-major tile
+__device__ __forceinline__ void st_half_row_sw128(uint8_t* tile, int row, int g, const float (&v)[32]) {
   uint8_t* prow = tile + row * 128;
 #pragma unroll
-  for (int c8 = 0; c8 < 8; ++c8) {
-    uint4 u = make_uint4(pack_bf16x2(v[8 * c8 + 0], v[8 * c8 + 1]), pack_bf16x2(v[8 * c8 + 2], v[8 * c8 + 3]),
-                         pack_bf16x2(v[8 * c8 + 4], v[8 * c8 + 5]), pack_bf16x2(v[8 * c8 + 6], v[8 * c8 + 7]));
+  for (int c = 0; c < 4; ++c) {
+    const int c8 = 4 * g + c;
+    uint4 u = make_uint4(pack_bf16x2(v[8 * c + 0], v[8 * c + 1]), pack_bf16x2(v[8 * c + 2], v[8 * c + 3]),
+                         pack_bf16x2(v[8 * c + 4], v[8 * c + 5]), pack_bf16x2(v[8 * c + 6], v[8 * c + 7]));
     *reinterpret_cast<uint4*>(prow + ((c8 ^ (row & 7)) << 4)) = u;
   }
 }
 
-__device__ __forceinline__ void tmem_ld64(uint32_t taddr, float (&v)[64]) {
-  float a[32], b[32];
-  tmem_ld32(taddr, a);
-  tmem_ld32(taddr + 32, b);
+// Epilogue phase A: thread (row r, column half g) moves accumulator columns [64 g, 64 g + 64) to staging row r.
+__device__ __forceinline__ void stage_acc(uint32_t tacc, float* stg, int r, int g) {
+  float* row = stg + r * STG_LD + 64 * g;
+  uint32_t a[32], b[32];
+  tmem_ld32_nw(tacc + 64 * g, a);
+  tmem_ld32_nw(tacc + 64 * g + 32, b);
+  tmem_wait_ld();
 #pragma unroll
-  for (int c = 0; c < 32; ++c) { v[c] = a[c]; v[32 + c] = b[c]; }
+  for (int i = 0; i < 32; ++i) { row[i] = __uint_as_float(a[i]); row[32 + i] = __uint_as_float(b[i]); }
 }
 
-// RoPE backward on a full 128-wide row held as 4 chunks of 32 (pairs j, j+64): dx_j = dy_j c + dy_{j+64} s,
-// dx_{j+64} = dy_{j+64} c - dy_j s
-__device__ __forceinline__ void rope_bwd_row(float (&r0)[32], float (&r1)[32], float (&r2)[32], float (&r3)[32],
-                                             const float2* cs) {
+// Epilogue phase B: elementwise warp w8 (0..7) writes staged rows [16 w8, 16 w8 + 16) to dst (bf16), lanes across
+// columns (coalesced), 8 rows in flight; with rope, applies the RoPE backward (pairs j, j+64):
+// dx_j = dy_j c + dy_{j+64} s, dx_{j+64} = dy_{j+64} c - dy_j s.
+__device__ __forceinline__ void store_rows(const float* stg, int w8, int lane, int row0, int n_valid,
+                                           bf16* dst, int ld, const float2* cs, bool rope) {
+  const int j = 2 * lane;   // this lane: columns j, j+1 and j+64, j+65
 #pragma unroll
-  for (int j = 0; j < 32; ++j) {
-    float2 e = cs[j];
-    float y1 = r0[j], y2 = r2[j];
-    r0[j] = y1 * e.x + y2 * e.y;
-    r2[j] = y2 * e.x - y1 * e.y;
-    e = cs[32 + j];
-    y1 = r1[j]; y2 = r3[j];
-    r1[j] = y1 * e.x + y2 * e.y;
-    r3[j] = y2 * e.x - y1 * e.y;
+  for (int half = 0; half < 2; ++half) {
+    float4 e[8];
+    float a0[8], a1[8], b0[8], b1[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int rr = w8 * 16 + half * 8 + u;
+      const float* s = stg + rr * STG_LD;
+      a0[u] = s[j]; a1[u] = s[j + 1]; b0[u] = s[64 + j]; b1[u] = s[65 + j];
+      if (rope && rr < n_valid) e[u] = *reinterpret_cast<const float4*>(cs + (size_t)(row0 + rr) * (HD / 2) + j);
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int rr = w8 * 16 + half * 8 + u;
+      if (rr >= n_valid) continue;
+      float x0 = a0[u], x1 = a1[u], y0 = b0[u], y1 = b1[u];
+      if (rope) {   // e = (c_j, s_j, c_j+1, s_j+1)
+        x0 = a0[u] * e[u].x + b0[u] * e[u].y; y0 = b0[u] * e[u].x - a0[u] * e[u].y;
+        x1 = a1[u] * e[u].z + b1[u] * e[u].w; y1 = b1[u] * e[u].z - a1[u] * e[u].w;
+      }
+      bf16* d = dst + (size_t)rr * ld;
+      *reinterpret_cast<uint32_t*>(d + j) = pack_bf16x2(x0, x1);
+      *reinterpret_cast<uint32_t*>(d + 64 + j) = pack_bf16x2(y0, y1);
+    }
   }
-}
-
-__device__ __forceinline__ void st_row32_bf16(bf16* dst, const float (&v)[32]) {
-  uint4* d = reinterpret_cast<uint4*>(dst);
-#pragma unroll
-  for (int q = 0; q < 4; ++q)
-    d[q] = make_uint4(pack_bf16x2(v[8 * q], v[8 * q + 1]), pack_bf16x2(v[8 * q + 2], v[8 * q + 3]),
-                      pack_bf16x2(v[8 * q + 4], v[8 * q + 5]), pack_bf16x2(v[8 * q + 6], v[8 * q + 7]));
 }
 
 // ======================================================================================= dK / dV kernel
@@ -101,26 +172,23 @@ constexpr int KV_ROWS = 128, QB = 64;
 constexpr int KV_TILE = KV_ROWS * HD * 2;      // 32 KB (2 atoms [128][64])
 constexpr int QB_TILE = QB * HD * 2;           // 16 KB (2 atoms [64][64])
 constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
-constexpr int SMEM_DKDV = 2 * KV_TILE + 4 * QB_TILE + 4 * PT_TILE + 1024;   // 193 KB
+constexpr int SMEM_DKDV = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;   // 225 KB
+static_assert(2 * KV_ROWS * STG_LD * 4 <= SMEM_DKDV - 1024, "dK/dV staging must fit in the freed buffers");
 
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
                         const __grid_constant__ CUtensorMap tmDO64, const TcBwdParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* sK = smem;
-  uint8_t* sV = sK + KV_TILE;
-  // stage b of each double buffer at base + b * tile
-  uint8_t* const sQ0 = sV + KV_TILE;              // Q stages
-  uint8_t* const sO0 = sQ0 + 2 * QB_TILE;         // dO stages
-  uint8_t* const sP0 = sO0 + 2 * QB_TILE;         // P^T
-  uint8_t* const sS0 = sP0 + 2 * PT_TILE;         // dS^T
-#define sQ(b) (sQ0 + (b) * QB_TILE)
-#define sO(b) (sO0 + (b) * QB_TILE)
-#define sP(b) (sP0 + (b) * PT_TILE)
-#define sS(b) (sS0 + (b) * PT_TILE)
-  __shared__ __align__(8) uint64_t bar_kv, full[2], empty[2], s_full[2], ew_done[2], acc_done;
+  uint8_t* const sK = smem;
+  uint8_t* const sV = sK + KV_TILE;
+  uint8_t* const sQ0 = sV + KV_TILE;                  // Q stages
+  uint8_t* const sO0 = sQ0 + STAGES * QB_TILE;        // dO stages
+  uint8_t* const sP0 = sO0 + STAGES * QB_TILE;        // P^T  (2 buffers)
+  uint8_t* const sS0 = sP0 + 2 * PT_TILE;             // dS^T (2 buffers)
+  __shared__ __align__(8) uint64_t bar_kv, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2], acc_done;
   __shared__ uint32_t tmem_sh;
+  __shared__ float s_lse[2][QB], s_D[2][QB];
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int2 kb = p.blocks[blockIdx.x];
@@ -130,12 +198,12 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   const int nqb = (L - k0 + QB - 1) / QB;      // q blocks [k0, L)
   const int nblk = rep * nqb;
 
+  TR_DECL
   if (threadIdx.x == 0) {
     tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO64);
     mbar_init(&bar_kv, 1);
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&full[i], 1); mbar_init(&empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], 4);
-    }
+    for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
     mbar_init(&acc_done, 1);
     fence_barrier_init();
   }
@@ -144,9 +212,7 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_sh;
-#define tS(b) (tmem + 64 * (b))
-#define tP(b) (tmem + 128 + 64 * (b))
-  const uint32_t tdV = tmem + 256, tdK = tmem + 384;
+  const uint32_t tdV = tmem + 256, tdK = tmem + 384;   // S^T buffers at 0/64, dP^T at 128/192
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
@@ -157,52 +223,59 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       tma_load_2d(sV, &tmQKV128, &bar_kv, vcol, base + k0);
       tma_load_2d(sV + 16384, &tmQKV128, &bar_kv, vcol + 64, base + k0);
       for (int it = 0; it < nblk; ++it) {
-        const int b = it & 1;
+        const int st = it % STAGES;
         const int h = hk * rep + it / nqb, q0 = k0 + (it % nqb) * QB;
-        bw_wait(&empty[b], ((it >> 1) & 1) ^ 1);
-        mbar_expect_tx(&full[b], 2 * QB_TILE);
-        tma_load_2d(sQ(b), &tmQKV64, &full[b], h * HD, base + q0);
-        tma_load_2d(sQ(b) + 8192, &tmQKV64, &full[b], h * HD + 64, base + q0);
-        tma_load_2d(sO(b), &tmDO64, &full[b], h * HD, base + q0);
-        tma_load_2d(sO(b) + 8192, &tmDO64, &full[b], h * HD + 64, base + q0);
+        bw_wait_idle(&empty[st], ((it / STAGES) & 1) ^ 1);
+        mbar_expect_tx(&full[st], 2 * QB_TILE);
+        uint8_t* q = sQ0 + st * QB_TILE;
+        uint8_t* o = sO0 + st * QB_TILE;
+        tma_load_2d(q, &tmQKV64, &full[st], h * HD, base + q0);
+        tma_load_2d(q + 8192, &tmQKV64, &full[st], h * HD + 64, base + q0);
+        tma_load_2d(o, &tmDO64, &full[st], h * HD, base + q0);
+        tma_load_2d(o + 8192, &tmDO64, &full[st], h * HD + 64, base + q0);
       }
     }
   } else if (warp == 1) {
     // ------------------------------------------------ MMA issuer
     constexpr uint32_t ID_S = umma_idesc_bf16(128, QB, 0);     // [128 kv] x [64 q], K = hd
     constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 kv] x [128 hd], K = 64 q, B MN-major
-    bw_wait(&bar_kv, 0);
+    bw_wait_idle(&bar_kv, 0);
+    TR_C(0)
     tc_fence_after();
     auto issue_acc = [&](int itp) {  // dV += P^T dO ; dK += dS^T Q   for block itp
-      const int bp = itp & 1;
-      bw_wait(&ew_done[bp], (itp >> 1) & 1);
+      const int bp = itp & 1, sp = itp % STAGES;
+      bw_wait_idle(&ew_done[bp], (itp >> 1) & 1);
+      TR_B(itp)
       tc_fence_after();
       __syncwarp();
       if (elect_one()) {
-        const uint32_t pa = smem_u32(sP(bp)), sa = smem_u32(sS(bp));
-        const uint32_t ob = smem_u32(sO(bp)), qb = smem_u32(sQ(bp));
+        const uint32_t pa = smem_u32(sP0 + bp * PT_TILE), sa = smem_u32(sS0 + bp * PT_TILE);
+        const uint32_t ob = smem_u32(sO0 + sp * QB_TILE), qb = smem_u32(sQ0 + sp * QB_TILE);
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk) {
           const uint32_t acc = (itp > 0 || kk > 0) ? 1u : 0u;
           tc_mma_bf16(tdV, umma_desc_sw128(pa + kk * 32, 16, 1024), umma_desc_sw128(ob + kk * 2048, 8192, 1024), ID_ACC, acc);
           tc_mma_bf16(tdK, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(qb + kk * 2048, 8192, 1024), ID_ACC, acc);
         }
-        tc_commit(&empty[bp]);   // frees the Q/dO stage and the P/dS buffer of block itp
+        tc_commit(&empty[sp]);     // Q/dO stage free
+        tc_commit(&pd_free[bp]);   // P^T/dS^T buffer free
       }
       __syncwarp();
     };
     for (int it = 0; it < nblk; ++it) {
-      const int b = it & 1;
-      bw_wait(&full[b], (it >> 1) & 1);
+      const int b = it & 1, st = it % STAGES;
+      bw_wait_idle(&full[st], (it / STAGES) & 1);
+      TR_A(it)
       tc_fence_after();
       __syncwarp();
       if (elect_one()) {
-        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(b)), o = smem_u32(sO(b));
+        const uint32_t k = smem_u32(sK), v = smem_u32(sV);
+        const uint32_t q = smem_u32(sQ0 + st * QB_TILE), o = smem_u32(sO0 + st * QB_TILE);
 #pragma unroll
         for (int kk = 0; kk < 8; ++kk) {
           const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
-          tc_mma_bf16(tS(b), umma_desc_sw128(k + offa, 16, 1024), umma_desc_sw128(q + offb, 16, 1024), ID_S, kk > 0);
-          tc_mma_bf16(tP(b), umma_desc_sw128(v + offa, 16, 1024), umma_desc_sw128(o + offb, 16, 1024), ID_S, kk > 0);
+          tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(k + offa, 16, 1024), umma_desc_sw128(q + offb, 16, 1024), ID_S, kk > 0);
+          tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(v + offa, 16, 1024), umma_desc_sw128(o + offb, 16, 1024), ID_S, kk > 0);
         }
         tc_commit(&s_full[b]);
       }
@@ -213,64 +286,70 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     __syncwarp();
     if (elect_one()) tc_commit(&acc_done);
     __syncwarp();
+    TR_C(1)
+    if (lane == 0) { TR_PRINT("MMA") }
   } else {
-    // ------------------------------------------------ elementwise warps (thread = key row = TMEM lane)
-    const int q4 = warp & 3;
-    const int r = q4 * 32 + lane;           // key row within the block
+    // ------------------------------------------------ elementwise warps (thread = key row = TMEM lane;
+    //                                                  warpgroup g owns query columns [32 g, 32 g + 32))
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
+    const int r = w4 * 32 + lane;           // key row within the block
     const int kpos = k0 + r;
-    const uint32_t lane_off = (uint32_t)(q4 * 32) << 16;
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_B;
     for (int it = 0; it < nblk; ++it) {
       const int b = it & 1;
       const int h = hk * rep + it / nqb, q0 = k0 + (it % nqb) * QB;
+      if (t < 2 * QB) {  // stage lse (log2 domain) and D of the block's 64 queries
+        const int c = t & (QB - 1), qpos = q0 + c;
+        const float* src = (t < QB ? p.lse : p.D) + (size_t)h * p.T + base + qpos;
+        const float v = qpos < L ? __ldg(src) : 0.f;
+        if (t < QB) s_lse[b][c] = v * LOG2E_B; else s_D[b][c] = v;
+      }
+      ew_sync();
       bw_wait(&s_full[b], (it >> 1) & 1);
+      TR_A(it)
       tc_fence_after();
       __syncwarp();
-      float s[64], dp[64];
-      tmem_ld64(tS(b) + lane_off, s);
-      tmem_ld64(tP(b) + lane_off, dp);
-      const float* lse_h = p.lse + (size_t)h * p.T + base;
-      const float* D_h = p.D + (size_t)h * p.T + base;
+      uint32_t su[32], du[32];
+      tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
+      tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+      tmem_wait_ld();
+      const int cmin = kpos - q0 - 32 * g;   // P = 0 for queries before the key (causal) ...
+      const int cmax = L - q0 - 32 * g;      // ... and past the end of the sequence
+      float pv[32], dsv[32];
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
-        const int qpos = q0 + c;
-        float pv = 0.f, dsv = 0.f;
-        if (qpos < L && kpos <= qpos) {
-          pv = exp2f(s[c] * sl2 - __ldg(lse_h + qpos) * LOG2E_B);
-          dsv = pv * (dp[c] - __ldg(D_h + qpos)) * p.scale;
-        }
-        s[c] = pv;
-        dp[c] = dsv;
+      for (int c = 0; c < 32; ++c) {
+        const bool ok = c >= cmin && c < cmax;
+        const float e = exp2f(__uint_as_float(su[c]) * sl2 - s_lse[b][32 * g + c]);
+        pv[c] = ok ? e : 0.f;
+        dsv[c] = ok ? e * (__uint_as_float(du[c]) - s_D[b][32 * g + c]) * p.scale : 0.f;
       }
-      // the P^T / dS^T buffer b was last read by the dV/dK MMAs of block it-2
-      if (it >= 2) bw_wait(&empty[b], ((it - 2) >> 1) & 1);
-      st_row64_sw128(sP(b), r, s);
-      st_row64_sw128(sS(b), r, dp);
+      if (it >= 2) bw_wait(&pd_free[b], ((it - 2) >> 1) & 1);
+      st_half_row_sw128(sP0 + b * PT_TILE, r, g, pv);
+      st_half_row_sw128(sS0 + b * PT_TILE, r, g, dsv);
       fence_proxy_async();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&ew_done[b]);
+      TR_B(it)
     }
+    TR_C(0)
     // ------------------------------------------------ epilogue: dK (RoPE bwd), dV rows -> dqkv
     bw_wait(&acc_done, 0);
+    TR_C(1)
     tc_fence_after();
     __syncwarp();
-    const bool rok = kpos < L;
-    float a0[32], a1[32], a2[32], a3[32];
-    tmem_ld32(tdK + lane_off, a0);
-    tmem_ld32(tdK + lane_off + 32, a1);
-    tmem_ld32(tdK + lane_off + 64, a2);
-    tmem_ld32(tdK + lane_off + 96, a3);
-    const int ps = rok ? kpos : 0;
-    rope_bwd_row(a0, a1, a2, a3, p.rope_cs + (size_t)ps * (HD / 2));
-    bf16* krow = p.dqkv + (size_t)(base + ps) * p.ld_dqkv + kcol;
-    if (rok) { st_row32_bf16(krow, a0); st_row32_bf16(krow + 32, a1); st_row32_bf16(krow + 64, a2); st_row32_bf16(krow + 96, a3); }
-    tmem_ld32(tdV + lane_off, a0);
-    tmem_ld32(tdV + lane_off + 32, a1);
-    tmem_ld32(tdV + lane_off + 64, a2);
-    tmem_ld32(tdV + lane_off + 96, a3);
-    bf16* vrow = p.dqkv + (size_t)(base + ps) * p.ld_dqkv + vcol;
-    if (rok) { st_row32_bf16(vrow, a0); st_row32_bf16(vrow + 32, a1); st_row32_bf16(vrow + 64, a2); st_row32_bf16(vrow + 96, a3); }
+    float* stgK = reinterpret_cast<float*>(smem);            // every MMA has completed: all buffers are free
+    float* stgV = stgK + KV_ROWS * STG_LD;
+    stage_acc(tdK + lane_off, stgK, r, g);
+    stage_acc(tdV + lane_off, stgV, r, g);
+    ew_sync();
+    TR_C(2)
+    const int nv = min(KV_ROWS, L - k0);
+    store_rows(stgK, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + kcol, p.ld_dqkv, p.rope_cs, true);
+    store_rows(stgV, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + vcol, p.ld_dqkv, p.rope_cs, false);
+    TR_C(3)
+    if (threadIdx.x == 64) { TR_PRINT("EW") }
   }
   tc_fence_before();
   __syncthreads();
@@ -285,21 +364,20 @@ constexpr int Q_ROWS = 128, KB = 64;
 constexpr int Q_TILE = Q_ROWS * HD * 2;       // 32 KB
 constexpr int KB_TILE = KB * HD * 2;          // 16 KB
 constexpr int DS_TILE = Q_ROWS * KB * 2;      // 16 KB
-constexpr int SMEM_DQ = 2 * Q_TILE + 4 * KB_TILE + 2 * DS_TILE + 1024;   // 161 KB
+constexpr int SMEM_DQ = 2 * Q_TILE + 2 * STAGES * KB_TILE + 2 * DS_TILE + 1024;   // 193 KB
+static_assert(Q_ROWS * STG_LD * 4 <= SMEM_DQ - 1024, "dQ staging must fit in the freed buffers");
 
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
                       const __grid_constant__ CUtensorMap tmDO128, const TcBwdParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* const sQ1 = smem;
-  uint8_t* const sO1 = sQ1 + Q_TILE;
-  uint8_t* const sK0 = sO1 + Q_TILE;
-  uint8_t* const sV0 = sK0 + 2 * KB_TILE;
-  uint8_t* const sS0 = sV0 + 2 * KB_TILE;
-#define sK(b) (sK0 + (b) * KB_TILE)
-#define sV(b) (sV0 + (b) * KB_TILE)
-  __shared__ __align__(8) uint64_t bar_q, full[2], empty[2], s_full[2], ew_done[2], acc_done;
+  uint8_t* const sQ = smem;
+  uint8_t* const sO = sQ + Q_TILE;
+  uint8_t* const sK0 = sO + Q_TILE;                  // K stages
+  uint8_t* const sV0 = sK0 + STAGES * KB_TILE;       // V stages
+  uint8_t* const sS0 = sV0 + STAGES * KB_TILE;       // dS (2 buffers)
+  __shared__ __align__(8) uint64_t bar_q, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2], acc_done;
   __shared__ uint32_t tmem_sh;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -312,9 +390,8 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   if (threadIdx.x == 0) {
     tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO128);
     mbar_init(&bar_q, 1);
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&full[i], 1); mbar_init(&empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], 4);
-    }
+    for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
     mbar_init(&acc_done, 1);
     fence_barrier_init();
   }
@@ -323,57 +400,61 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_sh;
-  const uint32_t tdQ = tmem + 256;
+  const uint32_t tdQ = tmem + 256;   // S buffers at 0/64, dP at 128/192
 
   if (warp == 0) {
     if (elect_one()) {
       mbar_expect_tx(&bar_q, 2 * Q_TILE);
-      tma_load_2d(sQ1, &tmQKV128, &bar_q, h * HD, base + q0);
-      tma_load_2d(sQ1 + 16384, &tmQKV128, &bar_q, h * HD + 64, base + q0);
-      tma_load_2d(sO1, &tmDO128, &bar_q, h * HD, base + q0);
-      tma_load_2d(sO1 + 16384, &tmDO128, &bar_q, h * HD + 64, base + q0);
+      tma_load_2d(sQ, &tmQKV128, &bar_q, h * HD, base + q0);
+      tma_load_2d(sQ + 16384, &tmQKV128, &bar_q, h * HD + 64, base + q0);
+      tma_load_2d(sO, &tmDO128, &bar_q, h * HD, base + q0);
+      tma_load_2d(sO + 16384, &tmDO128, &bar_q, h * HD + 64, base + q0);
       for (int it = 0; it < nkb; ++it) {
-        const int b = it & 1;
-        bw_wait(&empty[b], ((it >> 1) & 1) ^ 1);
-        mbar_expect_tx(&full[b], 2 * KB_TILE);
-        tma_load_2d(sK(b), &tmQKV64, &full[b], kcol, base + it * KB);
-        tma_load_2d(sK(b) + 8192, &tmQKV64, &full[b], kcol + 64, base + it * KB);
-        tma_load_2d(sV(b), &tmQKV64, &full[b], vcol, base + it * KB);
-        tma_load_2d(sV(b) + 8192, &tmQKV64, &full[b], vcol + 64, base + it * KB);
+        const int st = it % STAGES;
+        bw_wait_idle(&empty[st], ((it / STAGES) & 1) ^ 1);
+        mbar_expect_tx(&full[st], 2 * KB_TILE);
+        uint8_t* k = sK0 + st * KB_TILE;
+        uint8_t* v = sV0 + st * KB_TILE;
+        tma_load_2d(k, &tmQKV64, &full[st], kcol, base + it * KB);
+        tma_load_2d(k + 8192, &tmQKV64, &full[st], kcol + 64, base + it * KB);
+        tma_load_2d(v, &tmQKV64, &full[st], vcol, base + it * KB);
+        tma_load_2d(v + 8192, &tmQKV64, &full[st], vcol + 64, base + it * KB);
       }
     }
   } else if (warp == 1) {
     constexpr uint32_t ID_S = umma_idesc_bf16(128, KB, 0);     // [128 q] x [64 keys], K = hd
     constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 q] x [128 hd], K = 64 keys, B MN-major
-    bw_wait(&bar_q, 0);
+    bw_wait_idle(&bar_q, 0);
     tc_fence_after();
     auto issue_acc = [&](int itp) {  // dQ += dS K  for key block itp
-      const int bp = itp & 1;
-      bw_wait(&ew_done[bp], (itp >> 1) & 1);
+      const int bp = itp & 1, sp = itp % STAGES;
+      bw_wait_idle(&ew_done[bp], (itp >> 1) & 1);
       tc_fence_after();
       __syncwarp();
       if (elect_one()) {
-        const uint32_t sa = smem_u32(sS(bp)), kb_ = smem_u32(sK(bp));
+        const uint32_t sa = smem_u32(sS0 + bp * DS_TILE), kb_ = smem_u32(sK0 + sp * KB_TILE);
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk)
           tc_mma_bf16(tdQ, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(kb_ + kk * 2048, 8192, 1024), ID_ACC,
                       (itp > 0 || kk > 0) ? 1u : 0u);
-        tc_commit(&empty[bp]);
+        tc_commit(&empty[sp]);
+        tc_commit(&pd_free[bp]);
       }
       __syncwarp();
     };
     for (int it = 0; it < nkb; ++it) {
-      const int b = it & 1;
-      bw_wait(&full[b], (it >> 1) & 1);
+      const int b = it & 1, st = it % STAGES;
+      bw_wait_idle(&full[st], (it / STAGES) & 1);
       tc_fence_after();
       __syncwarp();
       if (elect_one()) {
-        const uint32_t q = smem_u32(sQ1), o = smem_u32(sO1), k = smem_u32(sK(b)), v = smem_u32(sV(b));
+        const uint32_t q = smem_u32(sQ), o = smem_u32(sO);
+        const uint32_t k = smem_u32(sK0 + st * KB_TILE), v = smem_u32(sV0 + st * KB_TILE);
 #pragma unroll
         for (int kk = 0; kk < 8; ++kk) {
           const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
-          tc_mma_bf16(tS(b), umma_desc_sw128(q + offa, 16, 1024), umma_desc_sw128(k + offb, 16, 1024), ID_S, kk > 0);
-          tc_mma_bf16(tP(b), umma_desc_sw128(o + offa, 16, 1024), umma_desc_sw128(v + offb, 16, 1024), ID_S, kk > 0);
+          tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(q + offa, 16, 1024), umma_desc_sw128(k + offb, 16, 1024), ID_S, kk > 0);
+          tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(o + offa, 16, 1024), umma_desc_sw128(v + offb, 16, 1024), ID_S, kk > 0);
         }
         tc_commit(&s_full[b]);
       }
@@ -385,10 +466,10 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     if (elect_one()) tc_commit(&acc_done);
     __syncwarp();
   } else {
-    const int q4 = warp & 3;
-    const int r = q4 * 32 + lane;           // query row
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2;   // warpgroup g owns key columns [32 g, 32 g + 32)
+    const int r = w4 * 32 + lane;           // query row
     const int qpos = q0 + r;
-    const uint32_t lane_off = (uint32_t)(q4 * 32) << 16;
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_B;
     const bool qok = qpos < L;
     const float lse2 = qok ? p.lse[(size_t)h * p.T + base + qpos] * LOG2E_B : 0.f;
@@ -398,18 +479,19 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       bw_wait(&s_full[b], (it >> 1) & 1);
       tc_fence_after();
       __syncwarp();
-      float s[64], dp[64];
-      tmem_ld64(tS(b) + lane_off, s);
-      tmem_ld64(tP(b) + lane_off, dp);
+      uint32_t su[32], du[32];
+      tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
+      tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+      tmem_wait_ld();
+      const int cmax = qok ? qpos - it * KB - 32 * g : -1;   // keys <= query
+      float dsv[32];
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
-        const int key = it * KB + c;
-        float dsv = 0.f;
-        if (qok && key <= qpos) dsv = exp2f(s[c] * sl2 - lse2) * (dp[c] - Dq) * p.scale;
-        dp[c] = dsv;
+      for (int c = 0; c < 32; ++c) {
+        const float v = exp2f(__uint_as_float(su[c]) * sl2 - lse2) * (__uint_as_float(du[c]) - Dq) * p.scale;
+        dsv[c] = c <= cmax ? v : 0.f;
       }
-      if (it >= 2) bw_wait(&empty[b], ((it - 2) >> 1) & 1);
-      st_row64_sw128(sS(b), r, dp);
+      if (it >= 2) bw_wait(&pd_free[b], ((it - 2) >> 1) & 1);
+      st_half_row_sw128(sS0 + b * DS_TILE, r, g, dsv);
       fence_proxy_async();
       tc_fence_before();
       __syncwarp();
@@ -418,15 +500,11 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     bw_wait(&acc_done, 0);
     tc_fence_after();
     __syncwarp();
-    float a0[32], a1[32], a2[32], a3[32];
-    tmem_ld32(tdQ + lane_off, a0);
-    tmem_ld32(tdQ + lane_off + 32, a1);
-    tmem_ld32(tdQ + lane_off + 64, a2);
-    tmem_ld32(tdQ + lane_off + 96, a3);
-    const int ps = qok ? qpos : 0;
-    rope_bwd_row(a0, a1, a2, a3, p.rope_cs + (size_t)ps * (HD / 2));
-    bf16* qrow = p.dqkv + (size_t)(base + ps) * p.ld_dqkv + h * HD;
-    if (qok) { st_row32_bf16(qrow, a0); st_row32_bf16(qrow + 32, a1); st_row32_bf16(qrow + 64, a2); st_row32_bf16(qrow + 96, a3); }
+    float* stg = reinterpret_cast<float*>(smem);
+    stage_acc(tdQ + lane_off, stg, r, g);
+    ew_sync();
+    const int nv = min(Q_ROWS, L - q0);
+    store_rows(stg, w8, lane, q0, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD, p.ld_dqkv, p.rope_cs, true);
   }
   tc_fence_before();
   __syncthreads();
@@ -456,9 +534,9 @@ int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaS
     cudaFuncSetAttribute(attn_bwd_dq_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DQ);
     attr = true;
   }
-  attn_bwd_dkdv_tc_kernel<<<dim3(n_blocks128, a.Hkv), 192, SMEM_DKDV, st>>>(mQKV128, mQKV64, mDO64, p);
+  attn_bwd_dkdv_tc_kernel<<<dim3(n_blocks128, a.Hkv), NTHREADS, SMEM_DKDV, st>>>(mQKV128, mQKV64, mDO64, p);
   ++g_launch_count;
-  attn_bwd_dq_tc_kernel<<<dim3(n_blocks128, a.H), 192, SMEM_DQ, st>>>(mQKV128, mQKV64, mDO128, p);
+  attn_bwd_dq_tc_kernel<<<dim3(n_blocks128, a.H), NTHREADS, SMEM_DQ, st>>>(mQKV128, mQKV64, mDO128, p);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }
