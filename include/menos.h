@@ -49,7 +49,7 @@ typedef enum {
   MENOS_ENOCLIENT = -3, /* unknown client id                                                     */
   MENOS_ESTATE = -4,    /* e.g. backward on a batch without a live forward, weights not loaded    */
   MENOS_ECUDA = -5,     /* CUDA error (sticky until menos_sync)                                   */
-  MENOS_ENCCL = -6      /* reserved: tensor-parallel communicator error                           */
+  MENOS_ENCCL = -6      /* tensor-parallel all-reduce callback failed (menos_tp_cfg)             */
 } menos_status;
 
 typedef struct menos_server menos_server;
@@ -67,7 +67,9 @@ typedef struct {
 
 /* One decoder layer's frozen base weights, natural (HF) layouts, bf16 row-major, host or device.
  * The library COPIES them into its single device copy (WeightStore); the caller may free them after the
- * call returns.  hd = d_model / n_heads. */
+ * call returns.  hd = d_model / n_heads.  Under tensor parallelism (opts->tp.world = W > 1) every projection
+ * is the rank's SHARD with H, H_kv, f replaced by H/W, H_kv/W, f/W in the shapes below (wo and wdown keep
+ * their d rows and hold the rank's columns); g1, g2 are full. */
 typedef struct {
   const void* wq;    /* [H*hd, d]     */
   const void* wk;    /* [H_kv*hd, d]  */
@@ -91,12 +93,35 @@ typedef struct {
   double lr, beta1, beta2, eps, weight_decay; /* torch.optim.AdamW semantics (scalars in double, as torch forms them) */
 } menos_adamw_cfg;
 
+/* Tensor parallelism (Llama-2-70B, BASELINE.json configs[4]).
+ * Megatron split of every server layer over `world` ranks, one process and one server object per GPU:
+ *   column-parallel: Wq, Wk, Wv (rank r holds heads [r*H/world, (r+1)*H/world) and the matching KV heads),
+ *                    W_gate, W_up (rows [r*f/world, (r+1)*f/world));
+ *   row-parallel:    Wo (columns of rank r's heads), W_down (columns [r*f/world, (r+1)*f/world)).
+ * Per layer the server calls `allreduce` four times (sum, in place, on the call's stream):
+ *   forward  : the o-proj and down-proj partial sums (fp32 [T, d]; rank 0's partial carries the residual);
+ *   backward : the gate|up-dX and qkv-dX partial sums (fp32 [T, d]).
+ * LoRA: column-parallel targets keep A [r, d] replicated and B [N/world, r] sharded; row-parallel targets keep
+ * A [r, K/world] sharded and B [d, r] replicated.  Row-parallel adapters fold into the existing all-reduce by
+ * linearity; the gradients of the replicated tensors (dA of q,k,v,gate,up; dB of o,down) are partial sums and
+ * are all-reduced once per backward per client (one fp32 call over a contiguous region).  No other exchange.
+ * The callback must leave identical bytes on every rank (NCCL / gloo all-reduce do).  It returns 0 on success;
+ * nonzero makes the server call fail with MENOS_ENCCL.  world <= 1: no tensor parallelism (replica). */
+enum { MENOS_DT_F32 = 0, MENOS_DT_BF16 = 1 };
+typedef int (*menos_allreduce_fn)(void* buf, size_t count, int dtype, void* stream, void* user);
+typedef struct {
+  int rank, world;              /* 0 <= rank < world; H, H_kv and d_ff divisible by world              */
+  menos_allreduce_fn allreduce; /* required when world > 1                                              */
+  void* user;                   /* passed back to allreduce                                             */
+} menos_tp_cfg;
+
 typedef struct {
   int max_clients;     /* registry capacity (default 64)                                     */
   int max_rank;        /* largest LoRA rank accepted (default 64)                             */
   int max_seq_len;     /* longest sequence (RoPE table rows; default 4096)                   */
   size_t arena_bytes;  /* activation arena I (Eq.3); 0 = free memory - 8 GiB    */
   int num_sms;         /* persistent-grid width; 0 = device SM count                          */
+  menos_tp_cfg tp;     /* tensor parallelism; zero-initialised = none                          */
 } menos_server_opts;
 
 /* forward flags */
@@ -144,6 +169,7 @@ MENOS_API int menos_batch_free(menos_server* s, menos_batch* batch);
 MENOS_API int menos_adapter_step(menos_server* s, int n, const int32_t* client_ids, void* stream);
 
 /* Host copies of one adapter tensor (fp32).  which: 0 = A [r, K], 1 = B [N, r], 2 = dA, 3 = dB,
+ * (under tensor parallelism K and N are the rank's local extents: see menos_tp_cfg; adapter_shape reports them)
  * 4 = m_A, 5 = m_B, 6 = v_A, 7 = v_B.  layer in 0..n_layers-1, target 0..6 (must be in the client's mask).
  * set_adapter accepts which 0..1 (A, B) and refreshes the bf16 copy.  Both synchronise the device. */
 MENOS_API int menos_adapter_shape(menos_server* s, int32_t id, int target, int* rows, int* cols);

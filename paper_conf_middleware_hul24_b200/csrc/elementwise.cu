@@ -28,6 +28,8 @@ __device__ __forceinline__ void st8b(bf16* p, const float (&v)[8]) {
   *reinterpret_cast<uint4*>(p) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
                                             pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
 }
+__device__ __forceinline__ void ld8(const bf16* p, float (&v)[8]) { ld8b(p, v); }
+__device__ __forceinline__ void ld8(const float* p, float (&v)[8]) { ld8f(p, v); }
 
 // ------------------------------------------------------------------ RMSNorm forward
 // y = x * rstd * g, rstd = rsqrt(mean(x^2) + eps); x fp32 residual stream [T, d]; y bf16 (GEMM operand);
@@ -61,7 +63,8 @@ __global__ void rmsnorm_fwd_kernel(const float* __restrict__ x, const float* __r
 // ------------------------------------------------------------------ RMSNorm backward (+ residual)
 // dx = resid + rstd*(gh - xh*mean(gh*xh)),  gh = dy*g,  xh = x*rstd.   dy bf16 (GEMM output), x / resid / dx
 // fp32 (residual streams); dxb = bf16 copy of dx for the next dX GEMM's A operand (optional).
-__global__ void rmsnorm_bwd_kernel(const bf16* __restrict__ dy, const float* __restrict__ x,
+template <typename TDY>
+__global__ void rmsnorm_bwd_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
                                    const float* __restrict__ g, const float* __restrict__ rstd,
                                    const float* __restrict__ resid, float* __restrict__ dx, bf16* __restrict__ dxb,
                                    int T, int d) {
@@ -72,7 +75,7 @@ __global__ void rmsnorm_bwd_kernel(const bf16* __restrict__ dy, const float* __r
   float dot = 0.f;
   for (int i = lane * 8; i < d; i += 256) {
     float a[8], b[8], gg[8];
-    ld8b(dy + ro + i, a);
+    ld8(dy + ro + i, a);
     ld8f(x + ro + i, b);
     ld8f(g + i, gg);
 #pragma unroll
@@ -82,7 +85,7 @@ __global__ void rmsnorm_bwd_kernel(const bf16* __restrict__ dy, const float* __r
   const float mean = dot * r / (float)d;  // mean(gh * xh) = r * mean(gh * x)
   for (int i = lane * 8; i < d; i += 256) {
     float a[8], b[8], c[8], gg[8], o[8];
-    ld8b(dy + ro + i, a);
+    ld8(dy + ro + i, a);
     ld8f(x + ro + i, b);
     ld8f(resid + ro + i, c);
     ld8f(g + i, gg);
@@ -144,8 +147,8 @@ __global__ void __launch_bounds__(256) rmsnorm_fwd_reg_kernel(const float* __res
   }
 }
 
-template <int NC>
-__global__ void __launch_bounds__(256) rmsnorm_bwd_reg_kernel(const bf16* __restrict__ dy, const float* __restrict__ x,
+template <int NC, typename TDY>
+__global__ void __launch_bounds__(256) rmsnorm_bwd_reg_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
                                                               const float* __restrict__ g, const float* __restrict__ rstd,
                                                               const float* __restrict__ resid, float* __restrict__ dx,
                                                               bf16* __restrict__ dxb, int T, int d) {
@@ -162,7 +165,7 @@ __global__ void __launch_bounds__(256) rmsnorm_bwd_reg_kernel(const bf16* __rest
     const int i = (c * 128 + t) * 8;
     if (ok && i < d) {
       float gg[8];
-      ld8b(dy + ro + i, a[c]);
+      ld8(dy + ro + i, a[c]);
       ld8f(x + ro + i, b[c]);
       ld8f(g + i, gg);
 #pragma unroll
@@ -290,23 +293,32 @@ int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int
   }
   return LAUNCH_CHECK();
 }
-int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
-                bf16* dxb, int T, int d, cudaStream_t st) {
+template <typename TDY>
+static int rmsnorm_bwd_t(const TDY* dy, const float* x, const float* g, const float* rstd, const float* resid,
+                         float* dx, bf16* dxb, int T, int d, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
   const int nc = (d + 1023) / 1024, grid = (T + 1) / 2;
   switch (nc) {
-    case 1: rmsnorm_bwd_reg_kernel<1><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 2: rmsnorm_bwd_reg_kernel<2><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 4: rmsnorm_bwd_reg_kernel<4><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 5: rmsnorm_bwd_reg_kernel<5><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 8: rmsnorm_bwd_reg_kernel<8><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 1: rmsnorm_bwd_reg_kernel<1, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 2: rmsnorm_bwd_reg_kernel<2, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 4: rmsnorm_bwd_reg_kernel<4, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 5: rmsnorm_bwd_reg_kernel<5, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 8: rmsnorm_bwd_reg_kernel<8, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
     default: {
       const int warps = 8;
-      rmsnorm_bwd_kernel<<<(T + warps - 1) / warps, warps * 32, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d);
+      rmsnorm_bwd_kernel<TDY><<<(T + warps - 1) / warps, warps * 32, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d);
     }
   }
   return LAUNCH_CHECK();
+}
+int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
+                bf16* dxb, int T, int d, cudaStream_t st) {
+  return rmsnorm_bwd_t(dy, x, g, rstd, resid, dx, dxb, T, d, st);
+}
+int rmsnorm_bwd_f32dy(const float* dy, const float* x, const float* g, const float* rstd, const float* resid,
+                      float* dx, bf16* dxb, int T, int d, cudaStream_t st) {
+  return rmsnorm_bwd_t(dy, x, g, rstd, resid, dx, dxb, T, d, st);
 }
 int convert_f32_to_bf16(const float* src, bf16* dst, long long n, cudaStream_t st) {
   if (n <= 0) return 0;

@@ -291,12 +291,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           float v[32];
           tmem_ld32(tb + c * 32, v);
           if (rok) {
-            const float4* r4 = reinterpret_cast<const float4*>(p.resid + (size_t)row * p.ldr + col);
             float4* o4 = reinterpret_cast<float4*>(p.outf + (size_t)row * p.ldo + col);
+            if (p.resid) {
+              const float4* r4 = reinterpret_cast<const float4*>(p.resid + (size_t)row * p.ldr + col);
 #pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              const float4 r = r4[q];
-              o4[q] = make_float4(v[4 * q] + r.x, v[4 * q + 1] + r.y, v[4 * q + 2] + r.z, v[4 * q + 3] + r.w);
+              for (int q = 0; q < 8; ++q) {
+                const float4 r = r4[q];
+                o4[q] = make_float4(v[4 * q] + r.x, v[4 * q + 1] + r.y, v[4 * q + 2] + r.z, v[4 * q + 3] + r.w);
+              }
+            } else {   // tensor-parallel partial sum (the residual is added by rank 0 only)
+#pragma unroll
+              for (int q = 0; q < 8; ++q) o4[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
             }
           }
         }

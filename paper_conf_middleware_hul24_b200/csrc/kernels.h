@@ -17,7 +17,7 @@ extern unsigned long long g_launch_count;
 // ---------------------------------------------------------------- tcgen05 GEMM
 enum EpiMode : int {
   EPI_STORE = 0,       // out = bf16(acc)
-  EPI_RESID = 1,       // outf = acc + residf   (fp32 residual stream)
+  EPI_RESID = 1,       // outf = acc + residf   (fp32 residual stream; resid == nullptr: outf = acc)
   EPI_ROPE = 2,        // columns < rope_cols rotated by RoPE at pos[row]; out = bf16
   EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu), out2 = bf16(silu(g) u)
   EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
@@ -75,6 +75,9 @@ int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int
 // dx = resid + rstd*(gh - xh*mean(gh*xh)), gh = dy*g, xh = x*rstd; dxb (optional) = bf16(dx)
 int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
                 bf16* dxb, int T, int d, cudaStream_t st);
+// same with an fp32 incoming gradient (tensor-parallel path: dy is the fp32 all-reduced dX partial sum)
+int rmsnorm_bwd_f32dy(const float* dy, const float* x, const float* g, const float* rstd, const float* resid,
+                      float* dx, bf16* dxb, int T, int d, cudaStream_t st);
 int convert_f32_to_bf16(const float* src, bf16* dst, long long n, cudaStream_t st);       // n % 8 == 0
 int convert_bf16_to_f32_vec(const bf16* src, float* dst, long long n, cudaStream_t st);   // n % 8 == 0
 int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st);

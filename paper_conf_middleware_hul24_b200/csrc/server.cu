@@ -92,7 +92,11 @@ enum { GQKV = 0, GO, GGU, GD, NG };
 static const int kTargetGroup[NT] = {GQKV, GQKV, GQKV, GO, GGU, GGU, GD};
 
 struct Dims {
+  // local (per tensor-parallel rank) extents: H, Hkv, f are the global ones / tp_world
   int d, H, Hkv, hd, f, fpad, Nq, Nkv, Nqkv;
+  int tp_rank, tp_world;
+  int K_glob[NT];                  // global input dim of each projection (LoRA A init bound, A slicing)
+  bool a_rep[NT];                  // A replicated across ranks (column-parallel); else B replicated (row-parallel)
   float eps, theta;
   int K_t[NT], N_t[NT];            // projection input/output dims (natural)
   int K_g[NG], N_g[NG], ldK_g[NG]; // group GEMM input dim, output dim, Acat leading dim
@@ -100,15 +104,20 @@ struct Dims {
   int rb_base[NT], rb_blk[NT], rb_stride[NT];
 };
 
-static Dims make_dims(const menos_model_cfg& c) {
+static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 1) {
   Dims D;
-  D.d = c.d_model; D.H = c.n_heads; D.Hkv = c.n_kv_heads; D.hd = c.d_model / c.n_heads;
-  D.f = c.d_ff; D.fpad = (int)align_up(c.d_ff, 128);
+  D.tp_rank = tp_rank; D.tp_world = tp_world;
+  D.d = c.d_model; D.H = c.n_heads / tp_world; D.Hkv = c.n_kv_heads / tp_world; D.hd = c.d_model / c.n_heads;
+  D.f = c.d_ff / tp_world; D.fpad = (int)align_up(D.f, 128);
   D.Nq = D.H * D.hd; D.Nkv = D.Hkv * D.hd; D.Nqkv = D.Nq + 2 * D.Nkv;
   D.eps = c.rms_eps; D.theta = c.rope_theta;
   const int K[NT] = {D.d, D.d, D.d, D.Nq, D.d, D.d, D.f};
   const int N[NT] = {D.Nq, D.Nkv, D.Nkv, D.d, D.f, D.f, D.d};
-  for (int t = 0; t < NT; ++t) { D.K_t[t] = K[t]; D.N_t[t] = N[t]; }
+  for (int t = 0; t < NT; ++t) {
+    D.K_t[t] = K[t]; D.N_t[t] = N[t];
+    D.a_rep[t] = !(t == TO || t == TD);
+    D.K_glob[t] = D.a_rep[t] ? K[t] : K[t] * tp_world;
+  }
   D.K_g[GQKV] = D.d;  D.N_g[GQKV] = D.Nqkv;    D.ldK_g[GQKV] = D.d;
   D.K_g[GO] = D.Nq;   D.N_g[GO] = D.d;         D.ldK_g[GO] = D.Nq;
   D.K_g[GGU] = D.d;   D.N_g[GGU] = 2 * D.fpad; D.ldK_g[GGU] = D.d;
@@ -177,6 +186,7 @@ struct Client {
   int sub[NT];                      // slot sub-offset of target t inside the group slot (j * rs), -1 if absent
   float* buf = nullptr;             // P | G | M | V, each n_params fp32
   size_t n_params = 0;
+  size_t n_rep = 0;                 // params [0, n_rep) are replicated across tensor-parallel ranks
   std::vector<long long> offA, offB;  // [layer * NT + t]
   float *P() const { return buf; }
   float *G() const { return buf + n_params; }
@@ -265,6 +275,7 @@ struct menos_server {
   Dims D{};
   int first_layer = 0, n_layers = 0, device = 0, num_sms = 148;
   menos_server_opts opts{};
+  menos_tp_cfg tp{0, 1, nullptr, nullptr};  // tensor parallelism (world 1 = replica)
   // WeightStore: one bf16 copy of every server layer, packed for the kernels
   uint8_t* wbuf = nullptr; size_t wbytes = 0;
   struct LW { bf16 *wqkv, *wo, *wgu, *wd; float *g1, *g2; };
@@ -471,10 +482,19 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
   if (prop.major != 10) FAIL(MENOS_ECUDA, "device %d is sm_%d%d; this library is built for sm_100a", device, prop.major, prop.minor);
   CUDA_TRY(cudaSetDevice(device));
 
-  std::unique_ptr<menos_server> s(new menos_server());
-  s->cfg = *cfg; s->D = make_dims(*cfg); s->first_layer = first_layer; s->n_layers = n_layers; s->device = device;
   menos_server_opts o{};
   if (opts) o = *opts;
+  menos_tp_cfg tp = o.tp;
+  if (tp.world <= 1) tp = menos_tp_cfg{0, 1, nullptr, nullptr};
+  if (tp.world > 1) {
+    if (tp.rank < 0 || tp.rank >= tp.world || !tp.allreduce) FAIL(MENOS_EINVAL, "bad tensor-parallel cfg");
+    if (cfg->n_heads % tp.world || cfg->n_kv_heads % tp.world || cfg->d_ff % tp.world)
+      FAIL(MENOS_EINVAL, "H=%d, H_kv=%d, f=%d not divisible by tp world %d", cfg->n_heads, cfg->n_kv_heads,
+           cfg->d_ff, tp.world);
+  }
+  std::unique_ptr<menos_server> s(new menos_server());
+  s->cfg = *cfg; s->D = make_dims(*cfg, tp.rank, tp.world); s->tp = tp;
+  s->first_layer = first_layer; s->n_layers = n_layers; s->device = device;
   if (o.max_clients <= 0) o.max_clients = 64;
   if (o.max_rank <= 0) o.max_rank = 64;
   if (o.max_seq_len <= 0) o.max_seq_len = 4096;
@@ -589,28 +609,39 @@ extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uin
   // parameter layout
   c.offA.assign((size_t)s->n_layers * NT, -1);
   c.offB.assign((size_t)s->n_layers * NT, -1);
+  // replicated tensors first (A of column-parallel targets, B of row-parallel ones), so that under tensor
+  // parallelism their gradient partial sums are one contiguous all-reduce (menos_tp_cfg); with world 1 the
+  // split is immaterial
   size_t n = 0;
-  for (int l = 0; l < s->n_layers; ++l)
-    for (int t = 0; t < NT; ++t) {
-      if (!(target_mask >> t & 1)) continue;
-      c.offA[l * NT + t] = (long long)n; n += (size_t)rank * D.K_t[t];
-      c.offB[l * NT + t] = (long long)n; n += (size_t)D.N_t[t] * rank;
-    }
+  for (int pass = 0; pass < 2; ++pass) {
+    for (int l = 0; l < s->n_layers; ++l)
+      for (int t = 0; t < NT; ++t) {
+        if (!(target_mask >> t & 1)) continue;
+        if ((pass == 0) == D.a_rep[t]) { c.offA[l * NT + t] = (long long)n; n += (size_t)rank * D.K_t[t]; }
+        else { c.offB[l * NT + t] = (long long)n; n += (size_t)D.N_t[t] * rank; }
+      }
+    if (pass == 0) c.n_rep = n;
+  }
   c.n_params = n;
   if (cudaMalloc(&c.buf, 4 * n * sizeof(float)) != cudaSuccess) { cudaGetLastError(); FAIL(MENOS_ENOMEM, "adapter state"); }
   CUDA_TRY(cudaMemset(c.buf, 0, 4 * n * sizeof(float)));
   // init: A ~ U(-1/sqrt(K), 1/sqrt(K)) (PEFT kaiming-uniform a=sqrt(5)), B = 0
   std::vector<float> host(n, 0.f);
   uint64_t st = init_seed * 0x2545F4914F6CDD1Dull + 1;
+  // the draw is over the GLOBAL [r, K] of every (layer, target) in the same order on every tensor-parallel
+  // rank; a row-parallel rank keeps its column slice, so the shards assemble the world-1 A exactly
   for (int l = 0; l < s->n_layers; ++l)
     for (int t = 0; t < NT; ++t) {
       if (!(target_mask >> t & 1)) continue;
-      const double bound = 1.0 / std::sqrt((double)D.K_t[t]);
+      const int Kg = D.K_glob[t], Kl = D.K_t[t];
+      const int c0 = D.a_rep[t] ? 0 : D.tp_rank * Kl;
+      const double bound = 1.0 / std::sqrt((double)Kg);
       const long long o = c.offA[l * NT + t];
-      for (long long i = 0; i < (long long)rank * D.K_t[t]; ++i) {
-        const double u = (double)(splitmix(st) >> 11) * (1.0 / 9007199254740992.0);
-        host[o + i] = (float)((2.0 * u - 1.0) * bound);
-      }
+      for (int i = 0; i < rank; ++i)
+        for (int k = 0; k < Kg; ++k) {
+          const double u = (double)(splitmix(st) >> 11) * (1.0 / 9007199254740992.0);
+          if (k >= c0 && k < c0 + Kl) host[o + (long long)i * Kl + (k - c0)] = (float)((2.0 * u - 1.0) * bound);
+        }
     }
   CUDA_TRY(cudaMemcpy(c.buf, host.data(), n * sizeof(float), cudaMemcpyHostToDevice));
   c.used = true;
@@ -1124,6 +1155,15 @@ static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
   return lora_tokred_run(b->d_tprobs, b->d_ttiles + L.tiles_off, L.n_tiles, L.max_n, st);
 }
 
+// tensor-parallel all-reduce (sum, in place, stream-ordered) through the caller's callback (menos_tp_cfg)
+static int tp_allreduce(menos_server* s, void* buf, size_t count, int dtype, cudaStream_t st) {
+  if (s->tp.world <= 1 || count == 0) return MENOS_OK;
+  const int rc = s->tp.allreduce(buf, count, dtype, (void*)st, s->tp.user);
+  if (rc) FAIL(MENOS_ENCCL, "tensor-parallel all-reduce failed (%d) on rank %d", rc, s->tp.rank);
+  return MENOS_OK;
+}
+static inline bool tp_on(const menos_server* s) { return s->tp.world > 1; }
+
 static GemmArgs gemm_base(menos_server* s) {
   GemmArgs a;
   memset(&a, 0, sizeof a);
@@ -1180,7 +1220,10 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
       a.mtile_extra = b->d_mtile[GO];
     }
     a.epi = EPI_RESID; a.outf = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
+    if (D.tp_rank != 0) a.resid = nullptr;  // row-parallel: rank 0's partial carries the residual
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
+    int rc = tp_allreduce(s, S.h, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: o-proj partial sums
+    if (rc) return rc;
   }
   // A5: RMSNorm2
   { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st)); }
@@ -1212,7 +1255,10 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
       a.mtile_extra = b->d_mtile[GD];
     }
     a.epi = EPI_RESID; a.outf = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
+    if (D.tp_rank != 0) a.resid = nullptr;
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
+    int rc = tp_allreduce(s, y, (size_t)T * D.d, MENOS_DT_F32, st);      // A16: down-proj partial sums
+    if (rc) return rc;
   }
   return MENOS_OK;
 }
@@ -1250,10 +1296,17 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GGU];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
+    if (tp_on(s)) { a.epi = EPI_RESID; a.outf = sc.xout; a.resid = nullptr; }  // fp32 partial for the all-reduce
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
+    int rc = tp_allreduce(s, sc.xout, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: gate|up-dX partial sums
+    if (rc) return rc;
   }
   if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
-  { ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st)); }
+  {
+    ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
+    if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
+    else K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
+  }
   // A10: O dX (+ LoRA o) -> dO
   if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
   {
@@ -1294,10 +1347,17 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GQKV];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
+    if (tp_on(s)) { a.epi = EPI_RESID; a.outf = sc.xout; a.resid = nullptr; }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
+    int rc = tp_allreduce(s, sc.xout, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: qkv-dX partial sums
+    if (rc) return rc;
   }
   if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
-  { ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st); K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st)); }
+  {
+    ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
+    if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
+    else K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
+  }
   return MENOS_OK;
 }
 
@@ -1420,6 +1480,13 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
     std::swap(dyf, dxf);
     std::swap(dyb, dxb);
   }
+  // A16: the replicated adapters' gradients (dA of column-parallel, dB of row-parallel targets) are partial
+  // sums over the ranks' shards; one contiguous fp32 all-reduce per client
+  if (tp_on(s))
+    for (int c : b->bclients) {
+      rc = tp_allreduce(s, s->clients[c].G(), s->clients[c].n_rep, MENOS_DT_F32, st);
+      if (rc) return rc;
+    }
   CUDA_TRY(cudaMemcpyAsync(g_s, dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
   cudaPointerAttributes pa;
   if (cudaPointerGetAttributes(&pa, g_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&

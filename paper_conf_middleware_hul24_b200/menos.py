@@ -39,9 +39,16 @@ class AdamWCfg(C.Structure):
                 ("weight_decay", C.c_double)]
 
 
+from .tp import ALLREDUCE_FN, wrap_allreduce  # noqa: E402
+
+
+class TPCfg(C.Structure):
+    _fields_ = [("rank", C.c_int), ("world", C.c_int), ("allreduce", ALLREDUCE_FN), ("user", C.c_void_p)]
+
+
 class ServerOpts(C.Structure):
     _fields_ = [("max_clients", C.c_int), ("max_rank", C.c_int), ("max_seq_len", C.c_int),
-                ("arena_bytes", C.c_size_t), ("num_sms", C.c_int)]
+                ("arena_bytes", C.c_size_t), ("num_sms", C.c_int), ("tp", TPCfg)]
 
 
 class Stats(C.Structure):
@@ -152,10 +159,19 @@ class Server:
 
     def __init__(self, d_model, n_heads, n_kv_heads, d_ff, n_layers, first_layer=1, rms_eps=1e-5,
                  rope_theta=1e4, weights=None, device=0, max_clients=64, max_rank=64, max_seq_len=4096,
-                 arena_bytes=0, num_sms=0):
+                 arena_bytes=0, num_sms=0, tp=None):
+        """tp = (rank, world, allreduce) for tensor parallelism (include/menos.h menos_tp_cfg): `weights` are
+        then the rank's shards (tp.shard_layer_weights) and `allreduce(buf, count, dtype, stream)` is an in-place
+        sum over the ranks (tp.make_torch_allreduce)."""
         self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta)
         self.n_layers = n_layers
-        opts = ServerOpts(max_clients, max_rank, max_seq_len, arena_bytes, num_sms)
+        tpc = TPCfg(0, 1, ALLREDUCE_FN(), None)
+        self._tp_cb = None
+        if tp is not None and tp[1] > 1:
+            self._tp_cb = wrap_allreduce(tp[2])   # kept alive as long as the server
+            tpc = TPCfg(tp[0], tp[1], self._tp_cb, None)
+        self.tp_rank, self.tp_world = (tp[0], tp[1]) if tp is not None else (0, 1)
+        opts = ServerOpts(max_clients, max_rank, max_seq_len, arena_bytes, num_sms, tpc)
         h = C.c_void_p()
         warr = None
         if weights is not None:
