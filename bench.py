@@ -131,18 +131,28 @@ def run_reference(args):
 
 
 # ------------------------------------------------------------------------------------------------ GPU arm
-def build_server(torch, w, device, seed, arena_gb):
+def build_server(torch, w, device, seed, arena_gb, tp=None):
+    """One server (replica, or tensor-parallel shard when tp = (rank, world, allreduce)).  Weights are drawn on
+    the GPU directly in the shapes this server holds (a shard draws its own values: perf runs never compare
+    bytes)."""
     from paper_conf_middleware_hul24_b200 import Server
     m = w.model
+    if arena_gb is None or arena_gb <= 0:   # everything the base copy leaves, minus headroom
+        free = torch.cuda.mem_get_info(device)[0]
+        W = tp[1] if tp else 1
+        P = m.n_layers * (2 * m.d_model * (m.n_heads + m.n_kv_heads) * m.head_dim + 3 * m.d_model * m.d_ff) // W
+        arena_gb = max(4.0, (free - 2 * P - (6 << 30)) / (1 << 30))
     srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
                  rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=None, device=device.index,
                  max_rank=16, max_seq_len=max(max(c.seq_lens) for c in w.clients),
-                 arena_bytes=int(arena_gb * (1 << 30)))
+                 arena_bytes=int(arena_gb * (1 << 30)), tp=tp)
     gen = torch.Generator(device=device)
     hd = m.head_dim
-    shapes = {"wq": (m.n_heads * hd, m.d_model), "wk": (m.n_kv_heads * hd, m.d_model),
-              "wv": (m.n_kv_heads * hd, m.d_model), "wo": (m.d_model, m.n_heads * hd),
-              "wgate": (m.d_ff, m.d_model), "wup": (m.d_ff, m.d_model), "wdown": (m.d_model, m.d_ff)}
+    W = tp[1] if tp else 1
+    Hl, Hkvl, fl = m.n_heads // W, m.n_kv_heads // W, m.d_ff // W
+    shapes = {"wq": (Hl * hd, m.d_model), "wk": (Hkvl * hd, m.d_model),
+              "wv": (Hkvl * hd, m.d_model), "wo": (m.d_model, Hl * hd),
+              "wgate": (fl, m.d_model), "wup": (fl, m.d_model), "wdown": (m.d_model, fl)}
     out_std = 0.02 / (2.0 * m.total_layers) ** 0.5   # same recipe as workloads.base_layer_weights (R17)
     for l in range(m.n_layers):
         gen.manual_seed(seed * 1000 + l)
@@ -189,14 +199,27 @@ def run_gpu(args):
     if os.environ.get("MENOS_ATTN_TC") is not None:   # kernel-variant switch for A/B measurements
         M.lib().menos_test_set_attn_tc(int(os.environ["MENOS_ATTN_TC"]))
     w = workload(args.workload, n_layers=args.layers)
-    # cfg2 (32 ragged clients): LPT partition over the ranks (strong scaling); otherwise every rank serves the
-    # workload's own client set on its replica (weak scaling)
-    strong = args.workload == "cfg2_7b_x32_ragged"
-    if strong:
+    # cfg2 / cfg3 (32 ragged 7B clients / 16 13B clients): LPT partition over the replica ranks (strong scaling);
+    # cfg4 (70B): tensor-parallel over the ranks, every rank sees all clients' tokens (strong scaling);
+    # otherwise every rank serves the workload's own client set on its replica (weak scaling)
+    tp_mode = args.workload.startswith("cfg4") or args.tp_shard_only > 1
+    strong = args.workload in ("cfg2_7b_x32_ragged", "cfg3_13b_x16") or tp_mode
+    tp = None
+    if tp_mode:
+        from paper_conf_middleware_hul24_b200 import tp as TPM
+        if args.tp_shard_only > 1:
+            # single-GPU compute-only timing of rank 0's shard of a W-way split: the all-reduce is a no-op, so
+            # this is NOT a bench value (no communication); it measures the per-GPU kernels of the TP path
+            if world != 1:
+                raise SystemExit("--tp-shard-only runs on one GPU")
+            tp = (0, args.tp_shard_only, lambda buf, n, dt, st: 0)
+        else:
+            tp = (rank, world, TPM.make_torch_allreduce(device=local)) if world > 1 else None
+    elif strong:
         w.clients = [w.clients[i] for i in workload_partition(w, world)[rank]]
     T = w.n_tokens
     d = w.model.d_model
-    srv = build_server(torch, w, device, seed=rank, arena_gb=args.arena_gb)
+    srv = build_server(torch, w, device, seed=rank, arena_gb=args.arena_gb, tp=tp)
     ids = register_clients(np, srv, w, seed=rank + 1)
     # waves: temporal sharing of the arena when the clients' saved activations do not fit at once
     mem = [srv.client_memory(ids[i], c.n_tokens) for i, c in enumerate(w.clients)]
@@ -219,7 +242,7 @@ def run_gpu(args):
     x_s, g_s = torch.empty_like(x_c), torch.empty_like(x_c)
     stream = torch.cuda.current_stream(device)
     T_all = T
-    if world > 1:
+    if world > 1 and not tp_mode:
         tt = torch.tensor([float(T)], device=device)
         dist.all_reduce(tt)
         T_all = int(tt.item())
@@ -331,7 +354,12 @@ def run_gpu(args):
             K_, N_ = target_dims(m, t)
             lora += 6 * c.rank * (K_ + N_) * c.n_tokens * m.n_layers
     step_flops = 4 * P * T + attn + lora
-    step_tflops = step_flops * (T_all / T) * args.steps / (ms / 1000.0) / 1e12
+    if tp_mode:   # every rank computes 1/W of the (replicated-token) step; the job does the whole step once
+        job_flops = step_flops / (args.tp_shard_only if args.tp_shard_only > 1 else 1)
+    else:
+        job_flops = step_flops * (T_all / T)
+    step_tflops = job_flops * args.steps / (ms / 1000.0) / 1e12
+    n_dev = world
 
     # HBM bytes per client (persistent A+O and the SAVE-forward arena share), Eq.3 accounting
     st = srv.stats()
@@ -356,11 +384,16 @@ def run_gpu(args):
                        "waves_per_step": len(waves), "server_layers": w.model.n_layers,
                        "lora": sorted({f"r{c.rank} {'+'.join(c.targets)}" for c in w.clients}),
                        "seq_lens": sorted({s for c in w.clients for s in c.seq_lens}),
-                       "parallelism": f"replica x{world} (clients partitioned, no collective)",
-                       "l2": "inputs larger than L2: 12.55 GB bf16 weights + ~28 GB saved activations streamed "
-                             "per step vs 126 MB L2"},
+                       "parallelism": (f"tensor-parallel x{world} (NCCL all-reduce per attention/MLP block)"
+                                       if tp_mode and args.tp_shard_only <= 1 else
+                                       f"rank-0 shard of TP-{args.tp_shard_only}, all-reduce elided: compute "
+                                       f"only, NOT a bench value" if tp_mode else
+                                       f"replica x{world} (clients partitioned, no collective)"),
+                       "l2": f"inputs larger than L2: {srv.stats()['base_bytes'] / 1e9:.2f} GB bf16 weights + "
+                             f"{sum(m_[1] for m_ in mem) / 1e9:.1f} GB saved activations "
+                             f"streamed per step vs 126 MB L2"},
             "roofline": roofline, "step_tflops": step_tflops,
-            "step_frac_of_peak": step_tflops / peak if peak else None,
+            "step_frac_of_peak": step_tflops / (peak * n_dev) if peak else None,
             "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
@@ -383,7 +416,10 @@ def main():
     ap.add_argument("--impl", default="menos", choices=["menos", "reference"])
     ap.add_argument("--workload", default="cfg1_7b_x4")
     ap.add_argument("--layers", type=int, default=None, help="truncate depth (debug only; not a bench value)")
-    ap.add_argument("--arena-gb", type=float, default=80.0)
+    ap.add_argument("--arena-gb", type=float, default=0.0, help="activation arena; 0 = all memory the base leaves")
+    ap.add_argument("--tp-shard-only", type=int, default=0,
+                    help="time rank 0's shard of a W-way tensor-parallel split on 1 GPU (no all-reduce; not a "
+                         "bench value)")
     ap.add_argument("--cpu-layers", type=int, default=6)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")

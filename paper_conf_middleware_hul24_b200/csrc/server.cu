@@ -297,6 +297,10 @@ struct menos_server {
   struct Slot { uint8_t* buf = nullptr; size_t bytes = 0; cudaEvent_t ev = nullptr; };
   Slot ring[kRing];
   int ring_next = 0;
+  // device copies of the AdamW tables (hyper-params, segments, work list): a ring reused once the kernel that
+  // last read an entry has completed (its event), so adapter_step never allocates on the hot path
+  Slot dring[kRing];
+  int dring_next = 0;
 };
 
 // =====================================================================================================
@@ -443,8 +447,18 @@ static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, c
   if (work.empty()) return MENOS_OK;
   const size_t b1 = hyp.size() * sizeof(AdamHyper), b2 = segs.size() * sizeof(AdamSeg), b3 = work.size() * sizeof(int4);
   const size_t o2 = align_up(b1, 256), o3 = o2 + align_up(b2, 256), tot = o3 + b3;
-  uint8_t* dbuf = nullptr;
-  CUDA_TRY(cudaMallocAsync((void**)&dbuf, tot, st));
+  auto& ds = s->dring[s->dring_next];
+  s->dring_next = (s->dring_next + 1) % menos_server::kRing;
+  if (ds.ev) CUDA_TRY(cudaEventSynchronize(ds.ev));
+  else CUDA_TRY(cudaEventCreateWithFlags(&ds.ev, cudaEventDisableTiming));
+  if (tot > ds.bytes) {
+    if (ds.buf) CUDA_TRY(cudaFree(ds.buf));
+    ds.buf = nullptr;
+    const size_t nb = std::max(align_up(tot * 5 / 4, 1 << 16), (size_t)1 << 20);
+    if (cudaMalloc(&ds.buf, nb) != cudaSuccess) { cudaGetLastError(); ds.bytes = 0; FAIL(MENOS_ENOMEM, "adamw tables"); }
+    ds.bytes = nb;
+  }
+  uint8_t* dbuf = ds.buf;
   std::vector<uint8_t> blob(tot);
   memcpy(blob.data(), hyp.data(), b1);
   memcpy(blob.data() + o2, segs.data(), b2);
@@ -457,7 +471,7 @@ static int run_adam(menos_server* s, const std::vector<int>& ids, bool update, c
     ProfScope ps(PC_ADAMW, 0, nparam * (update ? 30.0 : 6.0), st);
     K_TRY(adamw_run((AdamSeg*)(dbuf + o2), (int4*)(dbuf + o3), (int)work.size(), (AdamHyper*)dbuf, st));
   }
-  CUDA_TRY(cudaFreeAsync(dbuf, st));
+  CUDA_TRY(cudaEventRecord(ds.ev, st));
   return MENOS_OK;
 }
 
@@ -561,6 +575,10 @@ extern "C" void menos_server_destroy(menos_server* s) {
   if (s->arena_mem) cudaFree(s->arena_mem);
   for (auto& sl : s->ring) {
     if (sl.buf) cudaFreeHost(sl.buf);
+    if (sl.ev) cudaEventDestroy(sl.ev);
+  }
+  for (auto& sl : s->dring) {
+    if (sl.buf) cudaFree(sl.buf);
     if (sl.ev) cudaEventDestroy(sl.ev);
   }
   delete s;

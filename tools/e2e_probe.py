@@ -92,7 +92,7 @@ def main():
     t3 = time.perf_counter()
     print(f"host-buffer wall: fwd {(t1-t0)*1e3:.1f} ms, bwd {(t2-t1)*1e3:.1f} ms, step+sync {(t3-t2)*1e3:.1f} ms")
     # per-call device segments over 4 host-buffer steps
-    for it in range(4):
+    for it in range(int(os.environ.get('NSTEPS', '4'))):
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
         w0 = time.perf_counter()
         ev[0].record(st)
