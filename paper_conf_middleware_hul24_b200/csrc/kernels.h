@@ -103,7 +103,12 @@ struct AttnArgs {
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block
 int attn_fwd_tc(const AttnArgs& a, const int2* qblocks128, int n_qblocks128, cudaStream_t st);
-extern int g_attn_tc;  // head_dim 128 variant bitmask: 1 = tcgen05 forward, 2 = tcgen05 backward
+// persistent warp-specialized tcgen05 forward for head_dim 128 (attention_fwd_ws.cu); items = (seq, q0, head, -)
+int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st);
+void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out);
+// head_dim 128 variant bitmask: 1 = tcgen05 forward (2-pass), 2 = tcgen05 backward, 4 = persistent
+// warp-specialized tcgen05 forward (takes precedence over 1)
+extern int g_attn_tc;
 int attn_bwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 backward for head_dim 128 (attention_bwd_tc.cu); blocks128 = (seq, local start) per 128-row block
 int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaStream_t st);

@@ -252,6 +252,7 @@ struct menos_batch {
   bool save_a = false;
   int n_mt = 0, n_blocks = 0, n_blocks128 = 0;
   int2* d_blocks128 = nullptr;
+  int4* d_attn_items = nullptr; int n_attn_items = 0;   // persistent attention forward work list
   double pairs = 0;   // causal (query, key) pairs summed over sequences
   // device metadata
   uint8_t* meta = nullptr;  // arena
@@ -946,6 +947,9 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   for (int i = 0; i < b->n_seqs; ++i)
     for (int q = 0; q < b->seq_len[i]; q += 128) blocks128.push_back(make_int2(i, q));
   b->n_blocks128 = (int)blocks128.size();
+  std::vector<int4> attn_items;
+  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items);
+  b->n_attn_items = (int)attn_items.size();
   std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
   for (int g = 0; g < NG; ++g) {
     if (!b->g_active[g]) continue;
@@ -975,6 +979,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_pos = put(b->pos.data(), b->pos.size() * 4);
   const size_t o_blk = put(blocks.data(), blocks.size() * sizeof(int2));
   const size_t o_blk128 = put(blocks128.data(), blocks128.size() * sizeof(int2));
+  const size_t o_items = put(attn_items.data(), attn_items.size() * sizeof(int4));
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
 
@@ -1101,6 +1106,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   if (rc) return rc;
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
   b->d_blocks128 = (int2*)(meta + o_blk128);
+  b->d_attn_items = (int4*)(meta + o_items);
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
   b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
@@ -1222,7 +1228,8 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st);
-    if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+    if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, b->d_attn_items, b->n_attn_items, s->num_sms, st));
+    else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
     else K_TRY(attn_fwd(a, st));
   }
   // A4: O GEMM (+ LoRA o) + residual

@@ -94,14 +94,24 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
   cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
   const bool tc_fwd = hd == 128 && (g_attn_tc & 1), tc_bwd = hd == 128 && (g_attn_tc & 2);
-  rc = tc_fwd ? attn_fwd_tc(a, d_b128, (int)b128.size(), 0) : attn_fwd(a, 0);
+  const bool ws_fwd = hd == 128 && (g_attn_tc & 4);
+  std::vector<int4> items;
+  attn_ws_items(seq_len, n_seqs, H, items);
+  int4* d_items;
+  cudaMalloc(&d_items, std::max<size_t>(1, items.size()) * sizeof(int4));
+  cudaMemcpy(d_items, items.data(), items.size() * sizeof(int4), cudaMemcpyHostToDevice);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  rc = ws_fwd ? attn_fwd_ws(a, d_items, (int)items.size(), sms, 0)
+              : tc_fwd ? attn_fwd_tc(a, d_b128, (int)b128.size(), 0) : attn_fwd(a, 0);
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
     rc = tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
   }
   cudaError_t e = cudaDeviceSynchronize();
-  cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D); cudaFree(d_b128);
+  cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D); cudaFree(d_b128); cudaFree(d_items);
   if (rc != 0) return fail("attention launch rejected");
   if (e != cudaSuccess) return fail(cudaGetErrorString(e));
   return MENOS_OK;
@@ -194,12 +204,12 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
   return MENOS_OK;
 }
 
-// Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward, 2 = tcgen05 backward (dK/dV + dQ kernels).
-// The tcgen05 forward's serialized single-control-thread pipeline is still slower than the mma.sync kernel on the
-// 512-token workloads, so only the backward is on by default.
-namespace menos { int g_attn_tc = 2; }
+// Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward (2-pass, serialized), 2 = tcgen05 backward
+// (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1).
+// Default 6: the persistent tcgen05 forward (2.1x the mma.sync kernel at S = 512) and the tcgen05 backward.
+namespace menos { int g_attn_tc = 6; }
 extern "C" int menos_test_set_attn_tc(int mode) {
-  if (mode < 0 || mode > 3) { fail("attention mode must be in [0, 3]"); return MENOS_EINVAL; }
+  if (mode < 0 || mode > 7) { fail("attention mode must be in [0, 7]"); return MENOS_EINVAL; }
   menos::g_attn_tc = mode;
   return MENOS_OK;
 }
