@@ -129,15 +129,22 @@ __global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* _
 
 // ============================================================================ token-reduction kernel
 // C[m, n] = scale * sum_t P[t, map(m)] * Q[t, n]  over t in [0, T); tile (MT x NT) at (m0, n0)
+// 4-stage cp.async ring of 64-token stages (~54 KB of P / Q in flight per CTA): the reduction streams one client's
+// activations once, so bytes in flight, not math, set its speed
+constexpr int TR_BK = 64, TR_STAGES = 4;
+template <int MT, int NT>
+constexpr int tokred_smem_bytes() { return TR_STAGES * TR_BK * (MT + NT) * 2; }
+
 template <int MT, int NT>
 __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProblem* __restrict__ probs,
                                                           const int4* __restrict__ tiles) {
-  constexpr int BK = 32;                       // tokens per stage
+  constexpr int BK = TR_BK, NS = TR_STAGES;    // tokens per stage, stages
   constexpr int WM = MT >= 64 ? MT / 4 : MT;   // rows per warp (4 warps split M when MT is large)
   constexpr int WN = MT >= 64 ? NT : NT / 4;   // cols per warp (else split N)
   constexpr int NMI = WM / 16, NNJ = WN / 8;
-  __shared__ __align__(128) bf16 Ps[2][BK * MT];   // [token][m]
-  __shared__ __align__(128) bf16 Qs[2][BK * NT];   // [token][n]
+  extern __shared__ __align__(128) uint8_t tr_smem[];
+  bf16* Ps_base = reinterpret_cast<bf16*>(tr_smem);   // [NS][BK * MT]  ([token][m])
+  bf16* Qs_base = Ps_base + NS * BK * MT;             // [NS][BK * NT]  ([token][n])
   const int4 tl = tiles[blockIdx.x];
   const LoraTokRedProblem P = probs[tl.x];
   const int m0 = tl.y, n0 = tl.z;
@@ -147,17 +154,19 @@ __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProble
   const int pcol0 = (m0 / P.p_blk) * P.p_blk_stride + m0 % P.p_blk;
 
   auto load = [&](int buf, int t0) {
+    bf16* Ps = Ps_base + buf * BK * MT;
+    bf16* Qs = Qs_base + buf * BK * NT;
     for (int i = tid; i < BK * (MT / 8); i += 128) {
       const int r = i / (MT / 8), c = i % (MT / 8);
       const int tok = t0 + r;
       const bool ok = tok < P.T && m0 + c * 8 < P.M;
-      cp_async16(smem_u32(&Ps[buf][tsw<MT>(r, c)]), P.P + (ok ? (size_t)tok * P.ldp + pcol0 + c * 8 : 0), ok ? 16 : 0);
+      cp_async16(smem_u32(&Ps[tsw<MT>(r, c)]), P.P + (ok ? (size_t)tok * P.ldp + pcol0 + c * 8 : 0), ok ? 16 : 0);
     }
     for (int i = tid; i < BK * (NT / 8); i += 128) {
       const int r = i / (NT / 8), c = i % (NT / 8);
       const int tok = t0 + r;
       const bool ok = tok < P.T && n0 + c * 8 < P.N;
-      cp_async16(smem_u32(&Qs[buf][tsw<NT>(r, c)]), P.Q + (ok ? (size_t)tok * P.ldq + n0 + c * 8 : 0), ok ? 16 : 0);
+      cp_async16(smem_u32(&Qs[tsw<NT>(r, c)]), P.Q + (ok ? (size_t)tok * P.ldq + n0 + c * 8 : 0), ok ? 16 : 0);
     }
   };
 
@@ -167,14 +176,21 @@ __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProble
 #pragma unroll
     for (int j = 0; j < NNJ; ++j) acc[i][j][0] = acc[i][j][1] = acc[i][j][2] = acc[i][j][3] = 0.f;
   const int nk = (P.T + BK - 1) / BK;
-  load(0, 0);
-  cp_async_commit();
+#pragma unroll
+  for (int s = 0; s < NS - 1; ++s) {
+    if (s < nk) load(s, s * BK);
+    cp_async_commit();
+  }
   for (int kb = 0; kb < nk; ++kb) {
-    if (kb + 1 < nk) { load((kb + 1) & 1, (kb + 1) * BK); cp_async_commit(); cp_async_wait<1>(); }
-    else cp_async_wait<0>();
+    cp_async_wait<NS - 2>();
     __syncthreads();
-    const bf16* p_s = Ps[kb & 1];
-    const bf16* q_s = Qs[kb & 1];
+    {
+      const int nx = kb + NS - 1;
+      if (nx < nk) load(nx % NS, nx * BK);
+      cp_async_commit();
+    }
+    const bf16* p_s = Ps_base + (kb % NS) * BK * MT;
+    const bf16* q_s = Qs_base + (kb % NS) * BK * NT;
 #pragma unroll
     for (int kk = 0; kk < BK; kk += 16) {
       const int mat = lane >> 3, r = lane & 7;
@@ -197,8 +213,8 @@ __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProble
         }
       }
     }
-    __syncthreads();
   }
+  cp_async_wait<0>();
 #pragma unroll
   for (int i = 0; i < NMI; ++i)
 #pragma unroll
@@ -244,8 +260,16 @@ int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_til
 
 int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st) {
   if (n_tiles <= 0) return 0;
-  if (mt == 128) lora_tokred_kernel<128, 16><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
-  else if (mt == 16) lora_tokred_kernel<16, 128><<<n_tiles, 128, 0, st>>>(d_probs, d_tiles);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_tokred_kernel<128, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         tokred_smem_bytes<128, 16>());
+    cudaFuncSetAttribute(lora_tokred_kernel<16, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         tokred_smem_bytes<16, 128>());
+    attr = true;
+  }
+  if (mt == 128) lora_tokred_kernel<128, 16><<<n_tiles, 128, tokred_smem_bytes<128, 16>(), st>>>(d_probs, d_tiles);
+  else if (mt == 16) lora_tokred_kernel<16, 128><<<n_tiles, 128, tokred_smem_bytes<16, 128>(), st>>>(d_probs, d_tiles);
   else return -1;
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;

@@ -1061,6 +1061,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           p.C = U + (size_t)t0 * R + col; p.ldc = R;
           p.M = Tc; p.N = w; p.K = D.K_g[g]; p.scale = c.s;
           f.push_back(p);
+          if (g == GQKV) continue;   // q / k / v: per-target dU problems below
           // dU[t, col..col+w) = s * dY_c Bcat[:, col..]   (other targets' rows of Bcat are zero in these columns)
           LoraRowsProblem q{};
           q.A = dY + (size_t)t0 * ldy; q.lda = ldy;
@@ -1068,6 +1069,20 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           q.C = sc.dU[g] + (size_t)t0 * R + col; q.ldc = R;
           q.M = Tc; q.N = w; q.K = D.N_g[g]; q.scale = c.s;
           du.push_back(q);
+        }
+        if (g == GQKV) {
+          // q, k, v own contiguous row ranges of Bcat (and columns of dY): reduce each target over its own N_t
+          // columns only -- the other targets' columns multiply zero rows -- which also doubles the tile count
+          for (int t = TQ; t <= TV; ++t) {
+            if (!(c.mask >> t & 1)) continue;
+            LoraRowsProblem q{};
+            q.A = dY + (size_t)t0 * ldy + D.rb_base[t]; q.lda = ldy;
+            q.B = s->Bcat[g][l] + (size_t)D.rb_base[t] * s->cols[g].cap + c.col_off[g] + c.sub[t];
+            q.ldb = s->cols[g].cap; q.b_kn = 1;
+            q.C = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.ldc = R;
+            q.M = Tc; q.N = c.rs; q.K = D.N_t[t]; q.scale = c.s;
+            du.push_back(q);
+          }
         }
         // per target: dB = dY_t^T (s U_t), dA = dU_t^T X   (fp32, overwrite; reduced over this client only)
         for (int t = 0; t < NT; ++t) {
