@@ -64,7 +64,8 @@ MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A,
 
 /* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
    bit 1 = tcgen05 backward (else mma.sync), bit 2 = persistent warp-specialized tcgen05 forward (overrides
-   bit 0). Returns MENOS_EINVAL outside [0, 7]. */
+   bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1). Returns MENOS_EINVAL outside
+   [0, 15]. */
 MENOS_API int menos_test_set_attn_tc(int mode);
 
 MENOS_API const char* menos_testing_last_error(void);

@@ -97,20 +97,6 @@ __device__ __forceinline__ void bw_wait_idle(uint64_t* bar, uint32_t parity) {
   }
 }
 
-// 32 lanes x 32 fp32 columns without the trailing wait (batch several, then tmem_wait_ld)
-__device__ __forceinline__ void tmem_ld32_nw(uint32_t taddr, uint32_t (&r)[32]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
-      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-      : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-
 // write columns [32 g, 32 g + 32) (bf16) of one row of a [rows][64] SWIZZLE_128B K-major tile
 __device__ __forceinline__ void st_half_row_sw128(uint8_t* tile, int row, int g, const float (&v)[32]) {
   uint8_t* prow = tile + row * 128;
@@ -188,7 +174,7 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   uint8_t* const sS0 = sP0 + 2 * PT_TILE;             // dS^T (2 buffers)
   __shared__ __align__(8) uint64_t bar_kv, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2], acc_done;
   __shared__ uint32_t tmem_sh;
-  __shared__ float s_lse[2][QB], s_D[2][QB];
+  __shared__ __align__(16) float s_lse[2][QB], s_D[2][QB];
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int2 kb = p.blocks[blockIdx.x];
@@ -318,11 +304,19 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       const int cmax = L - q0 - 32 * g;      // ... and past the end of the sequence
       float pv[32], dsv[32];
 #pragma unroll
-      for (int c = 0; c < 32; ++c) {
-        const bool ok = c >= cmin && c < cmax;
-        const float e = exp2f(__uint_as_float(su[c]) * sl2 - s_lse[b][32 * g + c]);
-        pv[c] = ok ? e : 0.f;
-        dsv[c] = ok ? e * (__uint_as_float(du[c]) - s_D[b][32 * g + c]) * p.scale : 0.f;
+      for (int c4 = 0; c4 < 32; c4 += 4) {
+        const float4 lz = *reinterpret_cast<const float4*>(&s_lse[b][32 * g + c4]);
+        const float4 dz = *reinterpret_cast<const float4*>(&s_D[b][32 * g + c4]);
+        const float lzv[4] = {lz.x, lz.y, lz.z, lz.w}, dzv[4] = {dz.x, dz.y, dz.z, dz.w};
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int c = c4 + u;
+          const bool ok = c >= cmin && c < cmax;
+          const float x = fmaf(__uint_as_float(su[c]), sl2, -lzv[u]);
+          const float e = u == 3 ? poly_exp2(x) : fast_exp2(x);   // a quarter on the FMA pipe (SFU-bound loop)
+          pv[c] = ok ? e : 0.f;
+          dsv[c] = ok ? e * (__uint_as_float(du[c]) - dzv[u]) * p.scale : 0.f;
+        }
       }
       if (it >= 2) bw_wait(&pd_free[b], ((it - 2) >> 1) & 1);
       st_half_row_sw128(sP0 + b * PT_TILE, r, g, pv);
@@ -487,7 +481,9 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       float dsv[32];
 #pragma unroll
       for (int c = 0; c < 32; ++c) {
-        const float v = exp2f(__uint_as_float(su[c]) * sl2 - lse2) * (__uint_as_float(du[c]) - Dq) * p.scale;
+        const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+        const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);   // a quarter on the FMA pipe
+        const float v = e * (__uint_as_float(du[c]) - Dq) * p.scale;
         dsv[c] = c <= cmax ? v : 0.f;
       }
       if (it >= 2) bw_wait(&pd_free[b], ((it - 2) >> 1) & 1);

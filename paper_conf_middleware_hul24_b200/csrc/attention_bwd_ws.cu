@@ -1,0 +1,609 @@
+// Varlen causal flash-attention BACKWARD, persistent warp-specialized tcgen05 kernels, head_dim 128.
+// SURVEY.md §8(a) A11.  Same contract and math as attention_bwd_tc.cu (deterministic: no atomics; blocks never
+// cross a sequence, so never a client; GQA; RoPE backward applied to dq / dk before the store),
+// restructured so that the per-block fill / drain of the non-persistent kernels overlaps with useful work:
+//   * one CTA per SM loops over work items (dK/dV: (sequence, kv head, 128-key block); dQ: (sequence, head,
+//     128-query block)); the TMA producer loads the next item's resident operand (K|V, resp. Q|dO) as soon as the
+//     current item's last S / dP MMA has consumed it, and the streamed operand ring runs across item boundaries;
+//   * the MMA warp starts the next item's S / dP MMAs while the elementwise warps run the previous epilogue; only
+//     the first accumulation into dK|dV (resp. dQ) waits for the epilogue to have read the TMEM accumulators;
+//   * epilogue: each thread reads the accumulator columns j and j+64 of its row, applies the RoPE backward in
+//     registers, stages bf16 rows (swizzled) in the freed P/dS buffers and the warps write them row-contiguously.
+// Elementwise work: P = exp2(S c - lse) (a quarter on the FMA pipe), dS = P (dP - D) scale, bf16 packed into
+// 128B-swizzled K-major tiles for the accumulation MMAs.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace menos {
+
+bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
+                uint32_t br);
+
+namespace {
+
+constexpr int HD = 128, STAGES = 3, EW_WARPS = 8, NTHREADS = 64 + 32 * EW_WARPS;
+constexpr float LOG2E_W = 1.4426950408889634f;
+
+struct BwParams {
+  const int* cu_seqlens;
+  const int4* items;       // (seq, block start, head (dQ) / kv head (dK/dV), -)
+  int n_items;
+  const float* lse;        // [H, T] natural log
+  const float* D;          // [H, T]
+  bf16* dqkv; int ld_dqkv;
+  const float2* rope_cs;   // [max_pos][HD/2] (cos, sin)
+  int T, H, Hkv;
+  float scale;
+};
+
+__device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.b32 %0, 1, 0, P;\n\t}"
+                 : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  }
+}
+__device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
+
+// columns [32 g, 32 g + 32) (bf16) of one row of a [rows][64] SWIZZLE_128B K-major tile
+__device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const float (&v)[32]) {
+  uint8_t* prow = tile + row * 128;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const int c8 = 4 * g + c;
+    uint4 u = make_uint4(pack_bf16x2(v[8 * c + 0], v[8 * c + 1]), pack_bf16x2(v[8 * c + 2], v[8 * c + 3]),
+                         pack_bf16x2(v[8 * c + 4], v[8 * c + 5]), pack_bf16x2(v[8 * c + 6], v[8 * c + 7]));
+    *reinterpret_cast<uint4*>(prow + ((c8 ^ (row & 7)) << 4)) = u;
+  }
+}
+
+// Epilogue, fp32 staging of 64 accumulator rows (one TMEM lane-quadrant pair) in 32 KB: 16-byte chunk k (0..31) of
+// staged row rr at rr * 512 + ((k ^ (rr & 7)) << 4) (conflict-free for the row-per-lane writes)
+__device__ __forceinline__ float* stg32_at(uint8_t* stg, int rr, int k) {
+  return reinterpret_cast<float*>(stg + rr * 512 + ((k ^ (rr & 7)) << 4));
+}
+// this thread's TMEM row (staged row rr), columns [32g, 32g+32) and [64+32g, 64+32g+32)
+__device__ __forceinline__ void acc_row_to_stage32(uint32_t tacc, uint8_t* stg, int rr, int g) {
+  uint32_t a[32], b[32];
+  tmem_ld32_nw(tacc + 32 * g, a);
+  tmem_ld32_nw(tacc + 64 + 32 * g, b);
+  tmem_wait_ld();
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    *reinterpret_cast<uint4*>(stg32_at(stg, rr, 8 * g + c)) = make_uint4(a[4 * c], a[4 * c + 1], a[4 * c + 2], a[4 * c + 3]);
+    *reinterpret_cast<uint4*>(stg32_at(stg, rr, 16 + 8 * g + c)) = make_uint4(b[4 * c], b[4 * c + 1], b[4 * c + 2], b[4 * c + 3]);
+  }
+}
+// all elementwise warps: staged rows -> bf16 rows of dst (rows row0 + rr < n_valid), lanes across columns (the RoPE
+// table reads and the row stores are coalesced); with rope the RoPE backward at position pos0 + row0 + rr:
+// dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
+__device__ __forceinline__ void stage32_to_global(uint8_t* stg, int w8, int lane, int row0, int n_valid, bf16* dst,
+                                                  int ld, const float2* cs, int pos0, bool rope) {
+  const int jl = lane & 15, j = 4 * jl;
+#pragma unroll 2
+  for (int r2 = 0; r2 < 8; r2 += 2) {
+    const int rr = w8 * 8 + r2 + (lane >> 4), row = row0 + rr;
+    if (row >= n_valid) continue;
+    const float4 a = *reinterpret_cast<const float4*>(stg32_at(stg, rr, jl));
+    const float4 b = *reinterpret_cast<const float4*>(stg32_at(stg, rr, 16 + jl));
+    float x[4] = {a.x, a.y, a.z, a.w}, y[4] = {b.x, b.y, b.z, b.w};
+    if (rope) {
+      const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)(pos0 + row) * (HD / 2) + j);
+      const float4 e0 = c4[0], e1 = c4[1];   // (c_j, s_j, c_j+1, s_j+1), (c_j+2, s_j+2, c_j+3, s_j+3)
+      const float cc[4] = {e0.x, e0.z, e1.x, e1.z}, ss[4] = {e0.y, e0.w, e1.y, e1.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float xi = x[i] * cc[i] + y[i] * ss[i], yi = y[i] * cc[i] - x[i] * ss[i];
+        x[i] = xi; y[i] = yi;
+      }
+    }
+    bf16* d = dst + (size_t)row * ld;
+    *reinterpret_cast<uint2*>(d + j) = make_uint2(pack_bf16x2(x[0], x[1]), pack_bf16x2(x[2], x[3]));
+    *reinterpret_cast<uint2*>(d + 64 + j) = make_uint2(pack_bf16x2(y[0], y[1]), pack_bf16x2(y[2], y[3]));
+  }
+}
+// one 128-row accumulator through the 32 KB staging area in two 64-row rounds (TMEM lane quadrants 0-1, then
+// 2-3); with arrive, each warp arrives on acc_free right after its TMEM rows have been read
+__device__ __forceinline__ void acc_epilogue(uint32_t tacc_lane, uint8_t* stg, int w4, int w8, int lane, int g,
+                                             int n_valid, bf16* dst, int ld, const float2* cs, int pos0, bool rope,
+                                             uint64_t* acc_free_bar, bool arrive) {
+#pragma unroll 1
+  for (int half = 0; half < 2; ++half) {
+    if ((w4 >> 1) == half) {
+      acc_row_to_stage32(tacc_lane, stg, (w4 & 1) * 32 + lane, g);
+      if (arrive) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(acc_free_bar);
+      }
+    }
+    ew_sync();
+    stage32_to_global(stg, w8, lane, half * 64, n_valid, dst, ld, cs, pos0, rope);
+    ew_sync();
+  }
+}
+
+struct Geo { int base, L, blk0, head, n; };
+
+// -DMENOS_BWS_PROF: per-phase clock64 accounting (dK/dV kernel: one elementwise thread and the MMA lane)
+#ifdef MENOS_BWS_PROF
+__device__ unsigned long long g_bws_prof[16];
+#define BP_DECL long long bp_t = clock64(); unsigned long long bpr_[16] = {0};
+#define BP(k) do { const long long t_ = clock64(); bpr_[k] += t_ - bp_t; bp_t = t_; } while (0)
+#define BP_FLUSH(cond) do { if (cond) for (int k_ = 0; k_ < 16; ++k_) if (bpr_[k_]) atomicAdd(&g_bws_prof[k_], bpr_[k_]); } while (0)
+#else
+#define BP_DECL
+#define BP(k) do {} while (0)
+#define BP_FLUSH(cond) do {} while (0)
+#endif
+
+// ======================================================================================= dK / dV
+constexpr int KV_ROWS = 128, QB = 64;
+constexpr int KV_TILE = KV_ROWS * HD * 2;      // 32 KB (2 atoms [128][64])
+constexpr int QB_TILE = QB * HD * 2;           // 16 KB (2 atoms [64][64])
+constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
+constexpr int SMEM_DKDV = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;
+
+__global__ void __launch_bounds__(NTHREADS, 1)
+attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
+                        const __grid_constant__ CUtensorMap tmDO64, const BwParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* const sK = smem;
+  uint8_t* const sV = sK + KV_TILE;
+  uint8_t* const sQ0 = sV + KV_TILE;                  // Q stages
+  uint8_t* const sO0 = sQ0 + STAGES * QB_TILE;        // dO stages
+  uint8_t* const sP0 = sO0 + STAGES * QB_TILE;        // P^T  (2 buffers) -- dK staging in the epilogue
+  uint8_t* const sS0 = sP0 + 2 * PT_TILE;             // dS^T (2 buffers) -- dV staging in the epilogue
+  __shared__ __align__(8) uint64_t kv_full, kv_empty, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2];
+  __shared__ __align__(8) uint64_t acc_full, acc_free;
+  __shared__ uint32_t tmem_sh;
+  __shared__ __align__(16) float s_lse[2][QB], s_D[2][QB];
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int rep = p.H / p.Hkv;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO64);
+    mbar_init(&kv_full, 1); mbar_init(&kv_empty, 1);
+    for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
+    mbar_init(&acc_full, 1); mbar_init(&acc_free, EW_WARPS);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;
+  const uint32_t tdV = tmem + 256, tdK = tmem + 384;   // S^T buffers at 0/64, dP^T at 128/192
+
+  auto load_geo = [&](int item) {
+    Geo g{0, 0, 0, 0, 0};
+    if (item < p.n_items) {
+      const int4 it = p.items[item];
+      g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
+      g.n = rep * ((g.L - g.blk0 + QB - 1) / QB);      // (head of the group, 64-query block) pairs
+    }
+    return g;
+  };
+
+  if (warp == 0) {
+    // ------------------------------------------------ TMA producer
+    if (elect_one()) {
+      Geo nx = load_geo(blockIdx.x);
+      int it = 0, gb = 0;
+      for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+        const Geo G = nx;
+        nx = load_geo(item + gridDim.x);
+        const int k0 = G.blk0, hk = G.head, nqb = (G.L - k0 + QB - 1) / QB;
+        const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
+        wait_bar(&kv_empty, (it & 1) ^ 1);
+        mbar_expect_tx(&kv_full, 2 * KV_TILE);
+        tma_load_2d(sK, &tmQKV128, &kv_full, kcol, G.base + k0);
+        tma_load_2d(sK + 16384, &tmQKV128, &kv_full, kcol + 64, G.base + k0);
+        tma_load_2d(sV, &tmQKV128, &kv_full, vcol, G.base + k0);
+        tma_load_2d(sV + 16384, &tmQKV128, &kv_full, vcol + 64, G.base + k0);
+        for (int j = 0; j < G.n; ++j, ++gb) {
+          const int st = gb % STAGES;
+          const int h = hk * rep + j / nqb, q0 = k0 + (j % nqb) * QB;
+          wait_bar(&empty[st], ((gb / STAGES) & 1) ^ 1);
+          mbar_expect_tx(&full[st], 2 * QB_TILE);
+          uint8_t* q = sQ0 + st * QB_TILE;
+          uint8_t* o = sO0 + st * QB_TILE;
+          tma_load_2d(q, &tmQKV64, &full[st], h * HD, G.base + q0);
+          tma_load_2d(q + 8192, &tmQKV64, &full[st], h * HD + 64, G.base + q0);
+          tma_load_2d(o, &tmDO64, &full[st], h * HD, G.base + q0);
+          tma_load_2d(o + 8192, &tmDO64, &full[st], h * HD + 64, G.base + q0);
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    // ------------------------------------------------ MMA issuer
+    constexpr uint32_t ID_S = umma_idesc_bf16(128, QB, 0);     // [128 kv] x [64 q], K = hd
+    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 kv] x [128 hd], K = 64 q, B MN-major
+    Geo nx = load_geo(blockIdx.x);
+    BP_DECL
+    int it = 0, gb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = nx;
+      nx = load_geo(item + gridDim.x);
+      auto issue_acc = [&](int gp, int jp) {  // dV += P^T dO ; dK += dS^T Q   for global block gp (item block jp)
+        const int bp = gp & 1, sp = gp % STAGES;
+        BP(10);
+        wait_bar(&ew_done[bp], (gp >> 1) & 1);
+        BP(11);
+        if (jp == 0) wait_bar(&acc_free, (it & 1) ^ 1);   // previous item's epilogue has read dV / dK
+        BP(12);
+        tc_fence_after();
+        __syncwarp();
+        if (elect_one()) {
+          const uint32_t pa = smem_u32(sP0 + bp * PT_TILE), sa = smem_u32(sS0 + bp * PT_TILE);
+          const uint32_t ob = smem_u32(sO0 + sp * QB_TILE), qb = smem_u32(sQ0 + sp * QB_TILE);
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const uint32_t acc = (jp > 0 || kk > 0) ? 1u : 0u;
+            tc_mma_bf16(tdV, umma_desc_sw128(pa + kk * 32, 16, 1024), umma_desc_sw128(ob + kk * 2048, 8192, 1024), ID_ACC, acc);
+            tc_mma_bf16(tdK, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(qb + kk * 2048, 8192, 1024), ID_ACC, acc);
+          }
+          tc_commit(&empty[sp]);     // Q/dO stage free
+          tc_commit(&pd_free[bp]);   // P^T/dS^T buffer free
+        }
+        __syncwarp();
+        BP(13);
+      };
+      wait_bar(&kv_full, it & 1);
+      tc_fence_after();
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        const int b = gb & 1, st = gb % STAGES;
+        BP(10);
+        wait_bar(&full[st], (gb / STAGES) & 1);
+        BP(14);
+        tc_fence_after();
+        __syncwarp();
+        if (elect_one()) {
+          const uint32_t k = smem_u32(sK), v = smem_u32(sV);
+          const uint32_t q = smem_u32(sQ0 + st * QB_TILE), o = smem_u32(sO0 + st * QB_TILE);
+#pragma unroll
+          for (int kk = 0; kk < 8; ++kk) {
+            const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
+            tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(k + offa, 16, 1024), umma_desc_sw128(q + offb, 16, 1024), ID_S, kk > 0);
+            tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(v + offa, 16, 1024), umma_desc_sw128(o + offb, 16, 1024), ID_S, kk > 0);
+          }
+          tc_commit(&s_full[b]);
+          if (j == G.n - 1) tc_commit(&kv_empty);   // K / V free once the item's last S^T / dP^T completes
+        }
+        __syncwarp();
+        if (j > 0) issue_acc(gb - 1, j - 1);
+      }
+      if (G.n > 0) issue_acc(gb - 1, G.n - 1);
+      __syncwarp();
+      if (elect_one()) tc_commit(&acc_full);
+      __syncwarp();
+    }
+    BP(10);
+    BP_FLUSH(blockIdx.x < 8 && lane == 0);
+  } else {
+    // ------------------------------------------------ elementwise warps (thread = key row = TMEM lane;
+    //                                                  warpgroup g owns query columns [32 g, 32 g + 32))
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
+    const int r = w4 * 32 + lane;           // key row within the block
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
+    const float sl2 = p.scale * LOG2E_W;
+    Geo nx = load_geo(blockIdx.x);
+    BP_DECL
+    // lse (t < 64) or D (64 <= t < 128) of query t & 63 of (item G, block j); 0 outside the sequence / list
+    auto lse_d_load = [&](const Geo& G, int j) -> float {
+      if (t >= 2 * QB || G.n == 0) return 0.f;
+      const int nqb = (G.L - G.blk0 + QB - 1) / QB;
+      const int h = G.head * rep + j / nqb, qpos = G.blk0 + (j % nqb) * QB + (t & (QB - 1));
+      return qpos < G.L ? __ldg((t < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos) : 0.f;
+    };
+    float pre = 0.f;
+    int it = 0, gb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = nx;
+      nx = load_geo(item + gridDim.x);
+      const int k0 = G.blk0, L = G.L, base = G.base, nqb = (L - k0 + QB - 1) / QB;
+      const int kpos = k0 + r;
+      if (it == 0) pre = lse_d_load(G, 0);
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        const int b = gb & 1;
+        const int q0 = k0 + (j % nqb) * QB;
+        if (t < 2 * QB) {  // stage lse (log2 domain) and D of the block's 64 queries (loaded one block ahead)
+          const int c = t & (QB - 1);
+          if (t < QB) s_lse[b][c] = pre * LOG2E_W; else s_D[b][c] = pre * p.scale;   // D pre-scaled
+          pre = j + 1 < G.n ? lse_d_load(G, j + 1) : lse_d_load(nx, 0);
+        }
+        BP(0);
+        ew_sync();
+        BP(1);
+        wait_bar(&s_full[b], (gb >> 1) & 1);
+        BP(2);
+        tc_fence_after();
+        __syncwarp();
+        uint32_t su[32], du[32];
+        tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
+        tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+        tmem_wait_ld();
+        const int cmin = kpos - q0 - 32 * g;   // P = 0 for queries before the key (causal) ...
+        const int cmax = L - q0 - 32 * g;      // ... and past the end of the sequence
+        const bool full = cmin <= 0 && cmax >= 32;   // interior block: no mask in this row half
+        float pv[32], dsv[32];
+#pragma unroll
+        for (int c4 = 0; c4 < 32; c4 += 4) {
+          const float4 lz = *reinterpret_cast<const float4*>(&s_lse[b][32 * g + c4]);
+          const float4 dz = *reinterpret_cast<const float4*>(&s_D[b][32 * g + c4]);
+          const float lzv[4] = {lz.x, lz.y, lz.z, lz.w}, dzv[4] = {dz.x, dz.y, dz.z, dz.w};
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int c = c4 + u;
+            const bool ok = full || (c >= cmin && c < cmax);
+            const float x = fmaf(__uint_as_float(su[c]), sl2, -lzv[u]);
+            const float e = u == 3 ? poly_exp2(x) : fast_exp2(x);
+            pv[c] = ok ? e : 0.f;
+            dsv[c] = ok ? e * fmaf(__uint_as_float(du[c]), p.scale, -dzv[u]) : 0.f;
+          }
+        }
+        BP(3);
+        if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
+        BP(4);
+        st_half_row(sP0 + b * PT_TILE, r, g, pv);
+        st_half_row(sS0 + b * PT_TILE, r, g, dsv);
+        fence_proxy_async();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ew_done[b]);
+        BP(5);
+      }
+      // ------------------------------------------------ epilogue: dK (RoPE bwd), dV rows -> dqkv
+      BP(0);
+      wait_bar(&acc_full, it & 1);
+      BP(6);
+      tc_fence_after();
+      __syncwarp();
+      // all MMAs of this item completed: P^T / dS^T buffers are free for staging
+      const int nv = min(KV_ROWS, L - k0);
+      bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
+      acc_epilogue(tdK + lane_off, sP0, w4, w8, lane, g, nv, dst + (p.H + G.head) * HD, p.ld_dqkv, p.rope_cs, k0,
+                   true, &acc_free, false);
+      BP(7);
+      acc_epilogue(tdV + lane_off, sP0, w4, w8, lane, g, nv, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv,
+                   p.rope_cs, k0, false, &acc_free, true);
+      BP(8);
+    }
+    BP_FLUSH(blockIdx.x < 8 && t == 0);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<512>(tmem);
+  }
+}
+
+// ======================================================================================= dQ
+constexpr int Q_ROWS = 128, KB = 64;
+constexpr int Q_TILE = Q_ROWS * HD * 2;       // 32 KB
+constexpr int KB_TILE = KB * HD * 2;          // 16 KB
+constexpr int DS_TILE = Q_ROWS * KB * 2;      // 16 KB
+constexpr int SMEM_DQ = 2 * Q_TILE + 2 * STAGES * KB_TILE + 2 * DS_TILE + 1024;
+
+__global__ void __launch_bounds__(NTHREADS, 1)
+attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
+                      const __grid_constant__ CUtensorMap tmDO128, const BwParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* const sQ = smem;
+  uint8_t* const sO = sQ + Q_TILE;
+  uint8_t* const sK0 = sO + Q_TILE;                  // K stages
+  uint8_t* const sV0 = sK0 + STAGES * KB_TILE;       // V stages
+  uint8_t* const sS0 = sV0 + STAGES * KB_TILE;       // dS (2 buffers) -- dQ staging in the epilogue
+  __shared__ __align__(8) uint64_t q_full, q_empty, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2];
+  __shared__ __align__(8) uint64_t acc_full, acc_free;
+  __shared__ uint32_t tmem_sh;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO128);
+    mbar_init(&q_full, 1); mbar_init(&q_empty, 1);
+    for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
+    mbar_init(&acc_full, 1); mbar_init(&acc_free, EW_WARPS);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;
+  const uint32_t tdQ = tmem + 256;   // S buffers at 0/64, dP at 128/192
+
+  auto load_geo = [&](int item) {
+    Geo g{0, 0, 0, 0, 0};
+    if (item < p.n_items) {
+      const int4 it = p.items[item];
+      g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
+      g.n = (min(g.L, g.blk0 + Q_ROWS) + KB - 1) / KB;
+    }
+    return g;
+  };
+
+  if (warp == 0) {
+    if (elect_one()) {
+      Geo nx = load_geo(blockIdx.x);
+      int it = 0, gb = 0;
+      for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+        const Geo G = nx;
+        nx = load_geo(item + gridDim.x);
+        const int h = G.head, hk = h / (p.H / p.Hkv), q0 = G.blk0;
+        const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
+        wait_bar(&q_empty, (it & 1) ^ 1);
+        mbar_expect_tx(&q_full, 2 * Q_TILE);
+        tma_load_2d(sQ, &tmQKV128, &q_full, h * HD, G.base + q0);
+        tma_load_2d(sQ + 16384, &tmQKV128, &q_full, h * HD + 64, G.base + q0);
+        tma_load_2d(sO, &tmDO128, &q_full, h * HD, G.base + q0);
+        tma_load_2d(sO + 16384, &tmDO128, &q_full, h * HD + 64, G.base + q0);
+        for (int j = 0; j < G.n; ++j, ++gb) {
+          const int st = gb % STAGES;
+          wait_bar(&empty[st], ((gb / STAGES) & 1) ^ 1);
+          mbar_expect_tx(&full[st], 2 * KB_TILE);
+          uint8_t* k = sK0 + st * KB_TILE;
+          uint8_t* v = sV0 + st * KB_TILE;
+          tma_load_2d(k, &tmQKV64, &full[st], kcol, G.base + j * KB);
+          tma_load_2d(k + 8192, &tmQKV64, &full[st], kcol + 64, G.base + j * KB);
+          tma_load_2d(v, &tmQKV64, &full[st], vcol, G.base + j * KB);
+          tma_load_2d(v + 8192, &tmQKV64, &full[st], vcol + 64, G.base + j * KB);
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    constexpr uint32_t ID_S = umma_idesc_bf16(128, KB, 0);     // [128 q] x [64 keys], K = hd
+    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 q] x [128 hd], K = 64 keys, B MN-major
+    Geo nx = load_geo(blockIdx.x);
+    int it = 0, gb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = nx;
+      nx = load_geo(item + gridDim.x);
+      auto issue_acc = [&](int gp, int jp) {  // dQ += dS K
+        const int bp = gp & 1, sp = gp % STAGES;
+        wait_bar(&ew_done[bp], (gp >> 1) & 1);
+        if (jp == 0) wait_bar(&acc_free, (it & 1) ^ 1);
+        tc_fence_after();
+        __syncwarp();
+        if (elect_one()) {
+          const uint32_t sa = smem_u32(sS0 + bp * DS_TILE), kb_ = smem_u32(sK0 + sp * KB_TILE);
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            tc_mma_bf16(tdQ, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(kb_ + kk * 2048, 8192, 1024), ID_ACC,
+                        (jp > 0 || kk > 0) ? 1u : 0u);
+          tc_commit(&empty[sp]);
+          tc_commit(&pd_free[bp]);
+        }
+        __syncwarp();
+      };
+      wait_bar(&q_full, it & 1);
+      tc_fence_after();
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        const int b = gb & 1, st = gb % STAGES;
+        wait_bar(&full[st], (gb / STAGES) & 1);
+        tc_fence_after();
+        __syncwarp();
+        if (elect_one()) {
+          const uint32_t q = smem_u32(sQ), o = smem_u32(sO);
+          const uint32_t k = smem_u32(sK0 + st * KB_TILE), v = smem_u32(sV0 + st * KB_TILE);
+#pragma unroll
+          for (int kk = 0; kk < 8; ++kk) {
+            const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
+            tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(q + offa, 16, 1024), umma_desc_sw128(k + offb, 16, 1024), ID_S, kk > 0);
+            tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(o + offa, 16, 1024), umma_desc_sw128(v + offb, 16, 1024), ID_S, kk > 0);
+          }
+          tc_commit(&s_full[b]);
+          if (j == G.n - 1) tc_commit(&q_empty);   // Q / dO free once the item's last S / dP completes
+        }
+        __syncwarp();
+        if (j > 0) issue_acc(gb - 1, j - 1);
+      }
+      if (G.n > 0) issue_acc(gb - 1, G.n - 1);
+      __syncwarp();
+      if (elect_one()) tc_commit(&acc_full);
+      __syncwarp();
+    }
+  } else {
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2;   // warpgroup g owns key columns [32 g, 32 g + 32)
+    const int r = w4 * 32 + lane;           // query row
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
+    const float sl2 = p.scale * LOG2E_W;
+    Geo nx = load_geo(blockIdx.x);
+    int it = 0, gb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = nx;
+      nx = load_geo(item + gridDim.x);
+      const int h = G.head, q0 = G.blk0, L = G.L, base = G.base;
+      const int qpos = q0 + r;
+      const bool qok = qpos < L;
+      const float lse2 = qok ? p.lse[(size_t)h * p.T + base + qpos] * LOG2E_W : 0.f;
+      const float Dq = qok ? p.D[(size_t)h * p.T + base + qpos] * p.scale : 0.f;   // pre-scaled
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        const int b = gb & 1;
+        wait_bar(&s_full[b], (gb >> 1) & 1);
+        tc_fence_after();
+        __syncwarp();
+        uint32_t su[32], du[32];
+        tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
+        tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+        tmem_wait_ld();
+        const int cmax = qok ? qpos - j * KB - 32 * g : -1;   // keys <= query
+        float dsv[32];
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+          const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+          const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
+          const float v = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
+          dsv[c] = (cmax >= 31 || c <= cmax) ? v : 0.f;
+        }
+        if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
+        st_half_row(sS0 + b * DS_TILE, r, g, dsv);
+        fence_proxy_async();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ew_done[b]);
+      }
+      wait_bar(&acc_full, it & 1);
+      tc_fence_after();
+      __syncwarp();
+      const int nv = min(Q_ROWS, L - q0);
+      acc_epilogue(tdQ + lane_off, sS0, w4, w8, lane, g, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD,
+                   p.ld_dqkv, p.rope_cs, q0, true, &acc_free, true);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<512>(tmem);
+  }
+}
+
+}  // namespace
+
+#ifdef MENOS_BWS_PROF
+int attn_bws_prof_read(unsigned long long* out) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, g_bws_prof, sizeof(unsigned long long) * 16);
+  unsigned long long z[16] = {0};
+  cudaMemcpyToSymbol(g_bws_prof, z, sizeof z);
+  return 0;
+}
+#endif
+
+// items_kv: (seq, k0, kv head) per 128-key block for dK/dV; items_q: (seq, q0, head) per 128-query block for dQ
+int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                int num_sms, cudaStream_t st) {
+  if (a.hd != HD) return -1;
+  if (n_items_kv <= 0 && n_items_q <= 0) return 0;
+  CUtensorMap mQKV128, mQKV64, mDO64, mDO128;
+  if (!tma_map_2d(&mQKV128, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 128)) return -2;
+  if (!tma_map_2d(&mQKV64, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 64)) return -2;
+  if (!tma_map_2d(&mDO64, a.dO, a.T, a.H * HD, a.ld_do, 64, 64)) return -2;
+  if (!tma_map_2d(&mDO128, a.dO, a.T, a.H * HD, a.ld_do, 64, 128)) return -2;
+  BwParams p;
+  p.cu_seqlens = a.cu_seqlens; p.lse = a.lse; p.D = a.D; p.dqkv = a.dqkv;
+  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv; p.scale = a.scale;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(attn_bwd_dkdv_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DKDV);
+    cudaFuncSetAttribute(attn_bwd_dq_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DQ);
+    attr = true;
+  }
+  p.items = items_kv; p.n_items = n_items_kv;
+  attn_bwd_dkdv_ws_kernel<<<min(n_items_kv, num_sms), NTHREADS, SMEM_DKDV, st>>>(mQKV128, mQKV64, mDO64, p);
+  ++g_launch_count;
+  p.items = items_q; p.n_items = n_items_q;
+  attn_bwd_dq_ws_kernel<<<min(n_items_q, num_sms), NTHREADS, SMEM_DQ, st>>>(mQKV128, mQKV64, mDO128, p);
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+}  // namespace menos

@@ -15,6 +15,7 @@
 //   * warps 4-7 = softmax, one query row per thread (= TMEM lane): online softmax in the log2 domain with a
 //     lazy max (O in TMEM is rescaled only when a row max grows by more than 2^8; P values stay <= 256),
 //     P = exp2(S - m) in bf16 written into a 128B-swizzled smem tile that is the next PV MMA's A operand.
+#include <algorithm>
 #include "common.cuh"
 #include "kernels.h"
 
@@ -371,11 +372,21 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
 bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
                 uint32_t br);
 
-void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out) {
+void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order) {
   // (sequence, head) groups, q blocks of a group adjacent and largest first: the group's K/V stays in L2
+  const size_t first = out.size();
   for (int i = 0; i < n_seqs; ++i)
     for (int h = 0; h < H; ++h)
       for (int q = ((seq_len[i] - 1) / BQ) * BQ; q >= 0; q -= BQ) out.push_back(make_int4(i, q, h, 0));
+  if (order == 0) return;
+  // LPT for the static round-robin of the persistent grids: stable sort by work, largest first.  order 1:
+  // work ~ causal kv blocks of a query block (forward, dQ); order 2: ~ query blocks after a key block (dK/dV)
+  std::vector<int> len(seq_len, seq_len + n_seqs);
+  auto cost = [&](const int4& it) {
+    const int L = len[it.x];
+    return order == 1 ? std::min(L, it.y + BQ) : L - it.y;
+  };
+  std::stable_sort(out.begin() + first, out.end(), [&](const int4& a, const int4& b) { return cost(a) > cost(b); });
 }
 
 #ifdef MENOS_WS_PROF

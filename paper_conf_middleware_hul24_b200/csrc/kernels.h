@@ -105,10 +105,17 @@ int attn_fwd(const AttnArgs& a, cudaStream_t st);
 int attn_fwd_tc(const AttnArgs& a, const int2* qblocks128, int n_qblocks128, cudaStream_t st);
 // persistent warp-specialized tcgen05 forward for head_dim 128 (attention_fwd_ws.cu); items = (seq, q0, head, -)
 int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st);
-void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out);
+// order: 0 = (sequence, head) groups (L2 locality), 1 = largest forward / dQ work first, 2 = largest dK/dV first
+void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order = 0);
+// persistent warp-specialized tcgen05 backward for head_dim 128 (attention_bwd_ws.cu): items_kv = (seq, k0, kv
+// head, -) per 128-key block, items_q = (seq, q0, head, -) per 128-query block
+int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                int num_sms, cudaStream_t st);
 // head_dim 128 variant bitmask: 1 = tcgen05 forward (2-pass), 2 = tcgen05 backward, 4 = persistent
-// warp-specialized tcgen05 forward (takes precedence over 1)
+// warp-specialized tcgen05 forward (takes precedence over 1), 8 = persistent warp-specialized tcgen05 backward
+// (takes precedence over 2)
 extern int g_attn_tc;
+extern int g_attn_order;   // persistent attention work order: 1 = LPT (default), 0 = (sequence, head) grouped
 int attn_bwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 backward for head_dim 128 (attention_bwd_tc.cu); blocks128 = (seq, local start) per 128-row block
 int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaStream_t st);

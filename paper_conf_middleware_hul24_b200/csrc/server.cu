@@ -252,7 +252,9 @@ struct menos_batch {
   bool save_a = false;
   int n_mt = 0, n_blocks = 0, n_blocks128 = 0;
   int2* d_blocks128 = nullptr;
-  int4* d_attn_items = nullptr; int n_attn_items = 0;   // persistent attention forward work list
+  int4* d_attn_items = nullptr; int n_attn_items = 0;   // persistent attention work list (query blocks x heads)
+  int4* d_attn_items_kv = nullptr; int n_attn_items_kv = 0;   // key blocks x kv heads (dK/dV)
+  int4* d_attn_items_q = nullptr;                              // query blocks x heads, backward order (dQ)
   double pairs = 0;   // causal (query, key) pairs summed over sequences
   // device metadata
   uint8_t* meta = nullptr;  // arena
@@ -948,8 +950,12 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     for (int q = 0; q < b->seq_len[i]; q += 128) blocks128.push_back(make_int2(i, q));
   b->n_blocks128 = (int)blocks128.size();
   std::vector<int4> attn_items;
-  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items);
+  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items, g_attn_order ? 1 : 0);
   b->n_attn_items = (int)attn_items.size();
+  std::vector<int4> attn_items_kv, attn_items_q;
+  attn_ws_items(b->seq_len.data(), b->n_seqs, D.Hkv, attn_items_kv, g_attn_order ? 2 : 0);
+  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items_q, g_attn_order ? 1 : 0);
+  b->n_attn_items_kv = (int)attn_items_kv.size();
   std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
   for (int g = 0; g < NG; ++g) {
     if (!b->g_active[g]) continue;
@@ -980,6 +986,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_blk = put(blocks.data(), blocks.size() * sizeof(int2));
   const size_t o_blk128 = put(blocks128.data(), blocks128.size() * sizeof(int2));
   const size_t o_items = put(attn_items.data(), attn_items.size() * sizeof(int4));
+  const size_t o_items_kv = put(attn_items_kv.data(), attn_items_kv.size() * sizeof(int4));
+  const size_t o_items_q = put(attn_items_q.data(), attn_items_q.size() * sizeof(int4));
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
 
@@ -1122,6 +1130,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
   b->d_blocks128 = (int2*)(meta + o_blk128);
   b->d_attn_items = (int4*)(meta + o_items);
+  b->d_attn_items_kv = (int4*)(meta + o_items_kv);
+  b->d_attn_items_q = (int4*)(meta + o_items_q);
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
   b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
@@ -1372,7 +1382,9 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
     {
       ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * b->pairs, 0, st);
-      if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+      if (D.hd == 128 && (g_attn_tc & 8))
+        K_TRY(attn_bwd_ws(a, b->d_attn_items_kv, b->n_attn_items_kv, b->d_attn_items_q, b->n_attn_items, s->num_sms, st));
+      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, b->n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
     }
   }

@@ -96,7 +96,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   const bool tc_fwd = hd == 128 && (g_attn_tc & 1), tc_bwd = hd == 128 && (g_attn_tc & 2);
   const bool ws_fwd = hd == 128 && (g_attn_tc & 4);
   std::vector<int4> items;
-  attn_ws_items(seq_len, n_seqs, H, items);
+  attn_ws_items(seq_len, n_seqs, H, items, g_attn_order ? 1 : 0);
   int4* d_items;
   cudaMalloc(&d_items, std::max<size_t>(1, items.size()) * sizeof(int4));
   cudaMemcpy(d_items, items.data(), items.size() * sizeof(int4), cudaMemcpyHostToDevice);
@@ -108,7 +108,16 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
-    rc = tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+    std::vector<int4> items_kv;
+    attn_ws_items(seq_len, n_seqs, Hkv, items_kv, g_attn_order ? 2 : 0);
+    int4* d_items_kv;
+    cudaMalloc(&d_items_kv, std::max<size_t>(1, items_kv.size()) * sizeof(int4));
+    cudaMemcpy(d_items_kv, items_kv.data(), items_kv.size() * sizeof(int4), cudaMemcpyHostToDevice);
+    const bool ws_bwd = hd == 128 && (g_attn_tc & 8);
+    rc = ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
+                : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+    cudaDeviceSynchronize();
+    cudaFree(d_items_kv);
   }
   cudaError_t e = cudaDeviceSynchronize();
   cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D); cudaFree(d_b128); cudaFree(d_items);
@@ -205,11 +214,14 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
 }
 
 // Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward (2-pass, serialized), 2 = tcgen05 backward
-// (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1).
-// Default 6: the persistent tcgen05 forward (2.1x the mma.sync kernel at S = 512) and the tcgen05 backward.
-namespace menos { int g_attn_tc = 6; }
+// (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1),
+// 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; overrides 2).
+// Default 14: the persistent tcgen05 forward and backward (LPT work order, bit 4 selects (sequence, head) order).
+namespace menos { int g_attn_tc = 14; int g_attn_order = 1; }
 extern "C" int menos_test_set_attn_tc(int mode) {
-  if (mode < 0 || mode > 7) { fail("attention mode must be in [0, 7]"); return MENOS_EINVAL; }
+  if (mode < 0 || mode > 31) { fail("attention mode must be in [0, 31]"); return MENOS_EINVAL; }
+  menos::g_attn_order = (mode & 16) ? 0 : 1;   // bit 4: (sequence, head)-grouped work order instead of LPT
+  mode &= 15;
   menos::g_attn_tc = mode;
   return MENOS_OK;
 }

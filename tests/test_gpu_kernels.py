@@ -232,7 +232,9 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 6), (128, 8, 1, [130, 7, 256], 6),
+@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 14), (128, 8, 1, [130, 7, 256], 14),
+                                             (128, 2, 2, [512, 1024, 255], 14), (128, 3, 1, [2048, 1, 700], 14),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 6), (128, 8, 1, [130, 7, 256], 6),
                                              (128, 2, 2, [512, 1024, 255], 6), (128, 3, 1, [2048, 1, 700], 6),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 3), (128, 4, 2, [1, 17, 64, 129, 300], 0),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 2), (128, 8, 1, [130, 7, 256], 3),
