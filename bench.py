@@ -195,7 +195,7 @@ def run_gpu(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     device = torch.device("cuda", local)
     torch.cuda.set_device(device)
-    from paper_conf_middleware_hul24_b200.partition import plan_waves, workload_partition
+    from paper_conf_middleware_hul24_b200.partition import plan_waves_exact, workload_partition
     if os.environ.get("MENOS_ATTN_TC") is not None:   # kernel-variant switch for A/B measurements
         M.lib().menos_test_set_attn_tc(int(os.environ["MENOS_ATTN_TC"]))
     w = workload(args.workload, n_layers=args.layers)
@@ -223,8 +223,11 @@ def run_gpu(args):
     ids = register_clients(np, srv, w, seed=rank + 1)
     # waves: temporal sharing of the arena when the clients' saved activations do not fit at once
     mem = [srv.client_memory(ids[i], c.n_tokens) for i, c in enumerate(w.clients)]
-    cap = srv.stats()["arena_bytes"] - (256 << 20)
-    waves = plan_waves([m[1] for m in mem], [m[2] for m in mem], cap)
+    cap = srv.stats()["arena_bytes"] - (64 << 20)
+
+    def demand(idx):   # exact peak arena bytes of one batched call (menos_batch_memory)
+        return max(srv.batch_memory([ids[i] for i in idx], [w.clients[i].n_tokens for i in idx]))
+    waves = plan_waves_exact(len(w.clients), demand, cap)
     toff = [0]
     for c in w.clients:
         toff.append(toff[-1] + c.n_tokens)

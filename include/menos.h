@@ -151,6 +151,14 @@ MENOS_API int menos_unregister_client(menos_server* s, int32_t client_id);
 MENOS_API int menos_client_memory(menos_server* s, int32_t client_id, int n_tokens, size_t* persistent, size_t* fwd_bytes,
                         size_t* bwd_bytes);
 
+/* Exact arena demand of ONE batched call over these clients (n_tokens[i] tokens of client ids[i]): the peak arena
+ * bytes the forward (*fwd_bytes) and the backward (*bwd_bytes) of that batch need, including the per-call scratch
+ * block and the block-diagonal LoRA slot columns the batch spans (which depend on the set of clients, so a sum of
+ * per-client menos_client_memory figures is not exact).  flags as in menos_forward.  Used to form waves / admit
+ * clients (Alg.2) without ever hitting MENOS_ENOMEM. */
+MENOS_API int menos_batch_memory(menos_server* s, int n_clients, const int32_t* ids, const int32_t* n_tokens, int flags,
+                       size_t* fwd_bytes, size_t* bwd_bytes);
+
 /* Step 2: x_s = f_s(x_c).  n_seqs sequences; seq_client[i] (host) is the client of sequence i and
  * seq_len[i] (host) its length (>= 1, <= max_seq_len).  Sequences of one client must be contiguous
  * (client-major packing).  T = sum(seq_len).  x_c, x_s: [T, d] bf16 (host or device).

@@ -743,6 +743,39 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
   return MENOS_OK;
 }
 
+static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save);
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set);
+static size_t meta_bytes_bound(int T, int Ls, int n_clients);
+
+extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t* ids, const int32_t* n_tokens,
+                                  int flags, size_t* fwd_bytes, size_t* bwd_bytes) {
+  if (!s || n_clients < 0 || (n_clients > 0 && (!ids || !n_tokens))) FAIL(MENOS_EINVAL, "bad arguments");
+  const Dims& D = s->D;
+  int R[NG] = {0, 0, 0, 0};
+  bool save_a = false;
+  long long T = 0;
+  for (int i = 0; i < n_clients; ++i) {
+    const int id = ids[i];
+    if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+    if (n_tokens[i] < 0) FAIL(MENOS_EINVAL, "n_tokens < 0");
+    const Client& c = s->clients[id];
+    for (int g = 0; g < NG; ++g) if (c.width[g]) R[g] = std::max(R[g], c.col_off[g] + c.width[g]);
+    if (c.mask >> TD & 1) save_a = true;
+    T += n_tokens[i];
+  }
+  if (T > (1ll << 30)) FAIL(MENOS_EINVAL, "too many tokens");
+  for (int g = 0; g < NG; ++g) R[g] = (int)align_up(R[g], 64);
+  const bool nograd = flags & MENOS_FWD_NOGRAD;
+  const size_t meta = meta_bytes_bound((int)T, s->n_layers, n_clients);
+  // forward: scratch (+ the NOGRAD layer set) + slab (+ meta); backward of a NOGRAD batch re-forwards with SAVE
+  const size_t fwd = scratch_bytes_of(D, (int)T, R, nograd) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, !nograd) + meta;
+  const size_t bwd = scratch_bytes_of(D, (int)T, R, nograd) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, true) +
+                     (nograd ? slab_bytes_of(D, s->n_layers, (int)T, R, save_a, false) : 0) + 2 * meta;
+  if (fwd_bytes) *fwd_bytes = fwd;
+  if (bwd_bytes) *bwd_bytes = bwd;
+  return MENOS_OK;
+}
+
 extern "C" int menos_adapter_shape(menos_server* s, int32_t id, int target, int* rows, int* cols) {
   if (!s || !rows || !cols) FAIL(MENOS_EINVAL, "null argument");
   if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
@@ -919,24 +952,51 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
 }
 
 // Allocate the slab (saved activations or x_c copy) and upload all metadata incl. small-GEMM problem lists.
+// arena bytes of a batch's slab: the SAVE activations of every layer (I in Eq.3), or under NOGRAD
+// only the x_c copy; R_used = the batch's block-diagonal LoRA slot widths per group (0 = inactive)
+static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save) {
+  if (!save) return align_up((size_t)T * D.d * 4, 256);
+  size_t per_layer = 0;
+  auto A = [&](size_t n) { per_layer += align_up(n, 256); };
+  A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x (fp32), xn, rstd1
+  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
+  A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h (fp32), hn, rstd2
+  A((size_t)T * 2 * D.fpad * 2);                                            // gu
+  if (save_a) A((size_t)T * D.fpad * 2);
+  for (int g = 0; g < NG; ++g) if (R_used[g]) A((size_t)T * R_used[g] * 2);
+  return per_layer * Ls;
+}
+// arena bytes of the per-call scratch block (see get_scratch)
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set) {
+  size_t need = 0;
+  auto A = [&](size_t n) { need += align_up(n, 256); };
+  const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
+  A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout
+  A(db); A(db); A(db); A(db); A(db);                                          // dyb, dxb, dhb, dhn, io
+  A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * 2 * D.fpad * 2); A((size_t)T * D.fpad * 2);
+  A((size_t)D.H * T * 4);
+  for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
+  // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
+  if (nograd_set) {
+    A(db); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
+    A((size_t)T * 2 * D.fpad * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
+    for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
+  }
+  return need;
+}
+// generous bound of a batch's metadata block (segment tables, positions, tile maps, LoRA problem lists)
+static size_t meta_bytes_bound(int T, int Ls, int n_clients) {
+  return (size_t)64 * T + (size_t)Ls * (64 << 10) + (size_t)n_clients * Ls * 4096 + (1 << 20);
+}
+
 static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const LayerSave* ng, cudaStream_t st) {
   const Dims& D = s->D;
   const int T = b->T, Ls = s->n_layers;
   // ---- sizes
   const bool save = !b->nograd;
-  size_t ush = 0;
-  for (int g = 0; g < NG; ++g) if (b->g_active[g]) ush += (size_t)b->R_used[g] * 2;
-  size_t per_layer = 0;
-  auto A = [&](size_t n) { per_layer += align_up(n, 256); };
-  if (save) {
-    A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x (fp32), xn, rstd1
-    A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
-    A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h (fp32), hn, rstd2
-    A((size_t)T * 2 * D.fpad * 2);                                            // gu
-    if (b->save_a) A((size_t)T * D.fpad * 2);
-    for (int g = 0; g < NG; ++g) if (b->g_active[g]) A((size_t)T * b->R_used[g] * 2);
-  }
-  const size_t slab_bytes = save ? per_layer * Ls : align_up((size_t)T * D.d * 4, 256);
+  int R_act[NG];
+  for (int g = 0; g < NG; ++g) R_act[g] = b->g_active[g] ? b->R_used[g] : 0;
+  const size_t slab_bytes = slab_bytes_of(D, Ls, T, R_act, b->save_a, save);
   // ---- metadata blob
   std::vector<uint8_t> blob;
   auto put = [&](const void* p, size_t n) {
@@ -1142,22 +1202,12 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
 }
 
 // scratch (per server, grown to the largest batch; used only inside one call)
-static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc) {
+// nograd_set: also reserve the NOGRAD forward's layer buffers (only a MENOS_FWD_NOGRAD forward needs them; the
+// backward's re-forward writes into the batch's SAVE slab), so SAVE batches use exactly scratch_bytes_per_token
+static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set) {
   const Dims& D = s->D;
-  int rsum = 0;
-  for (int g = 0; g < NG; ++g) rsum += R_used[g];
-  size_t need = 0;
-  auto A = [&](size_t n) { need += align_up(n, 256); };
+  const size_t need = scratch_bytes_of(D, T, R_used, nograd_set);
   const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
-  A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout
-  A(db); A(db); A(db); A(db); A(db);                                          // dyb, dxb, dhb, dhn, io
-  A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * 2 * D.fpad * 2); A((size_t)T * D.fpad * 2);
-  A((size_t)D.H * T * 4);
-  for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
-  // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
-  A(db); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
-  A((size_t)T * 2 * D.fpad * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
-  for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   if (need > s->scratch_bytes) {
     if (s->scratch) s->arena.release(s->scratch);
     s->scratch = (uint8_t*)s->arena.alloc(need);
@@ -1440,7 +1490,7 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
   const Dims& D = s->D;
   const int T = b->T;
   Scratch sc;
-  rc = get_scratch(s, T, b->R_used, sc);
+  rc = get_scratch(s, T, b->R_used, sc, b->nograd);
   if (rc) return rc;
   LayerSave ng{};
   if (b->nograd) nograd_layer(s, T, b->R_used, sc, ng);
@@ -1500,7 +1550,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   const Dims& D = s->D;
   const int T = b->T;
   Scratch sc;
-  int rc = get_scratch(s, T, b->R_used, sc);
+  int rc = get_scratch(s, T, b->R_used, sc, false);
   if (rc) return rc;
   if (b->nograd) {
     // Alg.1 L10: re-forward with gradient preparation from the cached x_c; the SAVE slab is

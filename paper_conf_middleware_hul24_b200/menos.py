@@ -75,6 +75,7 @@ SIGNATURES = {
     "menos_register_client": (_I, [_P, _I, _F, C.c_uint32, C.POINTER(AdamWCfg), C.c_uint64, _PI32]),
     "menos_unregister_client": (_I, [_P, C.c_int32]),
     "menos_client_memory": (_I, [_P, C.c_int32, _I, C.POINTER(_S), C.POINTER(_S), C.POINTER(_S)]),
+    "menos_batch_memory": (_I, [_P, _I, _PI32, _PI32, _I, C.POINTER(_S), C.POINTER(_S)]),
     "menos_forward": (_I, [_P, _I, _PI32, _PI32, _P, _P, _I, _P, C.POINTER(_P)]),
     "menos_backward": (_I, [_P, _P, _P, _P, _P]),
     "menos_batch_free": (_I, [_P, _P]),
@@ -217,6 +218,13 @@ class Server:
         a, b, c = C.c_size_t(), C.c_size_t(), C.c_size_t()
         check(lib().menos_client_memory(self.h, cid, n_tokens, C.byref(a), C.byref(b), C.byref(c)))
         return a.value, b.value, c.value
+
+    def batch_memory(self, client_ids, n_tokens, flags=FWD_SAVE):
+        """(fwd_bytes, bwd_bytes): exact peak arena demand of one batched forward / backward over these clients."""
+        a, b = C.c_size_t(), C.c_size_t()
+        check(lib().menos_batch_memory(self.h, len(client_ids), _i32(client_ids), _i32(n_tokens), flags, C.byref(a),
+                                       C.byref(b)))
+        return a.value, b.value
 
     def adapter_shape(self, cid: int, target: str):
         r = (C.c_int * 2)()

@@ -65,3 +65,21 @@ def plan_waves(fwd_bytes, scratch_bytes, capacity: int) -> list[list[int]]:
     if cur:
         waves.append(cur)
     return waves
+
+
+def plan_waves_exact(n_clients: int, demand, capacity: int) -> list[list[int]]:
+    """Same greedy wave formation as plan_waves, with the EXACT peak arena demand of a candidate wave:
+    demand(list_of_client_indices) -> bytes (the library's menos_batch_memory, which accounts for the block-diagonal
+    LoRA slot columns a wave spans and the per-call scratch).  Clients keep batch order (client-major packing)."""
+    waves: list[list[int]] = []
+    cur: list[int] = []
+    for i in range(n_clients):
+        if demand([i]) > capacity:
+            raise MemoryError(f"client {i} needs {demand([i])} B > arena {capacity} B")
+        if cur and demand(cur + [i]) > capacity:
+            waves.append(cur)
+            cur = []
+        cur.append(i)
+    if cur:
+        waves.append(cur)
+    return waves

@@ -160,6 +160,45 @@ def test_enomem_returned_not_crash():
     srv.close()
 
 
+@pytest.mark.parametrize("flags", [0, 1])
+def test_batch_memory_is_exact_bound(flags):
+    """menos_batch_memory (the admission query, Alg.2 L2 PAPER.md:238): an arena of max(fwd, bwd) bytes runs the
+    batch (SAVE, or NOGRAD + re-forward) and the observed arena peak P stays below it, with at most the metadata
+    bound (<= 4 MB here) of slack; an arena just below P is refused with ENOMEM (never a crash)."""
+    from paper_conf_middleware_hul24_b200 import MenosError
+    m = MODELS["tiny"]
+    cl = [ClientCfg(4, 8.0, ("q", "v"), [33, 60]), ClientCfg(16, 32.0, TARGETS, [100]), ClientCfg(8, 16.0, ("o", "down"), [7])]
+    w = Workload("bm", m, cl)
+    inputs = make_inputs(w, seed=21)
+    weights, adapters, io = inputs
+    x = torch.from_numpy(np.concatenate([a for a, _ in io])).to(torch.bfloat16).cuda()
+
+    def run(cap):
+        srv = new_server(w, weights, arena_bytes=cap)
+        ids = register(srv, w, adapters)
+        sc, sl = [], []
+        for i, c in enumerate(cl):
+            sc += [ids[i]] * len(c.seq_lens)
+            sl += list(c.seq_lens)
+        need = max(srv.batch_memory(ids, [c.n_tokens for c in cl], flags))
+        try:
+            b = srv.forward(sc, sl, x, torch.empty_like(x), flags=flags)
+            srv.backward(b, x, torch.empty_like(x))
+            torch.cuda.synchronize()
+            return need, srv.stats()["arena_peak"], None
+        except MenosError as e:
+            return need, None, e
+        finally:
+            srv.close()
+
+    need, _, _ = run(1 << 30)
+    need2, peak, err = run(need)
+    assert err is None and need2 == need
+    assert peak <= need <= peak + (4 << 20)
+    _, _, err = run(peak - 4096)
+    assert err is not None and err.code == -2
+
+
 def test_host_buffers_e2e_path():
     """x_c / g_c given as (pinned) host buffers: same results as device buffers."""
     w = workload("cfg0_tiny")

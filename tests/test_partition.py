@@ -76,3 +76,16 @@ def test_plan_waves():
     assert plan_waves([90, 5], [5, 1], 96) == [[0], [1]]
     with pytest.raises(MemoryError):
         plan_waves([200], [1], 100)
+
+
+def test_plan_waves_exact_uses_joint_demand():
+    from paper_conf_middleware_hul24_b200.partition import plan_waves_exact
+    # joint demand grows faster than the sum (block-diagonal slot columns span the wave)
+    sizes = [10, 10, 10, 10]
+    demand = lambda idx: sum(sizes[i] for i in idx) + 5 * len(idx) ** 2
+    waves = plan_waves_exact(4, demand, 60)
+    assert waves == [[0, 1], [2, 3]]
+    assert all(demand(w) <= 60 for w in waves)
+    assert sorted(i for w in waves for i in w) == [0, 1, 2, 3]
+    with pytest.raises(MemoryError):
+        plan_waves_exact(1, lambda idx: 100, 60)
