@@ -158,12 +158,23 @@ MENOS_API int menos_client_memory(menos_server* s, int32_t client_id, int n_toke
  * clients (Alg.2) without ever hitting MENOS_ENOMEM. */
 MENOS_API int menos_batch_memory(menos_server* s, int n_clients, const int32_t* ids, const int32_t* n_tokens, int flags,
                        size_t* fwd_bytes, size_t* bwd_bytes);
+/* flags bit for menos_batch_memory: figures are ADDITIVE UPPER BOUNDS -- computed with the LoRA slot span and the
+ * saved-tensor set of every registered client instead of the batch's own, so for any partition of a batch into
+ * parts P_k, sum_k demand(P_k, MENOS_MEM_BOUND) >= demand(batch): every term is linear in tokens plus a nonnegative
+ * constant, and 256-byte rounding is subadditive.  The Alg.2 scheduler (menos_sched_*) ADDS per-client demands
+ * (PAPER.md:238-263); this keeps its accounting safe when the granted requests run as one batched call. */
+enum { MENOS_MEM_BOUND = 2 };
 
 /* Step 2: x_s = f_s(x_c).  n_seqs sequences; seq_client[i] (host) is the client of sequence i and
  * seq_len[i] (host) its length (>= 1, <= max_seq_len).  Sequences of one client must be contiguous
  * (client-major packing).  T = sum(seq_len).  x_c, x_s: [T, d] bf16 (host or device).
  * On success *batch is a handle that owns the saved activations (or the x_c copy under NOGRAD) until
- * menos_backward or menos_batch_free.  ENOMEM if the arena cannot hold them (form smaller waves). */
+ * menos_backward or menos_batch_free.  ENOMEM if the arena cannot hold them (form smaller waves).
+ * NOGRAD with batch == NULL: nothing is retained after the call (Alg.1 L6-7: compute x_s without caching, then
+ * release GPU memory); the caller keeps x_c for the later re-forward ("we just need to cache the
+ * forward activations for the re-forward computation") and runs it as a SAVE forward + backward.  This is the
+ * mode the Alg.2 scheduler loop uses: a backward wave may group clients whose forwards ran in different waves.
+ * SAVE requires batch != NULL. */
 MENOS_API int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_client, const int32_t* seq_len, const void* x_c,
                   void* x_s, int flags, void* stream, menos_batch** batch);
 
@@ -209,6 +220,44 @@ MENOS_API unsigned long long menos_launch_count(void);
 
 MENOS_API int menos_sync(menos_server* s);
 MENOS_API const char* menos_last_error(void);
+
+/* ---------------------------------------------------------------------------------------------------------------
+ * Task scheduler: Algorithm 2 of PAPER.md:235-263 (§4.2), FCFS + backfilling over GPU memory (SURVEY.md §8(f)
+ * NEXT-2).  Host-only (no CUDA; usable without a GPU).  It decides which waiting requests enter the batched
+ * menos_forward / menos_backward calls: every SCHEDULE (one per event) returns a list of grants, and the caller
+ * runs the FWD grants of that list as one batched NOGRAD menos_forward (Alg.1 L6) and the BWD grants as one
+ * batched re-forward + menos_backward + menos_adapter_step (Alg.1 L10-12), then reports each client's completion.
+ *
+ *   menos_sched_create(M_avail)          Alg.2 L1, L3, L4 (M_avail = bytes the scheduler may hand out)
+ *   menos_sched_set_demand(i, M_f, M_b)  Alg.2 L2 (e.g. menos_batch_memory(..., MENOS_MEM_BOUND) of client i
+ *                                        alone: those figures are additive, so a batch of granted requests
+ *                                        never exceeds the memory the grants reserved)
+ *   menos_sched_arrive(i, kind)          Alg.2 L7-9: x_c (kind FWD) or g_c (kind BWD) of client i arrived
+ *   menos_sched_complete(i)              Alg.2 L10-13: client i's task finished and released A[i]
+ * Grants are written to out[0..*n_out) in the order they were made: the FCFS head first (L16-22), then the
+ * backfilled requests in waiting-list order (L23-24).  out must hold max_clients entries (EINVAL otherwise, with
+ * the scheduler state already updated).  Errors: ENOCLIENT (id out of range / no demands), ESTATE (the client
+ * already has a request waiting or running, or complete() without a running task), ENOMEM (a demand larger than
+ * M_avail at create: it could never be granted and would block the FCFS head forever; nothing is enqueued).
+ * Not thread-safe: one event at a time (the paper's scheduler is one event loop, Alg.2 L5-6). */
+typedef struct menos_sched menos_sched;
+enum { MENOS_REQ_FWD = 0, MENOS_REQ_BWD = 1 };
+typedef struct {
+  int32_t client;  /* serving process S_i                                 */
+  int32_t kind;    /* MENOS_REQ_FWD / MENOS_REQ_BWD                        */
+  size_t bytes;    /* memory reserved for it: M_f[i] or M_b[i] (A[i])     */
+} menos_sched_grant;
+MENOS_API int menos_sched_create(size_t m_avail, int max_clients, menos_sched** out);
+MENOS_API void menos_sched_destroy(menos_sched* s);
+MENOS_API int menos_sched_set_demand(menos_sched* s, int32_t client, size_t m_f, size_t m_b);
+MENOS_API int menos_sched_arrive(menos_sched* s, int32_t client, int kind, menos_sched_grant* out, int max_out,
+                                 int* n_out);
+MENOS_API int menos_sched_complete(menos_sched* s, int32_t client, menos_sched_grant* out, int max_out, int* n_out);
+/* current M_avail, |W|, number of running tasks, and the first max_waiting entries of W (may be NULL) */
+MENOS_API int menos_sched_state(menos_sched* s, size_t* m_avail, int* n_waiting, int* n_running, int32_t* waiting,
+                                int max_waiting);
+/* decision latency of SCHEDULE ("less than 0.1 milliseconds"): count, mean and max in ns */
+MENOS_API int menos_sched_timing(menos_sched* s, long long* decisions, double* mean_ns, double* max_ns);
 
 #ifdef __cplusplus
 }

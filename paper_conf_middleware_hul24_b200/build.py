@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OUT_DIR = os.path.join(HERE, "_lib")
 LIB = os.path.join(OUT_DIR, "libmenos.so")
-SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_ws.cu", "attention_bwd_tc.cu", "attention_bwd_ws.cu", "lora.cu", "elementwise.cu", "server.cu", "testing.cu"]
+SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_ws.cu", "attention_bwd_tc.cu", "attention_bwd_ws.cu", "lora.cu", "elementwise.cu", "server.cu", "testing.cu", "sched.cpp"]
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"),
@@ -37,7 +37,7 @@ def build(verbose: bool = False, force: bool = False) -> str:
     jobs = []
     for src in SOURCES:
         s = os.path.join(CSRC, src)
-        o = os.path.join(OUT_DIR, src.replace(".cu", ".o"))
+        o = os.path.join(OUT_DIR, os.path.splitext(src)[0] + ".o")
         if force or _stale(o, [s] + headers):
             jobs.append([NVCC, *FLAGS, "-c", s, "-o", o])
 
@@ -51,7 +51,7 @@ def build(verbose: bool = False, force: bool = False) -> str:
                 sys.stderr.write(r.stdout + r.stderr)
             if r.returncode:
                 raise RuntimeError(f"nvcc failed: {' '.join(cmd)}")
-    objs = [os.path.join(OUT_DIR, s.replace(".cu", ".o")) for s in SOURCES]
+    objs = [os.path.join(OUT_DIR, os.path.splitext(s)[0] + ".o") for s in SOURCES]
     if force or jobs or not os.path.exists(LIB):
         cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", LIB, *objs,
                "-Xcompiler", "-fPIC"]

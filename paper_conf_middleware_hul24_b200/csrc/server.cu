@@ -34,6 +34,17 @@ static void set_err(const char* fmt, ...) {
   tl_err = buf;
 }
 #define FAIL(code, ...) do { set_err(__VA_ARGS__); return (code); } while (0)
+namespace menos {
+// shared with sched.cpp (the Alg.2 scheduler reports through the same thread-local message)
+void set_last_error(const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  tl_err = buf;
+}
+}  // namespace menos
 #define CUDA_TRY(x)                                                                         \
   do {                                                                                      \
     cudaError_t e_ = (x);                                                                   \
@@ -751,9 +762,17 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
                                   int flags, size_t* fwd_bytes, size_t* bwd_bytes) {
   if (!s || n_clients < 0 || (n_clients > 0 && (!ids || !n_tokens))) FAIL(MENOS_EINVAL, "bad arguments");
   const Dims& D = s->D;
+  if (flags & ~(MENOS_FWD_NOGRAD | MENOS_MEM_BOUND)) FAIL(MENOS_EINVAL, "bad flags %d", flags);
   int R[NG] = {0, 0, 0, 0};
   bool save_a = false;
   long long T = 0;
+  if (flags & MENOS_MEM_BOUND) {   // additive bound: the registry-wide slot span and saved-tensor set
+    for (const Client& c : s->clients) {
+      if (!c.used) continue;
+      for (int g = 0; g < NG; ++g) if (c.width[g]) R[g] = std::max(R[g], c.col_off[g] + c.width[g]);
+      if (c.mask >> TD & 1) save_a = true;
+    }
+  }
   for (int i = 0; i < n_clients; ++i) {
     const int id = ids[i];
     if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
@@ -1478,9 +1497,10 @@ static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, floa
 // =====================================================================================================
 extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_client, const int32_t* seq_len,
                              const void* x_c, void* x_s, int flags, void* stream, menos_batch** batch) {
-  if (!s || !batch || n_seqs <= 0 || !seq_client || !seq_len || !x_c || !x_s) FAIL(MENOS_EINVAL, "bad arguments");
+  if (!s || n_seqs <= 0 || !seq_client || !seq_len || !x_c || !x_s) FAIL(MENOS_EINVAL, "bad arguments");
   if (flags != MENOS_FWD_SAVE && flags != MENOS_FWD_NOGRAD) FAIL(MENOS_EINVAL, "bad flags %d", flags);
-  *batch = nullptr;
+  if (!batch && flags != MENOS_FWD_NOGRAD) FAIL(MENOS_EINVAL, "batch == NULL requires MENOS_FWD_NOGRAD");
+  if (batch) *batch = nullptr;
   for (int l = 0; l < s->n_layers; ++l) if (!s->loaded[l]) FAIL(MENOS_ESTATE, "layer %d weights not loaded", l);
   CUDA_TRY(cudaSetDevice(s->device));
   cudaStream_t st = (cudaStream_t)stream;
@@ -1530,6 +1550,10 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
       pa.type != cudaMemoryTypeManaged)
     CUDA_TRY(cudaStreamSynchronize(st));
   cudaGetLastError();
+  if (!batch) {   // NOGRAD, nothing retained (Alg.1 L7): later arena allocations are stream-ordered after this call
+    fail_free(MENOS_OK);
+    return MENOS_OK;
+  }
   *batch = b.release();
   return MENOS_OK;
 }

@@ -15,6 +15,8 @@ LIB_PATH = os.path.join(HERE, "_lib", "libmenos.so")
 TARGET_BITS = {"q": 1, "k": 2, "v": 4, "o": 8, "gate": 16, "up": 32, "down": 64}
 TARGET_INDEX = {"q": 0, "k": 1, "v": 2, "o": 3, "gate": 4, "up": 5, "down": 6}
 FWD_SAVE, FWD_NOGRAD = 0, 1
+MEM_BOUND = 2
+REQ_FWD, REQ_BWD = 0, 1
 WHICH = {"A": 0, "B": 1, "dA": 2, "dB": 3, "mA": 4, "mB": 5, "vA": 6, "vB": 7}
 STATUS = {0: "OK", -1: "EINVAL", -2: "ENOMEM", -3: "ENOCLIENT", -4: "ESTATE", -5: "ECUDA", -6: "ENCCL"}
 
@@ -55,6 +57,10 @@ class Stats(C.Structure):
     _fields_ = [("base_bytes", C.c_size_t), ("adapters_bytes", C.c_size_t), ("arena_bytes", C.c_size_t),
                 ("arena_used", C.c_size_t), ("arena_peak", C.c_size_t), ("n_clients", C.c_int),
                 ("num_sms", C.c_int)]
+
+
+class SchedGrant(C.Structure):
+    _fields_ = [("client", C.c_int32), ("kind", C.c_int32), ("bytes", C.c_size_t)]
 
 
 class KernelStat(C.Structure):
@@ -100,6 +106,13 @@ SIGNATURES = {
     "menos_test_gemm_time": (_I, [_I, _I, _I, _I, _P, _P, _P, _I, _P, _I, C.POINTER(C.c_float)]),
     "menos_test_set_attn_tc": (_I, [_I]),
     "menos_testing_last_error": (C.c_char_p, []),
+    "menos_sched_create": (_I, [_S, _I, C.POINTER(_P)]),
+    "menos_sched_destroy": (None, [_P]),
+    "menos_sched_set_demand": (_I, [_P, C.c_int32, _S, _S]),
+    "menos_sched_arrive": (_I, [_P, C.c_int32, _I, C.POINTER(SchedGrant), _I, C.POINTER(_I)]),
+    "menos_sched_complete": (_I, [_P, C.c_int32, C.POINTER(SchedGrant), _I, C.POINTER(_I)]),
+    "menos_sched_state": (_I, [_P, C.POINTER(_S), C.POINTER(_I), C.POINTER(_I), _PI32, _I]),
+    "menos_sched_timing": (_I, [_P, C.POINTER(C.c_longlong), C.POINTER(C.c_double), C.POINTER(C.c_double)]),
 }
 
 
@@ -248,11 +261,12 @@ class Server:
                                       v.ctypes.data_as(C.POINTER(C.c_float))))
 
     # ---------------------------------------------------------------- the hot path
-    def forward(self, seq_client, seq_len, x_c, x_s, flags=FWD_SAVE, stream=None) -> Batch:
+    def forward(self, seq_client, seq_len, x_c, x_s, flags=FWD_SAVE, stream=None, retain=True) -> Batch | None:
+        """retain=False (NOGRAD only): nothing is kept after the call (Alg.1 L6-7); returns None."""
         b = C.c_void_p()
         check(lib().menos_forward(self.h, len(seq_client), _i32(seq_client), _i32(seq_len), ptr(x_c), ptr(x_s),
-                                  flags, _stream(stream), C.byref(b)))
-        return Batch(self, b.value, int(sum(seq_len)))
+                                  flags, _stream(stream), C.byref(b) if retain else None))
+        return Batch(self, b.value, int(sum(seq_len))) if retain else None
 
     def backward(self, batch: Batch, g_c, g_s, stream=None):
         check(lib().menos_backward(self.h, batch.handle, ptr(g_c), ptr(g_s), _stream(stream)))
@@ -289,3 +303,53 @@ def profile_read() -> dict:
     check(lib().menos_profile_read(arr, 16, C.byref(n)))
     return {arr[i].name.decode(): {"launches": arr[i].launches, "ms": arr[i].ms, "flops": arr[i].flops,
                                    "bytes": arr[i].bytes} for i in range(n.value)}
+
+
+class Scheduler:
+    """Algorithm 2: FCFS + backfilling over GPU memory; native (menos_sched_*)."""
+
+    def __init__(self, m_avail: int, max_clients: int = 64):
+        h = C.c_void_p()
+        check(lib().menos_sched_create(m_avail, max_clients, C.byref(h)))
+        self.h, self.max_clients = h.value, max_clients
+        self._out = (SchedGrant * max_clients)()
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().menos_sched_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def set_demand(self, client: int, m_f: int, m_b: int):
+        check(lib().menos_sched_set_demand(self.h, client, m_f, m_b))
+
+    def _grants(self, n):
+        return [(self._out[i].client, self._out[i].kind, self._out[i].bytes) for i in range(n.value)]
+
+    def arrive(self, client: int, kind: int) -> list[tuple[int, int, int]]:
+        """Alg.2 L7-9; returns the grants [(client, kind, bytes)] of the SCHEDULE call, in grant order."""
+        n = C.c_int()
+        check(lib().menos_sched_arrive(self.h, client, kind, self._out, self.max_clients, C.byref(n)))
+        return self._grants(n)
+
+    def complete(self, client: int) -> list[tuple[int, int, int]]:
+        """Alg.2 L10-13."""
+        n = C.c_int()
+        check(lib().menos_sched_complete(self.h, client, self._out, self.max_clients, C.byref(n)))
+        return self._grants(n)
+
+    def state(self) -> dict:
+        a, w, r = C.c_size_t(), C.c_int(), C.c_int()
+        buf = (C.c_int32 * self.max_clients)()
+        check(lib().menos_sched_state(self.h, C.byref(a), C.byref(w), C.byref(r), buf, self.max_clients))
+        return {"m_avail": a.value, "waiting": list(buf[:w.value]), "n_running": r.value}
+
+    def timing(self) -> dict:
+        n, mean, mx = C.c_longlong(), C.c_double(), C.c_double()
+        check(lib().menos_sched_timing(self.h, C.byref(n), C.byref(mean), C.byref(mx)))
+        return {"decisions": n.value, "mean_ns": mean.value, "max_ns": mx.value}
