@@ -1227,7 +1227,7 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   const Dims& D = s->D;
   const size_t need = scratch_bytes_of(D, T, R_used, nograd_set);
   const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
-  if (need > s->scratch_bytes) {
+  if (need != s->scratch_bytes) {   // shrink-to-fit too: a stale large block must not outlive the call that needed it
     if (s->scratch) s->arena.release(s->scratch);
     s->scratch = (uint8_t*)s->arena.alloc(need);
     if (!s->scratch) { s->scratch_bytes = 0; FAIL(MENOS_ENOMEM, "arena: scratch needs %zu B", need); }
