@@ -144,6 +144,14 @@ MENOS_API void menos_server_destroy(menos_server* s);
  * rank 1..max_rank; alpha > 0; target_mask != 0.  Returns ENOMEM when the registry is full. */
 MENOS_API int menos_register_client(menos_server* s, int rank, float alpha, uint32_t target_mask, const menos_adamw_cfg* opt,
                           uint64_t init_seed, int32_t* client_id);
+/* Per-client cut point (clients choose how many layers they keep): the client
+ * holds layers [0, cut_layer) itself and its tokens enter the server segment at ABSOLUTE layer cut_layer
+ * (first_layer <= cut_layer < first_layer + n_layers); menos_register_client == cut_layer = first_layer.  The
+ * client has adapters only for layers >= cut_layer (get/set_adapter below it: EINVAL); its x_c is the input of
+ * layer cut_layer and its g_s the gradient there.  In a batch, clients must come in non-decreasing cut order
+ * (EINVAL otherwise): layer l then runs on the prefix of tokens whose client has cut <= l. */
+MENOS_API int menos_register_client_at(menos_server* s, int cut_layer, int rank, float alpha, uint32_t target_mask,
+                                       const menos_adamw_cfg* opt, uint64_t init_seed, int32_t* client_id);
 MENOS_API int menos_unregister_client(menos_server* s, int32_t client_id);
 
 /* Closed-form memory demands (Alg.2 L2): persistent A+O bytes of the client, and the arena

@@ -193,6 +193,7 @@ struct Client {
   uint32_t mask = 0;
   menos_adamw_cfg opt{};
   int step = 0;
+  int cut = 0;                      // first server layer (local index) the client's tokens enter (NEXT-3)
   int col_off[NG] = {0, 0, 0, 0}, width[NG] = {0, 0, 0, 0};
   int sub[NT];                      // slot sub-offset of target t inside the group slot (j * rs), -1 if absent
   float* buf = nullptr;             // P | G | M | V, each n_params fp32
@@ -263,10 +264,17 @@ struct menos_batch {
   bool save_a = false;
   int n_mt = 0, n_blocks = 0, n_blocks128 = 0;
   int2* d_blocks128 = nullptr;
-  int4* d_attn_items = nullptr; int n_attn_items = 0;   // persistent attention work list (query blocks x heads)
-  int4* d_attn_items_kv = nullptr; int n_attn_items_kv = 0;   // key blocks x kv heads (dK/dV)
-  int4* d_attn_items_q = nullptr;                              // query blocks x heads, backward order (dQ)
   double pairs = 0;   // causal (query, key) pairs summed over sequences
+  // per-client cut points: the batch is ordered by non-decreasing cut, so
+  // the clients active at layer l (cut <= l) are a prefix: tokens [0, Tl[l]), sequences [0, nseq_l[l])
+  std::vector<int> Tl, nseq_l, view_of;
+  struct AttnView {
+    int n_seqs = 0, n_blocks = 0, n_blocks128 = 0, n_items = 0, n_items_kv = 0;
+    double pairs = 0;
+    size_t o_items = 0, o_items_kv = 0, o_items_q = 0;
+    int4 *items = nullptr, *items_kv = nullptr, *items_q = nullptr;
+  };
+  std::vector<AttnView> views;
   // device metadata
   uint8_t* meta = nullptr;  // arena
   int* d_cu = nullptr; int* d_pos = nullptr; int2* d_blocks = nullptr;
@@ -392,7 +400,7 @@ static int grow_group(menos_server* s, int g, int need_end) {
 // AdamW / refresh segments of one client (both A and B of every targeted (layer, target))
 static void client_segments(menos_server* s, const Client& c, int hyp_idx, std::vector<AdamSeg>& segs) {
   const Dims& D = s->D;
-  for (int l = 0; l < s->n_layers; ++l)
+  for (int l = c.cut; l < s->n_layers; ++l)
     for (int t = 0; t < NT; ++t) {
       if (!(c.mask >> t & 1)) continue;
       const int g = kTargetGroup[t];
@@ -610,7 +618,16 @@ static uint64_t splitmix(uint64_t& x) {
 
 extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uint32_t target_mask,
                                      const menos_adamw_cfg* opt, uint64_t init_seed, int32_t* client_id) {
+  if (!s) FAIL(MENOS_EINVAL, "null server");
+  return menos_register_client_at(s, s->first_layer, rank, alpha, target_mask, opt, init_seed, client_id);
+}
+
+extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank, float alpha, uint32_t target_mask,
+                                        const menos_adamw_cfg* opt, uint64_t init_seed, int32_t* client_id) {
   if (!s || !client_id) FAIL(MENOS_EINVAL, "null server/id");
+  if (cut_layer < s->first_layer || cut_layer >= s->first_layer + s->n_layers)
+    FAIL(MENOS_EINVAL, "cut layer %d outside the server segment [%d, %d)", cut_layer, s->first_layer,
+         s->first_layer + s->n_layers);
   if (rank < 1 || rank > s->opts.max_rank) FAIL(MENOS_EINVAL, "rank %d outside [1, %d]", rank, s->opts.max_rank);
   if (!(alpha > 0.f) || target_mask == 0 || (target_mask >> NT)) FAIL(MENOS_EINVAL, "bad alpha/target mask");
   CUDA_TRY(cudaSetDevice(s->device));
@@ -621,6 +638,7 @@ extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uin
   Client c;
   c.rank = rank; c.rs = (int)align_up(rank, 16); c.alpha = alpha; c.s = alpha / (float)rank; c.mask = target_mask;
   c.opt = opt ? *opt : menos_adamw_cfg{1e-4, 0.9, 0.999, 1e-8, 0.01};
+  c.cut = cut_layer - s->first_layer;
   for (int t = 0; t < NT; ++t) c.sub[t] = -1;
   int cnt[NG] = {0, 0, 0, 0};
   for (int t = 0; t < NT; ++t)
@@ -646,7 +664,7 @@ extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uin
   // split is immaterial
   size_t n = 0;
   for (int pass = 0; pass < 2; ++pass) {
-    for (int l = 0; l < s->n_layers; ++l)
+    for (int l = c.cut; l < s->n_layers; ++l)   // no adapters below the client's cut
       for (int t = 0; t < NT; ++t) {
         if (!(target_mask >> t & 1)) continue;
         if ((pass == 0) == D.a_rep[t]) { c.offA[l * NT + t] = (long long)n; n += (size_t)rank * D.K_t[t]; }
@@ -662,7 +680,7 @@ extern "C" int menos_register_client(menos_server* s, int rank, float alpha, uin
   uint64_t st = init_seed * 0x2545F4914F6CDD1Dull + 1;
   // the draw is over the GLOBAL [r, K] of every (layer, target) in the same order on every tensor-parallel
   // rank; a row-parallel rank keeps its column slice, so the shards assemble the world-1 A exactly
-  for (int l = 0; l < s->n_layers; ++l)
+  for (int l = c.cut; l < s->n_layers; ++l)
     for (int t = 0; t < NT; ++t) {
       if (!(target_mask >> t & 1)) continue;
       const int Kg = D.K_glob[t], Kl = D.K_t[t];
@@ -814,6 +832,7 @@ static int adapter_ptr(menos_server* s, int32_t id, int layer, int target, int w
     FAIL(MENOS_EINVAL, "bad layer/target/which");
   Client& c = s->clients[id];
   if (!(c.mask >> target & 1)) FAIL(MENOS_EINVAL, "target %d not in client mask", target);
+  if (layer < c.cut) FAIL(MENOS_EINVAL, "layer %d is below client %d's cut (no adapter there)", layer, id);
   const bool isB = which & 1;
   const long long off = isB ? c.offB[layer * NT + target] : c.offA[layer * NT + target];
   *n = (size_t)c.rank * (isB ? s->D.N_t[target] : s->D.K_t[target]);
@@ -950,6 +969,18 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   }
   b->T = b->cu.back();
   const int T = b->T;
+  // per-client cuts: clients must come in non-decreasing cut order; layer l sees the prefix of clients with cut <= l
+  b->Tl.assign(s->n_layers, 0);
+  b->nseq_l.assign(s->n_layers, 0);
+  for (size_t k = 0; k < b->bclients.size(); ++k) {
+    const int cut = s->clients[b->bclients[k]].cut;
+    if (k > 0 && cut < s->clients[b->bclients[k - 1]].cut)
+      FAIL(MENOS_EINVAL, "clients must be ordered by non-decreasing cut layer (client %d)", b->bclients[k]);
+  }
+  for (int i = 0; i < n_seqs; ++i) {
+    const int cut = s->clients[b->seq_client[i]].cut;
+    for (int l = cut; l < s->n_layers; ++l) { b->Tl[l] = b->cu[i + 1]; b->nseq_l[l] = i + 1; }
+  }
   // LoRA groups active in this batch and their used slot width
   for (int c : b->bclients) {
     const Client& cl = s->clients[c];
@@ -1028,13 +1059,30 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   for (int i = 0; i < b->n_seqs; ++i)
     for (int q = 0; q < b->seq_len[i]; q += 128) blocks128.push_back(make_int2(i, q));
   b->n_blocks128 = (int)blocks128.size();
-  std::vector<int4> attn_items;
-  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items, g_attn_order ? 1 : 0);
-  b->n_attn_items = (int)attn_items.size();
-  std::vector<int4> attn_items_kv, attn_items_q;
-  attn_ws_items(b->seq_len.data(), b->n_seqs, D.Hkv, attn_items_kv, g_attn_order ? 2 : 0);
-  attn_ws_items(b->seq_len.data(), b->n_seqs, D.H, attn_items_q, g_attn_order ? 1 : 0);
-  b->n_attn_items_kv = (int)attn_items_kv.size();
+  // one attention view (work lists over the first n sequences) per distinct active prefix
+  b->views.clear();
+  b->view_of.assign(Ls, -1);
+  std::vector<std::vector<int4>> v_items, v_items_kv, v_items_q;
+  for (int l = 0; l < Ls; ++l) {
+    const int ns = b->nseq_l[l];
+    if (ns == 0) continue;
+    if (!b->views.empty() && b->views.back().n_seqs == ns) { b->view_of[l] = (int)b->views.size() - 1; continue; }
+    menos_batch::AttnView v;
+    v.n_seqs = ns;
+    for (int i = 0; i < ns; ++i) {
+      v.n_blocks += ceil_div(b->seq_len[i], 64);
+      v.n_blocks128 += ceil_div(b->seq_len[i], 128);
+      v.pairs += 0.5 * (double)b->seq_len[i] * (b->seq_len[i] + 1);
+    }
+    v_items.emplace_back(); v_items_kv.emplace_back(); v_items_q.emplace_back();
+    attn_ws_items(b->seq_len.data(), ns, D.H, v_items.back(), g_attn_order ? 1 : 0);
+    attn_ws_items(b->seq_len.data(), ns, D.Hkv, v_items_kv.back(), g_attn_order ? 2 : 0);
+    attn_ws_items(b->seq_len.data(), ns, D.H, v_items_q.back(), g_attn_order ? 1 : 0);
+    v.n_items = (int)v_items.back().size();
+    v.n_items_kv = (int)v_items_kv.back().size();
+    b->views.push_back(v);
+    b->view_of[l] = (int)b->views.size() - 1;
+  }
   std::vector<int2> mt((size_t)NG * b->n_mt, make_int2(0, 0));
   for (int g = 0; g < NG; ++g) {
     if (!b->g_active[g]) continue;
@@ -1064,9 +1112,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_pos = put(b->pos.data(), b->pos.size() * 4);
   const size_t o_blk = put(blocks.data(), blocks.size() * sizeof(int2));
   const size_t o_blk128 = put(blocks128.data(), blocks128.size() * sizeof(int2));
-  const size_t o_items = put(attn_items.data(), attn_items.size() * sizeof(int4));
-  const size_t o_items_kv = put(attn_items_kv.data(), attn_items_kv.size() * sizeof(int4));
-  const size_t o_items_q = put(attn_items_q.data(), attn_items_q.size() * sizeof(int4));
+  for (size_t v = 0; v < b->views.size(); ++v) {
+    b->views[v].o_items = put(v_items[v].data(), v_items[v].size() * sizeof(int4));
+    b->views[v].o_items_kv = put(v_items_kv[v].data(), v_items_kv[v].size() * sizeof(int4));
+    b->views[v].o_items_q = put(v_items_q[v].data(), v_items_q[v].size() * sizeof(int4));
+  }
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
 
@@ -1136,7 +1186,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       std::vector<LoraTokRedProblem> db, da;
       for (size_t k = 0; k < b->bclients.size(); ++k) {
         const Client& c = s->clients[b->bclients[k]];
-        if (!c.width[g]) continue;
+        if (!c.width[g] || c.cut > l) continue;   // not yet in the segment at this layer
         const int t0 = b->btok_off[k], Tc = b->btok_n[k];
         for (int j0 = 0; j0 < c.width[g]; j0 += 128) {
           const int w = std::min(128, c.width[g] - j0);
@@ -1208,9 +1258,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   if (rc) return rc;
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
   b->d_blocks128 = (int2*)(meta + o_blk128);
-  b->d_attn_items = (int4*)(meta + o_items);
-  b->d_attn_items_kv = (int4*)(meta + o_items_kv);
-  b->d_attn_items_q = (int4*)(meta + o_items_q);
+  for (auto& v : b->views) {
+    v.items = (int4*)(meta + v.o_items);
+    v.items_kv = (int4*)(meta + v.o_items_kv);
+    v.items_q = (int4*)(meta + v.o_items_q);
+  }
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
   b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
@@ -1294,7 +1346,9 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
                          bool use_lists, cudaStream_t st) {
   const Dims& D = s->D;
   const auto& W = s->W[l];
-  const int T = b->T;
+  const int T = b->Tl[l];
+  if (T == 0) return MENOS_OK;
+  const menos_batch::AttnView& V = b->views[b->view_of[l]];
   // A1: RMSNorm1 (fp32 residual in, bf16 GEMM operand out)
   { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st)); }
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
@@ -1319,11 +1373,11 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     AttnArgs a;
     memset(&a, 0, sizeof a);
     a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
-    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
-    a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * b->pairs, 0, st);
-    if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, b->d_attn_items, b->n_attn_items, s->num_sms, st));
-    else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = V.n_blocks; a.kvblocks = b->d_blocks;
+    a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * V.pairs, 0, st);
+    if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, V.items, V.n_items, s->num_sms, st));
+    else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, V.n_blocks128, st));
     else K_TRY(attn_fwd(a, st));
   }
   // A4: O GEMM (+ LoRA o) + residual
@@ -1389,7 +1443,9 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   const Dims& D = s->D;
   const auto& W = s->W[l];
   const LayerSave& S = b->L[l];
-  const int T = b->T;
+  const int T = b->Tl[l];
+  if (T == 0) return MENOS_OK;
+  const menos_batch::AttnView& V = b->views[b->view_of[l]];
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
   if (b->g_active[GD]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GD], st));
   {
@@ -1446,14 +1502,14 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     AttnArgs a;
     memset(&a, 0, sizeof a);
     a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
-    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = b->n_blocks; a.kvblocks = b->d_blocks;
-    a.n_kvblocks = b->n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = V.n_blocks; a.kvblocks = b->d_blocks;
+    a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
     {
-      ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * b->pairs, 0, st);
+      ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * V.pairs, 0, st);
       if (D.hd == 128 && (g_attn_tc & 8))
-        K_TRY(attn_bwd_ws(a, b->d_attn_items_kv, b->n_attn_items_kv, b->d_attn_items_q, b->n_attn_items, s->num_sms, st));
-      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, b->n_blocks128, st));
+        K_TRY(attn_bwd_ws(a, V.items_kv, V.n_items_kv, V.items_q, V.n_items, s->num_sms, st));
+      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, V.n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
     }
   }
@@ -1482,11 +1538,24 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   return MENOS_OK;
 }
 
+// NEXT-3: the clients whose cut is layer l enter there -- their x_c rows [Tl[l-1], Tl[l]) (kept in
+// the fp32 copy L[0].x of the whole batch input) join the residual stream x that layer l reads
+static int join_rows(menos_server* s, menos_batch* b, int l, float* x, cudaStream_t st) {
+  if (l <= 0 || l >= s->n_layers) return MENOS_OK;
+  const int lo = b->Tl[l - 1], hi = b->Tl[l];
+  if (hi == lo || x == b->L[0].x) return MENOS_OK;
+  const size_t d = (size_t)s->D.d;
+  CUDA_TRY(cudaMemcpyAsync(x + lo * d, b->L[0].x + lo * d, (size_t)(hi - lo) * d * 4, cudaMemcpyDeviceToDevice, st));
+  return MENOS_OK;
+}
+
 // full SAVE forward over all layers: X[0] = b->L[0].x (already filled), output -> xout (fp32)
 static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, float* xout, cudaStream_t st) {
   for (int l = 0; l < s->n_layers; ++l) {
     float* y = (l + 1 < s->n_layers) ? b->L[l + 1].x : xout;
     int rc = layer_forward(s, b, l, b->L[l].x, y, b->L[l], true, st);
+    if (rc) return rc;
+    rc = join_rows(s, b, l + 1, y, st);
     if (rc) return rc;
   }
   return MENOS_OK;
@@ -1536,6 +1605,8 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     for (int l = 0; l < s->n_layers; ++l) {
       float* y = ((s->n_layers - 1 - l) % 2 == 0) ? sc.xout : sc.dxf;
       rc = layer_forward(s, b.get(), l, x, y, ng, true, st);
+      if (rc) return fail_free(rc);
+      rc = join_rows(s, b.get(), l + 1, y, st);
       if (rc) return fail_free(rc);
       x = y;
     }
@@ -1600,11 +1671,18 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
     if (b->g_active[g]) CUDA_TRY(cudaMemsetAsync(sc.dU[g], 0, (size_t)T * b->R_used[g] * 2, st));
   float* dyf = sc.dyf; bf16* dyb = sc.dyb;
   float* dxf = sc.dxf; bf16* dxb = sc.dxb;
+  const bool mixed_cuts = b->Tl[0] != T;
   for (int l = s->n_layers - 1; l >= 0; --l) {
     rc = layer_backward(s, b, l, dyf, dyb, dxf, dxb, sc, st);
     if (rc) return rc;
     std::swap(dyf, dxf);
     std::swap(dyb, dxb);
+    if (mixed_cuts) {   // NEXT-3: the clients whose cut is layer l leave here; dx rows [Tl[l-1], Tl[l]) are their g_s
+      const int lo = l > 0 ? b->Tl[l - 1] : 0, hi = b->Tl[l];
+      if (hi > lo)
+        CUDA_TRY(cudaMemcpyAsync(sc.io + (size_t)lo * D.d, dyb + (size_t)lo * D.d, (size_t)(hi - lo) * D.d * 2,
+                                 cudaMemcpyDeviceToDevice, st));
+    }
   }
   // A16: the replicated adapters' gradients (dA of column-parallel, dB of row-parallel targets) are partial
   // sums over the ranks' shards; one contiguous fp32 all-reduce per client
@@ -1613,7 +1691,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
       rc = tp_allreduce(s, s->clients[c].G(), s->clients[c].n_rep, MENOS_DT_F32, st);
       if (rc) return rc;
     }
-  CUDA_TRY(cudaMemcpyAsync(g_s, dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(g_s, mixed_cuts ? sc.io : dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
   cudaPointerAttributes pa;
   if (cudaPointerGetAttributes(&pa, g_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&
       pa.type != cudaMemoryTypeManaged)

@@ -79,6 +79,7 @@ SIGNATURES = {
     "menos_server_load_layer": (_I, [_P, _I, C.POINTER(LayerWeights)]),
     "menos_server_destroy": (None, [_P]),
     "menos_register_client": (_I, [_P, _I, _F, C.c_uint32, C.POINTER(AdamWCfg), C.c_uint64, _PI32]),
+    "menos_register_client_at": (_I, [_P, _I, _I, _F, C.c_uint32, C.POINTER(AdamWCfg), C.c_uint64, _PI32]),
     "menos_unregister_client": (_I, [_P, C.c_int32]),
     "menos_client_memory": (_I, [_P, C.c_int32, _I, C.POINTER(_S), C.POINTER(_S), C.POINTER(_S)]),
     "menos_batch_memory": (_I, [_P, _I, _PI32, _PI32, _I, C.POINTER(_S), C.POINTER(_S)]),
@@ -215,13 +216,18 @@ class Server:
 
     # ---------------------------------------------------------------- clients
     def register_client(self, rank, alpha, targets=("q", "v"), lr=1e-4, betas=(0.9, 0.999), eps=1e-8,
-                        weight_decay=0.01, seed=0) -> int:
+                        weight_decay=0.01, seed=0, cut_layer=None) -> int:
+        """cut_layer (absolute layer index, NEXT-3): where the client's tokens enter; None = the segment's first."""
         mask = 0
         for t in targets:
             mask |= TARGET_BITS[t]
         opt = AdamWCfg(lr, betas[0], betas[1], eps, weight_decay)
         cid = C.c_int32()
-        check(lib().menos_register_client(self.h, rank, alpha, mask, C.byref(opt), seed, C.byref(cid)))
+        if cut_layer is None:
+            check(lib().menos_register_client(self.h, rank, alpha, mask, C.byref(opt), seed, C.byref(cid)))
+        else:
+            check(lib().menos_register_client_at(self.h, cut_layer, rank, alpha, mask, C.byref(opt), seed,
+                                                 C.byref(cid)))
         return cid.value
 
     def unregister_client(self, cid: int):

@@ -47,8 +47,11 @@ def new_server(w: Workload, weights, arena_bytes=0, max_rank=16, device="cuda:0"
 def register(srv, w: Workload, adapters, seed=0):
     ids = []
     for i, c in enumerate(w.clients):
-        cid = srv.register_client(c.rank, c.alpha, c.targets, seed=seed + i)
+        cid = srv.register_client(c.rank, c.alpha, c.targets, seed=seed + i,
+                                  cut_layer=(w.model.first_layer + c.cut) if c.cut else None)
         for l, d in enumerate(adapters[i]):
+            if l < c.cut:
+                continue   # no adapters below the client's cut
             for t, (A, B) in d.items():
                 srv.set_adapter(cid, l, t, "A", A)
                 srv.set_adapter(cid, l, t, "B", B)
@@ -87,7 +90,7 @@ def run_gpu_step(w: Workload, seed: int = 0, zero_b: bool = False, flags: int = 
         off += T
         gr = []
         if grads:
-            for l in range(m.n_layers):
+            for l in range(c.cut, m.n_layers):   # the client's layers (grads index 0 = its cut layer)
                 gr.append({t: (srv.get_adapter(ids[i], l, t, "dA"), srv.get_adapter(ids[i], l, t, "dB"))
                            for t in c.targets})
         out["grads"].append(gr)
@@ -107,7 +110,10 @@ def run_oracle_step(w: Workload, seed: int = 0, zero_b: bool = False, inputs=Non
         if clients is not None and i not in clients:
             out["x_s"].append(None); out["g_s"].append(None); out["grads"].append(None)
             continue
-        xs, gs, gr = O.client_step(io[i][0], io[i][1], c.seq_lens, weights, adapters[i], c.alpha / c.rank, m)
+        # a client with cut k runs the segment [k, L): the same oracle on the layers it sends its tokens through
+        mc = m.with_layers(m.n_layers - c.cut) if c.cut else m
+        xs, gs, gr = O.client_step(io[i][0], io[i][1], c.seq_lens, weights[c.cut:], adapters[i][c.cut:],
+                                   c.alpha / c.rank, mc)
         out["x_s"].append(xs)
         out["g_s"].append(gs)
         out["grads"].append(gr)

@@ -332,3 +332,27 @@ def test_paper_memory_figures():
         me = O.memory_menos(M, AO, 0, I, N)
         assert me <= sb + 1e-9 and sb <= v + 1e-9
         assert abs(v - N * (M + AO + I)) < 1e-9 and abs(me - (M + N * AO + I)) < 1e-9
+
+
+def test_segment_composes_at_a_cut():
+    """NEXT-3: a client with cut k runs the oracle's segment [k, L).  Pin the meaning of x_c / g_s at
+    a cut by composition: f_[0,L) = f_[k,L) o f_[0,k), and g_s of [0,L) equals g_s of [0,k) driven by the g_s that
+    [k,L) returns (chain rule); the adapter grads of layers >= k are those of the shorter segment (fp64)."""
+    import dataclasses
+    m = dataclasses.replace(MODELS["tiny"], n_layers=3, n_kv_heads=2)
+    c = ClientCfg(4, 8.0, ("q", "v", "down"), [9, 5])
+    W = [base_layer_weights(m, l, seed=21) for l in range(3)]
+    ad = client_adapters(m, c, seed=22)
+    x, g = client_inputs(m, c, seed=23)
+    s = c.alpha / c.rank
+    xs, gs, gr = O.client_step(x, g, c.seq_lens, W, ad, s, m, F64)
+    k = 1
+    mid, gmid, grk = O.client_step(x, np.zeros_like(x), c.seq_lens, W[:k], ad[:k], s, m.with_layers(k), F64)
+    xs2, gk, gr2 = O.client_step(mid, g, c.seq_lens, W[k:], ad[k:], s, m.with_layers(3 - k), F64)
+    _, gs2, gr1 = O.client_step(x, gk, c.seq_lens, W[:k], ad[:k], s, m.with_layers(k), F64)
+    np.testing.assert_allclose(xs2, xs, rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(gs2, gs, rtol=1e-10, atol=1e-12)
+    for l in range(3 - k):
+        for t in c.targets:
+            np.testing.assert_allclose(gr2[l][t][0], gr[k + l][t][0], rtol=1e-10, atol=1e-13)
+            np.testing.assert_allclose(gr2[l][t][1], gr[k + l][t][1], rtol=1e-10, atol=1e-13)

@@ -77,6 +77,7 @@ class ClientCfg:
     alpha: float
     targets: tuple[str, ...]
     seq_lens: list[int] = field(default_factory=list)
+    cut: int = 0   # local index of the first server layer this client's tokens enter (NEXT-3; 0 = segment start)
 
     @property
     def n_tokens(self) -> int:
