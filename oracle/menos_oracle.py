@@ -256,29 +256,121 @@ def layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
     return dx, grads
 
 
+# ============================================================ OPT decoder layer (NEXT-4)
+# OPT-1.3B and up: pre-LayerNorm (do_layer_norm_before), biases on every projection, ReLU MLP, learned positions
+# added by the client's embedding layer (so no positional term in the server segment).  Reading R23.
+def layernorm_fwd(x, g, b, eps):
+    """y = (x - mu) rstd g + b, mu = mean(x), rstd = 1/sqrt(var(x) + eps) (biased variance), last axis."""
+    mu = np.mean(x, axis=-1, keepdims=True)
+    xc = x - mu
+    rstd = 1.0 / np.sqrt(np.mean(xc * xc, axis=-1, keepdims=True) + eps)
+    return xc * rstd * g + b, rstd
+
+
+def layernorm_bwd(dy, x, g, rstd):
+    """dx of layernorm_fwd (g, b frozen): xh = (x - mu) rstd, gh = dy g,
+    dx = rstd (gh - mean(gh) - xh mean(gh xh))."""
+    xh = (x - np.mean(x, axis=-1, keepdims=True)) * rstd
+    gh = dy * g
+    return rstd * (gh - np.mean(gh, axis=-1, keepdims=True) - xh * np.mean(gh * xh, axis=-1, keepdims=True))
+
+
+def opt_layer_fwd(x, W, lora, s, cfg, dtype=np.float32):
+    """One OPT decoder layer on ONE sequence x [S, d]:  xn = LN1(x);  q,k,v = xn W^T + b (+LoRA);
+    O = causal attn (scale hd^-1/2);  h = x + O Wo^T + bo (+LoRA);  hn = LN2(h);
+    a = relu(hn W1^T + b1 (+LoRA up));  y = h + a W2^T + b2 (+LoRA down)."""
+    S, d = x.shape
+    H, hd = cfg.n_heads, cfg.head_dim
+    Wd = {k: _cast(v, dtype) for k, v in W.items()}
+    L = {t: (_cast(a, dtype), _cast(b, dtype)) for t, (a, b) in lora.items()}
+    c = {"x": x}
+    eps = dtype(cfg.rms_eps)
+    xn, c["rstd1"] = layernorm_fwd(x, Wd["g1"], Wd["b1"], eps)
+    c["xn"] = xn
+    U = {}
+    qp, U["q"] = proj_fwd(xn, Wd["wq"], L.get("q"), s)
+    kp, U["k"] = proj_fwd(xn, Wd["wk"], L.get("k"), s)
+    vp, U["v"] = proj_fwd(xn, Wd["wv"], L.get("v"), s)
+    q = (qp + Wd["bq"]).reshape(S, H, hd)
+    k = (kp + Wd["bk"]).reshape(S, H, hd)
+    v = (vp + Wd["bv"]).reshape(S, H, hd)
+    O, c["lse"] = attention_fwd(q, k, v)
+    c["q"], c["k"], c["v"] = q, k, v
+    Of = O.reshape(S, H * hd)
+    c["O"] = Of
+    ao, U["o"] = proj_fwd(Of, Wd["wo"], L.get("o"), s)
+    h = x + ao + Wd["bo"]
+    c["h"] = h
+    hn, c["rstd2"] = layernorm_fwd(h, Wd["g2"], Wd["b2"], eps)
+    c["hn"] = hn
+    z, U["up"] = proj_fwd(hn, Wd["wup"], L.get("up"), s)
+    a = np.maximum(z + Wd["bup"], 0)
+    c["a"] = a
+    md, U["down"] = proj_fwd(a, Wd["wdown"], L.get("down"), s)
+    y = h + md + Wd["bdown"]
+    c["U"] = U
+    return y, c
+
+
+def opt_layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
+    """Backward of opt_layer_fwd in exact reverse order; dx and {target: (dA, dB)}, no base or bias gradient."""
+    S = dy.shape[0]
+    H, hd = cfg.n_heads, cfg.head_dim
+    Wd = {k: _cast(v, dtype) for k, v in W.items()}
+    L = {t: (_cast(a, dtype), _cast(b, dtype)) for t, (a, b) in lora.items()}
+    U = c["U"]
+    grads = {}
+    da, gd = proj_bwd(dy, c["a"], Wd["wdown"], L.get("down"), s, U["down"])
+    if gd is not None:
+        grads["down"] = gd
+    dz = da * (c["a"] > 0)
+    dhn, gu = proj_bwd(dz, c["hn"], Wd["wup"], L.get("up"), s, U["up"])
+    if gu is not None:
+        grads["up"] = gu
+    dh = dy + layernorm_bwd(dhn, c["h"], Wd["g2"], c["rstd2"])
+    dO, go = proj_bwd(dh, c["O"], Wd["wo"], L.get("o"), s, U["o"])
+    if go is not None:
+        grads["o"] = go
+    dq, dk, dv = attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
+    dxn = np.zeros_like(c["xn"])
+    for t, dt in (("q", dq), ("k", dk), ("v", dv)):
+        dxt, gt_ = proj_bwd(dt.reshape(S, H * hd), c["xn"], Wd["w" + t], L.get(t), s, U[t])
+        dxn = dxn + dxt
+        if gt_ is not None:
+            grads[t] = gt_
+    dx = dh + layernorm_bwd(dxn, c["x"], Wd["g1"], c["rstd1"])
+    return dx, grads
+
+
+def _layer_fns(cfg):
+    return (opt_layer_fwd, opt_layer_bwd) if getattr(cfg, "arch", "llama") == "opt" else (layer_fwd, layer_bwd)
+
+
 # ============================================================ server segment
 def segment_fwd_bwd(x_c, g_c, weights, adapters, s, cfg, dtype=np.float32):
     """One client's ONE sequence through all server layers: forward from x_c, then
     backward from g_c (Alg.1 L10-11).
     weights: list over layers of base dicts; adapters: list over layers of {t: (A,B)}.
     Returns x_s, g_s, grads (list over layers of {t: (dA, dB)})."""
+    fwd, bwd = _layer_fns(cfg)
     x = np.asarray(x_c, dtype=dtype)
     caches = []
     for ell in range(cfg.n_layers):
-        x, cache = layer_fwd(x, weights[ell], adapters[ell], dtype(s), cfg, dtype)
+        x, cache = fwd(x, weights[ell], adapters[ell], dtype(s), cfg, dtype)
         caches.append(cache)
     x_s = x
     dy = np.asarray(g_c, dtype=dtype)
     grads = [None] * cfg.n_layers
     for ell in reversed(range(cfg.n_layers)):
-        dy, grads[ell] = layer_bwd(dy, caches[ell], weights[ell], adapters[ell], dtype(s), cfg, dtype)
+        dy, grads[ell] = bwd(dy, caches[ell], weights[ell], adapters[ell], dtype(s), cfg, dtype)
     return x_s, dy, grads
 
 
 def segment_fwd(x_c, weights, adapters, s, cfg, dtype=np.float32):
+    fwd, _ = _layer_fns(cfg)
     x = np.asarray(x_c, dtype=dtype)
     for ell in range(cfg.n_layers):
-        x, _ = layer_fwd(x, weights[ell], adapters[ell], dtype(s), cfg, dtype)
+        x, _ = fwd(x, weights[ell], adapters[ell], dtype(s), cfg, dtype)
     return x
 
 

@@ -33,6 +33,7 @@ class ModelCfg:
     rms_eps: float = 1e-5
     rope_theta: float = 10000.0
     model_layers: int = 0    # decoder layers of the full model (0: first_layer + n_layers)
+    arch: str = "llama"      # "llama" (RMSNorm, RoPE, SwiGLU) or "opt" (LayerNorm+bias, biases, ReLU; NEXT-4)
 
     @property
     def head_dim(self) -> int:
@@ -50,6 +51,9 @@ class ModelCfg:
 MODELS = {
     # tiny: BASELINE.json configs[0]
     "tiny": ModelCfg("tiny", 64, 4, 4, 172, 2, model_layers=3),
+    # OPT (NEXT-4): tiny, and OPT-1.3B (d 2048, 32 heads, ffn 8192, 24 layers) [ext, HF config]
+    "opt_tiny": ModelCfg("opt-tiny", 64, 4, 4, 256, 2, model_layers=3, arch="opt"),
+    "opt1.3b": ModelCfg("opt-1.3b", 2048, 32, 32, 8192, 23, model_layers=24, arch="opt"),
     # Llama-2-7B / 13B / 70B server segments (layers 2..L, 1-indexed) [ext]
     "7b": ModelCfg("llama2-7b", 4096, 32, 32, 11008, 31, model_layers=32),
     "13b": ModelCfg("llama2-13b", 5120, 40, 40, 13824, 39, model_layers=40),
@@ -141,6 +145,16 @@ def base_layer_weights(cfg: ModelCfg, layer: int, seed: int = 0) -> dict[str, np
     for j, g in enumerate(["g1", "g2"]):
         r = _rng(seed, layer, 100 + j)
         out[g] = bf16_round(1.0 + 0.1 * r.standard_normal(cfg.d_model, dtype=np.float32))
+    if cfg.arch == "opt":
+        # OPT: no gate; biases of q, k, v, o, fc1 (up), fc2 (down) and the LayerNorm biases ~ 0.02 N(0,1), nonzero
+        # so that every bias path is exercised (trained OPT biases are nonzero)
+        del out["wgate"]
+        for j, t in enumerate(["q", "k", "v", "o", "up", "down"]):
+            r = _rng(seed, layer, 200 + j)
+            out["b" + t] = bf16_round(0.02 * r.standard_normal(target_dims(cfg, t)[1], dtype=np.float32))
+        for j, bname in enumerate(["b1", "b2"]):
+            r = _rng(seed, layer, 300 + j)
+            out[bname] = bf16_round(0.1 * r.standard_normal(cfg.d_model, dtype=np.float32))
     return out
 
 
