@@ -137,11 +137,16 @@ def build_server(torch, w, device, seed, arena_gb, tp=None):
     bytes)."""
     from paper_conf_middleware_hul24_b200 import Server
     m = w.model
-    if arena_gb is None or arena_gb <= 0:   # everything the base copy leaves, minus headroom
+    if arena_gb is None or arena_gb <= 0:   # everything the base copy and the clients' adapters leave, minus headroom
+        from workloads import target_dims
         free = torch.cuda.mem_get_info(device)[0]
         W = tp[1] if tp else 1
         P = m.n_layers * (2 * m.d_model * (m.n_heads + m.n_kv_heads) * m.head_dim + 3 * m.d_model * m.d_ff) // W
-        arena_gb = max(4.0, (free - 2 * P - (6 << 30)) / (1 << 30))
+        # A + O per client: fp32 p, g, m, v (16 B/param) + bf16 slot tables (A and B, rank padded to 16, tables
+        # grown by doubling: x2)
+        ao = sum(m.n_layers * sum(target_dims(m, t)[0] + target_dims(m, t)[1] for t in c.targets)
+                 * (16 * c.rank + 2 * 2 * (-(-c.rank // 16) * 16)) for c in w.clients) // W
+        arena_gb = max(4.0, (free - 2 * P - ao - (6 << 30)) / (1 << 30))
     srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
                  rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=None, device=device.index,
                  max_rank=16, max_seq_len=max(max(c.seq_lens) for c in w.clients),

@@ -61,9 +61,18 @@ typedef struct {
   int n_heads;     /* H                                  */
   int n_kv_heads;  /* H_kv (GQA when < H)                 */
   int d_ff;        /* f (SwiGLU inner size)               */
-  float rms_eps;   /* RMSNorm epsilon (1e-5)              */
-  float rope_theta;/* RoPE base (1e4)                     */
+  float rms_eps;   /* RMSNorm epsilon (1e-5); LayerNorm epsilon for OPT */
+  float rope_theta;/* RoPE base (1e4); unused for OPT      */
+  int arch;        /* MENOS_ARCH_LLAMA (0, default) or MENOS_ARCH_OPT (1)  */
 } menos_model_cfg;
+
+/* Model families (SURVEY.md §8(f) NEXT-4; PAPER.md:292, :294 evaluate Llama 2 and OPT):
+ *   LLAMA: pre-RMSNorm, RoPE, no biases, SwiGLU MLP (gate, up, down), GQA allowed.
+ *   OPT  : pre-LayerNorm (do_layer_norm_before, OPT-1.3B and up) with gain and bias, learned positions (on the
+ *          client: the embedding layer is client-side), biases on q, k, v, o, fc1, fc2, ReLU MLP
+ *          y = h + fc2(relu(fc1(LN2(h)))).  n_kv_heads must equal n_heads.  LoRA targets q, k, v, o, up (= fc1)
+ *          and down (= fc2); gate does not exist (EINVAL). */
+enum { MENOS_ARCH_LLAMA = 0, MENOS_ARCH_OPT = 1 };
 
 /* One decoder layer's frozen base weights, natural (HF) layouts, bf16 row-major, host or device.
  * The library COPIES them into its single device copy (WeightStore); the caller may free them after the
@@ -78,8 +87,18 @@ typedef struct {
   const void* wgate; /* [f, d]        */
   const void* wup;   /* [f, d]        */
   const void* wdown; /* [d, f]        */
-  const void* g1;    /* [d] input RMSNorm gain          */
-  const void* g2;    /* [d] post-attention RMSNorm gain */
+  const void* g1;    /* [d] input RMSNorm gain          (OPT: self_attn_layer_norm weight) */
+  const void* g2;    /* [d] post-attention RMSNorm gain (OPT: final_layer_norm weight)     */
+  /* OPT only (NULL for Llama): biases and LayerNorm biases, bf16.  wgate is NULL for OPT; wup = fc1 [f, d],
+   * wdown = fc2 [d, f]. */
+  const void* bq;    /* [H*hd] */
+  const void* bk;    /* [H*hd] */
+  const void* bv;    /* [H*hd] */
+  const void* bo;    /* [d]    */
+  const void* bup;   /* [f]  fc1 bias */
+  const void* bdown; /* [d]  fc2 bias */
+  const void* b1;    /* [d]  self_attn_layer_norm bias */
+  const void* b2;    /* [d]  final_layer_norm bias     */
 } menos_layer_weights;
 
 /* LoRA target projections (bit mask).  PAPER.md:294 uses q,v. */

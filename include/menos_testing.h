@@ -31,7 +31,7 @@ MENOS_API int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int 
 
 /* Varlen causal flash attention forward + backward (A3, A11) on a packed qkv [T, (H+2Hkv)hd] (q,k post-RoPE):
  * O [T, H*hd], lse [H, T] fp32; if dO != NULL also dqkv [T, (H+2Hkv)hd] = gradients w.r.t. the PRE-RoPE
- * q, k and v (RoPE backward with theta applied).  seq_len: host [n_seqs]. */
+ * q, k and v (RoPE backward with theta applied; theta <= 0: no RoPE, as for OPT).  seq_len: host [n_seqs]. */
 MENOS_API int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, int Hkv, int hd, const void* qkv, void* O,
                          float* lse, const void* dO, void* dqkv, float theta);
 

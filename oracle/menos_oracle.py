@@ -275,7 +275,27 @@ def layernorm_bwd(dy, x, g, rstd):
     return rstd * (gh - np.mean(gh, axis=-1, keepdims=True) - xh * np.mean(gh * xh, axis=-1, keepdims=True))
 
 
-def opt_layer_fwd(x, W, lora, s, cfg, dtype=np.float32):
+def _bf16(a):
+    """Round to the nearest bf16 (ties to even), returned as float32: the kernel's GEMM-operand precision."""
+    u = np.ascontiguousarray(a, dtype=np.float32).view(np.uint32)
+    u = (u + (np.uint32(0x7FFF) + ((u >> 16) & np.uint32(1)))) & np.uint32(0xFFFF0000)
+    return u.view(np.float32)
+
+
+def relu_decision(hn, Wup, bup, lora, s):
+    """Reading R25: the ReLU mask is a decision taken by floating point, so the oracle takes it in the
+    kernel's precision for that op -- bf16 GEMM operands (hn, and the LoRA shrink output U), fp32 accumulation, fp32
+    bias -- instead of on its own fp32 pre-activation (which differs by bf16 rounding and would flip the sign of
+    near-zero entries).  Returns the boolean mask [S, f]."""
+    hb = _bf16(hn)
+    z = hb @ np.asarray(Wup, np.float32).T
+    if lora is not None:
+        A, B = lora
+        z = z + _bf16(np.float32(s) * (hb @ np.asarray(A, np.float32).T)) @ np.asarray(B, np.float32).T
+    return (z + np.asarray(bup, np.float32)) > 0
+
+
+def opt_layer_fwd(x, W, lora, s, cfg, dtype=np.float32, relu_mask_bf16=False):
     """One OPT decoder layer on ONE sequence x [S, d]:  xn = LN1(x);  q,k,v = xn W^T + b (+LoRA);
     O = causal attn (scale hd^-1/2);  h = x + O Wo^T + bo (+LoRA);  hn = LN2(h);
     a = relu(hn W1^T + b1 (+LoRA up));  y = h + a W2^T + b2 (+LoRA down)."""
@@ -304,7 +324,12 @@ def opt_layer_fwd(x, W, lora, s, cfg, dtype=np.float32):
     hn, c["rstd2"] = layernorm_fwd(h, Wd["g2"], Wd["b2"], eps)
     c["hn"] = hn
     z, U["up"] = proj_fwd(hn, Wd["wup"], L.get("up"), s)
-    a = np.maximum(z + Wd["bup"], 0)
+    if relu_mask_bf16:
+        c["mask"] = relu_decision(hn, W["wup"], W["bup"], lora.get("up"), s)
+        a = (z + Wd["bup"]) * c["mask"]
+    else:
+        a = np.maximum(z + Wd["bup"], 0)
+        c["mask"] = a > 0
     c["a"] = a
     md, U["down"] = proj_fwd(a, Wd["wdown"], L.get("down"), s)
     y = h + md + Wd["bdown"]
@@ -323,7 +348,7 @@ def opt_layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
     da, gd = proj_bwd(dy, c["a"], Wd["wdown"], L.get("down"), s, U["down"])
     if gd is not None:
         grads["down"] = gd
-    dz = da * (c["a"] > 0)
+    dz = da * c["mask"]
     dhn, gu = proj_bwd(dz, c["hn"], Wd["wup"], L.get("up"), s, U["up"])
     if gu is not None:
         grads["up"] = gu
@@ -342,17 +367,19 @@ def opt_layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
     return dx, grads
 
 
-def _layer_fns(cfg):
-    return (opt_layer_fwd, opt_layer_bwd) if getattr(cfg, "arch", "llama") == "opt" else (layer_fwd, layer_bwd)
+def _layer_fns(cfg, relu_mask_bf16=False):
+    if getattr(cfg, "arch", "llama") == "opt":
+        return (lambda *a, **k: opt_layer_fwd(*a, **k, relu_mask_bf16=relu_mask_bf16)), opt_layer_bwd
+    return layer_fwd, layer_bwd
 
 
 # ============================================================ server segment
-def segment_fwd_bwd(x_c, g_c, weights, adapters, s, cfg, dtype=np.float32):
+def segment_fwd_bwd(x_c, g_c, weights, adapters, s, cfg, dtype=np.float32, relu_mask_bf16=False):
     """One client's ONE sequence through all server layers: forward from x_c, then
     backward from g_c (Alg.1 L10-11).
     weights: list over layers of base dicts; adapters: list over layers of {t: (A,B)}.
     Returns x_s, g_s, grads (list over layers of {t: (dA, dB)})."""
-    fwd, bwd = _layer_fns(cfg)
+    fwd, bwd = _layer_fns(cfg, relu_mask_bf16)
     x = np.asarray(x_c, dtype=dtype)
     caches = []
     for ell in range(cfg.n_layers):
@@ -374,14 +401,15 @@ def segment_fwd(x_c, weights, adapters, s, cfg, dtype=np.float32):
     return x
 
 
-def client_step(x_c, g_c, seq_lens, weights, adapters, s, cfg, dtype=np.float32):
+def client_step(x_c, g_c, seq_lens, weights, adapters, s, cfg, dtype=np.float32, relu_mask_bf16=False):
     """One client: its sequences run independently (positions restart at 0, reading R5);
     LoRA grads are summed over all of the client's tokens (backward overwrites, reading R10).
     x_c, g_c: [T_c, d] client-major packed.  Returns x_s, g_s [T_c, d], grads."""
     outs, gins, total = [], [], None
     off = 0
     for S in seq_lens:
-        xs, gs, gr = segment_fwd_bwd(x_c[off:off + S], g_c[off:off + S], weights, adapters, s, cfg, dtype)
+        xs, gs, gr = segment_fwd_bwd(x_c[off:off + S], g_c[off:off + S], weights, adapters, s, cfg, dtype,
+                                     relu_mask_bf16)
         outs.append(xs)
         gins.append(gs)
         if total is None:

@@ -333,7 +333,7 @@ __global__ void __launch_bounds__(128) attn_bwd_dkdv_kernel(const AttnArgs a) {
 #pragma unroll
     for (int e = 0; e < 4; ++e) dk[i][e] *= a.scale;
   const int p0 = min(kr0, L - 1), p1 = min(kr0 + 8, L - 1);
-  rope_bwd_frag<HD>(dk, a.rope_cs, p0 < 0 ? 0 : p0, p1 < 0 ? 0 : p1);
+  if (a.rope_cs) rope_bwd_frag<HD>(dk, a.rope_cs, p0 < 0 ? 0 : p0, p1 < 0 ? 0 : p1);   // none for OPT
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
     const int kr = kr0 + r * 8;
@@ -455,7 +455,7 @@ __global__ void __launch_bounds__(128) attn_bwd_dq_kernel(const AttnArgs a) {
 #pragma unroll
     for (int e = 0; e < 4; ++e) dq[i][e] *= a.scale;
   const int p0 = min(qr0, L - 1), p1 = min(qr0 + 8, L - 1);
-  rope_bwd_frag<HD>(dq, a.rope_cs, p0, p1);
+  if (a.rope_cs) rope_bwd_frag<HD>(dq, a.rope_cs, p0, p1);
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
     const int qr = qr0 + r * 8;

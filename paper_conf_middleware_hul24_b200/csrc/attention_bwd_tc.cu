@@ -340,7 +340,7 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     ew_sync();
     TR_C(2)
     const int nv = min(KV_ROWS, L - k0);
-    store_rows(stgK, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + kcol, p.ld_dqkv, p.rope_cs, true);
+    store_rows(stgK, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + kcol, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
     store_rows(stgV, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + vcol, p.ld_dqkv, p.rope_cs, false);
     TR_C(3)
     if (threadIdx.x == 64) { TR_PRINT("EW") }
@@ -500,7 +500,7 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     stage_acc(tdQ + lane_off, stg, r, g);
     ew_sync();
     const int nv = min(Q_ROWS, L - q0);
-    store_rows(stg, w8, lane, q0, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD, p.ld_dqkv, p.rope_cs, true);
+    store_rows(stg, w8, lane, q0, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
   }
   tc_fence_before();
   __syncthreads();

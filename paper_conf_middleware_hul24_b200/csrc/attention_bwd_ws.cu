@@ -123,6 +123,54 @@ __device__ __forceinline__ void acc_epilogue(uint32_t tacc_lane, uint8_t* stg, i
   }
 }
 
+// Single-round epilogue: every elementwise thread converts its TMEM row (columns [32g, 32g+32) and [64+32g, ..),
+// i.e. the RoPE pairs (j, j+64)) to bf16 in registers -- RoPE backward applied there -- and writes it into a bf16
+// staging tile [128 rows][256 B] (16-byte chunk k of row rr at rr*256 + ((k ^ (rr & 15)) << 4)); the TMEM
+// accumulator is released right after the loads, then all warps store whole rows (2 rows per instruction).
+// Same fp32 ops in the same order as the staged-fp32 path: the bf16 result is bitwise identical.
+__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const float2* cs,
+                                                int pos, bool rope) {
+  uint32_t a[32], b[32];
+  tmem_ld32_nw(tacc + 32 * g, a);
+  tmem_ld32_nw(tacc + 64 + 32 * g, b);
+  tmem_wait_ld();
+  float x[32], y[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
+  if (rope) {   // dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
+    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + 32 * g);
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      const float4 e = __ldg(c4 + i);   // (c_2i, s_2i, c_2i+1, s_2i+1)
+      const float x0 = x[2 * i] * e.x + y[2 * i] * e.y, y0 = y[2 * i] * e.x - x[2 * i] * e.y;
+      const float x1 = x[2 * i + 1] * e.z + y[2 * i + 1] * e.w, y1 = y[2 * i + 1] * e.z - x[2 * i + 1] * e.w;
+      x[2 * i] = x0; y[2 * i] = y0; x[2 * i + 1] = x1; y[2 * i + 1] = y1;
+    }
+  }
+  uint8_t* row = stg + rr * 256;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
+                                pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
+    const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
+                                pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
+    *reinterpret_cast<uint4*>(row + (((4 * g + c) ^ (rr & 15)) << 4)) = ux;
+    *reinterpret_cast<uint4*>(row + (((8 + 4 * g + c) ^ (rr & 15)) << 4)) = uy;
+  }
+}
+// n_tiles staged bf16 tiles (32 KB apart) -> rows [0, n_valid) of dst[t] (row stride ld), 16 lanes per 256-B row
+__device__ __forceinline__ void stage16_store(const uint8_t* stg, int n_tiles, int w8, int lane, int n_valid,
+                                              bf16* dst0, bf16* dst1, int ld) {
+  const int k = lane & 15;
+#pragma unroll 4
+  for (int i = 0; i < 8 * n_tiles; ++i) {
+    const int R = i * 16 + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
+    if (rr >= n_valid) continue;
+    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 32768 + rr * 256 + ((k ^ (rr & 15)) << 4));
+    *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * ld + k * 8) = v;
+  }
+}
+
 struct Geo { int base, L, blk0, head, n; };
 
 // -DMENOS_BWS_PROF: per-phase clock64 accounting (dK/dV kernel: one elementwise thread and the MMA lane)
@@ -365,11 +413,16 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       // all MMAs of this item completed: P^T / dS^T buffers are free for staging
       const int nv = min(KV_ROWS, L - k0);
       bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
-      acc_epilogue(tdK + lane_off, sP0, w4, w8, lane, g, nv, dst + (p.H + G.head) * HD, p.ld_dqkv, p.rope_cs, k0,
-                   true, &acc_free, false);
+      // P^T / dS^T buffers (64 KB, contiguous) = bf16 staging of dK | dV
+      acc_row_to_bf16(tdK + lane_off, sP0, r, g, p.rope_cs, k0 + r, p.rope_cs != nullptr && r < nv);
+      acc_row_to_bf16(tdV + lane_off, sP0 + 32768, r, g, nullptr, 0, false);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free);   // the next item's dK / dV accumulation may start
       BP(7);
-      acc_epilogue(tdV + lane_off, sP0, w4, w8, lane, g, nv, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv,
-                   p.rope_cs, k0, false, &acc_free, true);
+      ew_sync();
+      stage16_store(sP0, 2, w8, lane, nv, dst + (p.H + G.head) * HD, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv);
+      ew_sync();
       BP(8);
     }
     BP_FLUSH(blockIdx.x < 8 && t == 0);
@@ -554,8 +607,15 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       tc_fence_after();
       __syncwarp();
       const int nv = min(Q_ROWS, L - q0);
-      acc_epilogue(tdQ + lane_off, sS0, w4, w8, lane, g, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD,
-                   p.ld_dqkv, p.rope_cs, q0, true, &acc_free, true);
+      // dS buffers (32 KB) = bf16 staging of dQ
+      acc_row_to_bf16(tdQ + lane_off, sS0, r, g, p.rope_cs, q0 + r, p.rope_cs != nullptr && r < nv);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free);
+      ew_sync();
+      bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
+      stage16_store(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
+      ew_sync();
     }
   }
   tc_fence_before();

@@ -1,6 +1,7 @@
 // HBM-bound row kernels: RMSNorm fwd/bwd, attention-backward row sums
 // (A11 prologue), fused multi-tensor AdamW over all stepped clients' adapters (A13, Alg.1 L12),
 // RoPE table.  One warp per row, 16-byte vector loads, warp-shuffle fp32 reductions.
+#include <type_traits>
 #include "common.cuh"
 #include "kernels.h"
 
@@ -272,6 +273,101 @@ __global__ void bf16_to_f32_kernel(const bf16* __restrict__ s, float* __restrict
     d[i] = __bfloat162float(s[i]);
 }
 
+// ------------------------------------------------------------------ LayerNorm (OPT, NEXT-4)
+// One warp per row, the row cached in registers (NCH 8-element chunks per lane, d <= 256 * NCH), two-pass
+// statistics in fp32.  fwd: y = (x - mu) * rstd * g + b.  bwd (+ residual; g, b frozen so no dg, db):
+// dx = resid + rstd * (gh - mean(gh) - xh * mean(gh * xh)), gh = dy * g, xh = (x - mu) * rstd; mu and rstd are
+// recomputed from x with the forward's own reduction order.
+template <int NCH>
+__device__ __forceinline__ void ln_stats(const float (&v)[NCH][8], int lane, int d, float eps, float& mu, float& r) {
+  float s = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c)
+    if ((c * 32 + lane) * 8 < d)
+#pragma unroll
+      for (int k = 0; k < 8; ++k) s += v[c][k];
+  mu = warp_sum(s) / (float)d;
+  float q = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c)
+    if ((c * 32 + lane) * 8 < d)
+#pragma unroll
+      for (int k = 0; k < 8; ++k) { const float e = v[c][k] - mu; q += e * e; }
+  r = rsqrtf(warp_sum(q) / (float)d + eps);
+}
+
+template <int NCH>
+__global__ void layernorm_fwd_kernel(const float* __restrict__ x, const float* __restrict__ g,
+                                     const float* __restrict__ b, bf16* __restrict__ y, float* __restrict__ rstd,
+                                     int T, int d, float eps) {
+  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (row >= T) return;
+  const float* xr = x + (size_t)row * d;
+  float v[NCH][8];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int i = (c * 32 + lane) * 8;
+    if (i < d) ld8f(xr + i, v[c]);
+  }
+  float mu, r;
+  ln_stats<NCH>(v, lane, d, eps, mu, r);
+  if (lane == 0) rstd[row] = r;
+  bf16* yr = y + (size_t)row * d;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int i = (c * 32 + lane) * 8;
+    if (i >= d) continue;
+    float gg[8], bb[8], o[8];
+    ld8f(g + i, gg);
+    ld8f(b + i, bb);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) o[k] = (v[c][k] - mu) * r * gg[k] + bb[k];
+    st8b(yr + i, o);
+  }
+}
+
+template <int NCH, typename TDY>
+__global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
+                                     const float* __restrict__ g, const float* __restrict__ resid,
+                                     float* __restrict__ dx, bf16* __restrict__ dxb, int T, int d, float eps) {
+  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (row >= T) return;
+  const size_t ro = (size_t)row * d;
+  float v[NCH][8], gh[NCH][8];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int i = (c * 32 + lane) * 8;
+    if (i < d) {
+      ld8f(x + ro + i, v[c]);
+      float a[8], gg[8];
+      ld8(dy + ro + i, a);
+      ld8f(g + i, gg);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) gh[c][k] = a[k] * gg[k];
+    }
+  }
+  float mu, r;
+  ln_stats<NCH>(v, lane, d, eps, mu, r);
+  float sg = 0.f, sgx = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c)
+    if ((c * 32 + lane) * 8 < d)
+#pragma unroll
+      for (int k = 0; k < 8; ++k) { sg += gh[c][k]; sgx += gh[c][k] * (v[c][k] - mu) * r; }
+  const float mg = warp_sum(sg) / (float)d, mgx = warp_sum(sgx) / (float)d;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int i = (c * 32 + lane) * 8;
+    if (i >= d) continue;
+    float rr[8], o[8];
+    ld8f(resid + ro + i, rr);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) o[k] = rr[k] + r * (gh[c][k] - mg - (v[c][k] - mu) * r * mgx);
+    st8f(dx + ro + i, o);
+    if (dxb) st8b(dxb + ro + i, o);
+  }
+}
+
 }  // namespace
 
 #define LAUNCH_CHECK() (++g_launch_count, cudaPeekAtLastError() == cudaSuccess ? 0 : -3)
@@ -353,6 +449,42 @@ int convert_bf16_to_f32(const bf16* src, float* dst, long long n, cudaStream_t s
   if (n <= 0) return 0;
   bf16_to_f32_kernel<<<1024, 256, 0, st>>>(src, dst, n);
   return LAUNCH_CHECK();
+}
+
+
+// ------------------------------------------------------------------ LayerNorm launchers (OPT)
+template <typename F>
+static int ln_dispatch(int d, F&& f) {
+  const int nch = (d + 255) / 256;
+  if (nch <= 1) return f(std::integral_constant<int, 1>{});
+  if (nch <= 2) return f(std::integral_constant<int, 2>{});
+  if (nch <= 4) return f(std::integral_constant<int, 4>{});
+  if (nch <= 8) return f(std::integral_constant<int, 8>{});
+  if (nch <= 16) return f(std::integral_constant<int, 16>{});
+  return -1;
+}
+int layernorm_fwd(const float* x, const float* g, const float* b, bf16* y, float* rstd, int T, int d, float eps,
+                  cudaStream_t st) {
+  if (T <= 0) return 0;
+  if (d % 8) return -1;
+  return ln_dispatch(d, [&](auto n) {
+    layernorm_fwd_kernel<decltype(n)::value><<<(T + 7) / 8, 256, 0, st>>>(x, g, b, y, rstd, T, d, eps);
+    return LAUNCH_CHECK();
+  });
+}
+template <typename TDY>
+static int layernorm_bwd_t(const TDY* dy, const float* x, const float* g, const float* resid, float* dx, bf16* dxb,
+                           int T, int d, float eps, cudaStream_t st) {
+  if (T <= 0) return 0;
+  if (d % 8) return -1;
+  return ln_dispatch(d, [&](auto n) {
+    layernorm_bwd_kernel<decltype(n)::value, TDY><<<(T + 7) / 8, 256, 0, st>>>(dy, x, g, resid, dx, dxb, T, d, eps);
+    return LAUNCH_CHECK();
+  });
+}
+int layernorm_bwd(const bf16* dy, const float* x, const float* g, const float* resid, float* dx, bf16* dxb, int T,
+                  int d, float eps, cudaStream_t st) {
+  return layernorm_bwd_t(dy, x, g, resid, dx, dxb, T, d, eps, st);
 }
 
 }  // namespace menos

@@ -49,10 +49,21 @@ struct KParams {
   float* outf;
   bf16* out2; int ldo2;
   const bf16* aux; int ldaux;
+  const float* bias;
   const float2* rope_cs;
   const int* pos;
   int head_dim, rope_cols;
 };
+
+// v[j] += bias[col + j] (fp32, 32 consecutive columns; col % 32 == 0)
+__device__ __forceinline__ void add_bias32(float (&v)[32], const float* bias, int col) {
+  const float4* b4 = reinterpret_cast<const float4*>(bias + col);
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const float4 b = __ldg(b4 + q);
+    v[4 * q] += b.x; v[4 * q + 1] += b.y; v[4 * q + 2] += b.z; v[4 * q + 3] += b.w;
+  }
+}
 
 __device__ __forceinline__ void store32(bf16* dst, const float (&v)[32]) {
   uint4* d = reinterpret_cast<uint4*>(dst);
@@ -272,7 +283,33 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (col >= p.N) break;
           float v[32];
           tmem_ld32(tb + c * 32, v);
+          if (p.bias) add_bias32(v, p.bias, col);
           if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
+        }
+      } else if (p.epi == EPI_RELU_FWD) {
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          if (p.bias) add_bias32(v, p.bias, col);
+#pragma unroll
+          for (int j = 0; j < 32; ++j) v[j] = fmaxf(v[j], 0.f);
+          if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
+        }
+      } else if (p.epi == EPI_RELU_BWD) {
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          if (rok) {
+            float a[32];
+            load32(p.aux + (size_t)row * p.ldaux + col, a);
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = a[j] > 0.f ? v[j] : 0.f;
+            store32(p.out + (size_t)row * p.ldo + col, v);
+          }
         }
       } else if (p.epi == 99 || p.epi == 98) {
         // tuning aid: drain TMEM without storing (isolates the mainloop)
@@ -284,25 +321,34 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         }
         if (sink == 12345.678f) p.out[0] = f2bf(sink);
       } else if (p.epi == EPI_RESID) {
-        // fp32 residual stream: outf = acc + resid
+        // fp32 residual stream: outf = acc (+ bias) + resid.  The chunk's 8 residual loads are all issued before
+        // the TMEM load and before any store: outf and resid may alias as far as the compiler knows, so loads
+        // interleaved with the stores would serialise into 8 HBM round trips per chunk.
         for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
+          float r[32];
+          const bool has_r = rok && p.resid;
+          if (has_r) {
+            const float4* r4 = reinterpret_cast<const float4*>(p.resid + (size_t)row * p.ldr + col);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const float4 x = __ldg(r4 + q);
+              r[4 * q] = x.x; r[4 * q + 1] = x.y; r[4 * q + 2] = x.z; r[4 * q + 3] = x.w;
+            }
+          } else {   // tensor-parallel partial sum (the residual is added by rank 0 only)
+#pragma unroll
+            for (int j = 0; j < 32; ++j) r[j] = 0.f;
+          }
           float v[32];
           tmem_ld32(tb + c * 32, v);
+          if (p.bias) add_bias32(v, p.bias, col);
           if (rok) {
             float4* o4 = reinterpret_cast<float4*>(p.outf + (size_t)row * p.ldo + col);
-            if (p.resid) {
-              const float4* r4 = reinterpret_cast<const float4*>(p.resid + (size_t)row * p.ldr + col);
 #pragma unroll
-              for (int q = 0; q < 8; ++q) {
-                const float4 r = r4[q];
-                o4[q] = make_float4(v[4 * q] + r.x, v[4 * q + 1] + r.y, v[4 * q + 2] + r.z, v[4 * q + 3] + r.w);
-              }
-            } else {   // tensor-parallel partial sum (the residual is added by rank 0 only)
-#pragma unroll
-              for (int q = 0; q < 8; ++q) o4[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-            }
+            for (int q = 0; q < 8; ++q)
+              o4[q] = make_float4(v[4 * q] + r[4 * q], v[4 * q + 1] + r[4 * q + 1], v[4 * q + 2] + r[4 * q + 2],
+                                  v[4 * q + 3] + r[4 * q + 3]);
           }
         }
       } else if (p.epi == EPI_ROPE) {
@@ -523,7 +569,7 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   p.M = a.M; p.N = a.N; p.K = a.K; p.kb_main = (a.K + BK - 1) / BK;
   p.R = a.R; p.mtile_extra = a.mtile_extra; p.ntile_extra = a.ntile_extra;
   p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr; p.outf = a.outf;
-  p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux;
+  p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux; p.bias = a.bias;
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
   const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);
   int sms = a.num_sms > 0 ? a.num_sms : 148;

@@ -21,6 +21,9 @@ enum EpiMode : int {
   EPI_ROPE = 2,        // columns < rope_cols rotated by RoPE at pos[row]; out = bf16
   EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu), out2 = bf16(silu(g) u)
   EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
+  EPI_RELU_FWD = 5,    // OPT fc1: out = bf16(relu(acc + bias))
+  EPI_RELU_BWD = 6,    // OPT fc2 dX: out = bf16(acc * (aux > 0)), aux = saved relu output
+  // EPI_STORE and EPI_RESID add `bias[col]` (fp32) when bias != nullptr (OPT projections)
 };
 
 struct GemmArgs {
@@ -40,7 +43,8 @@ struct GemmArgs {
   const float* resid; int ldr;     // EPI_RESID: fp32 residual in, fp32 `outf` out (ld = ldo)
   float* outf;
   bf16* out2; int ldo2;            // EPI_SWIGLU_FWD: a
-  const bf16* aux; int ldaux;      // EPI_SWIGLU_BWD: saved gu
+  const bf16* aux; int ldaux;      // EPI_SWIGLU_BWD: saved gu; EPI_RELU_BWD: saved relu output
+  const float* bias;               // [N] fp32 or nullptr (EPI_STORE, EPI_RESID, EPI_RELU_FWD)
   const float2* rope_cs;           // EPI_ROPE: [max_pos][hd/2] (cos, sin)
   const int* pos;                  // EPI_ROPE: per-row position
   int head_dim, rope_cols;
@@ -72,6 +76,12 @@ void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, st
 // ---------------------------------------------------------------- norms / elementwise
 // residual streams (x, h forward; dy, dh backward) are fp32; GEMM operands (xn, hn, dxn ...) are bf16
 int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st);
+// LayerNorm (OPT, NEXT-4): y = (x - mu) rstd g + b (bf16 out, rstd saved); bwd recomputes mu, rstd from x:
+// dx = resid + rstd (gh - mean(gh) - xh mean(gh xh)), gh = dy g; dxb = optional bf16 copy
+int layernorm_fwd(const float* x, const float* g, const float* b, bf16* y, float* rstd, int T, int d, float eps,
+                  cudaStream_t st);
+int layernorm_bwd(const bf16* dy, const float* x, const float* g, const float* resid, float* dx, bf16* dxb, int T,
+                  int d, float eps, cudaStream_t st);
 // dx = resid + rstd*(gh - xh*mean(gh*xh)), gh = dy*g, xh = x*rstd; dxb (optional) = bf16(dx)
 int rmsnorm_bwd(const bf16* dy, const float* x, const float* g, const float* rstd, const float* resid, float* dx,
                 bf16* dxb, int T, int d, cudaStream_t st);

@@ -105,6 +105,8 @@ static const int kTargetGroup[NT] = {GQKV, GQKV, GQKV, GO, GGU, GGU, GD};
 struct Dims {
   // local (per tensor-parallel rank) extents: H, Hkv, f are the global ones / tp_world
   int d, H, Hkv, hd, f, fpad, Nq, Nkv, Nqkv;
+  int arch;                        // MENOS_ARCH_LLAMA / MENOS_ARCH_OPT (NEXT-4)
+  int gu_cols;                     // columns of the saved MLP activation: [gate|up] 2*fpad (Llama), relu(fc1) fpad (OPT)
   int tp_rank, tp_world;
   int K_glob[NT];                  // global input dim of each projection (LoRA A init bound, A slicing)
   bool a_rep[NT];                  // A replicated across ranks (column-parallel); else B replicated (row-parallel)
@@ -122,6 +124,9 @@ static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 
   D.f = c.d_ff / tp_world; D.fpad = (int)align_up(D.f, 128);
   D.Nq = D.H * D.hd; D.Nkv = D.Hkv * D.hd; D.Nqkv = D.Nq + 2 * D.Nkv;
   D.eps = c.rms_eps; D.theta = c.rope_theta;
+  D.arch = c.arch;
+  const bool opt = c.arch == MENOS_ARCH_OPT;
+  D.gu_cols = opt ? D.fpad : 2 * D.fpad;
   const int K[NT] = {D.d, D.d, D.d, D.Nq, D.d, D.d, D.f};
   const int N[NT] = {D.Nq, D.Nkv, D.Nkv, D.d, D.f, D.f, D.d};
   for (int t = 0; t < NT; ++t) {
@@ -131,12 +136,13 @@ static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 
   }
   D.K_g[GQKV] = D.d;  D.N_g[GQKV] = D.Nqkv;    D.ldK_g[GQKV] = D.d;
   D.K_g[GO] = D.Nq;   D.N_g[GO] = D.d;         D.ldK_g[GO] = D.Nq;
-  D.K_g[GGU] = D.d;   D.N_g[GGU] = 2 * D.fpad; D.ldK_g[GGU] = D.d;
+  D.K_g[GGU] = D.d;   D.N_g[GGU] = D.gu_cols;  D.ldK_g[GGU] = D.d;
   D.K_g[GD] = D.f;    D.N_g[GD] = D.d;         D.ldK_g[GD] = D.fpad;
   const int big = 1 << 30;
   int base[NT] = {0, D.Nq, D.Nq + D.Nkv, 0, 0, 128, 0};
   int blk[NT] = {big, big, big, big, 128, 128, big};
   int str[NT] = {0, 0, 0, 0, 256, 256, 0};
+  if (opt) { base[TU] = 0; blk[TU] = big; str[TU] = 0; }   // fc1 rows, not interleaved (gate does not exist)
   for (int t = 0; t < NT; ++t) { D.rb_base[t] = base[t]; D.rb_blk[t] = blk[t]; D.rb_stride[t] = str[t]; }
   return D;
 }
@@ -300,7 +306,11 @@ struct menos_server {
   menos_tp_cfg tp{0, 1, nullptr, nullptr};  // tensor parallelism (world 1 = replica)
   // WeightStore: one bf16 copy of every server layer, packed for the kernels
   uint8_t* wbuf = nullptr; size_t wbytes = 0;
-  struct LW { bf16 *wqkv, *wo, *wgu, *wd; float *g1, *g2; };
+  struct LW {
+    bf16 *wqkv, *wo, *wgu, *wd;
+    float *g1, *g2;
+    float *be1, *be2, *bqkv, *bo, *bu, *bd;   // OPT: LayerNorm biases, projection biases (fp32; zero for Llama)
+  };
   std::vector<LW> W;
   std::vector<bool> loaded;
   // LoRA slot tables per layer per group (bf16): Bcat [N_g, cap], Acat [cap, ldK_g]
@@ -328,13 +338,47 @@ struct menos_server {
 // =====================================================================================================
 // helpers: weights
 // =====================================================================================================
+// OPT (NEXT-4): q|k|v, o as for Llama; fc1 -> wgu [fpad, d] (rows >= f zero), fc2 -> wd [d, fpad]; LayerNorm gains
+// and biases and the projection biases -> fp32
+static int upload_layer_opt(menos_server* s, int l, const menos_layer_weights* w) {
+  const Dims& D = s->D;
+  auto& L = s->W[l];
+  const size_t b2 = 2;
+  cudaStream_t st = 0;
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv, w->wq, (size_t)D.Nq * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)D.Nq * D.d, w->wk, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)(D.Nq + D.Nkv) * D.d, w->wv, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wo, w->wo, (size_t)D.d * D.Nq * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpyAsync(L.wgu, w->wup, (size_t)D.f * D.d * b2, cudaMemcpyDefault, st));
+  CUDA_TRY(cudaMemcpy2DAsync(L.wd, (size_t)D.fpad * b2, w->wdown, (size_t)D.f * b2, (size_t)D.f * b2, D.d,
+                             cudaMemcpyDefault, st));
+  struct V { const void* src; float* dst; int n; };
+  const V vs[] = {{w->g1, L.g1, D.d}, {w->g2, L.g2, D.d}, {w->b1, L.be1, D.d}, {w->b2, L.be2, D.d},
+                  {w->bo, L.bo, D.d}, {w->bdown, L.bd, D.d}, {w->bq, L.bqkv, D.Nq}, {w->bk, L.bqkv + D.Nq, D.Nkv},
+                  {w->bv, L.bqkv + D.Nq + D.Nkv, D.Nkv}, {w->bup, L.bu, D.f}};
+  bf16* tmp = nullptr;
+  CUDA_TRY(cudaMalloc(&tmp, (size_t)std::max(D.Nqkv, D.fpad) * b2));
+  for (const V& v : vs) {
+    CUDA_TRY(cudaMemcpyAsync(tmp, v.src, (size_t)v.n * b2, cudaMemcpyDefault, st));
+    K_TRY(convert_bf16_to_f32(tmp, v.dst, v.n, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+  }
+  CUDA_TRY(cudaFree(tmp));
+  s->loaded[l] = true;
+  return MENOS_OK;
+}
+
 static int upload_layer(menos_server* s, int l, const menos_layer_weights* w) {
   const Dims& D = s->D;
   auto& L = s->W[l];
   const size_t b2 = 2;
-  if (!w || !w->wq || !w->wk || !w->wv || !w->wo || !w->wgate || !w->wup || !w->wdown || !w->g1 || !w->g2)
+  const bool opt = D.arch == MENOS_ARCH_OPT;
+  if (!w || !w->wq || !w->wk || !w->wv || !w->wo || (!opt && !w->wgate) || !w->wup || !w->wdown || !w->g1 || !w->g2)
     FAIL(MENOS_EINVAL, "layer %d: null weight pointer", l);
+  if (opt && (!w->bq || !w->bk || !w->bv || !w->bo || !w->bup || !w->bdown || !w->b1 || !w->b2))
+    FAIL(MENOS_EINVAL, "layer %d: OPT needs every bias", l);
   cudaStream_t st = 0;
+  if (opt) return upload_layer_opt(s, l, w);
   CUDA_TRY(cudaMemcpyAsync(L.wqkv, w->wq, (size_t)D.Nq * D.d * b2, cudaMemcpyDefault, st));
   CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)D.Nq * D.d, w->wk, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
   CUDA_TRY(cudaMemcpyAsync(L.wqkv + (size_t)(D.Nq + D.Nkv) * D.d, w->wv, (size_t)D.Nkv * D.d * b2, cudaMemcpyDefault, st));
@@ -511,6 +555,9 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
   const int hd = cfg->d_model / cfg->n_heads;
   if (hd != 16 && hd != 32 && hd != 64 && hd != 128) FAIL(MENOS_EINVAL, "head_dim %d unsupported (16/32/64/128)", hd);
   if (cfg->d_model % 64) FAIL(MENOS_EINVAL, "d_model must be a multiple of 64");
+  if (cfg->arch != MENOS_ARCH_LLAMA && cfg->arch != MENOS_ARCH_OPT) FAIL(MENOS_EINVAL, "unknown arch %d", cfg->arch);
+  if (cfg->arch == MENOS_ARCH_OPT && cfg->n_kv_heads != cfg->n_heads) FAIL(MENOS_EINVAL, "OPT has no GQA");
+  if (cfg->arch == MENOS_ARCH_OPT && opts && opts->tp.world > 1) FAIL(MENOS_EINVAL, "tensor parallelism is Llama-only");
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) FAIL(MENOS_ECUDA, "no CUDA device %d", device);
   cudaDeviceProp prop;
@@ -540,8 +587,9 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
 
   // WeightStore: one allocation for all layers (a single preloaded copy)
   const size_t per = align_up((size_t)D.Nqkv * D.d * 2, 256) + align_up((size_t)D.d * D.Nq * 2, 256) +
-                     align_up((size_t)2 * D.fpad * D.d * 2, 256) + align_up((size_t)D.d * D.fpad * 2, 256) +
-                     2 * align_up((size_t)D.d * 4, 256);
+                     align_up((size_t)D.gu_cols * D.d * 2, 256) + align_up((size_t)D.d * D.fpad * 2, 256) +
+                     6 * align_up((size_t)D.d * 4, 256) + align_up((size_t)D.Nqkv * 4, 256) +   // g1 g2 be1 be2 bo bd
+                     align_up((size_t)D.fpad * 4, 256);
   s->wbytes = per * n_layers;
   if (cudaMalloc(&s->wbuf, s->wbytes) != cudaSuccess) { cudaGetLastError(); FAIL(MENOS_ENOMEM, "weight store (%zu B)", s->wbytes); }
   CUDA_TRY(cudaMemset(s->wbuf, 0, s->wbytes));
@@ -552,10 +600,16 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
     auto& L = s->W[l];
     L.wqkv = (bf16*)p; p += align_up((size_t)D.Nqkv * D.d * 2, 256);
     L.wo = (bf16*)p; p += align_up((size_t)D.d * D.Nq * 2, 256);
-    L.wgu = (bf16*)p; p += align_up((size_t)2 * D.fpad * D.d * 2, 256);
+    L.wgu = (bf16*)p; p += align_up((size_t)D.gu_cols * D.d * 2, 256);
     L.wd = (bf16*)p; p += align_up((size_t)D.d * D.fpad * 2, 256);
     L.g1 = (float*)p; p += align_up((size_t)D.d * 4, 256);
-    L.g2 = (float*)p;
+    L.g2 = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.be1 = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.be2 = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.bo = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.bd = (float*)p; p += align_up((size_t)D.d * 4, 256);
+    L.bqkv = (float*)p; p += align_up((size_t)D.Nqkv * 4, 256);
+    L.bu = (float*)p;
   }
   for (int g = 0; g < NG; ++g) { s->Bcat[g].assign(n_layers, nullptr); s->Acat[g].assign(n_layers, nullptr); }
   CUDA_TRY(cudaMalloc(&s->rope, (size_t)o.max_seq_len * (D.hd / 2) * sizeof(float2)));
@@ -630,6 +684,7 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
          s->first_layer + s->n_layers);
   if (rank < 1 || rank > s->opts.max_rank) FAIL(MENOS_EINVAL, "rank %d outside [1, %d]", rank, s->opts.max_rank);
   if (!(alpha > 0.f) || target_mask == 0 || (target_mask >> NT)) FAIL(MENOS_EINVAL, "bad alpha/target mask");
+  if (s->D.arch == MENOS_ARCH_OPT && (target_mask >> TG & 1)) FAIL(MENOS_EINVAL, "OPT has no gate projection");
   CUDA_TRY(cudaSetDevice(s->device));
   int id = -1;
   for (size_t i = 0; i < s->clients.size(); ++i) if (!s->clients[i].used) { id = (int)i; break; }
@@ -731,7 +786,7 @@ static size_t saved_bytes_per_token_layer(const Dims& D, bool save_a) {
   b += (size_t)D.d * 2 * 2;        // xn, hn
   b += (size_t)D.Nqkv * 2;         // qkv
   b += (size_t)D.Nq * 2;           // O
-  b += (size_t)2 * D.fpad * 2;     // gu
+  b += (size_t)D.gu_cols * 2;      // gu (OPT: relu(fc1))
   if (save_a) b += (size_t)D.fpad * 2;
   b += 4 * 2 + (size_t)D.H * 4;    // rstd1, rstd2, lse
   return b;
@@ -742,7 +797,7 @@ static size_t scratch_bytes_per_token(const Dims& D, int R_sum) {
   b += (size_t)D.d * 2 * 5;          // dyb, dxb, dhb, dhn, io staging (bf16)
   b += (size_t)D.Nq * 2;             // dO
   b += (size_t)D.Nqkv * 2;           // dqkv
-  b += (size_t)2 * D.fpad * 2;       // dgu
+  b += (size_t)D.gu_cols * 2;        // dgu
   b += (size_t)D.fpad * 2;           // a (when not saved)
   b += (size_t)D.H * 4;              // D rowsums
   b += (size_t)R_sum * 2;            // dU
@@ -761,7 +816,7 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
   size_t slots = 0;
   for (int g = 0; g < NG; ++g) slots += (size_t)c.width[g] * (D.N_g[g] + D.ldK_g[g]) * 2 * s->n_layers;
   if (persistent) *persistent = 16 * c.n_params + slots;
-  const bool save_a = (c.mask >> TD) & 1;
+  const bool save_a = ((c.mask >> TD) & 1) && D.arch != MENOS_ARCH_OPT;
   size_t ush = 0;
   for (int g = 0; g < NG; ++g) ush += (size_t)c.width[g] * 2;
   const size_t T = (size_t)n_tokens;
@@ -788,7 +843,7 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
     for (const Client& c : s->clients) {
       if (!c.used) continue;
       for (int g = 0; g < NG; ++g) if (c.width[g]) R[g] = std::max(R[g], c.col_off[g] + c.width[g]);
-      if (c.mask >> TD & 1) save_a = true;
+      if ((c.mask >> TD & 1) && D.arch != MENOS_ARCH_OPT) save_a = true;
     }
   }
   for (int i = 0; i < n_clients; ++i) {
@@ -797,7 +852,7 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
     if (n_tokens[i] < 0) FAIL(MENOS_EINVAL, "n_tokens < 0");
     const Client& c = s->clients[id];
     for (int g = 0; g < NG; ++g) if (c.width[g]) R[g] = std::max(R[g], c.col_off[g] + c.width[g]);
-    if (c.mask >> TD & 1) save_a = true;
+    if ((c.mask >> TD & 1) && D.arch != MENOS_ARCH_OPT) save_a = true;
     T += n_tokens[i];
   }
   if (T > (1ll << 30)) FAIL(MENOS_EINVAL, "too many tokens");
@@ -986,7 +1041,7 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
     const Client& cl = s->clients[c];
     for (int g = 0; g < NG; ++g)
       if (cl.width[g]) { b->g_active[g] = true; b->R_used[g] = std::max(b->R_used[g], cl.col_off[g] + cl.width[g]); }
-    if (cl.mask >> TD & 1) b->save_a = true;
+    if ((cl.mask >> TD & 1) && D.arch != MENOS_ARCH_OPT) b->save_a = true;
   }
   for (int g = 0; g < NG; ++g) b->R_used[g] = (int)align_up(b->R_used[g], 64);
   b->n_mt = ceil_div(T, 128);
@@ -1011,7 +1066,7 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
   A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x (fp32), xn, rstd1
   A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
   A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h (fp32), hn, rstd2
-  A((size_t)T * 2 * D.fpad * 2);                                            // gu
+  A((size_t)T * D.gu_cols * 2);                                             // gu
   if (save_a) A((size_t)T * D.fpad * 2);
   for (int g = 0; g < NG; ++g) if (R_used[g]) A((size_t)T * R_used[g] * 2);
   return per_layer * Ls;
@@ -1023,13 +1078,13 @@ static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool 
   const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
   A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout
   A(db); A(db); A(db); A(db); A(db);                                          // dyb, dxb, dhb, dhn, io
-  A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * 2 * D.fpad * 2); A((size_t)T * D.fpad * 2);
+  A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.gu_cols * 2); A((size_t)T * D.fpad * 2);
   A((size_t)D.H * T * 4);
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
   if (nograd_set) {
     A(db); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
-    A((size_t)T * 2 * D.fpad * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
+    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
     for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   }
   return need;
@@ -1133,8 +1188,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       S.x = (float*)take((size_t)T * D.d * 4); S.xn = (bf16*)take((size_t)T * D.d * 2); S.rstd1 = (float*)take((size_t)T * 4);
       S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2); S.lse = (float*)take((size_t)D.H * T * 4);
       S.h = (float*)take((size_t)T * D.d * 4); S.hn = (bf16*)take((size_t)T * D.d * 2); S.rstd2 = (float*)take((size_t)T * 4);
-      S.gu = (bf16*)take((size_t)T * 2 * D.fpad * 2);
-      S.a = b->save_a ? (bf16*)take((size_t)T * D.fpad * 2) : sc.a;
+      S.gu = (bf16*)take((size_t)T * D.gu_cols * 2);
+      S.a = D.arch == MENOS_ARCH_OPT ? S.gu : b->save_a ? (bf16*)take((size_t)T * D.fpad * 2) : sc.a;
       for (int g = 0; g < NG; ++g) S.U[g] = b->g_active[g] ? (bf16*)take((size_t)T * b->R_used[g] * 2) : nullptr;
     }
   } else {
@@ -1179,7 +1234,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       switch (g) {
         case GQKV: X = S.xn; ldx = D.d; dY = sc.dqkv; ldy = D.Nqkv; break;
         case GO: X = S.O; ldx = D.Nq; dY = sc.dhb; ldy = D.d; break;
-        case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = 2 * D.fpad; break;
+        case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = D.gu_cols; break;
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
       std::vector<LoraRowsProblem> f, du;
@@ -1291,7 +1346,7 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   sc.dyb = (bf16*)take(db); sc.dxb = (bf16*)take(db); sc.dhb = (bf16*)take(db); sc.dhn = (bf16*)take(db);
   sc.io = (bf16*)take(db);
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
-  sc.dgu = (bf16*)take((size_t)T * 2 * D.fpad * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
+  sc.dgu = (bf16*)take((size_t)T * D.gu_cols * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
   sc.Dsum = (float*)take((size_t)D.H * T * 4);
   for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
   return MENOS_OK;
@@ -1304,10 +1359,10 @@ static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scr
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
   S.xn = (bf16*)take((size_t)T * D.d * 2); S.h = (float*)take((size_t)T * D.d * 4);
   S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
-  S.gu = (bf16*)take((size_t)2 * T * D.fpad * 2); S.lse = (float*)take((size_t)D.H * T * 4);
+  S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * T * 4);
   S.rstd1 = (float*)take((size_t)T * 8); S.rstd2 = S.rstd1 + T;
   S.hn = sc.dhn;  // free during a forward
-  S.a = sc.a;
+  S.a = D.arch == MENOS_ARCH_OPT ? S.gu : sc.a;   // OPT: the down projection's input is relu(fc1), kept in gu
   for (int g = 0; g < NG; ++g) S.U[g] = (bf16*)take((size_t)T * R_used[g] * 2);
 }
 
@@ -1349,8 +1404,13 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
   const int T = b->Tl[l];
   if (T == 0) return MENOS_OK;
   const menos_batch::AttnView& V = b->views[b->view_of[l]];
-  // A1: RMSNorm1 (fp32 residual in, bf16 GEMM operand out)
-  { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st)); }
+  const bool opt = D.arch == MENOS_ARCH_OPT;
+  // A1: RMSNorm1 (OPT: LayerNorm1) (fp32 residual in, bf16 GEMM operand out)
+  {
+    ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st);
+    if (opt) K_TRY(layernorm_fwd(x, W.g1, W.be1, S.xn, S.rstd1, T, D.d, D.eps, st));
+    else K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st));
+  }
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
   if (b->g_active[GQKV]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
@@ -1366,6 +1426,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     }
     a.epi = EPI_ROPE; a.out = S.qkv; a.ldo = D.Nqkv;
     a.rope_cs = s->rope; a.pos = b->d_pos; a.head_dim = D.hd; a.rope_cols = D.Nq + D.Nkv;
+    if (opt) { a.epi = EPI_STORE; a.bias = W.bqkv; }   // OPT: biases, no RoPE (learned positions are client-side)
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A3: varlen causal flash attention
@@ -1393,13 +1454,18 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
       a.mtile_extra = b->d_mtile[GO];
     }
     a.epi = EPI_RESID; a.outf = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
+    if (opt) a.bias = W.bo;
     if (D.tp_rank != 0) a.resid = nullptr;  // row-parallel: rank 0's partial carries the residual
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     int rc = tp_allreduce(s, S.h, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: o-proj partial sums
     if (rc) return rc;
   }
-  // A5: RMSNorm2
-  { ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st); K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st)); }
+  // A5: RMSNorm2 (OPT: LayerNorm2)
+  {
+    ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st);
+    if (opt) K_TRY(layernorm_fwd(S.h, W.g2, W.be2, S.hn, S.rstd2, T, D.d, D.eps, st));
+    else K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st));
+  }
   // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
   if (b->g_active[GGU]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
@@ -1413,6 +1479,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
       a.mtile_extra = b->d_mtile[GGU];
     }
     a.epi = EPI_SWIGLU_FWD; a.out = S.gu; a.ldo = 2 * D.fpad; a.out2 = S.a; a.ldo2 = D.fpad;
+    if (opt) { a.N = D.fpad; a.epi = EPI_RELU_FWD; a.ldo = D.fpad; a.bias = W.bu; }   // OPT: a = relu(fc1(hn))
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   // A7: down GEMM (+ LoRA down) + residual
@@ -1428,6 +1495,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
       a.mtile_extra = b->d_mtile[GD];
     }
     a.epi = EPI_RESID; a.outf = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
+    if (opt) a.bias = W.bd;
     if (D.tp_rank != 0) a.resid = nullptr;
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     int rc = tp_allreduce(s, y, (size_t)T * D.d, MENOS_DT_F32, st);      // A16: down-proj partial sums
@@ -1446,6 +1514,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   const int T = b->Tl[l];
   if (T == 0) return MENOS_OK;
   const menos_batch::AttnView& V = b->views[b->view_of[l]];
+  const bool opt = D.arch == MENOS_ARCH_OPT;
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
   if (b->g_active[GD]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GD], st));
   {
@@ -1457,6 +1526,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GD];
     }
     a.epi = EPI_SWIGLU_BWD; a.out = sc.dgu; a.ldo = 2 * D.fpad; a.aux = S.gu; a.ldaux = 2 * D.fpad;
+    if (opt) { a.epi = EPI_RELU_BWD; a.ldo = D.fpad; a.ldaux = D.fpad; }   // dz = da * (relu(z) > 0)
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   if (b->g_active[GD]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GD], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GD], st)); }
@@ -1464,8 +1534,8 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   if (b->g_active[GGU]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GGU], st));
   {
     GemmArgs a = gemm_base(s);
-    a.M = T; a.N = D.d; a.K = 2 * D.fpad; a.b_mn_major = 1;
-    a.A = sc.dgu; a.lda = 2 * D.fpad; a.B = W.wgu; a.ldb = D.d;
+    a.M = T; a.N = D.d; a.K = D.gu_cols; a.b_mn_major = 1;
+    a.A = sc.dgu; a.lda = D.gu_cols; a.B = W.wgu; a.ldb = D.d;
     if (b->g_active[GGU]) {
       a.R = b->R_used[GGU]; a.A2 = sc.dU[GGU]; a.lda2 = a.R; a.B2 = s->Acat[GGU][l]; a.ldb2 = D.ldK_g[GGU];
       a.mtile_extra = b->d_mtile[GGU];
@@ -1479,7 +1549,8 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
   {
     ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
-    if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
+    if (opt) K_TRY(layernorm_bwd(sc.dhn, S.h, W.g2, dyf, sc.dhf, sc.dhb, T, D.d, D.eps, st));
+    else if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
     else K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
   }
   // A10: O dX (+ LoRA o) -> dO
@@ -1504,7 +1575,8 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
     a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = V.n_blocks; a.kvblocks = b->d_blocks;
     a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv; a.rope_cs = s->rope;
+    a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv;
+    a.rope_cs = opt ? nullptr : s->rope;   // OPT: no RoPE backward
     {
       ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * V.pairs, 0, st);
       if (D.hd == 128 && (g_attn_tc & 8))
@@ -1532,7 +1604,8 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
   {
     ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
-    if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
+    if (opt) K_TRY(layernorm_bwd(sc.dhn, S.x, W.g1, sc.dhf, dxf, dxb, T, D.d, D.eps, st));
+    else if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
     else K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
   }
   return MENOS_OK;
@@ -1720,7 +1793,7 @@ extern "C" int menos_test_batch_tensor(menos_server* s, menos_batch* b, int laye
     case 3: src = S.O; n = T * D.Nq * 2; break;
     case 4: src = S.h; n = T * D.d * 4; break;
     case 5: src = S.hn; n = T * D.d * 2; break;
-    case 6: src = S.gu; n = T * 2 * D.fpad * 2; break;
+    case 6: src = S.gu; n = T * D.gu_cols * 2; break;
     case 7: src = S.a; n = T * D.fpad * 2; break;
     case 8: case 9: case 10: case 11: src = S.U[which - 8]; n = src ? T * b->R_used[which - 8] * 2 : 0; break;
     case 12: src = S.lse; n = (size_t)D.H * T * 4; break;

@@ -107,7 +107,8 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
               : tc_fwd ? attn_fwd_tc(a, d_b128, (int)b128.size(), 0) : attn_fwd(a, 0);
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
-    a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv; a.rope_cs = d_cs;
+    a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv;
+    a.rope_cs = theta > 0.f ? d_cs : nullptr;   // theta <= 0: no RoPE backward (OPT)
     std::vector<int4> items_kv;
     attn_ws_items(seq_len, n_seqs, Hkv, items_kv, g_attn_order ? 2 : 0);
     int4* d_items_kv;

@@ -15,6 +15,7 @@ LIB_PATH = os.path.join(HERE, "_lib", "libmenos.so")
 TARGET_BITS = {"q": 1, "k": 2, "v": 4, "o": 8, "gate": 16, "up": 32, "down": 64}
 TARGET_INDEX = {"q": 0, "k": 1, "v": 2, "o": 3, "gate": 4, "up": 5, "down": 6}
 FWD_SAVE, FWD_NOGRAD = 0, 1
+ARCH = {"llama": 0, "opt": 1}
 MEM_BOUND = 2
 REQ_FWD, REQ_BWD = 0, 1
 WHICH = {"A": 0, "B": 1, "dA": 2, "dB": 3, "mA": 4, "mB": 5, "vA": 6, "vB": 7}
@@ -29,11 +30,12 @@ class MenosError(RuntimeError):
 
 class ModelCfg(C.Structure):
     _fields_ = [("d_model", C.c_int), ("n_heads", C.c_int), ("n_kv_heads", C.c_int), ("d_ff", C.c_int),
-                ("rms_eps", C.c_float), ("rope_theta", C.c_float)]
+                ("rms_eps", C.c_float), ("rope_theta", C.c_float), ("arch", C.c_int)]
 
 
 class LayerWeights(C.Structure):
-    _fields_ = [(n, C.c_void_p) for n in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")]
+    _fields_ = [(n, C.c_void_p) for n in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2",
+                                          "bq", "bk", "bv", "bo", "bup", "bdown", "b1", "b2")]
 
 
 class AdamWCfg(C.Structure):
@@ -174,11 +176,11 @@ class Server:
 
     def __init__(self, d_model, n_heads, n_kv_heads, d_ff, n_layers, first_layer=1, rms_eps=1e-5,
                  rope_theta=1e4, weights=None, device=0, max_clients=64, max_rank=64, max_seq_len=4096,
-                 arena_bytes=0, num_sms=0, tp=None):
+                 arena_bytes=0, num_sms=0, tp=None, arch="llama"):
         """tp = (rank, world, allreduce) for tensor parallelism (include/menos.h menos_tp_cfg): `weights` are
         then the rank's shards (tp.shard_layer_weights) and `allreduce(buf, count, dtype, stream)` is an in-place
         sum over the ranks (tp.make_torch_allreduce)."""
-        self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta)
+        self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta, ARCH[arch])
         self.n_layers = n_layers
         tpc = TPCfg(0, 1, ALLREDUCE_FN(), None)
         self._tp_cb = None
@@ -197,7 +199,7 @@ class Server:
 
     @staticmethod
     def _lw(w: dict) -> LayerWeights:
-        return LayerWeights(*[ptr(w[k]) for k in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")])
+        return LayerWeights(*[ptr(w.get(k)) for k, _ in LayerWeights._fields_])
 
     def load_layer(self, layer: int, w: dict):
         lw = self._lw(w)

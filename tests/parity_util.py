@@ -34,13 +34,13 @@ def new_server(w: Workload, weights, arena_bytes=0, max_rank=16, device="cuda:0"
     m = w.model
     wl = []
     for W in weights:
-        wl.append({k: _bf16(W[k]) for k in ("wq", "wk", "wv", "wo", "wgate", "wup", "wdown", "g1", "g2")})
+        wl.append({k: _bf16(v) for k, v in W.items()})
     names = {"wq": "wq", "wk": "wk", "wv": "wv", "wo": "wo", "wgate": "wgate", "wup": "wup", "wdown": "wdown"}
     del names
     max_seq = max(max(c.seq_lens) for c in w.clients)
     srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
                  rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=wl, max_rank=max_rank,
-                 max_seq_len=max(max_seq, 64), arena_bytes=arena_bytes)
+                 max_seq_len=max(max_seq, 64), arena_bytes=arena_bytes, arch=m.arch)
     return srv
 
 
@@ -112,8 +112,9 @@ def run_oracle_step(w: Workload, seed: int = 0, zero_b: bool = False, inputs=Non
             continue
         # a client with cut k runs the segment [k, L): the same oracle on the layers it sends its tokens through
         mc = m.with_layers(m.n_layers - c.cut) if c.cut else m
+        # OPT: the ReLU mask is a floating-point decision; the oracle takes it in the kernel's precision (R25)
         xs, gs, gr = O.client_step(io[i][0], io[i][1], c.seq_lens, weights[c.cut:], adapters[i][c.cut:],
-                                   c.alpha / c.rank, mc)
+                                   c.alpha / c.rank, mc, relu_mask_bf16=(m.arch == "opt"))
         out["x_s"].append(xs)
         out["g_s"].append(gs)
         out["grads"].append(gr)

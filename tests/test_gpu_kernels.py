@@ -239,8 +239,12 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
                                              (128, 4, 2, [1, 17, 64, 129, 300], 3), (128, 4, 2, [1, 17, 64, 129, 300], 0),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 2), (128, 8, 1, [130, 7, 256], 3),
                                              (128, 2, 2, [512, 1024, 255], 3), (128, 2, 2, [512, 1024, 255], 0),
-                                             (16, 4, 4, [16, 16, 3], 3), (64, 8, 1, [200, 65], 3)])
+                                             (16, 4, 4, [16, 16, 3], 3), (64, 8, 1, [200, 65], 3),
+                                             (128, 4, 4, [1, 17, 64, 129, 300], -14), (64, 4, 4, [200, 65], -3)])
 def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
+    """tc < 0: kernel variant |tc| with no RoPE (theta 0: the OPT path, NEXT-4)."""
+    rope = tc >= 0
+    tc = abs(tc)
     from paper_conf_middleware_hul24_b200.menos import check
     check(lib().menos_test_set_attn_tc(tc), testing=True)
     T = sum(lens)
@@ -253,7 +257,7 @@ def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
     dqkv = torch.zeros(T, N, dtype=torch.bfloat16, device="cuda")
     dO_d = dev(dO)  # keep a reference: a temporary's memory would be recycled before the call
     rc = lib().menos_test_attention(len(lens), i32(lens), H, Hkv, hd, qkv_d.data_ptr(), O_d.data_ptr(),
-                                    lse.data_ptr(), dO_d.data_ptr(), dqkv.data_ptr(), 1e4)
+                                    lse.data_ptr(), dO_d.data_ptr(), dqkv.data_ptr(), 1e4 if rope else 0.0)
     check(rc, testing=True)
     got_O, got_lse, got_d = host(O_d), lse.cpu().numpy(), host(dqkv)
     t0 = 0
@@ -266,8 +270,9 @@ def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
         np.testing.assert_allclose(got_lse[:, t0:t0 + L], lb, rtol=2e-3, atol=2e-3)
         # backward uses the GPU's bf16 O (as the kernel does) only through D; compare with the oracle
         dq, dk, dv = O.attention_bwd(dO[t0:t0 + L].reshape(L, H, hd), q, k, v)
-        cos, sin = O.rope_cos_sin(L, hd, 1e4, np.float32)
-        dq, dk = O.rope_bwd(dq, cos, sin), O.rope_bwd(dk, cos, sin)
+        if rope:
+            cos, sin = O.rope_cos_sin(L, hd, 1e4, np.float32)
+            dq, dk = O.rope_bwd(dq, cos, sin), O.rope_bwd(dk, cos, sin)
         ref = np.concatenate([dq.reshape(L, -1), dk.reshape(L, -1), dv.reshape(L, -1)], 1)
         g = got_d[t0:t0 + L]
         scale = np.max(np.abs(ref))

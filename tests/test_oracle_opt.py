@@ -140,3 +140,27 @@ def test_opt_zero_b_is_base_and_models_registered():
     np.testing.assert_array_equal(y0, y1)
     m = MODELS["opt1.3b"]
     assert (m.d_model, m.n_heads, m.d_ff, m.total_layers, m.head_dim) == (2048, 32, 8192, 24, 64)
+
+
+def test_relu_decision_in_kernel_precision_differs_only_where_ambiguous():
+    """Reading R25: with relu_mask_bf16 the oracle decides the ReLU mask on bf16 operands (the kernel's precision).
+    Pin: the decision agrees with the exact fp64 sign wherever the exact pre-activation is farther from 0 than the
+    a-priori bound of the bf16 operand rounding, |z - z_bf16| <= 2^-8 (sum_k |hn_k W_k| + LoRA terms), and flips are
+    rare; elsewhere both signs are correct results."""
+    cfg = opt_cfg()
+    W = base_layer_weights(cfg, 0, seed=61)
+    c = ClientCfg(8, 16.0, ("up",), [200])
+    lora = client_adapters(cfg, c, seed=62)[0]
+    x, _ = client_inputs(cfg, c, seed=63)
+    s = c.alpha / c.rank
+    _, cache = O.opt_layer_fwd(x.astype(F64), W, lora, s, cfg, F64)
+    hn = cache["hn"]
+    A, B = (a.astype(F64) for a in lora["up"])
+    z = hn @ W["wup"].astype(F64).T + s * (hn @ A.T) @ B.T + W["bup"].astype(F64)
+    mask = O.relu_decision(hn, W["wup"], W["bup"], lora["up"], s)
+    bound = 2.0 ** -8 * (np.abs(hn) @ np.abs(W["wup"].astype(F64)).T
+                         + s * (np.abs(hn) @ np.abs(A).T) @ np.abs(B).T * 2.0) + 1e-6 * np.abs(z)
+    flips = mask != (z > 0)
+    assert np.all(np.abs(z[flips]) <= bound[flips])
+    assert np.all(mask[np.abs(z) > bound] == (z[np.abs(z) > bound] > 0))
+    assert flips.mean() < 5e-3
