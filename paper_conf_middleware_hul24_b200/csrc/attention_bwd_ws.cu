@@ -57,72 +57,6 @@ __device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const
   }
 }
 
-// Epilogue, fp32 staging of 64 accumulator rows (one TMEM lane-quadrant pair) in 32 KB: 16-byte chunk k (0..31) of
-// staged row rr at rr * 512 + ((k ^ (rr & 7)) << 4) (conflict-free for the row-per-lane writes)
-__device__ __forceinline__ float* stg32_at(uint8_t* stg, int rr, int k) {
-  return reinterpret_cast<float*>(stg + rr * 512 + ((k ^ (rr & 7)) << 4));
-}
-// this thread's TMEM row (staged row rr), columns [32g, 32g+32) and [64+32g, 64+32g+32)
-__device__ __forceinline__ void acc_row_to_stage32(uint32_t tacc, uint8_t* stg, int rr, int g) {
-  uint32_t a[32], b[32];
-  tmem_ld32_nw(tacc + 32 * g, a);
-  tmem_ld32_nw(tacc + 64 + 32 * g, b);
-  tmem_wait_ld();
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {
-    *reinterpret_cast<uint4*>(stg32_at(stg, rr, 8 * g + c)) = make_uint4(a[4 * c], a[4 * c + 1], a[4 * c + 2], a[4 * c + 3]);
-    *reinterpret_cast<uint4*>(stg32_at(stg, rr, 16 + 8 * g + c)) = make_uint4(b[4 * c], b[4 * c + 1], b[4 * c + 2], b[4 * c + 3]);
-  }
-}
-// all elementwise warps: staged rows -> bf16 rows of dst (rows row0 + rr < n_valid), lanes across columns (the RoPE
-// table reads and the row stores are coalesced); with rope the RoPE backward at position pos0 + row0 + rr:
-// dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
-__device__ __forceinline__ void stage32_to_global(uint8_t* stg, int w8, int lane, int row0, int n_valid, bf16* dst,
-                                                  int ld, const float2* cs, int pos0, bool rope) {
-  const int jl = lane & 15, j = 4 * jl;
-#pragma unroll 2
-  for (int r2 = 0; r2 < 8; r2 += 2) {
-    const int rr = w8 * 8 + r2 + (lane >> 4), row = row0 + rr;
-    if (row >= n_valid) continue;
-    const float4 a = *reinterpret_cast<const float4*>(stg32_at(stg, rr, jl));
-    const float4 b = *reinterpret_cast<const float4*>(stg32_at(stg, rr, 16 + jl));
-    float x[4] = {a.x, a.y, a.z, a.w}, y[4] = {b.x, b.y, b.z, b.w};
-    if (rope) {
-      const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)(pos0 + row) * (HD / 2) + j);
-      const float4 e0 = c4[0], e1 = c4[1];   // (c_j, s_j, c_j+1, s_j+1), (c_j+2, s_j+2, c_j+3, s_j+3)
-      const float cc[4] = {e0.x, e0.z, e1.x, e1.z}, ss[4] = {e0.y, e0.w, e1.y, e1.w};
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float xi = x[i] * cc[i] + y[i] * ss[i], yi = y[i] * cc[i] - x[i] * ss[i];
-        x[i] = xi; y[i] = yi;
-      }
-    }
-    bf16* d = dst + (size_t)row * ld;
-    *reinterpret_cast<uint2*>(d + j) = make_uint2(pack_bf16x2(x[0], x[1]), pack_bf16x2(x[2], x[3]));
-    *reinterpret_cast<uint2*>(d + 64 + j) = make_uint2(pack_bf16x2(y[0], y[1]), pack_bf16x2(y[2], y[3]));
-  }
-}
-// one 128-row accumulator through the 32 KB staging area in two 64-row rounds (TMEM lane quadrants 0-1, then
-// 2-3); with arrive, each warp arrives on acc_free right after its TMEM rows have been read
-__device__ __forceinline__ void acc_epilogue(uint32_t tacc_lane, uint8_t* stg, int w4, int w8, int lane, int g,
-                                             int n_valid, bf16* dst, int ld, const float2* cs, int pos0, bool rope,
-                                             uint64_t* acc_free_bar, bool arrive) {
-#pragma unroll 1
-  for (int half = 0; half < 2; ++half) {
-    if ((w4 >> 1) == half) {
-      acc_row_to_stage32(tacc_lane, stg, (w4 & 1) * 32 + lane, g);
-      if (arrive) {
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(acc_free_bar);
-      }
-    }
-    ew_sync();
-    stage32_to_global(stg, w8, lane, half * 64, n_valid, dst, ld, cs, pos0, rope);
-    ew_sync();
-  }
-}
-
 // Single-round epilogue: every elementwise thread converts its TMEM row (columns [32g, 32g+32) and [64+32g, ..),
 // i.e. the RoPE pairs (j, j+64)) to bf16 in registers -- RoPE backward applied there -- and writes it into a bf16
 // staging tile [128 rows][256 B] (16-byte chunk k of row rr at rr*256 + ((k ^ (rr & 15)) << 4)); the TMEM

@@ -55,6 +55,10 @@ struct KParams {
   int head_dim, rope_cols;
 };
 
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+
 // v[j] += bias[col + j] (fp32, 32 consecutive columns; col % 32 == 0)
 __device__ __forceinline__ void add_bias32(float (&v)[32], const float* bias, int col) {
   const float4* b4 = reinterpret_cast<const float4*>(bias + col);
@@ -271,6 +275,26 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     for (int t = cluster_id; t < total; t += n_clusters) {
       int m, n;
       tile_coords(t, num_m, num_n, m, n);
+      {
+        // L2 prefetch of the epilogue's HBM inputs for this row while the tile's MMAs still run: residual (fp32,
+        // 8 x 128 B lines), saved g|u (SwiGLU bwd: 2 x 4 x 128 B) or relu output (4 x 128 B)
+        const int prow = m * C::TILE_M + rank * BM + q * 32 + lane;
+        const int pn0 = n * BN;
+        if (prow < p.M) {
+          if (p.epi == EPI_RESID && p.resid) {
+            const float* r = p.resid + (size_t)prow * p.ldr + pn0;
+            for (int c = 0; c < 8 && pn0 + c * 32 < p.N; ++c) prefetch_l2(r + c * 32);
+          } else if (p.epi == EPI_SWIGLU_BWD) {
+            for (int h = 0; h < 2 && pn0 + h * 128 < p.N; ++h) {
+              const bf16* a = p.aux + (size_t)prow * p.ldaux + ((pn0 + h * 128) >> 7) * 256;
+              for (int c = 0; c < 2; ++c) { prefetch_l2(a + c * 64); prefetch_l2(a + 128 + c * 64); }
+            }
+          } else if (p.epi == EPI_RELU_BWD) {
+            const bf16* a = p.aux + (size_t)prow * p.ldaux + pn0;
+            for (int c = 0; c < 4 && pn0 + c * 64 < p.N; ++c) prefetch_l2(a + c * 64);
+          }
+        }
+      }
       mbar_wait(&tfull_bar[acc], acc_phase);
       tc_fence_after();
       const int row = m * C::TILE_M + rank * BM + q * 32 + lane;

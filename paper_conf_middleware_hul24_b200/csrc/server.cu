@@ -17,6 +17,7 @@
 
 #include "../../include/menos.h"
 #include "../../include/menos_testing.h"
+#include <type_traits>
 #include "kernels.h"
 
 using namespace menos;
@@ -293,6 +294,12 @@ struct menos_batch {
   // saved activations (SAVE) or x_c copy (NOGRAD)
   uint8_t* slab = nullptr;
   std::vector<LayerSave> L;
+  // LoRA side problem lists reference the per-call scratch block (dY, dU); the scratch may move between this
+  // batch's forward and its backward (another call of a different size in between), so the host copies are kept
+  // and relocated before the backward (relocate_scratch_refs)
+  std::vector<LoraRowsProblem> h_rprobs;
+  std::vector<LoraTokRedProblem> h_tprobs;
+  uint8_t* scratch_base = nullptr; size_t scratch_span = 0;
 };
 
 // =====================================================================================================
@@ -1321,6 +1328,9 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
   b->d_rprobs = (LoraRowsProblem*)(meta + o_rp);
+  b->h_rprobs = std::move(rprobs);
+  b->h_tprobs = std::move(tprobs);
+  b->scratch_base = s->scratch; b->scratch_span = s->scratch_bytes;
   b->d_rtiles = (int2*)(meta + o_rt);
   b->d_tprobs = (LoraTokRedProblem*)(meta + o_tp);
   b->d_ttiles = (int4*)(meta + o_tt);
@@ -1710,6 +1720,28 @@ extern "C" int menos_batch_free(menos_server* s, menos_batch* b) {
   return MENOS_OK;
 }
 
+// Shift every problem-list pointer into the batch's forward-time scratch block to the current block (same T and
+// slot widths => same internal offsets, get_scratch) and re-upload the lists (stream-ordered, pinned ring).
+static int relocate_scratch_refs(menos_server* s, menos_batch* b, cudaStream_t st) {
+  if (b->scratch_base == s->scratch || b->scratch_base == nullptr) return MENOS_OK;
+  const uint8_t* lo = b->scratch_base;
+  const uint8_t* hi = lo + b->scratch_span;
+  const ptrdiff_t delta = s->scratch - b->scratch_base;
+  auto mv = [&](auto*& p) {
+    const uint8_t* q = reinterpret_cast<const uint8_t*>(p);
+    if (q >= lo && q < hi) p = reinterpret_cast<std::remove_reference_t<decltype(p)>>(const_cast<uint8_t*>(q) + delta);
+  };
+  for (auto& p : b->h_rprobs) { mv(p.A); mv(p.B); mv(p.C); }
+  for (auto& p : b->h_tprobs) { mv(p.P); mv(p.Q); mv(p.C); }
+  int rc = 0;
+  if (!b->h_rprobs.empty()) rc = upload(s, b->d_rprobs, b->h_rprobs.data(), b->h_rprobs.size() * sizeof(LoraRowsProblem), st);
+  if (!rc && !b->h_tprobs.empty())
+    rc = upload(s, b->d_tprobs, b->h_tprobs.data(), b->h_tprobs.size() * sizeof(LoraTokRedProblem), st);
+  if (rc) return rc;
+  b->scratch_base = s->scratch; b->scratch_span = s->scratch_bytes;
+  return MENOS_OK;
+}
+
 extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, void* g_s, void* stream) {
   if (!s || !b || !g_c || !g_s) FAIL(MENOS_EINVAL, "bad arguments");
   for (int c : b->bclients) if (!s->clients[c].used) FAIL(MENOS_ESTATE, "client %d unregistered since forward", c);
@@ -1734,6 +1766,9 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
     s->arena.release(old_meta);   // stream-ordered reuse: later users run after these copies
     s->arena.release(old_slab);
     rc = forward_save(s, b, sc, sc.xout, st);
+    if (rc) return rc;
+  } else {
+    rc = relocate_scratch_refs(s, b, st);
     if (rc) return rc;
   }
   // g_c (bf16) -> the bf16 copy of the incoming gradient and the fp32 gradient residual stream

@@ -216,3 +216,34 @@ def test_host_buffers_e2e_path():
     np.testing.assert_array_equal(xs.float().numpy(), np.concatenate(dev_out["x_s"]))
     np.testing.assert_array_equal(gs.float().numpy(), np.concatenate(dev_out["g_s"]))
     srv.close()
+
+
+def test_interleaved_save_batches_bitwise():
+    """Two SAVE batches of different sizes outstanding at once (forward A, forward B, backward A, backward B):
+    the per-call scratch block moves in between, and A's backward must still equal A run alone (bitwise)."""
+    m = MODELS["tiny"]
+    wa = Workload("a", m, [ClientCfg(4, 8.0, ("q", "v", "down"), [30, 9])])
+    wb = Workload("b", m, [ClientCfg(8, 16.0, TARGETS, [200, 77])])
+    ia, ib = make_inputs(wa, seed=31), make_inputs(wb, seed=32)
+    ib = (ia[0], ib[1], ib[2])   # one shared base
+    ref_a, ref_b = run_gpu_step(wa, inputs=ia), run_gpu_step(wb, inputs=ib)
+    w = Workload("ab", m, wa.clients + wb.clients)
+    srv = new_server(w, ia[0])
+    ids = register(srv, w, ia[1] + ib[1])
+    from tests.parity_util import _bf16
+    xa, ga = (_bf16(np.concatenate([a for a, _ in ia[2]]), "cuda"), _bf16(np.concatenate([g for _, g in ia[2]]), "cuda"))
+    xb, gb = (_bf16(np.concatenate([a for a, _ in ib[2]]), "cuda"), _bf16(np.concatenate([g for _, g in ib[2]]), "cuda"))
+    xsa, gsa, xsb, gsb = (torch.empty_like(t) for t in (xa, ga, xb, gb))
+    ba = srv.forward([ids[0]] * 2, [30, 9], xa, xsa)
+    bb = srv.forward([ids[1]] * 2, [200, 77], xb, xsb)
+    srv.backward(ba, ga, gsa)
+    srv.backward(bb, gb, gsb)
+    torch.cuda.synchronize()
+    assert np.array_equal(xsa.float().cpu().numpy(), ref_a["x_s"][0])
+    assert np.array_equal(gsa.float().cpu().numpy(), ref_a["g_s"][0])
+    assert np.array_equal(xsb.float().cpu().numpy(), ref_b["x_s"][0])
+    assert np.array_equal(gsb.float().cpu().numpy(), ref_b["g_s"][0])
+    for l in range(m.n_layers):
+        for t in ("q", "v", "down"):
+            assert np.array_equal(srv.get_adapter(ids[0], l, t, "dA"), ref_a["grads"][0][l][t][0])
+    srv.close()
