@@ -150,7 +150,7 @@ def build_server(torch, w, device, seed, arena_gb, tp=None):
     srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
                  rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=None, device=device.index,
                  max_rank=16, max_seq_len=max(max(c.seq_lens) for c in w.clients),
-                 arena_bytes=int(arena_gb * (1 << 30)), tp=tp)
+                 arena_bytes=int(arena_gb * (1 << 30)), tp=tp, arch=m.arch)
     gen = torch.Generator(device=device)
     hd = m.head_dim
     W = tp[1] if tp else 1
@@ -166,6 +166,12 @@ def build_server(torch, w, device, seed, arena_gb, tp=None):
               for k, s in shapes.items()}
         for gname in ("g1", "g2"):
             lw[gname] = (1 + 0.1 * torch.randn(m.d_model, generator=gen, device=device)).to(torch.bfloat16)
+        if m.arch == "opt":   # OPT (NEXT-4): no gate; biases and LayerNorm biases (workloads.base_layer_weights recipe)
+            del lw["wgate"]
+            for bname, n in (("bq", Hl * hd), ("bk", Hkvl * hd), ("bv", Hkvl * hd), ("bo", m.d_model),
+                             ("bup", fl), ("bdown", m.d_model), ("b1", m.d_model), ("b2", m.d_model)):
+                sd = 0.1 if bname in ("b1", "b2") else 0.02
+                lw[bname] = (sd * torch.randn(n, generator=gen, device=device)).to(torch.bfloat16)
         srv.load_layer(l, lw)
         del lw
     torch.cuda.synchronize(device)
@@ -351,8 +357,9 @@ def run_gpu(args):
     # algorithmic FLOPs of the whole step (no recompute credit, no base dW): 4 P + attention + LoRA
     m = w.model
     hd = m.head_dim
+    mlp_mats = 2 if m.arch == "opt" else 3   # OPT: fc1, fc2; Llama: gate, up, down
     P = m.n_layers * (m.d_model * (m.n_heads + 2 * m.n_kv_heads) * hd + m.d_model * m.n_heads * hd
-                      + 3 * m.d_model * m.d_ff)
+                      + mlp_mats * m.d_model * m.d_ff)
     pairs = sum(s * (s + 1) / 2 for c in w.clients for s in c.seq_lens)
     attn = 12 * hd * m.n_heads * pairs * m.n_layers
     lora = 0.0

@@ -98,46 +98,50 @@ __global__ void rmsnorm_bwd_kernel(const TDY* __restrict__ dy, const float* __re
 }
 
 // ------------------------------------------------------------------ single-pass RMSNorm (row cached in registers)
-// 128 threads per row, 8-element chunks, up to NC chunks per thread (d <= 128 * 8 * NC); block = 2 rows.
-template <int NC>
+// TPR threads per row (128, or 256 for wide rows such as d = 8192), 8-element chunks, up to NC chunks per thread
+// (d <= TPR * 8 * NC); block = 256 threads = 256 / TPR rows.
+template <int TPR>
 __device__ __forceinline__ float block_row_sum(float v, float* red, int wr) {
-  // reduce over the 4 warps of this row's 128 threads
+  // reduce over the TPR / 32 warps of this row's threads (fixed order)
+  constexpr int W = TPR / 32;
   v = warp_sum(v);
-  const int lane = threadIdx.x & 31, w = (threadIdx.x >> 5) & 3;
-  if (lane == 0) red[wr * 4 + w] = v;
+  const int lane = threadIdx.x & 31, w = (threadIdx.x % TPR) >> 5;
+  if (lane == 0) red[wr * W + w] = v;
   __syncthreads();
-  const float s = red[wr * 4 + 0] + red[wr * 4 + 1] + red[wr * 4 + 2] + red[wr * 4 + 3];
+  float s = red[wr * W];
+#pragma unroll
+  for (int k = 1; k < W; ++k) s += red[wr * W + k];
   return s;
 }
 
-template <int NC>
+template <int NC, int TPR>
 __global__ void __launch_bounds__(256) rmsnorm_fwd_reg_kernel(const float* __restrict__ x, const float* __restrict__ g,
                                                               bf16* __restrict__ y, float* __restrict__ rstd, int T,
                                                               int d, float eps) {
   __shared__ float red[8];
-  const int wr = threadIdx.x >> 7, t = threadIdx.x & 127;
-  const int row = blockIdx.x * 2 + wr;
+  const int wr = threadIdx.x / TPR, t = threadIdx.x % TPR;
+  const int row = blockIdx.x * (256 / TPR) + wr;
   const bool ok = row < T;
   const float* xr = x + (size_t)(ok ? row : 0) * d;
   float v[NC][8];
   float ss = 0.f;
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
-    const int i = (c * 128 + t) * 8;
+    const int i = (c * TPR + t) * 8;
     if (ok && i < d) {
       ld8f(xr + i, v[c]);
 #pragma unroll
       for (int k = 0; k < 8; ++k) ss += v[c][k] * v[c][k];
     }
   }
-  ss = block_row_sum<NC>(ss, red, wr);
+  ss = block_row_sum<TPR>(ss, red, wr);
   const float r = rsqrtf(ss / (float)d + eps);
   if (!ok) return;
   if (t == 0) rstd[row] = r;
   bf16* yr = y + (size_t)row * d;
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
-    const int i = (c * 128 + t) * 8;
+    const int i = (c * TPR + t) * 8;
     if (i < d) {
       float gg[8];
       ld8f(g + i, gg);
@@ -148,42 +152,42 @@ __global__ void __launch_bounds__(256) rmsnorm_fwd_reg_kernel(const float* __res
   }
 }
 
-template <int NC, typename TDY>
+template <int NC, int TPR, typename TDY>
 __global__ void __launch_bounds__(256) rmsnorm_bwd_reg_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
                                                               const float* __restrict__ g, const float* __restrict__ rstd,
                                                               const float* __restrict__ resid, float* __restrict__ dx,
                                                               bf16* __restrict__ dxb, int T, int d) {
   __shared__ float red[8];
-  const int wr = threadIdx.x >> 7, t = threadIdx.x & 127;
-  const int row = blockIdx.x * 2 + wr;
+  const int wr = threadIdx.x / TPR, t = threadIdx.x % TPR;
+  const int row = blockIdx.x * (256 / TPR) + wr;
   const bool ok = row < T;
   const size_t ro = (size_t)(ok ? row : 0) * d;
   const float r = ok ? rstd[row] : 0.f;
-  float a[NC][8], b[NC][8];
+  float a[NC][8], b[NC][8], res[NC][8];
   float dot = 0.f;
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
-    const int i = (c * 128 + t) * 8;
+    const int i = (c * TPR + t) * 8;
     if (ok && i < d) {
       float gg[8];
       ld8(dy + ro + i, a[c]);
       ld8f(x + ro + i, b[c]);
+      ld8f(resid + ro + i, res[c]);   // issued with the others: its latency overlaps the row reduction
       ld8f(g + i, gg);
 #pragma unroll
       for (int k = 0; k < 8; ++k) { a[c][k] *= gg[k]; dot += a[c][k] * b[c][k]; }   // a = gh = dy * g
     }
   }
-  dot = block_row_sum<NC>(dot, red, wr);
+  dot = block_row_sum<TPR>(dot, red, wr);
   if (!ok) return;
   const float mean = dot * r / (float)d;
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
-    const int i = (c * 128 + t) * 8;
+    const int i = (c * TPR + t) * 8;
     if (i < d) {
-      float res[8], o[8];
-      ld8f(resid + ro + i, res);
+      float o[8];
 #pragma unroll
-      for (int k = 0; k < 8; ++k) o[k] = res[k] + r * (a[c][k] - b[c][k] * r * mean);
+      for (int k = 0; k < 8; ++k) o[k] = res[c][k] + r * (a[c][k] - b[c][k] * r * mean);
       st8f(dx + ro + i, o);
       if (dxb) st8b(dxb + ro + i, o);
     }
@@ -375,13 +379,13 @@ __global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __
 int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
-  const int nc = (d + 1023) / 1024, grid = (T + 1) / 2;
+  const int nc = (d + 1023) / 1024, g2 = (T + 1) / 2;
   switch (nc) {  // single pass: the row stays in registers between the reduction and the write
-    case 1: rmsnorm_fwd_reg_kernel<1><<<grid, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-    case 2: rmsnorm_fwd_reg_kernel<2><<<grid, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-    case 4: rmsnorm_fwd_reg_kernel<4><<<grid, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-    case 5: rmsnorm_fwd_reg_kernel<5><<<grid, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-    case 8: rmsnorm_fwd_reg_kernel<8><<<grid, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 1: rmsnorm_fwd_reg_kernel<1, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 2: rmsnorm_fwd_reg_kernel<2, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 3: case 4: rmsnorm_fwd_reg_kernel<4, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 5: rmsnorm_fwd_reg_kernel<5, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 6: case 7: case 8: rmsnorm_fwd_reg_kernel<4, 256><<<T, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
     default: {
       const int warps = 8;
       rmsnorm_fwd_kernel<<<(T + warps - 1) / warps, warps * 32, 0, st>>>(x, g, y, rstd, T, d, eps);
@@ -394,13 +398,14 @@ static int rmsnorm_bwd_t(const TDY* dy, const float* x, const float* g, const fl
                          float* dx, bf16* dxb, int T, int d, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
-  const int nc = (d + 1023) / 1024, grid = (T + 1) / 2;
+  const int nc = (d + 1023) / 1024, g2 = (T + 1) / 2;
   switch (nc) {
-    case 1: rmsnorm_bwd_reg_kernel<1, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 2: rmsnorm_bwd_reg_kernel<2, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 4: rmsnorm_bwd_reg_kernel<4, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 5: rmsnorm_bwd_reg_kernel<5, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-    case 8: rmsnorm_bwd_reg_kernel<8, TDY><<<grid, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 1: rmsnorm_bwd_reg_kernel<1, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 2: rmsnorm_bwd_reg_kernel<2, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 3: case 4: rmsnorm_bwd_reg_kernel<4, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 5: rmsnorm_bwd_reg_kernel<5, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 6: case 7: case 8:   // wide rows (70B: d = 8192): one row per 256 threads keeps 4 chunks per thread
+      rmsnorm_bwd_reg_kernel<4, 256, TDY><<<T, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
     default: {
       const int warps = 8;
       rmsnorm_bwd_kernel<TDY><<<(T + warps - 1) / warps, warps * 32, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d);

@@ -50,6 +50,7 @@ struct KParams {
   bf16* out2; int ldo2;
   const bf16* aux; int ldaux;
   const float* bias;
+  float* dsum; int dsum_ld, dsum_hd;
   const float2* rope_cs;
   const int* pos;
   int head_dim, rope_cols;
@@ -289,7 +290,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               const bf16* a = p.aux + (size_t)prow * p.ldaux + ((pn0 + h * 128) >> 7) * 256;
               for (int c = 0; c < 2; ++c) { prefetch_l2(a + c * 64); prefetch_l2(a + 128 + c * 64); }
             }
-          } else if (p.epi == EPI_RELU_BWD) {
+          } else if (p.epi == EPI_RELU_BWD || p.epi == EPI_STORE_DSUM) {
             const bf16* a = p.aux + (size_t)prow * p.ldaux + pn0;
             for (int c = 0; c < 4 && pn0 + c * 64 < p.N; ++c) prefetch_l2(a + c * 64);
           }
@@ -309,6 +310,25 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           tmem_ld32(tb + c * 32, v);
           if (p.bias) add_bias32(v, p.bias, col);
           if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
+        }
+      } else if (p.epi == EPI_STORE_DSUM) {
+        float dot = 0.f;
+        for (int c = 0; c < 8; ++c) {
+          const int col = n0 + c * 32;
+          if (col >= p.N) break;
+          float v[32];
+          tmem_ld32(tb + c * 32, v);
+          if (rok) {
+            float o[32];
+            load32(p.aux + (size_t)row * p.ldaux + col, o);
+            store32(p.out + (size_t)row * p.ldo + col, v);
+#pragma unroll
+            for (int j = 0; j < 32; ++j) dot += __bfloat162float(__float2bfloat16_rn(v[j])) * o[j];
+            if ((col + 32) % p.dsum_hd == 0) {
+              p.dsum[(size_t)(col / p.dsum_hd) * p.dsum_ld + row] = dot;
+              dot = 0.f;
+            }
+          }
         }
       } else if (p.epi == EPI_RELU_FWD) {
         for (int c = 0; c < 8; ++c) {
@@ -570,6 +590,7 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
   if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;
   if ((a.epi == EPI_SWIGLU_FWD && a.N % 256) || (a.epi == EPI_SWIGLU_BWD && a.N % 128)) return -1;
+  if (a.epi == EPI_STORE_DSUM && (a.dsum_hd <= 0 || a.dsum_hd % 32 || !a.dsum || !a.aux)) return -1;
   const int CG = g_gemm_cta_group == 1 ? 1 : 2;
   const uint32_t bbox = BN / CG;  // B rows (K-major) staged per CTA
   CUtensorMap mA, mB, mA2, mB2;
@@ -594,6 +615,7 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   p.R = a.R; p.mtile_extra = a.mtile_extra; p.ntile_extra = a.ntile_extra;
   p.epi = a.epi; p.out = a.out; p.ldo = a.ldo; p.resid = a.resid; p.ldr = a.ldr; p.outf = a.outf;
   p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux; p.bias = a.bias;
+  p.dsum = a.dsum; p.dsum_ld = a.dsum_ld; p.dsum_hd = a.dsum_hd;
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
   const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);
   int sms = a.num_sms > 0 ? a.num_sms : 148;

@@ -23,6 +23,9 @@ enum EpiMode : int {
   EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
   EPI_RELU_FWD = 5,    // OPT fc1: out = bf16(relu(acc + bias))
   EPI_RELU_BWD = 6,    // OPT fc2 dX: out = bf16(acc * (aux > 0)), aux = saved relu output
+  EPI_STORE_DSUM = 7,  // o-proj dX: out = dO = bf16(acc), and per head h of width dsum_hd (% 32 == 0):
+                       // dsum[h * dsum_ld + row] = sum_j bf16(dO)[row, j] * aux[row, j] (aux = saved O): the
+                       // attention backward's D = rowsum(dO . O), fused so dO and O are not re-read
   // EPI_STORE and EPI_RESID add `bias[col]` (fp32) when bias != nullptr (OPT projections)
 };
 
@@ -45,6 +48,7 @@ struct GemmArgs {
   bf16* out2; int ldo2;            // EPI_SWIGLU_FWD: a
   const bf16* aux; int ldaux;      // EPI_SWIGLU_BWD: saved gu; EPI_RELU_BWD: saved relu output
   const float* bias;               // [N] fp32 or nullptr (EPI_STORE, EPI_RESID, EPI_RELU_FWD)
+  float* dsum; int dsum_ld, dsum_hd;   // EPI_STORE_DSUM
   const float2* rope_cs;           // EPI_ROPE: [max_pos][hd/2] (cos, sin)
   const int* pos;                  // EPI_ROPE: per-row position
   int head_dim, rope_cols;

@@ -1563,7 +1563,8 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     else if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
     else K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
   }
-  // A10: O dX (+ LoRA o) -> dO
+  // A10: O dX (+ LoRA o) -> dO (and, for head_dim % 32 == 0, the attention backward's row sums D)
+  const bool fuse_dsum = D.hd % 32 == 0;
   if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
   {
     GemmArgs a = gemm_base(s);
@@ -1574,11 +1575,17 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GO];
     }
     a.epi = EPI_STORE; a.out = sc.dO; a.ldo = D.Nq;
+    if (fuse_dsum) {   // A11 prologue fused: D = rowsum(dO . O) per head from the epilogue's bf16 dO
+      a.epi = EPI_STORE_DSUM; a.aux = S.O; a.ldaux = D.Nq; a.dsum = sc.Dsum; a.dsum_ld = T; a.dsum_hd = D.hd;
+    }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
   if (b->g_active[GO]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GO], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GO], st)); }
   // A11: attention backward (+ RoPE backward) -> dqkv
-  { ProfScope ps(PC_ATTN_PREP, 0, (double)T * (4.0 * D.Nq + 4 * D.H), st); K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st)); }
+  if (!fuse_dsum) {
+    ProfScope ps(PC_ATTN_PREP, 0, (double)T * (4.0 * D.Nq + 4 * D.H), st);
+    K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st));
+  }
   {
     AttnArgs a;
     memset(&a, 0, sizeof a);

@@ -289,7 +289,7 @@ def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
         t0 += L
 
 
-@pytest.mark.parametrize("T,d", [(7, 64), (1000, 4096)])
+@pytest.mark.parametrize("T,d", [(7, 64), (1000, 4096), (33, 5120), (65, 8192), (9, 3072)])
 def test_rmsnorm_fwd_bwd(T, d):
     from paper_conf_middleware_hul24_b200.menos import check
     rng = np.random.default_rng(61)

@@ -226,6 +226,12 @@ def workload(name: str, n_layers: int | None = None) -> Workload:
         m = MODELS["13b"]
         cl = [ClientCfg(16, 32.0, TARGETS, [2048]) for _ in range(16)]
         w = Workload(name, m, cl, 8, "Llama-2-13B, 16 clients r=16 all projections, 1 x 2048")
+    elif name == "opt13_x16_paper":
+        # NEXT-4 extra (not a BASELINE config): the paper's OPT setting -- OPT-1.3B server layers
+        # 2..24, LoRA r=8 alpha=16 on q,v, batch 16 x S~100 per client (S15) -- with 16 clients on one GPU
+        m = MODELS["opt1.3b"]
+        cl = [ClientCfg(8, 16.0, ("q", "v"), [100] * 16) for _ in range(16)]
+        w = Workload(name, m, cl, 1, "OPT-1.3B, 16 clients r=8 q,v, batch 16 x 100 (paper's OPT setting)")
     elif name == "cfg4_70b_tp8_x16":
         m = MODELS["70b"]
         cl = [ClientCfg(8, 16.0, ("q", "v"), [1024, 1024]) for _ in range(16)]
