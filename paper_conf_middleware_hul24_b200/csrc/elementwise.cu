@@ -338,6 +338,14 @@ __global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __
   if (row >= T) return;
   const size_t ro = (size_t)row * d;
   float v[NCH][8], gh[NCH][8];
+  // residual loads first: in flight during the loads and reductions below instead of after them
+  const float4* rr4 = reinterpret_cast<const float4*>(resid + ro);
+  float4 rq[NCH][2];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int i = (c * 32 + lane) * 8;
+    if (i < d) { rq[c][0] = rr4[i / 4]; rq[c][1] = rr4[i / 4 + 1]; }
+  }
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
     const int i = (c * 32 + lane) * 8;
@@ -363,8 +371,8 @@ __global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __
   for (int c = 0; c < NCH; ++c) {
     const int i = (c * 32 + lane) * 8;
     if (i >= d) continue;
-    float rr[8], o[8];
-    ld8f(resid + ro + i, rr);
+    const float rr[8] = {rq[c][0].x, rq[c][0].y, rq[c][0].z, rq[c][0].w, rq[c][1].x, rq[c][1].y, rq[c][1].z, rq[c][1].w};
+    float o[8];
 #pragma unroll
     for (int k = 0; k < 8; ++k) o[k] = rr[k] + r * (gh[c][k] - mg - (v[c][k] - mu) * r * mgx);
     st8f(dx + ro + i, o);
