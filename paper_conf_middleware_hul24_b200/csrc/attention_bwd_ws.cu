@@ -21,7 +21,13 @@ bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols,
 
 namespace {
 
-constexpr int HD = 128, STAGES = 3, EW_WARPS = 8, NTHREADS = 64 + 32 * EW_WARPS;
+#ifndef MENOS_BWS_EW
+#define MENOS_BWS_EW 8
+#endif
+// EW_WARPS elementwise warps: EW_WARPS / 4 per TMEM lane quadrant, each thread owning CPT of a block's 64 columns
+constexpr int HD = 128, STAGES = 3, EW_WARPS = MENOS_BWS_EW, NTHREADS = 64 + 32 * EW_WARPS;
+constexpr int CPT = 64 / (EW_WARPS / 4);
+static_assert(CPT == 16 || CPT == 32, "EW_WARPS must be 8 or 16");
 constexpr float LOG2E_W = 1.4426950408889634f;
 
 struct BwParams {
@@ -45,12 +51,27 @@ __device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
 }
 __device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
 
-// columns [32 g, 32 g + 32) (bf16) of one row of a [rows][64] SWIZZLE_128B K-major tile
-__device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const float (&v)[32]) {
+// CPT consecutive TMEM columns (32x32b.x16 / .x32), no wait
+template <int N>
+__device__ __forceinline__ void tmem_ldc_nw(uint32_t taddr, uint32_t (&r)[N]) {
+  if constexpr (N == 32) {
+    tmem_ld32_nw(taddr, r);
+  } else {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+  }
+}
+
+// columns [CPT g, CPT g + CPT) (bf16) of one row of a [rows][64] SWIZZLE_128B K-major tile
+__device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const float (&v)[CPT]) {
   uint8_t* prow = tile + row * 128;
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
-    const int c8 = 4 * g + c;
+  for (int c = 0; c < CPT / 8; ++c) {
+    const int c8 = (CPT / 8) * g + c;
     uint4 u = make_uint4(pack_bf16x2(v[8 * c + 0], v[8 * c + 1]), pack_bf16x2(v[8 * c + 2], v[8 * c + 3]),
                          pack_bf16x2(v[8 * c + 4], v[8 * c + 5]), pack_bf16x2(v[8 * c + 6], v[8 * c + 7]));
     *reinterpret_cast<uint4*>(prow + ((c8 ^ (row & 7)) << 4)) = u;
@@ -64,17 +85,17 @@ __device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const
 // Same fp32 ops in the same order as the staged-fp32 path: the bf16 result is bitwise identical.
 __device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const float2* cs,
                                                 int pos, bool rope) {
-  uint32_t a[32], b[32];
-  tmem_ld32_nw(tacc + 32 * g, a);
-  tmem_ld32_nw(tacc + 64 + 32 * g, b);
+  uint32_t a[CPT], b[CPT];
+  tmem_ldc_nw(tacc + CPT * g, a);
+  tmem_ldc_nw(tacc + 64 + CPT * g, b);
   tmem_wait_ld();
-  float x[32], y[32];
+  float x[CPT], y[CPT];
 #pragma unroll
-  for (int i = 0; i < 32; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
+  for (int i = 0; i < CPT; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
   if (rope) {   // dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
-    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + 32 * g);
+    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + CPT * g);
 #pragma unroll
-    for (int i = 0; i < 16; ++i) {
+    for (int i = 0; i < CPT / 2; ++i) {
       const float4 e = __ldg(c4 + i);   // (c_2i, s_2i, c_2i+1, s_2i+1)
       const float x0 = x[2 * i] * e.x + y[2 * i] * e.y, y0 = y[2 * i] * e.x - x[2 * i] * e.y;
       const float x1 = x[2 * i + 1] * e.z + y[2 * i + 1] * e.w, y1 = y[2 * i + 1] * e.z - x[2 * i + 1] * e.w;
@@ -83,13 +104,13 @@ __device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int
   }
   uint8_t* row = stg + rr * 256;
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
+  for (int c = 0; c < CPT / 8; ++c) {
     const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
                                 pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
     const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
                                 pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
-    *reinterpret_cast<uint4*>(row + (((4 * g + c) ^ (rr & 15)) << 4)) = ux;
-    *reinterpret_cast<uint4*>(row + (((8 + 4 * g + c) ^ (rr & 15)) << 4)) = uy;
+    *reinterpret_cast<uint4*>(row + ((((CPT / 8) * g + c) ^ (rr & 15)) << 4)) = ux;
+    *reinterpret_cast<uint4*>(row + (((8 + (CPT / 8) * g + c) ^ (rr & 15)) << 4)) = uy;
   }
 }
 // n_tiles staged bf16 tiles (32 KB apart) -> rows [0, n_valid) of dst[t] (row stride ld), 16 lanes per 256-B row
@@ -97,8 +118,8 @@ __device__ __forceinline__ void stage16_store(const uint8_t* stg, int n_tiles, i
                                               bf16* dst0, bf16* dst1, int ld) {
   const int k = lane & 15;
 #pragma unroll 4
-  for (int i = 0; i < 8 * n_tiles; ++i) {
-    const int R = i * 16 + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
+  for (int i = 0; i < 128 * n_tiles / (2 * EW_WARPS); ++i) {
+    const int R = i * (2 * EW_WARPS) + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
     if (rr >= n_valid) continue;
     const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 32768 + rr * 256 + ((k ^ (rr & 15)) << 4));
     *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * ld + k * 8) = v;
@@ -267,7 +288,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     BP_FLUSH(blockIdx.x < 8 && lane == 0);
   } else {
     // ------------------------------------------------ elementwise warps (thread = key row = TMEM lane;
-    //                                                  warpgroup g owns query columns [32 g, 32 g + 32))
+    //                                                  warp group g owns query columns [CPT g, CPT g + CPT))
     const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
     const int r = w4 * 32 + lane;           // key row within the block
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
@@ -304,18 +325,18 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         BP(2);
         tc_fence_after();
         __syncwarp();
-        uint32_t su[32], du[32];
-        tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
-        tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+        uint32_t su[CPT], du[CPT];
+        tmem_ldc_nw(tmem + 64 * b + CPT * g + lane_off, su);
+        tmem_ldc_nw(tmem + 128 + 64 * b + CPT * g + lane_off, du);
         tmem_wait_ld();
-        const int cmin = kpos - q0 - 32 * g;   // P = 0 for queries before the key (causal) ...
-        const int cmax = L - q0 - 32 * g;      // ... and past the end of the sequence
-        const bool full = cmin <= 0 && cmax >= 32;   // interior block: no mask in this row half
-        float pv[32], dsv[32];
+        const int cmin = kpos - q0 - CPT * g;   // P = 0 for queries before the key (causal) ...
+        const int cmax = L - q0 - CPT * g;      // ... and past the end of the sequence
+        const bool full = cmin <= 0 && cmax >= CPT;   // interior block: no mask in this row's columns
+        float pv[CPT], dsv[CPT];
 #pragma unroll
-        for (int c4 = 0; c4 < 32; c4 += 4) {
-          const float4 lz = *reinterpret_cast<const float4*>(&s_lse[b][32 * g + c4]);
-          const float4 dz = *reinterpret_cast<const float4*>(&s_D[b][32 * g + c4]);
+        for (int c4 = 0; c4 < CPT; c4 += 4) {
+          const float4 lz = *reinterpret_cast<const float4*>(&s_lse[b][CPT * g + c4]);
+          const float4 dz = *reinterpret_cast<const float4*>(&s_D[b][CPT * g + c4]);
           const float lzv[4] = {lz.x, lz.y, lz.z, lz.w}, dzv[4] = {dz.x, dz.y, dz.z, dz.w};
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
@@ -498,7 +519,7 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       __syncwarp();
     }
   } else {
-    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2;   // warpgroup g owns key columns [32 g, 32 g + 32)
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2;   // warp group g owns key columns [CPT g, CPT g + CPT)
     const int r = w4 * 32 + lane;           // query row
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_W;
@@ -517,18 +538,18 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         wait_bar(&s_full[b], (gb >> 1) & 1);
         tc_fence_after();
         __syncwarp();
-        uint32_t su[32], du[32];
-        tmem_ld32_nw(tmem + 64 * b + 32 * g + lane_off, su);
-        tmem_ld32_nw(tmem + 128 + 64 * b + 32 * g + lane_off, du);
+        uint32_t su[CPT], du[CPT];
+        tmem_ldc_nw(tmem + 64 * b + CPT * g + lane_off, su);
+        tmem_ldc_nw(tmem + 128 + 64 * b + CPT * g + lane_off, du);
         tmem_wait_ld();
-        const int cmax = qok ? qpos - j * KB - 32 * g : -1;   // keys <= query
-        float dsv[32];
+        const int cmax = qok ? qpos - j * KB - CPT * g : -1;   // keys <= query
+        float dsv[CPT];
 #pragma unroll
-        for (int c = 0; c < 32; ++c) {
+        for (int c = 0; c < CPT; ++c) {
           const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
           const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
           const float v = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
-          dsv[c] = (cmax >= 31 || c <= cmax) ? v : 0.f;
+          dsv[c] = (cmax >= CPT - 1 || c <= cmax) ? v : 0.f;
         }
         if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
         st_half_row(sS0 + b * DS_TILE, r, g, dsv);
