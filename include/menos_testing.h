@@ -41,7 +41,7 @@ MENOS_API int menos_test_rmsnorm(int T, int d, const float* x, const float* g, f
                                  const void* dy, const float* resid, float* dx, void* dxb);
 
 /* Copy one saved intermediate of a live SAVE batch to host (debugging / white-box tests).
- * which: 0 x, 1 xn, 2 qkv, 3 O, 4 h, 5 hn, 6 gu, 7 a, 8 U_qkv, 9 U_o, 10 U_gu, 11 U_down (bf16), 12 lse (fp32 [H,T]).
+ * which: 0 x, 1 xn, 2 qkv, 3 O, 4 h, 5 hn, 6 gu (Llama: warp-tile order, see gu_tile_off in gemm_tcgen05.cu), 7 a, 8 U_qkv, 9 U_o, 10 U_gu, 11 U_down (bf16), 12 lse (fp32 [H,T]).
  * *bytes receives the size; host_out may be NULL to query it. */
 MENOS_API int menos_test_batch_tensor(menos_server* s, menos_batch* b, int layer, int which, void* host_out,
                                       size_t* bytes);

@@ -20,7 +20,7 @@ SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"),
-         "--expt-relaxed-constexpr"]
+         "--expt-relaxed-constexpr"] + os.environ.get("MENOS_NVCC_DEFS", "").split()   # tuning variants only
 
 
 def _stale(obj: str, srcs: list[str]) -> bool:

@@ -19,8 +19,8 @@ enum EpiMode : int {
   EPI_STORE = 0,       // out = bf16(acc)
   EPI_RESID = 1,       // outf = acc + residf   (fp32 residual stream; resid == nullptr: outf = acc)
   EPI_ROPE = 2,        // columns < rope_cols rotated by RoPE at pos[row]; out = bf16
-  EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu), out2 = bf16(silu(g) u)
-  EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu; out = dgu (interleaved like gu)
+  EPI_SWIGLU_FWD = 3,  // tile = [128 gate | 128 up]: out = bf16(acc) (saved gu, warp-tile order, see gu_tile_off), out2 = bf16(silu(g) u)
+  EPI_SWIGLU_BWD = 4,  // acc = da over f columns; aux = saved gu (warp-tile order); out = dgu (row-major, interleaved like gu)
   EPI_RELU_FWD = 5,    // OPT fc1: out = bf16(relu(acc + bias))
   EPI_RELU_BWD = 6,    // OPT fc2 dX: out = bf16(acc * (aux > 0)), aux = saved relu output
   EPI_STORE_DSUM = 7,  // o-proj dX: out = dO = bf16(acc), and per head h of width dsum_hd (% 32 == 0):

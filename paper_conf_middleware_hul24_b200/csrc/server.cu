@@ -1564,7 +1564,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     else K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
   }
   // A10: O dX (+ LoRA o) -> dO (and, for head_dim % 32 == 0, the attention backward's row sums D)
-  const bool fuse_dsum = D.hd % 32 == 0;
+  const bool fuse_dsum = D.hd % 32 == 0 && 128 % D.hd == 0;
   if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
   {
     GemmArgs a = gemm_base(s);

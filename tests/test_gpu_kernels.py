@@ -203,8 +203,20 @@ def test_gemm_rope_epilogue(hd, H, Hkv):
     assert maxrel(host(out), ref) < 1e-2
 
 
+def untile_gu(buf):
+    """Saved g|u is stored in warp-tile order (gemm_tcgen05.cu gu_tile_off): rows in groups of 32 (n rows in the
+    tail group), inside a group the 16-byte unit (row, col // 8) at group_base + ((col // 8) * n + row % 32) * 8."""
+    T, W = buf.shape
+    flat, out = buf.reshape(-1), np.empty_like(buf)
+    for g0 in range(0, T, 32):
+        n = min(32, T - g0)
+        blk = flat[g0 * W:(g0 + n) * W].reshape(W // 8, n, 8)      # [unit, row, 8]
+        out[g0:g0 + n] = blk.transpose(1, 0, 2).reshape(n, W)
+    return out
+
+
 def test_gemm_swiglu_fwd_and_bwd_epilogues():
-    T, d, f = 260, 128, 256     # f multiple of 128; interleaved gu layout [128 gate | 128 up] per block
+    T, d, f = 260, 128, 384     # f multiple of 128 (the last da tile is half full); interleaved gu layout [128 gate | 128 up] per block
     x = rnd((T, d), 41)
     Wg, Wu = rnd((f, d), 42, 0.1), rnd((f, d), 43, 0.1)
     Wgu = np.zeros((2 * f, d), np.float32)
@@ -221,7 +233,7 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     dy, Wd = rnd((T, dout), 44), rnd((dout, f), 45, 0.1)
     dgu = torch.empty(T, 2 * f, dtype=torch.bfloat16, device="cuda")
     gemm(T, f, dout, 1, dev(dy), dev(Wd), epi=4, out=dgu, aux=gu, ldaux=2 * f, ldo=2 * f)
-    gu_h = host(gu)
+    gu_h = untile_gu(host(gu))
     g_b = np.concatenate([gu_h[:, fb * 256:fb * 256 + 128] for fb in range(f // 128)], 1)
     u_b = np.concatenate([gu_h[:, fb * 256 + 128:fb * 256 + 256] for fb in range(f // 128)], 1)
     dg, du = O.swiglu_bwd(dy @ Wd, g_b, u_b)

@@ -11,12 +11,8 @@
 // * CG = 2 (default): a CTA pair (cluster of 2, cta_group::2) computes a 256 x 256 tile with one M=256 UMMA per
 //   K=16 step; each CTA stages its 128 rows of A and its 128-column half of B (halving the smem traffic per SM).
 //   CG = 1: one CTA computes 128 x 256.
-// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread, leader CTA), warps 2.. = EPW epilogue
-//   warps (TMEM -> registers -> fused epilogue -> global).  EPW = 4 (default): one warp per TMEM lane quadrant;
-//   EPW = 8 (-DMENOS_GEMM_EPW=8): two per quadrant, each owning 128 of the tile's 256 columns (measured 4% faster
-//   on the SwiGLU-bwd epilogue but capped at 168 registers and spilling, so not the default).  Epilogues that read
-//   HBM (SwiGLU bwd, D row sums) issue the next chunk's loads before the current chunk's TMEM load.  Two TMEM
-//   accumulators (2 x 256 fp32 columns) let the
+// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread, leader CTA), warps 2-5 = epilogue
+//   (TMEM -> registers -> fused epilogue -> global).  Two TMEM accumulators (2 x 256 fp32 columns) let the
 //   epilogue of tile i overlap the MMAs of tile i+1.  Persistent grid; tiles rasterised in groups of 16
 //   M-tiles so a wave's A rows and B panels stay L2-resident.
 #include <mutex>
@@ -29,12 +25,7 @@ namespace menos {
 
 namespace {
 constexpr int BM = 128, BN = 256, BK = 64;
-#ifndef MENOS_GEMM_EPW
-#define MENOS_GEMM_EPW 4
-#endif
-constexpr int EPW = MENOS_GEMM_EPW;           // epilogue warps (4 or 8): 1 or 2 per TMEM lane quadrant
-constexpr int NTHREADS = 64 + 32 * EPW;
-constexpr int EPC = 8 / (EPW / 4);            // 32-column chunks of a 256-column tile per epilogue warp
+constexpr int NTHREADS = 192;
 constexpr int GROUP_M = 16;
 
 template <int CG> struct Cfg {
@@ -101,26 +92,6 @@ __device__ __forceinline__ void load32(const bf16* src, float (&v)[32]) {
     v[8 * q + 4] = c.x; v[8 * q + 5] = c.y; v[8 * q + 6] = d.x; v[8 * q + 7] = d.y;
   }
 }
-// Saved SwiGLU inputs g|u live in WARP-TILE order: rows in groups of 32 (one epilogue warp's rows);
-// inside a group of n rows (32, or T % 32 for the tail group) the 16-byte unit (row, 8-column unit col/8) sits at
-// group_base + ((col/8) * n + row % 32) * 8 elements.  One warp instruction over its 32 rows then touches 512
-// contiguous bytes, where the row-major layout touched 32 rows x 16 B (two requests per 32-byte sector).  Only the
-// SwiGLU forward epilogue writes this buffer and only the SwiGLU backward epilogue reads it.
-__device__ __forceinline__ size_t gu_tile_off(int row, int col, int T, int W) {
-  const int g0 = row & ~31, n = min(32, T - g0);
-  return (size_t)g0 * W + ((size_t)(col >> 3) * n + (row & 31)) * 8;
-}
-__device__ __forceinline__ void store32_tiled(bf16* base, int row, int col, int T, int W, const float (&v)[32]) {
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    uint4 u;
-    u.x = pack_bf16x2(v[8 * q + 0], v[8 * q + 1]);
-    u.y = pack_bf16x2(v[8 * q + 2], v[8 * q + 3]);
-    u.z = pack_bf16x2(v[8 * q + 4], v[8 * q + 5]);
-    u.w = pack_bf16x2(v[8 * q + 6], v[8 * q + 7]);
-    *reinterpret_cast<uint4*>(base + gu_tile_off(row, col + 8 * q, T, W)) = u;
-  }
-}
 // RoPE inside one 32-column chunk for head_dim = 2*HALF <= 32 (pairs (j, j+HALF) of each head)
 template <int HALF>
 __device__ __forceinline__ void rope_small(const float (&v)[32], float (&o)[32], const float2* cs) {
@@ -184,7 +155,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     tma_prefetch(&tmA); tma_prefetch(&tmB);
     if (p.R > 0) { tma_prefetch(&tmA2); tma_prefetch(&tmB2); }
     for (int s = 0; s < C::STAGES; ++s) { mbar_init(&full_bar[s], 1); mbar_init(&empty_bar[s], 1); }
-    for (int s = 0; s < 2; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], EPW * CG); }
+    for (int s = 0; s < 2; ++s) { mbar_init(&tfull_bar[s], 1); mbar_init(&tempty_bar[s], 4 * CG); }
     fence_barrier_init();
   }
   if (warp == 1) {
@@ -299,9 +270,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else {
-    // ------------------------------------------------ epilogue warps 2..9 (both CTAs)
+    // ------------------------------------------------ epilogue warps 2..5 (both CTAs)
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
-    const int cb = ((warp - 2) >> 2) * EPC, ce = cb + EPC;   // this warp's 32-column chunks [cb, ce)
     int acc = 0; uint32_t acc_phase = 0;
     for (int t = cluster_id; t < total; t += n_clusters) {
       int m, n;
@@ -310,24 +280,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         // L2 prefetch of the epilogue's HBM inputs for this row while the tile's MMAs still run: residual (fp32,
         // 8 x 128 B lines), saved g|u (SwiGLU bwd: 2 x 4 x 128 B) or relu output (4 x 128 B)
         const int prow = m * C::TILE_M + rank * BM + q * 32 + lane;
-        const int pn0 = n * BN + cb * 32, pn1 = min(n * BN + ce * 32, p.N);
+        const int pn0 = n * BN;
         if (prow < p.M) {
           if (p.epi == EPI_RESID && p.resid) {
-            const float* r = p.resid + (size_t)prow * p.ldr;
-            for (int col = pn0; col < pn1; col += 32) prefetch_l2(r + col);
+            const float* r = p.resid + (size_t)prow * p.ldr + pn0;
+            for (int c = 0; c < 8 && pn0 + c * 32 < p.N; ++c) prefetch_l2(r + c * 32);
           } else if (p.epi == EPI_SWIGLU_BWD) {
-            // per 128-column block, this warp's g and its u are two contiguous runs (warp-tile order): the lanes
-            // prefetch them line by line
-            const int r0 = prow & ~31, nrow = min(32, p.M - r0);
-            for (int col = pn0; col < pn1; col += 128) {
-              const int gcol = (col >> 7) * 256 + (col & 127);
-              const int run = min(128, pn1 - col) * nrow;   // elements
-              const bf16* g = p.aux + gu_tile_off(r0, gcol, p.M, 2 * p.N);
-              for (int e = lane * 64; e < run; e += 32 * 64) { prefetch_l2(g + e); prefetch_l2(g + 128 * nrow + e); }
+            for (int h = 0; h < 2 && pn0 + h * 128 < p.N; ++h) {
+              const bf16* a = p.aux + (size_t)prow * p.ldaux + ((pn0 + h * 128) >> 7) * 256;
+              for (int c = 0; c < 2; ++c) { prefetch_l2(a + c * 64); prefetch_l2(a + 128 + c * 64); }
             }
           } else if (p.epi == EPI_RELU_BWD || p.epi == EPI_STORE_DSUM) {
-            const bf16* a = p.aux + (size_t)prow * p.ldaux;
-            for (int col = pn0; col < pn1; col += 64) prefetch_l2(a + col);
+            const bf16* a = p.aux + (size_t)prow * p.ldaux + pn0;
+            for (int c = 0; c < 4 && pn0 + c * 64 < p.N; ++c) prefetch_l2(a + c * 64);
           }
         }
       }
@@ -338,7 +303,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const uint32_t tb = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
       const int n0 = n * BN;
       if (p.epi == EPI_STORE) {
-        for (int c = cb; c < cb + EPC; ++c) {
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
           float v[32];
@@ -347,38 +312,18 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
         }
       } else if (p.epi == EPI_STORE_DSUM) {
-        // the next chunk's O loads are issued before this chunk's TMEM load (see EPI_SWIGLU_BWD)
-        const int cl = min(cb + EPC, (p.N - n0 + 31) / 32);
-        uint4 oq[4];
-        auto ld_o = [&](int c, uint4 (&r)[4]) {
-          const uint4* a = reinterpret_cast<const uint4*>(p.aux + (size_t)row * p.ldaux + n0 + c * 32);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) r[i] = a[i];
-        };
-        if (rok && cb < cl) ld_o(cb, oq);
         float dot = 0.f;
-#pragma unroll 1
-        for (int c = cb; c < cl; ++c) {
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
-          uint4 o0[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) o0[i] = oq[i];
-          if (rok && c + 1 < cl) ld_o(c + 1, oq);
+          if (col >= p.N) break;
           float v[32];
           tmem_ld32(tb + c * 32, v);
           if (rok) {
+            float o[32];
+            load32(p.aux + (size_t)row * p.ldaux + col, o);
             store32(p.out + (size_t)row * p.ldo + col, v);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              const uint32_t ow[4] = {o0[i].x, o0[i].y, o0[i].z, o0[i].w};
-#pragma unroll
-              for (int h = 0; h < 4; ++h) {
-                const float2 o2 = unpack_bf16x2(ow[h]);
-                const int j = 8 * i + 2 * h;
-                dot += __bfloat162float(__float2bfloat16_rn(v[j])) * o2.x;
-                dot += __bfloat162float(__float2bfloat16_rn(v[j + 1])) * o2.y;
-              }
-            }
+            for (int j = 0; j < 32; ++j) dot += __bfloat162float(__float2bfloat16_rn(v[j])) * o[j];
             if ((col + 32) % p.dsum_hd == 0) {
               p.dsum[(size_t)(col / p.dsum_hd) * p.dsum_ld + row] = dot;
               dot = 0.f;
@@ -386,7 +331,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           }
         }
       } else if (p.epi == EPI_RELU_FWD) {
-        for (int c = cb; c < cb + EPC; ++c) {
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
           float v[32];
@@ -397,7 +342,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (rok) store32(p.out + (size_t)row * p.ldo + col, v);
         }
       } else if (p.epi == EPI_RELU_BWD) {
-        for (int c = cb; c < cb + EPC; ++c) {
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
           float v[32];
@@ -413,17 +358,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       } else if (p.epi == 99 || p.epi == 98) {
         // tuning aid: drain TMEM without storing (isolates the mainloop)
         float sink = 0.f;
-        for (int c = cb; c < cb + EPC; ++c) {
+        for (int c = 0; c < 8; ++c) {
           float v[32];
           tmem_ld32(tb + c * 32, v);
-          sink += v[0] + v[31];
+          sink += v[c];
         }
         if (sink == 12345.678f) p.out[0] = f2bf(sink);
       } else if (p.epi == EPI_RESID) {
         // fp32 residual stream: outf = acc (+ bias) + resid.  The chunk's 8 residual loads are all issued before
         // the TMEM load and before any store: outf and resid may alias as far as the compiler knows, so loads
         // interleaved with the stores would serialise into 8 HBM round trips per chunk.
-        for (int c = cb; c < cb + EPC; ++c) {
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
           if (col >= p.N) break;
           float r[32];
@@ -455,7 +400,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         const int ps = rok ? p.pos[row] : 0;
         const float2* cs = p.rope_cs + (size_t)ps * half;
         if (half >= 32) {
-          for (int c = cb; c < cb + EPC; ++c) {
+          for (int c = 0; c < 8; ++c) {
             const int col = n0 + c * 32;
             if (col >= p.N) break;
             if ((col % hd) >= half) continue;           // handled as a partner chunk
@@ -479,7 +424,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             }
           }
         } else {
-          for (int c = cb; c < cb + EPC; ++c) {
+          for (int c = 0; c < 8; ++c) {
             const int col = n0 + c * 32;
             if (col >= p.N) break;
             float v[32], o[32];
@@ -496,13 +441,13 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         }
       } else if (p.epi == EPI_SWIGLU_FWD) {
         // tile = [128 gate | 128 up] of f block n; a[:, n*128 + j] = silu(g_j) * u_j
-        for (int c = cb / 2; c < cb / 2 + EPC / 2; ++c) {
+        for (int c = 0; c < 4; ++c) {
           float g[32], u[32];
           tmem_ld32(tb + c * 32, g);
           tmem_ld32(tb + (c + 4) * 32, u);
           if (rok) {
-            store32_tiled(p.out, row, n0 + c * 32, p.M, p.N, g);          // saved g|u: warp-tile order
-            store32_tiled(p.out, row, n0 + 128 + c * 32, p.M, p.N, u);
+            store32(p.out + (size_t)row * p.ldo + n0 + c * 32, g);
+            store32(p.out + (size_t)row * p.ldo + n0 + 128 + c * 32, u);
             float a[32];
 #pragma unroll
             for (int j = 0; j < 32; ++j) a[j] = g[j] * sigmoidf_(g[j]) * u[j];
@@ -510,47 +455,27 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           }
         }
       } else if (p.epi == EPI_SWIGLU_BWD) {
-        // acc = da over f columns; gu saved interleaved in 128-blocks: g at fb*256+jj, u at fb*256+128+jj.
-        // The next chunk's g|u loads are issued before this chunk's TMEM load: the TMEM wait is a compiler memory
-        // barrier, so without this each chunk's HBM round trip would serialise behind the previous chunk.
-        const int cl = min(cb + EPC, (p.N - n0 + 31) / 32);
-        uint4 gq[4], uq[4];
-        auto ld_gu = [&](int c, uint4 (&gr)[4], uint4 (&ur)[4]) {
-          const int col = n0 + c * 32, gcol = (col >> 7) * 256 + (col & 127);   // g column; u is 128 further
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            gr[i] = *reinterpret_cast<const uint4*>(p.aux + gu_tile_off(row, gcol + 8 * i, p.M, 2 * p.N));
-            ur[i] = *reinterpret_cast<const uint4*>(p.aux + gu_tile_off(row, gcol + 128 + 8 * i, p.M, 2 * p.N));
-          }
-        };
-        if (rok && cb < cl) ld_gu(cb, gq, uq);
-#pragma unroll 1
-        for (int c = cb; c < cl; ++c) {
+        // acc = da over f columns; gu saved interleaved in 128-blocks: g at fb*256+jj, u at fb*256+128+jj
+        for (int c = 0; c < 8; ++c) {
           const int col = n0 + c * 32;
-          uint4 g0[4], u0[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) { g0[i] = gq[i]; u0[i] = uq[i]; }
-          if (rok && c + 1 < cl) ld_gu(c + 1, gq, uq);
+          if (col >= p.N) break;
           float da[32];
           tmem_ld32(tb + c * 32, da);
           if (rok) {
             const int fb = col >> 7, jj = col & 127;
-            uint4* og = reinterpret_cast<uint4*>(p.out + (size_t)row * p.ldo + fb * 256 + jj);
+            const size_t gofs = (size_t)row * p.ldaux + fb * 256 + jj;
+            float g[32], u[32], dg[32], du[32];
+            load32(p.aux + gofs, g);
+            load32(p.aux + gofs + 128, u);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {   // 8 columns at a time: packed straight into the 16-byte stores
-              const uint32_t gw[4] = {g0[i].x, g0[i].y, g0[i].z, g0[i].w}, uw[4] = {u0[i].x, u0[i].y, u0[i].z, u0[i].w};
-              uint32_t dgw[4], duw[4];
-#pragma unroll
-              for (int h = 0; h < 4; ++h) {
-                const float2 g2 = unpack_bf16x2(gw[h]), u2 = unpack_bf16x2(uw[h]);
-                const float d0 = da[8 * i + 2 * h], d1 = da[8 * i + 2 * h + 1];
-                const float s0 = sigmoidf_(g2.x), s1 = sigmoidf_(g2.y);
-                dgw[h] = pack_bf16x2(d0 * u2.x * s0 * (1.0f + g2.x * (1.0f - s0)), d1 * u2.y * s1 * (1.0f + g2.y * (1.0f - s1)));
-                duw[h] = pack_bf16x2(d0 * g2.x * s0, d1 * g2.y * s1);
-              }
-              og[i] = make_uint4(dgw[0], dgw[1], dgw[2], dgw[3]);
-              og[16 + i] = make_uint4(duw[0], duw[1], duw[2], duw[3]);
+            for (int j = 0; j < 32; ++j) {
+              const float sg = sigmoidf_(g[j]);
+              dg[j] = da[j] * u[j] * sg * (1.0f + g[j] * (1.0f - sg));
+              du[j] = da[j] * g[j] * sg;
             }
+            const size_t oofs = (size_t)row * p.ldo + fb * 256 + jj;
+            store32(p.out + oofs, dg);
+            store32(p.out + oofs + 128, du);
           }
         }
       }
@@ -665,10 +590,7 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
   if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;
   if ((a.epi == EPI_SWIGLU_FWD && a.N % 256) || (a.epi == EPI_SWIGLU_BWD && a.N % 128)) return -1;
-  // the epilogue warps split a tile's 256 columns in 128-column halves: a head (RoPE pairs, D row sums) must not
-  // straddle two halves
-  if (a.epi == EPI_STORE_DSUM && (a.dsum_hd <= 0 || a.dsum_hd % 32 || 128 % a.dsum_hd || !a.dsum || !a.aux)) return -1;
-  if (a.epi == EPI_ROPE && (a.head_dim <= 0 || 128 % a.head_dim)) return -1;
+  if (a.epi == EPI_STORE_DSUM && (a.dsum_hd <= 0 || a.dsum_hd % 32 || !a.dsum || !a.aux)) return -1;
   const int CG = g_gemm_cta_group == 1 ? 1 : 2;
   const uint32_t bbox = BN / CG;  // B rows (K-major) staged per CTA
   CUtensorMap mA, mB, mA2, mB2;

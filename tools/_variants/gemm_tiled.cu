@@ -11,12 +11,10 @@
 // * CG = 2 (default): a CTA pair (cluster of 2, cta_group::2) computes a 256 x 256 tile with one M=256 UMMA per
 //   K=16 step; each CTA stages its 128 rows of A and its 128-column half of B (halving the smem traffic per SM).
 //   CG = 1: one CTA computes 128 x 256.
-// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread, leader CTA), warps 2.. = EPW epilogue
-//   warps (TMEM -> registers -> fused epilogue -> global).  EPW = 4 (default): one warp per TMEM lane quadrant;
-//   EPW = 8 (-DMENOS_GEMM_EPW=8): two per quadrant, each owning 128 of the tile's 256 columns (measured 4% faster
-//   on the SwiGLU-bwd epilogue but capped at 168 registers and spilling, so not the default).  Epilogues that read
-//   HBM (SwiGLU bwd, D row sums) issue the next chunk's loads before the current chunk's TMEM load.  Two TMEM
-//   accumulators (2 x 256 fp32 columns) let the
+// * Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer (one thread, leader CTA), warps 2-9 = epilogue
+//   (TMEM -> registers -> fused epilogue -> global); two warps per TMEM lane quadrant, each owning 128 of the
+//   tile's 256 columns, so the epilogues that read HBM (SwiGLU bwd, residual, D row sums) have twice the loads in
+//   flight per row.  Two TMEM accumulators (2 x 256 fp32 columns) let the
 //   epilogue of tile i overlap the MMAs of tile i+1.  Persistent grid; tiles rasterised in groups of 16
 //   M-tiles so a wave's A rows and B panels stay L2-resident.
 #include <mutex>
@@ -30,7 +28,7 @@ namespace menos {
 namespace {
 constexpr int BM = 128, BN = 256, BK = 64;
 #ifndef MENOS_GEMM_EPW
-#define MENOS_GEMM_EPW 4
+#define MENOS_GEMM_EPW 8
 #endif
 constexpr int EPW = MENOS_GEMM_EPW;           // epilogue warps (4 or 8): 1 or 2 per TMEM lane quadrant
 constexpr int NTHREADS = 64 + 32 * EPW;
