@@ -1,6 +1,6 @@
 // Segmented multi-client LoRA side contractions (SURVEY.md §8(a) A2/A4/A6/A7 shrink, A8-A12 LoRA backward).
 //
-//   rows kernel (one client's 64-token block, full reduction):
+//   rows kernel (one client's ROWS_BM-token block, full reduction):
 //     shrink   U_c  = s_c * X_c A_c^T      (B operand = A_cat rows   [W, K], "nk")
 //     dU       dU_c = s_c * dY_c B_c       (B operand = B_cat        [K, W], "kn")
 //   token-reduction kernel (reduce over ONE client's tokens, fixed order -> deterministic, no atomics):
@@ -29,12 +29,18 @@ __device__ __forceinline__ int tsw(int row, int chunk) {
 // C[t, j] = scale * sum_k A[t, k] * Bop(j, k) for t in [m0, m0+64), j in [0, NT)
 // 4-stage cp.async ring of 128-wide K tiles: ~96-192 KB of X / dY in flight per SM, enough to stream the
 // activations at HBM rate with one CTA per 64-token block.
-constexpr int ROWS_BM = 64, ROWS_BK = 128, ROWS_STAGES = 4;
+#ifndef MENOS_LORA_ROWS_BM
+#define MENOS_LORA_ROWS_BM 64
+#endif
+// ROWS_BM tokens per CTA, one warp per 16 of them.  64 (default) vs 32 measured at cfg1 shapes
+// (profiles/r1n_lora_rows_bm.txt): 32-token blocks double the CTAs but each CTA still re-stages the whole
+// [N, K] adapter operand from L2, so the shrink is no faster and the per-target dU is 38% slower.
+constexpr int ROWS_BM = MENOS_LORA_ROWS_BM, ROWS_BK = 128, ROWS_STAGES = 4, ROWS_NTH = ROWS_BM / 16 * 32;
 template <int NT>
 constexpr int rows_smem_bytes() { return ROWS_STAGES * (ROWS_BM + NT) * ROWS_BK * 2; }
 
 template <int NT>
-__global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* __restrict__ probs,
+__global__ void __launch_bounds__(ROWS_NTH) lora_rows_kernel(const LoraRowsProblem* __restrict__ probs,
                                                         const int2* __restrict__ tiles) {
   constexpr int BM = ROWS_BM, BK = ROWS_BK, NNT = NT / 8, NS = ROWS_STAGES;
   extern __shared__ __align__(128) uint8_t rows_smem[];
@@ -48,21 +54,21 @@ __global__ void __launch_bounds__(128) lora_rows_kernel(const LoraRowsProblem* _
   auto load = [&](int buf, int k0) {
     bf16* As = As_base + buf * BM * BK;
     bf16* Bs = Bs_base + buf * NT * BK;
-    for (int i = tid; i < BM * (BK / 8); i += 128) {
+    for (int i = tid; i < BM * (BK / 8); i += ROWS_NTH) {
       const int r = i / (BK / 8), c = i % (BK / 8);
       const int gr = m0 + r, gk = k0 + c * 8;
       const bool ok = gr < P.M && gk < P.K;
       cp_async16(smem_u32(&As[tsw<BK>(r, c)]), P.A + (ok ? (size_t)gr * P.lda + gk : 0), ok ? 16 : 0);
     }
     if (!P.b_kn) {
-      for (int i = tid; i < NT * (BK / 8); i += 128) {
+      for (int i = tid; i < NT * (BK / 8); i += ROWS_NTH) {
         const int r = i / (BK / 8), c = i % (BK / 8);
         const int gk = k0 + c * 8;
         const bool ok = r < P.N && gk < P.K;
         cp_async16(smem_u32(&Bs[tsw<BK>(r, c)]), P.B + (ok ? (size_t)r * P.ldb + gk : 0), ok ? 16 : 0);
       }
     } else {
-      for (int i = tid; i < BK * (NT / 8); i += 128) {
+      for (int i = tid; i < BK * (NT / 8); i += ROWS_NTH) {
         const int r = i / (NT / 8), c = i % (NT / 8);
         const int gk = k0 + r;
         const bool ok = gk < P.K && c * 8 < P.N;
@@ -233,7 +239,7 @@ __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProble
 
 void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out) {
   for (int i = 0; i < n; ++i)
-    for (int m = 0; m < probs[i].M; m += 64) out.push_back(make_int2(i, m));
+    for (int m = 0; m < probs[i].M; m += ROWS_BM) out.push_back(make_int2(i, m));
 }
 void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out) {
   for (int i = 0; i < n; ++i)
@@ -250,9 +256,9 @@ int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_til
     cudaFuncSetAttribute(lora_rows_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem_bytes<128>());
     attr = true;
   }
-  if (max_n <= 32) lora_rows_kernel<32><<<n_tiles, 128, rows_smem_bytes<32>(), st>>>(d_probs, d_tiles);
-  else if (max_n <= 64) lora_rows_kernel<64><<<n_tiles, 128, rows_smem_bytes<64>(), st>>>(d_probs, d_tiles);
-  else if (max_n <= 128) lora_rows_kernel<128><<<n_tiles, 128, rows_smem_bytes<128>(), st>>>(d_probs, d_tiles);
+  if (max_n <= 32) lora_rows_kernel<32><<<n_tiles, ROWS_NTH, rows_smem_bytes<32>(), st>>>(d_probs, d_tiles);
+  else if (max_n <= 64) lora_rows_kernel<64><<<n_tiles, ROWS_NTH, rows_smem_bytes<64>(), st>>>(d_probs, d_tiles);
+  else if (max_n <= 128) lora_rows_kernel<128><<<n_tiles, ROWS_NTH, rows_smem_bytes<128>(), st>>>(d_probs, d_tiles);
   else return -1;
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
