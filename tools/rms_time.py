@@ -3,8 +3,10 @@ Each call ends in a device sync, so the per-call time includes one launch + sync
 Prints one JSON line: us per fwd, us per bwd (fwd+bwd minus fwd), and GB/s against DESIGN's algorithmic bytes
 (fwd 6d+4 B/token, bwd 16d+4 B/token with the bf16 copy)."""
 import json
+import os
 import sys
 import torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_middleware_hul24_b200.menos import lib, check
 
 T, d = (int(a) for a in sys.argv[1:3]) if len(sys.argv) > 2 else (8192, 4096)
