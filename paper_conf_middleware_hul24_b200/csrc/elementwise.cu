@@ -382,6 +382,9 @@ __global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __
 
 }  // namespace
 
+#ifndef MENOS_RMS_WIDE4K
+#define MENOS_RMS_WIDE4K 1
+#endif
 #define LAUNCH_CHECK() (++g_launch_count, cudaPeekAtLastError() == cudaSuccess ? 0 : -3)
 
 int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int d, float eps, cudaStream_t st) {
@@ -391,12 +394,13 @@ int rmsnorm_fwd(const float* x, const float* g, bf16* y, float* rstd, int T, int
   switch (nc) {  // single pass: the row stays in registers between the reduction and the write
     case 1: rmsnorm_fwd_reg_kernel<1, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
     case 2: rmsnorm_fwd_reg_kernel<2, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-#if MENOS_RMS_WIDE4K   // tuning variant: one row per 256 threads, 2 chunks per thread
+#if MENOS_RMS_WIDE4K   // one row per 256 threads, 2-3 chunks per thread (r1q: bwd 100 -> 80 us at 8192 x 4096)
     case 3: case 4: rmsnorm_fwd_reg_kernel<2, 256><<<T, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+    case 5: rmsnorm_fwd_reg_kernel<3, 256><<<T, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
 #else
     case 3: case 4: rmsnorm_fwd_reg_kernel<4, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
-#endif
     case 5: rmsnorm_fwd_reg_kernel<5, 128><<<g2, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
+#endif
     case 6: case 7: case 8: rmsnorm_fwd_reg_kernel<4, 256><<<T, 256, 0, st>>>(x, g, y, rstd, T, d, eps); break;
     default: {
       const int warps = 8;
@@ -416,10 +420,11 @@ static int rmsnorm_bwd_t(const TDY* dy, const float* x, const float* g, const fl
     case 2: rmsnorm_bwd_reg_kernel<2, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
 #if MENOS_RMS_WIDE4K
     case 3: case 4: rmsnorm_bwd_reg_kernel<2, 256, TDY><<<T, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+    case 5: rmsnorm_bwd_reg_kernel<3, 256, TDY><<<T, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
 #else
     case 3: case 4: rmsnorm_bwd_reg_kernel<4, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
-#endif
     case 5: rmsnorm_bwd_reg_kernel<5, 128, TDY><<<g2, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
+#endif
     case 6: case 7: case 8:   // wide rows (70B: d = 8192): one row per 256 threads keeps 4 chunks per thread
       rmsnorm_bwd_reg_kernel<4, 256, TDY><<<T, 256, 0, st>>>(dy, x, g, rstd, resid, dx, dxb, T, d); break;
     default: {
