@@ -278,48 +278,71 @@ __global__ void bf16_to_f32_kernel(const bf16* __restrict__ s, float* __restrict
 }
 
 // ------------------------------------------------------------------ LayerNorm (OPT, NEXT-4)
-// One warp per row, the row cached in registers (NCH 8-element chunks per lane, d <= 256 * NCH), two-pass
+// WPR warps per row, the row cached in registers (NCH 8-element chunks per lane, d <= 256 * WPR * NCH), two-pass
 // statistics in fp32.  fwd: y = (x - mu) * rstd * g + b.  bwd (+ residual; g, b frozen so no dg, db):
 // dx = resid + rstd * (gh - mean(gh) - xh * mean(gh * xh)), gh = dy * g, xh = (x - mu) * rstd; mu and rstd are
 // recomputed from x with the forward's own reduction order.
-template <int NCH>
-__device__ __forceinline__ void ln_stats(const float (&v)[NCH][8], int lane, int d, float eps, float& mu, float& r) {
+// WPR warps per row (1 for d <= 1024, 2 above: d = 2048 at one warp per row held 215 registers in the backward,
+// one CTA per SM); the row sums go warp_sum -> shared slots of the row's warps (fixed order), the same helper in
+// fwd and bwd so the backward's recomputed mu / rstd equal the forward's bit for bit.
+template <int WPR>
+__device__ __forceinline__ float ln_row_sum(float v, float* red) {
+  v = warp_sum(v);
+  if constexpr (WPR == 1) {
+    return v;
+  } else {
+    const int w = threadIdx.x >> 5, base = (w / WPR) * WPR;
+    if ((threadIdx.x & 31) == 0) red[w] = v;
+    __syncthreads();
+    float s = red[base];
+#pragma unroll
+    for (int k = 1; k < WPR; ++k) s += red[base + k];
+    __syncthreads();   // red is reused by the next reduction
+    return s;
+  }
+}
+
+template <int NCH, int WPR>
+__device__ __forceinline__ void ln_stats(const float (&v)[NCH][8], int tr, int d, float eps, float& mu, float& r,
+                                         float* red) {
   float s = 0.f;
 #pragma unroll
   for (int c = 0; c < NCH; ++c)
-    if ((c * 32 + lane) * 8 < d)
+    if ((c * 32 * WPR + tr) * 8 < d)
 #pragma unroll
       for (int k = 0; k < 8; ++k) s += v[c][k];
-  mu = warp_sum(s) / (float)d;
+  mu = ln_row_sum<WPR>(s, red) / (float)d;
   float q = 0.f;
 #pragma unroll
   for (int c = 0; c < NCH; ++c)
-    if ((c * 32 + lane) * 8 < d)
+    if ((c * 32 * WPR + tr) * 8 < d)
 #pragma unroll
       for (int k = 0; k < 8; ++k) { const float e = v[c][k] - mu; q += e * e; }
-  r = rsqrtf(warp_sum(q) / (float)d + eps);
+  r = rsqrtf(ln_row_sum<WPR>(q, red) / (float)d + eps);
 }
 
-template <int NCH>
-__global__ void layernorm_fwd_kernel(const float* __restrict__ x, const float* __restrict__ g,
-                                     const float* __restrict__ b, bf16* __restrict__ y, float* __restrict__ rstd,
-                                     int T, int d, float eps) {
-  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  if (row >= T) return;
-  const float* xr = x + (size_t)row * d;
+template <int NCH, int WPR>
+__global__ void __launch_bounds__(256) layernorm_fwd_kernel(const float* __restrict__ x, const float* __restrict__ g,
+                                                            const float* __restrict__ b, bf16* __restrict__ y,
+                                                            float* __restrict__ rstd, int T, int d, float eps) {
+  __shared__ float red[8];
+  const int row = blockIdx.x * (8 / WPR) + threadIdx.x / (32 * WPR), tr = threadIdx.x % (32 * WPR);
+  const bool ok = row < T;   // no early return: the row sums may synchronise the CTA
+  const float* xr = x + (size_t)(ok ? row : 0) * d;
   float v[NCH][8];
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int i = (c * 32 + lane) * 8;
+    const int i = (c * 32 * WPR + tr) * 8;
     if (i < d) ld8f(xr + i, v[c]);
   }
   float mu, r;
-  ln_stats<NCH>(v, lane, d, eps, mu, r);
-  if (lane == 0) rstd[row] = r;
+  ln_stats<NCH, WPR>(v, tr, d, eps, mu, r, red);
+  if (!ok) return;
+  if (tr == 0) rstd[row] = r;
   bf16* yr = y + (size_t)row * d;
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int i = (c * 32 + lane) * 8;
+    const int i = (c * 32 * WPR + tr) * 8;
     if (i >= d) continue;
     float gg[8], bb[8], o[8];
     ld8f(g + i, gg);
@@ -330,25 +353,27 @@ __global__ void layernorm_fwd_kernel(const float* __restrict__ x, const float* _
   }
 }
 
-template <int NCH, typename TDY>
-__global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
-                                     const float* __restrict__ g, const float* __restrict__ resid,
-                                     float* __restrict__ dx, bf16* __restrict__ dxb, int T, int d, float eps) {
-  const int row = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-  if (row >= T) return;
-  const size_t ro = (size_t)row * d;
+template <int NCH, int WPR, typename TDY>
+__global__ void __launch_bounds__(256) layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __restrict__ x,
+                                                            const float* __restrict__ g,
+                                                            const float* __restrict__ resid, float* __restrict__ dx,
+                                                            bf16* __restrict__ dxb, int T, int d, float eps) {
+  __shared__ float red[8];
+  const int row = blockIdx.x * (8 / WPR) + threadIdx.x / (32 * WPR), tr = threadIdx.x % (32 * WPR);
+  const bool ok = row < T;
+  const size_t ro = (size_t)(ok ? row : 0) * d;
   float v[NCH][8], gh[NCH][8];
   // residual loads first: in flight during the loads and reductions below instead of after them
   const float4* rr4 = reinterpret_cast<const float4*>(resid + ro);
   float4 rq[NCH][2];
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int i = (c * 32 + lane) * 8;
+    const int i = (c * 32 * WPR + tr) * 8;
     if (i < d) { rq[c][0] = rr4[i / 4]; rq[c][1] = rr4[i / 4 + 1]; }
   }
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int i = (c * 32 + lane) * 8;
+    const int i = (c * 32 * WPR + tr) * 8;
     if (i < d) {
       ld8f(x + ro + i, v[c]);
       float a[8], gg[8];
@@ -359,17 +384,18 @@ __global__ void layernorm_bwd_kernel(const TDY* __restrict__ dy, const float* __
     }
   }
   float mu, r;
-  ln_stats<NCH>(v, lane, d, eps, mu, r);
+  ln_stats<NCH, WPR>(v, tr, d, eps, mu, r, red);
   float sg = 0.f, sgx = 0.f;
 #pragma unroll
   for (int c = 0; c < NCH; ++c)
-    if ((c * 32 + lane) * 8 < d)
+    if ((c * 32 * WPR + tr) * 8 < d)
 #pragma unroll
       for (int k = 0; k < 8; ++k) { sg += gh[c][k]; sgx += gh[c][k] * (v[c][k] - mu) * r; }
-  const float mg = warp_sum(sg) / (float)d, mgx = warp_sum(sgx) / (float)d;
+  const float mg = ln_row_sum<WPR>(sg, red) / (float)d, mgx = ln_row_sum<WPR>(sgx, red) / (float)d;
+  if (!ok) return;
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int i = (c * 32 + lane) * 8;
+    const int i = (c * 32 * WPR + tr) * 8;
     if (i >= d) continue;
     const float rr[8] = {rq[c][0].x, rq[c][0].y, rq[c][0].z, rq[c][0].w, rq[c][1].x, rq[c][1].y, rq[c][1].z, rq[c][1].w};
     float o[8];
@@ -480,21 +506,24 @@ int convert_bf16_to_f32(const bf16* src, float* dst, long long n, cudaStream_t s
 
 // ------------------------------------------------------------------ LayerNorm launchers (OPT)
 template <typename F>
-static int ln_dispatch(int d, F&& f) {
+static int ln_dispatch(int d, F&& f) {   // (chunks per lane, warps per row); d <= 4096 as before
+  using std::integral_constant;
   const int nch = (d + 255) / 256;
-  if (nch <= 1) return f(std::integral_constant<int, 1>{});
-  if (nch <= 2) return f(std::integral_constant<int, 2>{});
-  if (nch <= 4) return f(std::integral_constant<int, 4>{});
-  if (nch <= 8) return f(std::integral_constant<int, 8>{});
-  if (nch <= 16) return f(std::integral_constant<int, 16>{});
+  if (nch <= 1) return f(integral_constant<int, 1>{}, integral_constant<int, 1>{});
+  if (nch <= 2) return f(integral_constant<int, 2>{}, integral_constant<int, 1>{});
+  if (nch <= 4) return f(integral_constant<int, 4>{}, integral_constant<int, 1>{});
+  if (nch <= 8) return f(integral_constant<int, 4>{}, integral_constant<int, 2>{});
+  if (nch <= 16) return f(integral_constant<int, 4>{}, integral_constant<int, 4>{});
   return -1;
 }
 int layernorm_fwd(const float* x, const float* g, const float* b, bf16* y, float* rstd, int T, int d, float eps,
                   cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
-  return ln_dispatch(d, [&](auto n) {
-    layernorm_fwd_kernel<decltype(n)::value><<<(T + 7) / 8, 256, 0, st>>>(x, g, b, y, rstd, T, d, eps);
+  return ln_dispatch(d, [&](auto n, auto w) {
+    constexpr int RPB = 8 / decltype(w)::value;   // rows per 256-thread CTA
+    layernorm_fwd_kernel<decltype(n)::value, decltype(w)::value><<<(T + RPB - 1) / RPB, 256, 0, st>>>(
+        x, g, b, y, rstd, T, d, eps);
     return LAUNCH_CHECK();
   });
 }
@@ -503,8 +532,10 @@ static int layernorm_bwd_t(const TDY* dy, const float* x, const float* g, const 
                            int T, int d, float eps, cudaStream_t st) {
   if (T <= 0) return 0;
   if (d % 8) return -1;
-  return ln_dispatch(d, [&](auto n) {
-    layernorm_bwd_kernel<decltype(n)::value, TDY><<<(T + 7) / 8, 256, 0, st>>>(dy, x, g, resid, dx, dxb, T, d, eps);
+  return ln_dispatch(d, [&](auto n, auto w) {
+    constexpr int RPB = 8 / decltype(w)::value;
+    layernorm_bwd_kernel<decltype(n)::value, decltype(w)::value, TDY><<<(T + RPB - 1) / RPB, 256, 0, st>>>(
+        dy, x, g, resid, dx, dxb, T, d, eps);
     return LAUNCH_CHECK();
   });
 }

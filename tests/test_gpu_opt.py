@@ -9,6 +9,7 @@ import pytest
 
 from tests.parity_util import compare_step, make_inputs, run_gpu_step, run_oracle_step, act_err
 from workloads import ClientCfg, MODELS, Workload
+from workloads.synth import ModelCfg
 
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
@@ -35,6 +36,15 @@ def test_opt_1p3b_width_two_layers():
     w = Workload("opt13_2l", m, [ClientCfg(8, 16.0, ("q", "v"), [100, 100, 57]),
                                  ClientCfg(16, 32.0, OPT_T, [200, 33])])
     assert_ok(compare_step(run_gpu_step(w, seed=22), run_oracle_step(w, seed=22)))
+
+
+@pytest.mark.parametrize("d,heads,ffn", [(4096, 32, 16384), (1024, 16, 4096)])
+def test_opt_layernorm_widths_one_layer(d, heads, ffn):
+    """LayerNorm launch shapes other than 1.3B's: d = 4096 (OPT-6.7B widths, head_dim 128 -> tcgen05 attention;
+    four warps per row) and d = 1024 (one warp per row); 1 server layer, ragged sequences."""
+    m = ModelCfg(f"opt-d{d}", d, heads, heads, ffn, 1, model_layers=2, arch="opt")
+    w = Workload(f"opt_d{d}", m, [ClientCfg(8, 16.0, ("q", "v"), [130, 5]), ClientCfg(16, 32.0, OPT_T, [77])])
+    assert_ok(compare_step(run_gpu_step(w, seed=23), run_oracle_step(w, seed=23)))
 
 
 def test_opt_invariants_zero_b_and_batched_alone():
