@@ -331,7 +331,7 @@ def run_gpu(args):
     peak = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
     traffic = None
     tp = os.path.join(ROOT, "profiles", "gemm_traffic.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and args.workload == "cfg1_7b_x4" and not args.layers:   # measured at cfg1's shapes only
         try:
             traffic = json.load(open(tp)).get("bytes_per_launch")
         except Exception:
