@@ -85,48 +85,141 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------------ CPU oracle
-def oracle_sample(n_layers: int = 2, n_seqs: int = 4, seq: int = 512):
-    """Time the CPU oracle (as it stands) on a bounded sample of the cfg1 workload: one client's batch
-    (n_seqs x seq tokens) through n_layers of the 31 server layers, fwd + bwd.  Returns tokens/s scaled to
-    the full 31-layer segment."""
+_ORACLE_CACHE = {}
+
+
+def _oracle_weights(n_layers: int):
+    """Base weights of the first n_layers Llama-2-7B server layers (fp32, the parity recipe), generated once."""
+    from workloads import MODELS, base_layer_weights
+    key = n_layers
+    if key not in _ORACLE_CACHE:
+        _ORACLE_CACHE.clear()
+        m = MODELS["7b"].with_layers(n_layers)
+        _ORACLE_CACHE[key] = (m, [base_layer_weights(m, l, seed=0) for l in range(n_layers)])
+    return _ORACLE_CACHE[key]
+
+
+def oracle_layers_that_fit() -> int:
+    """All 31 server layers (cfg1 full depth) when the host holds their fp32 weights (25 GB) plus working space;
+    otherwise the most that fit, and the line says so."""
+    full = 31
+    try:
+        import psutil
+        avail = psutil.virtual_memory().available
+    except Exception:
+        return full
+    per_layer = 202_383_360 * 4 * 1.2
+    return max(1, min(full, int((avail - (12 << 30)) // per_layer)))
+
+
+def oracle_sample(seq: int = 512, n_layers: int | None = None):
+    """Time the CPU oracle (as it stands, never tuned) on a bounded sample of the cfg1 workload: ONE sequence of `seq`
+    tokens of one cfg1 client (r = 8 on q, v) through the Llama-2-7B server segment, forward + backward.  Full depth
+    (31 layers) unless the host cannot hold the fp32 weights; then the truncation is stated and scaled."""
     import numpy as np
     from oracle import menos_oracle as O
-    from workloads import ClientCfg, MODELS, base_layer_weights, client_adapters, client_inputs
+    from workloads import ClientCfg, client_adapters, client_inputs
     cores = len(os.sched_getaffinity(0))
-    m = MODELS["7b"].with_layers(n_layers)
-    c = ClientCfg(8, 16.0, ("q", "v"), [seq] * n_seqs)
-    W = [base_layer_weights(m, l, seed=0) for l in range(n_layers)]
+    full = 31
+    n_layers = n_layers or oracle_layers_that_fit()
+    m, W = _oracle_weights(n_layers)
+    c = ClientCfg(8, 16.0, ("q", "v"), [seq])
     ad = client_adapters(m, c, seed=1)
     x, g = client_inputs(m, c, seed=2)
     t0 = time.perf_counter()
     O.client_step(x, g, c.seq_lens, W, ad, c.alpha / c.rank, m)
     dt = time.perf_counter() - t0
-    full = MODELS["7b"].n_layers
-    tps = c.n_tokens / (dt * full / n_layers)
-    return {"value": tps, "unit": "tokens/s", "cores": cores, "kind": "oracle",
-            "sample": f"1 client x {n_seqs} seq x {seq} tokens through {n_layers} of {full} Llama-2-7B server "
-                      f"layers (fwd+bwd, fp32 numpy, {dt:.1f} s), scaled to the {full}-layer segment"}
+    scale = full / n_layers
+    tps = c.n_tokens / (dt * scale)
+    depth = (f"all {full} Llama-2-7B server layers" if n_layers == full else
+             f"{n_layers} of {full} Llama-2-7B server layers (host RAM bound), time scaled x{scale:.2f} to {full}")
+    return {"value": tps, "unit": "tokens/s", "cores": cores, "kind": "oracle", "sample_s": dt,
+            "sample_tokens": c.n_tokens, "sample_layers": n_layers,
+            "sample": f"1 cfg1 sequence of {seq} tokens (r=8 q,v) through {depth}, fwd+bwd, fp32 numpy on {cores} "
+                      f"host threads: {dt:.2f} s"}
 
 
 def run_reference(args):
+    """The reference arm for this tier = the CPU oracle as it stands, rank 0 only.  Each step is a
+    bounded sample of our arm's workload: one 128-token sequence of a cfg1 client through the whole 31-layer segment
+    (no depth extrapolation when the host holds the weights); value = tokens/s of that sample."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    seq = 128
     for _ in range(args.warmup):
-        oracle_sample(1, 1, 512)
-    vals = []
-    for _ in range(args.steps):
-        vals.append(oracle_sample(1, 1, 512))
+        oracle_sample(seq)
+    vals = [oracle_sample(seq) for _ in range(args.steps)]
     v = statistics.median([r["value"] for r in vals])
+    s_med = statistics.median([r["sample_s"] for r in vals])
     cb = dict(vals[-1])
     cb["value"] = v
+    w = args.workload or "cfg1_7b_x4"
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 512 / v * 1000.0, "higher_is_better": True,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": s_med * 1000.0, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": "cfg1_7b_x4", "model": "llama2-7b", "sample": cb["sample"]},
+            "config": {"workload": w, "model": "llama2-7b", "measured_sample": cb["sample"],
+                       "sample_tokens_per_step": cb["sample_tokens"], "sample_layers": cb["sample_layers"],
+                       "note": "ms_per_step is the measured time of one sample step, not of the whole workload"},
             "cpu_baseline": cb, "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0,
                                         "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------ launcher
+def _free_port() -> int:
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def spawn_ranks(args) -> int:
+    """`python bench.py --gpus N` without a torchrun environment: re-exec this script under torchrun with N ranks
+    (one process per GPU, 127.0.0.1 rendezvous), NCCL init logs on stderr; rank 0 prints the JSON line."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__), *sys.argv[1:]]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env.setdefault("OMP_NUM_THREADS", "4")
+    return subprocess.run(cmd, env=env).returncode
+
+
+def rank_plan(w, world: int, rank: int, tp_mode: bool, strong: bool):
+    """The clients this rank serves: all of them (weak scaling / tensor parallel) or its LPT share (strong)."""
+    from paper_conf_middleware_hul24_b200.partition import workload_partition
+    if strong and not tp_mode:
+        return workload_partition(w, world)[rank]
+    return list(range(len(w.clients)))
+
+
+def run_dry(args):
+    """Launcher check without the library or a GPU: every rank computes its client share; rank 0 prints the rank map
+    as one JSON line (gloo all_gather when world > 1)."""
+    import torch.distributed as dist
+    from workloads import workload
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if world > 1:
+        dist.init_process_group("gloo")
+    w = workload(args.workload)
+    tp_mode = args.workload.startswith("cfg4")
+    strong = args.workload in ("cfg2_7b_x32_ragged", "cfg3_13b_x16") or tp_mode
+    mine = rank_plan(w, world, rank, tp_mode, strong)
+    info = {"rank": rank, "pid": os.getpid(), "clients": mine, "tokens": sum(w.clients[i].n_tokens for i in mine)}
+    allinfo = [None] * world
+    if world > 1:
+        dist.all_gather_object(allinfo, info)
+    else:
+        allinfo = [info]
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "metric": METRIC, "n_gpus": world, "ranks_seen": len(allinfo),
+                          "config": {"workload": args.workload, "scaling": "strong" if strong else "weak",
+                                     "per_rank": allinfo}}))
+    if world > 1:
+        dist.destroy_process_group()
     return 0
 
 
@@ -201,6 +294,9 @@ def run_gpu(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch with torchrun or let bench.py "
+                         f"spawn the ranks)")
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
@@ -227,11 +323,17 @@ def run_gpu(args):
         else:
             tp = (rank, world, TPM.make_torch_allreduce(device=local)) if world > 1 else None
     elif strong:
-        w.clients = [w.clients[i] for i in workload_partition(w, world)[rank]]
+        w.clients = [w.clients[i] for i in rank_plan(w, world, rank, tp_mode, strong)]
     T = w.n_tokens
     d = w.model.d_model
+    torch.cuda.synchronize(device)
+    free0 = torch.cuda.mem_get_info(device)[0]
     srv = build_server(torch, w, device, seed=rank, arena_gb=args.arena_gb, tp=tp)
+    torch.cuda.synchronize(device)
+    free1 = torch.cuda.mem_get_info(device)[0]
     ids = register_clients(np, srv, w, seed=rank + 1)
+    torch.cuda.synchronize(device)
+    free2 = torch.cuda.mem_get_info(device)[0]
     # waves: temporal sharing of the arena when the clients' saved activations do not fit at once
     mem = [srv.client_memory(ids[i], c.n_tokens) for i, c in enumerate(w.clients)]
     cap = srv.stats()["arena_bytes"] - (64 << 20)
@@ -239,6 +341,13 @@ def run_gpu(args):
     def demand(idx):   # exact peak arena bytes of one batched call (menos_batch_memory)
         return max(srv.batch_memory([ids[i] for i in idx], [w.clients[i].n_tokens for i in idx]))
     waves = plan_waves_exact(len(w.clients), demand, cap)
+    props = torch.cuda.get_device_properties(device)
+    my_info = {"rank": rank, "device": str(getattr(props, "uuid", local)),
+               "clients": len(w.clients), "tokens": T, "waves": len(waves)}
+    per_rank = [my_info]
+    if world > 1:
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, my_info)
     toff = [0]
     for c in w.clients:
         toff.append(toff[-1] + c.n_tokens)
@@ -387,6 +496,15 @@ def run_gpu(args):
     Nc = len(w.clients)
     hbm = {"base_M_bytes_once_per_gpu": Mb, "per_client_persistent_AO_bytes": AO,
            "per_client_arena_I_bytes": statistics.mean(p["arena_I"] for p in per_client),
+           "measured": {
+               "how": "cudaMemGetInfo deltas around menos_server_create (base + arena + tables) and around the "
+                      "clients' registration (A+O: fp32 p, g, m, v + bf16 slot tables incl. their growth); arena "
+                      "high-water mark of the step from the library's allocator",
+               "server_create_bytes": free0 - free1, "arena_bytes": st["arena_bytes"],
+               "base_and_tables_bytes": free0 - free1 - st["arena_bytes"],
+               "per_client_persistent_AO_bytes": (free1 - free2) / max(1, Nc),
+               "arena_peak_bytes_per_token": st["arena_peak"] / max(1, max(
+                   sum(w.clients[i].n_tokens for i in wv) for wv in waves))},
            "persistent_reduction_vs_vanilla": 1.0 - (Mb + Nc * AO) / (Nc * (Mb + AO)),
            "paper_reference": "PAPER.md:352: -72.2% for 4 Llama-2-7B clients on a V100 (fp32; context only)"}
 
@@ -397,6 +515,7 @@ def run_gpu(args):
             "config": {"workload": args.workload, "model": w.model.name, "clients_per_gpu": len(w.clients),
                        "tokens_per_gpu_step": T, "tokens_per_step_all_gpus": T_all,
                        "waves_per_step": len(waves), "server_layers": w.model.n_layers,
+                       "per_rank": per_rank, "gpus_active": len({r["device"] for r in per_rank}),
                        "lora": sorted({f"r{c.rank} {'+'.join(c.targets)}" for c in w.clients}),
                        "seq_lens": sorted({s for c in w.clients for s in c.seq_lens}),
                        "parallelism": (f"tensor-parallel x{world} (NCCL all-reduce per attention/MLP block)"
@@ -412,7 +531,7 @@ def run_gpu(args):
             "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
-            line["cpu_baseline"] = oracle_sample(args.cpu_layers, 4, 512)
+            line["cpu_baseline"] = oracle_sample(512)
         except Exception as ex:  # never let the baseline kill the bench line
             line["cpu_baseline"] = {"value": None, "error": repr(ex)}
     if rank == 0:
@@ -429,20 +548,27 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="menos", choices=["menos", "reference"])
-    ap.add_argument("--workload", default="cfg1_7b_x4")
+    ap.add_argument("--workload", default=None,
+                    help="default: cfg1_7b_x4 at --gpus 1, cfg2_7b_x32_ragged (LPT over the ranks) at --gpus > 1")
     ap.add_argument("--layers", type=int, default=None, help="truncate depth (debug only; not a bench value)")
     ap.add_argument("--arena-gb", type=float, default=0.0, help="activation arena; 0 = all memory the base leaves")
     ap.add_argument("--tp-shard-only", type=int, default=0,
                     help="time rank 0's shard of a W-way tensor-parallel split on 1 GPU (no all-reduce; not a "
                          "bench value)")
-    ap.add_argument("--cpu-layers", type=int, default=6)
+    ap.add_argument("--dry-run", action="store_true", help="launcher check: no library, no GPU; print the rank map")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.workload is None:
+        args.workload = "cfg1_7b_x4" if args.gpus == 1 else "cfg2_7b_x32_ragged"
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args)
     if args.impl == "reference":
         return run_reference(args)
+    if args.dry_run:
+        return run_dry(args)
     return run_gpu(args)
 
 

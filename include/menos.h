@@ -192,6 +192,14 @@ MENOS_API int menos_batch_memory(menos_server* s, int n_clients, const int32_t* 
  * (PAPER.md:238-263); this keeps its accounting safe when the granted requests run as one batched call. */
 enum { MENOS_MEM_BOUND = 2 };
 
+/* Stream rule: every forward / backward / adapter_step of one server must be issued on ONE stream (the first such
+ * call binds it; a different stream later returns MENOS_EINVAL).  Arena slabs and the scratch block are released on
+ * the host as soon as their last kernel is enqueued and reused in stream order, which is only safe on one stream.
+ * Live batches: a SAVE batch (or a retained NOGRAD batch) returned by menos_forward is "live" until menos_backward or
+ * menos_batch_free.  While any SAVE batch is live, a registration that would grow the LoRA slot tables returns
+ * MENOS_ESTATE (the batch's precomputed LoRA problem lists point into them); a client that belongs to a live batch
+ * cannot be unregistered (MENOS_ESTATE), so its id cannot be reused under the batch either. */
+
 /* Step 2: x_s = f_s(x_c).  n_seqs sequences; seq_client[i] (host) is the client of sequence i and
  * seq_len[i] (host) its length (>= 1, <= max_seq_len).  Sequences of one client must be contiguous
  * (client-major packing).  T = sum(seq_len).  x_c, x_s: [T, d] bf16 (host or device).
@@ -262,8 +270,8 @@ MENOS_API const char* menos_last_error(void);
  *   menos_sched_arrive(i, kind)          Alg.2 L7-9: x_c (kind FWD) or g_c (kind BWD) of client i arrived
  *   menos_sched_complete(i)              Alg.2 L10-13: client i's task finished and released A[i]
  * Grants are written to out[0..*n_out) in the order they were made: the FCFS head first (L16-22), then the
- * backfilled requests in waiting-list order (L23-24).  out must hold max_clients entries (EINVAL otherwise, with
- * the scheduler state already updated).  Errors: ENOCLIENT (id out of range / no demands), ESTATE (the client
+ * backfilled requests in waiting-list order (L23-24).  out must hold max_clients entries (max_out >= max_clients;
+ * EINVAL otherwise, checked before anything changes).  Errors: ENOCLIENT (id out of range / no demands), ESTATE (the client
  * already has a request waiting or running, or complete() without a running task), ENOMEM (a demand larger than
  * M_avail at create: it could never be granted and would block the FCFS head forever; nothing is enqueued).
  * Not thread-safe: one event at a time (the paper's scheduler is one event loop, Alg.2 L5-6). */

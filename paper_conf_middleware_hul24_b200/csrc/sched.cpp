@@ -111,6 +111,8 @@ MENOS_API int menos_sched_arrive(menos_sched* s, int32_t client, int kind, menos
                                  int* n_out) {                                                  // L7-9
   if (n_out) *n_out = 0;
   if (!s || (max_out > 0 && !out)) SFAIL(MENOS_EINVAL, "sched_arrive: bad arguments");
+  // one SCHEDULE can grant every waiting client: out must hold max_clients entries, checked BEFORE any state change
+  if (max_out < (int)s->cl.size()) SFAIL(MENOS_EINVAL, "sched_arrive: out holds %d < max_clients %zu", max_out, s->cl.size());
   if (kind != MENOS_REQ_FWD && kind != MENOS_REQ_BWD) SFAIL(MENOS_EINVAL, "sched_arrive: bad kind %d", kind);
   if (client < 0 || client >= (int32_t)s->cl.size() || !s->cl[client].known)
     SFAIL(MENOS_ENOCLIENT, "sched_arrive: client %d has no demands (menos_sched_set_demand)", client);
@@ -128,6 +130,7 @@ MENOS_API int menos_sched_complete(menos_sched* s, int32_t client, menos_sched_g
                                    int* n_out) {                                                // L10-13
   if (n_out) *n_out = 0;
   if (!s || (max_out > 0 && !out)) SFAIL(MENOS_EINVAL, "sched_complete: bad arguments");
+  if (max_out < (int)s->cl.size()) SFAIL(MENOS_EINVAL, "sched_complete: out holds %d < max_clients %zu", max_out, s->cl.size());
   if (client < 0 || client >= (int32_t)s->cl.size()) SFAIL(MENOS_ENOCLIENT, "sched: client %d out of range", client);
   auto& c = s->cl[client];
   if (c.state != 2) SFAIL(MENOS_ESTATE, "sched_complete: client %d has no running task", client);

@@ -241,6 +241,10 @@ struct ColAlloc {
     if (newcap > cap) release(cap, newcap - cap);
     cap = newcap;
   }
+  bool fits(int w) const {
+    for (const auto& kv : free_) if (kv.second >= w) return true;
+    return false;
+  }
   int max_end() const {  // end of the highest allocated column
     int end = cap;
     auto it = free_.rbegin();
@@ -300,6 +304,8 @@ struct menos_batch {
   std::vector<LoraRowsProblem> h_rprobs;
   std::vector<LoraTokRedProblem> h_tprobs;
   uint8_t* scratch_base = nullptr; size_t scratch_span = 0;
+  // live-batch accounting (menos_server::batch_refs / live_save): set when the handle is returned to the caller
+  bool counted = false, counted_save = false;
 };
 
 // =====================================================================================================
@@ -340,7 +346,24 @@ struct menos_server {
   // last read an entry has completed (its event), so adapter_step never allocates on the hot path
   Slot dring[kRing];
   int dring_next = 0;
+  // live batches: a SAVE batch's LoRA problem lists hold raw slot-table pointers, leading dimensions and each
+  // client's gradient buffer, so while one is alive the slot tables may not move (registration that would grow them
+  // returns MENOS_ESTATE) and none of its clients may be unregistered (MENOS_ESTATE)
+  int live_save = 0;
+  std::vector<int> batch_refs;   // per client id: live batches that contain it
+  // the one stream this server's work is ordered on (arena slabs and the scratch block are reused in stream order):
+  // bound by the first forward / backward / adapter_step, any other stream afterwards is MENOS_EINVAL
+  bool stream_bound = false;
+  cudaStream_t stream = nullptr;
 };
+
+static int bind_stream(menos_server* s, cudaStream_t st) {
+  if (!s->stream_bound) { s->stream_bound = true; s->stream = st; return MENOS_OK; }
+  if (s->stream != st)
+    FAIL(MENOS_EINVAL, "server work must stay on one stream (bound to %p, got %p): arena memory is reused in "
+         "stream order", (void*)s->stream, (void*)st);
+  return MENOS_OK;
+}
 
 // =====================================================================================================
 // helpers: weights
@@ -622,6 +645,7 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
   CUDA_TRY(cudaMalloc(&s->rope, (size_t)o.max_seq_len * (D.hd / 2) * sizeof(float2)));
   K_TRY(fill_rope_table(s->rope, o.max_seq_len, D.hd, D.theta, 0));
   s->clients.resize(o.max_clients);
+  s->batch_refs.assign(o.max_clients, 0);
   if (w) {
     for (int l = 0; l < n_layers; ++l) {
       int rc = upload_layer(s.get(), l, &w[l]);
@@ -696,6 +720,14 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
   int id = -1;
   for (size_t i = 0; i < s->clients.size(); ++i) if (!s->clients[i].used) { id = (int)i; break; }
   if (id < 0) FAIL(MENOS_ENOMEM, "client registry full (%d)", s->opts.max_clients);
+  if (s->live_save > 0) {   // the slot tables may not move under a live SAVE batch (its problem lists point into them)
+    int cnt0[NG] = {0, 0, 0, 0};
+    for (int t = 0; t < NT; ++t) if (target_mask >> t & 1) cnt0[kTargetGroup[t]]++;
+    for (int g = 0; g < NG; ++g)
+      if (cnt0[g] && !s->cols[g].fits(cnt0[g] * (int)align_up(rank, 16)))
+        FAIL(MENOS_ESTATE, "registration would grow the LoRA slot tables while %d SAVE batch(es) are alive; run their "
+             "backward (or menos_batch_free) first", s->live_save);
+  }
   const Dims& D = s->D;
   Client c;
   c.rank = rank; c.rs = (int)align_up(rank, 16); c.alpha = alpha; c.s = alpha / (float)rank; c.mask = target_mask;
@@ -768,6 +800,9 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
 extern "C" int menos_unregister_client(menos_server* s, int32_t id) {
   if (!s) FAIL(MENOS_EINVAL, "null server");
   if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
+  if (s->batch_refs[id] > 0)
+    FAIL(MENOS_ESTATE, "client %d is in %d live batch(es); run their backward (or menos_batch_free) first", id,
+         s->batch_refs[id]);
   CUDA_TRY(cudaSetDevice(s->device));
   CUDA_TRY(cudaDeviceSynchronize());
   Client& c = s->clients[id];
@@ -945,6 +980,7 @@ extern "C" int menos_adapter_step(menos_server* s, int n, const int32_t* ids, vo
     v.push_back(ids[i]);
   }
   CUDA_TRY(cudaSetDevice(s->device));
+  if (int rc0 = bind_stream(s, (cudaStream_t)stream)) return rc0;
   return run_adam(s, v, true, (cudaStream_t)stream);
 }
 
@@ -1663,6 +1699,7 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
   for (int l = 0; l < s->n_layers; ++l) if (!s->loaded[l]) FAIL(MENOS_ESTATE, "layer %d weights not loaded", l);
   CUDA_TRY(cudaSetDevice(s->device));
   cudaStream_t st = (cudaStream_t)stream;
+  if (int rc0 = bind_stream(s, st)) return rc0;
   std::unique_ptr<menos_batch> b;
   int rc = build_batch(s, n_seqs, seq_client, seq_len, flags == MENOS_FWD_NOGRAD, b);
   if (rc) return rc;
@@ -1715,12 +1752,17 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     fail_free(MENOS_OK);
     return MENOS_OK;
   }
+  b->counted = true;
+  for (int c : b->bclients) s->batch_refs[c]++;
+  if (!b->nograd) { b->counted_save = true; s->live_save++; }
   *batch = b.release();
   return MENOS_OK;
 }
 
 extern "C" int menos_batch_free(menos_server* s, menos_batch* b) {
   if (!s || !b) FAIL(MENOS_EINVAL, "null argument");
+  if (b->counted) for (int c : b->bclients) s->batch_refs[c]--;
+  if (b->counted_save) s->live_save--;
   if (b->slab) s->arena.release(b->slab);
   if (b->meta) s->arena.release(b->meta);
   delete b;
@@ -1754,6 +1796,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   for (int c : b->bclients) if (!s->clients[c].used) FAIL(MENOS_ESTATE, "client %d unregistered since forward", c);
   CUDA_TRY(cudaSetDevice(s->device));
   cudaStream_t st = (cudaStream_t)stream;
+  if (int rc0 = bind_stream(s, st)) return rc0;
   const Dims& D = s->D;
   const int T = b->T;
   Scratch sc;

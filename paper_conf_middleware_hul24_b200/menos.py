@@ -166,6 +166,30 @@ def _i32(seq):
     return arr
 
 
+def _check_act(name: str, x, n_tokens: int, d_model: int, device: int | None):
+    """x_c / x_s / g_c / g_s must be bf16, contiguous, [sum(seq_len), d_model], on the server's GPU or in host memory:
+    the library trusts T from seq_len, so a short, strided or fp32 buffer would be read / written out of bounds."""
+    if isinstance(x, int):
+        return   # raw address: the caller vouches for it (include/menos.h)
+    want = n_tokens * d_model
+    if hasattr(x, "data_ptr"):
+        import torch
+        if x.dtype != torch.bfloat16:
+            raise MenosError(-1, f"{name}: dtype {x.dtype}, expected torch.bfloat16")
+        if not x.is_contiguous():
+            raise MenosError(-1, f"{name}: not contiguous")
+        if x.numel() != want:
+            raise MenosError(-1, f"{name}: {tuple(x.shape)} has {x.numel()} elements, expected [{n_tokens}, {d_model}]")
+        if x.is_cuda and device is not None and x.device.index != device:
+            raise MenosError(-1, f"{name}: on cuda:{x.device.index}, the server is on cuda:{device}")
+        return
+    if hasattr(x, "ctypes"):   # numpy: raw bf16 bits
+        if x.dtype.itemsize != 2 or not x.flags["C_CONTIGUOUS"] or x.size != want:
+            raise MenosError(-1, f"{name}: numpy buffer must be contiguous 2-byte bf16 bits of [{n_tokens}, {d_model}]")
+        return
+    raise TypeError(f"{name}: unsupported buffer type {type(x)}")
+
+
 class Batch:
     def __init__(self, server: "Server", handle: int, n_tokens: int):
         self.server, self.handle, self.n_tokens = server, handle, n_tokens
@@ -182,6 +206,7 @@ class Server:
         sum over the ranks (tp.make_torch_allreduce)."""
         self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta, ARCH[arch])
         self.n_layers = n_layers
+        self.device = device
         tpc = TPCfg(0, 1, ALLREDUCE_FN(), None)
         self._tp_cb = None
         if tp is not None and tp[1] > 1:
@@ -271,12 +296,17 @@ class Server:
     # ---------------------------------------------------------------- the hot path
     def forward(self, seq_client, seq_len, x_c, x_s, flags=FWD_SAVE, stream=None, retain=True) -> Batch | None:
         """retain=False (NOGRAD only): nothing is kept after the call (Alg.1 L6-7); returns None."""
+        T = int(sum(seq_len))
+        _check_act("x_c", x_c, T, self.cfg.d_model, self.device)
+        _check_act("x_s", x_s, T, self.cfg.d_model, self.device)
         b = C.c_void_p()
         check(lib().menos_forward(self.h, len(seq_client), _i32(seq_client), _i32(seq_len), ptr(x_c), ptr(x_s),
                                   flags, _stream(stream), C.byref(b) if retain else None))
         return Batch(self, b.value, int(sum(seq_len))) if retain else None
 
     def backward(self, batch: Batch, g_c, g_s, stream=None):
+        _check_act("g_c", g_c, batch.n_tokens, self.cfg.d_model, self.device)
+        _check_act("g_s", g_s, batch.n_tokens, self.cfg.d_model, self.device)
         check(lib().menos_backward(self.h, batch.handle, ptr(g_c), ptr(g_s), _stream(stream)))
         batch.handle = None
 
@@ -284,6 +314,17 @@ class Server:
         if batch.handle:
             check(lib().menos_batch_free(self.h, batch.handle))
             batch.handle = None
+
+    def batch_tensor(self, batch: Batch, layer: int, which: int):
+        """White-box test hook (include/menos_testing.h menos_test_batch_tensor): one saved intermediate of a live
+        SAVE batch as raw bytes (numpy uint8); the caller interprets dtype / shape."""
+        import numpy as np
+        n = C.c_size_t()
+        check(lib().menos_test_batch_tensor(self.h, batch.handle, layer, which, None, C.byref(n)), testing=False)
+        out = np.empty(n.value, np.uint8)
+        if n.value:
+            check(lib().menos_test_batch_tensor(self.h, batch.handle, layer, which, out.ctypes.data, C.byref(n)))
+        return out
 
     def adapter_step(self, client_ids, stream=None):
         check(lib().menos_adapter_step(self.h, len(client_ids), _i32(client_ids), _stream(stream)))

@@ -3,7 +3,9 @@
 run_gpu_step  : drives libmenos.so through its C-ABI (paper_conf_middleware_hul24_b200.Server).
 run_oracle_step: the CPU oracle (oracle/menos_oracle.py) on the same seeded inputs.
 compare_step  : BASELINE.json north_star bars -- activations max|d|/max|ref| <= 2e-2, every gradient tensor
-                cosine >= 0.999 (DESIGN.md §"Tolerances").
+                cosine >= 0.999 (DESIGN.md §"Tolerances") -- applied to x_s and g_s AND to the segment's branch
+                deltas x_s - x_c and g_s - g_c (so an identity map, a dropped branch or a dropped adapter cannot hide
+                behind the residual stream; tests/test_mutants.py proves each such mutant fails).
 """
 from __future__ import annotations
 
@@ -20,9 +22,9 @@ def _bf16(a, device="cpu"):
     return torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(torch.bfloat16).to(device).contiguous()
 
 
-def make_inputs(w: Workload, seed: int = 0, zero_b: bool = False, outlier: bool = False):
+def make_inputs(w: Workload, seed: int = 0, zero_b: bool = False, outlier: bool = False, recipe: str = "default"):
     m = w.model
-    weights = [base_layer_weights(m, l, seed=seed) for l in range(m.n_layers)]
+    weights = [base_layer_weights(m, l, seed=seed, recipe=recipe) for l in range(m.n_layers)]
     adapters = [client_adapters(m, c, seed=1000 + 17 * seed + i, zero_b=zero_b) for i, c in enumerate(w.clients)]
     io = [client_inputs(m, c, seed=2000 + 17 * seed + i, outlier=outlier) for i, c in enumerate(w.clients)]
     return weights, adapters, io
@@ -80,7 +82,7 @@ def run_gpu_step(w: Workload, seed: int = 0, zero_b: bool = False, flags: int = 
     b = srv.forward(seq_client, seq_len, x, xs, flags=flags)
     srv.backward(b, g, gs)
     torch.cuda.synchronize()
-    out = {"x_s": [], "g_s": [], "grads": []}
+    out = {"x_s": [], "g_s": [], "grads": [], "x_c": [a for a, _ in io], "g_c": [b for _, b in io]}
     off = 0
     xs_h, gs_h = xs.float().cpu().numpy(), gs.float().cpu().numpy()
     for i, c in enumerate(w.clients):
@@ -105,16 +107,15 @@ def run_oracle_step(w: Workload, seed: int = 0, zero_b: bool = False, inputs=Non
     from oracle import menos_oracle as O
     m = w.model
     weights, adapters, io = inputs if inputs is not None else make_inputs(w, seed, zero_b)
-    out = {"x_s": [], "g_s": [], "grads": []}
+    out = {"x_s": [], "g_s": [], "grads": [], "x_c": [a for a, _ in io], "g_c": [b for _, b in io]}
     for i, c in enumerate(w.clients):
         if clients is not None and i not in clients:
             out["x_s"].append(None); out["g_s"].append(None); out["grads"].append(None)
             continue
         # a client with cut k runs the segment [k, L): the same oracle on the layers it sends its tokens through
         mc = m.with_layers(m.n_layers - c.cut) if c.cut else m
-        # OPT: the ReLU mask is a floating-point decision; the oracle takes it in the kernel's precision (R25)
         xs, gs, gr = O.client_step(io[i][0], io[i][1], c.seq_lens, weights[c.cut:], adapters[i][c.cut:],
-                                   c.alpha / c.rank, mc, relu_mask_bf16=(m.arch == "opt"))
+                                   c.alpha / c.rank, mc)
         out["x_s"].append(xs)
         out["g_s"].append(gs)
         out["grads"].append(gr)
@@ -144,6 +145,12 @@ def compare_step(gpu, ora, clients=None):
         rep[f"c{i}.x_s"] = {"metric": e, "ok": e <= ACT_TOL, "kind": "maxrel"}
         cg = cosine(gpu["g_s"][i], ora["g_s"][i])
         rep[f"c{i}.g_s"] = {"metric": cg, "ok": cg >= COS_TOL, "kind": "cos"}
+        # branch deltas: what the segment adds to its input / to the incoming gradient
+        xc, gc = np.asarray(ora["x_c"][i], np.float64), np.asarray(ora["g_c"][i], np.float64)
+        e = act_err(gpu["x_s"][i] - xc, ora["x_s"][i] - xc)
+        rep[f"c{i}.x_s-x_c"] = {"metric": e, "ok": e <= ACT_TOL, "kind": "maxrel"}
+        cg = cosine(gpu["g_s"][i] - gc, ora["g_s"][i] - gc)
+        rep[f"c{i}.g_s-g_c"] = {"metric": cg, "ok": cg >= COS_TOL, "kind": "cos"}
         for l, d in enumerate(gpu["grads"][i]):
             for t, (dA, dB) in d.items():
                 oA, oB = ora["grads"][i][l][t]

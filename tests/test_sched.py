@@ -176,6 +176,25 @@ def test_native_errors():
     assert s.complete(0) == [] and s.state()["m_avail"] == 100
 
 
+def test_native_short_out_buffer_changes_nothing():
+    """a grant buffer smaller than max_clients is rejected BEFORE any state change (no client is left
+    marked running with its memory deducted and no grant reported)."""
+    import ctypes as C
+    M = _native()
+    s = M.Scheduler(100, 4)
+    for i in range(4):
+        s.set_demand(i, 10, 10)
+    out = (M.SchedGrant * 2)()
+    n = C.c_int()
+    rc = M.lib().menos_sched_arrive(s.h, 0, M.REQ_FWD, out, 2, C.byref(n))
+    assert rc == -1 and n.value == 0
+    assert s.state() == {"m_avail": 100, "waiting": [], "n_running": 0}
+    assert s.arrive(0, M.REQ_FWD) == [(0, M.REQ_FWD, 10)]
+    rc = M.lib().menos_sched_complete(s.h, 0, out, 3, C.byref(n))
+    assert rc == -1 and s.state() == {"m_avail": 90, "waiting": [], "n_running": 1}
+    assert s.complete(0) == [] and s.state()["m_avail"] == 100
+
+
 def test_native_decision_latency():
     """the scheduler takes less than 0.1 ms per decision (the paper's Python one).  64 clients,
     a full waiting list; mean and max of the native SCHEDULE call."""

@@ -126,21 +126,44 @@ def _rng(*key: int) -> np.random.Generator:
     return np.random.Generator(np.random.PCG64(list(key)))
 
 
-def base_layer_weights(cfg: ModelCfg, layer: int, seed: int = 0) -> dict[str, np.ndarray]:
+RECIPES = ("default", "plain")
+
+
+def is_small(cfg: ModelCfg) -> bool:
+    """The tiny parity configs (d < 1024): weights are width-scaled (reading R26)."""
+    return cfg.d_model < 1024
+
+
+def weight_std(cfg: ModelCfg, t: str, recipe: str = "default") -> float:
+    """Init std of base projection t:
+    * tiny configs (R26): 1/sqrt(K) for every projection, so each attention / MLP branch is O(1) against the
+      residual stream as it is at Llama-2 width (0.02 = 1.28/sqrt(4096)); with 0.02 at d = 64 the branches are ~1%
+      of the residual and a kernel that dropped one would still pass the activation bar;
+    * Llama-2 widths, recipe "plain": N(0, 0.02^2) everywhere (Llama init std, SURVEY.md §8(d));
+    * Llama-2 widths, recipe "default" (R27): q, k, v, gate, up 0.02; the residual-branch outputs o and down use the
+      GPT-2 / Megatron depth-scaled std 0.02 / sqrt(2 L) (L = decoder layers of the whole model), so a 31-79 layer
+      random residual stream grows like a trained pre-norm network's instead of doubling every few layers."""
+    K, _ = target_dims(cfg, t)
+    if is_small(cfg):
+        return 1.0 / np.sqrt(K)
+    if recipe == "plain" or t not in ("o", "down"):
+        return 0.02
+    return 0.02 / np.sqrt(2.0 * cfg.total_layers)
+
+
+def base_layer_weights(cfg: ModelCfg, layer: int, seed: int = 0, recipe: str = "default") -> dict[str, np.ndarray]:
     """Frozen base weights of one decoder layer, natural (HF) layouts, fp32 bf16-representable.
 
-    W ~ N(0, 0.02^2) (Llama init std) for q, k, v, gate, up; the residual-branch output projections o and
-    down use the GPT-2 / Megatron scaled init std 0.02 / sqrt(2 L) (L = total decoder layers of the model),
-    so the residual stream evolves like a trained pre-norm network instead of a chaotic random one
-    (reading R17).  Gains g = 1 + 0.1 N(0,1).
+    W ~ N(0, weight_std(cfg, t, recipe)^2) (readings R26 / R27); gains g = 1 + 0.1 N(0,1).
     """
+    if recipe not in RECIPES:
+        raise KeyError(recipe)
     out = {}
     names = ["q", "k", "v", "o", "gate", "up", "down"]
-    out_std = 0.02 / np.sqrt(2.0 * cfg.total_layers)
     for i, t in enumerate(names):
         K, N = target_dims(cfg, t)
         r = _rng(seed, layer, i)
-        std = out_std if t in ("o", "down") else 0.02
+        std = weight_std(cfg, t, recipe)
         out["w" + t] = bf16_round(r.standard_normal((N, K), dtype=np.float32) * np.float32(std))
     for j, g in enumerate(["g1", "g2"]):
         r = _rng(seed, layer, 100 + j)
@@ -163,9 +186,12 @@ def client_adapters(cfg: ModelCfg, c: ClientCfg, seed: int, zero_b: bool = False
     """Per server layer: {target: (A [r, K], B [N, r])}, fp32 bf16-representable.
 
     A ~ U(-1/sqrt(K), 1/sqrt(K)) (PEFT kaiming-uniform a=sqrt(5) bound);
-    B ~ N(0, 0.02^2), nonzero so that dA != 0 (zero for invariant (b)).
+    B ~ N(0, 0.02^2), nonzero so that dA != 0 (zero for invariant (b)).  Tiny configs (R26): B ~ N(0, 0.25/r), so
+    the LoRA delta s (x A^T) B^T is a sizeable fraction of its projection (as for a trained adapter) and a kernel
+    that dropped one client's adapter fails the activation bar.
     """
     layers = []
+    b_std = np.sqrt(0.25 / c.rank) if is_small(cfg) else 0.02
     for ell in range(cfg.n_layers):
         d = {}
         for ti, t in enumerate(TARGETS):
@@ -178,7 +204,7 @@ def client_adapters(cfg: ModelCfg, c: ClientCfg, seed: int, zero_b: bool = False
             if zero_b:
                 B = np.zeros((N, c.rank), np.float32)
             else:
-                B = bf16_round(r.standard_normal((N, c.rank), dtype=np.float32) * np.float32(0.02))
+                B = bf16_round(r.standard_normal((N, c.rank), dtype=np.float32) * np.float32(b_std))
             d[t] = (A, B)
         layers.append(d)
     return layers
