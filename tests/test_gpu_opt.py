@@ -80,3 +80,51 @@ def test_opt_rejects_gate_target():
     with pytest.raises(MenosError):
         srv.register_client(4, 8.0, ("gate",))
     srv.close()
+
+
+def test_relu_mask_valid():
+    """The ReLU mask is a decision several answers satisfy near z = 0 (where bf16 rounding of the GEMM operands can
+    flip the sign).  Check the kernel's OWN decision (the saved a = relu(fc1) of a SAVE batch, a > 0) against the exact
+    fp64 sign of the oracle's pre-activation z = fc1(LN2(h)) + LoRA: they must agree wherever |z| exceeds the a-priori
+    bf16 bound tau = 2^-8 * sum_k |hn_k| |W_k| (+ the LoRA term), with a x4 margin from layer 1 on for the propagated
+    input differences; and the band |z| <= tau must be a small fraction of the entries."""
+    from tests.test_gpu_whitebox import gpu_layer_values
+    from oracle import menos_oracle as O
+    w = Workload("opt_relu", MODELS["opt_tiny"], [ClientCfg(8, 16.0, OPT_T, [33, 1, 70]),
+                                                  ClientCfg(16, 32.0, ("v", "up", "down"), [129])])
+    inputs = make_inputs(w, seed=27)
+    weights, adapters, io = inputs
+    gpu = gpu_layer_values(w, inputs)
+    m = w.model
+    F = np.float64
+    zs, taus = [[] for _ in range(m.n_layers)], [[] for _ in range(m.n_layers)]
+    for i, c in enumerate(w.clients):
+        off = 0
+        s = c.alpha / c.rank
+        for S in c.seq_lens:
+            x = np.asarray(io[i][0][off:off + S], F)
+            off += S
+            for l in range(m.n_layers):
+                W = {k: np.asarray(v, F) for k, v in weights[l].items()}
+                y, cache = O.opt_layer_fwd(x, W, {t: (np.asarray(a, F), np.asarray(b, F))
+                                                  for t, (a, b) in adapters[i][l].items()}, s, m, F)
+                hn = cache["hn"]
+                z = hn @ W["wup"].T + W["bup"]
+                tau = 2.0 ** -8 * (np.abs(hn) @ np.abs(W["wup"]).T)
+                if "up" in adapters[i][l]:
+                    A, B = (np.asarray(v, F) for v in adapters[i][l]["up"])
+                    U = hn @ A.T
+                    z = z + s * U @ B.T
+                    tau = tau + 2.0 ** -8 * s * ((np.abs(hn) @ np.abs(A).T) + np.abs(U)) @ np.abs(B).T
+                zs[l].append(z)
+                taus[l].append(tau)
+                x = y
+    band_total = 0
+    for l in range(m.n_layers):
+        z, tau = np.concatenate(zs[l]), np.concatenate(taus[l]) * (1.0 if l == 0 else 4.0)
+        gm = gpu[l]["a"][:, :m.d_ff] > 0
+        clear = np.abs(z) > tau
+        assert np.array_equal(gm[clear], (z > 0)[clear]), (l, int(np.sum(gm[clear] != (z > 0)[clear])))
+        band_total += int(np.sum(~clear))
+        assert np.mean(~clear) < 0.05, (l, float(np.mean(~clear)))
+    print("entries inside the rounding band:", band_total)
