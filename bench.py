@@ -319,9 +319,13 @@ def run_gpu(args):
             # this is NOT a bench value (no communication); it measures the per-GPU kernels of the TP path
             if world != 1:
                 raise SystemExit("--tp-shard-only runs on one GPU")
-            tp = (0, args.tp_shard_only, lambda buf, n, dt, st: 0)
+            tp = (0, args.tp_shard_only, lambda op, snd, rcv, n, dt, st: 0)
         else:
-            tp = (rank, world, TPM.make_torch_allreduce(device=local)) if world > 1 else None
+            # NCCL driven by the library (no Python on the per-layer path): rank 0's unique id, broadcast once
+            ids_ = [TPM.nccl_unique_id() if rank == 0 else None]
+            if world > 1:
+                dist.broadcast_object_list(ids_, src=0)
+            tp = (rank, world, ids_[0]) if world > 1 else None
     elif strong:
         w.clients = [w.clients[i] for i in rank_plan(w, world, rank, tp_mode, strong)]
     T = w.n_tokens

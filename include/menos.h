@@ -113,26 +113,48 @@ typedef struct {
 } menos_adamw_cfg;
 
 /* Tensor parallelism (Llama-2-70B, BASELINE.json configs[4]).
- * Megatron split of every server layer over `world` ranks, one process and one server object per GPU:
+ * Megatron split of every server layer over `world` ranks, one process and one server object per GPU, with
+ * SEQUENCE PARALLELISM for everything outside the split GEMMs:
  *   column-parallel: Wq, Wk, Wv (rank r holds heads [r*H/world, (r+1)*H/world) and the matching KV heads),
  *                    W_gate, W_up (rows [r*f/world, (r+1)*f/world));
- *   row-parallel:    Wo (columns of rank r's heads), W_down (columns [r*f/world, (r+1)*f/world)).
- * Per layer the server calls `allreduce` four times (sum, in place, on the call's stream):
- *   forward  : the o-proj and down-proj partial sums (fp32 [T, d]; rank 0's partial carries the residual);
- *   backward : the gate|up-dX and qkv-dX partial sums (fp32 [T, d]).
+ *   row-parallel:    Wo (columns of rank r's heads), W_down (columns [r*f/world, (r+1)*f/world));
+ *   token-parallel:  the residual streams (x, h forward; dy, dh backward), RMSNorm forward / backward and their
+ *                    saved statistics: rank r owns token rows [r*Tl, (r+1)*Tl), Tl = ceil(T / world) (the last rank's
+ *                    rows past T are padding and never read).
+ * Exchanges per layer, all bf16 [*, d] (the payload of one all-reduce split into its two halves):
+ *   forward : all-gather of RMSNorm1's and RMSNorm2's outputs (the column-parallel GEMMs read every token);
+ *             reduce-scatter of the o-proj and down-proj partial sums (the residual add then runs on the rank's rows);
+ *   backward: all-gather of the incoming gradient dy and of dh (the row-parallel dX GEMMs read every token);
+ *             reduce-scatter of the gate|up-dX and qkv-dX partial sums (RMSNorm backward runs on the rank's rows).
+ * x_c / g_c are read at the rank's own rows; x_s / g_s are all-gathered so every rank returns the whole [T, d].
  * LoRA: column-parallel targets keep A [r, d] replicated and B [N/world, r] sharded; row-parallel targets keep
- * A [r, K/world] sharded and B [d, r] replicated.  Row-parallel adapters fold into the existing all-reduce by
- * linearity; the gradients of the replicated tensors (dA of q,k,v,gate,up; dB of o,down) are partial sums and
- * are all-reduced once per backward per client (one fp32 call over a contiguous region).  No other exchange.
- * The callback must leave identical bytes on every rank (NCCL / gloo all-reduce do).  It returns 0 on success;
- * nonzero makes the server call fail with MENOS_ENCCL.  world <= 1: no tensor parallelism (replica). */
+ * A [r, K/world] sharded and B [d, r] replicated.  Row-parallel adapters fold into the reduce-scatter by linearity;
+ * the gradients of the replicated tensors (dA of q,k,v,gate,up; dB of o,down) are partial sums and are all-reduced
+ * (fp32) once per backward per client over a contiguous region.  No other exchange.
+ * Transport: if `nccl_id` is non-NULL (128 bytes from menos_tp_unique_id on rank 0, broadcast by the caller) the
+ * library creates an NCCL communicator and issues the collectives itself on the call's stream (NCCL over NVLink /
+ * NVSwitch; `collective` is ignored).  Otherwise `collective` is called (e.g. torch.distributed over gloo); it must
+ * be stream-ordered w.r.t. `stream` and leave identical bytes on every rank.  Nonzero return: MENOS_ENCCL.
+ * world <= 1 and nccl_id == NULL: no tensor parallelism (replica).  world == 1 with nccl_id: the sequence-parallel
+ * schedule on one rank (test vehicle for the NCCL transport). */
 enum { MENOS_DT_F32 = 0, MENOS_DT_BF16 = 1 };
-typedef int (*menos_allreduce_fn)(void* buf, size_t count, int dtype, void* stream, void* user);
+enum { MENOS_COLL_ALLREDUCE = 0, MENOS_COLL_ALLGATHER = 1, MENOS_COLL_REDUCE_SCATTER = 2 };
+/* ALLREDUCE: in-place sum of `count` elements (send == recv).  ALLGATHER: send holds `count` elements, recv
+ * world * count (rank-major).  REDUCE_SCATTER: send holds world * count, recv gets this rank's `count` of the sum. */
+typedef int (*menos_collective_fn)(int op, const void* send, void* recv, size_t count, int dtype, void* stream,
+                                   void* user);
 typedef struct {
-  int rank, world;              /* 0 <= rank < world; H, H_kv and d_ff divisible by world              */
-  menos_allreduce_fn allreduce; /* required when world > 1                                              */
-  void* user;                   /* passed back to allreduce                                             */
+  int rank, world;                /* 0 <= rank < world; H, H_kv and d_ff divisible by world               */
+  menos_collective_fn collective; /* caller transport (used when nccl_id == NULL)                          */
+  void* user;                     /* passed back to collective                                             */
+  const void* nccl_id;            /* 128-byte ncclUniqueId, or NULL                                        */
 } menos_tp_cfg;
+/* 128-byte NCCL unique id for menos_tp_cfg.nccl_id (call on one rank, broadcast to the others).  ENCCL if NCCL is
+ * not loadable. */
+MENOS_API int menos_tp_unique_id(void* out128);
+/* Collectives this server has issued on the tensor-parallel path and their payload bytes (an all-reduce counts its
+ * buffer, an all-gather / reduce-scatter world x one rank's share). */
+MENOS_API int menos_tp_stats(menos_server* s, long long* calls, double* bytes);
 
 typedef struct {
   int max_clients;     /* registry capacity (default 64)                                     */

@@ -64,9 +64,14 @@ MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A,
 
 /* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
    bit 1 = tcgen05 backward (else mma.sync), bit 2 = persistent warp-specialized tcgen05 forward (overrides
-   bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1). Returns MENOS_EINVAL outside
-   [0, 15]. */
+   bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1), bit 4 = (sequence, head)-grouped
+   work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1; default mode 46).
+   Returns MENOS_EINVAL outside [0, 63]. */
 MENOS_API int menos_test_set_attn_tc(int mode);
+
+/* Tuning aid: per-phase clock64 totals of the one-pass attention backward's role threads (16 counters, cleared by the
+ * read) when libmenos.so was built with -DMENOS_ABF_PROF (MENOS_NVCC_DEFS); zeros otherwise. */
+MENOS_API int menos_test_abf_prof(unsigned long long* out16);
 
 MENOS_API const char* menos_testing_last_error(void);
 

@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OUT_DIR = os.path.join(HERE, "_lib")
 LIB = os.path.join(OUT_DIR, "libmenos.so")
-SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_ws.cu", "attention_bwd_tc.cu", "attention_bwd_ws.cu", "lora.cu", "elementwise.cu", "server.cu", "testing.cu", "sched.cpp"]
+SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_ws.cu", "attention_bwd_tc.cu", "attention_bwd_ws.cu", "attention_bwd_fused.cu", "lora.cu", "elementwise.cu", "server.cu", "testing.cu", "sched.cpp", "comm.cpp"]
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"),
@@ -54,7 +54,7 @@ def build(verbose: bool = False, force: bool = False) -> str:
     objs = [os.path.join(OUT_DIR, os.path.splitext(s)[0] + ".o") for s in SOURCES]
     if force or jobs or not os.path.exists(LIB):
         cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", LIB, *objs,
-               "-Xcompiler", "-fPIC"]
+               "-Xcompiler", "-fPIC", "-ldl"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode:
             sys.stderr.write(r.stdout + r.stderr)

@@ -389,6 +389,15 @@ void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out
   std::stable_sort(out.begin() + first, out.end(), [&](const int4& a, const int4& b) { return cost(a) > cost(b); });
 }
 
+// (sequence, kv head) items of the one-pass backward, LPT: longest sequence first (stable)
+void attn_seq_items(const int* seq_len, int n_seqs, int Hkv, std::vector<int4>& out) {
+  const size_t first = out.size();
+  for (int i = 0; i < n_seqs; ++i)
+    for (int h = 0; h < Hkv; ++h) out.push_back(make_int4(i, 0, h, 0));
+  std::stable_sort(out.begin() + first, out.end(),
+                   [&](const int4& a, const int4& b) { return seq_len[a.x] > seq_len[b.x]; });
+}
+
 #ifdef MENOS_WS_PROF
 int attn_ws_prof_read(unsigned long long* out) {
   cudaDeviceSynchronize();

@@ -208,6 +208,18 @@ __global__ void bf16_to_f32_vec_kernel(const bf16* __restrict__ s, float* __rest
     st8f(d + 8 * i, v);
   }
 }
+// out = x + float(delta): the sequence-parallel residual add after a reduce-scatter (A16); x, out fp32, delta bf16
+__global__ void add_bf16_f32_kernel(const float* x, const bf16* __restrict__ delta, float* out,
+                                    long long n8) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n8; i += (long long)gridDim.x * blockDim.x) {
+    float a[8], b[8];
+    ld8f(x + 8 * i, a);
+    ld8b(delta + 8 * i, b);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) a[k] += b[k];
+    st8f(out + 8 * i, a);
+  }
+}
 
 // ------------------------------------------------------------------ D = rowsum(dO * O) per (token, head)
 __global__ void attn_prep_kernel(const bf16* __restrict__ dO, const bf16* __restrict__ O, float* __restrict__ D,
@@ -478,6 +490,12 @@ int convert_bf16_to_f32_vec(const bf16* src, float* dst, long long n, cudaStream
   if (n <= 0) return 0;
   if (n % 8) return -1;
   bf16_to_f32_vec_kernel<<<1184, 256, 0, st>>>(src, dst, n / 8);
+  return LAUNCH_CHECK();
+}
+int add_bf16_to_f32(const float* x, const bf16* delta, float* out, long long n, cudaStream_t st) {
+  if (n <= 0) return 0;
+  if (n % 8) return -1;
+  add_bf16_f32_kernel<<<1184, 256, 0, st>>>(x, delta, out, n / 8);
   return LAUNCH_CHECK();
 }
 int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st) {

@@ -95,6 +95,8 @@ int rmsnorm_bwd_f32dy(const float* dy, const float* x, const float* g, const flo
 int convert_f32_to_bf16(const float* src, bf16* dst, long long n, cudaStream_t st);       // n % 8 == 0
 int convert_bf16_to_f32_vec(const bf16* src, float* dst, long long n, cudaStream_t st);   // n % 8 == 0
 int attn_bwd_prep(const bf16* dO, const bf16* O, float* D, int T, int H, int hd, cudaStream_t st);
+// out = x + float(delta) (fp32 residual add of a bf16 reduce-scatter result; n % 8 == 0); out may alias x
+int add_bf16_to_f32(const float* x, const bf16* delta, float* out, long long n, cudaStream_t st);
 
 // ---------------------------------------------------------------- attention (varlen causal, GQA)
 struct AttnArgs {
@@ -113,6 +115,8 @@ struct AttnArgs {
   const float* D;                // [H, T]
   bf16* dqkv; int ld_dqkv;       // dq/dk/dv written pre-RoPE (RoPE backward applied)
   const float2* rope_cs;         // [max_pos][hd/2]
+  // one-pass backward (attention_bwd_fused.cu): per-thread ordered fp32 dQ accumulation
+  float* dq_acc;                 // [T, H*hd] fp32 scratch
 };
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block
@@ -125,9 +129,14 @@ void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out
 // head, -) per 128-key block, items_q = (seq, q0, head, -) per 128-query block
 int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
                 int num_sms, cudaStream_t st);
+// one-pass persistent tcgen05 backward for head_dim 128 (attention_bwd_fused.cu): items = (seq, -, kv head, -), one
+// per (sequence, kv head), longest sequence first (attn_seq_items)
+int attn_bwd_fused(const AttnArgs& a, const int4* items_seq, int n_items, int num_sms, cudaStream_t st);
+void attn_seq_items(const int* seq_len, int n_seqs, int Hkv, std::vector<int4>& out);
+int attn_bwd_fused_prof(unsigned long long* out16);   // tuning: per-phase cycles (-DMENOS_ABF_PROF builds)
 // head_dim 128 variant bitmask: 1 = tcgen05 forward (2-pass), 2 = tcgen05 backward, 4 = persistent
 // warp-specialized tcgen05 forward (takes precedence over 1), 8 = persistent warp-specialized tcgen05 backward
-// (takes precedence over 2)
+// (takes precedence over 2), 32 = one-pass fused tcgen05 backward (takes precedence over 8 and 2)
 extern int g_attn_tc;
 extern int g_attn_order;   // persistent attention work order: 1 = LPT (default), 0 = (sequence, head) grouped
 int attn_bwd(const AttnArgs& a, cudaStream_t st);

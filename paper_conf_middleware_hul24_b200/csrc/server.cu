@@ -19,6 +19,7 @@
 #include "../../include/menos_testing.h"
 #include <type_traits>
 #include "kernels.h"
+#include "comm.h"
 
 using namespace menos;
 
@@ -109,6 +110,7 @@ struct Dims {
   int arch;                        // MENOS_ARCH_LLAMA / MENOS_ARCH_OPT (NEXT-4)
   int gu_cols;                     // columns of the saved MLP activation: [gate|up] 2*fpad (Llama), relu(fc1) fpad (OPT)
   int tp_rank, tp_world;
+  bool sp;                         // tensor parallel with sequence-parallel residual streams (include/menos.h)
   int K_glob[NT];                  // global input dim of each projection (LoRA A init bound, A slicing)
   bool a_rep[NT];                  // A replicated across ranks (column-parallel); else B replicated (row-parallel)
   float eps, theta;
@@ -118,9 +120,9 @@ struct Dims {
   int rb_base[NT], rb_blk[NT], rb_stride[NT];
 };
 
-static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 1) {
+static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 1, bool sp = false) {
   Dims D;
-  D.tp_rank = tp_rank; D.tp_world = tp_world;
+  D.tp_rank = tp_rank; D.tp_world = tp_world; D.sp = sp;
   D.d = c.d_model; D.H = c.n_heads / tp_world; D.Hkv = c.n_kv_heads / tp_world; D.hd = c.d_model / c.n_heads;
   D.f = c.d_ff / tp_world; D.fpad = (int)align_up(D.f, 128);
   D.Nq = D.H * D.hd; D.Nkv = D.Hkv * D.hd; D.Nqkv = D.Nq + 2 * D.Nkv;
@@ -146,6 +148,15 @@ static Dims make_dims(const menos_model_cfg& c, int tp_rank = 0, int tp_world = 
   if (opt) { base[TU] = 0; blk[TU] = big; str[TU] = 0; }   // fc1 rows, not interleaved (gate does not exist)
   for (int t = 0; t < NT; ++t) { D.rb_base[t] = base[t]; D.rb_blk[t] = blk[t]; D.rb_stride[t] = str[t]; }
   return D;
+}
+
+// token rows under sequence parallelism: rank r owns rows [r*Tloc, (r+1)*Tloc), Tpad = world*Tloc >= T (the last
+// rank's rows past T are padding); without it Tloc = Tpad = T
+struct Rows { int T, Tloc, Tpad, row0; };
+static inline Rows rows_of(const Dims& D, int T) {
+  if (!D.sp) return Rows{T, T, T, 0};
+  const int loc = ceil_div(T, D.tp_world);
+  return Rows{T, loc, loc * D.tp_world, loc * D.tp_rank};
 }
 
 // =====================================================================================================
@@ -280,10 +291,10 @@ struct menos_batch {
   // the clients active at layer l (cut <= l) are a prefix: tokens [0, Tl[l]), sequences [0, nseq_l[l])
   std::vector<int> Tl, nseq_l, view_of;
   struct AttnView {
-    int n_seqs = 0, n_blocks = 0, n_blocks128 = 0, n_items = 0, n_items_kv = 0;
+    int n_seqs = 0, n_blocks = 0, n_blocks128 = 0, n_items = 0, n_items_kv = 0, n_items_seq = 0;
     double pairs = 0;
-    size_t o_items = 0, o_items_kv = 0, o_items_q = 0;
-    int4 *items = nullptr, *items_kv = nullptr, *items_q = nullptr;
+    size_t o_items = 0, o_items_kv = 0, o_items_q = 0, o_items_seq = 0;
+    int4 *items = nullptr, *items_kv = nullptr, *items_q = nullptr, *items_seq = nullptr;
   };
   std::vector<AttnView> views;
   // device metadata
@@ -316,7 +327,8 @@ struct menos_server {
   Dims D{};
   int first_layer = 0, n_layers = 0, device = 0, num_sms = 148;
   menos_server_opts opts{};
-  menos_tp_cfg tp{0, 1, nullptr, nullptr};  // tensor parallelism (world 1 = replica)
+  menos_tp_cfg tp{0, 1, nullptr, nullptr, nullptr};  // tensor parallelism (world 1 = replica)
+  Comm comm;                                          // its transport (comm.cpp): NCCL or the caller's callback
   // WeightStore: one bf16 copy of every server layer, packed for the kernels
   uint8_t* wbuf = nullptr; size_t wbytes = 0;
   struct LW {
@@ -598,15 +610,18 @@ extern "C" int menos_server_create(const menos_model_cfg* cfg, int first_layer, 
   menos_server_opts o{};
   if (opts) o = *opts;
   menos_tp_cfg tp = o.tp;
-  if (tp.world <= 1) tp = menos_tp_cfg{0, 1, nullptr, nullptr};
-  if (tp.world > 1) {
-    if (tp.rank < 0 || tp.rank >= tp.world || !tp.allreduce) FAIL(MENOS_EINVAL, "bad tensor-parallel cfg");
+  if (tp.world <= 1 && !tp.nccl_id) tp = menos_tp_cfg{0, 1, nullptr, nullptr, nullptr};
+  if (tp.world < 1) tp.world = 1;
+  if (tp.world > 1 || tp.nccl_id) {
+    if (tp.rank < 0 || tp.rank >= tp.world || (!tp.collective && !tp.nccl_id)) FAIL(MENOS_EINVAL, "bad tensor-parallel cfg");
     if (cfg->n_heads % tp.world || cfg->n_kv_heads % tp.world || cfg->d_ff % tp.world)
       FAIL(MENOS_EINVAL, "H=%d, H_kv=%d, f=%d not divisible by tp world %d", cfg->n_heads, cfg->n_kv_heads,
            cfg->d_ff, tp.world);
   }
   std::unique_ptr<menos_server> s(new menos_server());
-  s->cfg = *cfg; s->D = make_dims(*cfg, tp.rank, tp.world); s->tp = tp;
+  s->cfg = *cfg; s->D = make_dims(*cfg, tp.rank, tp.world, tp.world > 1 || tp.nccl_id != nullptr); s->tp = tp;
+  if (int rc = s->comm.init(tp, device)) return rc;
+  s->tp.nccl_id = nullptr;   // the caller's id buffer is not kept
   s->first_layer = first_layer; s->n_layers = n_layers; s->device = device;
   if (o.max_clients <= 0) o.max_clients = 64;
   if (o.max_rank <= 0) o.max_rank = 64;
@@ -680,6 +695,7 @@ extern "C" void menos_server_destroy(menos_server* s) {
   if (s->wbuf) cudaFree(s->wbuf);
   if (s->rope) cudaFree(s->rope);
   if (s->arena_mem) cudaFree(s->arena_mem);
+  s->comm.destroy();
   for (auto& sl : s->ring) {
     if (sl.buf) cudaFreeHost(sl.buf);
     if (sl.ev) cudaEventDestroy(sl.ev);
@@ -1034,13 +1050,20 @@ extern "C" int menos_sync(menos_server* s) {
 
 extern "C" const char* menos_last_error(void) { return tl_err.c_str(); }
 
+extern "C" int menos_tp_stats(menos_server* s, long long* calls, double* bytes) {
+  if (!s || !calls || !bytes) FAIL(MENOS_EINVAL, "null argument");
+  *calls = s->comm.calls; *bytes = s->comm.bytes;
+  return MENOS_OK;
+}
+
 // =====================================================================================================
 // batch construction (BatchPacker)
 // =====================================================================================================
 struct Scratch {
-  float *dyf, *dxf, *dhf, *xout;     // fp32 residual streams (gradient ping-pong, dh, forward output)
-  bf16 *dyb, *dxb, *dhb;             // bf16 copies (A operands of the dX GEMMs, LoRA dY)
-  bf16 *dhn, *dO, *dqkv, *dgu, *a, *io;  // io: bf16 staging of x_c / x_s / g_c / g_s
+  float *dyf, *dxf, *dhf, *xout;     // fp32 residual streams (gradient ping-pong, dh, forward output); local rows
+  bf16 *dyb, *dxb, *dhb;             // bf16 copies (A operands of the dX GEMMs, LoRA dY); local rows
+  bf16 *dhn, *dO, *dqkv, *dgu, *a, *io;  // io: bf16 staging of x_c / x_s / g_c / g_s ([Tpad, d])
+  bf16 *gath, *rsout;                // sequence parallel: all-gathered dy / dh [Tpad, d]; reduce-scatter output [Tloc, d]
   float* Dsum;
   bf16* dU[NG];
 };
@@ -1075,6 +1098,9 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
     if (k > 0 && cut < s->clients[b->bclients[k - 1]].cut)
       FAIL(MENOS_EINVAL, "clients must be ordered by non-decreasing cut layer (client %d)", b->bclients[k]);
   }
+  if (D.sp)
+    for (int c : b->bclients)
+      if (s->clients[c].cut != 0) FAIL(MENOS_EINVAL, "per-client cut points are not supported with tensor parallelism");
   for (int i = 0; i < n_seqs; ++i) {
     const int cut = s->clients[b->seq_client[i]].cut;
     for (int l = cut; l < s->n_layers; ++l) { b->Tl[l] = b->cu[i + 1]; b->nseq_l[l] = i + 1; }
@@ -1103,12 +1129,13 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
 // arena bytes of a batch's slab: the SAVE activations of every layer (I in Eq.3), or under NOGRAD
 // only the x_c copy; R_used = the batch's block-diagonal LoRA slot widths per group (0 = inactive)
 static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save) {
-  if (!save) return align_up((size_t)T * D.d * 4, 256);
+  const Rows R = rows_of(D, T);   // sequence parallel: x, h, rstd local; xn, hn all-gathered
+  if (!save) return align_up((size_t)R.Tloc * D.d * 4, 256);
   size_t per_layer = 0;
   auto A = [&](size_t n) { per_layer += align_up(n, 256); };
-  A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // x (fp32), xn, rstd1
-  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);  // qkv, O, lse
-  A((size_t)T * D.d * 4); A((size_t)T * D.d * 2); A((size_t)T * 4);        // h (fp32), hn, rstd2
+  A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // x (fp32), xn, rstd1
+  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);        // qkv, O, lse
+  A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // h (fp32), hn, rstd2
   A((size_t)T * D.gu_cols * 2);                                             // gu
   if (save_a) A((size_t)T * D.fpad * 2);
   for (int g = 0; g < NG; ++g) if (R_used[g]) A((size_t)T * R_used[g] * 2);
@@ -1118,16 +1145,18 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
 static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set) {
   size_t need = 0;
   auto A = [&](size_t n) { need += align_up(n, 256); };
-  const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
-  A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout
-  A(db); A(db); A(db); A(db); A(db);                                          // dyb, dxb, dhb, dhn, io
+  const Rows Rw = rows_of(D, T);
+  const size_t df = (size_t)Rw.Tloc * D.d * 4, db = (size_t)Rw.Tloc * D.d * 2, dp = (size_t)Rw.Tpad * D.d * 2;
+  A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout (local rows)
+  A(db); A(db); A(db); A(dp); A(dp);                                          // dyb, dxb, dhb (local), dhn, io
+  if (D.sp) { A(dp); A(db); }                                                 // gathered dy / dh, reduce-scatter out
   A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.gu_cols * 2); A((size_t)T * D.fpad * 2);
-  A((size_t)D.H * T * 4);
+  A((size_t)D.H * T * 4);                                                     // Dsum
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
   if (nograd_set) {
-    A(db); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
-    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * T * 4); A((size_t)T * 8);
+    A(dp); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
+    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * T * 4); A((size_t)Rw.Tloc * 8); A(dp);
     for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   }
   return need;
@@ -1160,7 +1189,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   // one attention view (work lists over the first n sequences) per distinct active prefix
   b->views.clear();
   b->view_of.assign(Ls, -1);
-  std::vector<std::vector<int4>> v_items, v_items_kv, v_items_q;
+  std::vector<std::vector<int4>> v_items, v_items_kv, v_items_q, v_items_seq;
   for (int l = 0; l < Ls; ++l) {
     const int ns = b->nseq_l[l];
     if (ns == 0) continue;
@@ -1175,9 +1204,12 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     v_items.emplace_back(); v_items_kv.emplace_back(); v_items_q.emplace_back();
     attn_ws_items(b->seq_len.data(), ns, D.H, v_items.back(), g_attn_order ? 1 : 0);
     attn_ws_items(b->seq_len.data(), ns, D.Hkv, v_items_kv.back(), g_attn_order ? 2 : 0);
+    v_items_seq.emplace_back();
+    attn_seq_items(b->seq_len.data(), ns, D.Hkv, v_items_seq.back());
     attn_ws_items(b->seq_len.data(), ns, D.H, v_items_q.back(), g_attn_order ? 1 : 0);
     v.n_items = (int)v_items.back().size();
     v.n_items_kv = (int)v_items_kv.back().size();
+    v.n_items_seq = (int)v_items_seq.back().size();
     b->views.push_back(v);
     b->view_of[l] = (int)b->views.size() - 1;
   }
@@ -1214,6 +1246,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->views[v].o_items = put(v_items[v].data(), v_items[v].size() * sizeof(int4));
     b->views[v].o_items_kv = put(v_items_kv[v].data(), v_items_kv[v].size() * sizeof(int4));
     b->views[v].o_items_q = put(v_items_q[v].data(), v_items_q[v].size() * sizeof(int4));
+    b->views[v].o_items_seq = put(v_items_seq[v].data(), v_items_seq[v].size() * sizeof(int4));
   }
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
@@ -1223,14 +1256,17 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   if (!slab) FAIL(MENOS_ENOMEM, "arena: batch needs %zu B, %zu of %zu B in use", slab_bytes, s->arena.used, s->arena.cap);
   b->slab = slab;
   b->L.assign(Ls, LayerSave{});
+  const Rows Rw = rows_of(D, T);
   if (save) {
     uint8_t* p = slab;
     auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
     for (int l = 0; l < Ls; ++l) {
       LayerSave& S = b->L[l];
-      S.x = (float*)take((size_t)T * D.d * 4); S.xn = (bf16*)take((size_t)T * D.d * 2); S.rstd1 = (float*)take((size_t)T * 4);
+      S.x = (float*)take((size_t)Rw.Tloc * D.d * 4); S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
+      S.rstd1 = (float*)take((size_t)Rw.Tloc * 4);
       S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2); S.lse = (float*)take((size_t)D.H * T * 4);
-      S.h = (float*)take((size_t)T * D.d * 4); S.hn = (bf16*)take((size_t)T * D.d * 2); S.rstd2 = (float*)take((size_t)T * 4);
+      S.h = (float*)take((size_t)Rw.Tloc * D.d * 4); S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
+      S.rstd2 = (float*)take((size_t)Rw.Tloc * 4);
       S.gu = (bf16*)take((size_t)T * D.gu_cols * 2);
       S.a = D.arch == MENOS_ARCH_OPT ? S.gu : b->save_a ? (bf16*)take((size_t)T * D.fpad * 2) : sc.a;
       for (int g = 0; g < NG; ++g) S.U[g] = b->g_active[g] ? (bf16*)take((size_t)T * b->R_used[g] * 2) : nullptr;
@@ -1266,7 +1302,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   };
   for (int l = 0; l < Ls; ++l) {
     const LayerSave& S = save ? b->L[l] : *ng;
-    bf16* dyl = ((Ls - 1 - l) % 2 == 0) ? sc.dyb : sc.dxb;  // bf16 copy of layer l's incoming gradient
+    // bf16 copy of layer l's incoming gradient (sequence parallel: its all-gather, which also holds dh later)
+    bf16* dyl = D.sp ? sc.gath : ((Ls - 1 - l) % 2 == 0) ? sc.dyb : sc.dxb;
     for (int g = 0; g < NG; ++g) {
       if (!b->g_active[g]) continue;
       const int R = b->R_used[g];
@@ -1276,7 +1313,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       bf16* U = S.U[g];
       switch (g) {
         case GQKV: X = S.xn; ldx = D.d; dY = sc.dqkv; ldy = D.Nqkv; break;
-        case GO: X = S.O; ldx = D.Nq; dY = sc.dhb; ldy = D.d; break;
+        case GO: X = S.O; ldx = D.Nq; dY = D.sp ? sc.gath : sc.dhb; ldy = D.d; break;
         case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = D.gu_cols; break;
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
@@ -1360,6 +1397,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     v.items = (int4*)(meta + v.o_items);
     v.items_kv = (int4*)(meta + v.o_items_kv);
     v.items_q = (int4*)(meta + v.o_items_q);
+    v.items_seq = (int4*)(meta + v.o_items_seq);
   }
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
@@ -1379,7 +1417,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
 static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set) {
   const Dims& D = s->D;
   const size_t need = scratch_bytes_of(D, T, R_used, nograd_set);
-  const size_t df = (size_t)T * D.d * 4, db = (size_t)T * D.d * 2;
+  const Rows Rw = rows_of(D, T);
+  const size_t df = (size_t)Rw.Tloc * D.d * 4, db = (size_t)Rw.Tloc * D.d * 2, dp = (size_t)Rw.Tpad * D.d * 2;
   if (need != s->scratch_bytes) {   // shrink-to-fit too: a stale large block must not outlive the call that needed it
     if (s->scratch) s->arena.release(s->scratch);
     s->scratch = (uint8_t*)s->arena.alloc(need);
@@ -1389,8 +1428,10 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   uint8_t* p = s->scratch;
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
   sc.dyf = (float*)take(df); sc.dxf = (float*)take(df); sc.dhf = (float*)take(df); sc.xout = (float*)take(df);
-  sc.dyb = (bf16*)take(db); sc.dxb = (bf16*)take(db); sc.dhb = (bf16*)take(db); sc.dhn = (bf16*)take(db);
-  sc.io = (bf16*)take(db);
+  sc.dyb = (bf16*)take(db); sc.dxb = (bf16*)take(db); sc.dhb = (bf16*)take(db); sc.dhn = (bf16*)take(dp);
+  sc.io = (bf16*)take(dp);
+  sc.gath = sc.rsout = nullptr;
+  if (D.sp) { sc.gath = (bf16*)take(dp); sc.rsout = (bf16*)take(db); }
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
   sc.dgu = (bf16*)take((size_t)T * D.gu_cols * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
   sc.Dsum = (float*)take((size_t)D.H * T * 4);
@@ -1401,13 +1442,14 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
 // NOGRAD layer buffers carved after the regular scratch (same arena block)
 static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scratch& sc, LayerSave& S) {
   const Dims& D = s->D;
+  const Rows Rw = rows_of(D, T);
   uint8_t* p = (uint8_t*)(sc.dU[NG - 1]) + align_up((size_t)T * R_used[NG - 1] * 2, 256);
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
-  S.xn = (bf16*)take((size_t)T * D.d * 2); S.h = (float*)take((size_t)T * D.d * 4);
+  S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2); S.h = (float*)take((size_t)Rw.Tloc * D.d * 4);
   S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
   S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * T * 4);
-  S.rstd1 = (float*)take((size_t)T * 8); S.rstd2 = S.rstd1 + T;
-  S.hn = sc.dhn;  // free during a forward
+  S.rstd1 = (float*)take((size_t)Rw.Tloc * 8); S.rstd2 = S.rstd1 + Rw.Tloc;
+  S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
   S.a = D.arch == MENOS_ARCH_OPT ? S.gu : sc.a;   // OPT: the down projection's input is relu(fc1), kept in gu
   for (int g = 0; g < NG; ++g) S.U[g] = (bf16*)take((size_t)T * R_used[g] * 2);
 }
@@ -1429,11 +1471,19 @@ static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
 // tensor-parallel all-reduce (sum, in place, stream-ordered) through the caller's callback (menos_tp_cfg)
 static int tp_allreduce(menos_server* s, void* buf, size_t count, int dtype, cudaStream_t st) {
   if (s->tp.world <= 1 || count == 0) return MENOS_OK;
-  const int rc = s->tp.allreduce(buf, count, dtype, (void*)st, s->tp.user);
-  if (rc) FAIL(MENOS_ENCCL, "tensor-parallel all-reduce failed (%d) on rank %d", rc, s->tp.rank);
-  return MENOS_OK;
+  return s->comm.run(MENOS_COLL_ALLREDUCE, buf, buf, count, dtype, st);
 }
 static inline bool tp_on(const menos_server* s) { return s->tp.world > 1; }
+
+// sequence parallel (A16): all-gather of the rank's [Tloc, d] rows (already in place at buf + row0 d) into [Tpad, d]
+static int sp_gather(menos_server* s, const Rows& R, bf16* buf, cudaStream_t st) {
+  return s->comm.run(MENOS_COLL_ALLGATHER, buf + (size_t)R.row0 * s->D.d, buf, (size_t)R.Tloc * s->D.d, MENOS_DT_BF16, st);
+}
+// reduce-scatter of a [Tpad, d] partial sum (rows past T zeroed) into the rank's [Tloc, d] rows
+static int sp_scatter(menos_server* s, const Rows& R, bf16* part, bf16* out, cudaStream_t st) {
+  if (R.Tpad > R.T) CUDA_TRY(cudaMemsetAsync(part + (size_t)R.T * s->D.d, 0, (size_t)(R.Tpad - R.T) * s->D.d * 2, st));
+  return s->comm.run(MENOS_COLL_REDUCE_SCATTER, part, out, (size_t)R.Tloc * s->D.d, MENOS_DT_BF16, st);
+}
 
 static GemmArgs gemm_base(menos_server* s) {
   GemmArgs a;
@@ -1443,20 +1493,25 @@ static GemmArgs gemm_base(menos_server* s) {
 }
 
 // forward of layer l: x -> y; S holds the destinations of every intermediate
+// x, y: the layer's fp32 residual stream in / out (sequence parallel: the rank's Tloc rows)
 static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x, float* y, const LayerSave& S,
-                         bool use_lists, cudaStream_t st) {
+                         const Scratch& sc, bool use_lists, cudaStream_t st) {
   const Dims& D = s->D;
   const auto& W = s->W[l];
   const int T = b->Tl[l];
   if (T == 0) return MENOS_OK;
+  const Rows R = rows_of(D, T);
   const menos_batch::AttnView& V = b->views[b->view_of[l]];
   const bool opt = D.arch == MENOS_ARCH_OPT;
-  // A1: RMSNorm1 (OPT: LayerNorm1) (fp32 residual in, bf16 GEMM operand out)
+  // A1: RMSNorm1 (OPT: LayerNorm1) (fp32 residual in, bf16 GEMM operand out); sequence parallel: on the rank's rows,
+  // written in place into the all-gather buffer
   {
-    ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st);
-    if (opt) K_TRY(layernorm_fwd(x, W.g1, W.be1, S.xn, S.rstd1, T, D.d, D.eps, st));
-    else K_TRY(rmsnorm_fwd(x, W.g1, S.xn, S.rstd1, T, D.d, D.eps, st));
+    ProfScope ps(PC_NORM, 0, (double)R.Tloc * (6.0 * D.d + 4), st);
+    bf16* xn = S.xn + (size_t)R.row0 * D.d;
+    if (opt) K_TRY(layernorm_fwd(x, W.g1, W.be1, xn, S.rstd1, R.Tloc, D.d, D.eps, st));
+    else K_TRY(rmsnorm_fwd(x, W.g1, xn, S.rstd1, R.Tloc, D.d, D.eps, st));
   }
+  if (D.sp) { int rc = sp_gather(s, R, S.xn, st); if (rc) return rc; }   // A16: every token's xn for the QKV GEMM
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
   if (b->g_active[GQKV]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
@@ -1501,17 +1556,22 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     }
     a.epi = EPI_RESID; a.outf = S.h; a.ldo = D.d; a.resid = x; a.ldr = D.d;
     if (opt) a.bias = W.bo;
-    if (D.tp_rank != 0) a.resid = nullptr;  // row-parallel: rank 0's partial carries the residual
+    if (D.sp) { a.epi = EPI_STORE; a.out = sc.dhn; a.outf = nullptr; a.resid = nullptr; }   // row-parallel partial
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
-    int rc = tp_allreduce(s, S.h, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: o-proj partial sums
-    if (rc) return rc;
+    if (D.sp) {   // A16: reduce-scatter of the o-proj partial sums, then the residual add on the rank's rows
+      int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st);
+      if (rc) return rc;
+      K_TRY(add_bf16_to_f32(x, sc.rsout, S.h, (long long)R.Tloc * D.d, st));
+    }
   }
   // A5: RMSNorm2 (OPT: LayerNorm2)
   {
-    ProfScope ps(PC_NORM, 0, (double)T * (6.0 * D.d + 4), st);
-    if (opt) K_TRY(layernorm_fwd(S.h, W.g2, W.be2, S.hn, S.rstd2, T, D.d, D.eps, st));
-    else K_TRY(rmsnorm_fwd(S.h, W.g2, S.hn, S.rstd2, T, D.d, D.eps, st));
+    ProfScope ps(PC_NORM, 0, (double)R.Tloc * (6.0 * D.d + 4), st);
+    bf16* hn = S.hn + (size_t)R.row0 * D.d;
+    if (opt) K_TRY(layernorm_fwd(S.h, W.g2, W.be2, hn, S.rstd2, R.Tloc, D.d, D.eps, st));
+    else K_TRY(rmsnorm_fwd(S.h, W.g2, hn, S.rstd2, R.Tloc, D.d, D.eps, st));
   }
+  if (D.sp) { int rc = sp_gather(s, R, S.hn, st); if (rc) return rc; }   // A16: every token's hn for gate|up
   // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
   if (b->g_active[GGU]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
@@ -1542,10 +1602,13 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     }
     a.epi = EPI_RESID; a.outf = y; a.ldo = D.d; a.resid = S.h; a.ldr = D.d;
     if (opt) a.bias = W.bd;
-    if (D.tp_rank != 0) a.resid = nullptr;
+    if (D.sp) { a.epi = EPI_STORE; a.out = sc.dhn; a.outf = nullptr; a.resid = nullptr; }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
-    int rc = tp_allreduce(s, y, (size_t)T * D.d, MENOS_DT_F32, st);      // A16: down-proj partial sums
-    if (rc) return rc;
+    if (D.sp) {   // A16: reduce-scatter of the down-proj partial sums, residual add on the rank's rows
+      int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st);
+      if (rc) return rc;
+      K_TRY(add_bf16_to_f32(S.h, sc.rsout, y, (long long)R.Tloc * D.d, st));
+    }
   }
   return MENOS_OK;
 }
@@ -1561,6 +1624,13 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   if (T == 0) return MENOS_OK;
   const menos_batch::AttnView& V = b->views[b->view_of[l]];
   const bool opt = D.arch == MENOS_ARCH_OPT;
+  const Rows R = rows_of(D, T);
+  if (D.sp) {   // A16: every token's incoming gradient for the row-parallel down-dX GEMM (and LoRA down)
+    CUDA_TRY(cudaMemcpyAsync(sc.gath + (size_t)R.row0 * D.d, dy, (size_t)R.Tloc * D.d * 2, cudaMemcpyDeviceToDevice, st));
+    int rc = sp_gather(s, R, sc.gath, st);
+    if (rc) return rc;
+    dy = sc.gath;
+  }
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
   if (b->g_active[GD]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GD], st));
   {
@@ -1587,17 +1657,22 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GGU];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
-    if (tp_on(s)) { a.epi = EPI_RESID; a.outf = sc.xout; a.resid = nullptr; }  // fp32 partial for the all-reduce
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
-    int rc = tp_allreduce(s, sc.xout, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: gate|up-dX partial sums
-    if (rc) return rc;
+    if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: gate|up-dX partials
   }
   if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
   {
-    ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
-    if (opt) K_TRY(layernorm_bwd(sc.dhn, S.h, W.g2, dyf, sc.dhf, sc.dhb, T, D.d, D.eps, st));
-    else if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
-    else K_TRY(rmsnorm_bwd(sc.dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, T, D.d, st));
+    ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
+    const bf16* dhn = D.sp ? sc.rsout : sc.dhn;
+    if (opt) K_TRY(layernorm_bwd(dhn, S.h, W.g2, dyf, sc.dhf, sc.dhb, R.Tloc, D.d, D.eps, st));
+    else K_TRY(rmsnorm_bwd(dhn, S.h, W.g2, S.rstd2, dyf, sc.dhf, sc.dhb, R.Tloc, D.d, st));
+  }
+  bf16* dh_all = sc.dhb;   // the O-dX GEMM's A operand: every token's dh
+  if (D.sp) {               // A16
+    CUDA_TRY(cudaMemcpyAsync(sc.gath + (size_t)R.row0 * D.d, sc.dhb, (size_t)R.Tloc * D.d * 2, cudaMemcpyDeviceToDevice, st));
+    int rc = sp_gather(s, R, sc.gath, st);
+    if (rc) return rc;
+    dh_all = sc.gath;
   }
   // A10: O dX (+ LoRA o) -> dO (and, for head_dim % 32 == 0, the attention backward's row sums D)
   const bool fuse_dsum = D.hd % 32 == 0 && 128 % D.hd == 0;
@@ -1605,7 +1680,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
-    a.A = sc.dhb; a.lda = D.d; a.B = W.wo; a.ldb = D.Nq;
+    a.A = dh_all; a.lda = D.d; a.B = W.wo; a.ldb = D.Nq;
     if (b->g_active[GO]) {
       a.R = b->R_used[GO]; a.A2 = sc.dU[GO]; a.lda2 = a.R; a.B2 = s->Acat[GO][l]; a.ldb2 = D.ldK_g[GO];
       a.mtile_extra = b->d_mtile[GO];
@@ -1630,9 +1705,13 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv;
     a.rope_cs = opt ? nullptr : s->rope;   // OPT: no RoPE backward
+    // one-pass backward: dQ accumulates in fp32 in the forward-output buffer (free during the backward: Nq <= d)
+    a.dq_acc = sc.xout;
     {
       ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * V.pairs, 0, st);
-      if (D.hd == 128 && (g_attn_tc & 8))
+      if (D.hd == 128 && (g_attn_tc & 32))
+        K_TRY(attn_bwd_fused(a, V.items_seq, V.n_items_seq, s->num_sms, st));
+      else if (D.hd == 128 && (g_attn_tc & 8))
         K_TRY(attn_bwd_ws(a, V.items_kv, V.n_items_kv, V.items_q, V.n_items, s->num_sms, st));
       else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, V.n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
@@ -1649,17 +1728,15 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
       a.mtile_extra = b->d_mtile[GQKV];
     }
     a.epi = EPI_STORE; a.out = sc.dhn; a.ldo = D.d;
-    if (tp_on(s)) { a.epi = EPI_RESID; a.outf = sc.xout; a.resid = nullptr; }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
-    int rc = tp_allreduce(s, sc.xout, (size_t)T * D.d, MENOS_DT_F32, st);   // A16: qkv-dX partial sums
-    if (rc) return rc;
+    if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: qkv-dX partials
   }
   if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
   {
-    ProfScope ps(PC_NORM, 0, (double)T * (16.0 * D.d + 4), st);
-    if (opt) K_TRY(layernorm_bwd(sc.dhn, S.x, W.g1, sc.dhf, dxf, dxb, T, D.d, D.eps, st));
-    else if (tp_on(s)) K_TRY(rmsnorm_bwd_f32dy(sc.xout, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
-    else K_TRY(rmsnorm_bwd(sc.dhn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, T, D.d, st));
+    ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
+    const bf16* dxn = D.sp ? sc.rsout : sc.dhn;
+    if (opt) K_TRY(layernorm_bwd(dxn, S.x, W.g1, sc.dhf, dxf, dxb, R.Tloc, D.d, D.eps, st));
+    else K_TRY(rmsnorm_bwd(dxn, S.x, W.g1, S.rstd1, sc.dhf, dxf, dxb, R.Tloc, D.d, st));
   }
   return MENOS_OK;
 }
@@ -1679,7 +1756,7 @@ static int join_rows(menos_server* s, menos_batch* b, int l, float* x, cudaStrea
 static int forward_save(menos_server* s, menos_batch* b, const Scratch& sc, float* xout, cudaStream_t st) {
   for (int l = 0; l < s->n_layers; ++l) {
     float* y = (l + 1 < s->n_layers) ? b->L[l + 1].x : xout;
-    int rc = layer_forward(s, b, l, b->L[l].x, y, b->L[l], true, st);
+    int rc = layer_forward(s, b, l, b->L[l].x, y, b->L[l], sc, true, st);
     if (rc) return rc;
     rc = join_rows(s, b, l + 1, y, st);
     if (rc) return rc;
@@ -1717,9 +1794,12 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     if (b->meta) s->arena.release(b->meta);
     return code;
   };
-  // x_c (bf16, host or device) -> staging -> the fp32 residual stream X[0]
+  // x_c (bf16, host or device) -> staging -> the fp32 residual stream X[0] (sequence parallel: the rank's rows;
+  // padding rows zero)
+  const Rows R = rows_of(D, T);
+  if (R.Tpad > T) CUDA_TRY(cudaMemsetAsync(sc.io + (size_t)T * D.d, 0, (size_t)(R.Tpad - T) * D.d * 2, st));
   if (cudaMemcpyAsync(sc.io, x_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess ||
-      convert_bf16_to_f32_vec(sc.io, b->L[0].x, (long long)T * D.d, st) != 0) {
+      convert_bf16_to_f32_vec(sc.io + (size_t)R.row0 * D.d, b->L[0].x, (long long)R.Tloc * D.d, st) != 0) {
     set_err("copy of x_c failed");
     return fail_free(MENOS_ECUDA);
   }
@@ -1731,15 +1811,19 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
     const float* x = b->L[0].x;
     for (int l = 0; l < s->n_layers; ++l) {
       float* y = ((s->n_layers - 1 - l) % 2 == 0) ? sc.xout : sc.dxf;
-      rc = layer_forward(s, b.get(), l, x, y, ng, true, st);
+      rc = layer_forward(s, b.get(), l, x, y, ng, sc, true, st);
       if (rc) return fail_free(rc);
       rc = join_rows(s, b.get(), l + 1, y, st);
       if (rc) return fail_free(rc);
       x = y;
     }
   }
-  if (convert_f32_to_bf16(sc.xout, sc.io, (long long)T * D.d, st) != 0 ||
-      cudaMemcpyAsync(x_s, sc.io, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
+  if (convert_f32_to_bf16(sc.xout, sc.io + (size_t)R.row0 * D.d, (long long)R.Tloc * D.d, st) != 0) {
+    set_err("conversion of x_s failed");
+    return fail_free(MENOS_ECUDA);
+  }
+  if (D.sp) { rc = sp_gather(s, R, sc.io, st); if (rc) return fail_free(rc); }   // every rank returns all of x_s
+  if (cudaMemcpyAsync(x_s, sc.io, (size_t)T * D.d * 2, cudaMemcpyDefault, st) != cudaSuccess) {
     set_err("copy of x_s failed");
     return fail_free(MENOS_ECUDA);
   }
@@ -1799,6 +1883,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   if (int rc0 = bind_stream(s, st)) return rc0;
   const Dims& D = s->D;
   const int T = b->T;
+  const Rows R = rows_of(D, T);
   Scratch sc;
   int rc = get_scratch(s, T, b->R_used, sc, false);
   if (rc) return rc;
@@ -1812,7 +1897,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
     b->nograd = false;
     rc = finalize_batch(s, b, sc, nullptr, st);
     if (rc) { b->nograd = true; b->slab = old_slab; b->meta = old_meta; return rc; }
-    CUDA_TRY(cudaMemcpyAsync(b->L[0].x, xc, (size_t)T * D.d * 4, cudaMemcpyDeviceToDevice, st));
+    CUDA_TRY(cudaMemcpyAsync(b->L[0].x, xc, (size_t)R.Tloc * D.d * 4, cudaMemcpyDeviceToDevice, st));
     s->arena.release(old_meta);   // stream-ordered reuse: later users run after these copies
     s->arena.release(old_slab);
     rc = forward_save(s, b, sc, sc.xout, st);
@@ -1821,9 +1906,16 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
     rc = relocate_scratch_refs(s, b, st);
     if (rc) return rc;
   }
-  // g_c (bf16) -> the bf16 copy of the incoming gradient and the fp32 gradient residual stream
-  CUDA_TRY(cudaMemcpyAsync(sc.dyb, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
-  K_TRY(convert_bf16_to_f32_vec(sc.dyb, sc.dyf, (long long)T * D.d, st));
+  // g_c (bf16) -> the bf16 copy of the incoming gradient and the fp32 gradient residual stream (sequence parallel:
+  // the rank's rows, padding rows zero)
+  if (D.sp) {
+    if (R.Tpad > T) CUDA_TRY(cudaMemsetAsync(sc.io + (size_t)T * D.d, 0, (size_t)(R.Tpad - T) * D.d * 2, st));
+    CUDA_TRY(cudaMemcpyAsync(sc.io, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+    CUDA_TRY(cudaMemcpyAsync(sc.dyb, sc.io + (size_t)R.row0 * D.d, (size_t)R.Tloc * D.d * 2, cudaMemcpyDeviceToDevice, st));
+  } else {
+    CUDA_TRY(cudaMemcpyAsync(sc.dyb, g_c, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  }
+  K_TRY(convert_bf16_to_f32_vec(sc.dyb, sc.dyf, (long long)R.Tloc * D.d, st));
   // the block-diagonal dU scratch: zero once (a batch's slot positions are the same in every layer)
   for (int g = 0; g < NG; ++g)
     if (b->g_active[g]) CUDA_TRY(cudaMemsetAsync(sc.dU[g], 0, (size_t)T * b->R_used[g] * 2, st));
@@ -1849,7 +1941,12 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
       rc = tp_allreduce(s, s->clients[c].G(), s->clients[c].n_rep, MENOS_DT_F32, st);
       if (rc) return rc;
     }
-  CUDA_TRY(cudaMemcpyAsync(g_s, mixed_cuts ? sc.io : dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
+  if (D.sp) {   // every rank returns all of g_s
+    CUDA_TRY(cudaMemcpyAsync(sc.io + (size_t)R.row0 * D.d, dyb, (size_t)R.Tloc * D.d * 2, cudaMemcpyDeviceToDevice, st));
+    rc = sp_gather(s, R, sc.io, st);
+    if (rc) return rc;
+  }
+  CUDA_TRY(cudaMemcpyAsync(g_s, (mixed_cuts || D.sp) ? sc.io : dyb, (size_t)T * D.d * 2, cudaMemcpyDefault, st));
   cudaPointerAttributes pa;
   if (cudaPointerGetAttributes(&pa, g_s) == cudaSuccess && pa.type != cudaMemoryTypeDevice &&
       pa.type != cudaMemoryTypeManaged)
@@ -1869,14 +1966,15 @@ extern "C" int menos_test_batch_tensor(menos_server* s, menos_batch* b, int laye
   const Dims& D = s->D;
   const LayerSave& S = b->L[layer];
   const size_t T = b->T;
+  const Rows R = rows_of(D, b->T);   // sequence parallel: x, h are the rank's rows; xn, hn all-gathered (padded)
   const void* src = nullptr;
   size_t n = 0;
   switch (which) {
-    case 0: src = S.x; n = T * D.d * 4; break;
+    case 0: src = S.x; n = (size_t)R.Tloc * D.d * 4; break;
     case 1: src = S.xn; n = T * D.d * 2; break;
     case 2: src = S.qkv; n = T * D.Nqkv * 2; break;
     case 3: src = S.O; n = T * D.Nq * 2; break;
-    case 4: src = S.h; n = T * D.d * 4; break;
+    case 4: src = S.h; n = (size_t)R.Tloc * D.d * 4; break;
     case 5: src = S.hn; n = T * D.d * 2; break;
     case 6: src = S.gu; n = T * D.gu_cols * 2; break;
     case 7: src = S.a; n = T * D.fpad * 2; break;

@@ -115,10 +115,22 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
     cudaMalloc(&d_items_kv, std::max<size_t>(1, items_kv.size()) * sizeof(int4));
     cudaMemcpy(d_items_kv, items_kv.data(), items_kv.size() * sizeof(int4), cudaMemcpyHostToDevice);
     const bool ws_bwd = hd == 128 && (g_attn_tc & 8);
-    rc = ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
-                : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+    const bool fused_bwd = hd == 128 && (g_attn_tc & 32);
+    float* d_acc = nullptr;
+    std::vector<int4> items_seq;
+    int4* d_items_seq = nullptr;
+    if (fused_bwd) {
+      attn_seq_items(seq_len, n_seqs, Hkv, items_seq);
+      cudaMalloc(&d_items_seq, items_seq.size() * sizeof(int4));
+      cudaMemcpy(d_items_seq, items_seq.data(), items_seq.size() * sizeof(int4), cudaMemcpyHostToDevice);
+      cudaMalloc(&d_acc, (size_t)T * H * hd * sizeof(float));
+      a.dq_acc = d_acc;
+    }
+    rc = fused_bwd ? attn_bwd_fused(a, d_items_seq, (int)items_seq.size(), sms, 0)
+         : ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
+                  : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
     cudaDeviceSynchronize();
-    cudaFree(d_items_kv);
+    cudaFree(d_items_kv); cudaFree(d_acc); cudaFree(d_items_seq);
   }
   cudaError_t e = cudaDeviceSynchronize();
   cudaFree(d_cu); cudaFree(d_blk); cudaFree(d_cs); cudaFree(d_D); cudaFree(d_b128); cudaFree(d_items);
@@ -218,11 +230,16 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
 // (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1),
 // 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; overrides 2).
 // Default 14: the persistent tcgen05 forward and backward (LPT work order, bit 4 selects (sequence, head) order).
-namespace menos { int g_attn_tc = 14; int g_attn_order = 1; }
+namespace menos { int g_attn_tc = 46; int g_attn_order = 1; }
+extern "C" int menos_test_abf_prof(unsigned long long* out16) {
+  if (!out16) return fail("null output");
+  return menos::attn_bwd_fused_prof(out16);
+}
+
 extern "C" int menos_test_set_attn_tc(int mode) {
-  if (mode < 0 || mode > 31) { fail("attention mode must be in [0, 31]"); return MENOS_EINVAL; }
+  if (mode < 0 || mode > 63) { fail("attention mode must be in [0, 63]"); return MENOS_EINVAL; }
   menos::g_attn_order = (mode & 16) ? 0 : 1;   // bit 4: (sequence, head)-grouped work order instead of LPT
-  mode &= 15;
+  mode &= 47;                                  // bit 5: one-pass fused backward
   menos::g_attn_tc = mode;
   return MENOS_OK;
 }

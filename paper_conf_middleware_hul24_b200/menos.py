@@ -43,11 +43,12 @@ class AdamWCfg(C.Structure):
                 ("weight_decay", C.c_double)]
 
 
-from .tp import ALLREDUCE_FN, wrap_allreduce  # noqa: E402
+from .tp import COLLECTIVE_FN, wrap_collective  # noqa: E402
 
 
 class TPCfg(C.Structure):
-    _fields_ = [("rank", C.c_int), ("world", C.c_int), ("allreduce", ALLREDUCE_FN), ("user", C.c_void_p)]
+    _fields_ = [("rank", C.c_int), ("world", C.c_int), ("collective", COLLECTIVE_FN), ("user", C.c_void_p),
+                ("nccl_id", C.c_void_p)]
 
 
 class ServerOpts(C.Structure):
@@ -97,6 +98,8 @@ SIGNATURES = {
     "menos_profile_enable": (_I, [_I]),
     "menos_profile_read": (_I, [C.POINTER(KernelStat), _I, C.POINTER(_I)]),
     "menos_sync": (_I, [_P]),
+    "menos_tp_unique_id": (_I, [_P]),
+    "menos_tp_stats": (_I, [_P, C.POINTER(C.c_longlong), C.POINTER(C.c_double)]),
     "menos_last_error": (C.c_char_p, []),
     "menos_test_gemm": (_I, [_I, _I, _I, _I, _P, _I, _P, _I, _P, _I, _P, _I, _I, _PI32, _I, _P, _I, _P, _I, _P, _I,
                              _P, _I, _I, _I, _PI32, _F, _I]),
@@ -108,6 +111,7 @@ SIGNATURES = {
     "menos_test_set_gemm_cta_group": (_I, [_I]),
     "menos_test_gemm_time": (_I, [_I, _I, _I, _I, _P, _P, _P, _I, _P, _I, C.POINTER(C.c_float)]),
     "menos_test_set_attn_tc": (_I, [_I]),
+    "menos_test_abf_prof": (_I, [C.POINTER(C.c_ulonglong)]),
     "menos_testing_last_error": (C.c_char_p, []),
     "menos_sched_create": (_I, [_S, _I, C.POINTER(_P)]),
     "menos_sched_destroy": (None, [_P]),
@@ -201,17 +205,22 @@ class Server:
     def __init__(self, d_model, n_heads, n_kv_heads, d_ff, n_layers, first_layer=1, rms_eps=1e-5,
                  rope_theta=1e4, weights=None, device=0, max_clients=64, max_rank=64, max_seq_len=4096,
                  arena_bytes=0, num_sms=0, tp=None, arch="llama"):
-        """tp = (rank, world, allreduce) for tensor parallelism (include/menos.h menos_tp_cfg): `weights` are
-        then the rank's shards (tp.shard_layer_weights) and `allreduce(buf, count, dtype, stream)` is an in-place
-        sum over the ranks (tp.make_torch_allreduce)."""
+        """tp = (rank, world, transport) for tensor parallelism (include/menos.h menos_tp_cfg): `weights` are then the
+        rank's shards (tp.shard_layer_weights); transport is either the 128-byte NCCL unique id (bytes, from
+        tp.nccl_unique_id on rank 0, broadcast by the caller: the library drives NCCL itself) or a Python collective
+        (op, send, recv, count, dtype, stream) -> int (tp.make_torch_collective)."""
         self.cfg = ModelCfg(d_model, n_heads, n_kv_heads, d_ff, rms_eps, rope_theta, ARCH[arch])
         self.n_layers = n_layers
         self.device = device
-        tpc = TPCfg(0, 1, ALLREDUCE_FN(), None)
-        self._tp_cb = None
-        if tp is not None and tp[1] > 1:
-            self._tp_cb = wrap_allreduce(tp[2])   # kept alive as long as the server
-            tpc = TPCfg(tp[0], tp[1], self._tp_cb, None)
+        tpc = TPCfg(0, 1, COLLECTIVE_FN(), None, None)
+        self._tp_cb = self._tp_id = None
+        if tp is not None and (tp[1] > 1 or isinstance(tp[2], (bytes, bytearray))):
+            if isinstance(tp[2], (bytes, bytearray)):
+                self._tp_id = C.create_string_buffer(bytes(tp[2]), 128)
+                tpc = TPCfg(tp[0], tp[1], COLLECTIVE_FN(), None, C.cast(self._tp_id, C.c_void_p))
+            else:
+                self._tp_cb = wrap_collective(tp[2])   # kept alive as long as the server
+                tpc = TPCfg(tp[0], tp[1], self._tp_cb, None, None)
         self.tp_rank, self.tp_world = (tp[0], tp[1]) if tp is not None else (0, 1)
         opts = ServerOpts(max_clients, max_rank, max_seq_len, arena_bytes, num_sms, tpc)
         h = C.c_void_p()
@@ -336,6 +345,12 @@ class Server:
 
     def sync(self):
         check(lib().menos_sync(self.h))
+
+    def tp_stats(self) -> dict:
+        """Collectives the tensor-parallel path issued and their payload bytes (menos_tp_stats)."""
+        n, b = C.c_longlong(), C.c_double()
+        check(lib().menos_tp_stats(self.h, C.byref(n), C.byref(b)))
+        return {"calls": n.value, "bytes": b.value}
 
 
 def launch_count() -> int:

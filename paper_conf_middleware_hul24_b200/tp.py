@@ -1,9 +1,9 @@
 """Tensor parallelism for the largest model (Llama-2-70B, BASELINE.json configs[4]).
 
 Host-side logic only (argument marshalling): which slice of every base weight and LoRA adapter a rank holds, how the
-shards reassemble, and the all-reduce callback `menos_tp_cfg.allreduce` (include/menos.h) implemented with
-torch.distributed (NCCL over NVLink on a multi-GPU box; gloo for the single-GPU / CPU tests).  Every step of the
-path still runs in libmenos.so; the library calls the callback at the four per-layer exchange points.
+shards reassemble, the NCCL unique id handshake (the library then drives NCCL itself), and a torch.distributed
+collective callback (`menos_tp_cfg.collective`, include/menos.h) for the single-GPU gloo tests.  Every step of the
+path runs in libmenos.so.
 
 Split (Megatron, the paper's P:133 "more GPUs" reading for a model that does not fit one GPU's share):
   column-parallel q, k, v (heads), gate, up (rows of f): LoRA A [r, d] replicated, B [N/W, r] sharded;
@@ -70,8 +70,10 @@ def gather_adapter(t: str, shards: list, which: str = "grad"):
     return np.concatenate(As, axis=1), Bs[0]
 
 
-# ------------------------------------------------------------------------------------------- all-reduce callback
-ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_size_t, C.c_int, C.c_void_p, C.c_void_p)
+# ------------------------------------------------------------------------------------------- collectives
+# include/menos.h menos_collective_fn: (op, send, recv, count, dtype, stream, user) -> int
+COLLECTIVE_FN = C.CFUNCTYPE(C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_int, C.c_void_p, C.c_void_p)
+OP_ALLREDUCE, OP_ALLGATHER, OP_REDUCE_SCATTER = 0, 1, 2
 
 
 class _CudaArray:
@@ -82,43 +84,77 @@ class _CudaArray:
                                          "strides": None}
 
 
-def make_torch_allreduce(group=None, device=None):
-    """A Python callable (buf, count, dtype, stream) -> int for menos_tp_cfg.allreduce: an in-place SUM
-    all-reduce of the device buffer with torch.distributed on `group`, ordered on the library's stream
-    (the collective waits for the work queued on `stream`; later work on `stream` waits for the collective)."""
+def make_torch_collective(group=None, device=None):
+    """A Python callable (op, send, recv, count, dtype, stream) -> int for menos_tp_cfg.collective, implemented with
+    torch.distributed on `group` and ordered on the library's stream.  Used for the single-GPU tests (gloo: ranks share
+    one GPU, which NCCL does not allow); multi-GPU runs give the library an NCCL id instead (menos_tp_unique_id) so no
+    Python runs on the per-layer path.  gloo has no reduce-scatter: it is an all-reduce of the full buffer followed by
+    a copy of this rank's chunk (same sum, more bytes)."""
     import torch
     import torch.distributed as dist
     dev = torch.device("cuda", torch.cuda.current_device() if device is None else device)
-    views: dict = {}
+    gloo = dist.get_backend(group) == "gloo"
 
-    def fn(buf: int, count: int, dtype: int, stream: int) -> int:
-        key = (buf, count, dtype)
-        t = views.get(key)
-        if t is None:
-            if len(views) > 256:
-                views.clear()
-            if dtype == 0:
-                t = torch.as_tensor(_CudaArray(buf, count, "<f4"), device=dev)
-            else:
-                t = torch.as_tensor(_CudaArray(buf, count, "<i2"), device=dev).view(torch.bfloat16)
-            views[key] = t
+    def view(ptr: int, n: int, dtype: int):
+        if dtype == 0:
+            return torch.as_tensor(_CudaArray(ptr, n, "<f4"), device=dev)
+        return torch.as_tensor(_CudaArray(ptr, n, "<i2"), device=dev).view(torch.bfloat16)
+
+    def fn(op: int, send: int, recv: int, count: int, dtype: int, stream: int) -> int:
+        world = dist.get_world_size(group)
+        rank = dist.get_rank(group)
         s = torch.cuda.ExternalStream(stream, device=dev) if stream else torch.cuda.default_stream(dev)
         with torch.cuda.stream(s):
-            dist.all_reduce(t, group=group)
+            if op == OP_ALLREDUCE:
+                t = view(recv, count, dtype)
+                if gloo and dtype == 1:   # sum in fp32, one rounding to bf16 at the end (as NCCL's bf16 kernels do)
+                    f = t.float()
+                    dist.all_reduce(f, group=group)
+                    t.copy_(f)
+                else:
+                    dist.all_reduce(t, group=group)
+            elif op == OP_ALLGATHER:
+                out = view(recv, count * world, dtype)
+                src = view(send, count, dtype)
+                if gloo:
+                    parts = [torch.empty_like(src) for _ in range(world)]
+                    dist.all_gather(parts, src.clone(), group=group)
+                    out.copy_(torch.cat(parts))
+                else:
+                    dist.all_gather_into_tensor(out, src, group=group)
+            elif op == OP_REDUCE_SCATTER:
+                src = view(send, count * world, dtype)
+                out = view(recv, count, dtype)
+                if gloo:
+                    f = src.float()
+                    dist.all_reduce(f, group=group)
+                    out.copy_(f[rank * count:(rank + 1) * count])
+                else:
+                    dist.reduce_scatter_tensor(out, src, group=group)
+            else:
+                return 1
         return 0
 
     return fn
 
 
-def wrap_allreduce(fn):
-    """ctypes callback around a Python all-reduce callable; exceptions become a nonzero status (MENOS_ENCCL)."""
+def nccl_unique_id(lib=None) -> bytes:
+    """128-byte NCCL unique id from libmenos (menos_tp_unique_id); rank 0 makes it, the caller broadcasts it."""
+    from .menos import check, lib as _lib
+    buf = C.create_string_buffer(128)
+    check((lib or _lib()).menos_tp_unique_id(buf))
+    return buf.raw
+
+
+def wrap_collective(fn):
+    """ctypes callback around a Python collective; exceptions become a nonzero status (MENOS_ENCCL)."""
     import traceback
 
-    def cb(buf, count, dtype, stream, user):
+    def cb(op, send, recv, count, dtype, stream, user):
         try:
-            return int(fn(buf or 0, int(count), int(dtype), stream or 0) or 0)
+            return int(fn(int(op), send or 0, recv or 0, int(count), int(dtype), stream or 0) or 0)
         except Exception:
             traceback.print_exc()
             return 1
 
-    return ALLREDUCE_FN(cb)
+    return COLLECTIVE_FN(cb)

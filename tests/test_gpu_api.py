@@ -35,10 +35,10 @@ def test_live_save_batch_blocks_table_growth_and_unregister():
     srv, ids, x, g, sc, sl = _setup()
     xs, gs = torch.empty_like(x), torch.empty_like(x)
     b = srv.forward(sc, sl, x, xs)
-    # growth needed: the q/v slot table holds 64 columns, filled by 2 clients x 2 targets x 16; a rank-64 client
-    # (2 x 64 columns) cannot fit
+    # growth needed: the q/k/v slot table holds 64 columns, filled by 2 clients x 2 targets x 16; a client with
+    # 3 targets x 16 columns cannot fit
     with pytest.raises(MenosError) as e:
-        srv.register_client(64, 128.0, ("q", "v"))
+        srv.register_client(16, 32.0, ("q", "k", "v"))
     assert e.value.code == -4
     with pytest.raises(MenosError) as e:
         srv.unregister_client(ids[0])
@@ -46,7 +46,7 @@ def test_live_save_batch_blocks_table_growth_and_unregister():
     srv.backward(b, g, gs)
     torch.cuda.synchronize()
     # after the backward both are allowed
-    cid = srv.register_client(64, 128.0, ("q", "v"))
+    cid = srv.register_client(16, 32.0, ("q", "k", "v"))
     srv.unregister_client(cid)
     srv.close()
 

@@ -244,7 +244,23 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 14), (128, 8, 1, [130, 7, 256], 14),
+DEFAULT_ATTN_MODE = 46   # testing.cu g_attn_tc default: persistent tcgen05 forward + one-pass fused backward
+
+
+@pytest.fixture(autouse=True)
+def _restore_attention_mode():
+    """Kernel-variant tests switch the library-global attention variant; restore the production default afterwards so
+    the end-to-end tests of later modules run the default kernels."""
+    yield
+    from paper_conf_middleware_hul24_b200.menos import check
+    check(lib().menos_test_set_attn_tc(DEFAULT_ATTN_MODE), testing=True)
+
+
+@pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 46), (128, 8, 1, [130, 7, 256], 46),
+                                             (128, 2, 2, [512, 1024, 255], 46), (128, 3, 1, [2048, 1, 700], 46),
+                                             (128, 8, 8, [512] * 16 + [77], 46), (128, 8, 1, [1024] * 3 + [33], 46),
+                                             (128, 4, 4, [1, 17, 64, 129, 300], -46),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 14), (128, 8, 1, [130, 7, 256], 14),
                                              (128, 2, 2, [512, 1024, 255], 14), (128, 3, 1, [2048, 1, 700], 14),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 6), (128, 8, 1, [130, 7, 256], 6),
                                              (128, 2, 2, [512, 1024, 255], 6), (128, 3, 1, [2048, 1, 700], 6),
@@ -385,3 +401,22 @@ def test_lora_tokred_gate_up_block_remap():
     check(lib().menos_test_lora_tokred(dgud.data_ptr() + 128 * 2, Ud.data_ptr(), out.data_ptr(), f, r, T, 2 * f, 16,
                                        r, 128, 256, 1.0, 128), testing=True)   # "up" target: base column 128
     assert maxrel(out.cpu().numpy(), du.T @ U[:, :r]) < 1e-2
+
+
+def test_fused_attention_backward_deterministic():
+    """The one-pass backward adds each dQ block's contributions in a fixed order (ordered counters): two runs give
+    bitwise identical dq, dk, dv, also with more work items than SMs (persistent loop, waits across CTAs)."""
+    from paper_conf_middleware_hul24_b200.menos import check
+    check(lib().menos_test_set_attn_tc(46), testing=True)
+    lens, H, Hkv, hd = [700, 1024, 3, 512, 129] * 6, 8, 2, 128
+    T, N = sum(lens), (H + 2 * Hkv) * hd
+    qkv_d, dO_d = dev(rnd((T, N), 71)), dev(rnd((T, H * hd), 72))
+    outs = []
+    for _ in range(2):
+        O_d = torch.empty(T, H * hd, dtype=torch.bfloat16, device="cuda")
+        lse = torch.empty(H, T, dtype=torch.float32, device="cuda")
+        dqkv = torch.zeros(T, N, dtype=torch.bfloat16, device="cuda")
+        check(lib().menos_test_attention(len(lens), i32(lens), H, Hkv, hd, qkv_d.data_ptr(), O_d.data_ptr(),
+                                         lse.data_ptr(), dO_d.data_ptr(), dqkv.data_ptr(), 1e4), testing=True)
+        outs.append(dqkv.clone())
+    assert torch.equal(outs[0], outs[1])

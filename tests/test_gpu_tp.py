@@ -1,11 +1,13 @@
 """Tensor-parallel server segment on the GPU (include/menos.h menos_tp_cfg), checked
 against the UNSHARDED CPU oracle.
 
-Two ranks share cuda:0 (the only GPU a test box has): each process creates its own libmenos server shard with
-tp = (rank, 2, torch.distributed all-reduce over gloo), loads its weight / adapter shards
-(paper_conf_middleware_hul24_b200.tp), and runs forward(SAVE or NOGRAD) + backward + adapter_step on the full
-replicated batch.  The library calls the all-reduce at the four per-layer exchange points and once per backward
-for the replicated adapters' gradients; everything else runs in its kernels.  Bars as in test_gpu_parity.py:
+Several ranks share cuda:0 (the only GPU a test box has; NCCL refuses two ranks on one GPU): each process creates its
+own libmenos server shard with tp = (rank, world, torch.distributed collective over gloo), loads its weight / adapter
+shards (paper_conf_middleware_hul24_b200.tp), and runs forward(SAVE or NOGRAD) + backward + adapter_step.  The
+library runs the sequence-parallel schedule: bf16 all-gathers of the norm outputs / incoming gradients and bf16
+reduce-scatters of the row-parallel partial sums (8 per layer), plus one fp32 all-reduce of the replicated adapters'
+gradients per client per backward; everything else runs in its kernels.  The NCCL transport (the library drives
+NCCL itself from a broadcast unique id) is exercised at world 1 on one GPU.  Bars as in test_gpu_parity.py:
 activations max|d|/max|ref| <= 2e-2, cosine >= 0.999 on every gradient tensor (gathered over the shards).
 """
 import os
@@ -29,7 +31,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, wl, flags, q):
+def _worker(rank, world, port, wl, flags, q, transport="gloo"):
     import torch.distributed as dist
     from paper_conf_middleware_hul24_b200 import Server
     from paper_conf_middleware_hul24_b200 import tp as TP
@@ -44,9 +46,15 @@ def _worker(rank, world, port, wl, flags, q):
         for W in weights:
             Ws = TP.shard_layer_weights(W, rank, world, m.n_heads, m.n_kv_heads, hd, m.d_ff)
             shards.append({k: torch.from_numpy(np.ascontiguousarray(v)).to(torch.bfloat16).cuda() for k, v in Ws.items()})
+        del weights
+        if transport == "nccl":   # the library drives NCCL itself from rank 0's unique id (broadcast here)
+            uid = [TP.nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            tpc = (rank, world, uid[0])
+        else:
+            tpc = (rank, world, TP.make_torch_collective())
         srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
-                     weights=shards, max_rank=16, max_seq_len=1024, arena_bytes=2 << 30,
-                     tp=(rank, world, TP.make_torch_allreduce()))
+                     weights=shards, max_rank=16, max_seq_len=1024, arena_bytes=2 << 30, tp=tpc)
         ids = []
         for i, c in enumerate(wl.clients):
             cid = srv.register_client(c.rank, c.alpha, c.targets, seed=i)
@@ -72,7 +80,7 @@ def _worker(rank, world, port, wl, flags, q):
         torch.cuda.synchronize()
         params = [[{t: (srv.get_adapter(ids[i], l, t, "A"), srv.get_adapter(ids[i], l, t, "B")) for t in c.targets}
                    for l in range(m.n_layers)] for i, c in enumerate(wl.clients)]
-        q.put((rank, xs.float().cpu().numpy(), gs.float().cpu().numpy(), grads, params))
+        q.put((rank, xs.float().cpu().numpy(), gs.float().cpu().numpy(), grads, params, srv.tp_stats()))
         srv.close()
     except Exception as e:  # surface the failure to the parent instead of hanging it
         import traceback
@@ -81,15 +89,15 @@ def _worker(rank, world, port, wl, flags, q):
         dist.destroy_process_group()
 
 
-def _run(wl, flags=0, world=2):
+def _run(wl, flags=0, world=2, transport="gloo"):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, wl, flags, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, wl, flags, q, transport)) for r in range(world)]
     for p in procs:
         p.start()
-    res = sorted([q.get(timeout=600) for _ in procs], key=lambda r: r[0])
+    res = sorted([q.get(timeout=1200) for _ in procs], key=lambda r: r[0])
     for p in procs:
         p.join(timeout=120)
     for r in res:
@@ -97,11 +105,17 @@ def _run(wl, flags=0, world=2):
     return res
 
 
-def _check(wl, res, world=2):
+def _check(wl, res, world=2, flags=0):
     from oracle import menos_oracle as O
     from paper_conf_middleware_hul24_b200 import tp as TP
     m = wl.model
     weights, adapters, io = make_inputs(wl, seed=11)
+    # sequence-parallel exchanges: per layer 4 all-gathers + 4 reduce-scatters of bf16 [T, d] (fwd + bwd), 2 more
+    # all-gathers for x_s / g_s, one fp32 all-reduce per client of the replicated adapter gradients
+    if world > 1:
+        st = res[0][5]
+        per_layer = 8 if flags == 0 else 12   # NOGRAD: the forward's exchanges again in the backward's re-forward
+        assert st["calls"] == per_layer * m.n_layers + 2 + len(wl.clients), st
     for r in range(1, world):          # replicated outputs are bitwise identical on every rank
         assert np.array_equal(res[r][1], res[0][1])
         assert np.array_equal(res[r][2], res[0][2])
@@ -144,4 +158,22 @@ def test_tp2_70b_like_hd128_qv_and_nograd():
     wl = Workload("tp_hd128", MODEL_70B_LIKE,
                   [ClientCfg(8, 16.0, ("q", "v"), [300, 129]), ClientCfg(16, 32.0, ("q", "v", "o", "down"), [256])])
     _check(wl, _run(wl))
-    _check(wl, _run(wl, flags=1))   # MENOS_FWD_NOGRAD: the re-forward inside backward exchanges the same way
+    _check(wl, _run(wl, flags=1), flags=1)   # MENOS_FWD_NOGRAD: the re-forward inside backward exchanges the same way
+
+
+def test_tp8_at_llama2_70b_width():
+    """BASELINE configs[4] shard shapes: Llama-2-70B widths (d 8192, 64 heads of 128, 8 KV heads, f 28672) split 8
+    ways, so every rank holds 8 query heads, 1 KV head and f/8 = 3584 (the cfg4 per-GPU shapes); 2 layers, two clients
+    (q,v r=8 and q,v,o,down r=16), T = 407 tokens (not a multiple of 8: the last rank's padding rows are exercised)."""
+    m = ModelCfg("llama2-70b-2l", 8192, 64, 8, 28672, 2, model_layers=80)
+    wl = Workload("tp8_70b", m, [ClientCfg(8, 16.0, ("q", "v"), [200, 57]),
+                                 ClientCfg(16, 32.0, ("q", "v", "o", "down"), [150])])
+    _check(wl, _run(wl, world=8), world=8)
+
+
+def test_nccl_transport_world1():
+    """The library-driven NCCL path (menos_tp_unique_id -> menos_tp_cfg.nccl_id -> ncclCommInitRank) running the
+    sequence-parallel schedule at world 1 on the one GPU: results match the oracle like every other configuration."""
+    wl = Workload("tp_nccl1", MODEL_70B_LIKE,
+                  [ClientCfg(8, 16.0, ("q", "v"), [100, 29]), ClientCfg(16, 32.0, ("q", "v", "o", "down"), [64])])
+    _check(wl, _run(wl, world=1, transport="nccl"), world=1)

@@ -3,11 +3,13 @@ world_size 2.
 
 Each rank holds the shards `paper_conf_middleware_hul24_b200.tp` assigns (column-parallel q,k,v,gate,up;
 row-parallel o,down; LoRA A replicated / B sharded for column targets, A sharded / B replicated for row targets)
-and runs the exchange plan libmenos.so implements: all-reduce of the o-proj and down-proj partial sums (rank 0's
-partial carries the residual), of the gate|up-dX and qkv-dX partial sums, and once per backward of the
-replicated adapters' gradient partial sums.  The shard arithmetic is composed from oracle primitives; the result
-must equal the UNSHARDED oracle (fp64, up to re-association).  This pins the host-side shard layout and the
-placement of every collective that the GPU path's TP mode relies on.
+and runs the SEQUENCE-PARALLEL exchange plan libmenos.so implements: the residual streams and the norms live on the
+rank's token rows [r*Tl, (r+1)*Tl) (Tl = ceil(T / world), the last rank padded); per layer the norm outputs and the
+incoming gradients dy, dh are all-gathered, the o / down partial sums (forward) and gate|up-dX / qkv-dX partial sums
+(backward) are reduce-scattered, and once per backward the replicated adapters' gradient partial sums are
+all-reduced; x_s and g_s are all-gathered at the end.  The shard arithmetic is composed from oracle primitives; the
+result must equal the UNSHARDED oracle (fp64, up to re-association).  This pins the host-side shard layout, the row
+split and the placement of every collective that the GPU path's tensor-parallel mode relies on.
 """
 import os
 import socket
@@ -22,7 +24,7 @@ from paper_conf_middleware_hul24_b200 import tp as TP
 from workloads import ClientCfg, ModelCfg, TARGETS, base_layer_weights, client_adapters, client_inputs
 
 CFG = ModelCfg("tiny-gqa-tp", 64, 4, 2, 172, 2, model_layers=3)   # H=4, H_kv=2 (GQA), f=172 -> 2 ranks
-CLIENT = ClientCfg(4, 8.0, TARGETS, [16, 9])                       # all 7 targets, ragged sequences
+CLIENT = ClientCfg(4, 8.0, TARGETS, [16, 9])                       # all 7 targets, ragged sequences: T = 25 (odd)
 F64 = np.float64
 
 
@@ -30,6 +32,49 @@ def _allreduce(x):
     t = torch.from_numpy(np.ascontiguousarray(x))
     dist.all_reduce(t)
     return t.numpy()
+
+
+def _rows(T):
+    world, rank = dist.get_world_size(), dist.get_rank()
+    loc = -(-T // world)
+    return loc, loc * world, loc * rank
+
+
+def _gather(x_loc, T):
+    """all-gather of the ranks' [Tl, d] rows -> [T, d] (padding rows dropped)."""
+    parts = [torch.empty_like(torch.from_numpy(x_loc)) for _ in range(dist.get_world_size())]
+    dist.all_gather(parts, torch.from_numpy(np.ascontiguousarray(x_loc)))
+    return torch.cat(parts).numpy()[:T]
+
+
+def _scatter(part, T):
+    """reduce-scatter of a [T, d] partial sum (padded to world * Tl rows) -> this rank's [Tl, d] rows."""
+    loc, pad, r0 = _rows(T)
+    full = np.zeros((pad, part.shape[1]), part.dtype)
+    full[:T] = part
+    return _allreduce(full)[r0:r0 + loc]
+
+
+def _attn_fwd(q, k, v, lens):
+    outs, off = [], 0
+    for S in lens:
+        o, _ = O.attention_fwd(q[off:off + S], k[off:off + S], v[off:off + S])
+        outs.append(o)
+        off += S
+    return np.concatenate(outs)
+
+
+def _attn_bwd(dO, q, k, v, lens):
+    res, off = [], 0
+    for S in lens:
+        res.append(O.attention_bwd(dO[off:off + S], q[off:off + S], k[off:off + S], v[off:off + S]))
+        off += S
+    return [np.concatenate([r[i] for r in res]) for i in range(3)]
+
+
+def _rope(lens, hd):
+    cs, ss = zip(*[O.rope_cos_sin(S, hd, CFG.rope_theta, F64) for S in lens])
+    return np.concatenate(cs), np.concatenate(ss)
 
 
 def _shard_layer(rank, world, W, lora):
@@ -41,28 +86,28 @@ def _shard_layer(rank, world, W, lora):
             {t: (np.asarray(a, F64), np.asarray(b, F64)) for t, (a, b) in Ls.items()})
 
 
-def _tp_layer_fwd(rank, x, W, L, s, H, Hkv):
-    S = x.shape[0]
+def _tp_layer_fwd(x_loc, T, lens, W, L, s, H, Hkv):
     hd = CFG.head_dim
-    c = {"x": x}
-    xn, c["rstd1"] = O.rmsnorm_fwd(x, W["g1"], CFG.rms_eps)
+    c = {"x": x_loc}
+    xn_loc, c["rstd1"] = O.rmsnorm_fwd(x_loc, W["g1"], CFG.rms_eps)
+    xn = _gather(xn_loc, T)                                           # exchange: all-gather xn
     c["xn"] = xn
     U = {}
     qp, U["q"] = O.proj_fwd(xn, W["wq"], L.get("q"), s)
     kp, U["k"] = O.proj_fwd(xn, W["wk"], L.get("k"), s)
     vp, U["v"] = O.proj_fwd(xn, W["wv"], L.get("v"), s)
-    cos, sin = O.rope_cos_sin(S, hd, CFG.rope_theta, F64)
+    cos, sin = _rope(lens, hd)
     c["cos"], c["sin"] = cos, sin
-    q = O.rope_fwd(qp.reshape(S, H, hd), cos, sin)
-    k = O.rope_fwd(kp.reshape(S, Hkv, hd), cos, sin)
-    v = vp.reshape(S, Hkv, hd)
-    Oa, _ = O.attention_fwd(q, k, v)
+    q = O.rope_fwd(qp.reshape(T, H, hd), cos, sin)
+    k = O.rope_fwd(kp.reshape(T, Hkv, hd), cos, sin)
+    v = vp.reshape(T, Hkv, hd)
     c["q"], c["k"], c["v"] = q, k, v
-    c["O"] = Oa.reshape(S, H * hd)
+    c["O"] = _attn_fwd(q, k, v, lens).reshape(T, H * hd)
     ao, U["o"] = O.proj_fwd(c["O"], W["wo"], L.get("o"), s)          # row-parallel partial (+ s U_r B^T)
-    h = _allreduce((x if rank == 0 else 0.0) + ao)                    # exchange 1
-    c["h"] = h
-    hn, c["rstd2"] = O.rmsnorm_fwd(h, W["g2"], CFG.rms_eps)
+    h_loc = x_loc + _scatter(ao, T)                                   # exchange: reduce-scatter, residual add
+    c["h"] = h_loc
+    hn_loc, c["rstd2"] = O.rmsnorm_fwd(h_loc, W["g2"], CFG.rms_eps)
+    hn = _gather(hn_loc, T)                                           # exchange: all-gather hn
     c["hn"] = hn
     gt, U["gate"] = O.proj_fwd(hn, W["wgate"], L.get("gate"), s)
     up, U["up"] = O.proj_fwd(hn, W["wup"], L.get("up"), s)
@@ -70,33 +115,41 @@ def _tp_layer_fwd(rank, x, W, L, s, H, Hkv):
     a = O.silu(gt) * up
     c["a"] = a
     md, U["down"] = O.proj_fwd(a, W["wdown"], L.get("down"), s)
-    y = _allreduce((h if rank == 0 else 0.0) + md)                    # exchange 2
+    y_loc = h_loc + _scatter(md, T)                                   # exchange: reduce-scatter, residual add
     c["U"] = U
-    return y, c
+    return y_loc, c
 
 
-def _tp_layer_bwd(dy, c, W, L, s, H, Hkv):
-    S = dy.shape[0]
+def _tp_layer_bwd(dy_loc, T, lens, c, W, L, s, H, Hkv):
     hd = CFG.head_dim
     U = c["U"]
     g = {}
+    dy = _gather(dy_loc, T)                                           # exchange: all-gather dy
     da, g["down"] = O.proj_bwd(dy, c["a"], W["wdown"], L.get("down"), s, U["down"])
     dgt, dup = O.swiglu_bwd(da, c["gt"], c["up"])
     dg, g["gate"] = O.proj_bwd(dgt, c["hn"], W["wgate"], L.get("gate"), s, U["gate"])
     du, g["up"] = O.proj_bwd(dup, c["hn"], W["wup"], L.get("up"), s, U["up"])
-    dhn = _allreduce(dg + du)                                         # exchange 3
-    dh = dy + O.rmsnorm_bwd(dhn, c["h"], W["g2"], c["rstd2"])
+    dhn_loc = _scatter(dg + du, T)                                    # exchange: reduce-scatter
+    dh_loc = dy_loc + O.rmsnorm_bwd(dhn_loc, c["h"], W["g2"], c["rstd2"])
+    dh = _gather(dh_loc, T)                                           # exchange: all-gather dh
     dO, g["o"] = O.proj_bwd(dh, c["O"], W["wo"], L.get("o"), s, U["o"])
-    dq, dk, dv = O.attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
-    dqp = O.rope_bwd(dq, c["cos"], c["sin"]).reshape(S, H * hd)
-    dkp = O.rope_bwd(dk, c["cos"], c["sin"]).reshape(S, Hkv * hd)
+    dq, dk, dv = _attn_bwd(dO.reshape(T, H, hd), c["q"], c["k"], c["v"], lens)
+    dqp = O.rope_bwd(dq, c["cos"], c["sin"]).reshape(T, H * hd)
+    dkp = O.rope_bwd(dk, c["cos"], c["sin"]).reshape(T, Hkv * hd)
     dxn = 0.0
-    for t, d_t in (("q", dqp), ("k", dkp), ("v", dv.reshape(S, Hkv * hd))):
+    for t, d_t in (("q", dqp), ("k", dkp), ("v", dv.reshape(T, Hkv * hd))):
         dxt, g[t] = O.proj_bwd(d_t, c["xn"], W["w" + t], L.get(t), s, U[t])
         dxn = dxn + dxt
-    dxn = _allreduce(dxn)                                             # exchange 4
-    dx = dh + O.rmsnorm_bwd(dxn, c["x"], W["g1"], c["rstd1"])
-    return dx, g
+    dxn_loc = _scatter(dxn, T)                                        # exchange: reduce-scatter
+    dx_loc = dh_loc + O.rmsnorm_bwd(dxn_loc, c["x"], W["g1"], c["rstd1"])
+    return dx_loc, g
+
+
+def _local(x, T):
+    loc, pad, r0 = _rows(T)
+    full = np.zeros((pad, x.shape[1]), x.dtype)
+    full[:T] = x
+    return full[r0:r0 + loc]
 
 
 def _worker(rank, world, port, q):
@@ -108,29 +161,24 @@ def _worker(rank, world, port, q):
         ad = client_adapters(CFG, CLIENT, seed=5)
         x_c, g_c = client_inputs(CFG, CLIENT, seed=6)
         s = CLIENT.alpha / CLIENT.rank
+        T, lens = CLIENT.n_tokens, CLIENT.seq_lens
         shards = [_shard_layer(rank, world, Wf[l], ad[l]) for l in range(CFG.n_layers)]
-        xs_all, gs_all, grads = [], [], [{} for _ in range(CFG.n_layers)]
-        off = 0
-        for S in CLIENT.seq_lens:
-            x = x_c[off:off + S].astype(F64)
-            caches = []
-            for l in range(CFG.n_layers):
-                x, c = _tp_layer_fwd(rank, x, *shards[l], s, H, Hkv)
-                caches.append(c)
-            xs_all.append(x)
-            dy = g_c[off:off + S].astype(F64)
-            for l in reversed(range(CFG.n_layers)):
-                dy, gl = _tp_layer_bwd(dy, caches[l], *shards[l], s, H, Hkv)
-                for t, (dA, dB) in gl.items():
-                    pa, pb = grads[l].get(t, (0.0, 0.0))
-                    grads[l][t] = (pa + dA, pb + dB)
-            gs_all.append(dy)
-            off += S
+        x = _local(x_c.astype(F64), T)
+        caches = []
+        for l in range(CFG.n_layers):
+            x, c = _tp_layer_fwd(x, T, lens, *shards[l], s, H, Hkv)
+            caches.append(c)
+        xs = _gather(x, T)                                            # x_s on every rank
+        dy = _local(g_c.astype(F64), T)
+        grads = [None] * CFG.n_layers
+        for l in reversed(range(CFG.n_layers)):
+            dy, grads[l] = _tp_layer_bwd(dy, T, lens, caches[l], *shards[l], s, H, Hkv)
+        gs = _gather(dy, T)
         # once per backward: the replicated adapters' gradient partial sums
         for l in range(CFG.n_layers):
             for t, (dA, dB) in grads[l].items():
                 grads[l][t] = (_allreduce(dA), dB) if t in TP.COLUMN_PARALLEL else (dA, _allreduce(dB))
-        q.put((rank, np.concatenate(xs_all), np.concatenate(gs_all), grads))
+        q.put((rank, xs, gs, grads))
     finally:
         dist.destroy_process_group()
 
