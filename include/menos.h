@@ -101,12 +101,19 @@ typedef struct {
   const void* b2;    /* [d]  final_layer_norm bias     */
 } menos_layer_weights;
 
-/* LoRA target projections (bit mask).  PAPER.md:294 uses q,v. */
+/* LoRA target projections (bit mask).  PAPER.md:294 uses q,v.
+ * MENOS_T_PREFIX: prefix tuning instead of LoRA (SURVEY.md §8(f) NEXT-3; PAPER.md:59 §2.1, :121 §3.1; Li & Liang [16]):
+ * the client holds, per server layer, P = `rank` learned key and value vectors per KV head which every query of its
+ * sequences attends to in addition to its causal keys (one softmax over both; the prefix keys are used as given, no
+ * RoPE; sequence positions stay 0-based -- DESIGN.md R28).  It must be the client's only target (alpha is ignored);
+ * not available with tensor parallelism, and a batch holding a prefix client cannot mix cut points.  Init
+ * N(0, 1).  get/set_adapter target index 7: which A = prefix keys [P, H_kv*hd], B = prefix values [P, H_kv*hd]
+ * (dA / dB their gradients, summed over the client's tokens). */
 enum {
   MENOS_T_Q = 1, MENOS_T_K = 2, MENOS_T_V = 4, MENOS_T_O = 8,
-  MENOS_T_GATE = 16, MENOS_T_UP = 32, MENOS_T_DOWN = 64
+  MENOS_T_GATE = 16, MENOS_T_UP = 32, MENOS_T_DOWN = 64, MENOS_T_PREFIX = 128
 };
-/* target index (0..6) used by get/set_adapter: q, k, v, o, gate, up, down */
+/* target index (0..7) used by get/set_adapter: q, k, v, o, gate, up, down, prefix */
 
 typedef struct {
   double lr, beta1, beta2, eps, weight_decay; /* torch.optim.AdamW semantics (scalars in double, as torch forms them) */

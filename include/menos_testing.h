@@ -65,7 +65,8 @@ MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A,
 /* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
    bit 1 = tcgen05 backward (else mma.sync), bit 2 = persistent warp-specialized tcgen05 forward (overrides
    bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1), bit 4 = (sequence, head)-grouped
-   work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1; default mode 46).
+   work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1).  Default mode 14
+   (persistent forward + two-kernel persistent backward: measured faster than the one-pass kernel).
    Returns MENOS_EINVAL outside [0, 63]. */
 MENOS_API int menos_test_set_attn_tc(int mode);
 

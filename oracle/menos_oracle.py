@@ -126,6 +126,62 @@ def attention_bwd(dO, q, k, v):
     return dq, dk, dv
 
 
+# ============================================================ prefix-tuning attention (NEXT-3; reading R28)
+def attention_prefix_fwd(q, k, v, pk, pv):
+    """Prefix tuning (§2.1, Li & Liang [16]; a client may pick it instead of LoRA): the layer
+    holds P learned key/value vectors per KV head, pk/pv [P, Hkv, hd], which every query of the sequence attends to
+    in addition to its causal keys -- one softmax over [prefix | causal keys], scale hd^-1/2 (reading R28: prefix
+    keys are used as given, no RoPE; the sequence keeps positions 0..S-1).  Returns O [S,H,hd], lse [H,S]."""
+    S, H, hd = q.shape
+    P = pk.shape[0]
+    rep = H // k.shape[1]
+    scale = 1.0 / np.sqrt(hd)
+    O = np.zeros_like(q)
+    lse = np.zeros((H, S), dtype=q.dtype)
+    mask = np.concatenate([np.zeros((S, P), dtype=bool), np.triu(np.ones((S, S), dtype=bool), 1)], axis=1)
+    for h in range(H):
+        kh = np.concatenate([pk[:, h // rep, :], k[:, h // rep, :]])
+        vh = np.concatenate([pv[:, h // rep, :], v[:, h // rep, :]])
+        s = (q[:, h, :] @ kh.T) * scale
+        s = np.where(mask, -np.inf, s)
+        m = np.max(s, axis=-1, keepdims=True)
+        e = np.exp(s - m)
+        z = np.sum(e, axis=-1, keepdims=True)
+        O[:, h, :] = (e / z) @ vh
+        lse[h] = (m + np.log(z))[:, 0]
+    return O, lse
+
+
+def attention_prefix_bwd(dO, q, k, v, pk, pv):
+    """Backward of attention_prefix_fwd (same textbook softmax backward over the concatenated keys):
+    returns dq, dk, dv, dpk, dpv (GQA: kv-head and prefix gradients sum over the heads of their group)."""
+    S, H, hd = q.shape
+    P = pk.shape[0]
+    rep = H // k.shape[1]
+    scale = 1.0 / np.sqrt(hd)
+    dq, dk, dv = np.zeros_like(q), np.zeros_like(k), np.zeros_like(v)
+    dpk, dpv = np.zeros_like(pk), np.zeros_like(pv)
+    mask = np.concatenate([np.zeros((S, P), dtype=bool), np.triu(np.ones((S, S), dtype=bool), 1)], axis=1)
+    for h in range(H):
+        kv = h // rep
+        kh = np.concatenate([pk[:, kv, :], k[:, kv, :]])
+        vh = np.concatenate([pv[:, kv, :], v[:, kv, :]])
+        s = (q[:, h, :] @ kh.T) * scale
+        s = np.where(mask, -np.inf, s)
+        e = np.exp(s - np.max(s, axis=-1, keepdims=True))
+        Pm = e / np.sum(e, axis=-1, keepdims=True)
+        dvh = Pm.T @ dO[:, h, :]
+        dP = dO[:, h, :] @ vh.T
+        dS = Pm * (dP - np.sum(Pm * dP, axis=-1, keepdims=True))
+        dq[:, h, :] = (dS @ kh) * scale
+        dkh = (dS.T @ q[:, h, :]) * scale
+        dpk[:, kv, :] += dkh[:P]
+        dk[:, kv, :] += dkh[P:]
+        dpv[:, kv, :] += dvh[:P]
+        dv[:, kv, :] += dvh[P:]
+    return dq, dk, dv, dpk, dpv
+
+
 # ============================================================ SwiGLU (reading R4)
 def sigmoid(x):
     return 1.0 / (1.0 + np.exp(-x))
@@ -194,7 +250,11 @@ def layer_fwd(x, W, lora, s, cfg, dtype=np.float32):
     q = rope_fwd(qp.reshape(S, H, hd), cos, sin)
     k = rope_fwd(kp.reshape(S, Hkv, hd), cos, sin)
     v = vp.reshape(S, Hkv, hd)
-    O, c["lse"] = attention_fwd(q, k, v)
+    if "prefix" in L:   # prefix-tuning client (NEXT-3): the layer's learned prefix keys / values join the attention
+        pk, pv = (a.reshape(-1, Hkv, hd) for a in L["prefix"])
+        O, c["lse"] = attention_prefix_fwd(q, k, v, pk, pv)
+    else:
+        O, c["lse"] = attention_fwd(q, k, v)
     c["q"], c["k"], c["v"] = q, k, v
     Of = O.reshape(S, H * hd)
     c["O"] = Of
@@ -241,7 +301,12 @@ def layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
     if go is not None:
         grads["o"] = go
     # A11: attention backward, then RoPE backward
-    dq, dk, dv = attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
+    if "prefix" in L:
+        pk, pv = (a.reshape(-1, Hkv, hd) for a in L["prefix"])
+        dq, dk, dv, dpk, dpv = attention_prefix_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"], pk, pv)
+        grads["prefix"] = (dpk.reshape(pk.shape[0], -1), dpv.reshape(pv.shape[0], -1))
+    else:
+        dq, dk, dv = attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
     dqp = rope_bwd(dq, c["cos"], c["sin"]).reshape(S, H * hd)
     dkp = rope_bwd(dk, c["cos"], c["sin"]).reshape(S, Hkv * hd)
     dvp = dv.reshape(S, Hkv * hd)
@@ -314,7 +379,11 @@ def opt_layer_fwd(x, W, lora, s, cfg, dtype=np.float32, relu_mask_bf16=False):
     q = (qp + Wd["bq"]).reshape(S, H, hd)
     k = (kp + Wd["bk"]).reshape(S, H, hd)
     v = (vp + Wd["bv"]).reshape(S, H, hd)
-    O, c["lse"] = attention_fwd(q, k, v)
+    if "prefix" in L:   # prefix tuning (NEXT-3, R28): no RoPE in OPT, so exactly as for Llama minus the rotation
+        pk, pv = (a.reshape(-1, H, hd) for a in L["prefix"])
+        O, c["lse"] = attention_prefix_fwd(q, k, v, pk, pv)
+    else:
+        O, c["lse"] = attention_fwd(q, k, v)
     c["q"], c["k"], c["v"] = q, k, v
     Of = O.reshape(S, H * hd)
     c["O"] = Of
@@ -356,7 +425,12 @@ def opt_layer_bwd(dy, c, W, lora, s, cfg, dtype=np.float32):
     dO, go = proj_bwd(dh, c["O"], Wd["wo"], L.get("o"), s, U["o"])
     if go is not None:
         grads["o"] = go
-    dq, dk, dv = attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
+    if "prefix" in L:
+        pk, pv = (a.reshape(-1, H, hd) for a in L["prefix"])
+        dq, dk, dv, dpk, dpv = attention_prefix_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"], pk, pv)
+        grads["prefix"] = (dpk.reshape(pk.shape[0], -1), dpv.reshape(pv.shape[0], -1))
+    else:
+        dq, dk, dv = attention_bwd(dO.reshape(S, H, hd), c["q"], c["k"], c["v"])
     dxn = np.zeros_like(c["xn"])
     for t, dt in (("q", dq), ("k", dk), ("v", dv)):
         dxt, gt_ = proj_bwd(dt.reshape(S, H * hd), c["xn"], Wd["w" + t], L.get(t), s, U[t])

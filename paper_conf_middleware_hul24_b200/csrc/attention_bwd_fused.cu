@@ -5,8 +5,8 @@
 // head of the GQA group, 64-query block at or after the key block).  S^T = K Q^T, dP^T = V dO^T and
 // P^T = exp2(S^T c - lse), dS^T = P^T (dP^T - D) scale are computed ONCE per (key block, query block) and feed all
 // three gradient products:
-//     dV_j += P^T dO        dK_j += dS^T Q        dQ_i^T = K_j^T dS^T       (10 hd MMA FLOP per causal pair,
-// against 14 hd and twice the exponentials for the previous separate dK/dV and dQ kernels).
+//     dV_j += P^T dO        dK_j += dS^T Q        dQ_i = dS K_j (two 64-query blocks per MMA, M = 128)
+// (10 hd MMA FLOP per causal pair, against 14 hd and twice the exponentials for the separate dK/dV and dQ kernels).
 //
 // dV_j, dK_j accumulate in TMEM over the key block's query blocks and are written once per key block.  dQ_i collects
 // one contribution per key block j <= i; since one CTA owns all key blocks of the (sequence, kv head), every dQ element
@@ -21,8 +21,11 @@
 //                the block's lse and D staged beside them by the warp's lanes
 //   warp 1       MMA issuer (tcgen05.mma, one elected lane)
 //   warps 2-9    softmax-gradient warps: one TMEM lane (= key row) per thread, 32 query columns each
-//   warps 10-13  dQ drain: one TMEM lane (= head-dim index) per thread; TMEM -> ordered fp32 accumulate -> bf16
-// TMEM (512 columns): S^T 0..63 | dP^T 64..127 | dQ^T x2 128..255 | dV 256..383 | dK 384..511.
+//   warps 2-9    (also, once per key block, the dK (RoPE backward) / dV epilogue, straight from TMEM to global)
+//   warps 10-13  dQ drain: one TMEM lane (= query row of a block pair) per thread, all 128 head dims (the RoPE pairs
+//                are in-thread): TMEM -> program-ordered fp32 accumulate -> RoPE backward -> bf16
+// TMEM (512 columns): S^T 0..63 | dP^T 64..127 | dQ (a block pair: 128 query rows x 128 hd) 128..255 | dV 256..383 |
+// dK 384..511.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -44,7 +47,7 @@ constexpr int KV_TILE = KV_ROWS * HD * 2;      // 32 KB (2 SW128 atoms [128][64]
 constexpr int QB_TILE = QB * HD * 2;           // 16 KB (2 atoms [64][64])
 constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
 constexpr int SMEM_FUSED = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;
-constexpr uint32_t T_S = 0, T_DP = 64, T_DQ = 128, T_DV = 256, T_DK = 384;
+constexpr uint32_t T_S = 0, T_DP = 64, T_DQ = 128, T_DV = 256, T_DK = 384;   // TMEM columns
 
 struct FParams {
   const int* cu_seqlens;
@@ -61,6 +64,7 @@ struct FParams {
                            // exchange (results wrong for 1, 3)
 };
 
+__device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
 __device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
   uint32_t ok = 0;
   while (!ok) {
@@ -68,9 +72,14 @@ __device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
                  : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   }
 }
-__device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
-__device__ __forceinline__ void dr_sync() { asm volatile("bar.sync 2, %0;" ::"n"(32 * DR_WARPS) : "memory"); }
 
+
+// bf16x2 pack with round-to-nearest-even on the integer pipe (finite inputs): offloads the conversion unit
+__device__ __forceinline__ uint32_t pack_bf16x2_alu(float lo, float hi) {
+  const uint32_t a = __float_as_uint(lo), b = __float_as_uint(hi);
+  const uint32_t ra = a + 0x7FFFu + ((a >> 16) & 1u), rb = b + 0x7FFFu + ((b >> 16) & 1u);
+  return __byte_perm(ra, rb, 0x7632);
+}
 
 // Instruction descriptor kind::f16 with both operand majors selectable (bit 15: A MN-major, bit 16: B MN-major).
 __host__ __device__ constexpr uint32_t idesc_ab(int M, int N, int a_mn, int b_mn) {
@@ -85,51 +94,6 @@ __device__ __forceinline__ void st_half_row_packed(uint8_t* tile, int row, int g
     const int c8 = (CPT / 8) * g + c;
     *reinterpret_cast<uint4*>(prow + ((c8 ^ (row & 7)) << 4)) =
         make_uint4(u[4 * c], u[4 * c + 1], u[4 * c + 2], u[4 * c + 3]);
-  }
-}
-
-// TMEM accumulator row (columns [32g, 32g+32) and [64+32g, ..): the RoPE pairs) -> bf16, RoPE backward applied in
-// registers, into a staging tile [128 rows][256 B] (16-byte chunk k of row rr at rr*256 + ((k ^ (rr & 15)) << 4))
-__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const float2* cs,
-                                                int pos, bool rope) {
-  uint32_t a[CPT], b[CPT];
-  tmem_ld32_nw(tacc + CPT * g, a);
-  tmem_ld32_nw(tacc + 64 + CPT * g, b);
-  tmem_wait_ld();
-  float x[CPT], y[CPT];
-#pragma unroll
-  for (int i = 0; i < CPT; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
-  if (rope) {   // dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
-    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + CPT * g);
-#pragma unroll
-    for (int i = 0; i < CPT / 2; ++i) {
-      const float4 e = __ldg(c4 + i);
-      const float x0 = x[2 * i] * e.x + y[2 * i] * e.y, y0 = y[2 * i] * e.x - x[2 * i] * e.y;
-      const float x1 = x[2 * i + 1] * e.z + y[2 * i + 1] * e.w, y1 = y[2 * i + 1] * e.z - x[2 * i + 1] * e.w;
-      x[2 * i] = x0; y[2 * i] = y0; x[2 * i + 1] = x1; y[2 * i + 1] = y1;
-    }
-  }
-  uint8_t* row = stg + rr * 256;
-#pragma unroll
-  for (int c = 0; c < CPT / 8; ++c) {
-    const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
-                                pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
-    const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
-                                pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
-    *reinterpret_cast<uint4*>(row + ((((CPT / 8) * g + c) ^ (rr & 15)) << 4)) = ux;
-    *reinterpret_cast<uint4*>(row + (((8 + (CPT / 8) * g + c) ^ (rr & 15)) << 4)) = uy;
-  }
-}
-// two staged bf16 tiles (32 KB apart) -> rows [0, n_valid) of dst0 / dst1 (row stride ld), 16 lanes per 256-B row
-__device__ __forceinline__ void stage16_store(const uint8_t* stg, int w8, int lane, int n_valid, bf16* dst0,
-                                              bf16* dst1, int ld) {
-  const int k = lane & 15;
-#pragma unroll 4
-  for (int i = 0; i < 128 * 2 / (2 * EW_WARPS); ++i) {
-    const int R = i * (2 * EW_WARPS) + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
-    if (rr >= n_valid) continue;
-    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 32768 + rr * 256 + ((k ^ (rr & 15)) << 4));
-    *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * ld + k * 8) = v;
   }
 }
 
@@ -167,9 +131,9 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   const int rep = p.H / p.Hkv;
   if (threadIdx.x == 0) {
     tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO64);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < 2; ++i) {   // dq_full / dq_free: only [0] is used (one dQ accumulator)
       mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], 1);
-      mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1 + DR_WARPS);   // MMA commit + drain
+      mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1);
       mbar_init(&dq_full[i], 1); mbar_init(&dq_free[i], DR_WARPS);
     }
     for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 2); mbar_init(&empty[i], 1); }   // TMA tx + lse/D stores
@@ -261,22 +225,26 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     // ------------------------------------------------ MMA issuer
     constexpr uint32_t ID_S = idesc_ab(128, QB, 0, 0);    // S^T, dP^T: [128 kv] x [64 q], K = hd
     constexpr uint32_t ID_ACC = idesc_ab(128, HD, 0, 1);  // dV, dK: [128 kv] x [128 hd], K = 64 q, B MN-major
-    constexpr uint32_t ID_DQ = idesc_ab(128, QB, 1, 1);   // dQ^T: [128 hd] x [64 q], K = 128 kv, A and B MN-major
+    constexpr uint32_t ID_DQ = idesc_ab(128, HD, 1, 1);   // dQ: [128 q (two blocks)] x [128 hd], K = 128 kv
     PF_DECL
-    int kvit = 0, gb = 0;
+    int kvit = 0, gb = 0, npair = 0, use[2] = {0, 0};
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
       const Geo G = load_geo(item);
       for (int j = 0; j < G.nkv; ++j, ++kvit) {
         const int kb = kvit & 1, vb = kb ^ 1, n = rep * nqb_of(G, j);
         const uint32_t k_s = smem_u32(sX0 + kb * KV_TILE), v_s = smem_u32(sX0 + vb * KV_TILE);
-        auto issue_acc = [&](int gp, int jp) {  // dV += P^T dO ; dK += dS^T Q ; dQ^T = K^T dS^T   (block gp)
-          const int bp = gp & 1, sp = gp % STAGES;
+        // dV += P^T dO ; dK += dS^T Q for block jp (P/dS buffer jp & 1); after the second block of a pair (or a
+        // unit's unpaired last block) dQ[2 x 64 q][hd] = dS (both dS^T buffers read MN-major as one M = 128 operand:
+        // they sit 16 KB apart = one M-atom stride) . K_j
+        auto issue_acc = [&](int gp, int jp) {
+          const int bp = jp & 1, sp = gp % STAGES;
+          const bool dq_now = (jp & 1) || jp == n - 1;
           PF(6);
-          wait_bar(&ew_done[bp], (gp >> 1) & 1);
+          wait_bar(&ew_done[bp], use[bp] & 1);
           PF(3);
           if (jp == 0) wait_bar(&acc_free, (kvit & 1) ^ 1);   // previous key block's epilogue has read dV / dK
           PF(4);
-          wait_bar(&dq_free[bp], ((gp >> 1) & 1) ^ 1);        // the drain has read dQ^T of block gp - 2
+          if (dq_now) wait_bar(&dq_free[0], (npair & 1) ^ 1);   // the drain has read the previous pair's dQ
           PF(5);
           tc_fence_after();
           __syncwarp();
@@ -289,18 +257,22 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
               tc_mma_bf16(tmem + T_DV, umma_desc_sw128(pa + kk * 32, 16, 1024), umma_desc_sw128(ob + kk * 2048, 8192, 1024), ID_ACC, acc);
               tc_mma_bf16(tmem + T_DK, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(qb + kk * 2048, 8192, 1024), ID_ACC, acc);
             }
-            // dQ^T[hd][q] = sum_kv K[kv][hd] dS^T[kv][q]: A = K tile read MN-major (hd contiguous, 2 atoms of 64),
-            // B = dS^T tile read MN-major (q contiguous, 1 atom); K-steps of 16 key rows = 2048 B
-#pragma unroll
-            for (int kk = 0; kk < 8; ++kk)
-              tc_mma_bf16(tmem + T_DQ + 64 * bp, umma_desc_sw128(k_s + kk * 2048, 16384, 1024),
-                          umma_desc_sw128(sa + kk * 2048, 16384, 1024), ID_DQ, kk > 0 ? 1u : 0u);
             tc_commit(&empty[sp]);     // Q/dO stage free
-            tc_commit(&pd_free[bp]);   // P^T/dS^T buffer free
-            tc_commit(&dq_full[bp]);   // dQ^T ready for the drain
+            if (dq_now) {
+              const uint32_t s0 = smem_u32(sS0);
+#pragma unroll
+              for (int kk = 0; kk < 8; ++kk)   // K-steps of 16 key rows = 2048 B in both the dS^T tiles and K
+                tc_mma_bf16(tmem + T_DQ, umma_desc_sw128(s0 + kk * 2048, 16384, 1024),
+                            umma_desc_sw128(k_s + kk * 2048, 16384, 1024), ID_DQ, kk > 0 ? 1u : 0u);
+              tc_commit(&dq_full[0]);
+              tc_commit(&pd_free[0]);                  // both P^T/dS^T buffers read for the last time
+              if (jp & 1) tc_commit(&pd_free[1]);
+            }
             if (jp == n - 1) { tc_commit(&x_empty[kb]); tc_commit(&acc_full); }   // K read for the last time
           }
           __syncwarp();
+          ++use[bp];
+          if (dq_now) ++npair;
         };
         PF(6);
         wait_bar(&x_full[kb], kvit & 1);
@@ -353,7 +325,7 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_F;
     PF_DECL
-    int kvit = 0, gb = 0;
+    int kvit = 0, gb = 0, use[2] = {0, 0};
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
       const Geo G = load_geo(item);
       for (int j = 0; j < G.nkv; ++j, ++kvit) {
@@ -361,7 +333,7 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         const int kpos = k0 + r;
         PF(8);
         for (int jj = 0; jj < n; ++jj, ++gb) {
-          const int b = gb & 1, st = gb % STAGES;
+          const int b = jj & 1, st = gb % STAGES;
           int h, q0;
           blk(G, j, nqb, jj, h, q0);
           PF(8);
@@ -392,15 +364,19 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
               const int c = c4 + u;
               const bool ok = fullb || (c >= cmin && c < cmax);
               const float x = fmaf(__uint_as_float(su[c]), sl2, -lzv[u]);
-              const float e = u == 3 ? poly_exp2(x) : fast_exp2(x);
+              const float e = (u == 3 || ((p.dbg == 4 || p.dbg == 6) && u == 1)) ? poly_exp2(x) : fast_exp2(x);
               pv[u] = ok ? e : 0.f;
               dsv[u] = ok ? e * fmaf(__uint_as_float(du[c]), p.scale, -dzv[u]) : 0.f;
             }
-            pk[c4 / 2] = pack_bf16x2(pv[0], pv[1]); pk[c4 / 2 + 1] = pack_bf16x2(pv[2], pv[3]);
+            if (p.dbg == 5 || p.dbg == 6) {
+              pk[c4 / 2] = pack_bf16x2_alu(pv[0], pv[1]); pk[c4 / 2 + 1] = pack_bf16x2_alu(pv[2], pv[3]);
+            } else {
+              pk[c4 / 2] = pack_bf16x2(pv[0], pv[1]); pk[c4 / 2 + 1] = pack_bf16x2(pv[2], pv[3]);
+            }
             dk[c4 / 2] = pack_bf16x2(dsv[0], dsv[1]); dk[c4 / 2 + 1] = pack_bf16x2(dsv[2], dsv[3]);
           }
           PF(8);
-          if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
+          wait_bar(&pd_free[b], (use[b] & 1) ^ 1);   // the buffer's previous block has been read by its MMAs
           PF(9);
           st_half_row_packed(sP0 + b * PT_TILE, r, g, pk);
           st_half_row_packed(sS0 + b * PT_TILE, r, g, dk);
@@ -408,127 +384,200 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive(&ew_done[b]);
+          ++use[b];
         }
-        // ---------------------------------------------- epilogue of key block j: dK (RoPE bwd), dV rows -> dqkv
+        // ---------------------------------------------- epilogue of key block j: key row r, columns [32g, 32g+32) of
+        // dK (and their RoPE partners 64 + ..., in-thread) and of dV -> bf16 rows staged (swizzled) in the P^T / dS^T
+        // buffers (all of the key block's MMAs are done), then written by whole rows; the first half of the thread's
+        // RoPE table row is fetched before the wait for the key block's last MMA
+        const int nv = min(KV_ROWS, G.L - k0), kr = k0 + r;
+        const bool rope = p.rope_cs != nullptr && r < nv;
+        const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)(r < nv ? kr : 0) * (HD / 2) + CPT * g);
+        float4 cs8[8];
+        if (rope) {
+#pragma unroll
+          for (int k = 0; k < 8; ++k) cs8[k] = __ldg(c4 + k);
+        }
         PF(8);
         wait_bar(&acc_full, kvit & 1);
-        {   // the staging below reuses all four P^T / dS^T buffers: wait until the drain released the last two blocks'
-          const int gl = gb - 1;
-          wait_bar(&pd_free[gl & 1], (gl >> 1) & 1);
-          if (gl >= 1) wait_bar(&pd_free[(gl - 1) & 1], ((gl - 1) >> 1) & 1);
-        }
         PF(10);
         tc_fence_after();
         __syncwarp();
-        const int nv = min(KV_ROWS, G.L - k0);
-        bf16* dst = p.dqkv + (size_t)(G.base + k0) * p.ld_dqkv;
-        acc_row_to_bf16(tmem + T_DK + lane_off, sP0, r, g, p.rope_cs, k0 + r, p.rope_cs != nullptr && r < nv);
-        acc_row_to_bf16(tmem + T_DV + lane_off, sP0 + 32768, r, g, nullptr, 0, false);
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&acc_free);
+        uint8_t* row_k = sP0 + r * 256;            // dK staging tile [128 rows][256 B]
+        uint8_t* row_v = sP0 + 32768 + r * 256;    // dV staging tile
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {           // 16 dims of the thread's 32 at a time (and their partners)
+          uint32_t ka[16], kb2[16];
+          asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                       : "=r"(ka[0]), "=r"(ka[1]), "=r"(ka[2]), "=r"(ka[3]), "=r"(ka[4]), "=r"(ka[5]), "=r"(ka[6]), "=r"(ka[7]),
+                         "=r"(ka[8]), "=r"(ka[9]), "=r"(ka[10]), "=r"(ka[11]), "=r"(ka[12]), "=r"(ka[13]), "=r"(ka[14]), "=r"(ka[15])
+                       : "r"(tmem + T_DK + CPT * g + 16 * hh + lane_off));
+          asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                       : "=r"(kb2[0]), "=r"(kb2[1]), "=r"(kb2[2]), "=r"(kb2[3]), "=r"(kb2[4]), "=r"(kb2[5]), "=r"(kb2[6]), "=r"(kb2[7]),
+                         "=r"(kb2[8]), "=r"(kb2[9]), "=r"(kb2[10]), "=r"(kb2[11]), "=r"(kb2[12]), "=r"(kb2[13]), "=r"(kb2[14]), "=r"(kb2[15])
+                       : "r"(tmem + T_DK + 64 + CPT * g + 16 * hh + lane_off));
+          tmem_wait_ld();
+          float x[16], y[16];
+#pragma unroll
+          for (int k = 0; k < 16; ++k) { x[k] = __uint_as_float(ka[k]); y[k] = __uint_as_float(kb2[k]); }
+          if (rope) {   // dx_i = dy_i c + dy_{i+64} s ; dx_{i+64} = dy_{i+64} c - dy_i s
+            if (hh == 1) {
+#pragma unroll
+              for (int k = 0; k < 8; ++k) cs8[k] = __ldg(c4 + 8 + k);
+            }
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+              const float4 e = cs8[k];
+              const float x0 = x[2 * k] * e.x + y[2 * k] * e.y, y0 = y[2 * k] * e.x - x[2 * k] * e.y;
+              const float x1 = x[2 * k + 1] * e.z + y[2 * k + 1] * e.w, y1 = y[2 * k + 1] * e.z - x[2 * k + 1] * e.w;
+              x[2 * k] = x0; y[2 * k] = y0; x[2 * k + 1] = x1; y[2 * k + 1] = y1;
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < 2; ++k) {   // 16-byte chunk c of the row at ((c ^ (r & 15)) << 4)
+            const int ck = (CPT / 8) * g + 2 * hh + k;
+            *reinterpret_cast<uint4*>(row_k + ((ck ^ (r & 15)) << 4)) =
+                make_uint4(pack_bf16x2(x[8 * k], x[8 * k + 1]), pack_bf16x2(x[8 * k + 2], x[8 * k + 3]),
+                           pack_bf16x2(x[8 * k + 4], x[8 * k + 5]), pack_bf16x2(x[8 * k + 6], x[8 * k + 7]));
+            *reinterpret_cast<uint4*>(row_k + (((8 + ck) ^ (r & 15)) << 4)) =
+                make_uint4(pack_bf16x2(y[8 * k], y[8 * k + 1]), pack_bf16x2(y[8 * k + 2], y[8 * k + 3]),
+                           pack_bf16x2(y[8 * k + 4], y[8 * k + 5]), pack_bf16x2(y[8 * k + 6], y[8 * k + 7]));
+          }
+        }
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {   // dV columns [32g, 32g+32) and [64+32g, ..)
+          uint32_t va[32];
+          tmem_ld32_nw(tmem + T_DV + 64 * hh + CPT * g + lane_off, va);
+          tmem_wait_ld();
+          if (hh == 1) {
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&acc_free);   // dK / dV read: the next key block may accumulate
+          }
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int ck = 8 * hh + (CPT / 8) * g + k;
+            *reinterpret_cast<uint4*>(row_v + ((ck ^ (r & 15)) << 4)) =
+                make_uint4(pack_bf16x2(__uint_as_float(va[8 * k]), __uint_as_float(va[8 * k + 1])),
+                           pack_bf16x2(__uint_as_float(va[8 * k + 2]), __uint_as_float(va[8 * k + 3])),
+                           pack_bf16x2(__uint_as_float(va[8 * k + 4]), __uint_as_float(va[8 * k + 5])),
+                           pack_bf16x2(__uint_as_float(va[8 * k + 6]), __uint_as_float(va[8 * k + 7])));
+          }
+        }
         ew_sync();
-        stage16_store(sP0, w8, lane, nv, dst + (p.H + G.hk) * HD, dst + (p.H + p.Hkv + G.hk) * HD, p.ld_dqkv);
+        {   // whole rows: 16 lanes x 16 B per 256-byte row, 2 rows per instruction
+          bf16* dst0 = p.dqkv + (size_t)(G.base + k0) * p.ld_dqkv + (p.H + G.hk) * HD;
+          bf16* dst1 = dst0 + p.Hkv * HD;
+          const int kq = lane & 15;
+#pragma unroll 4
+          for (int i = 0; i < 128 * 2 / (2 * EW_WARPS); ++i) {
+            const int R = i * (2 * EW_WARPS) + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
+            if (rr >= nv) continue;
+            const uint4 v = *reinterpret_cast<const uint4*>(sP0 + t * 32768 + rr * 256 + ((kq ^ (rr & 15)) << 4));
+            *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * p.ld_dqkv + kq * 8) = v;
+          }
+        }
         ew_sync();
         PF(11);
       }
     }
     PF_FLUSH(threadIdx.x == 64);
   } else {
-    // ------------------------------------------------ dQ drain (thread = head-dim index d = TMEM lane).  The CTA owns
-    // every key block of its (sequence, kv head), so each dQ element is only ever touched by THIS thread: the
-    // contributions of key blocks j = 0, 1, ... are ordered by program order alone (store, then red.add, then the
-    // last one loads) -- deterministic, no cross-CTA synchronisation.  The last contributor exchanges the RoPE partner
-    // d ^ 64 (another warp) through the block's P^T / dS^T buffers, which it holds until it arrives on pd_free.
+    // ------------------------------------------------ dQ drain: thread = one query row of a block pair (TMEM lane:
+    // rows 0-63 the pair's first block, 64-127 its second), all 128 head dims -- the RoPE pairs (d, d + 64) are in the
+    // same thread.  The CTA owns every key block of its (sequence, kv head), so each dQ element is touched only by the
+    // thread that owns its row: the contributions of key blocks j = 0, 1, ... are ordered by program order alone
+    // (j = 0 stores, later blocks red.add, the last one loads the sum) -- deterministic without cross-CTA sync.
     const int w4 = warp & 3;
-    const int d = w4 * 32 + lane;
+    const int r = w4 * 32 + lane, mem = r >> 6, qr = r & 63;
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const int ldq = p.H * HD;
     const bool rope = p.rope_cs != nullptr && p.dbg != 3;
-    const int i = d & 63;
-    const float sgn = d < 64 ? 1.f : -1.f;             // dx_d = dy_d c + dy_{d+64} s ; dx_{d+64} = dy_{d+64} c - dy_d s
     PF_DECL
-    int gb = 0;
+    int npair = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
       const Geo G = load_geo(item);
       for (int j = 0; j < G.nkv; ++j) {
         const int nqb = nqb_of(G, j), n = rep * nqb;
-        for (int jj = 0; jj < n; ++jj, ++gb) {
-          const int b = gb & 1;
-          int h, q0;
-          blk(G, j, nqb, jj, h, q0);
-          const bool last = j == q0 / KV_ROWS;          // contributors to queries [q0, q0 + 64): key blocks 0..last
-          const int nv = min(QB, G.L - q0);
-          float* acc = p.dq_acc + (size_t)(G.base + q0) * ldq + h * HD + d;
-          float pre[32];                                 // the last contributor's partial sum (first half), loaded
-          if (last && j > 0 && p.dbg != 1) {             // ahead of the TMEM wait
-#pragma unroll
-            for (int c = 0; c < 32; ++c) pre[c] = c < nv ? __ldcg(acc + (size_t)c * ldq) : 0.f;
-          }
+        for (int jp = 0; jp < n; jp += 2, ++npair) {
+          const int jj = jp + mem;
+          int h = 0, q0 = 0;
+          if (jj < n) blk(G, j, nqb, jj, h, q0);
+          const int q = q0 + qr;
+          const bool active = jj < n && q < G.L && p.dbg != 1;
+          const bool last = j == q0 / KV_ROWS;        // contributors to query q: key blocks 0..last
+          float* acc = p.dq_acc + (size_t)(G.base + q) * ldq + h * HD;
           PF(14);
-          wait_bar(&dq_full[b], (gb >> 1) & 1);
+          wait_bar(&dq_full[0], npair & 1);
           PF(12);
           tc_fence_after();
           __syncwarp();
-          uint32_t u0[32], u1[32];
-          tmem_ld32_nw(tmem + T_DQ + 64 * b + lane_off, u0);
-          tmem_ld32_nw(tmem + T_DQ + 64 * b + 32 + lane_off, u1);
-          tmem_wait_ld();
-          tc_fence_before();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&dq_free[b]);
-          if (p.dbg == 1 || !last) {
-            if (p.dbg != 1) {
 #pragma unroll
-              for (int half = 0; half < 2; ++half) {
-                const uint32_t (&u)[32] = half ? u1 : u0;
-                float* a0 = acc + (size_t)(32 * half) * ldq;
-                const int nh = nv - 32 * half;
-                if (j == 0) {
+          for (int c = 0; c < 2; ++c) {   // columns [32c, 32c+32) and their RoPE partners [64+32c, ..)
+            uint32_t ua[32], ub[32];
+            tmem_ld32_nw(tmem + T_DQ + 32 * c + lane_off, ua);
+            tmem_ld32_nw(tmem + T_DQ + 64 + 32 * c + lane_off, ub);
+            tmem_wait_ld();
+            if (c == 1) {
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive(&dq_free[0]);
+            }
+            if (!active) continue;
+            float4* a0 = reinterpret_cast<float4*>(acc + 32 * c);
+            float4* a1 = reinterpret_cast<float4*>(acc + 64 + 32 * c);
+            if (!last) {
+              if (j == 0) {
 #pragma unroll
-                  for (int c = 0; c < 32; ++c) if (c < nh) __stcg(a0 + (size_t)c * ldq, __uint_as_float(u[c]));
-                } else {
+                for (int k = 0; k < 8; ++k) {
+                  __stcg(a0 + k, make_float4(__uint_as_float(ua[4 * k]), __uint_as_float(ua[4 * k + 1]),
+                                             __uint_as_float(ua[4 * k + 2]), __uint_as_float(ua[4 * k + 3])));
+                  __stcg(a1 + k, make_float4(__uint_as_float(ub[4 * k]), __uint_as_float(ub[4 * k + 1]),
+                                             __uint_as_float(ub[4 * k + 2]), __uint_as_float(ub[4 * k + 3])));
+                }
+              } else {
 #pragma unroll
-                  for (int c = 0; c < 32; ++c)
-                    if (c < nh) asm volatile("red.relaxed.gpu.global.add.f32 [%0], %1;" ::"l"(a0 + (size_t)c * ldq),
-                                             "f"(__uint_as_float(u[c])) : "memory");
+                for (int k = 0; k < 8; ++k) {
+                  asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(a0 + k),
+                               "r"(ua[4 * k]), "r"(ua[4 * k + 1]), "r"(ua[4 * k + 2]), "r"(ua[4 * k + 3]) : "memory");
+                  asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(a1 + k),
+                               "r"(ub[4 * k]), "r"(ub[4 * k + 1]), "r"(ub[4 * k + 2]), "r"(ub[4 * k + 3]) : "memory");
                 }
               }
+              continue;
             }
-            if (lane == 0) mbar_arrive(&pd_free[b]);   // the block's P^T / dS^T buffers were not needed
-            PF(13);
-            continue;
-          }
-          // complete sums -> [q][d] fp32 staging in the block's P^T (queries 0-31) / dS^T (32-63) buffers
-          // (conflict-free), then the RoPE backward reads the partner d ^ 64 from there
-          float* stg0 = reinterpret_cast<float*>(sP0 + b * PT_TILE);
-          float* stg1 = reinterpret_cast<float*>(sS0 + b * PT_TILE);
+            float x[32], y[32];
 #pragma unroll
-          for (int c = 0; c < 32; ++c) stg0[c * HD + d] = __uint_as_float(u0[c]) + (j > 0 ? pre[c] : 0.f);
-          if (j > 0) {
+            for (int k = 0; k < 32; ++k) { x[k] = __uint_as_float(ua[k]); y[k] = __uint_as_float(ub[k]); }
+            if (j > 0) {
 #pragma unroll
-            for (int c = 0; c < 32; ++c) pre[c] = 32 + c < nv ? __ldcg(acc + (size_t)(32 + c) * ldq) : 0.f;
-          }
+              for (int k = 0; k < 8; ++k) {
+                const float4 e = __ldcg(a0 + k), f = __ldcg(a1 + k);
+                x[4 * k] += e.x; x[4 * k + 1] += e.y; x[4 * k + 2] += e.z; x[4 * k + 3] += e.w;
+                y[4 * k] += f.x; y[4 * k + 1] += f.y; y[4 * k + 2] += f.z; y[4 * k + 3] += f.w;
+              }
+            }
+            if (rope) {   // dx_d = dy_d c + dy_{d+64} s ; dx_{d+64} = dy_{d+64} c - dy_d s   (d = 32c + k)
+              const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)q * (HD / 2) + 32 * c);
 #pragma unroll
-          for (int c = 0; c < 32; ++c) stg1[c * HD + d] = __uint_as_float(u1[c]) + (j > 0 ? pre[c] : 0.f);
-          bf16* out = p.dqkv + (size_t)(G.base + q0) * p.ld_dqkv + h * HD + d;
-          dr_sync();
-          const float2* cs = p.rope_cs + (size_t)q0 * (HD / 2) + i;
-#pragma unroll 8
-          for (int c = 0; c < nv; ++c) {
-            const float* sg = c < 32 ? stg0 : stg1;
-            const float x = sg[(c & 31) * HD + d];
-            if (rope) {
-              const float xp = sg[(c & 31) * HD + (d ^ 64)];
-              const float2 e = __ldg(cs + (size_t)c * (HD / 2));
-              out[(size_t)c * p.ld_dqkv] = f2bf(x * e.x + sgn * xp * e.y);
-            } else {
-              out[(size_t)c * p.ld_dqkv] = f2bf(x);
+              for (int k = 0; k < 16; ++k) {
+                const float4 e = __ldg(c4 + k);   // (cos, sin) of dims 2k, 2k + 1
+                const float x0 = x[2 * k] * e.x + y[2 * k] * e.y, y0 = y[2 * k] * e.x - x[2 * k] * e.y;
+                const float x1 = x[2 * k + 1] * e.z + y[2 * k + 1] * e.w, y1 = y[2 * k + 1] * e.z - x[2 * k + 1] * e.w;
+                x[2 * k] = x0; y[2 * k] = y0; x[2 * k + 1] = x1; y[2 * k + 1] = y1;
+              }
+            }
+            uint4* o0 = reinterpret_cast<uint4*>(p.dqkv + (size_t)(G.base + q) * p.ld_dqkv + h * HD + 32 * c);
+            uint4* o1 = reinterpret_cast<uint4*>(p.dqkv + (size_t)(G.base + q) * p.ld_dqkv + h * HD + 64 + 32 * c);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              o0[k] = make_uint4(pack_bf16x2(x[8 * k], x[8 * k + 1]), pack_bf16x2(x[8 * k + 2], x[8 * k + 3]),
+                                 pack_bf16x2(x[8 * k + 4], x[8 * k + 5]), pack_bf16x2(x[8 * k + 6], x[8 * k + 7]));
+              o1[k] = make_uint4(pack_bf16x2(y[8 * k], y[8 * k + 1]), pack_bf16x2(y[8 * k + 2], y[8 * k + 3]),
+                                 pack_bf16x2(y[8 * k + 4], y[8 * k + 5]), pack_bf16x2(y[8 * k + 6], y[8 * k + 7]));
             }
           }
-          dr_sync();                                     // partner reads done: the buffers go back to the pipeline
-          if (lane == 0) mbar_arrive(&pd_free[b]);
-          PF(14);
+          PF(13);
         }
       }
     }

@@ -143,6 +143,25 @@ int attn_bwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 backward for head_dim 128 (attention_bwd_tc.cu); blocks128 = (seq, local start) per 128-row block
 int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaStream_t st);
 
+// ---------------------------------------------------------------- prefix tuning (prefix.cu; NEXT-3, R28)
+struct PrefixClient {        // one prefix-tuning client of a batch
+  const bf16* table;         // bf16 prefix [layers from first_layer][2 (k, v)][n][Nkv]
+  float* grad;               // fp32 gradient, same layout
+  int n;                     // prefix length P
+  int first_layer;           // the client's cut (local layer index)
+  int seq0, seq1;            // its sequences [seq0, seq1) in the batch
+};
+// ext row r: src[r].x >= 0 -> copy qkv row src[r].x; else prefix row (src[r].y & 0xFFFF) of batch client
+// (src[r].y >> 16): q = 0, k / v from that client's table at `layer`
+int prefix_gather(const bf16* qkv, int ld, const int2* src, int n_rows, const PrefixClient* pc, int layer, int Nq,
+                  int Nkv, bf16* out, cudaStream_t st);
+int rows_map(const bf16* src, int lds, const int* map, int n_rows, int width, bf16* dst, int ldd, cudaStream_t st);
+int lse_map(const float* src, int n_src, const int* map, int n_rows, int H, float* dst, cudaStream_t st);
+int dqkv_from_ext(const bf16* ext, const int* ext_row, int T, int H, int Hkv, int hd, const float2* cs, const int* pos,
+                  bf16* dqkv, cudaStream_t st);
+int prefix_grad(const bf16* dqkv_ext, int Nq, int Nkv, const PrefixClient* pc, int n_pc, int total_rows,
+                const int* seq_ext0, int layer, cudaStream_t st);
+
 // ---------------------------------------------------------------- AdamW + bf16 refresh
 struct AdamSeg {              // one (client, layer, target, A|B) parameter block
   long long p_off;            // offset into the client's flat fp32 buffers

@@ -101,6 +101,7 @@ static inline int ceil_div(int a, int b) { return (a + b - 1) / b; }
 // target / group geometry
 // =====================================================================================================
 enum { TQ = 0, TK, TV, TO, TG, TU, TD, NT };
+constexpr int TPFX = 7;   // target index of the prefix-tuning adapter in get/set_adapter (MENOS_T_PREFIX, NEXT-3)
 enum { GQKV = 0, GO, GGU, GD, NG };
 static const int kTargetGroup[NT] = {GQKV, GQKV, GQKV, GO, GGU, GGU, GD};
 
@@ -218,6 +219,8 @@ struct Client {
   size_t n_params = 0;
   size_t n_rep = 0;                 // params [0, n_rep) are replicated across tensor-parallel ranks
   std::vector<long long> offA, offB;  // [layer * NT + t]
+  int n_prefix = 0;                 // prefix tuning (NEXT-3, R28): P prefix rows per layer; params [layer >= cut][k|v][P][Nkv]
+  bf16* pfx = nullptr;              // its bf16 copy, same layout (read by the attention's prefix gather)
   float *P() const { return buf; }
   float *G() const { return buf + n_params; }
   float *M() const { return buf + 2 * n_params; }
@@ -317,6 +320,19 @@ struct menos_batch {
   uint8_t* scratch_base = nullptr; size_t scratch_span = 0;
   // live-batch accounting (menos_server::batch_refs / live_save): set when the handle is returned to the caller
   bool counted = false, counted_save = false;
+  // prefix tuning (NEXT-3, R28): the attention runs on an EXTENDED batch in which every sequence of a prefix client
+  // is preceded by the client's P prefix rows (q = 0, k / v = the layer's prefix); Text = its rows (T without)
+  bool has_pfx = false;
+  int Text = 0, n_pc = 0, pc_rows = 0;
+  std::vector<int> ext_len;           // per sequence: P + L
+  AttnView xview;                     // attention work lists over the extension (prefix batches have no mixed cuts)
+  int* d_cu_ext = nullptr; int2* d_blocks_ext = nullptr; int2* d_blocks128_ext = nullptr;
+  int2* d_ext_src = nullptr;          // per ext row: (token row, -) or (-1, client slot << 16 | prefix row)
+  int* d_ext_tok = nullptr;           // per ext row: token row or -1
+  int* d_tok_ext = nullptr;           // per token: its ext row
+  int* d_seq_ext0 = nullptr;          // per sequence: its first ext row
+  PrefixClient* d_pc = nullptr;
+  double pairs_ext = 0;
 };
 
 // =====================================================================================================
@@ -486,6 +502,17 @@ static int grow_group(menos_server* s, int g, int need_end) {
 // AdamW / refresh segments of one client (both A and B of every targeted (layer, target))
 static void client_segments(menos_server* s, const Client& c, int hyp_idx, std::vector<AdamSeg>& segs) {
   const Dims& D = s->D;
+  if (c.n_prefix) {   // prefix keys and values of every layer: rows P, cols Nkv, bf16 copy in the same layout
+    for (int l = c.cut; l < s->n_layers; ++l)
+      for (int kv = 0; kv < 2; ++kv) {
+        AdamSeg a{};
+        a.p_off = ((long long)(l - c.cut) * 2 + kv) * c.n_prefix * D.Nkv; a.rows = c.n_prefix; a.cols = D.Nkv;
+        a.client = hyp_idx; a.dst = c.pfx + a.p_off; a.dst_ld = D.Nkv; a.is_b = 0;
+        a.row_blk = 1 << 30; a.row_blk_stride = 0; a.row_base = 0;
+        segs.push_back(a);
+      }
+    return;
+  }
   for (int l = c.cut; l < s->n_layers; ++l)
     for (int t = 0; t < NT; ++t) {
       if (!(c.mask >> t & 1)) continue;
@@ -689,7 +716,7 @@ extern "C" void menos_server_destroy(menos_server* s) {
   if (!s) return;
   cudaSetDevice(s->device);
   cudaDeviceSynchronize();
-  for (auto& c : s->clients) if (c.buf) cudaFree(c.buf);
+  for (auto& c : s->clients) { if (c.buf) cudaFree(c.buf); if (c.pfx) cudaFree(c.pfx); }
   for (int g = 0; g < NG; ++g)
     for (int l = 0; l < s->n_layers; ++l) { if (s->Bcat[g][l]) cudaFree(s->Bcat[g][l]); if (s->Acat[g][l]) cudaFree(s->Acat[g][l]); }
   if (s->wbuf) cudaFree(s->wbuf);
@@ -730,7 +757,10 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
     FAIL(MENOS_EINVAL, "cut layer %d outside the server segment [%d, %d)", cut_layer, s->first_layer,
          s->first_layer + s->n_layers);
   if (rank < 1 || rank > s->opts.max_rank) FAIL(MENOS_EINVAL, "rank %d outside [1, %d]", rank, s->opts.max_rank);
-  if (!(alpha > 0.f) || target_mask == 0 || (target_mask >> NT)) FAIL(MENOS_EINVAL, "bad alpha/target mask");
+  const bool prefix = (target_mask >> TPFX) & 1;
+  if (!(alpha > 0.f) || target_mask == 0 || (target_mask >> (TPFX + 1))) FAIL(MENOS_EINVAL, "bad alpha/target mask");
+  if (prefix && target_mask != (1u << TPFX)) FAIL(MENOS_EINVAL, "a prefix-tuning client has no LoRA targets");
+  if (prefix && s->D.sp) FAIL(MENOS_EINVAL, "prefix tuning is not supported with tensor parallelism");
   if (s->D.arch == MENOS_ARCH_OPT && (target_mask >> TG & 1)) FAIL(MENOS_EINVAL, "OPT has no gate projection");
   CUDA_TRY(cudaSetDevice(s->device));
   int id = -1;
@@ -773,7 +803,11 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
   // parallelism their gradient partial sums are one contiguous all-reduce (menos_tp_cfg); with world 1 the
   // split is immaterial
   size_t n = 0;
-  for (int pass = 0; pass < 2; ++pass) {
+  if (prefix) {   // [layer >= cut][k | v][P][Nkv]; no LoRA, nothing replicated
+    c.n_prefix = rank;
+    for (int l = c.cut; l < s->n_layers; ++l) n += (size_t)2 * rank * D.Nkv;
+  }
+  for (int pass = 0; pass < 2 && !prefix; ++pass) {
     for (int l = c.cut; l < s->n_layers; ++l)   // no adapters below the client's cut
       for (int t = 0; t < NT; ++t) {
         if (!(target_mask >> t & 1)) continue;
@@ -803,6 +837,14 @@ extern "C" int menos_register_client_at(menos_server* s, int cut_layer, int rank
           if (k >= c0 && k < c0 + Kl) host[o + (long long)i * Kl + (k - c0)] = (float)((2.0 * u - 1.0) * bound);
         }
     }
+  if (prefix) {   // prefix keys / values ~ N(0, 1) (PEFT's embedding init), Box-Muller on the same stream
+    for (size_t i = 0; i < n; ++i) {
+      const double u1 = ((double)(splitmix(st) >> 11) + 1.0) * (1.0 / 9007199254740993.0);
+      const double u2 = (double)(splitmix(st) >> 11) * (1.0 / 9007199254740992.0);
+      host[i] = (float)(std::sqrt(-2.0 * std::log(u1)) * std::cos(6.283185307179586 * u2));
+    }
+    if (cudaMalloc(&c.pfx, n * sizeof(bf16)) != cudaSuccess) { cudaGetLastError(); cudaFree(c.buf); FAIL(MENOS_ENOMEM, "prefix table"); }
+  }
   CUDA_TRY(cudaMemcpy(c.buf, host.data(), n * sizeof(float), cudaMemcpyHostToDevice));
   c.used = true;
   s->clients[id] = c;
@@ -832,6 +874,7 @@ extern "C" int menos_unregister_client(menos_server* s, int32_t id) {
     s->cols[g].release(c.col_off[g], c.width[g]);
   }
   CUDA_TRY(cudaFree(c.buf));
+  if (c.pfx) CUDA_TRY(cudaFree(c.pfx));
   s->clients[id] = Client();
   CUDA_TRY(cudaDeviceSynchronize());
   return MENOS_OK;
@@ -873,6 +916,7 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
   // A + O: fp32 p, g, m, v + the bf16 slot-table copy (Acat rows + Bcat columns incl. rank padding)
   size_t slots = 0;
   for (int g = 0; g < NG; ++g) slots += (size_t)c.width[g] * (D.N_g[g] + D.ldK_g[g]) * 2 * s->n_layers;
+  if (c.pfx) slots += 2 * c.n_params;   // prefix tuning: the bf16 copy of the prefix table
   if (persistent) *persistent = 16 * c.n_params + slots;
   const bool save_a = ((c.mask >> TD) & 1) && D.arch != MENOS_ARCH_OPT;
   size_t ush = 0;
@@ -885,8 +929,8 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
   return MENOS_OK;
 }
 
-static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save);
-static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set);
+static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save, int Text);
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text);
 static size_t meta_bytes_bound(int T, int Ls, int n_clients);
 
 extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t* ids, const int32_t* n_tokens,
@@ -896,7 +940,7 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
   if (flags & ~(MENOS_FWD_NOGRAD | MENOS_MEM_BOUND)) FAIL(MENOS_EINVAL, "bad flags %d", flags);
   int R[NG] = {0, 0, 0, 0};
   bool save_a = false;
-  long long T = 0;
+  long long T = 0, Text = 0;   // prefix clients: bound on the extension, assuming one-token sequences
   if (flags & MENOS_MEM_BOUND) {   // additive bound: the registry-wide slot span and saved-tensor set
     for (const Client& c : s->clients) {
       if (!c.used) continue;
@@ -912,15 +956,18 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
     for (int g = 0; g < NG; ++g) if (c.width[g]) R[g] = std::max(R[g], c.col_off[g] + c.width[g]);
     if ((c.mask >> TD & 1) && D.arch != MENOS_ARCH_OPT) save_a = true;
     T += n_tokens[i];
+    Text += (long long)n_tokens[i] * (1 + c.n_prefix);
   }
   if (T > (1ll << 30)) FAIL(MENOS_EINVAL, "too many tokens");
   for (int g = 0; g < NG; ++g) R[g] = (int)align_up(R[g], 64);
   const bool nograd = flags & MENOS_FWD_NOGRAD;
-  const size_t meta = meta_bytes_bound((int)T, s->n_layers, n_clients);
+  const size_t meta = meta_bytes_bound((int)(T + Text), s->n_layers, n_clients);
   // forward: scratch (+ the NOGRAD layer set) + slab (+ meta); backward of a NOGRAD batch re-forwards with SAVE
-  const size_t fwd = scratch_bytes_of(D, (int)T, R, nograd) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, !nograd) + meta;
-  const size_t bwd = scratch_bytes_of(D, (int)T, R, nograd) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, true) +
-                     (nograd ? slab_bytes_of(D, s->n_layers, (int)T, R, save_a, false) : 0) + 2 * meta;
+  if (Text > (1ll << 30)) FAIL(MENOS_EINVAL, "too many tokens");
+  const int Tx = (int)Text;
+  const size_t fwd = scratch_bytes_of(D, (int)T, R, nograd, Tx) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, !nograd, Tx) + meta;
+  const size_t bwd = scratch_bytes_of(D, (int)T, R, nograd, Tx) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, true, Tx) +
+                     (nograd ? slab_bytes_of(D, s->n_layers, (int)T, R, save_a, false, Tx) : 0) + 2 * meta;
   if (fwd_bytes) *fwd_bytes = fwd;
   if (bwd_bytes) *bwd_bytes = bwd;
   return MENOS_OK;
@@ -929,9 +976,13 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
 extern "C" int menos_adapter_shape(menos_server* s, int32_t id, int target, int* rows, int* cols) {
   if (!s || !rows || !cols) FAIL(MENOS_EINVAL, "null argument");
   if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
-  if (target < 0 || target >= NT) FAIL(MENOS_EINVAL, "bad target");
+  if (target < 0 || target > TPFX) FAIL(MENOS_EINVAL, "bad target");
   const Client& c = s->clients[id];
   if (!(c.mask >> target & 1)) FAIL(MENOS_EINVAL, "target %d not in client mask", target);
+  if (target == TPFX) {   // prefix keys (A) and values (B): [P, Nkv] each
+    rows[0] = rows[1] = c.n_prefix; cols[0] = cols[1] = s->D.Nkv;
+    return MENOS_OK;
+  }
   rows[0] = c.rank; cols[0] = s->D.K_t[target];   // A [r, K]
   rows[1] = s->D.N_t[target]; cols[1] = c.rank;   // B [N, r]
   return MENOS_OK;
@@ -941,12 +992,20 @@ static int adapter_ptr(menos_server* s, int32_t id, int layer, int target, int w
                        Client** cp) {
   if (!s) FAIL(MENOS_EINVAL, "null server");
   if (id < 0 || id >= (int)s->clients.size() || !s->clients[id].used) FAIL(MENOS_ENOCLIENT, "unknown client %d", id);
-  if (layer < 0 || layer >= s->n_layers || target < 0 || target >= NT || which < 0 || which > 7)
+  if (layer < 0 || layer >= s->n_layers || target < 0 || target > TPFX || which < 0 || which > 7)
     FAIL(MENOS_EINVAL, "bad layer/target/which");
   Client& c = s->clients[id];
   if (!(c.mask >> target & 1)) FAIL(MENOS_EINVAL, "target %d not in client mask", target);
   if (layer < c.cut) FAIL(MENOS_EINVAL, "layer %d is below client %d's cut (no adapter there)", layer, id);
   const bool isB = which & 1;
+  if (target == TPFX) {   // A = prefix keys, B = prefix values, [P, Nkv] each
+    const long long off = ((long long)(layer - c.cut) * 2 + (isB ? 1 : 0)) * c.n_prefix * s->D.Nkv;
+    *n = (size_t)c.n_prefix * s->D.Nkv;
+    float* base = which < 2 ? c.P() : which < 4 ? c.G() : which < 6 ? c.M() : c.V();
+    *p = base + off;
+    *cp = &c;
+    return MENOS_OK;
+  }
   const long long off = isB ? c.offB[layer * NT + target] : c.offA[layer * NT + target];
   *n = (size_t)c.rank * (isB ? s->D.N_t[target] : s->D.K_t[target]);
   float* base = which < 2 ? c.P() : which < 4 ? c.G() : which < 6 ? c.M() : c.V();
@@ -978,7 +1037,8 @@ extern "C" int menos_set_adapter(menos_server* s, int32_t id, int layer, int tar
   std::vector<AdamSeg> all, one;
   client_segments(s, *c, 0, all);
   for (auto& sg : all) {
-    const long long want = which ? c->offB[layer * NT + target] : c->offA[layer * NT + target];
+    const long long want = target == TPFX ? (long long)(p - c->P())
+                                          : which ? c->offB[layer * NT + target] : c->offA[layer * NT + target];
     if (sg.p_off == want) one.push_back(sg);
   }
   rc = run_adam(s, {id}, false, 0, &one);
@@ -1064,6 +1124,8 @@ struct Scratch {
   bf16 *dyb, *dxb, *dhb;             // bf16 copies (A operands of the dX GEMMs, LoRA dY); local rows
   bf16 *dhn, *dO, *dqkv, *dgu, *a, *io;  // io: bf16 staging of x_c / x_s / g_c / g_s ([Tpad, d])
   bf16 *gath, *rsout;                // sequence parallel: all-gathered dy / dh [Tpad, d]; reduce-scatter output [Tloc, d]
+  bf16 *qkv_x, *O_x, *dO_x, *dqkv_x; // prefix-tuning extension [Text, .] (nullptr without prefix clients)
+  float *D_x, *dqacc_x;
   float* Dsum;
   bf16* dU[NG];
 };
@@ -1090,6 +1152,24 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   }
   b->T = b->cu.back();
   const int T = b->T;
+  // prefix tuning: the extension's sequence lengths
+  b->ext_len.resize(n_seqs);
+  b->Text = 0;
+  for (int i = 0; i < n_seqs; ++i) {
+    const Client& c = s->clients[b->seq_client[i]];
+    if (c.n_prefix) b->has_pfx = true;
+    b->ext_len[i] = c.n_prefix + b->seq_len[i];
+    b->Text += b->ext_len[i];
+    b->pairs_ext += 0.5 * (double)b->ext_len[i] * (b->ext_len[i] + 1);
+  }
+  if (b->has_pfx) {
+    if (D.sp) FAIL(MENOS_EINVAL, "prefix tuning is not supported with tensor parallelism");
+    for (int c : b->bclients)
+      if (s->clients[c].cut != 0) FAIL(MENOS_EINVAL, "a batch with prefix-tuning clients cannot mix cut points");
+    for (int i = 0; i < n_seqs; ++i)
+      if (b->ext_len[i] > s->opts.max_seq_len)
+        FAIL(MENOS_EINVAL, "sequence %d: prefix + length %d exceeds max_seq_len %d", i, b->ext_len[i], s->opts.max_seq_len);
+  }
   // per-client cuts: clients must come in non-decreasing cut order; layer l sees the prefix of clients with cut <= l
   b->Tl.assign(s->n_layers, 0);
   b->nseq_l.assign(s->n_layers, 0);
@@ -1128,13 +1208,14 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
 // Allocate the slab (saved activations or x_c copy) and upload all metadata incl. small-GEMM problem lists.
 // arena bytes of a batch's slab: the SAVE activations of every layer (I in Eq.3), or under NOGRAD
 // only the x_c copy; R_used = the batch's block-diagonal LoRA slot widths per group (0 = inactive)
-static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save) {
+// Text: rows of the prefix-tuning extension (== T without prefix clients); lse is kept for the extension
+static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save, int Text) {
   const Rows R = rows_of(D, T);   // sequence parallel: x, h, rstd local; xn, hn all-gathered
   if (!save) return align_up((size_t)R.Tloc * D.d * 4, 256);
   size_t per_layer = 0;
   auto A = [&](size_t n) { per_layer += align_up(n, 256); };
   A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // x (fp32), xn, rstd1
-  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * T * 4);        // qkv, O, lse
+  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * std::max(T, Text) * 4);   // qkv, O, lse
   A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // h (fp32), hn, rstd2
   A((size_t)T * D.gu_cols * 2);                                             // gu
   if (save_a) A((size_t)T * D.fpad * 2);
@@ -1142,7 +1223,7 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
   return per_layer * Ls;
 }
 // arena bytes of the per-call scratch block (see get_scratch)
-static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set) {
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text) {
   size_t need = 0;
   auto A = [&](size_t n) { need += align_up(n, 256); };
   const Rows Rw = rows_of(D, T);
@@ -1150,13 +1231,17 @@ static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool 
   A(df); A(df); A(df); A(df);                                                 // dyf, dxf, dhf, xout (local rows)
   A(db); A(db); A(db); A(dp); A(dp);                                          // dyb, dxb, dhb (local), dhn, io
   if (D.sp) { A(dp); A(db); }                                                 // gathered dy / dh, reduce-scatter out
+  if (Text > T) {   // prefix-tuning extension: qkv, O, dO, dqkv, D (fp32), the one-pass backward's dQ sums (fp32)
+    A((size_t)Text * D.Nqkv * 2); A((size_t)Text * D.Nq * 2); A((size_t)Text * D.Nq * 2);
+    A((size_t)Text * D.Nqkv * 2); A((size_t)D.H * Text * 4); A((size_t)Text * D.Nq * 4);
+  }
   A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.gu_cols * 2); A((size_t)T * D.fpad * 2);
   A((size_t)D.H * T * 4);                                                     // Dsum
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
   if (nograd_set) {
     A(dp); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
-    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * T * 4); A((size_t)Rw.Tloc * 8); A(dp);
+    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * std::max(T, Text) * 4); A((size_t)Rw.Tloc * 8); A(dp);
     for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   }
   return need;
@@ -1173,7 +1258,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const bool save = !b->nograd;
   int R_act[NG];
   for (int g = 0; g < NG; ++g) R_act[g] = b->g_active[g] ? b->R_used[g] : 0;
-  const size_t slab_bytes = slab_bytes_of(D, Ls, T, R_act, b->save_a, save);
+  const size_t slab_bytes = slab_bytes_of(D, Ls, T, R_act, b->save_a, save, b->Text);
   // ---- metadata blob
   std::vector<uint8_t> blob;
   auto put = [&](const void* p, size_t n) {
@@ -1248,6 +1333,56 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->views[v].o_items_q = put(v_items_q[v].data(), v_items_q[v].size() * sizeof(int4));
     b->views[v].o_items_seq = put(v_items_seq[v].data(), v_items_seq[v].size() * sizeof(int4));
   }
+  // prefix tuning: the extended batch's segment tables, row maps and attention work lists (one view)
+  size_t o_xcu = 0, o_xblk = 0, o_xblk128 = 0, o_xsrc = 0, o_xtok = 0, o_tokx = 0, o_seqx = 0, o_pc = 0;
+  size_t o_xit = 0, o_xitkv = 0, o_xitq = 0, o_xitseq = 0;
+  if (b->has_pfx) {
+    const std::vector<int>& xl = b->ext_len;
+    std::vector<int> xcu(1, 0), xtok, tokx(T), seqx(b->n_seqs);
+    std::vector<int2> xsrc, xb64, xb128;
+    std::vector<PrefixClient> pcs;
+    std::vector<int> slot_of(s->clients.size(), -1);
+    for (size_t k = 0; k < b->bclients.size(); ++k) {
+      const Client& c = s->clients[b->bclients[k]];
+      if (!c.n_prefix) continue;
+      PrefixClient pc{};
+      pc.table = c.pfx; pc.grad = c.G(); pc.n = c.n_prefix; pc.first_layer = c.cut;
+      pc.seq0 = pc.seq1 = -1;
+      slot_of[b->bclients[k]] = (int)pcs.size();
+      pcs.push_back(pc);
+    }
+    for (int i = 0; i < b->n_seqs; ++i) {
+      const int cid = b->seq_client[i], P = s->clients[cid].n_prefix;
+      seqx[i] = xcu.back();
+      if (P) {
+        PrefixClient& pc = pcs[slot_of[cid]];
+        if (pc.seq0 < 0) pc.seq0 = i;
+        pc.seq1 = i + 1;
+      }
+      for (int p = 0; p < P; ++p) { xsrc.push_back(make_int2(-1, slot_of[cid] << 16 | p)); xtok.push_back(-1); }
+      for (int t = b->cu[i]; t < b->cu[i + 1]; ++t) { tokx[t] = (int)xsrc.size(); xsrc.push_back(make_int2(t, 0)); xtok.push_back(t); }
+      xcu.push_back(xcu.back() + xl[i]);
+      for (int q = 0; q < xl[i]; q += 64) xb64.push_back(make_int2(i, q));
+      for (int q = 0; q < xl[i]; q += 128) xb128.push_back(make_int2(i, q));
+    }
+    b->n_pc = (int)pcs.size();
+    b->pc_rows = 0;
+    for (auto& pc : pcs) b->pc_rows += pc.n;
+    std::vector<int4> xi, xikv, xiq, xiseq;
+    attn_ws_items(xl.data(), b->n_seqs, D.H, xi, g_attn_order ? 1 : 0);
+    attn_ws_items(xl.data(), b->n_seqs, D.Hkv, xikv, g_attn_order ? 2 : 0);
+    attn_ws_items(xl.data(), b->n_seqs, D.H, xiq, g_attn_order ? 1 : 0);
+    attn_seq_items(xl.data(), b->n_seqs, D.Hkv, xiseq);
+    menos_batch::AttnView& xv = b->xview;
+    xv.n_seqs = b->n_seqs; xv.n_blocks = (int)xb64.size(); xv.n_blocks128 = (int)xb128.size(); xv.pairs = b->pairs_ext;
+    xv.n_items = (int)xi.size(); xv.n_items_kv = (int)xikv.size(); xv.n_items_seq = (int)xiseq.size();
+    o_xcu = put(xcu.data(), xcu.size() * 4); o_xblk = put(xb64.data(), xb64.size() * sizeof(int2));
+    o_xblk128 = put(xb128.data(), xb128.size() * sizeof(int2)); o_xsrc = put(xsrc.data(), xsrc.size() * sizeof(int2));
+    o_xtok = put(xtok.data(), xtok.size() * 4); o_tokx = put(tokx.data(), tokx.size() * 4);
+    o_seqx = put(seqx.data(), seqx.size() * 4); o_pc = put(pcs.data(), pcs.size() * sizeof(PrefixClient));
+    o_xit = put(xi.data(), xi.size() * sizeof(int4)); o_xitkv = put(xikv.data(), xikv.size() * sizeof(int4));
+    o_xitq = put(xiq.data(), xiq.size() * sizeof(int4)); o_xitseq = put(xiseq.data(), xiseq.size() * sizeof(int4));
+  }
   const size_t o_mt = put(mt.data(), mt.size() * sizeof(int2));
   const size_t o_nt = put(ntq.data(), ntq.size());
 
@@ -1264,7 +1399,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       LayerSave& S = b->L[l];
       S.x = (float*)take((size_t)Rw.Tloc * D.d * 4); S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
       S.rstd1 = (float*)take((size_t)Rw.Tloc * 4);
-      S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2); S.lse = (float*)take((size_t)D.H * T * 4);
+      S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
+      S.lse = (float*)take((size_t)D.H * std::max(T, b->Text) * 4);
       S.h = (float*)take((size_t)Rw.Tloc * D.d * 4); S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
       S.rstd2 = (float*)take((size_t)Rw.Tloc * 4);
       S.gu = (bf16*)take((size_t)T * D.gu_cols * 2);
@@ -1392,6 +1528,14 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   int rc = upload(s, meta, blob.data(), blob.size(), st);
   if (rc) return rc;
   b->d_cu = (int*)(meta + o_cu); b->d_pos = (int*)(meta + o_pos); b->d_blocks = (int2*)(meta + o_blk);
+  if (b->has_pfx) {
+    b->d_cu_ext = (int*)(meta + o_xcu); b->d_blocks_ext = (int2*)(meta + o_xblk);
+    b->d_blocks128_ext = (int2*)(meta + o_xblk128); b->d_ext_src = (int2*)(meta + o_xsrc);
+    b->d_ext_tok = (int*)(meta + o_xtok); b->d_tok_ext = (int*)(meta + o_tokx); b->d_seq_ext0 = (int*)(meta + o_seqx);
+    b->d_pc = (PrefixClient*)(meta + o_pc);
+    b->xview.items = (int4*)(meta + o_xit); b->xview.items_kv = (int4*)(meta + o_xitkv);
+    b->xview.items_q = (int4*)(meta + o_xitq); b->xview.items_seq = (int4*)(meta + o_xitseq);
+  }
   b->d_blocks128 = (int2*)(meta + o_blk128);
   for (auto& v : b->views) {
     v.items = (int4*)(meta + v.o_items);
@@ -1414,9 +1558,9 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
 // scratch (per server, grown to the largest batch; used only inside one call)
 // nograd_set: also reserve the NOGRAD forward's layer buffers (only a MENOS_FWD_NOGRAD forward needs them; the
 // backward's re-forward writes into the batch's SAVE slab), so SAVE batches use exactly scratch_bytes_per_token
-static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set) {
+static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set, int Text) {
   const Dims& D = s->D;
-  const size_t need = scratch_bytes_of(D, T, R_used, nograd_set);
+  const size_t need = scratch_bytes_of(D, T, R_used, nograd_set, Text);
   const Rows Rw = rows_of(D, T);
   const size_t df = (size_t)Rw.Tloc * D.d * 4, db = (size_t)Rw.Tloc * D.d * 2, dp = (size_t)Rw.Tpad * D.d * 2;
   if (need != s->scratch_bytes) {   // shrink-to-fit too: a stale large block must not outlive the call that needed it
@@ -1432,6 +1576,12 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   sc.io = (bf16*)take(dp);
   sc.gath = sc.rsout = nullptr;
   if (D.sp) { sc.gath = (bf16*)take(dp); sc.rsout = (bf16*)take(db); }
+  sc.qkv_x = sc.O_x = sc.dO_x = sc.dqkv_x = nullptr; sc.D_x = sc.dqacc_x = nullptr;
+  if (Text > T) {
+    sc.qkv_x = (bf16*)take((size_t)Text * D.Nqkv * 2); sc.O_x = (bf16*)take((size_t)Text * D.Nq * 2);
+    sc.dO_x = (bf16*)take((size_t)Text * D.Nq * 2); sc.dqkv_x = (bf16*)take((size_t)Text * D.Nqkv * 2);
+    sc.D_x = (float*)take((size_t)D.H * Text * 4); sc.dqacc_x = (float*)take((size_t)Text * D.Nq * 4);
+  }
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
   sc.dgu = (bf16*)take((size_t)T * D.gu_cols * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
   sc.Dsum = (float*)take((size_t)D.H * T * 4);
@@ -1440,14 +1590,14 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
 }
 
 // NOGRAD layer buffers carved after the regular scratch (same arena block)
-static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scratch& sc, LayerSave& S) {
+static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scratch& sc, LayerSave& S, int Text) {
   const Dims& D = s->D;
   const Rows Rw = rows_of(D, T);
   uint8_t* p = (uint8_t*)(sc.dU[NG - 1]) + align_up((size_t)T * R_used[NG - 1] * 2, 256);
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
   S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2); S.h = (float*)take((size_t)Rw.Tloc * D.d * 4);
   S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
-  S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * T * 4);
+  S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * std::max(T, Text) * 4);
   S.rstd1 = (float*)take((size_t)Rw.Tloc * 8); S.rstd2 = S.rstd1 + Rw.Tloc;
   S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
   S.a = D.arch == MENOS_ARCH_OPT ? S.gu : sc.a;   // OPT: the down projection's input is relu(fc1), kept in gu
@@ -1530,17 +1680,27 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     if (opt) { a.epi = EPI_STORE; a.bias = W.bqkv; }   // OPT: biases, no RoPE (learned positions are client-side)
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  // A3: varlen causal flash attention
+  // A3: varlen causal flash attention (prefix tuning, NEXT-3: on the extension -- every prefix client's sequence is
+  // preceded by its P prefix rows, so causal attention over it is "the whole prefix plus the causal keys", R28)
   {
+    const bool xp = b->has_pfx;
+    const menos_batch::AttnView& AV = xp ? b->xview : V;
+    if (xp)
+      K_TRY(prefix_gather(S.qkv, D.Nqkv, b->d_ext_src, b->Text, b->d_pc, l, D.Nq, D.Nkv, sc.qkv_x, st));
     AttnArgs a;
     memset(&a, 0, sizeof a);
-    a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
-    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = V.n_blocks; a.kvblocks = b->d_blocks;
-    a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * V.pairs, 0, st);
-    if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, V.items, V.n_items, s->num_sms, st));
-    else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, b->d_blocks128, V.n_blocks128, st));
-    else K_TRY(attn_fwd(a, st));
+    a.qkv = xp ? sc.qkv_x : S.qkv; a.ld_qkv = D.Nqkv; a.O = xp ? sc.O_x : S.O; a.ld_o = D.Nq; a.lse = S.lse;
+    a.cu_seqlens = xp ? b->d_cu_ext : b->d_cu;
+    const int2* blk64 = xp ? b->d_blocks_ext : b->d_blocks;
+    a.qblocks = blk64; a.n_qblocks = AV.n_blocks; a.kvblocks = blk64; a.n_kvblocks = AV.n_blocks;
+    a.T = xp ? b->Text : T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    {
+      ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * AV.pairs, 0, st);
+      if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, AV.items, AV.n_items, s->num_sms, st));
+      else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
+      else K_TRY(attn_fwd(a, st));
+    }
+    if (xp) K_TRY(rows_map(sc.O_x, D.Nq, b->d_tok_ext, T, D.Nq, S.O, D.Nq, st));   // drop the prefix rows' outputs
   }
   // A4: O GEMM (+ LoRA o) + residual
   if (b->g_active[GO]) {
@@ -1698,23 +1858,40 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     K_TRY(attn_bwd_prep(sc.dO, S.O, sc.Dsum, T, D.H, D.hd, st));
   }
   {
+    // prefix tuning (NEXT-3): the backward runs on the extension too -- dO and D are zero on the prefix rows (their
+    // outputs were dropped), the kernels skip the RoPE backward (prefix keys are not rotated, R28) and it is applied
+    // when the sequence rows are copied back; the prefix rows' dk, dv become the prefix gradients
+    const bool xp = b->has_pfx;
+    const menos_batch::AttnView& AV = xp ? b->xview : V;
+    if (xp) {
+      K_TRY(rows_map(sc.dO, D.Nq, b->d_ext_tok, b->Text, D.Nq, sc.dO_x, D.Nq, st));
+      K_TRY(lse_map(sc.Dsum, T, b->d_ext_tok, b->Text, D.H, sc.D_x, st));
+      K_TRY(prefix_gather(S.qkv, D.Nqkv, b->d_ext_src, b->Text, b->d_pc, l, D.Nq, D.Nkv, sc.qkv_x, st));
+    }
     AttnArgs a;
     memset(&a, 0, sizeof a);
-    a.qkv = S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
-    a.cu_seqlens = b->d_cu; a.qblocks = b->d_blocks; a.n_qblocks = V.n_blocks; a.kvblocks = b->d_blocks;
-    a.n_kvblocks = V.n_blocks; a.T = T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
-    a.dO = sc.dO; a.ld_do = D.Nq; a.D = sc.Dsum; a.dqkv = sc.dqkv; a.ld_dqkv = D.Nqkv;
-    a.rope_cs = opt ? nullptr : s->rope;   // OPT: no RoPE backward
+    a.qkv = xp ? sc.qkv_x : S.qkv; a.ld_qkv = D.Nqkv; a.O = S.O; a.ld_o = D.Nq; a.lse = S.lse;
+    a.cu_seqlens = xp ? b->d_cu_ext : b->d_cu;
+    const int2* blk64 = xp ? b->d_blocks_ext : b->d_blocks;
+    a.qblocks = blk64; a.n_qblocks = AV.n_blocks; a.kvblocks = blk64; a.n_kvblocks = AV.n_blocks;
+    a.T = xp ? b->Text : T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
+    a.dO = xp ? sc.dO_x : sc.dO; a.ld_do = D.Nq; a.D = xp ? sc.D_x : sc.Dsum;
+    a.dqkv = xp ? sc.dqkv_x : sc.dqkv; a.ld_dqkv = D.Nqkv;
+    a.rope_cs = (opt || xp) ? nullptr : s->rope;   // OPT: no RoPE backward; extension: applied on the copy back
     // one-pass backward: dQ accumulates in fp32 in the forward-output buffer (free during the backward: Nq <= d)
-    a.dq_acc = sc.xout;
+    a.dq_acc = xp ? sc.dqacc_x : sc.xout;
     {
-      ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * V.pairs, 0, st);
+      ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * AV.pairs, 0, st);
       if (D.hd == 128 && (g_attn_tc & 32))
-        K_TRY(attn_bwd_fused(a, V.items_seq, V.n_items_seq, s->num_sms, st));
+        K_TRY(attn_bwd_fused(a, AV.items_seq, AV.n_items_seq, s->num_sms, st));
       else if (D.hd == 128 && (g_attn_tc & 8))
-        K_TRY(attn_bwd_ws(a, V.items_kv, V.n_items_kv, V.items_q, V.n_items, s->num_sms, st));
-      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, b->d_blocks128, V.n_blocks128, st));
+        K_TRY(attn_bwd_ws(a, AV.items_kv, AV.n_items_kv, AV.items_q, AV.n_items, s->num_sms, st));
+      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
+    }
+    if (xp) {
+      K_TRY(dqkv_from_ext(sc.dqkv_x, b->d_tok_ext, T, D.H, D.Hkv, D.hd, opt ? nullptr : s->rope, b->d_pos, sc.dqkv, st));
+      K_TRY(prefix_grad(sc.dqkv_x, D.Nq, D.Nkv, b->d_pc, b->n_pc, b->pc_rows, b->d_seq_ext0, l, st));
     }
   }
   // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
@@ -1783,10 +1960,10 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
   const Dims& D = s->D;
   const int T = b->T;
   Scratch sc;
-  rc = get_scratch(s, T, b->R_used, sc, b->nograd);
+  rc = get_scratch(s, T, b->R_used, sc, b->nograd, b->Text);
   if (rc) return rc;
   LayerSave ng{};
-  if (b->nograd) nograd_layer(s, T, b->R_used, sc, ng);
+  if (b->nograd) nograd_layer(s, T, b->R_used, sc, ng, b->Text);
   rc = finalize_batch(s, b.get(), sc, &ng, st);
   if (rc) return rc;
   auto fail_free = [&](int code) {
@@ -1885,7 +2062,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   const int T = b->T;
   const Rows R = rows_of(D, T);
   Scratch sc;
-  int rc = get_scratch(s, T, b->R_used, sc, false);
+  int rc = get_scratch(s, T, b->R_used, sc, false, b->Text);
   if (rc) return rc;
   if (b->nograd) {
     // Alg.1 L10: re-forward with gradient preparation from the cached x_c; the SAVE slab is

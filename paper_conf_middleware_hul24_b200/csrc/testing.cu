@@ -230,7 +230,7 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
 // (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1),
 // 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; overrides 2).
 // Default 14: the persistent tcgen05 forward and backward (LPT work order, bit 4 selects (sequence, head) order).
-namespace menos { int g_attn_tc = 46; int g_attn_order = 1; }
+namespace menos { int g_attn_tc = 14; int g_attn_order = 1; }
 extern "C" int menos_test_abf_prof(unsigned long long* out16) {
   if (!out16) return fail("null output");
   return menos::attn_bwd_fused_prof(out16);

@@ -39,7 +39,8 @@ def new_server(w: Workload, weights, arena_bytes=0, max_rank=16, device="cuda:0"
         wl.append({k: _bf16(v) for k, v in W.items()})
     names = {"wq": "wq", "wk": "wk", "wv": "wv", "wo": "wo", "wgate": "wgate", "wup": "wup", "wdown": "wdown"}
     del names
-    max_seq = max(max(c.seq_lens) for c in w.clients)
+    # prefix-tuning clients (rank = P) attend over P + S rows: the library bounds that by max_seq_len too
+    max_seq = max(max(c.seq_lens) + (c.rank if "prefix" in c.targets else 0) for c in w.clients)
     srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
                  rms_eps=m.rms_eps, rope_theta=m.rope_theta, weights=wl, max_rank=max_rank,
                  max_seq_len=max(max_seq, 64), arena_bytes=arena_bytes, arch=m.arch)

@@ -244,7 +244,7 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-DEFAULT_ATTN_MODE = 46   # testing.cu g_attn_tc default: persistent tcgen05 forward + one-pass fused backward
+DEFAULT_ATTN_MODE = 14   # testing.cu g_attn_tc default: persistent tcgen05 forward + two-kernel persistent backward
 
 
 @pytest.fixture(autouse=True)

@@ -25,7 +25,14 @@ def tiny_mix():
     return Workload("tiny_mix", m, cl)
 
 
-CONFIGS = {"cfg0": (lambda: workload("cfg0_tiny"), 0), "tiny_mix": (tiny_mix, 3)}
+def prefix_mix():
+    from workloads import PREFIX
+    return Workload("prefix_mix", MODELS["tiny"], [ClientCfg(4, 8.0, ("q", "v"), [16, 16]),
+                                                   ClientCfg(4, 1.0, (PREFIX,), [9, 20]),
+                                                   ClientCfg(2, 1.0, (PREFIX,), [1, 30, 5])])
+
+
+CONFIGS = {"cfg0": (lambda: workload("cfg0_tiny"), 0), "tiny_mix": (tiny_mix, 3), "prefix_mix": (prefix_mix, 5)}
 
 
 @contextlib.contextmanager
@@ -83,6 +90,14 @@ def mutant(name, w, inputs):
     if name == "attention_skipped":
         with patched(attention_fwd=_attn_zero_fwd, attention_bwd=_attn_zero_bwd):
             return run_oracle_step(w, inputs=inputs)
+    if name == "prefix_ignored":     # the attention of prefix clients runs without their prefix (grads left correct)
+        if not any("prefix" in c.targets for c in w.clients):
+            return None
+        good = run_oracle_step(w, inputs=inputs)
+        ad = [[{t: v for t, v in d.items() if t != "prefix"} for d in a] for a in adapters]
+        bad = run_oracle_step(w, inputs=(weights, ad, io))
+        bad["grads"] = good["grads"]
+        return bad
     if name == "rope_off":
         with patched(rope_fwd=lambda x, c, s: x, rope_bwd=lambda dy, c, s: dy):
             return run_oracle_step(w, inputs=inputs)
@@ -130,7 +145,7 @@ def mutant(name, w, inputs):
     raise KeyError(name)
 
 
-MUTANTS = ["mlp_dropped", "attention_skipped", "rope_off", "gqa_modulo", "client_lora_dropped", "lora_scale_one",
+MUTANTS = ["mlp_dropped", "attention_skipped", "prefix_ignored", "rope_off", "gqa_modulo", "client_lora_dropped", "lora_scale_one",
            "sequences_not_separated", "last_sequence_grads_only", "identity"]
 
 

@@ -164,3 +164,34 @@ def test_relu_decision_in_kernel_precision_differs_only_where_ambiguous():
     assert np.all(np.abs(z[flips]) <= bound[flips])
     assert np.all(mask[np.abs(z) > bound] == (z[np.abs(z) > bound] > 0))
     assert flips.mean() < 5e-3
+
+
+def test_opt_prefix_finite_differences_fp64():
+    """Prefix tuning on the OPT layer (R28, no RoPE): finite differences of the prefix grads over 2 layers."""
+    import dataclasses
+    from workloads import PREFIX
+    cfg = dataclasses.replace(MODELS["opt_tiny"], n_layers=2, d_model=32, n_heads=4, n_kv_heads=4, d_ff=48)
+    Ws = [base_layer_weights(cfg, l, seed=71) for l in range(2)]
+    c = ClientCfg(2, 1.0, (PREFIX,), [5, 3])
+    ad = client_adapters(cfg, c, seed=72)
+    x, g = client_inputs(cfg, c, seed=73)
+    x, g = x.astype(np.float64), g.astype(np.float64)
+    _, _, gr = O.client_step(x, g, c.seq_lens, Ws, ad, 1.0, cfg, np.float64)
+
+    def loss(ll):
+        return float(np.sum(O.client_step(x, np.zeros_like(g), c.seq_lens, Ws, ll, 1.0, cfg, np.float64)[0] * g))
+
+    r = np.random.default_rng(74)
+    for ell in range(2):
+        for which in (0, 1):
+            base = ad[ell][PREFIX][which]
+            dirp = r.standard_normal(base.shape)
+
+            def with_p(pp):
+                ll = [dict(d) for d in ad]
+                Pk, Pv = ll[ell][PREFIX]
+                ll[ell][PREFIX] = (pp, Pv) if which == 0 else (Pk, pp)
+                return ll
+            fd = (loss(with_p(base + 1e-6 * dirp)) - loss(with_p(base - 1e-6 * dirp))) / 2e-6
+            an = np.sum(gr[ell][PREFIX][which] * dirp)
+            assert abs(fd - an) < 1e-6 * max(1.0, abs(fd)), (ell, which, fd, an)

@@ -439,3 +439,86 @@ def test_segment_composes_at_a_cut():
         for t in c.targets:
             np.testing.assert_allclose(gr2[l][t][0], gr[k + l][t][0], rtol=1e-10, atol=1e-13)
             np.testing.assert_allclose(gr2[l][t][1], gr[k + l][t][1], rtol=1e-10, atol=1e-13)
+
+
+# ------------------------------------------------------------------ prefix tuning (NEXT-3, reading R28)
+def _sdpa_prefix(q, k, v, pk, pv):
+    """torch SDPA (fp64) over [prefix | sequence] keys with an explicit mask: prefix always visible, causal inside the
+    sequence; GQA by repeating kv heads (HF repeat_kv)."""
+    S, H, hd = q.shape
+    P, Hkv = pk.shape[0], k.shape[1]
+    rep = H // Hkv
+    qt = q.permute(1, 0, 2)[None]
+    kk = torch.cat([pk, k]).repeat_interleave(rep, dim=1).permute(1, 0, 2)[None]
+    vv = torch.cat([pv, v]).repeat_interleave(rep, dim=1).permute(1, 0, 2)[None]
+    mask = torch.cat([torch.ones(S, P, dtype=torch.bool), torch.tril(torch.ones(S, S, dtype=torch.bool))], dim=1)
+    return torch.nn.functional.scaled_dot_product_attention(qt, kk, vv, attn_mask=mask)[0].permute(1, 0, 2)
+
+
+@pytest.mark.parametrize("H,Hkv,P", [(4, 4, 3), (4, 2, 5), (2, 1, 1)])
+def test_prefix_attention_vs_sdpa_autograd_fp64(H, Hkv, P):
+    r = np.random.default_rng(91)
+    S, hd = 9, 16
+    q, k, v = (r.standard_normal((S, n, hd)) for n in (H, Hkv, Hkv))
+    pk, pv = r.standard_normal((P, Hkv, hd)), r.standard_normal((P, Hkv, hd))
+    dO = r.standard_normal((S, H, hd))
+    O_, lse = O.attention_prefix_fwd(q, k, v, pk, pv)
+    ts = [torch.from_numpy(a).requires_grad_(True) for a in (q, k, v, pk, pv)]
+    ref = _sdpa_prefix(*ts)
+    np.testing.assert_allclose(O_, ref.detach().numpy(), rtol=1e-10, atol=1e-12)
+    ref.backward(torch.from_numpy(dO))
+    got = O.attention_prefix_bwd(dO, q, k, v, pk, pv)
+    for g, t in zip(got, ts):
+        np.testing.assert_allclose(g, t.grad.numpy(), rtol=1e-9, atol=1e-11)
+    # lse closed form at row 0: log(sum_j<P exp(s_0j) + exp(s_00)) per head
+    sc = 1.0 / np.sqrt(hd)
+    for h in range(H):
+        kv = h // (H // Hkv)
+        s0 = np.concatenate([pk[:, kv] @ q[0, h], [k[0, kv] @ q[0, h]]]) * sc
+        assert abs(lse[h, 0] - np.log(np.sum(np.exp(s0)))) < 1e-12
+
+
+def test_prefix_attention_reduces_to_causal_without_prefix():
+    r = np.random.default_rng(92)
+    q, k, v = (r.standard_normal((7, n, 8)) for n in (4, 2, 2))
+    empty = np.zeros((0, 2, 8))
+    a, la = O.attention_prefix_fwd(q, k, v, empty, empty)
+    b, lb = O.attention_fwd(q, k, v)
+    np.testing.assert_allclose(a, b, rtol=1e-13)
+    np.testing.assert_allclose(la, lb, rtol=1e-13)
+    dO = r.standard_normal(q.shape)
+    for x, y in zip(O.attention_prefix_bwd(dO, q, k, v, empty, empty)[:3], O.attention_bwd(dO, q, k, v)):
+        np.testing.assert_allclose(x, y, rtol=1e-12, atol=1e-14)
+
+
+def test_prefix_finite_differences_client_fp64():
+    """dL/dPk, dL/dPv of a prefix-tuning client over 2 layers and 2 sequences (summed over the client's tokens) by
+    central differences of L = sum(G * x_s)."""
+    import dataclasses
+    from workloads import PREFIX
+    cfg = dataclasses.replace(MODELS["tiny"], n_layers=2, n_kv_heads=2, d_model=32, n_heads=4, d_ff=48)
+    Ws = [base_layer_weights(cfg, l, seed=93) for l in range(2)]
+    c = ClientCfg(3, 1.0, (PREFIX,), [6, 4])
+    ad = client_adapters(cfg, c, seed=94)
+    x, g = client_inputs(cfg, c, seed=95)
+    x, g = x.astype(F64), g.astype(F64)
+    xs, gs, gr = O.client_step(x, g, c.seq_lens, Ws, ad, 1.0, cfg, F64)
+
+    def loss(ll):
+        return float(np.sum(O.client_step(x, np.zeros_like(g), c.seq_lens, Ws, ll, 1.0, cfg, F64)[0] * g))
+
+    r = np.random.default_rng(96)
+    eps = 1e-6
+    for ell in range(2):
+        for which in (0, 1):
+            base = ad[ell][PREFIX][which]
+            dirp = r.standard_normal(base.shape)
+
+            def with_p(pp):
+                ll = [dict(d) for d in ad]
+                Pk, Pv = ll[ell][PREFIX]
+                ll[ell][PREFIX] = (pp, Pv) if which == 0 else (Pk, pp)
+                return ll
+            fd = (loss(with_p(base + eps * dirp)) - loss(with_p(base - eps * dirp))) / (2 * eps)
+            an = np.sum(gr[ell][PREFIX][which] * dirp)
+            assert abs(fd - an) < 1e-6 * max(1.0, abs(fd)), (ell, which, fd, an)

@@ -39,14 +39,21 @@ def main():
     dqkv = torch.empty(T, N, dtype=torch.bfloat16, device="cuda")
     arr = (C.c_int32 * len(lens))(*lens)
     out = (C.c_ulonglong * 16)()
+    import time
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for it in range(3):
         lib.menos_test_abf_prof(out)   # clear
+        ev0.record()
         M.check(lib.menos_test_attention(len(lens), arr, H, Hkv, hd, qkv.data_ptr(), O.data_ptr(), lse.data_ptr(),
                                          dO.data_ptr(), dqkv.data_ptr(), 1e4), testing=True)
+        ev1.record()
+        torch.cuda.synchronize()
+        ms = ev0.elapsed_time(ev1)
         lib.menos_test_abf_prof(out)
     v = [int(x) for x in out]
     tot = max(sum(v[0:7]), 1)
-    print(json.dumps({"shape": {"lens": spec, "H": H, "Hkv": Hkv},
+    print(json.dumps({"shape": {"lens": spec, "H": H, "Hkv": Hkv}, "fwd_bwd_call_ms": round(ms, 3),
+                      "dbg": os.environ.get("MENOS_ABF_DBG", "0"),
                       "phases_frac_of_mma_total": {NAMES[k]: round(v[k] / tot, 4) for k in range(15)},
                       "mma_total_cycles": tot}, indent=1))
 

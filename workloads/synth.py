@@ -13,12 +13,15 @@ import numpy as np
 
 __all__ = [
     "ModelCfg", "ClientCfg", "Workload", "TARGETS", "MODELS", "target_dims",
-    "bf16_round", "bf16_bits", "bits_to_f32", "base_layer_weights", "client_adapters",
+    "bf16_round", "bf16_bits", "bits_to_f32", "base_layer_weights", "client_adapters", "PREFIX",
     "client_inputs", "workload", "WORKLOAD_NAMES",
 ]
 
 # LoRA target projections, in the bit order of include/menos.h (MENOS_T_*).
 TARGETS = ("q", "k", "v", "o", "gate", "up", "down")
+# Prefix tuning (NEXT-3): a client with targets == (PREFIX,) holds, per server layer, P = `rank`
+# learned key and value vectors per KV head ("A" = prefix keys, "B" = prefix values, both [P, H_kv * hd]).
+PREFIX = "prefix"
 
 
 @dataclass(frozen=True)
@@ -62,8 +65,11 @@ MODELS = {
 
 
 def target_dims(cfg: ModelCfg, t: str) -> tuple[int, int]:
-    """(K_in, N_out) of projection t: y[.., N] = x[.., K] W[N, K]^T."""
+    """(K_in, N_out) of projection t: y[.., N] = x[.., K] W[N, K]^T.  For PREFIX: (0, H_kv * hd), the width of one
+    prefix key / value row."""
     d, hd = cfg.d_model, cfg.head_dim
+    if t == PREFIX:
+        return 0, cfg.n_kv_heads * hd
     return {
         "q": (d, cfg.n_heads * hd),
         "k": (d, cfg.n_kv_heads * hd),
@@ -194,6 +200,13 @@ def client_adapters(cfg: ModelCfg, c: ClientCfg, seed: int, zero_b: bool = False
     b_std = np.sqrt(0.25 / c.rank) if is_small(cfg) else 0.02
     for ell in range(cfg.n_layers):
         d = {}
+        if PREFIX in c.targets:   # prefix keys / values ~ N(0, 1) (PEFT's nn.Embedding init; O(1) like the layer's k, v)
+            r = _rng(seed, ell, 50)
+            N = target_dims(cfg, PREFIX)[1]
+            d[PREFIX] = (bf16_round(r.standard_normal((c.rank, N), dtype=np.float32)),
+                         bf16_round(r.standard_normal((c.rank, N), dtype=np.float32)))
+            layers.append(d)
+            continue
         for ti, t in enumerate(TARGETS):
             if t not in c.targets:
                 continue
