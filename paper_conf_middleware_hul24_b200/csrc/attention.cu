@@ -332,7 +332,8 @@ __global__ void __launch_bounds__(128) attn_bwd_dkdv_kernel(const AttnArgs a) {
   for (int i = 0; i < NON; ++i)
 #pragma unroll
     for (int e = 0; e < 4; ++e) dk[i][e] *= a.scale;
-  const int p0 = min(kr0, L - 1), p1 = min(kr0 + 8, L - 1);
+  const int sh = a.pos_shift ? a.pos_shift[kb.x] : 0;   // prefix rows of an extended batch: position < 0 -> identity
+  const int p0 = min(kr0, L - 1) - sh, p1 = min(kr0 + 8, L - 1) - sh;
   if (a.rope_cs) rope_bwd_frag<HD>(dk, a.rope_cs, p0 < 0 ? 0 : p0, p1 < 0 ? 0 : p1);   // none for OPT
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
@@ -454,8 +455,9 @@ __global__ void __launch_bounds__(128) attn_bwd_dq_kernel(const AttnArgs a) {
   for (int i = 0; i < NON; ++i)
 #pragma unroll
     for (int e = 0; e < 4; ++e) dq[i][e] *= a.scale;
-  const int p0 = min(qr0, L - 1), p1 = min(qr0 + 8, L - 1);
-  if (a.rope_cs) rope_bwd_frag<HD>(dq, a.rope_cs, p0, p1);
+  const int sh = a.pos_shift ? a.pos_shift[qb.x] : 0;
+  const int p0 = min(qr0, L - 1) - sh, p1 = min(qr0 + 8, L - 1) - sh;
+  if (a.rope_cs) rope_bwd_frag<HD>(dq, a.rope_cs, p0 < 0 ? 0 : p0, p1 < 0 ? 0 : p1);
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
     const int qr = qr0 + r * 8;

@@ -58,6 +58,7 @@ struct FParams {
   bf16* dqkv; int ld_dqkv;
   const float2* rope_cs;   // [max_pos][HD/2] (cos, sin) or nullptr (no RoPE: OPT)
   float* dq_acc;           // [T, H*HD] fp32 partial sums of dQ
+  const int* pos_shift;    // [n_seqs] prefix rows before each sequence (extended batch) or nullptr
   int T, H, Hkv;
   float scale;
   int dbg;                 // tuning only (MENOS_ABF_DBG): 1 drain skips the global accumulation, 3 no RoPE
@@ -391,8 +392,10 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         // buffers (all of the key block's MMAs are done), then written by whole rows; the first half of the thread's
         // RoPE table row is fetched before the wait for the key block's last MMA
         const int nv = min(KV_ROWS, G.L - k0), kr = k0 + r;
+        const int sh = p.pos_shift ? p.pos_shift[G.seq] : 0;   // prefix rows: position < 0 -> identity (R28)
         const bool rope = p.rope_cs != nullptr && r < nv;
-        const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)(r < nv ? kr : 0) * (HD / 2) + CPT * g);
+        const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)(r < nv ? max(0, kr - sh) : 0) * (HD / 2) +
+                                                           CPT * g);
         float4 cs8[8];
         if (rope) {
 #pragma unroll
@@ -558,7 +561,8 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
               }
             }
             if (rope) {   // dx_d = dy_d c + dy_{d+64} s ; dx_{d+64} = dy_{d+64} c - dy_d s   (d = 32c + k)
-              const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)q * (HD / 2) + 32 * c);
+              const int sh = p.pos_shift ? p.pos_shift[G.seq] : 0;
+              const float4* c4 = reinterpret_cast<const float4*>(p.rope_cs + (size_t)max(0, q - sh) * (HD / 2) + 32 * c);
 #pragma unroll
               for (int k = 0; k < 16; ++k) {
                 const float4 e = __ldg(c4 + k);   // (cos, sin) of dims 2k, 2k + 1
@@ -616,7 +620,7 @@ int attn_bwd_fused(const AttnArgs& a, const int4* items_seq, int n_items, int nu
   if (!tma_map_2d(&mDO64, a.dO, a.T, a.H * HD, a.ld_do, 64, 64)) return -2;
   FParams p;
   p.cu_seqlens = a.cu_seqlens; p.items = items_seq; p.n_items = n_items; p.lse = a.lse; p.D = a.D;
-  p.dqkv = a.dqkv; p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.dq_acc = a.dq_acc;
+  p.dqkv = a.dqkv; p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.dq_acc = a.dq_acc; p.pos_shift = a.pos_shift;
   p.T = a.T; p.H = a.H; p.Hkv = a.Hkv; p.scale = a.scale;
   static const int dbg = getenv("MENOS_ABF_DBG") ? atoi(getenv("MENOS_ABF_DBG")) : 0;
   p.dbg = dbg;

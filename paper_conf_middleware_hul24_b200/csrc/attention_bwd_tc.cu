@@ -35,6 +35,7 @@ struct TcBwdParams {
   const float* D;          // [H, T]
   bf16* dqkv; int ld_dqkv;
   const float2* rope_cs;   // [max_pos][HD/2] (cos, sin)
+  const int* pos_shift;    // [n_seqs] prefix rows before each sequence (extended batch) or nullptr
   int T, H, Hkv;
   float scale;
 };
@@ -135,7 +136,7 @@ __device__ __forceinline__ void store_rows(const float* stg, int w8, int lane, i
       const int rr = w8 * 16 + half * 8 + u;
       const float* s = stg + rr * STG_LD;
       a0[u] = s[j]; a1[u] = s[j + 1]; b0[u] = s[64 + j]; b1[u] = s[65 + j];
-      if (rope && rr < n_valid) e[u] = *reinterpret_cast<const float4*>(cs + (size_t)(row0 + rr) * (HD / 2) + j);
+      if (rope && rr < n_valid) e[u] = *reinterpret_cast<const float4*>(cs + (size_t)max(0, row0 + rr) * (HD / 2) + j);
     }
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
@@ -340,7 +341,8 @@ attn_bwd_dkdv_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     ew_sync();
     TR_C(2)
     const int nv = min(KV_ROWS, L - k0);
-    store_rows(stgK, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + kcol, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
+    store_rows(stgK, w8, lane, k0 - (p.pos_shift ? p.pos_shift[kb.x] : 0), nv,
+               p.dqkv + (size_t)(base + k0) * p.ld_dqkv + kcol, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
     store_rows(stgV, w8, lane, k0, nv, p.dqkv + (size_t)(base + k0) * p.ld_dqkv + vcol, p.ld_dqkv, p.rope_cs, false);
     TR_C(3)
     if (threadIdx.x == 64) { TR_PRINT("EW") }
@@ -500,7 +502,8 @@ attn_bwd_dq_tc_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     stage_acc(tdQ + lane_off, stg, r, g);
     ew_sync();
     const int nv = min(Q_ROWS, L - q0);
-    store_rows(stg, w8, lane, q0, nv, p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
+    store_rows(stg, w8, lane, q0 - (p.pos_shift ? p.pos_shift[qb.x] : 0), nv,
+               p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD, p.ld_dqkv, p.rope_cs, p.rope_cs != nullptr);
   }
   tc_fence_before();
   __syncthreads();
@@ -523,7 +526,8 @@ int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaS
   if (!tma_map_2d(&mDO128, a.dO, a.T, a.H * HD, a.ld_do, 64, 128)) return -2;
   TcBwdParams p;
   p.cu_seqlens = a.cu_seqlens; p.blocks = blocks128; p.lse = a.lse; p.D = a.D; p.dqkv = a.dqkv;
-  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv; p.scale = a.scale;
+  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.pos_shift = a.pos_shift; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv;
+  p.scale = a.scale;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(attn_bwd_dkdv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DKDV);

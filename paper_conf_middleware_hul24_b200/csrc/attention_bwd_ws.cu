@@ -1,4 +1,5 @@
-// Varlen causal flash-attention BACKWARD, persistent warp-specialized tcgen05 kernels, head_dim 128.
+// Varlen causal flash-attention BACKWARD, persistent warp-specialized tcgen05 kernels, head_dim 128 or 64 (OPT-1.3B,
+// NEXT-4: one 128-byte swizzle atom per head row; the RoPE pairs are (j, j + hd/2)).
 // SURVEY.md §8(a) A11.  Same contract and math as attention_bwd_tc.cu (deterministic: no atomics; blocks never
 // cross a sequence, so never a client; GQA; RoPE backward applied to dq / dk before the store),
 // restructured so that the per-block fill / drain of the non-persistent kernels overlaps with useful work:
@@ -25,7 +26,7 @@ namespace {
 #define MENOS_BWS_EW 8
 #endif
 // EW_WARPS elementwise warps: EW_WARPS / 4 per TMEM lane quadrant, each thread owning CPT of a block's 64 columns
-constexpr int HD = 128, STAGES = 3, EW_WARPS = MENOS_BWS_EW, NTHREADS = 64 + 32 * EW_WARPS;
+constexpr int STAGES = 3, EW_WARPS = MENOS_BWS_EW, NTHREADS = 64 + 32 * EW_WARPS;
 constexpr int CPT = 64 / (EW_WARPS / 4);
 static_assert(CPT == 16 || CPT == 32, "EW_WARPS must be 8 or 16");
 constexpr float LOG2E_W = 1.4426950408889634f;
@@ -37,7 +38,8 @@ struct BwParams {
   const float* lse;        // [H, T] natural log
   const float* D;          // [H, T]
   bf16* dqkv; int ld_dqkv;
-  const float2* rope_cs;   // [max_pos][HD/2] (cos, sin)
+  const float2* rope_cs;   // [max_pos][hd/2] (cos, sin)
+  const int* pos_shift;    // [n_seqs] prefix rows before each sequence (extended batch) or nullptr
   int T, H, Hkv;
   float scale;
 };
@@ -83,50 +85,56 @@ __device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const
 // staging tile [128 rows][256 B] (16-byte chunk k of row rr at rr*256 + ((k ^ (rr & 15)) << 4)); the TMEM
 // accumulator is released right after the loads, then all warps store whole rows (2 rows per instruction).
 // Same fp32 ops in the same order as the staged-fp32 path: the bf16 result is bitwise identical.
+// (HD 64: columns [16g, 16g+16) and [32+16g, ..), rows of 128 B with chunk k at ((k ^ (rr & 7)) << 4).)
+template <int HD>
 __device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const float2* cs,
                                                 int pos, bool rope) {
-  uint32_t a[CPT], b[CPT];
-  tmem_ldc_nw(tacc + CPT * g, a);
-  tmem_ldc_nw(tacc + 64 + CPT * g, b);
+  constexpr int EC = HD / 4, NCH = HD / 8;   // columns per group per half, 16-byte chunks per row
+  uint32_t a[EC], b[EC];
+  tmem_ldc_nw(tacc + EC * g, a);
+  tmem_ldc_nw(tacc + HD / 2 + EC * g, b);
   tmem_wait_ld();
-  float x[CPT], y[CPT];
+  float x[EC], y[EC];
 #pragma unroll
-  for (int i = 0; i < CPT; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
-  if (rope) {   // dx_j = dy_j c + dy_{j+64} s,  dx_{j+64} = dy_{j+64} c - dy_j s
-    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + CPT * g);
+  for (int i = 0; i < EC; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
+  if (rope) {   // dx_j = dy_j c + dy_{j+hd/2} s,  dx_{j+hd/2} = dy_{j+hd/2} c - dy_j s
+    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + EC * g);
 #pragma unroll
-    for (int i = 0; i < CPT / 2; ++i) {
+    for (int i = 0; i < EC / 2; ++i) {
       const float4 e = __ldg(c4 + i);   // (c_2i, s_2i, c_2i+1, s_2i+1)
       const float x0 = x[2 * i] * e.x + y[2 * i] * e.y, y0 = y[2 * i] * e.x - x[2 * i] * e.y;
       const float x1 = x[2 * i + 1] * e.z + y[2 * i + 1] * e.w, y1 = y[2 * i + 1] * e.z - x[2 * i + 1] * e.w;
       x[2 * i] = x0; y[2 * i] = y0; x[2 * i + 1] = x1; y[2 * i + 1] = y1;
     }
   }
-  uint8_t* row = stg + rr * 256;
+  uint8_t* row = stg + rr * (HD * 2);
 #pragma unroll
-  for (int c = 0; c < CPT / 8; ++c) {
+  for (int c = 0; c < EC / 8; ++c) {
     const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
                                 pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
     const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
                                 pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
-    *reinterpret_cast<uint4*>(row + ((((CPT / 8) * g + c) ^ (rr & 15)) << 4)) = ux;
-    *reinterpret_cast<uint4*>(row + (((8 + (CPT / 8) * g + c) ^ (rr & 15)) << 4)) = uy;
+    *reinterpret_cast<uint4*>(row + ((((EC / 8) * g + c) ^ (rr & (NCH - 1))) << 4)) = ux;
+    *reinterpret_cast<uint4*>(row + (((NCH / 2 + (EC / 8) * g + c) ^ (rr & (NCH - 1))) << 4)) = uy;
   }
 }
-// n_tiles staged bf16 tiles (32 KB apart) -> rows [0, n_valid) of dst[t] (row stride ld), 16 lanes per 256-B row
+// n_tiles staged bf16 tiles (128 rows each, 128 * 2 HD bytes apart) -> rows [0, n_valid) of dst[t] (row stride ld):
+// HD / 8 lanes per row, 256 / HD rows per store instruction
+template <int HD>
 __device__ __forceinline__ void stage16_store(const uint8_t* stg, int n_tiles, int w8, int lane, int n_valid,
                                               bf16* dst0, bf16* dst1, int ld) {
-  const int k = lane & 15;
+  constexpr int NCH = HD / 8, RPI = 32 / NCH, ROWB = HD * 2;
+  const int k = lane % NCH;
 #pragma unroll 4
-  for (int i = 0; i < 128 * n_tiles / (2 * EW_WARPS); ++i) {
-    const int R = i * (2 * EW_WARPS) + w8 * 2 + (lane >> 4), t = R >> 7, rr = R & 127;
+  for (int i = 0; i < 128 * n_tiles / (RPI * EW_WARPS); ++i) {
+    const int R = i * (RPI * EW_WARPS) + w8 * RPI + lane / NCH, t = R >> 7, rr = R & 127;
     if (rr >= n_valid) continue;
-    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 32768 + rr * 256 + ((k ^ (rr & 15)) << 4));
+    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 128 * ROWB + rr * ROWB + ((k ^ (rr & (NCH - 1))) << 4));
     *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * ld + k * 8) = v;
   }
 }
 
-struct Geo { int base, L, blk0, head, n; };
+struct Geo { int base, L, blk0, head, n, sh; };   // sh: RoPE position shift of the sequence (prefix rows)
 
 // -DMENOS_BWS_PROF: per-phase clock64 accounting (dK/dV kernel: one elementwise thread and the MMA lane)
 #ifdef MENOS_BWS_PROF
@@ -142,14 +150,19 @@ __device__ unsigned long long g_bws_prof[16];
 
 // ======================================================================================= dK / dV
 constexpr int KV_ROWS = 128, QB = 64;
-constexpr int KV_TILE = KV_ROWS * HD * 2;      // 32 KB (2 atoms [128][64])
-constexpr int QB_TILE = QB * HD * 2;           // 16 KB (2 atoms [64][64])
 constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
-constexpr int SMEM_DKDV = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;
+constexpr int KVA = KV_ROWS * 128, QBA = QB * 128;   // one SW128 atom (64 columns) of a K / V tile, of a Q / dO tile
+template <int HD> struct DkdvGeo {
+  static constexpr int KV_TILE = KV_ROWS * HD * 2;   // HD 128: 32 KB (2 atoms [128][64]); 64: 16 KB
+  static constexpr int QB_TILE = QB * HD * 2;        // 16 KB (2 atoms [64][64]); 8 KB
+  static constexpr int SMEM = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;
+};
 
+template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
                         const __grid_constant__ CUtensorMap tmDO64, const BwParams p) {
+  constexpr int KV_TILE = DkdvGeo<HD>::KV_TILE, QB_TILE = DkdvGeo<HD>::QB_TILE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* const sK = smem;
@@ -181,10 +194,11 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   const uint32_t tdV = tmem + 256, tdK = tmem + 384;   // S^T buffers at 0/64, dP^T at 128/192
 
   auto load_geo = [&](int item) {
-    Geo g{0, 0, 0, 0, 0};
+    Geo g{0, 0, 0, 0, 0, 0};
     if (item < p.n_items) {
       const int4 it = p.items[item];
       g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
+      g.sh = p.pos_shift ? p.pos_shift[it.x] : 0;
       g.n = rep * ((g.L - g.blk0 + QB - 1) / QB);      // (head of the group, 64-query block) pairs
     }
     return g;
@@ -202,10 +216,11 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
         wait_bar(&kv_empty, (it & 1) ^ 1);
         mbar_expect_tx(&kv_full, 2 * KV_TILE);
-        tma_load_2d(sK, &tmQKV128, &kv_full, kcol, G.base + k0);
-        tma_load_2d(sK + 16384, &tmQKV128, &kv_full, kcol + 64, G.base + k0);
-        tma_load_2d(sV, &tmQKV128, &kv_full, vcol, G.base + k0);
-        tma_load_2d(sV + 16384, &tmQKV128, &kv_full, vcol + 64, G.base + k0);
+#pragma unroll
+        for (int a = 0; a < HD / 64; ++a) {
+          tma_load_2d(sK + a * KVA, &tmQKV128, &kv_full, kcol + 64 * a, G.base + k0);
+          tma_load_2d(sV + a * KVA, &tmQKV128, &kv_full, vcol + 64 * a, G.base + k0);
+        }
         for (int j = 0; j < G.n; ++j, ++gb) {
           const int st = gb % STAGES;
           const int h = hk * rep + j / nqb, q0 = k0 + (j % nqb) * QB;
@@ -213,10 +228,11 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
           mbar_expect_tx(&full[st], 2 * QB_TILE);
           uint8_t* q = sQ0 + st * QB_TILE;
           uint8_t* o = sO0 + st * QB_TILE;
-          tma_load_2d(q, &tmQKV64, &full[st], h * HD, G.base + q0);
-          tma_load_2d(q + 8192, &tmQKV64, &full[st], h * HD + 64, G.base + q0);
-          tma_load_2d(o, &tmDO64, &full[st], h * HD, G.base + q0);
-          tma_load_2d(o + 8192, &tmDO64, &full[st], h * HD + 64, G.base + q0);
+#pragma unroll
+          for (int a = 0; a < HD / 64; ++a) {
+            tma_load_2d(q + a * QBA, &tmQKV64, &full[st], h * HD + 64 * a, G.base + q0);
+            tma_load_2d(o + a * QBA, &tmDO64, &full[st], h * HD + 64 * a, G.base + q0);
+          }
         }
       }
     }
@@ -224,7 +240,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   } else if (warp == 1) {
     // ------------------------------------------------ MMA issuer
     constexpr uint32_t ID_S = umma_idesc_bf16(128, QB, 0);     // [128 kv] x [64 q], K = hd
-    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 kv] x [128 hd], K = 64 q, B MN-major
+    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 kv] x [hd], K = 64 q, B MN-major
     Geo nx = load_geo(blockIdx.x);
     BP_DECL
     int it = 0, gb = 0;
@@ -268,8 +284,8 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
           const uint32_t k = smem_u32(sK), v = smem_u32(sV);
           const uint32_t q = smem_u32(sQ0 + st * QB_TILE), o = smem_u32(sO0 + st * QB_TILE);
 #pragma unroll
-          for (int kk = 0; kk < 8; ++kk) {
-            const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
+          for (int kk = 0; kk < HD / 16; ++kk) {
+            const uint32_t offa = (kk >> 2) * KVA + (kk & 3) * 32, offb = (kk >> 2) * QBA + (kk & 3) * 32;
             tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(k + offa, 16, 1024), umma_desc_sw128(q + offb, 16, 1024), ID_S, kk > 0);
             tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(v + offa, 16, 1024), umma_desc_sw128(o + offb, 16, 1024), ID_S, kk > 0);
           }
@@ -369,14 +385,14 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       const int nv = min(KV_ROWS, L - k0);
       bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
       // P^T / dS^T buffers (64 KB, contiguous) = bf16 staging of dK | dV
-      acc_row_to_bf16(tdK + lane_off, sP0, r, g, p.rope_cs, k0 + r, p.rope_cs != nullptr && r < nv);
-      acc_row_to_bf16(tdV + lane_off, sP0 + 32768, r, g, nullptr, 0, false);
+      acc_row_to_bf16<HD>(tdK + lane_off, sP0, r, g, p.rope_cs, max(0, k0 + r - G.sh), p.rope_cs != nullptr && r < nv);
+      acc_row_to_bf16<HD>(tdV + lane_off, sP0 + 128 * HD * 2, r, g, nullptr, 0, false);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_free);   // the next item's dK / dV accumulation may start
       BP(7);
       ew_sync();
-      stage16_store(sP0, 2, w8, lane, nv, dst + (p.H + G.head) * HD, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv);
+      stage16_store<HD>(sP0, 2, w8, lane, nv, dst + (p.H + G.head) * HD, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv);
       ew_sync();
       BP(8);
     }
@@ -392,14 +408,19 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
 
 // ======================================================================================= dQ
 constexpr int Q_ROWS = 128, KB = 64;
-constexpr int Q_TILE = Q_ROWS * HD * 2;       // 32 KB
-constexpr int KB_TILE = KB * HD * 2;          // 16 KB
 constexpr int DS_TILE = Q_ROWS * KB * 2;      // 16 KB
-constexpr int SMEM_DQ = 2 * Q_TILE + 2 * STAGES * KB_TILE + 2 * DS_TILE + 1024;
+constexpr int QA = Q_ROWS * 128, KBA = KB * 128;   // one SW128 atom of a Q / dO tile, of a K / V stage
+template <int HD> struct DqGeo {
+  static constexpr int Q_TILE = Q_ROWS * HD * 2;   // HD 128: 32 KB; 64: 16 KB
+  static constexpr int KB_TILE = KB * HD * 2;      // 16 KB; 8 KB
+  static constexpr int SMEM = 2 * Q_TILE + 2 * STAGES * KB_TILE + 2 * DS_TILE + 1024;
+};
 
+template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
                       const __grid_constant__ CUtensorMap tmDO128, const BwParams p) {
+  constexpr int Q_TILE = DqGeo<HD>::Q_TILE, KB_TILE = DqGeo<HD>::KB_TILE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* const sQ = smem;
@@ -428,10 +449,11 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   const uint32_t tdQ = tmem + 256;   // S buffers at 0/64, dP at 128/192
 
   auto load_geo = [&](int item) {
-    Geo g{0, 0, 0, 0, 0};
+    Geo g{0, 0, 0, 0, 0, 0};
     if (item < p.n_items) {
       const int4 it = p.items[item];
       g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
+      g.sh = p.pos_shift ? p.pos_shift[it.x] : 0;
       g.n = (min(g.L, g.blk0 + Q_ROWS) + KB - 1) / KB;
     }
     return g;
@@ -448,27 +470,29 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
         wait_bar(&q_empty, (it & 1) ^ 1);
         mbar_expect_tx(&q_full, 2 * Q_TILE);
-        tma_load_2d(sQ, &tmQKV128, &q_full, h * HD, G.base + q0);
-        tma_load_2d(sQ + 16384, &tmQKV128, &q_full, h * HD + 64, G.base + q0);
-        tma_load_2d(sO, &tmDO128, &q_full, h * HD, G.base + q0);
-        tma_load_2d(sO + 16384, &tmDO128, &q_full, h * HD + 64, G.base + q0);
+#pragma unroll
+        for (int a = 0; a < HD / 64; ++a) {
+          tma_load_2d(sQ + a * QA, &tmQKV128, &q_full, h * HD + 64 * a, G.base + q0);
+          tma_load_2d(sO + a * QA, &tmDO128, &q_full, h * HD + 64 * a, G.base + q0);
+        }
         for (int j = 0; j < G.n; ++j, ++gb) {
           const int st = gb % STAGES;
           wait_bar(&empty[st], ((gb / STAGES) & 1) ^ 1);
           mbar_expect_tx(&full[st], 2 * KB_TILE);
           uint8_t* k = sK0 + st * KB_TILE;
           uint8_t* v = sV0 + st * KB_TILE;
-          tma_load_2d(k, &tmQKV64, &full[st], kcol, G.base + j * KB);
-          tma_load_2d(k + 8192, &tmQKV64, &full[st], kcol + 64, G.base + j * KB);
-          tma_load_2d(v, &tmQKV64, &full[st], vcol, G.base + j * KB);
-          tma_load_2d(v + 8192, &tmQKV64, &full[st], vcol + 64, G.base + j * KB);
+#pragma unroll
+          for (int a = 0; a < HD / 64; ++a) {
+            tma_load_2d(k + a * KBA, &tmQKV64, &full[st], kcol + 64 * a, G.base + j * KB);
+            tma_load_2d(v + a * KBA, &tmQKV64, &full[st], vcol + 64 * a, G.base + j * KB);
+          }
         }
       }
     }
     __syncwarp();
   } else if (warp == 1) {
     constexpr uint32_t ID_S = umma_idesc_bf16(128, KB, 0);     // [128 q] x [64 keys], K = hd
-    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 q] x [128 hd], K = 64 keys, B MN-major
+    constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 q] x [hd], K = 64 keys, B MN-major
     Geo nx = load_geo(blockIdx.x);
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
@@ -502,8 +526,8 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
           const uint32_t q = smem_u32(sQ), o = smem_u32(sO);
           const uint32_t k = smem_u32(sK0 + st * KB_TILE), v = smem_u32(sV0 + st * KB_TILE);
 #pragma unroll
-          for (int kk = 0; kk < 8; ++kk) {
-            const uint32_t offa = (kk >> 2) * 16384 + (kk & 3) * 32, offb = (kk >> 2) * 8192 + (kk & 3) * 32;
+          for (int kk = 0; kk < HD / 16; ++kk) {
+            const uint32_t offa = (kk >> 2) * QA + (kk & 3) * 32, offb = (kk >> 2) * KBA + (kk & 3) * 32;
             tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(q + offa, 16, 1024), umma_desc_sw128(k + offb, 16, 1024), ID_S, kk > 0);
             tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(o + offa, 16, 1024), umma_desc_sw128(v + offb, 16, 1024), ID_S, kk > 0);
           }
@@ -563,13 +587,13 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       __syncwarp();
       const int nv = min(Q_ROWS, L - q0);
       // dS buffers (32 KB) = bf16 staging of dQ
-      acc_row_to_bf16(tdQ + lane_off, sS0, r, g, p.rope_cs, q0 + r, p.rope_cs != nullptr && r < nv);
+      acc_row_to_bf16<HD>(tdQ + lane_off, sS0, r, g, p.rope_cs, max(0, q0 + r - G.sh), p.rope_cs != nullptr && r < nv);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_free);
       ew_sync();
       bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
-      stage16_store(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
+      stage16_store<HD>(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
       ew_sync();
     }
   }
@@ -594,10 +618,9 @@ int attn_bws_prof_read(unsigned long long* out) {
 #endif
 
 // items_kv: (seq, k0, kv head) per 128-key block for dK/dV; items_q: (seq, q0, head) per 128-query block for dQ
-int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
-                int num_sms, cudaStream_t st) {
-  if (a.hd != HD) return -1;
-  if (n_items_kv <= 0 && n_items_q <= 0) return 0;
+template <int HD>
+static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                         int num_sms, cudaStream_t st) {
   CUtensorMap mQKV128, mQKV64, mDO64, mDO128;
   if (!tma_map_2d(&mQKV128, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 128)) return -2;
   if (!tma_map_2d(&mQKV64, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 64)) return -2;
@@ -605,20 +628,31 @@ int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const i
   if (!tma_map_2d(&mDO128, a.dO, a.T, a.H * HD, a.ld_do, 64, 128)) return -2;
   BwParams p;
   p.cu_seqlens = a.cu_seqlens; p.lse = a.lse; p.D = a.D; p.dqkv = a.dqkv;
-  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv; p.scale = a.scale;
+  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.pos_shift = a.pos_shift; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv;
+  p.scale = a.scale;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(attn_bwd_dkdv_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DKDV);
-    cudaFuncSetAttribute(attn_bwd_dq_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_DQ);
+    cudaFuncSetAttribute(attn_bwd_dkdv_ws_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, DkdvGeo<HD>::SMEM);
+    cudaFuncSetAttribute(attn_bwd_dq_ws_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, DqGeo<HD>::SMEM);
     attr = true;
   }
   p.items = items_kv; p.n_items = n_items_kv;
-  attn_bwd_dkdv_ws_kernel<<<min(n_items_kv, num_sms), NTHREADS, SMEM_DKDV, st>>>(mQKV128, mQKV64, mDO64, p);
+  if (n_items_kv > 0)
+    attn_bwd_dkdv_ws_kernel<HD><<<min(n_items_kv, num_sms), NTHREADS, DkdvGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO64, p);
   ++g_launch_count;
   p.items = items_q; p.n_items = n_items_q;
-  attn_bwd_dq_ws_kernel<<<min(n_items_q, num_sms), NTHREADS, SMEM_DQ, st>>>(mQKV128, mQKV64, mDO128, p);
+  if (n_items_q > 0)
+    attn_bwd_dq_ws_kernel<HD><<<min(n_items_q, num_sms), NTHREADS, DqGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO128, p);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                int num_sms, cudaStream_t st) {
+  if (n_items_kv <= 0 && n_items_q <= 0) return 0;
+  if (a.hd == 128) return launch_bwd_ws<128>(a, items_kv, n_items_kv, items_q, n_items_q, num_sms, st);
+  if (a.hd == 64) return launch_bwd_ws<64>(a, items_kv, n_items_kv, items_q, n_items_q, num_sms, st);
+  return -1;
 }
 
 }  // namespace menos

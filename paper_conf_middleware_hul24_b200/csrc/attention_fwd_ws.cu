@@ -1,5 +1,5 @@
 // Varlen causal flash-attention FORWARD, persistent and warp-specialized on the 5th-gen tensor cores
-// (tcgen05 / TMEM / TMA), head_dim 128.  SURVEY.md §8(a) A3.  Same contract as attn_fwd_kernel (attention.cu):
+// (tcgen05 / TMEM / TMA), head_dim 128 (Llama-2, OPT-6.7B+) or 64 (OPT-1.3B: NEXT-4; one 128-byte swizzle atom per row).  SURVEY.md §8(a) A3.  Same contract as attn_fwd_kernel (attention.cu):
 // a work item never crosses a sequence (so never a client: PAPER.md:428), GQA head h -> kv head h / (H/Hkv),
 // LSE saved for the backward.
 //
@@ -22,11 +22,15 @@
 namespace menos {
 namespace {
 
-constexpr int HD = 128, BQ = 128, BKV = 64, K_STAGES = 4, V_STAGES = 4;
-constexpr int Q_BYTES = BQ * HD * 2;                 // 32 KB: 2 SW128 atoms [128][64]
-constexpr int K_BYTES = BKV * HD * 2;                // 16 KB: 2 atoms [64][64] (V tiles likewise)
+constexpr int BQ = 128, BKV = 64, K_STAGES = 4, V_STAGES = 4;
+constexpr int QA_BYTES = BQ * 64 * 2;                // one SW128 atom of Q: [128 rows][64 cols] = 16 KB
+constexpr int KA_BYTES = BKV * 64 * 2;               // one atom of a K / V tile: [64][64] = 8 KB
 constexpr int P_BYTES = BQ * BKV * 2;                // 16 KB: 1 atom [128][64]
-constexpr int SMEM_WS = 2 * Q_BYTES + (K_STAGES + V_STAGES) * K_BYTES + 2 * P_BYTES + 1024;
+template <int HD> struct FwdGeo {
+  static constexpr int Q_BYTES = BQ * HD * 2;        // HD 128: 2 atoms; 64: 1
+  static constexpr int K_BYTES = BKV * HD * 2;
+  static constexpr int SMEM = 2 * Q_BYTES + (K_STAGES + V_STAGES) * K_BYTES + 2 * P_BYTES + 1024;
+};
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float RESCALE_THRESHOLD = 8.0f;            // log2 units
 constexpr int NTHREADS = 256;
@@ -63,9 +67,11 @@ __device__ __forceinline__ void wait_spin(uint64_t* bar, uint32_t parity) {
   }
 }
 
+template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                    const WsParams p) {
+  constexpr int Q_BYTES = FwdGeo<HD>::Q_BYTES, K_BYTES = FwdGeo<HD>::K_BYTES;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;                                   // [2][Q_BYTES]
@@ -94,7 +100,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_sh;
-  // TMEM columns: S[0] 0..63, S[1] 64..127, O[0] 128..255, O[1] 256..383
+  // TMEM columns: S[0] 0..63, S[1] 64..127, O[0] 128..128+HD, O[1] 256..256+HD
   const uint32_t tS0 = tmem, tO0 = tmem + 128;
 
   // work-item geometry; every role loads the NEXT item's geometry at the top of the current one (two dependent
@@ -129,15 +135,15 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           wait_spin(&q_empty[qb], ((it >> 1) & 1) ^ 1);
           uint8_t* q = sQ + qb * Q_BYTES;
           mbar_expect_tx(&q_full[qb], Q_BYTES);
-          tma_load_2d(q, &tmQ, &q_full[qb], qcol, base + q0);
-          tma_load_2d(q + Q_BYTES / 2, &tmQ, &q_full[qb], qcol + 64, base + q0);
+#pragma unroll
+          for (int a = 0; a < HD / 64; ++a) tma_load_2d(q + a * QA_BYTES, &tmQ, &q_full[qb], qcol + 64 * a, base + q0);
           for (int j = 0; j < nkv; ++j, ++kc) {
             const int s = kc % K_STAGES;
             wait_spin(&k_empty[s], ((kc / K_STAGES) & 1) ^ 1);
             uint8_t* k = sK + s * K_BYTES;
             mbar_expect_tx(&k_full[s], K_BYTES);
-            tma_load_2d(k, &tmKV, &k_full[s], kcol, base + j * BKV);
-            tma_load_2d(k + K_BYTES / 2, &tmKV, &k_full[s], kcol + 64, base + j * BKV);
+#pragma unroll
+            for (int a = 0; a < HD / 64; ++a) tma_load_2d(k + a * KA_BYTES, &tmKV, &k_full[s], kcol + 64 * a, base + j * BKV);
           }
         } else {
           const int vcol = (p.H + p.Hkv + hk) * HD;
@@ -146,8 +152,8 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
             wait_spin(&v_empty[s], ((kc / V_STAGES) & 1) ^ 1);
             uint8_t* v = sV + s * K_BYTES;
             mbar_expect_tx(&v_full[s], K_BYTES);
-            tma_load_2d(v, &tmKV, &v_full[s], vcol, base + j * BKV);
-            tma_load_2d(v + K_BYTES / 2, &tmKV, &v_full[s], vcol + 64, base + j * BKV);
+#pragma unroll
+            for (int a = 0; a < HD / 64; ++a) tma_load_2d(v + a * KA_BYTES, &tmKV, &v_full[s], vcol + 64 * a, base + j * BKV);
           }
         }
       }
@@ -165,7 +171,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
       item_geom(nxt, item, base, L, q0, h, nkv);
       const int qb = it & 1, ob = it & 1;
       const uint32_t tO = tO0 + ob * 128;
-      wait_spin(&q_full[qb], (it >> 1) & 1);
+      wait_spin(&q_full[qb], (it >> 1) & 1);   // (TMEM: O[ob] at 128 + 128 ob, HD columns)
       const uint32_t qa = smem_u32(sQ + qb * Q_BYTES);
       int prev_kv = 0, prev_b = 0, prev_sc = 0;
       auto issue_pv = [&](int j, int gkv, int b, int gsc) {
@@ -183,7 +189,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
 #pragma unroll
           for (int kk = 0; kk < BKV / 16; ++kk) {
             const uint64_t ad = umma_desc_sw128(pa + kk * 32, 16, 1024);
-            const uint64_t bd = umma_desc_sw128(vb + kk * 2048, 8192, 1024);
+            const uint64_t bd = umma_desc_sw128(vb + kk * 2048, KA_BYTES, 1024);
             tc_mma_bf16(tO, ad, bd, IDESC_PV, (j > 0 || kk > 0) ? 1u : 0u);
           }
           tc_commit(&pv_done[b]);
@@ -203,8 +209,8 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           const uint32_t ka = smem_u32(sK + s * K_BYTES);
 #pragma unroll
           for (int kk = 0; kk < HD / 16; ++kk) {
-            const uint64_t ad = umma_desc_sw128(qa + (kk >> 2) * (Q_BYTES / 2) + (kk & 3) * 32, 16, 1024);
-            const uint64_t bd = umma_desc_sw128(ka + (kk >> 2) * (K_BYTES / 2) + (kk & 3) * 32, 16, 1024);
+            const uint64_t ad = umma_desc_sw128(qa + (kk >> 2) * QA_BYTES + (kk & 3) * 32, 16, 1024);
+            const uint64_t bd = umma_desc_sw128(ka + (kk >> 2) * KA_BYTES + (kk & 3) * 32, 16, 1024);
             tc_mma_bf16(tS0 + b * 64, ad, bd, IDESC_S, kk > 0 ? 1u : 0u);
           }
           tc_commit(&s_full[b]);
@@ -275,7 +281,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
             tc_fence_after();
             const float f = need ? exp2f(m_used - mx) : 1.f;
 #pragma unroll 1
-            for (int c = 0; c < 4; ++c) {
+            for (int c = 0; c < HD / 32; ++c) {
               float o[32];
               tmem_ld32(tO + c * 32, o);
 #pragma unroll
@@ -320,9 +326,9 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
       tc_fence_after();
       const bool rok = qpos < L;
       const float inv = 1.f / l;
-      uint32_t o[4][32];
+      uint32_t o[HD / 32][32];
 #pragma unroll
-      for (int c = 0; c < 4; ++c) tmem_ld32_nw(tO + c * 32, o[c]);
+      for (int c = 0; c < HD / 32; ++c) tmem_ld32_nw(tO + c * 32, o[c]);
       tmem_wait_ld();
       // stage this warp's 32 rows (256 B each) in its own P rows (free: every PV of this item has completed), then
       // write them out row-contiguously: one store instruction covers 2 full rows instead of 32 scattered ones
@@ -332,7 +338,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           return sP + (c >> 3) * P_BYTES + (wq * 32 + r) * 128 + (((c & 7) ^ (r & 7)) << 4);
         };
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
+        for (int c = 0; c < HD / 32; ++c)
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
             const uint32_t* w = o[c] + 8 * q;
@@ -343,9 +349,10 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
                            pack_bf16x2(__uint_as_float(w[6]) * inv, __uint_as_float(w[7]) * inv));
           }
         __syncwarp();
-        const int half = lane >> 4, c = lane & 15;
+        constexpr int LPR = HD / 8, RPI = 32 / LPR;   // lanes per staged row (16-byte chunks), rows per instruction
+        const int half = lane / LPR, c = lane % LPR;
 #pragma unroll 4
-        for (int r2 = 0; r2 < 32; r2 += 2) {
+        for (int r2 = 0; r2 < 32; r2 += RPI) {
           const int r = r2 + half, qp = q0 + wq * 32 + r;
           const uint4 u = *reinterpret_cast<const uint4*>(stage(r, c));
           if (qp < L) *reinterpret_cast<uint4*>(p.O + (size_t)(base + qp) * p.ld_o + h * HD + c * 8) = u;
@@ -408,9 +415,8 @@ int attn_ws_prof_read(unsigned long long* out) {
 }
 #endif
 
-int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st) {
-  if (a.hd != HD) return -1;
-  if (n_items <= 0) return 0;
+template <int HD>
+static int launch_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st) {
   CUtensorMap mQ, mKV;
   if (!tma_map_2d(&mQ, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, BQ)) return -2;
   if (!tma_map_2d(&mKV, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, BKV)) return -2;
@@ -419,13 +425,20 @@ int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, 
   p.T = a.T; p.H = a.H; p.Hkv = a.Hkv; p.scale = a.scale;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(attn_fwd_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_WS);
+    cudaFuncSetAttribute(attn_fwd_ws_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, FwdGeo<HD>::SMEM);
     attr = true;
   }
   const int grid = n_items < num_sms ? n_items : num_sms;
-  attn_fwd_ws_kernel<<<grid, NTHREADS, SMEM_WS, st>>>(mQ, mKV, p);
+  attn_fwd_ws_kernel<HD><<<grid, NTHREADS, FwdGeo<HD>::SMEM, st>>>(mQ, mKV, p);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st) {
+  if (n_items <= 0) return 0;
+  if (a.hd == 128) return launch_fwd_ws<128>(a, items, n_items, num_sms, st);
+  if (a.hd == 64) return launch_fwd_ws<64>(a, items, n_items, num_sms, st);
+  return -1;
 }
 
 }  // namespace menos

@@ -117,6 +117,9 @@ struct AttnArgs {
   const float2* rope_cs;         // [max_pos][hd/2]
   // one-pass backward (attention_bwd_fused.cu): per-thread ordered fp32 dQ accumulation
   float* dq_acc;                 // [T, H*hd] fp32 scratch
+  // prefix tuning (NEXT-3): per sequence, the number of prefix rows in front of it in this (extended) batch: the RoPE
+  // backward uses position = row - shift (clamped at 0, the identity rotation: prefix rows are not rotated, R28)
+  const int* pos_shift;          // [n_seqs] or nullptr
 };
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
 // tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block

@@ -331,6 +331,7 @@ struct menos_batch {
   int* d_ext_tok = nullptr;           // per ext row: token row or -1
   int* d_tok_ext = nullptr;           // per token: its ext row
   int* d_seq_ext0 = nullptr;          // per sequence: its first ext row
+  int* d_seq_shift = nullptr;         // per sequence: its client's prefix length (RoPE position shift in the kernels)
   PrefixClient* d_pc = nullptr;
   double pairs_ext = 0;
 };
@@ -1334,11 +1335,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->views[v].o_items_seq = put(v_items_seq[v].data(), v_items_seq[v].size() * sizeof(int4));
   }
   // prefix tuning: the extended batch's segment tables, row maps and attention work lists (one view)
-  size_t o_xcu = 0, o_xblk = 0, o_xblk128 = 0, o_xsrc = 0, o_xtok = 0, o_tokx = 0, o_seqx = 0, o_pc = 0;
+  size_t o_xcu = 0, o_xblk = 0, o_xblk128 = 0, o_xsrc = 0, o_xtok = 0, o_tokx = 0, o_seqx = 0, o_pc = 0, o_seqsh = 0;
   size_t o_xit = 0, o_xitkv = 0, o_xitq = 0, o_xitseq = 0;
   if (b->has_pfx) {
     const std::vector<int>& xl = b->ext_len;
-    std::vector<int> xcu(1, 0), xtok, tokx(T), seqx(b->n_seqs);
+    std::vector<int> xcu(1, 0), xtok, tokx(T), seqx(b->n_seqs), seqsh(b->n_seqs);
     std::vector<int2> xsrc, xb64, xb128;
     std::vector<PrefixClient> pcs;
     std::vector<int> slot_of(s->clients.size(), -1);
@@ -1354,6 +1355,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     for (int i = 0; i < b->n_seqs; ++i) {
       const int cid = b->seq_client[i], P = s->clients[cid].n_prefix;
       seqx[i] = xcu.back();
+      seqsh[i] = P;
       if (P) {
         PrefixClient& pc = pcs[slot_of[cid]];
         if (pc.seq0 < 0) pc.seq0 = i;
@@ -1380,6 +1382,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     o_xblk128 = put(xb128.data(), xb128.size() * sizeof(int2)); o_xsrc = put(xsrc.data(), xsrc.size() * sizeof(int2));
     o_xtok = put(xtok.data(), xtok.size() * 4); o_tokx = put(tokx.data(), tokx.size() * 4);
     o_seqx = put(seqx.data(), seqx.size() * 4); o_pc = put(pcs.data(), pcs.size() * sizeof(PrefixClient));
+    o_seqsh = put(seqsh.data(), seqsh.size() * 4);
     o_xit = put(xi.data(), xi.size() * sizeof(int4)); o_xitkv = put(xikv.data(), xikv.size() * sizeof(int4));
     o_xitq = put(xiq.data(), xiq.size() * sizeof(int4)); o_xitseq = put(xiseq.data(), xiseq.size() * sizeof(int4));
   }
@@ -1533,6 +1536,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->d_blocks128_ext = (int2*)(meta + o_xblk128); b->d_ext_src = (int2*)(meta + o_xsrc);
     b->d_ext_tok = (int*)(meta + o_xtok); b->d_tok_ext = (int*)(meta + o_tokx); b->d_seq_ext0 = (int*)(meta + o_seqx);
     b->d_pc = (PrefixClient*)(meta + o_pc);
+    b->d_seq_shift = (int*)(meta + o_seqsh);
     b->xview.items = (int4*)(meta + o_xit); b->xview.items_kv = (int4*)(meta + o_xitkv);
     b->xview.items_q = (int4*)(meta + o_xitq); b->xview.items_seq = (int4*)(meta + o_xitseq);
   }
@@ -1696,7 +1700,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     a.T = xp ? b->Text : T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     {
       ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * AV.pairs, 0, st);
-      if (D.hd == 128 && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, AV.items, AV.n_items, s->num_sms, st));
+      if ((D.hd == 128 || D.hd == 64) && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, AV.items, AV.n_items, s->num_sms, st));
       else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
       else K_TRY(attn_fwd(a, st));
     }
@@ -1877,20 +1881,23 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.T = xp ? b->Text : T; a.H = D.H; a.Hkv = D.Hkv; a.hd = D.hd; a.scale = 1.f / std::sqrt((float)D.hd);
     a.dO = xp ? sc.dO_x : sc.dO; a.ld_do = D.Nq; a.D = xp ? sc.D_x : sc.Dsum;
     a.dqkv = xp ? sc.dqkv_x : sc.dqkv; a.ld_dqkv = D.Nqkv;
-    a.rope_cs = (opt || xp) ? nullptr : s->rope;   // OPT: no RoPE backward; extension: applied on the copy back
+    a.rope_cs = opt ? nullptr : s->rope;   // OPT: no RoPE backward
+    a.pos_shift = xp ? b->d_seq_shift : nullptr;   // extension: positions shifted back by the prefix, prefix rows unrotated
     // one-pass backward: dQ accumulates in fp32 in the forward-output buffer (free during the backward: Nq <= d)
     a.dq_acc = xp ? sc.dqacc_x : sc.xout;
     {
       ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * AV.pairs, 0, st);
       if (D.hd == 128 && (g_attn_tc & 32))
         K_TRY(attn_bwd_fused(a, AV.items_seq, AV.n_items_seq, s->num_sms, st));
-      else if (D.hd == 128 && (g_attn_tc & 8))
+      else if ((D.hd == 128 || D.hd == 64) && (g_attn_tc & 8))
         K_TRY(attn_bwd_ws(a, AV.items_kv, AV.n_items_kv, AV.items_q, AV.n_items, s->num_sms, st));
       else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
     }
     if (xp) {
-      K_TRY(dqkv_from_ext(sc.dqkv_x, b->d_tok_ext, T, D.H, D.Hkv, D.hd, opt ? nullptr : s->rope, b->d_pos, sc.dqkv, st));
+      // the kernels applied the RoPE backward at the true positions: the sequence rows are copied back as they are
+      // (the same kernel epilogue as without prefix clients, so a LoRA client's results do not depend on them)
+      K_TRY(dqkv_from_ext(sc.dqkv_x, b->d_tok_ext, T, D.H, D.Hkv, D.hd, nullptr, b->d_pos, sc.dqkv, st));
       K_TRY(prefix_grad(sc.dqkv_x, D.Nq, D.Nkv, b->d_pc, b->n_pc, b->pc_rows, b->d_seq_ext0, l, st));
     }
   }
@@ -2156,7 +2163,7 @@ extern "C" int menos_test_batch_tensor(menos_server* s, menos_batch* b, int laye
     case 6: src = S.gu; n = T * D.gu_cols * 2; break;
     case 7: src = S.a; n = T * D.fpad * 2; break;
     case 8: case 9: case 10: case 11: src = S.U[which - 8]; n = src ? T * b->R_used[which - 8] * 2 : 0; break;
-    case 12: src = S.lse; n = (size_t)D.H * T * 4; break;
+    case 12: src = S.lse; n = (size_t)D.H * std::max<size_t>(T, b->Text) * 4; break;   // prefix: [H, Text]
     default: FAIL(MENOS_EINVAL, "bad which");
   }
   *bytes = n;

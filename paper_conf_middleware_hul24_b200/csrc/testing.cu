@@ -94,7 +94,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
   cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
   const bool tc_fwd = hd == 128 && (g_attn_tc & 1), tc_bwd = hd == 128 && (g_attn_tc & 2);
-  const bool ws_fwd = hd == 128 && (g_attn_tc & 4);
+  const bool ws_fwd = (hd == 128 || hd == 64) && (g_attn_tc & 4);
   std::vector<int4> items;
   attn_ws_items(seq_len, n_seqs, H, items, g_attn_order ? 1 : 0);
   int4* d_items;
@@ -114,7 +114,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
     int4* d_items_kv;
     cudaMalloc(&d_items_kv, std::max<size_t>(1, items_kv.size()) * sizeof(int4));
     cudaMemcpy(d_items_kv, items_kv.data(), items_kv.size() * sizeof(int4), cudaMemcpyHostToDevice);
-    const bool ws_bwd = hd == 128 && (g_attn_tc & 8);
+    const bool ws_bwd = (hd == 128 || hd == 64) && (g_attn_tc & 8);
     const bool fused_bwd = hd == 128 && (g_attn_tc & 32);
     float* d_acc = nullptr;
     std::vector<int4> items_seq;

@@ -260,6 +260,7 @@ def _restore_attention_mode():
                                              (128, 2, 2, [512, 1024, 255], 46), (128, 3, 1, [2048, 1, 700], 46),
                                              (128, 8, 8, [512] * 16 + [77], 46), (128, 8, 1, [1024] * 3 + [33], 46),
                                              (128, 4, 4, [1, 17, 64, 129, 300], -46),
+                                             (64, 8, 1, [200, 65, 1], 14), (64, 4, 4, [200, 65, 1000, 3], -14),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 14), (128, 8, 1, [130, 7, 256], 14),
                                              (128, 2, 2, [512, 1024, 255], 14), (128, 3, 1, [2048, 1, 700], 14),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 6), (128, 8, 1, [130, 7, 256], 6),

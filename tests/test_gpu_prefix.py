@@ -27,7 +27,8 @@ def prefix_mix(m):
 
 @pytest.mark.parametrize("m", [MODELS["tiny"], dataclasses.replace(MODELS["tiny"], n_kv_heads=2),
                                ModelCfg("hd128", 512, 4, 2, 1024, 2, model_layers=3),   # tcgen05 attention kernels
-                               MODELS["opt_tiny"]], ids=["tiny", "tiny_gqa", "hd128_gqa", "opt_tiny"])
+                               ModelCfg("opt-small", 256, 4, 4, 1024, 2, model_layers=3, arch="opt")],
+                         ids=["tiny", "tiny_gqa", "hd128_gqa", "opt_small_hd64"])
 def test_prefix_clients_mixed_with_lora(m):
     w = prefix_mix(m)
     if m.arch == "opt":   # OPT has no gate projection

@@ -54,7 +54,7 @@ def _worker(rank, world, port, wl, flags, q, transport="gloo"):
         else:
             tpc = (rank, world, TP.make_torch_collective())
         srv = Server(m.d_model, m.n_heads, m.n_kv_heads, m.d_ff, m.n_layers, first_layer=m.first_layer,
-                     weights=shards, max_rank=16, max_seq_len=1024, arena_bytes=2 << 30, tp=tpc)
+                     weights=shards, max_rank=16, max_seq_len=1024, arena_bytes=1 << 30, tp=tpc)
         ids = []
         for i, c in enumerate(wl.clients):
             cid = srv.register_client(c.rank, c.alpha, c.targets, seed=i)
@@ -90,7 +90,10 @@ def _worker(rank, world, port, wl, flags, q, transport="gloo"):
 
 
 def _run(wl, flags=0, world=2, transport="gloo"):
+    import gc
     import torch.multiprocessing as mp
+    gc.collect()                 # the workers share this GPU: release what earlier tests left in this process
+    torch.cuda.empty_cache()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()

@@ -136,8 +136,11 @@ RECIPES = ("default", "plain")
 
 
 def is_small(cfg: ModelCfg) -> bool:
-    """The tiny parity configs (d < 1024): weights are width-scaled (reading R26)."""
-    return cfg.d_model < 1024
+    """The tiny Llama parity configs (d < 1024): weights are width-scaled (reading R26).  OPT keeps the
+    Llama-width recipe at every size: with O(1) branches its ReLU MLP's fc1 LoRA grads are ill-conditioned in bf16 --
+    an exact-bf16 evaluation of the oracle itself reaches only cos 0.9985-0.9991 (tools/bf16_emulation.py) -- so no
+    bf16 kernel could meet the bar there; the OPT white-box test checks every intermediate instead."""
+    return cfg.d_model < 1024 and cfg.arch != "opt"
 
 
 def weight_std(cfg: ModelCfg, t: str, recipe: str = "default") -> float:
