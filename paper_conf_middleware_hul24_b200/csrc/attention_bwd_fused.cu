@@ -405,7 +405,7 @@ attn_bwd_fused_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         wait_bar(&acc_full, kvit & 1);
         PF(10);
         tc_fence_after();
-        __syncwarp();
+        ew_sync();   // every warp's last P^T / dS^T stores precede the staging writes (visible to racecheck)
         uint8_t* row_k = sP0 + r * 256;            // dK staging tile [128 rows][256 B]
         uint8_t* row_v = sP0 + 32768 + r * 256;    // dV staging tile
 #pragma unroll

@@ -380,7 +380,8 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       wait_bar(&acc_full, it & 1);
       BP(6);
       tc_fence_after();
-      __syncwarp();
+      ew_sync();   // order every warp's last P^T / dS^T stores before the staging writes (the mbarrier chain through
+                   // the MMAs already does; the named barrier makes it visible to compute-sanitizer racecheck)
       // all MMAs of this item completed: P^T / dS^T buffers are free for staging
       const int nv = min(KV_ROWS, L - k0);
       bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
@@ -584,7 +585,7 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       }
       wait_bar(&acc_full, it & 1);
       tc_fence_after();
-      __syncwarp();
+      ew_sync();   // as in the dK / dV epilogue: the dS^T stores of every warp precede the staging writes
       const int nv = min(Q_ROWS, L - q0);
       // dS buffers (32 KB) = bf16 staging of dQ
       acc_row_to_bf16<HD>(tdQ + lane_off, sS0, r, g, p.rope_cs, max(0, q0 + r - G.sh), p.rope_cs != nullptr && r < nv);

@@ -1,11 +1,12 @@
 // Per-phase clock accounting of the persistent dK/dV backward kernel at the cfg1 shape (tuning aid).
-// Build: nvcc ... -DMENOS_BWS_PROF attention_bwd_ws.cu + this driver (see tools/README or DESIGN.md).
+// Build (on the GPU box): MENOS_NVCC_DEFS=-DMENOS_BWS_PROF python -m paper_conf_middleware_hul24_b200.build -f, then
+//   nvcc -std=c++17 -gencode arch=compute_100a,code=sm_100a tools/attn_bwd_phases.cu -I<pkg>/csrc <pkg>/_lib/*.o -lcuda -ldl
 #include <cstdio>
 #include <vector>
 #include <cmath>
 #include <cstring>
 #include "../paper_conf_middleware_hul24_b200/csrc/kernels.h"
-namespace menos { int attn_bws_prof_read(unsigned long long* out); int g_attn_order = 1; }
+namespace menos { int attn_bws_prof_read(unsigned long long* out); extern int g_attn_order; }
 using namespace menos;
 int main() {
   const int nseq = 16, S = 512, H = 32, Hkv = 32, hd = 128, T = nseq * S, N = (H + 2 * Hkv) * hd;
