@@ -30,6 +30,24 @@ constexpr int STAGES = 3, EW_WARPS = MENOS_BWS_EW, NTHREADS = 64 + 32 * EW_WARPS
 constexpr int CPT = 64 / (EW_WARPS / 4);
 static_assert(CPT == 16 || CPT == 32, "EW_WARPS must be 8 or 16");
 constexpr float LOG2E_W = 1.4426950408889634f;
+// MENOS_BWS_TMEM_P (default 1): the elementwise warps write P^T / dS^T (dK/dV kernel) and dS (dQ kernel) as packed
+// bf16 into the TMEM columns of the S / dP tile they have just read, and the accumulation MMAs take them as the A
+// operand from TMEM ("ts" form): no shared-memory round trip (16-32 KB of stores and MMA operand reads per block),
+// no proxy fence, no buffer-free barrier.  0: the shared-memory path (tuning A/B only).
+#ifndef MENOS_BWS_TMEM_P
+#define MENOS_BWS_TMEM_P 1
+#endif
+#if MENOS_BWS_TMEM_P
+static_assert(CPT == 32, "the packed TMEM operand layout assumes two 32-column thread groups (8 elementwise warps)");
+#endif
+// TMEM column (relative to the tile) of K-chunk kk (16 queries / keys) of a packed operand: thread group g wrote its
+// 32 columns' values into the first 16 of the 32 columns it had read (columns [32 g, 32 g + 16))
+__device__ __forceinline__ uint32_t packed_col(int kk) { return (uint32_t)((kk & 1) * 8 + (kk >> 1) * 32); }
+// pack CPT fp32 values into CPT / 2 bf16x2 words (even column in the low half)
+__device__ __forceinline__ void pack_row(const float (&v)[CPT], uint32_t (&u)[CPT / 2]) {
+#pragma unroll
+  for (int i = 0; i < CPT / 2; ++i) u[i] = pack_bf16x2(v[2 * i], v[2 * i + 1]);
+}
 
 struct BwParams {
   const int* cu_seqlens;
@@ -81,15 +99,26 @@ __device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const
 }
 
 // Single-round epilogue: every elementwise thread converts its TMEM row (columns [32g, 32g+32) and [64+32g, ..),
-// i.e. the RoPE pairs (j, j+64)) to bf16 in registers -- RoPE backward applied there -- and writes it into a bf16
-// staging tile [128 rows][256 B] (16-byte chunk k of row rr at rr*256 + ((k ^ (rr & 15)) << 4)); the TMEM
-// accumulator is released right after the loads, then all warps store whole rows (2 rows per instruction).
-// Same fp32 ops in the same order as the staged-fp32 path: the bf16 result is bitwise identical.
-// (HD 64: columns [16g, 16g+16) and [32+16g, ..), rows of 128 B with chunk k at ((k ^ (rr & 7)) << 4).)
+// i.e. the RoPE pairs (j, j+64)) to bf16 in registers -- RoPE backward applied there, with the (cos, sin) pairs
+// loaded BEFORE the wait for the accumulator (rope_cs_load) so the table's L2 latency hides behind it -- and writes it
+// into a bf16 staging matrix in the TMA SWIZZLE_128B layout: HD / 64 atoms of [128 rows][128 B], 16-byte chunk k
+// of row rr at atom (k / 8), rr * 128 + (((k % 8) ^ (rr & 7)) << 4).  The x half (columns < HD/2) lands in the first
+// half of the atoms, the y half in the second.  A full 128-row block leaves by TMA store (one thread, async: the
+// warps go on with the next item); a sequence's ragged last block by row-masked 16-byte stores (stage16_store).
+// Same fp32 ops in the same order as before: the bf16 result is bitwise identical.
 template <int HD>
-__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const float2* cs,
-                                                int pos, bool rope) {
-  constexpr int EC = HD / 4, NCH = HD / 8;   // columns per group per half, 16-byte chunks per row
+struct RopeCS { float4 v[HD / 8]; };   // (c_2i, s_2i, c_2i+1, s_2i+1) for the thread's HD/4 pairs
+template <int HD>
+__device__ __forceinline__ void rope_cs_load(RopeCS<HD>& c, const float2* cs, int pos, int g, bool rope) {
+  if (!rope) return;
+  const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + (HD / 4) * g);
+#pragma unroll
+  for (int i = 0; i < HD / 8; ++i) c.v[i] = __ldg(c4 + i);
+}
+template <int HD>
+__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const RopeCS<HD>& cs,
+                                                bool rope) {
+  constexpr int EC = HD / 4;   // columns per group per half
   uint32_t a[EC], b[EC];
   tmem_ldc_nw(tacc + EC * g, a);
   tmem_ldc_nw(tacc + HD / 2 + EC * g, b);
@@ -98,42 +127,65 @@ __device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int
 #pragma unroll
   for (int i = 0; i < EC; ++i) { x[i] = __uint_as_float(a[i]); y[i] = __uint_as_float(b[i]); }
   if (rope) {   // dx_j = dy_j c + dy_{j+hd/2} s,  dx_{j+hd/2} = dy_{j+hd/2} c - dy_j s
-    const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + EC * g);
 #pragma unroll
     for (int i = 0; i < EC / 2; ++i) {
-      const float4 e = __ldg(c4 + i);   // (c_2i, s_2i, c_2i+1, s_2i+1)
+      const float4 e = cs.v[i];
       const float x0 = x[2 * i] * e.x + y[2 * i] * e.y, y0 = y[2 * i] * e.x - x[2 * i] * e.y;
       const float x1 = x[2 * i + 1] * e.z + y[2 * i + 1] * e.w, y1 = y[2 * i + 1] * e.z - x[2 * i + 1] * e.w;
       x[2 * i] = x0; y[2 * i] = y0; x[2 * i + 1] = x1; y[2 * i + 1] = y1;
     }
   }
-  uint8_t* row = stg + rr * (HD * 2);
+  uint8_t* row = stg + rr * 128;
 #pragma unroll
   for (int c = 0; c < EC / 8; ++c) {
     const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
                                 pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
     const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
                                 pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
-    *reinterpret_cast<uint4*>(row + ((((EC / 8) * g + c) ^ (rr & (NCH - 1))) << 4)) = ux;
-    *reinterpret_cast<uint4*>(row + (((NCH / 2 + (EC / 8) * g + c) ^ (rr & (NCH - 1))) << 4)) = uy;
+    const int kx = (EC / 8) * g + c, ky = HD / 16 + kx;   // 16-byte chunk indices of the row
+    *reinterpret_cast<uint4*>(row + (kx >> 3) * 16384 + (((kx & 7) ^ (rr & 7)) << 4)) = ux;
+    *reinterpret_cast<uint4*>(row + (ky >> 3) * 16384 + (((ky & 7) ^ (rr & 7)) << 4)) = uy;
   }
 }
-// n_tiles staged bf16 tiles (128 rows each, 128 * 2 HD bytes apart) -> rows [0, n_valid) of dst[t] (row stride ld):
-// HD / 8 lanes per row, 256 / HD rows per store instruction
+// n_tiles staged bf16 matrices (128 rows each, 128 * 2 HD bytes apart, atom layout above) -> rows [0, n_valid) of
+// dst[t] (row stride ld): HD / 8 lanes per row, 256 / HD rows per store instruction
 template <int HD>
 __device__ __forceinline__ void stage16_store(const uint8_t* stg, int n_tiles, int w8, int lane, int n_valid,
                                               bf16* dst0, bf16* dst1, int ld) {
-  constexpr int NCH = HD / 8, RPI = 32 / NCH, ROWB = HD * 2;
+  constexpr int NCH = HD / 8, RPI = 32 / NCH, MATB = 128 * HD * 2;
   const int k = lane % NCH;
 #pragma unroll 4
   for (int i = 0; i < 128 * n_tiles / (RPI * EW_WARPS); ++i) {
     const int R = i * (RPI * EW_WARPS) + w8 * RPI + lane / NCH, t = R >> 7, rr = R & 127;
     if (rr >= n_valid) continue;
-    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * 128 * ROWB + rr * ROWB + ((k ^ (rr & (NCH - 1))) << 4));
+    const uint4 v = *reinterpret_cast<const uint4*>(stg + t * MATB + (k >> 3) * 16384 + rr * 128 +
+                                                    (((k & 7) ^ (rr & 7)) << 4));
     *reinterpret_cast<uint4*>((t ? dst1 : dst0) + (size_t)rr * ld + k * 8) = v;
   }
 }
+// one staged matrix (HD / 64 atoms) -> 128 rows of dqkv from (row, col) by TMA store; called by one thread after the
+// staging writes, fence.proxy.async and a barrier
+template <int HD>
+__device__ __forceinline__ void stage_tma_store(const CUtensorMap* m, const uint8_t* stg, int row, int col) {
+#pragma unroll
+  for (int a = 0; a < HD / 64; ++a) tma_store_2d(m, stg + a * 16384, col + 64 * a, row);
+}
 
+// Work-item geometry, pipelined so that no role stalls on global loads at an item boundary: the items entry of
+// item + 2G is loaded at the top of item, the sequence's cu_seqlens / pos_shift entries of item + G (whose items entry
+// arrived one item earlier) too, and both are consumed one item later.
+struct ItemPipe {
+  int4 raw;         // items[i + 2G] (x = -1: past the end)
+  int4 cur;         // items[i + G]
+  int c0, c1, sh;   // cu_seqlens[cur.x], cu_seqlens[cur.x + 1], pos_shift[cur.x]
+};
+__device__ __forceinline__ int4 item_at(const int4* items, int n, int i) {
+  return i < n ? items[i] : make_int4(-1, 0, 0, 0);
+}
+__device__ __forceinline__ void ip_fetch(ItemPipe& q, const int* cu, const int* ps) {
+  q.c0 = 0; q.c1 = 0; q.sh = 0;
+  if (q.cur.x >= 0) { q.c0 = cu[q.cur.x]; q.c1 = cu[q.cur.x + 1]; q.sh = ps ? ps[q.cur.x] : 0; }
+}
 struct Geo { int base, L, blk0, head, n, sh; };   // sh: RoPE position shift of the sequence (prefix rows)
 
 // -DMENOS_BWS_PROF: per-phase clock64 accounting (dK/dV kernel: one elementwise thread and the MMA lane)
@@ -148,6 +200,35 @@ __device__ unsigned long long g_bws_prof[16];
 #define BP_FLUSH(cond) do {} while (0)
 #endif
 
+// P = exp2(S c - lse) (every fourth on the FMA pipe), dS = P (dP - D) scale for the thread's CPT columns; MASK: the
+// causal / sequence-end mask (columns outside [cmin, cmax) are 0) -- interior blocks take the unmasked instance
+template <bool MASK>
+__device__ __forceinline__ void pds_math(const uint32_t (&su)[CPT], const uint32_t (&du)[CPT], const float* lse_s,
+                                         const float* d_s, float sl2, float scale, int cmin, int cmax,
+                                         float (&pv)[CPT], float (&dsv)[CPT]) {
+#pragma unroll
+  for (int c4 = 0; c4 < CPT; c4 += 4) {
+    const float4 lz = *reinterpret_cast<const float4*>(lse_s + c4);
+    const float4 dz = *reinterpret_cast<const float4*>(d_s + c4);
+    const float lzv[4] = {lz.x, lz.y, lz.z, lz.w}, dzv[4] = {dz.x, dz.y, dz.z, dz.w};
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int c = c4 + u;
+      const float x = fmaf(__uint_as_float(su[c]), sl2, -lzv[u]);
+      const float e = u == 3 ? poly_exp2(x) : fast_exp2(x);
+      const float ds = e * fmaf(__uint_as_float(du[c]), scale, -dzv[u]);
+      if (MASK) {
+        const bool ok = c >= cmin && c < cmax;
+        pv[c] = ok ? e : 0.f;
+        dsv[c] = ok ? ds : 0.f;
+      } else {
+        pv[c] = e;
+        dsv[c] = ds;
+      }
+    }
+  }
+}
+
 // ======================================================================================= dK / dV
 constexpr int KV_ROWS = 128, QB = 64;
 constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
@@ -161,7 +242,8 @@ template <int HD> struct DkdvGeo {
 template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
-                        const __grid_constant__ CUtensorMap tmDO64, const BwParams p) {
+                        const __grid_constant__ CUtensorMap tmDO64, const __grid_constant__ CUtensorMap tmOut,
+                        const BwParams p) {
   constexpr int KV_TILE = DkdvGeo<HD>::KV_TILE, QB_TILE = DkdvGeo<HD>::QB_TILE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -193,25 +275,31 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   const uint32_t tmem = tmem_sh;
   const uint32_t tdV = tmem + 256, tdK = tmem + 384;   // S^T buffers at 0/64, dP^T at 128/192
 
-  auto load_geo = [&](int item) {
-    Geo g{0, 0, 0, 0, 0, 0};
-    if (item < p.n_items) {
-      const int4 it = p.items[item];
-      g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
-      g.sh = p.pos_shift ? p.pos_shift[it.x] : 0;
-      g.n = rep * ((g.L - g.blk0 + QB - 1) / QB);      // (head of the group, 64-query block) pairs
-    }
+  auto ip_init = [&](ItemPipe& q) {
+    q.cur = item_at(p.items, p.n_items, blockIdx.x);
+    ip_fetch(q, p.cu_seqlens, p.pos_shift);
+    q.raw = item_at(p.items, p.n_items, blockIdx.x + gridDim.x);
+  };
+  auto ip_advance = [&](ItemPipe& q, int item) {   // at the top of `item`: q moves on to item + G
+    q.cur = q.raw;
+    ip_fetch(q, p.cu_seqlens, p.pos_shift);
+    q.raw = item_at(p.items, p.n_items, item + 2 * gridDim.x);
+  };
+  auto decode = [&](const ItemPipe& q) {
+    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh};
+    g.n = rep * ((g.L - g.blk0 + QB - 1) / QB);      // (head of the group, 64-query block) pairs; 0 past the end
     return g;
   };
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
     if (elect_one()) {
-      Geo nx = load_geo(blockIdx.x);
+      ItemPipe ip;
+      ip_init(ip);
       int it = 0, gb = 0;
       for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-        const Geo G = nx;
-        nx = load_geo(item + gridDim.x);
+        const Geo G = decode(ip);
+        ip_advance(ip, item);
         const int k0 = G.blk0, hk = G.head, nqb = (G.L - k0 + QB - 1) / QB;
         const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
         wait_bar(&kv_empty, (it & 1) ^ 1);
@@ -241,12 +329,13 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     // ------------------------------------------------ MMA issuer
     constexpr uint32_t ID_S = umma_idesc_bf16(128, QB, 0);     // [128 kv] x [64 q], K = hd
     constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 kv] x [hd], K = 64 q, B MN-major
-    Geo nx = load_geo(blockIdx.x);
+    ItemPipe ip;
+    ip_init(ip);
     BP_DECL
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-      const Geo G = nx;
-      nx = load_geo(item + gridDim.x);
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
       auto issue_acc = [&](int gp, int jp) {  // dV += P^T dO ; dK += dS^T Q   for global block gp (item block jp)
         const int bp = gp & 1, sp = gp % STAGES;
         BP(10);
@@ -257,8 +346,18 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         tc_fence_after();
         __syncwarp();
         if (elect_one()) {
-          const uint32_t pa = smem_u32(sP0 + bp * PT_TILE), sa = smem_u32(sS0 + bp * PT_TILE);
           const uint32_t ob = smem_u32(sO0 + sp * QB_TILE), qb = smem_u32(sQ0 + sp * QB_TILE);
+#if MENOS_BWS_TMEM_P
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {   // A = P^T / dS^T packed in the S^T / dP^T tiles of buffer bp
+            const uint32_t acc = (jp > 0 || kk > 0) ? 1u : 0u;
+            tc_mma_bf16_ts(tdV, tmem + 64 * bp + packed_col(kk), umma_desc_sw128(ob + kk * 2048, 8192, 1024), ID_ACC, acc);
+            tc_mma_bf16_ts(tdK, tmem + 128 + 64 * bp + packed_col(kk), umma_desc_sw128(qb + kk * 2048, 8192, 1024), ID_ACC,
+                           acc);
+          }
+          tc_commit(&empty[sp]);     // Q/dO stage free
+#else
+          const uint32_t pa = smem_u32(sP0 + bp * PT_TILE), sa = smem_u32(sS0 + bp * PT_TILE);
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk) {
             const uint32_t acc = (jp > 0 || kk > 0) ? 1u : 0u;
@@ -267,11 +366,14 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
           }
           tc_commit(&empty[sp]);     // Q/dO stage free
           tc_commit(&pd_free[bp]);   // P^T/dS^T buffer free
+#endif
         }
         __syncwarp();
         BP(13);
       };
+      BP(10);
       wait_bar(&kv_full, it & 1);
+      BP(15);
       tc_fence_after();
       for (int j = 0; j < G.n; ++j, ++gb) {
         const int b = gb & 1, st = gb % STAGES;
@@ -309,7 +411,8 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     const int r = w4 * 32 + lane;           // key row within the block
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_W;
-    Geo nx = load_geo(blockIdx.x);
+    ItemPipe ip;
+    ip_init(ip);
     BP_DECL
     // lse (t < 64) or D (64 <= t < 128) of query t & 63 of (item G, block j); 0 outside the sequence / list
     auto lse_d_load = [&](const Geo& G, int j) -> float {
@@ -318,21 +421,38 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       const int h = G.head * rep + j / nqb, qpos = G.blk0 + (j % nqb) * QB + (t & (QB - 1));
       return qpos < G.L ? __ldg((t < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos) : 0.f;
     };
-    float pre = 0.f;
+    // the stager threads' lse / D values run two blocks ahead of their use (the loads' latency -- L2 or HBM -- then
+    // hides behind two blocks of work): v_cur for this block, v_nxt for the next; a value whose block lies beyond the
+    // next item (items of one block) is loaded when it becomes the next one (nxt_ok = false)
+    float v_cur = 0.f, v_nxt = 0.f;
+    bool cur_ok = false, nxt_ok = false;
+    bool tma_pending = false;   // this thread (t == 0) has TMA stores reading the staging buffers
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-      const Geo G = nx;
-      nx = load_geo(item + gridDim.x);
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
       const int k0 = G.blk0, L = G.L, base = G.base, nqb = (L - k0 + QB - 1) / QB;
       const int kpos = k0 + r;
-      if (it == 0) pre = lse_d_load(G, 0);
       for (int j = 0; j < G.n; ++j, ++gb) {
         const int b = gb & 1;
         const int q0 = k0 + (j % nqb) * QB;
-        if (t < 2 * QB) {  // stage lse (log2 domain) and D of the block's 64 queries (loaded one block ahead)
+        if (t < 2 * QB) {  // stage lse (log2 domain) and D of the block's 64 queries
           const int c = t & (QB - 1);
-          if (t < QB) s_lse[b][c] = pre * LOG2E_W; else s_D[b][c] = pre * p.scale;   // D pre-scaled
-          pre = j + 1 < G.n ? lse_d_load(G, j + 1) : lse_d_load(nx, 0);
+          if (!cur_ok) v_cur = lse_d_load(G, j);
+          if (t < QB) s_lse[b][c] = v_cur * LOG2E_W; else s_D[b][c] = v_cur * p.scale;   // D pre-scaled
+          BP(9);
+          v_cur = v_nxt; cur_ok = nxt_ok;
+          if (!cur_ok) {   // the next block's value was not issued two blocks ago: issue it now
+            v_cur = j + 1 < G.n ? lse_d_load(G, j + 1) : lse_d_load(decode(ip), 0);
+            cur_ok = true;
+          }
+          nxt_ok = true;
+          if (j + 2 < G.n) {
+            v_nxt = lse_d_load(G, j + 2);
+          } else {
+            const Geo N = decode(ip);
+            if (j + 2 - G.n < N.n) v_nxt = lse_d_load(N, j + 2 - G.n); else nxt_ok = false;
+          }
         }
         BP(0);
         ew_sync();
@@ -347,56 +467,80 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         tmem_wait_ld();
         const int cmin = kpos - q0 - CPT * g;   // P = 0 for queries before the key (causal) ...
         const int cmax = L - q0 - CPT * g;      // ... and past the end of the sequence
-        const bool full = cmin <= 0 && cmax >= CPT;   // interior block: no mask in this row's columns
         float pv[CPT], dsv[CPT];
-#pragma unroll
-        for (int c4 = 0; c4 < CPT; c4 += 4) {
-          const float4 lz = *reinterpret_cast<const float4*>(&s_lse[b][CPT * g + c4]);
-          const float4 dz = *reinterpret_cast<const float4*>(&s_D[b][CPT * g + c4]);
-          const float lzv[4] = {lz.x, lz.y, lz.z, lz.w}, dzv[4] = {dz.x, dz.y, dz.z, dz.w};
-#pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const int c = c4 + u;
-            const bool ok = full || (c >= cmin && c < cmax);
-            const float x = fmaf(__uint_as_float(su[c]), sl2, -lzv[u]);
-            const float e = u == 3 ? poly_exp2(x) : fast_exp2(x);
-            pv[c] = ok ? e : 0.f;
-            dsv[c] = ok ? e * fmaf(__uint_as_float(du[c]), p.scale, -dzv[u]) : 0.f;
-          }
-        }
+        if (cmin <= 0 && cmax >= CPT)   // interior: no mask in this row's columns
+          pds_math<false>(su, du, &s_lse[b][CPT * g], &s_D[b][CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
+        else
+          pds_math<true>(su, du, &s_lse[b][CPT * g], &s_D[b][CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
         BP(3);
+#if MENOS_BWS_TMEM_P
+        {   // P^T, dS^T -> the first 16 of the 32 S^T / dP^T columns this thread group read
+          uint32_t up[CPT / 2], ud[CPT / 2];
+          pack_row(pv, up);
+          pack_row(dsv, ud);
+          tmem_st16_nw(tmem + 64 * b + 32 * g + lane_off, up);
+          tmem_st16_nw(tmem + 128 + 64 * b + 32 * g + lane_off, ud);
+          tmem_wait_st();
+        }
+        BP(4);
+#else
         if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
+        if (j == 0 && tma_pending) {   // the previous item's dK / dV TMA stores have read the staging buffers
+          if (t == 0) bulk_wait_read0();
+          ew_sync();
+          tma_pending = false;
+        }
         BP(4);
         st_half_row(sP0 + b * PT_TILE, r, g, pv);
         st_half_row(sS0 + b * PT_TILE, r, g, dsv);
         fence_proxy_async();
+#endif
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&ew_done[b]);
         BP(5);
       }
       // ------------------------------------------------ epilogue: dK (RoPE bwd), dV rows -> dqkv
+      const int nv = min(KV_ROWS, L - k0);
+      const bool rope = p.rope_cs != nullptr && r < nv;
+      RopeCS<HD> csk;
+      rope_cs_load<HD>(csk, p.rope_cs, max(0, k0 + r - G.sh), g, rope);   // in flight during the wait below
       BP(0);
       wait_bar(&acc_full, it & 1);
       BP(6);
       tc_fence_after();
+#if MENOS_BWS_TMEM_P
+      if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's TMA stores have read the staging
+      tma_pending = false;
+#endif
       ew_sync();   // order every warp's last P^T / dS^T stores before the staging writes (the mbarrier chain through
                    // the MMAs already does; the named barrier makes it visible to compute-sanitizer racecheck)
-      // all MMAs of this item completed: P^T / dS^T buffers are free for staging
-      const int nv = min(KV_ROWS, L - k0);
-      bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
-      // P^T / dS^T buffers (64 KB, contiguous) = bf16 staging of dK | dV
-      acc_row_to_bf16<HD>(tdK + lane_off, sP0, r, g, p.rope_cs, max(0, k0 + r - G.sh), p.rope_cs != nullptr && r < nv);
-      acc_row_to_bf16<HD>(tdV + lane_off, sP0 + 128 * HD * 2, r, g, nullptr, 0, false);
+      // all MMAs of this item completed: P^T / dS^T buffers (64 KB, contiguous) = bf16 staging of dK | dV
+      acc_row_to_bf16<HD>(tdK + lane_off, sP0, r, g, csk, rope);
+      acc_row_to_bf16<HD>(tdV + lane_off, sP0 + 128 * HD * 2, r, g, csk, false);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_free);   // the next item's dK / dV accumulation may start
       BP(7);
-      ew_sync();
-      stage16_store<HD>(sP0, 2, w8, lane, nv, dst + (p.H + G.head) * HD, dst + (p.H + p.Hkv + G.head) * HD, p.ld_dqkv);
-      ew_sync();
+      if (nv == KV_ROWS) {   // full block: TMA stores, the warps go on with the next item
+        fence_proxy_async();
+        ew_sync();
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sP0, base + k0, (p.H + G.head) * HD);
+          stage_tma_store<HD>(&tmOut, sP0 + 128 * HD * 2, base + k0, (p.H + p.Hkv + G.head) * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+      } else {               // the sequence's ragged last block: row-masked stores
+        bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
+        ew_sync();
+        stage16_store<HD>(sP0, 2, w8, lane, nv, dst + (p.H + G.head) * HD, dst + (p.H + p.Hkv + G.head) * HD,
+                          p.ld_dqkv);
+        ew_sync();
+      }
       BP(8);
     }
+    if (t == 0) bulk_wait0();
     BP_FLUSH(blockIdx.x < 8 && t == 0);
   }
   tc_fence_before();
@@ -420,7 +564,8 @@ template <int HD> struct DqGeo {
 template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
-                      const __grid_constant__ CUtensorMap tmDO128, const BwParams p) {
+                      const __grid_constant__ CUtensorMap tmDO128, const __grid_constant__ CUtensorMap tmOut,
+                      const BwParams p) {
   constexpr int Q_TILE = DqGeo<HD>::Q_TILE, KB_TILE = DqGeo<HD>::KB_TILE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -449,24 +594,30 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   const uint32_t tmem = tmem_sh;
   const uint32_t tdQ = tmem + 256;   // S buffers at 0/64, dP at 128/192
 
-  auto load_geo = [&](int item) {
-    Geo g{0, 0, 0, 0, 0, 0};
-    if (item < p.n_items) {
-      const int4 it = p.items[item];
-      g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.blk0 = it.y; g.head = it.z;
-      g.sh = p.pos_shift ? p.pos_shift[it.x] : 0;
-      g.n = (min(g.L, g.blk0 + Q_ROWS) + KB - 1) / KB;
-    }
+  auto ip_init = [&](ItemPipe& q) {
+    q.cur = item_at(p.items, p.n_items, blockIdx.x);
+    ip_fetch(q, p.cu_seqlens, p.pos_shift);
+    q.raw = item_at(p.items, p.n_items, blockIdx.x + gridDim.x);
+  };
+  auto ip_advance = [&](ItemPipe& q, int item) {
+    q.cur = q.raw;
+    ip_fetch(q, p.cu_seqlens, p.pos_shift);
+    q.raw = item_at(p.items, p.n_items, item + 2 * gridDim.x);
+  };
+  auto decode = [&](const ItemPipe& q) {
+    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh};
+    g.n = (min(g.L, g.blk0 + Q_ROWS) + KB - 1) / KB;   // 0 past the end
     return g;
   };
 
   if (warp == 0) {
     if (elect_one()) {
-      Geo nx = load_geo(blockIdx.x);
+      ItemPipe ip;
+      ip_init(ip);
       int it = 0, gb = 0;
       for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-        const Geo G = nx;
-        nx = load_geo(item + gridDim.x);
+        const Geo G = decode(ip);
+        ip_advance(ip, item);
         const int h = G.head, hk = h / (p.H / p.Hkv), q0 = G.blk0;
         const int kcol = (p.H + hk) * HD, vcol = (p.H + p.Hkv + hk) * HD;
         wait_bar(&q_empty, (it & 1) ^ 1);
@@ -494,11 +645,12 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   } else if (warp == 1) {
     constexpr uint32_t ID_S = umma_idesc_bf16(128, KB, 0);     // [128 q] x [64 keys], K = hd
     constexpr uint32_t ID_ACC = umma_idesc_bf16(128, HD, 1);   // [128 q] x [hd], K = 64 keys, B MN-major
-    Geo nx = load_geo(blockIdx.x);
+    ItemPipe ip;
+    ip_init(ip);
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-      const Geo G = nx;
-      nx = load_geo(item + gridDim.x);
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
       auto issue_acc = [&](int gp, int jp) {  // dQ += dS K
         const int bp = gp & 1, sp = gp % STAGES;
         wait_bar(&ew_done[bp], (gp >> 1) & 1);
@@ -506,13 +658,22 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         tc_fence_after();
         __syncwarp();
         if (elect_one()) {
-          const uint32_t sa = smem_u32(sS0 + bp * DS_TILE), kb_ = smem_u32(sK0 + sp * KB_TILE);
+          const uint32_t kb_ = smem_u32(sK0 + sp * KB_TILE);
+#if MENOS_BWS_TMEM_P
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)   // A = dS packed in the S tile of buffer bp
+            tc_mma_bf16_ts(tdQ, tmem + 64 * bp + packed_col(kk), umma_desc_sw128(kb_ + kk * 2048, 8192, 1024), ID_ACC,
+                           (jp > 0 || kk > 0) ? 1u : 0u);
+          tc_commit(&empty[sp]);
+#else
+          const uint32_t sa = smem_u32(sS0 + bp * DS_TILE);
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk)
             tc_mma_bf16(tdQ, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(kb_ + kk * 2048, 8192, 1024), ID_ACC,
                         (jp > 0 || kk > 0) ? 1u : 0u);
           tc_commit(&empty[sp]);
           tc_commit(&pd_free[bp]);
+#endif
         }
         __syncwarp();
       };
@@ -544,20 +705,30 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       __syncwarp();
     }
   } else {
-    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2;   // warp group g owns key columns [CPT g, CPT g + CPT)
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;   // warp group g owns key columns [CPT g, CPT g + CPT)
     const int r = w4 * 32 + lane;           // query row
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     const float sl2 = p.scale * LOG2E_W;
-    Geo nx = load_geo(blockIdx.x);
+    ItemPipe ip;
+    ip_init(ip);
+    // lse (log2 domain) and pre-scaled D of this thread's query row in item G; loaded one item ahead
+    auto row_stats = [&](const Geo& G, float& l2, float& dq) {
+      const int qpos = G.blk0 + r;
+      const bool ok = G.n > 0 && qpos < G.L;
+      l2 = ok ? __ldg(p.lse + (size_t)G.head * p.T + G.base + qpos) : 0.f;
+      dq = ok ? __ldg(p.D + (size_t)G.head * p.T + G.base + qpos) : 0.f;
+    };
+    float lse_n = 0.f, D_n = 0.f;
+    bool tma_pending = false;
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
-      const Geo G = nx;
-      nx = load_geo(item + gridDim.x);
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
       const int h = G.head, q0 = G.blk0, L = G.L, base = G.base;
       const int qpos = q0 + r;
       const bool qok = qpos < L;
-      const float lse2 = qok ? p.lse[(size_t)h * p.T + base + qpos] * LOG2E_W : 0.f;
-      const float Dq = qok ? p.D[(size_t)h * p.T + base + qpos] * p.scale : 0.f;   // pre-scaled
+      if (it == 0) row_stats(G, lse_n, D_n);
+      const float lse2 = lse_n * LOG2E_W, Dq = D_n * p.scale;   // Dq pre-scaled
       for (int j = 0; j < G.n; ++j, ++gb) {
         const int b = gb & 1;
         wait_bar(&s_full[b], (gb >> 1) & 1);
@@ -569,34 +740,76 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         tmem_wait_ld();
         const int cmax = qok ? qpos - j * KB - CPT * g : -1;   // keys <= query
         float dsv[CPT];
+        if (cmax >= CPT - 1) {   // no masked column in this row
 #pragma unroll
-        for (int c = 0; c < CPT; ++c) {
-          const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
-          const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
-          const float v = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
-          dsv[c] = (cmax >= CPT - 1 || c <= cmax) ? v : 0.f;
+          for (int c = 0; c < CPT; ++c) {
+            const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+            const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
+            dsv[c] = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+            const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
+            const float v = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
+            dsv[c] = c <= cmax ? v : 0.f;
+          }
         }
+        if (j == 0) row_stats(decode(ip), lse_n, D_n);   // next item's row statistics (its geometry has arrived)
+#if MENOS_BWS_TMEM_P
+        {   // dS -> the first 16 of the 32 S columns this thread group read
+          uint32_t ud[CPT / 2];
+          pack_row(dsv, ud);
+          tmem_st16_nw(tmem + 64 * b + 32 * g + lane_off, ud);
+          tmem_wait_st();
+        }
+#else
         if (gb >= 2) wait_bar(&pd_free[b], ((gb - 2) >> 1) & 1);
+        if (j == 0 && tma_pending) {   // the previous item's dQ TMA store has read the staging buffers
+          if (t == 0) bulk_wait_read0();
+          ew_sync();
+          tma_pending = false;
+        }
         st_half_row(sS0 + b * DS_TILE, r, g, dsv);
         fence_proxy_async();
+#endif
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&ew_done[b]);
       }
+      const int nv = min(Q_ROWS, L - q0);
+      const bool rope = p.rope_cs != nullptr && r < nv;
+      RopeCS<HD> csq;
+      rope_cs_load<HD>(csq, p.rope_cs, max(0, q0 + r - G.sh), g, rope);   // in flight during the wait below
       wait_bar(&acc_full, it & 1);
       tc_fence_after();
+#if MENOS_BWS_TMEM_P
+      if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's TMA store has read the staging
+      tma_pending = false;
+#endif
       ew_sync();   // as in the dK / dV epilogue: the dS^T stores of every warp precede the staging writes
-      const int nv = min(Q_ROWS, L - q0);
       // dS buffers (32 KB) = bf16 staging of dQ
-      acc_row_to_bf16<HD>(tdQ + lane_off, sS0, r, g, p.rope_cs, max(0, q0 + r - G.sh), p.rope_cs != nullptr && r < nv);
+      acc_row_to_bf16<HD>(tdQ + lane_off, sS0, r, g, csq, rope);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_free);
-      ew_sync();
-      bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
-      stage16_store<HD>(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
-      ew_sync();
+      if (nv == Q_ROWS) {
+        fence_proxy_async();
+        ew_sync();
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sS0, base + q0, h * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+      } else {
+        ew_sync();
+        bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
+        stage16_store<HD>(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
+        ew_sync();
+      }
     }
+    if (t == 0) bulk_wait0();
   }
   tc_fence_before();
   __syncthreads();
@@ -622,8 +835,9 @@ int attn_bws_prof_read(unsigned long long* out) {
 template <int HD>
 static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
                          int num_sms, cudaStream_t st) {
-  CUtensorMap mQKV128, mQKV64, mDO64, mDO128;
+  CUtensorMap mQKV128, mQKV64, mDO64, mDO128, mOut;
   if (!tma_map_2d(&mQKV128, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 128)) return -2;
+  if (!tma_map_2d(&mOut, a.dqkv, a.T, (a.H + 2 * a.Hkv) * HD, a.ld_dqkv, 64, 128)) return -2;   // dK / dV / dQ stores
   if (!tma_map_2d(&mQKV64, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 64)) return -2;
   if (!tma_map_2d(&mDO64, a.dO, a.T, a.H * HD, a.ld_do, 64, 64)) return -2;
   if (!tma_map_2d(&mDO128, a.dO, a.T, a.H * HD, a.ld_do, 64, 128)) return -2;
@@ -639,11 +853,13 @@ static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv
   }
   p.items = items_kv; p.n_items = n_items_kv;
   if (n_items_kv > 0)
-    attn_bwd_dkdv_ws_kernel<HD><<<min(n_items_kv, num_sms), NTHREADS, DkdvGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO64, p);
+    attn_bwd_dkdv_ws_kernel<HD><<<min(n_items_kv, num_sms), NTHREADS, DkdvGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO64,
+                                                                                                mOut, p);
   ++g_launch_count;
   p.items = items_q; p.n_items = n_items_q;
   if (n_items_q > 0)
-    attn_bwd_dq_ws_kernel<HD><<<min(n_items_q, num_sms), NTHREADS, DqGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO128, p);
+    attn_bwd_dq_ws_kernel<HD><<<min(n_items_q, num_sms), NTHREADS, DqGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO128,
+                                                                                            mOut, p);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }

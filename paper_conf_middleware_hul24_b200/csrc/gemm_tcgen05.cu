@@ -21,6 +21,7 @@
 //   M-tiles so a wave's A rows and B panels stay L2-resident.
 #include <mutex>
 #include <unordered_map>
+#include <cstdlib>
 #include <cstring>
 #include "common.cuh"
 #include "kernels.h"
@@ -35,7 +36,7 @@ constexpr int BM = 128, BN = 256, BK = 64;
 constexpr int EPW = MENOS_GEMM_EPW;           // epilogue warps (4 or 8): 1 or 2 per TMEM lane quadrant
 constexpr int NTHREADS = 64 + 32 * EPW;
 constexpr int EPC = 8 / (EPW / 4);            // 32-column chunks of a 256-column tile per epilogue warp
-constexpr int GROUP_M = 16;
+constexpr int GROUP_M = 16;   // default rasterisation group; MENOS_GEMM_GROUP_M overrides (tuning)
 
 template <int CG> struct Cfg {
   static constexpr int A_STAGE = BM * BK * 2;                 // 16 KB (this CTA's 128 rows)
@@ -63,6 +64,7 @@ struct KParams {
   const float2* rope_cs;
   const int* pos;
   int head_dim, rope_cols;
+  int group_m;             // rasterisation group (m-tiles per group)
 };
 
 #ifndef MENOS_GEMM_EPI_PREFETCH
@@ -138,11 +140,11 @@ __device__ __forceinline__ void rope_small(const float (&v)[32], float (&o)[32],
 __device__ __forceinline__ float sigmoidf_(float x) { return 1.0f / (1.0f + __expf(-x)); }
 
 // grouped rasterisation: groups of GROUP_M m-tiles; inside a group m runs fastest
-__device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int& m, int& n) {
-  const int per_group = GROUP_M * num_n;
+__device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int group_m, int& m, int& n) {
+  const int per_group = group_m * num_n;
   const int g = t / per_group;
-  const int first = g * GROUP_M;
-  const int gs = min(num_m - first, GROUP_M);
+  const int first = g * group_m;
+  const int gs = min(num_m - first, group_m);
   const int tin = t - g * per_group;
   m = first + tin % gs;
   n = tin / gs;
@@ -205,7 +207,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       int stage = 0; uint32_t phase = 0;
       for (int t = cluster_id; t < total; t += n_clusters) {
         int m, n, col0, n16;
-        tile_coords(t, num_m, num_n, m, n);
+        tile_coords(t, num_m, num_n, p.group_m, m, n);
         tile_extra<CG>(p, m, n, col0, n16);
         const int nkb = p.kb_main + (n16 + 3) / 4;
         const int arow = m * C::TILE_M + rank * BM;
@@ -261,7 +263,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       int acc = 0; uint32_t acc_phase = 0;
       for (int t = cluster_id; t < total; t += n_clusters) {
         int m, n, col0, n16;
-        tile_coords(t, num_m, num_n, m, n);
+        tile_coords(t, num_m, num_n, p.group_m, m, n);
         tile_extra<CG>(p, m, n, col0, n16);
         const int nkb = p.kb_main + (n16 + 3) / 4;
         mbar_wait(&tempty_bar[acc], acc_phase ^ 1);
@@ -308,7 +310,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     int acc = 0; uint32_t acc_phase = 0;
     for (int t = cluster_id; t < total; t += n_clusters) {
       int m, n;
-      tile_coords(t, num_m, num_n, m, n);
+      tile_coords(t, num_m, num_n, p.group_m, m, n);
       {
         // L2 prefetch of the epilogue's HBM inputs for this row while the tile's MMAs still run: residual (fp32,
         // 8 x 128 B lines), saved g|u (SwiGLU bwd: 2 x 4 x 128 B) or relu output (4 x 128 B)
@@ -698,6 +700,8 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   p.out2 = a.out2; p.ldo2 = a.ldo2; p.aux = a.aux; p.ldaux = a.ldaux; p.bias = a.bias;
   p.dsum = a.dsum; p.dsum_ld = a.dsum_ld; p.dsum_hd = a.dsum_hd;
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
+  static const int group_env = [] { const char* e = getenv("MENOS_GEMM_GROUP_M"); return e ? atoi(e) : 0; }();
+  p.group_m = group_env > 0 ? group_env : GROUP_M;
   const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);
   int sms = a.num_sms > 0 ? a.num_sms : 148;
   int clusters = sms / CG;

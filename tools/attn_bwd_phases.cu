@@ -38,7 +38,7 @@ int main() {
   float ms; cudaEventElapsedTime(&ms, e0, e1);
   attn_bws_prof_read(pr);
   printf("err %s  %.1f us per dkdv+dq launch pair\n", cudaGetErrorString(cudaGetLastError()), ms * 100.f);
-  const char* nm[16] = {"ew lse stage/loop", "ew ew_sync", "ew wait S", "ew tmem+math", "ew wait pd_free", "ew store P/dS+arrive", "ew epi wait acc", "ew epi tmem->stage", "ew epi copy-out", "-", "mma loop", "mma wait ew_done", "mma wait acc_free", "mma issue acc", "mma wait Q/dO", "-"};
+  const char* nm[16] = {"ew lse stage/loop", "ew ew_sync", "ew wait S", "ew tmem+math", "ew pack+TMEM st (or pd_free wait)", "ew arrive (or smem P/dS store)", "ew epi wait acc", "ew epi tmem->stage", "ew epi copy-out", "ew lse: value wait+store", "mma loop", "mma wait ew_done", "mma wait acc_free", "mma issue acc", "mma wait Q/dO", "mma wait K/V (item start)"};
   unsigned long long te = 0, tm = 0;
   for (int k = 0; k < 10; ++k) te += pr[k];
   for (int k = 10; k < 16; ++k) tm += pr[k];
