@@ -27,7 +27,7 @@ namespace {
 #endif
 // EW_WARPS elementwise warps: EW_WARPS / 4 per TMEM lane quadrant, each thread owning CPT of a block's 64 columns
 constexpr int STAGES = 3, EW_WARPS = MENOS_BWS_EW, NTHREADS = 64 + 32 * EW_WARPS;
-constexpr int CPT = 64 / (EW_WARPS / 4);
+constexpr int NGRP = EW_WARPS / 4, CPT = 64 / NGRP;   // column groups per lane quadrant, columns per thread
 static_assert(CPT == 16 || CPT == 32, "EW_WARPS must be 8 or 16");
 constexpr float LOG2E_W = 1.4426950408889634f;
 // MENOS_BWS_TMEM_P (default 1): the elementwise warps write P^T / dS^T (dK/dV kernel) and dS (dQ kernel) as packed
@@ -37,12 +37,27 @@ constexpr float LOG2E_W = 1.4426950408889634f;
 #ifndef MENOS_BWS_TMEM_P
 #define MENOS_BWS_TMEM_P 1
 #endif
-#if MENOS_BWS_TMEM_P
-static_assert(CPT == 32, "the packed TMEM operand layout assumes two 32-column thread groups (8 elementwise warps)");
+// MENOS_BWS_ALT (default 1, needs MENOS_BWS_TMEM_P and 8 elementwise warps): the elementwise warps form two groups of
+// four (one warp per TMEM lane quadrant) that take ALTERNATE blocks -- group = block parity = its S / dP buffer -- and a
+// thread owns all 64 columns of its row in its group's blocks (two halves of 32).  The SM's TMEM read port moves
+// 64 B / cycle, so a block's S + dP (64 KB) takes ~1000 cycles to read: with both groups on the same block every warp
+// waits for the port, then every warp computes; alternating, one group's loads overlap the other group's arithmetic.
+// The dK / dV epilogue stages dK, then dV, through one 32 KB buffer (frees 32 KB of shared memory for the lse / D ring).
+#ifndef MENOS_BWS_ALT
+#define MENOS_BWS_ALT MENOS_BWS_TMEM_P
+#endif
+#if MENOS_BWS_ALT
+static_assert(MENOS_BWS_TMEM_P && EW_WARPS == 8, "MENOS_BWS_ALT needs the TMEM operand path and 8 elementwise warps");
 #endif
 // TMEM column (relative to the tile) of K-chunk kk (16 queries / keys) of a packed operand: thread group g wrote its
-// 32 columns' values into the first 16 of the 32 columns it had read (columns [32 g, 32 g + 16))
-__device__ __forceinline__ uint32_t packed_col(int kk) { return (uint32_t)((kk & 1) * 8 + (kk >> 1) * 32); }
+// CPT columns' values into the first CPT / 2 of the CPT columns it had read (columns [CPT g, CPT g + CPT / 2))
+__device__ __forceinline__ uint32_t packed_col(int kk) {
+  return (uint32_t)((kk * 16 / CPT) * CPT + (kk * 16 % CPT) / 2);
+}
+template <int N>
+__device__ __forceinline__ void tmem_st_half(uint32_t taddr, const uint32_t (&u)[N]) {
+  if constexpr (N == 16) tmem_st16_nw(taddr, u); else tmem_st8_nw(taddr, u);
+}
 // pack CPT fp32 values into CPT / 2 bf16x2 words (even column in the low half)
 __device__ __forceinline__ void pack_row(const float (&v)[CPT], uint32_t (&u)[CPT / 2]) {
 #pragma unroll
@@ -76,6 +91,10 @@ template <int N>
 __device__ __forceinline__ void tmem_ldc_nw(uint32_t taddr, uint32_t (&r)[N]) {
   if constexpr (N == 32) {
     tmem_ld32_nw(taddr, r);
+  } else if constexpr (N == 8) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr));
   } else {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
@@ -107,18 +126,20 @@ __device__ __forceinline__ void st_half_row(uint8_t* tile, int row, int g, const
 // warps go on with the next item); a sequence's ragged last block by row-masked 16-byte stores (stage16_store).
 // Same fp32 ops in the same order as before: the bf16 result is bitwise identical.
 template <int HD>
-struct RopeCS { float4 v[HD / 8]; };   // (c_2i, s_2i, c_2i+1, s_2i+1) for the thread's HD/4 pairs
+struct RopeCS { float4 v[HD / (4 * NGRP)]; };   // (c_2i, s_2i, c_2i+1, s_2i+1) for the thread's HD / (2 NGRP) pairs
 template <int HD>
 __device__ __forceinline__ void rope_cs_load(RopeCS<HD>& c, const float2* cs, int pos, int g, bool rope) {
   if (!rope) return;
-  const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + (HD / 4) * g);
+  const float4* c4 = reinterpret_cast<const float4*>(cs + (size_t)pos * (HD / 2) + (HD / (2 * NGRP)) * g);
 #pragma unroll
-  for (int i = 0; i < HD / 8; ++i) c.v[i] = __ldg(c4 + i);
+  for (int i = 0; i < HD / (4 * NGRP); ++i) c.v[i] = __ldg(c4 + i);
 }
+// the thread's accumulator row chunk -> bf16 (RoPE backward applied when rope): x half (columns < HD/2) in ux, y in uy
 template <int HD>
-__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const RopeCS<HD>& cs,
-                                                bool rope) {
-  constexpr int EC = HD / 4;   // columns per group per half
+struct RowPack { uint4 x[HD / (16 * NGRP)], y[HD / (16 * NGRP)]; };
+template <int HD>
+__device__ __forceinline__ void acc_row_pack(uint32_t tacc, int g, const RopeCS<HD>& cs, bool rope, RowPack<HD>& o) {
+  constexpr int EC = HD / (2 * NGRP);   // columns per group per half
   uint32_t a[EC], b[EC];
   tmem_ldc_nw(tacc + EC * g, a);
   tmem_ldc_nw(tacc + HD / 2 + EC * g, b);
@@ -135,17 +156,31 @@ __device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int
       x[2 * i] = x0; y[2 * i] = y0; x[2 * i + 1] = x1; y[2 * i + 1] = y1;
     }
   }
+#pragma unroll
+  for (int c = 0; c < EC / 8; ++c) {
+    o.x[c] = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
+                        pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
+    o.y[c] = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
+                        pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
+  }
+}
+template <int HD>
+__device__ __forceinline__ void stage_row(uint8_t* stg, int rr, int g, const RowPack<HD>& o) {
+  constexpr int EC = HD / (2 * NGRP);
   uint8_t* row = stg + rr * 128;
 #pragma unroll
   for (int c = 0; c < EC / 8; ++c) {
-    const uint4 ux = make_uint4(pack_bf16x2(x[8 * c], x[8 * c + 1]), pack_bf16x2(x[8 * c + 2], x[8 * c + 3]),
-                                pack_bf16x2(x[8 * c + 4], x[8 * c + 5]), pack_bf16x2(x[8 * c + 6], x[8 * c + 7]));
-    const uint4 uy = make_uint4(pack_bf16x2(y[8 * c], y[8 * c + 1]), pack_bf16x2(y[8 * c + 2], y[8 * c + 3]),
-                                pack_bf16x2(y[8 * c + 4], y[8 * c + 5]), pack_bf16x2(y[8 * c + 6], y[8 * c + 7]));
     const int kx = (EC / 8) * g + c, ky = HD / 16 + kx;   // 16-byte chunk indices of the row
-    *reinterpret_cast<uint4*>(row + (kx >> 3) * 16384 + (((kx & 7) ^ (rr & 7)) << 4)) = ux;
-    *reinterpret_cast<uint4*>(row + (ky >> 3) * 16384 + (((ky & 7) ^ (rr & 7)) << 4)) = uy;
+    *reinterpret_cast<uint4*>(row + (kx >> 3) * 16384 + (((kx & 7) ^ (rr & 7)) << 4)) = o.x[c];
+    *reinterpret_cast<uint4*>(row + (ky >> 3) * 16384 + (((ky & 7) ^ (rr & 7)) << 4)) = o.y[c];
   }
+}
+template <int HD>
+__device__ __forceinline__ void acc_row_to_bf16(uint32_t tacc, uint8_t* stg, int rr, int g, const RopeCS<HD>& cs,
+                                                bool rope) {
+  RowPack<HD> o;
+  acc_row_pack<HD>(tacc, g, cs, rope, o);
+  stage_row<HD>(stg, rr, g, o);
 }
 // n_tiles staged bf16 matrices (128 rows each, 128 * 2 HD bytes apart, atom layout above) -> rows [0, n_valid) of
 // dst[t] (row stride ld): HD / 8 lanes per row, 256 / HD rows per store instruction
@@ -236,7 +271,7 @@ constexpr int KVA = KV_ROWS * 128, QBA = QB * 128;   // one SW128 atom (64 colum
 template <int HD> struct DkdvGeo {
   static constexpr int KV_TILE = KV_ROWS * HD * 2;   // HD 128: 32 KB (2 atoms [128][64]); 64: 16 KB
   static constexpr int QB_TILE = QB * HD * 2;        // 16 KB (2 atoms [64][64]); 8 KB
-  static constexpr int SMEM = 2 * KV_TILE + 2 * STAGES * QB_TILE + 4 * PT_TILE + 1024;
+  static constexpr int SMEM = 2 * KV_TILE + 2 * STAGES * QB_TILE + (MENOS_BWS_ALT ? 2 : 4) * PT_TILE + 1024;
 };
 
 template <int HD>
@@ -256,7 +291,14 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   __shared__ __align__(8) uint64_t kv_full, kv_empty, full[STAGES], empty[STAGES], s_full[2], ew_done[2], pd_free[2];
   __shared__ __align__(8) uint64_t acc_full, acc_free;
   __shared__ uint32_t tmem_sh;
-  __shared__ __align__(16) float s_lse[2][QB], s_D[2][QB];
+#if MENOS_BWS_ALT
+  // lse (log2 domain) | D (pre-scaled) of a block's 64 queries, per warp group a ring of 2 filled by cp.async one
+  // group block (two blocks) ahead
+  __shared__ __align__(16) float s_ld[2][2][2 * QB];
+#else
+  // lse (log2 domain) | D (pre-scaled) of a block's 64 queries, ring of 3 blocks filled by cp.async two blocks ahead
+  __shared__ __align__(16) float s_ld[3][2 * QB];
+#endif
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rep = p.H / p.Hkv;
@@ -264,7 +306,9 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO64);
     mbar_init(&kv_full, 1); mbar_init(&kv_empty, 1);
     for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], MENOS_BWS_ALT ? EW_WARPS / 2 : EW_WARPS); mbar_init(&pd_free[i], 1);
+    }
     mbar_init(&acc_full, 1); mbar_init(&acc_free, EW_WARPS);
     fence_barrier_init();
   }
@@ -405,6 +449,138 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     BP(10);
     BP_FLUSH(blockIdx.x < 8 && lane == 0);
   } else {
+#if MENOS_BWS_ALT
+    // ------------------------------------------------ elementwise warps: group gr = w8 / 4 takes the blocks of parity
+    //                                                  gr; thread = key row = TMEM lane, all 64 query columns
+    const int w4 = warp & 3, w8 = warp - 2, gr = w8 >> 2, t = threadIdx.x - 64, tt = t & 127;
+    const int r = w4 * 32 + lane;           // key row within the block
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
+    const float sl2 = p.scale * LOG2E_W;
+    ItemPipe ip;
+    ip_init(ip);
+    BP_DECL
+    auto gsync = [&]() {   // the group's four warps
+      if (gr == 0) asm volatile("bar.sync 2, 128;" ::: "memory"); else asm volatile("bar.sync 3, 128;" ::: "memory");
+    };
+    // lse (tt < 64) / D (64 <= tt < 128) of query tt & 63 of block jj of G -> s_ld[gr][slot][tt] by cp.async (0 outside)
+    auto issue = [&](int slot, const Geo& G, int jj) {
+      const float* src = p.lse;
+      int sz = 0;
+      if (jj < G.n) {
+        const int nqb = (G.L - G.blk0 + QB - 1) / QB;
+        const int h = G.head * rep + jj / nqb, qpos = G.blk0 + (jj % nqb) * QB + (tt & (QB - 1));
+        if (qpos < G.L) { src = (tt < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos; sz = 4; }
+      }
+      cp_async4(smem_u32(&s_ld[gr][slot][tt]), src, sz);
+    };
+    bool have_cur = false;      // this block's copy was issued one group block ago
+    bool tma_pending = false;   // this thread (t == 0) has TMA stores reading the staging buffer
+    int it = 0, gb = 0, kb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
+      const int k0 = G.blk0, L = G.L, base = G.base, nqb = (L - k0 + QB - 1) / QB;
+      const int kpos = k0 + r;
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        if ((gb & 1) != gr) continue;
+        const int q0 = k0 + (j % nqb) * QB, sl = kb & 1;
+        if (!have_cur) { issue(sl, G, j); cp_async_commit(); }
+        cp_async_wait<0>();
+        s_ld[gr][sl][tt] *= tt < QB ? LOG2E_W : p.scale;   // lse to the log2 domain, D pre-scaled
+        BP(9);
+        gsync();
+        BP(1);
+        {   // the group's next block (gb + 2): its copy now, when its item is known (else at its turn)
+          const Geo N = j + 2 >= G.n ? decode(ip) : G;
+          have_cur = true;
+          if (j + 2 < G.n) issue(sl ^ 1, G, j + 2);
+          else if (j + 2 - G.n < N.n) issue(sl ^ 1, N, j + 2 - G.n);
+          else have_cur = false;
+          cp_async_commit();
+        }
+        BP(0);
+        wait_bar(&s_full[gr], (gb >> 1) & 1);
+        BP(2);
+        tc_fence_after();
+        __syncwarp();
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {   // query columns [32 hf, 32 hf + 32)
+          uint32_t su[CPT], du[CPT];
+          tmem_ldc_nw(tmem + 64 * gr + 32 * hf + lane_off, su);
+          tmem_ldc_nw(tmem + 128 + 64 * gr + 32 * hf + lane_off, du);
+          tmem_wait_ld();
+          const int cmin = kpos - q0 - 32 * hf;   // P = 0 for queries before the key (causal) ...
+          const int cmax = L - q0 - 32 * hf;      // ... and past the end of the sequence
+          float pv[CPT], dsv[CPT];
+          if (cmin <= 0 && cmax >= CPT)
+            pds_math<false>(su, du, &s_ld[gr][sl][32 * hf], &s_ld[gr][sl][QB + 32 * hf], sl2, p.scale, cmin, cmax, pv,
+                            dsv);
+          else
+            pds_math<true>(su, du, &s_ld[gr][sl][32 * hf], &s_ld[gr][sl][QB + 32 * hf], sl2, p.scale, cmin, cmax, pv,
+                           dsv);
+          uint32_t up[CPT / 2], ud[CPT / 2];
+          pack_row(pv, up);
+          pack_row(dsv, ud);
+          tmem_st_half(tmem + 64 * gr + 32 * hf + lane_off, up);
+          tmem_st_half(tmem + 128 + 64 * gr + 32 * hf + lane_off, ud);
+        }
+        BP(3);
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ew_done[gr]);
+        ++kb;
+        BP(5);
+      }
+      // ------------------------------------------------ epilogue: dK (RoPE bwd), then dV, through one 32 KB staging
+      const int nv = min(KV_ROWS, L - k0);
+      const bool rope = p.rope_cs != nullptr && r < nv, full = nv == KV_ROWS;
+      RopeCS<HD> csk;
+      rope_cs_load<HD>(csk, p.rope_cs, max(0, k0 + r - G.sh), gr, rope);   // in flight during the wait below
+      BP(0);
+      wait_bar(&acc_full, it & 1);
+      BP(6);
+      tc_fence_after();
+      if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's dV store has read the staging
+      tma_pending = false;
+      ew_sync();
+      bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
+      acc_row_to_bf16<HD>(tdK + lane_off, sP0, r, gr, csk, rope);
+      RowPack<HD> vpk;
+      acc_row_pack<HD>(tdV + lane_off, gr, csk, false, vpk);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free);   // the next item's dK / dV accumulation may start
+      BP(7);
+      if (full) fence_proxy_async();
+      ew_sync();
+      if (full) {
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sP0, base + k0, (p.H + G.head) * HD);
+          bulk_commit();
+          bulk_wait_read0();
+        }
+      } else {
+        stage16_store<HD>(sP0, 1, w8, lane, nv, dst + (p.H + G.head) * HD, dst, p.ld_dqkv);
+      }
+      ew_sync();
+      stage_row<HD>(sP0, r, gr, vpk);
+      if (full) {
+        fence_proxy_async();
+        ew_sync();
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sP0, base + k0, (p.H + p.Hkv + G.head) * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+      } else {
+        ew_sync();
+        stage16_store<HD>(sP0, 1, w8, lane, nv, dst + (p.H + p.Hkv + G.head) * HD, dst, p.ld_dqkv);
+        ew_sync();
+      }
+      BP(8);
+    }
+#else
     // ------------------------------------------------ elementwise warps (thread = key row = TMEM lane;
     //                                                  warp group g owns query columns [CPT g, CPT g + CPT))
     const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
@@ -414,18 +590,21 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     ItemPipe ip;
     ip_init(ip);
     BP_DECL
-    // lse (t < 64) or D (64 <= t < 128) of query t & 63 of (item G, block j); 0 outside the sequence / list
-    auto lse_d_load = [&](const Geo& G, int j) -> float {
-      if (t >= 2 * QB || G.n == 0) return 0.f;
-      const int nqb = (G.L - G.blk0 + QB - 1) / QB;
-      const int h = G.head * rep + j / nqb, qpos = G.blk0 + (j % nqb) * QB + (t & (QB - 1));
-      return qpos < G.L ? __ldg((t < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos) : 0.f;
+    // the stager threads' (t < 128) lse / D values arrive by 4-byte cp.async two blocks ahead of their use (ring
+    // s_ld[gb % 3]; issued after block gb's barrier, when every thread is done with block gb - 1's slot), so their
+    // latency (L2 or HBM) hides behind two blocks of work without a register dependency; a value whose block lies
+    // beyond the next item (items of one block) is issued one block ahead instead
+    auto issue = [&](int slot, const Geo& G, int jj) {
+      const float* src = p.lse;
+      int sz = 0;
+      if (jj < G.n) {
+        const int nqb = (G.L - G.blk0 + QB - 1) / QB;
+        const int h = G.head * rep + jj / nqb, qpos = G.blk0 + (jj % nqb) * QB + (t & (QB - 1));
+        if (qpos < G.L) { src = (t < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos; sz = 4; }
+      }
+      cp_async4(smem_u32(&s_ld[slot][t]), src, sz);
     };
-    // the stager threads' lse / D values run two blocks ahead of their use (the loads' latency -- L2 or HBM -- then
-    // hides behind two blocks of work): v_cur for this block, v_nxt for the next; a value whose block lies beyond the
-    // next item (items of one block) is loaded when it becomes the next one (nxt_ok = false)
-    float v_cur = 0.f, v_nxt = 0.f;
-    bool cur_ok = false, nxt_ok = false;
+    bool nxt_issued = false, cur_wait0 = true;
     bool tma_pending = false;   // this thread (t == 0) has TMA stores reading the staging buffers
     int it = 0, gb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
@@ -434,29 +613,30 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       const int k0 = G.blk0, L = G.L, base = G.base, nqb = (L - k0 + QB - 1) / QB;
       const int kpos = k0 + r;
       for (int j = 0; j < G.n; ++j, ++gb) {
-        const int b = gb & 1;
+        const int b = gb & 1, sl = gb % 3;
         const int q0 = k0 + (j % nqb) * QB;
-        if (t < 2 * QB) {  // stage lse (log2 domain) and D of the block's 64 queries
-          const int c = t & (QB - 1);
-          if (!cur_ok) v_cur = lse_d_load(G, j);
-          if (t < QB) s_lse[b][c] = v_cur * LOG2E_W; else s_D[b][c] = v_cur * p.scale;   // D pre-scaled
+        if (t < 2 * QB) {   // this block's value: wait for its copy, scale in place
+          if (gb == 0) { issue(0, G, 0); cp_async_commit(); }
+          if (cur_wait0) cp_async_wait<0>(); else cp_async_wait<1>();
+          s_ld[sl][t] *= t < QB ? LOG2E_W : p.scale;   // lse to the log2 domain, D pre-scaled
           BP(9);
-          v_cur = v_nxt; cur_ok = nxt_ok;
-          if (!cur_ok) {   // the next block's value was not issued two blocks ago: issue it now
-            v_cur = j + 1 < G.n ? lse_d_load(G, j + 1) : lse_d_load(decode(ip), 0);
-            cur_ok = true;
-          }
-          nxt_ok = true;
-          if (j + 2 < G.n) {
-            v_nxt = lse_d_load(G, j + 2);
-          } else {
-            const Geo N = decode(ip);
-            if (j + 2 - G.n < N.n) v_nxt = lse_d_load(N, j + 2 - G.n); else nxt_ok = false;
-          }
         }
         BP(0);
         ew_sync();
         BP(1);
+        if (t < 2 * QB) {   // copies of block gb + 1 (if not issued a block ago) and gb + 2 (if its item is known)
+          const Geo N = j + 2 >= G.n ? decode(ip) : G;
+          const bool late = !nxt_issued;
+          if (late) {
+            if (j + 1 < G.n) issue((gb + 1) % 3, G, j + 1); else issue((gb + 1) % 3, N, j + 1 - G.n);
+          }
+          nxt_issued = true;
+          if (j + 2 < G.n) issue((gb + 2) % 3, G, j + 2);
+          else if (j + 2 - G.n < N.n) issue((gb + 2) % 3, N, j + 2 - G.n);
+          else nxt_issued = false;
+          cp_async_commit();
+          cur_wait0 = late;
+        }
         wait_bar(&s_full[b], (gb >> 1) & 1);
         BP(2);
         tc_fence_after();
@@ -469,17 +649,17 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         const int cmax = L - q0 - CPT * g;      // ... and past the end of the sequence
         float pv[CPT], dsv[CPT];
         if (cmin <= 0 && cmax >= CPT)   // interior: no mask in this row's columns
-          pds_math<false>(su, du, &s_lse[b][CPT * g], &s_D[b][CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
+          pds_math<false>(su, du, &s_ld[sl][CPT * g], &s_ld[sl][QB + CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
         else
-          pds_math<true>(su, du, &s_lse[b][CPT * g], &s_D[b][CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
+          pds_math<true>(su, du, &s_ld[sl][CPT * g], &s_ld[sl][QB + CPT * g], sl2, p.scale, cmin, cmax, pv, dsv);
         BP(3);
 #if MENOS_BWS_TMEM_P
         {   // P^T, dS^T -> the first 16 of the 32 S^T / dP^T columns this thread group read
           uint32_t up[CPT / 2], ud[CPT / 2];
           pack_row(pv, up);
           pack_row(dsv, ud);
-          tmem_st16_nw(tmem + 64 * b + 32 * g + lane_off, up);
-          tmem_st16_nw(tmem + 128 + 64 * b + 32 * g + lane_off, ud);
+          tmem_st_half(tmem + 64 * b + CPT * g + lane_off, up);
+          tmem_st_half(tmem + 128 + 64 * b + CPT * g + lane_off, ud);
           tmem_wait_st();
         }
         BP(4);
@@ -540,6 +720,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       }
       BP(8);
     }
+#endif
     if (t == 0) bulk_wait0();
     BP_FLUSH(blockIdx.x < 8 && t == 0);
   }
@@ -583,7 +764,9 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     tma_prefetch(&tmQKV128); tma_prefetch(&tmQKV64); tma_prefetch(&tmDO128);
     mbar_init(&q_full, 1); mbar_init(&q_empty, 1);
     for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], EW_WARPS); mbar_init(&pd_free[i], 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&s_full[i], 1); mbar_init(&ew_done[i], MENOS_BWS_ALT ? EW_WARPS / 2 : EW_WARPS); mbar_init(&pd_free[i], 1);
+    }
     mbar_init(&acc_full, 1); mbar_init(&acc_free, EW_WARPS);
     fence_barrier_init();
   }
@@ -705,6 +888,103 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
       __syncwarp();
     }
   } else {
+#if MENOS_BWS_ALT
+    // group gr = w8 / 4 takes the key blocks of parity gr (its S / dP buffer); thread = query row, all 64 key columns
+    const int w4 = warp & 3, w8 = warp - 2, gr = w8 >> 2, t = threadIdx.x - 64;
+    const int r = w4 * 32 + lane;           // query row
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
+    const float sl2 = p.scale * LOG2E_W;
+    ItemPipe ip;
+    ip_init(ip);
+    // lse (log2 domain) and pre-scaled D of this thread's query row in item G; loaded one item ahead
+    auto row_stats = [&](const Geo& G, float& l2, float& dq) {
+      const int qpos = G.blk0 + r;
+      const bool ok = G.n > 0 && qpos < G.L;
+      l2 = ok ? __ldg(p.lse + (size_t)G.head * p.T + G.base + qpos) : 0.f;
+      dq = ok ? __ldg(p.D + (size_t)G.head * p.T + G.base + qpos) : 0.f;
+    };
+    float lse_n = 0.f, D_n = 0.f;
+    bool tma_pending = false;
+    int it = 0, gb = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const Geo G = decode(ip);
+      ip_advance(ip, item);
+      const int h = G.head, q0 = G.blk0, L = G.L, base = G.base;
+      const int qpos = q0 + r;
+      const bool qok = qpos < L;
+      if (it == 0) row_stats(G, lse_n, D_n);
+      const float lse2 = lse_n * LOG2E_W, Dq = D_n * p.scale;   // Dq pre-scaled
+      bool stats_next = false;
+      for (int j = 0; j < G.n; ++j, ++gb) {
+        if ((gb & 1) != gr) continue;
+        wait_bar(&s_full[gr], (gb >> 1) & 1);
+        tc_fence_after();
+        __syncwarp();
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {   // key columns [32 hf, 32 hf + 32)
+          uint32_t su[CPT], du[CPT];
+          tmem_ldc_nw(tmem + 64 * gr + 32 * hf + lane_off, su);
+          tmem_ldc_nw(tmem + 128 + 64 * gr + 32 * hf + lane_off, du);
+          tmem_wait_ld();
+          const int cmax = qok ? qpos - j * KB - 32 * hf : -1;   // keys <= query
+          float dsv[CPT];
+          if (cmax >= CPT - 1) {   // no masked column
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) {
+              const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+              const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
+              dsv[c] = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
+            }
+          } else {
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) {
+              const float x = fmaf(__uint_as_float(su[c]), sl2, -lse2);
+              const float e = (c & 3) == 3 ? poly_exp2(x) : fast_exp2(x);
+              const float v = e * fmaf(__uint_as_float(du[c]), p.scale, -Dq);
+              dsv[c] = c <= cmax ? v : 0.f;
+            }
+          }
+          uint32_t ud[CPT / 2];
+          pack_row(dsv, ud);
+          tmem_st_half(tmem + 64 * gr + 32 * hf + lane_off, ud);
+        }
+        if (!stats_next) { row_stats(decode(ip), lse_n, D_n); stats_next = true; }   // next item's (geometry arrived)
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ew_done[gr]);
+      }
+      if (!stats_next) row_stats(decode(ip), lse_n, D_n);   // this group had no block in the item
+      const int nv = min(Q_ROWS, L - q0);
+      const bool rope = p.rope_cs != nullptr && r < nv;
+      RopeCS<HD> csq;
+      rope_cs_load<HD>(csq, p.rope_cs, max(0, q0 + r - G.sh), gr, rope);   // in flight during the wait below
+      wait_bar(&acc_full, it & 1);
+      tc_fence_after();
+      if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's TMA store has read the staging
+      tma_pending = false;
+      ew_sync();
+      // dS buffers (32 KB) = bf16 staging of dQ
+      acc_row_to_bf16<HD>(tdQ + lane_off, sS0, r, gr, csq, rope);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free);
+      if (nv == Q_ROWS) {
+        fence_proxy_async();
+        ew_sync();
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sS0, base + q0, h * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+      } else {
+        ew_sync();
+        bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
+        stage16_store<HD>(sS0, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
+        ew_sync();
+      }
+    }
+#else
     const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;   // warp group g owns key columns [CPT g, CPT g + CPT)
     const int r = w4 * 32 + lane;           // query row
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
@@ -761,7 +1041,7 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         {   // dS -> the first 16 of the 32 S columns this thread group read
           uint32_t ud[CPT / 2];
           pack_row(dsv, ud);
-          tmem_st16_nw(tmem + 64 * b + 32 * g + lane_off, ud);
+          tmem_st_half(tmem + 64 * b + CPT * g + lane_off, ud);
           tmem_wait_st();
         }
 #else
@@ -809,6 +1089,7 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
         ew_sync();
       }
     }
+#endif
     if (t == 0) bulk_wait0();
   }
   tc_fence_before();
