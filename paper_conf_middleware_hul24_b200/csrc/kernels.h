@@ -67,15 +67,37 @@ struct LoraRowsProblem {
 };
 // token reduction: C[m, n] = scale * sum_t P[t, map(m)] * Q[t, n]   (fp32 out, overwrite)
 //   map(m) = (m / p_blk) * p_blk_stride + m % p_blk   (gate/up interleaved 128-blocks)
+//   output rows may be split in segments (one client's q|k|v or gate|up dA in one pass over X): row m goes to
+//   segment m / m_seg (C, C1, C2) at row m % m_seg, and only rows with m % m_seg < m_valid are written
+//   (m_seg <= 0: one segment; m_valid <= 0: every row)
 struct LoraTokRedProblem {
   const bf16* P; const bf16* Q; float* C;
   int M, N, T, ldp, ldq, ldc, p_blk, p_blk_stride;
+  float scale;
+  float* C1; float* C2;
+  int m_seg, m_valid;
+};
+// fused dU + dB of one (client, target) in ONE pass over its dY columns:
+//   dB[m, n]  = sum_t dY[t, map(m)] U[t, n]                                  (fp32 [Nt, rank], overwrite)
+//   W[s][t,n] = sum_{m in slab s} dY[t, map(m)] B[map(m), n]                 (fp32 partials, [n_slabs][T][rank])
+//   dU[t, n]  = bf16(scale * sum_s W[s][t, n])  for n < rank, 0 for rank <= n < rs   (second, tiny kernel)
+// U = the saved s * X A^T of the target, B = its Bcat rows (indexed like dY's columns), map as above.
+struct LoraDUBProblem {
+  const bf16* dY; const bf16* U; const bf16* B;
+  float* dB; float* W; bf16* dU;
+  int Nt, rank, rs, T, ldy, ldu, ldb, lddu, p_blk, p_blk_stride, n_slabs;
   float scale;
 };
 int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st);
 int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st);
 void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out);
 void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out);
+// dU/dB slab width (dY columns per CTA) used for n_slabs
+constexpr int LORA_DUB_MT = 128;
+// grid: (max n_slabs * ceil(max rank / 16), n_probs); CTAs past a problem's slabs exit
+int lora_dub_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, int max_rank, cudaStream_t st);
+// grid: (ceil(max T * rs / 256), n_probs)
+int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max_elems, cudaStream_t st);
 
 // ---------------------------------------------------------------- norms / elementwise
 // residual streams (x, h forward; dy, dh backward) are fp32; GEMM operands (xn, hn, dxn ...) are bf16

@@ -35,14 +35,18 @@ __device__ __forceinline__ int tsw(int row, int chunk) {
 // ROWS_BM tokens per CTA, one warp per 16 of them.  64 (default) vs 32 measured at cfg1 shapes
 // (profiles/r1n_lora_rows_bm.txt): 32-token blocks double the CTAs but each CTA still re-stages the whole
 // [N, K] adapter operand from L2, so the shrink is no faster and the per-target dU is 38% slower.
-constexpr int ROWS_BM = MENOS_LORA_ROWS_BM, ROWS_BK = 128, ROWS_STAGES = 4, ROWS_NTH = ROWS_BM / 16 * 32;
+// Stages: as many 128-wide K tiles as ~196 KB of shared memory holds (one CTA per SM): the shrink has one CTA per
+// 64 tokens (128 CTAs at cfg1), so the bytes each SM keeps in flight set its HBM rate (4 stages: 1.9 TB/s, r2bb)
+constexpr int ROWS_BM = MENOS_LORA_ROWS_BM, ROWS_BK = 128, ROWS_NTH = ROWS_BM / 16 * 32;
 template <int NT>
-constexpr int rows_smem_bytes() { return ROWS_STAGES * (ROWS_BM + NT) * ROWS_BK * 2; }
+__host__ __device__ constexpr int rows_stages() { return NT <= 32 ? 8 : NT <= 64 ? 6 : 4; }
+template <int NT>
+constexpr int rows_smem_bytes() { return rows_stages<NT>() * (ROWS_BM + NT) * ROWS_BK * 2; }
 
 template <int NT>
 __global__ void __launch_bounds__(ROWS_NTH) lora_rows_kernel(const LoraRowsProblem* __restrict__ probs,
                                                         const int2* __restrict__ tiles) {
-  constexpr int BM = ROWS_BM, BK = ROWS_BK, NNT = NT / 8, NS = ROWS_STAGES;
+  constexpr int BM = ROWS_BM, BK = ROWS_BK, NNT = NT / 8, NS = rows_stages<NT>();
   extern __shared__ __align__(128) uint8_t rows_smem[];
   bf16* As_base = reinterpret_cast<bf16*>(rows_smem);                 // [NS][BM * BK]
   bf16* Bs_base = As_base + NS * BM * BK;                             // [NS][NT * BK]  ("nk": [NT][BK]; "kn": [BK][NT])
@@ -230,9 +234,182 @@ __global__ void __launch_bounds__(128) lora_tokred_kernel(const LoraTokRedProble
         const int r = m0 + wm0 + i * 16 + g + h * 8;
         const int c = n0 + wn0 + j * 8 + 2 * t;
         if (r >= P.M) continue;
-        if (c < P.N) P.C[(size_t)r * P.ldc + c] = acc[i][j][2 * h] * P.scale;
-        if (c + 1 < P.N) P.C[(size_t)r * P.ldc + c + 1] = acc[i][j][2 * h + 1] * P.scale;
+        const int seg = P.m_seg > 0 ? r / P.m_seg : 0, mr = P.m_seg > 0 ? r % P.m_seg : r;
+        if (P.m_valid > 0 && mr >= P.m_valid) continue;
+        float* C = seg == 0 ? P.C : seg == 1 ? P.C1 : P.C2;
+        if (c < P.N) C[(size_t)mr * P.ldc + c] = acc[i][j][2 * h] * P.scale;
+        if (c + 1 < P.N) C[(size_t)mr * P.ldc + c + 1] = acc[i][j][2 * h + 1] * P.scale;
       }
+}
+
+// ============================================================================ fused dU + dB kernel
+// CTA = (problem, slab of MT dY columns, 16-wide rank tile); streams the client's T tokens once in 64-token stages
+// (4-stage cp.async ring of the [64, MT] dY tile and the [64, 16] U tile).  Per stage:
+//   dB[slab, n]  += dY_tile^T U_tile     (accumulated in registers over all tokens; one fixed order)
+//   W[slab][t, n] = dY_tile B_slab       (this slab's share of dU for the stage's tokens, written once)
+// Replaces the two passes (dU rows kernel + dB token reduction) that each read dY from HBM.
+constexpr int DUB_BK = 64, DUB_STAGES = 4, DUB_NT = 16;
+template <int MT>
+constexpr int dub_smem_bytes() { return DUB_STAGES * DUB_BK * (MT + DUB_NT) * 2 + MT * DUB_NT * 2; }
+
+// NJ: n8 tiles of the 16-wide rank tile that carry data (1 when rank <= 8: half the MMAs, which the kernel needs --
+// at r = 8 it does 8 MACs per dY byte on mma.sync)
+template <int MT, int NJ>
+__global__ void __launch_bounds__(128) lora_dub_kernel(const LoraDUBProblem* __restrict__ probs, int n_rt) {
+  constexpr int BK = DUB_BK, NS = DUB_STAGES, NT = DUB_NT;
+  constexpr int WM = MT / 4, NMI = WM / 16;   // dB: each warp owns WM of the slab's columns
+  constexpr int CPR = MT / 8;                 // 16-byte chunks per dY row of a stage
+  static_assert(128 % CPR == 0, "one fixed chunk column per thread");
+  extern __shared__ __align__(128) uint8_t dub_smem[];
+  bf16* Ps_base = reinterpret_cast<bf16*>(dub_smem);   // [NS][BK * MT]  ([token][m])
+  bf16* Us_base = Ps_base + NS * BK * MT;              // [NS][BK * NT]  ([token][n])
+  bf16* Bs = Us_base + NS * BK * NT;                   // [MT * NT]      ([m][n])
+  const LoraDUBProblem P = probs[blockIdx.y];
+  const int slab = blockIdx.x / n_rt, n0 = (blockIdx.x % n_rt) * NT;
+  if (slab >= P.n_slabs || n0 >= P.rank) return;
+  const int m0 = slab * MT;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
+  // the slab's dY columns are contiguous (p_blk is a multiple of MT, host-checked)
+  const int pcol0 = (m0 / P.p_blk) * P.p_blk_stride + m0 % P.p_blk;
+
+  // this slab's B rows (indexed like dY's columns), once
+  for (int i = tid; i < MT * (NT / 8); i += 128) {
+    const int r = i / (NT / 8), c = i % (NT / 8);
+    const bool ok = m0 + r < P.Nt && n0 + c * 8 < P.rs;
+    cp_async16(smem_u32(&Bs[tsw<NT>(r, c)]), P.B + (ok ? (size_t)(pcol0 + r) * P.ldb + n0 + c * 8 : 0), ok ? 16 : 0);
+  }
+  // per-thread fixed dY chunk column, rows r0 + (128 / CPR) k
+  const int yc = tid % CPR, yr0 = tid / CPR;
+  const bool ycol_ok = m0 + yc * 8 < P.Nt;
+  const bf16* ysrc = P.dY + pcol0 + yc * 8;
+  const int uc = tid & 1, ur0 = tid >> 1;   // U: 2 chunks per row (NT = 16)
+  const bool ucol_ok = n0 + uc * 8 < P.rank;
+  const bf16* usrc = P.U + n0 + uc * 8;
+  auto load = [&](int buf, int t0) {
+    bf16* Ps = Ps_base + buf * BK * MT;
+    bf16* Us = Us_base + buf * BK * NT;
+#pragma unroll
+    for (int r = yr0; r < BK; r += 128 / CPR) {
+      const int tok = t0 + r;
+      const bool ok = ycol_ok && tok < P.T;
+      cp_async16(smem_u32(&Ps[tsw<MT>(r, yc)]), ok ? ysrc + (size_t)tok * P.ldy : P.dY, ok ? 16 : 0);
+    }
+    if (ur0 < BK) {
+      const int tok = t0 + ur0;
+      const bool ok = ucol_ok && tok < P.T;
+      cp_async16(smem_u32(&Us[tsw<NT>(ur0, uc)]), ok ? usrc + (size_t)tok * P.ldu : P.U, ok ? 16 : 0);
+    }
+  };
+
+  float accb[NMI][NJ][4];
+#pragma unroll
+  for (int i = 0; i < NMI; ++i)
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) accb[i][j][0] = accb[i][j][1] = accb[i][j][2] = accb[i][j][3] = 0.f;
+  const int nk = (P.T + BK - 1) / BK;
+#pragma unroll
+  for (int s = 0; s < NS - 1; ++s) {
+    if (s < nk) load(s, s * BK);
+    cp_async_commit();   // the first group also carries the B slab
+  }
+  const int mat = lane >> 3, rr = lane & 7;
+  float* const Wb = P.W + (size_t)slab * P.T * P.rank;
+  for (int kb = 0; kb < nk; ++kb) {
+    cp_async_wait<NS - 2>();
+    __syncthreads();
+    {
+      const int nx = kb + NS - 1;
+      if (nx < nk) load(nx % NS, nx * BK);
+      cp_async_commit();
+    }
+    const bf16* p_s = Ps_base + (kb % NS) * BK * MT;
+    const bf16* u_s = Us_base + (kb % NS) * BK * NT;
+    // dB: A(m, k=token) = dY^T via transposed ldmatrix, B(k=token, n) = U
+#pragma unroll
+    for (int kk = 0; kk < BK; kk += 16) {
+      uint32_t a[NMI][4];
+#pragma unroll
+      for (int i = 0; i < NMI; ++i) {
+        const int row = kk + (mat >> 1) * 8 + rr, col = warp * WM + i * 16 + (mat & 1) * 8;
+        ldsm_x4_t(smem_u32(p_s + tsw<MT>(row, col >> 3)), a[i][0], a[i][1], a[i][2], a[i][3]);
+      }
+      uint32_t b[4];
+      {
+        const int row = kk + (mat & 1) * 8 + rr, col = (mat >> 1) * 8;
+        ldsm_x4_t(smem_u32(u_s + tsw<NT>(row, col >> 3)), b[0], b[1], b[2], b[3]);
+      }
+#pragma unroll
+      for (int i = 0; i < NMI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) mma_bf16_16816(accb[i][j], a[i], b[2 * j], b[2 * j + 1]);
+    }
+    // dU share: warp w takes the stage's tokens 16w..16w+15, reduction over the slab's MT columns (two independent
+    // accumulator chains when NJ = 1, summed at the end in a fixed order)
+    {
+      float accu[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+      for (int kk = 0; kk < MT; kk += 16) {
+        uint32_t a[4], b[4];
+        {
+          const int row = warp * 16 + (mat & 1) * 8 + rr, col = kk + (mat >> 1) * 8;
+          ldsm_x4(smem_u32(p_s + tsw<MT>(row, col >> 3)), a[0], a[1], a[2], a[3]);
+        }
+        {
+          const int row = kk + (mat & 1) * 8 + rr, col = (mat >> 1) * 8;
+          ldsm_x4_t(smem_u32(Bs + tsw<NT>(row, col >> 3)), b[0], b[1], b[2], b[3]);
+        }
+        if (NJ == 2) {
+          mma_bf16_16816(accu[0], a, b[0], b[1]);
+          mma_bf16_16816(accu[1], a, b[2], b[3]);
+        } else {
+          mma_bf16_16816(accu[(kk >> 4) & 1], a, b[0], b[1]);
+        }
+      }
+      if (NJ == 1)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) accu[0][e] += accu[1][e];
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int tok = kb * BK + warp * 16 + g + h * 8;
+          const int n = n0 + j * 8 + 2 * t;
+          if (tok >= P.T) continue;
+          float* w = Wb + (size_t)tok * P.rank + n;
+          if (n < P.rank) w[0] = accu[j][2 * h];
+          if (n + 1 < P.rank) w[1] = accu[j][2 * h + 1];
+        }
+    }
+  }
+  cp_async_wait<0>();
+#pragma unroll
+  for (int i = 0; i < NMI; ++i)
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int m = m0 + warp * WM + i * 16 + g + h * 8;
+        const int n = n0 + j * 8 + 2 * t;
+        if (m >= P.Nt) continue;
+        float* d = P.dB + (size_t)m * P.rank + n;
+        if (n < P.rank) d[0] = accb[i][j][2 * h];
+        if (n + 1 < P.rank) d[1] = accb[i][j][2 * h + 1];
+      }
+}
+
+// dU[t, n] = bf16(scale * sum over slabs, in slab order, of W[s][t, n]); zero in the slot's padding columns
+__global__ void __launch_bounds__(256) lora_du_reduce_kernel(const LoraDUBProblem* __restrict__ probs) {
+  const LoraDUBProblem P = probs[blockIdx.y];
+  const long long e = (long long)blockIdx.x * 256 + threadIdx.x;
+  if (e >= (long long)P.T * P.rs) return;
+  const int tok = (int)(e / P.rs), n = (int)(e % P.rs);
+  float s = 0.f;
+  if (n < P.rank) {
+    const float* w = P.W + (size_t)tok * P.rank + n;
+    const size_t step = (size_t)P.T * P.rank;
+    for (int i = 0; i < P.n_slabs; ++i) s += w[i * step];
+  }
+  P.dU[(size_t)tok * P.lddu + n] = __float2bfloat16_rn(s * P.scale);
 }
 
 }  // namespace
@@ -272,11 +449,42 @@ int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n
                          tokred_smem_bytes<128, 16>());
     cudaFuncSetAttribute(lora_tokred_kernel<16, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          tokred_smem_bytes<16, 128>());
+    cudaFuncSetAttribute(lora_tokred_kernel<32, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         tokred_smem_bytes<32, 128>());
+    cudaFuncSetAttribute(lora_tokred_kernel<64, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         tokred_smem_bytes<64, 128>());
     attr = true;
   }
   if (mt == 128) lora_tokred_kernel<128, 16><<<n_tiles, 128, tokred_smem_bytes<128, 16>(), st>>>(d_probs, d_tiles);
   else if (mt == 16) lora_tokred_kernel<16, 128><<<n_tiles, 128, tokred_smem_bytes<16, 128>(), st>>>(d_probs, d_tiles);
+  else if (mt == 32) lora_tokred_kernel<32, 128><<<n_tiles, 128, tokred_smem_bytes<32, 128>(), st>>>(d_probs, d_tiles);
+  else if (mt == 64) lora_tokred_kernel<64, 128><<<n_tiles, 128, tokred_smem_bytes<64, 128>(), st>>>(d_probs, d_tiles);
   else return -1;
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int lora_dub_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, int max_rank, cudaStream_t st) {
+  if (n_probs <= 0 || max_slabs <= 0 || max_rank <= 0) return 0;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_dub_kernel<LORA_DUB_MT, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         dub_smem_bytes<LORA_DUB_MT>());
+    cudaFuncSetAttribute(lora_dub_kernel<LORA_DUB_MT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         dub_smem_bytes<LORA_DUB_MT>());
+    attr = true;
+  }
+  const int n_rt = (max_rank + DUB_NT - 1) / DUB_NT;
+  const dim3 grid(max_slabs * n_rt, n_probs);
+  if (max_rank <= 8) lora_dub_kernel<LORA_DUB_MT, 1><<<grid, 128, dub_smem_bytes<LORA_DUB_MT>(), st>>>(d_probs, n_rt);
+  else lora_dub_kernel<LORA_DUB_MT, 2><<<grid, 128, dub_smem_bytes<LORA_DUB_MT>(), st>>>(d_probs, n_rt);
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max_elems, cudaStream_t st) {
+  if (n_probs <= 0 || max_elems <= 0) return 0;
+  lora_du_reduce_kernel<<<dim3((unsigned)((max_elems + 255) / 256), n_probs), 256, 0, st>>>(d_probs);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }

@@ -276,7 +276,10 @@ struct LayerSave {
   float *rstd1, *rstd2, *lse;
   bf16* U[NG];
 };
-struct SGList { int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0; };
+struct SGList {
+  int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0;
+  int max_rank = 0; long long max_elems = 0;   // fused dU+dB lists: widest rank, largest T * rs
+};
 
 struct menos_batch {
   int T = 0, n_seqs = 0;
@@ -307,8 +310,10 @@ struct menos_batch {
   uint8_t* d_ntile_qkv = nullptr;
   LoraRowsProblem* d_rprobs = nullptr; int2* d_rtiles = nullptr;
   LoraTokRedProblem* d_tprobs = nullptr; int4* d_ttiles = nullptr;
-  // per layer, per group: fwd shrink, bwd dU, bwd dB, bwd dA
-  std::vector<SGList> sg_fwd, sg_du, sg_db, sg_da;  // [layer * NG + g]
+  LoraDUBProblem* d_dprobs = nullptr;
+  // per layer, per group: fwd shrink, bwd fused dU + dB (one pass over dY per target), bwd dA (one pass over X per
+  // client and group)
+  std::vector<SGList> sg_fwd, sg_dub, sg_da;  // [layer * NG + g]
   // saved activations (SAVE) or x_c copy (NOGRAD)
   uint8_t* slab = nullptr;
   std::vector<LayerSave> L;
@@ -317,6 +322,7 @@ struct menos_batch {
   // and relocated before the backward (relocate_scratch_refs)
   std::vector<LoraRowsProblem> h_rprobs;
   std::vector<LoraTokRedProblem> h_tprobs;
+  std::vector<LoraDUBProblem> h_dprobs;
   uint8_t* scratch_base = nullptr; size_t scratch_span = 0;
   // live-batch accounting (menos_server::batch_refs / live_save): set when the handle is returned to the caller
   bool counted = false, counted_save = false;
@@ -1128,6 +1134,7 @@ struct Scratch {
   bf16 *qkv_x, *O_x, *dO_x, *dqkv_x; // prefix-tuning extension [Text, .] (nullptr without prefix clients)
   float *D_x, *dqacc_x;
   float* Dsum;
+  float* wsp;                        // fused dU + dB: per-slab fp32 dU partials (one group at a time)
   bf16* dU[NG];
 };
 
@@ -1198,8 +1205,7 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   (void)D;
   // small-GEMM problem lists are filled later (need layer buffers); reserve host vectors here
   b->sg_fwd.resize((size_t)s->n_layers * NG);
-  b->sg_du.resize((size_t)s->n_layers * NG);
-  b->sg_db.resize((size_t)s->n_layers * NG);
+  b->sg_dub.resize((size_t)s->n_layers * NG);
   b->sg_da.resize((size_t)s->n_layers * NG);
 
   out = std::move(b);
@@ -1224,6 +1230,20 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
   return per_layer * Ls;
 }
 // arena bytes of the per-call scratch block (see get_scratch)
+// fused dU + dB partials of one group's problems: sum over clients and targets of ceil(N_t/128) * T_c * rank * 4 B,
+// bounded per token by (max over the group's targets of ceil(N_t/128)) * (slot span R_used[g]) * 4 B
+static size_t wsp_bytes_of(const Dims& D, int T, const int R_used[NG]) {
+  size_t w = 0;
+  for (int g = 0; g < NG; ++g) {
+    if (!R_used[g]) continue;
+    int ms = 0;
+    for (int t = 0; t < NT; ++t)
+      if (kTargetGroup[t] == g) ms = std::max(ms, (D.N_t[t] + LORA_DUB_MT - 1) / LORA_DUB_MT);
+    w = std::max(w, (size_t)ms * R_used[g] * 4);
+  }
+  return w * (size_t)T;
+}
+
 static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text) {
   size_t need = 0;
   auto A = [&](size_t n) { need += align_up(n, 256); };
@@ -1238,6 +1258,7 @@ static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool 
   }
   A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.gu_cols * 2); A((size_t)T * D.fpad * 2);
   A((size_t)D.H * T * 4);                                                     // Dsum
+  A(wsp_bytes_of(D, T, R_used));                                              // dU partials
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
   if (nograd_set) {
@@ -1419,6 +1440,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   std::vector<int2> rtiles;
   std::vector<LoraTokRedProblem> tprobs;
   std::vector<int4> ttiles;
+  std::vector<LoraDUBProblem> dprobs;
   auto add_rows = [&](SGList& L, const std::vector<LoraRowsProblem>& ps) {
     L.probs_off = (int)rprobs.size(); L.n_probs = (int)ps.size(); L.tiles_off = (int)rtiles.size();
     std::vector<int2> tl;
@@ -1456,8 +1478,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         case GGU: X = S.hn; ldx = D.d; dY = sc.dgu; ldy = D.gu_cols; break;
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
-      std::vector<LoraRowsProblem> f, du;
-      std::vector<LoraTokRedProblem> db, da;
+      std::vector<LoraRowsProblem> f;
+      std::vector<LoraDUBProblem> dub;
+      std::vector<LoraTokRedProblem> da;
+      size_t woff = 0;   // fp32 offset of the next problem's dU partials in sc.wsp (the group's lists run in turn)
+      int da_w = 0;
       for (size_t k = 0; k < b->bclients.size(); ++k) {
         const Client& c = s->clients[b->bclients[k]];
         if (!c.width[g] || c.cut > l) continue;   // not yet in the segment at this layer
@@ -1472,59 +1497,63 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           p.C = U + (size_t)t0 * R + col; p.ldc = R;
           p.M = Tc; p.N = w; p.K = D.K_g[g]; p.scale = c.s;
           f.push_back(p);
-          if (g == GQKV) continue;   // q / k / v: per-target dU problems below
-          // dU[t, col..col+w) = s * dY_c Bcat[:, col..]   (other targets' rows of Bcat are zero in these columns)
-          LoraRowsProblem q{};
-          q.A = dY + (size_t)t0 * ldy; q.lda = ldy;
-          q.B = s->Bcat[g][l] + col; q.ldb = s->cols[g].cap; q.b_kn = 1;
-          q.C = sc.dU[g] + (size_t)t0 * R + col; q.ldc = R;
-          q.M = Tc; q.N = w; q.K = D.N_g[g]; q.scale = c.s;
-          du.push_back(q);
         }
-        if (g == GQKV) {
-          // q, k, v own contiguous row ranges of Bcat (and columns of dY): reduce each target over its own N_t
-          // columns only -- the other targets' columns multiply zero rows -- which also doubles the tile count
-          for (int t = TQ; t <= TV; ++t) {
-            if (!(c.mask >> t & 1)) continue;
-            LoraRowsProblem q{};
-            q.A = dY + (size_t)t0 * ldy + D.rb_base[t]; q.lda = ldy;
-            q.B = s->Bcat[g][l] + (size_t)D.rb_base[t] * s->cols[g].cap + c.col_off[g] + c.sub[t];
-            q.ldb = s->cols[g].cap; q.b_kn = 1;
-            q.C = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.ldc = R;
-            q.M = Tc; q.N = c.rs; q.K = D.N_t[t]; q.scale = c.s;
-            du.push_back(q);
-          }
-        }
-        // per target: dB = dY_t^T (s U_t), dA = dU_t^T X   (fp32, overwrite; reduced over this client only)
+        // per target, ONE pass over its dY columns: dB = dY_t^T (s U_t) and dU_t = s dY_t B_t (per-slab partials,
+        // then a fixed-order slab sum); targets own contiguous (gate/up: 128-interleaved) row ranges of Bcat
+        LoraTokRedProblem pa{};
+        int nseg = 0;
         for (int t = 0; t < NT; ++t) {
           if (kTargetGroup[t] != g || !(c.mask >> t & 1)) continue;
-          LoraTokRedProblem pb{};
-          pb.P = dY + (size_t)t0 * ldy + D.rb_base[t]; pb.ldp = ldy;
-          pb.p_blk = D.rb_blk[t]; pb.p_blk_stride = D.rb_stride[t];
-          pb.Q = U + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pb.ldq = R;
-          pb.C = c.G() + c.offB[l * NT + t]; pb.ldc = c.rank;
-          pb.M = D.N_t[t]; pb.N = c.rank; pb.T = Tc; pb.scale = 1.f;
-          db.push_back(pb);
-          LoraTokRedProblem pa{};
-          pa.P = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; pa.ldp = R;
-          pa.p_blk = 1 << 30; pa.p_blk_stride = 0;
-          pa.Q = X + (size_t)t0 * ldx; pa.ldq = ldx;
-          pa.C = c.G() + c.offA[l * NT + t]; pa.ldc = D.K_t[t];
-          pa.M = c.rank; pa.N = D.K_t[t]; pa.T = Tc; pa.scale = 1.f;
-          da.push_back(pa);
+          LoraDUBProblem q{};
+          q.dY = dY + (size_t)t0 * ldy + D.rb_base[t]; q.ldy = ldy;
+          q.p_blk = D.rb_blk[t]; q.p_blk_stride = D.rb_stride[t];
+          q.U = U + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.ldu = R;
+          q.B = s->Bcat[g][l] + (size_t)D.rb_base[t] * s->cols[g].cap + c.col_off[g] + c.sub[t];
+          q.ldb = s->cols[g].cap;
+          q.dB = c.G() + c.offB[l * NT + t];
+          q.W = sc.wsp + woff;
+          q.dU = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.lddu = R;
+          q.Nt = D.N_t[t]; q.rank = c.rank; q.rs = c.rs; q.T = Tc; q.scale = c.s;
+          q.n_slabs = (q.Nt + LORA_DUB_MT - 1) / LORA_DUB_MT;
+          if (q.p_blk % LORA_DUB_MT) FAIL(MENOS_EINVAL, "LoRA row block %d not a multiple of %d", q.p_blk, LORA_DUB_MT);
+          woff += (size_t)q.n_slabs * Tc * c.rank;
+          dub.push_back(q);
+          // dA of every target of the group in one pass over X: dU columns [sub_t, sub_t + rank) -> dA_t rows
+          float* Ct = c.G() + c.offA[l * NT + t];
+          if (nseg == 0) pa.C = Ct; else if (nseg == 1) pa.C1 = Ct; else pa.C2 = Ct;
+          pa.N = D.K_t[t]; pa.ldc = D.K_t[t];
+          ++nseg;
         }
+        pa.P = sc.dU[g] + (size_t)t0 * R + c.col_off[g]; pa.ldp = R;
+        pa.p_blk = 1 << 30; pa.p_blk_stride = 0;
+        pa.Q = X + (size_t)t0 * ldx; pa.ldq = ldx;
+        pa.M = c.width[g]; pa.T = Tc; pa.scale = 1.f;
+        pa.m_seg = c.rs; pa.m_valid = c.rank;
+        da.push_back(pa);
+        da_w = std::max(da_w, c.width[g]);
       }
       const size_t li = (size_t)l * NG + g;
       add_rows(b->sg_fwd[li], f);
-      add_rows(b->sg_du[li], du);
-      add_tokred(b->sg_db[li], db, 128, 16);
-      add_tokred(b->sg_da[li], da, 16, 128);
+      {
+        SGList& Ld = b->sg_dub[li];
+        Ld.probs_off = (int)dprobs.size(); Ld.n_probs = (int)dub.size();
+        for (const auto& q : dub) {
+          Ld.flops += 4.0 * q.Nt * q.rank * q.T;
+          Ld.max_n = std::max(Ld.max_n, q.n_slabs);
+          Ld.max_rank = std::max(Ld.max_rank, q.rank);
+          Ld.max_elems = std::max(Ld.max_elems, (long long)q.T * q.rs);
+        }
+        dprobs.insert(dprobs.end(), dub.begin(), dub.end());
+      }
+      const int da_mt = da_w <= 16 ? 16 : da_w <= 32 ? 32 : 64;
+      add_tokred(b->sg_da[li], da, da_mt, 128);
     }
   }
   const size_t o_rp = put(rprobs.data(), rprobs.size() * sizeof(LoraRowsProblem));
   const size_t o_rt = put(rtiles.data(), rtiles.size() * sizeof(int2));
   const size_t o_tp = put(tprobs.data(), tprobs.size() * sizeof(LoraTokRedProblem));
   const size_t o_tt = put(ttiles.data(), ttiles.size() * sizeof(int4));
+  const size_t o_dp = put(dprobs.data(), dprobs.size() * sizeof(LoraDUBProblem));
   uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
   if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
   b->meta = meta;
@@ -1556,6 +1585,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->d_rtiles = (int2*)(meta + o_rt);
   b->d_tprobs = (LoraTokRedProblem*)(meta + o_tp);
   b->d_ttiles = (int4*)(meta + o_tt);
+  b->d_dprobs = (LoraDUBProblem*)(meta + o_dp);
+  b->h_dprobs = std::move(dprobs);
   return MENOS_OK;
 }
 
@@ -1589,6 +1620,7 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
   sc.dgu = (bf16*)take((size_t)T * D.gu_cols * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
   sc.Dsum = (float*)take((size_t)D.H * T * 4);
+  sc.wsp = (float*)take(wsp_bytes_of(D, T, R_used));
   for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
   return MENOS_OK;
 }
@@ -1615,6 +1647,14 @@ static int run_rows(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
   return lora_rows_run(b->d_rprobs, b->d_rtiles + L.tiles_off, L.n_tiles, L.max_n, st);
+}
+// fused dU + dB (one pass over each target's dY), then the fixed-order slab sum into the bf16 dU slot columns
+static int run_dub(menos_batch* b, const SGList& L, cudaStream_t st) {
+  if (L.n_probs == 0) return 0;
+  ProfScope ps(PC_LORA, L.flops, 0, st);
+  int rc = lora_dub_run(b->d_dprobs + L.probs_off, L.n_probs, L.max_n, L.max_rank, st);
+  if (rc) return rc;
+  return lora_du_reduce_run(b->d_dprobs + L.probs_off, L.n_probs, L.max_elems, st);
 }
 static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
@@ -1796,7 +1836,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     dy = sc.gath;
   }
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
-  if (b->g_active[GD]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GD], st));
+  if (b->g_active[GD]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GD], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.fpad; a.K = D.d; a.b_mn_major = 1;
@@ -1809,9 +1849,9 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     if (opt) { a.epi = EPI_RELU_BWD; a.ldo = D.fpad; a.ldaux = D.fpad; }   // dz = da * (relu(z) > 0)
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GD]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GD], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GD], st)); }
+  if (b->g_active[GD]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GD], st));
   // A9: gate/up dX (+ LoRA) -> dhn; RMSNorm2 backward + residual -> dh
-  if (b->g_active[GGU]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GGU], st));
+  if (b->g_active[GGU]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GGU], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = D.gu_cols; a.b_mn_major = 1;
@@ -1824,7 +1864,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: gate|up-dX partials
   }
-  if (b->g_active[GGU]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GGU], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st)); }
+  if (b->g_active[GGU]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st));
   {
     ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
     const bf16* dhn = D.sp ? sc.rsout : sc.dhn;
@@ -1840,7 +1880,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   }
   // A10: O dX (+ LoRA o) -> dO (and, for head_dim % 32 == 0, the attention backward's row sums D)
   const bool fuse_dsum = D.hd % 32 == 0 && 128 % D.hd == 0;
-  if (b->g_active[GO]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GO], st));
+  if (b->g_active[GO]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GO], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
@@ -1855,7 +1895,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GO]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GO], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GO], st)); }
+  if (b->g_active[GO]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GO], st));
   // A11: attention backward (+ RoPE backward) -> dqkv
   if (!fuse_dsum) {
     ProfScope ps(PC_ATTN_PREP, 0, (double)T * (4.0 * D.Nq + 4 * D.H), st);
@@ -1902,7 +1942,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     }
   }
   // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
-  if (b->g_active[GQKV]) K_TRY(run_rows(b, b->sg_du[(size_t)l * NG + GQKV], st));
+  if (b->g_active[GQKV]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GQKV], st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = D.Nqkv; a.b_mn_major = 1;
@@ -1915,7 +1955,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: qkv-dX partials
   }
-  if (b->g_active[GQKV]) { K_TRY(run_tokred(b, b->sg_db[(size_t)l * NG + GQKV], st)); K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st)); }
+  if (b->g_active[GQKV]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st));
   {
     ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
     const bf16* dxn = D.sp ? sc.rsout : sc.dhn;
@@ -2049,11 +2089,14 @@ static int relocate_scratch_refs(menos_server* s, menos_batch* b, cudaStream_t s
     if (q >= lo && q < hi) p = reinterpret_cast<std::remove_reference_t<decltype(p)>>(const_cast<uint8_t*>(q) + delta);
   };
   for (auto& p : b->h_rprobs) { mv(p.A); mv(p.B); mv(p.C); }
-  for (auto& p : b->h_tprobs) { mv(p.P); mv(p.Q); mv(p.C); }
+  for (auto& p : b->h_tprobs) { mv(p.P); mv(p.Q); mv(p.C); mv(p.C1); mv(p.C2); }
+  for (auto& p : b->h_dprobs) { mv(p.dY); mv(p.U); mv(p.B); mv(p.dB); mv(p.W); mv(p.dU); }
   int rc = 0;
   if (!b->h_rprobs.empty()) rc = upload(s, b->d_rprobs, b->h_rprobs.data(), b->h_rprobs.size() * sizeof(LoraRowsProblem), st);
   if (!rc && !b->h_tprobs.empty())
     rc = upload(s, b->d_tprobs, b->h_tprobs.data(), b->h_tprobs.size() * sizeof(LoraTokRedProblem), st);
+  if (!rc && !b->h_dprobs.empty())
+    rc = upload(s, b->d_dprobs, b->h_dprobs.data(), b->h_dprobs.size() * sizeof(LoraDUBProblem), st);
   if (rc) return rc;
   b->scratch_base = s->scratch; b->scratch_span = s->scratch_bytes;
   return MENOS_OK;

@@ -36,6 +36,21 @@ def test_tiny_all_targets_gqa_ragged_mixed_ranks():
     assert_report(rep)
 
 
+def test_tiny_ranks_above_16():
+    """Ranks 24 and 32: the fused dU + dB kernel runs two 16-wide rank tiles per slab, and a q|k|v slot of 96
+    columns takes the one-pass dA over two 64-row tiles (three output segments)."""
+    m = dataclasses.replace(MODELS["tiny"], n_heads=4, n_kv_heads=2)
+    cl = [ClientCfg(32, 64.0, ("q", "v", "gate", "up"), [33, 90]), ClientCfg(24, 48.0, TARGETS, [57]),
+          ClientCfg(4, 8.0, ("v",), [16])]
+    w = Workload("tiny_big_rank", m, cl)
+    inputs = make_inputs(w, seed=11)
+    srv = new_server(w, inputs[0], max_rank=64)
+    ids = register(srv, w, inputs[1])
+    rep = compare_step(run_gpu_step(w, inputs=inputs, srv=srv, ids=ids), run_oracle_step(w, inputs=inputs))
+    srv.close()
+    assert_report(rep)
+
+
 def test_zero_b_equals_base_bitwise():
     """Invariant (b): with B = 0 the LoRA contribution is exactly zero, whatever the targets."""
     m = MODELS["tiny"]
