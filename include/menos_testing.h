@@ -65,10 +65,16 @@ MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A,
 /* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
    bit 1 = tcgen05 backward (else mma.sync), bit 2 = persistent warp-specialized tcgen05 forward (overrides
    bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1), bit 4 = (sequence, head)-grouped
-   work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1).  Default mode 14
-   (persistent forward + two-kernel persistent backward: measured faster than the one-pass kernel).
-   Returns MENOS_EINVAL outside [0, 63]. */
+   work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1), bit 6 (with bit 3)
+   = dS-stored backward: the dK/dV kernel also stores bf16 dS^T tiles and dQ = dS K is computed from them, so S, P and
+   dP are evaluated once per (key, query) pair.  Default mode 78 (persistent forward + dS-stored
+   persistent backward).  Returns MENOS_EINVAL outside [0, 127]. */
 MENOS_API int menos_test_set_attn_tc(int mode);
+
+/* dS-stored backward: most 16 KB dS^T tiles one chunk may use (default 32768 = 512 MB; the server reserves
+   min(this, what the batch needs) in its scratch and runs larger batches in chunks of (sequence, kv head) units).
+   Small values force chunking (tests).  MENOS_EINVAL if tiles < 1. */
+MENOS_API int menos_test_set_ds_cap(long long tiles);
 
 /* Tuning aid: per-phase clock64 totals of the one-pass attention backward's role threads (16 counters, cleared by the
  * read) when libmenos.so was built with -DMENOS_ABF_PROF (MENOS_NVCC_DEFS); zeros otherwise. */

@@ -12,6 +12,7 @@
 //     registers, stages bf16 rows (swizzled) in the freed P/dS buffers and the warps write them row-contiguously.
 // Elementwise work: P = exp2(S c - lse) (a quarter on the FMA pipe), dS = P (dP - D) scale, bf16 packed into
 // 128B-swizzled K-major tiles for the accumulation MMAs.
+#include <algorithm>
 #include "common.cuh"
 #include "kernels.h"
 
@@ -75,7 +76,22 @@ struct BwParams {
   const int* pos_shift;    // [n_seqs] prefix rows before each sequence (extended batch) or nullptr
   int T, H, Hkv;
   float scale;
+  // dS^T tiles for the dQ pass (attn_bwd_dq_ds_kernel) or nullptr: the dK/dV kernel stores every block's bf16
+  // dS^T [128 keys][64 queries] at tile ds_tile(...) of `ds`; ds_base[seq * Hkv + kv head] = first tile of the unit
+  bf16* ds;
+  const int* ds_base;
 };
+
+// dS^T tiles of one sequence of length L and one head: key block kb (128 keys) pairs with the 64-query blocks
+// qb = 2 kb .. nqb - 1 (causal); tiles are numbered key block by key block
+__host__ __device__ __forceinline__ int ds_tiles_of(int L) {
+  const int nqb = (L + 63) / 64, nkb = (L + 127) / 128;
+  return nkb * nqb - nkb * (nkb - 1);
+}
+__device__ __forceinline__ int ds_tile_in_head(int L, int kb, int qb) {
+  const int nqb = (L + 63) / 64;
+  return kb * nqb - kb * (kb - 1) + (qb - 2 * kb);
+}
 
 __device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
   uint32_t ok = 0;
@@ -221,7 +237,7 @@ __device__ __forceinline__ void ip_fetch(ItemPipe& q, const int* cu, const int* 
   q.c0 = 0; q.c1 = 0; q.sh = 0;
   if (q.cur.x >= 0) { q.c0 = cu[q.cur.x]; q.c1 = cu[q.cur.x + 1]; q.sh = ps ? ps[q.cur.x] : 0; }
 }
-struct Geo { int base, L, blk0, head, n, sh; };   // sh: RoPE position shift of the sequence (prefix rows)
+struct Geo { int base, L, blk0, head, n, sh, seq; };   // sh: RoPE position shift of the sequence (prefix rows)
 
 // -DMENOS_BWS_PROF: per-phase clock64 accounting (dK/dV kernel: one elementwise thread and the MMA lane)
 #ifdef MENOS_BWS_PROF
@@ -278,7 +294,7 @@ template <int HD>
 __global__ void __launch_bounds__(NTHREADS, 1)
 attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid_constant__ CUtensorMap tmQKV64,
                         const __grid_constant__ CUtensorMap tmDO64, const __grid_constant__ CUtensorMap tmOut,
-                        const BwParams p) {
+                        const __grid_constant__ CUtensorMap tmDS, const BwParams p) {
   constexpr int KV_TILE = DkdvGeo<HD>::KV_TILE, QB_TILE = DkdvGeo<HD>::QB_TILE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -330,7 +346,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     q.raw = item_at(p.items, p.n_items, item + 2 * gridDim.x);
   };
   auto decode = [&](const ItemPipe& q) {
-    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh};
+    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh, q.cur.x};
     g.n = rep * ((g.L - g.blk0 + QB - 1) / QB);      // (head of the group, 64-query block) pairs; 0 past the end
     return g;
   };
@@ -481,12 +497,19 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       ip_advance(ip, item);
       const int k0 = G.blk0, L = G.L, base = G.base, nqb = (L - k0 + QB - 1) / QB;
       const int kpos = k0 + r;
+      // dS^T tiles of this unit (sequence, kv head) for the dQ pass
+      const int ds_unit = (p.ds && G.n > 0) ? __ldg(p.ds_base + G.seq * p.Hkv + G.head) : 0;
       for (int j = 0; j < G.n; ++j, ++gb) {
         if ((gb & 1) != gr) continue;
         const int q0 = k0 + (j % nqb) * QB, sl = kb & 1;
+        // dS^T of this block -> the group's staging tile (128-byte swizzled rows) -> one TMA store (dS-stored variant)
+        // (sP0: idle between item epilogues; group gr stages in its half)
+        uint8_t* const ds_stg = sP0 + gr * PT_TILE + r * 128;
+        const bool ds_lead = p.ds != nullptr && w4 == 0 && lane == 0;
         if (!have_cur) { issue(sl, G, j); cp_async_commit(); }
         cp_async_wait<0>();
         s_ld[gr][sl][tt] *= tt < QB ? LOG2E_W : p.scale;   // lse to the log2 domain, D pre-scaled
+        if (p.ds && w4 == 0 && lane == 0) bulk_wait_read0();   // the group's staging tile is free again
         BP(9);
         gsync();
         BP(1);
@@ -523,12 +546,29 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
           pack_row(dsv, ud);
           tmem_st_half(tmem + 64 * gr + 32 * hf + lane_off, up);
           tmem_st_half(tmem + 128 + 64 * gr + 32 * hf + lane_off, ud);
+          if (p.ds) {   // the same bf16 dS^T row (queries 32 hf .. 32 hf + 31): four 16-byte chunks of the staged row
+#pragma unroll
+            for (int c = 0; c < CPT / 8; ++c) {
+              const int c8 = (CPT / 8) * hf + c;
+              *reinterpret_cast<uint4*>(ds_stg + ((c8 ^ (r & 7)) << 4)) =
+                  make_uint4(ud[4 * c], ud[4 * c + 1], ud[4 * c + 2], ud[4 * c + 3]);
+            }
+          }
         }
         BP(3);
         tmem_wait_st();
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&ew_done[gr]);
+        if (p.ds) {   // the staged dS^T tile leaves by TMA (async; the leader waits for its read before the next fill)
+          fence_proxy_async();
+          gsync();
+          if (ds_lead) {
+            const int tile = ds_unit + (j / nqb) * ds_tiles_of(L) + ds_tile_in_head(L, k0 / KV_ROWS, q0 / QB);
+            tma_store_2d(&tmDS, sP0 + gr * PT_TILE, 0, tile * KV_ROWS);
+            bulk_commit();
+          }
+        }
         ++kb;
         BP(5);
       }
@@ -542,6 +582,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       BP(6);
       tc_fence_after();
       if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's dV store has read the staging
+      if (p.ds && w4 == 0 && lane == 0) bulk_wait_read0();   // ... and the groups' dS^T stores (same buffer)
       tma_pending = false;
       ew_sync();
       bf16* dst = p.dqkv + (size_t)(base + k0) * p.ld_dqkv;
@@ -576,6 +617,10 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       } else {
         ew_sync();
         stage16_store<HD>(sP0, 1, w8, lane, nv, dst + (p.H + p.Hkv + G.head) * HD, dst, p.ld_dqkv);
+        ew_sync();
+      }
+      if (p.ds) {   // the next item's dS^T staging reuses sP0: the dV store must have read it
+        if (t == 0 && tma_pending) { bulk_wait_read0(); tma_pending = false; }
         ew_sync();
       }
       BP(8);
@@ -721,7 +766,7 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       BP(8);
     }
 #endif
-    if (t == 0) bulk_wait0();
+    if (t == 0 || (p.ds && (warp & 3) == 0 && lane == 0)) bulk_wait0();   // epilogue / dS^T stores complete
     BP_FLUSH(blockIdx.x < 8 && t == 0);
   }
   tc_fence_before();
@@ -788,7 +833,7 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
     q.raw = item_at(p.items, p.n_items, item + 2 * gridDim.x);
   };
   auto decode = [&](const ItemPipe& q) {
-    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh};
+    Geo g{q.c0, q.c1 - q.c0, q.cur.y, q.cur.z, 0, q.sh, q.cur.x};
     g.n = (min(g.L, g.blk0 + Q_ROWS) + KB - 1) / KB;   // 0 past the end
     return g;
   };
@@ -1100,6 +1145,153 @@ attn_bwd_dq_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __grid
   }
 }
 
+// ======================================================================================= dQ from stored dS^T
+// dQ[q, :] = sum over key blocks kb <= q-block of dS[q, keys of kb] K[keys of kb, :], with dS^T read back from the
+// tiles the dK/dV kernel stored (bf16 [128 keys][64 queries], linear; TMA applies the 128-byte swizzle), so S, P and
+// dP are computed ONCE per (key, query) pair: this pass is a memory-bound varlen GEMM (M = 128 queries = two
+// 64-query tiles read as one MN-major A operand one M-atom apart, N = head_dim, K = 128 keys per block).
+// Roles: warp 0 TMA (dS^T pair + K block per stage, 3-stage ring across items), warp 1 MMA (dQ in one of two TMEM
+// accumulators, so an item's epilogue overlaps the next item's MMAs), warps 2-9 the epilogue (RoPE backward, bf16,
+// TMA store) exactly as in attn_bwd_dq_ws_kernel.
+constexpr int DSQ_STAGES = 3;
+template <int HD> struct DqDsGeo {
+  static constexpr int DS2 = 2 * KV_ROWS * QB * 2;   // two dS^T tiles: 32 KB
+  static constexpr int KT = KV_ROWS * HD * 2;        // K block: 32 KB (HD 128) / 16 KB
+  static constexpr int STAGE = DS2 + KT;
+  static constexpr int STG = Q_ROWS * HD * 2;        // bf16 staging of one dQ block
+  static constexpr int SMEM = DSQ_STAGES * STAGE + STG + 1024;
+};
+static_assert(DqDsGeo<128>::SMEM <= 232448, "dQ-from-dS shared memory");
+
+template <int HD>
+__global__ void __launch_bounds__(NTHREADS, 1)
+attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_constant__ CUtensorMap tmQKV128,
+                      const __grid_constant__ CUtensorMap tmOut, const BwParams p) {
+  using Gm = DqDsGeo<HD>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* const sStage = smem;                              // [stage][dS^T pair | K block]
+  uint8_t* const sStg = smem + DSQ_STAGES * Gm::STAGE;       // dQ staging
+  __shared__ __align__(8) uint64_t full[DSQ_STAGES], empty[DSQ_STAGES], acc_full[2], acc_free[2];
+  __shared__ uint32_t tmem_sh;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int rep = p.H / p.Hkv;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmDS); tma_prefetch(&tmQKV128);
+    for (int i = 0; i < DSQ_STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_free[i], EW_WARPS); }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<2 * HD>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;
+  // item -> (sequence geometry, q0, head); items are read directly (the producer runs ahead of everyone else)
+  auto geo = [&](int item, int& base, int& L, int& q0, int& h, int& seq) {
+    const int4 it = p.items[item];
+    seq = it.x; q0 = it.y; h = it.z;
+    base = p.cu_seqlens[seq]; L = p.cu_seqlens[seq + 1] - base;
+  };
+
+  if (warp == 0) {
+    if (elect_one()) {
+      int gb = 0;
+      for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
+        int base, L, q0, h, seq;
+        geo(item, base, L, q0, h, seq);
+        const int hk = h / rep;
+        const int t_head = __ldg(p.ds_base + seq * p.Hkv + hk) + (h - hk * rep) * ds_tiles_of(L);
+        const int kcol = (p.H + hk) * HD;
+        for (int kb = 0; kb <= q0 / KV_ROWS; ++kb, ++gb) {
+          const int st = gb % DSQ_STAGES;
+          wait_bar(&empty[st], ((gb / DSQ_STAGES) & 1) ^ 1);
+          mbar_expect_tx(&full[st], Gm::STAGE);
+          uint8_t* sd = sStage + st * Gm::STAGE;
+          const int tile = t_head + ds_tile_in_head(L, kb, q0 / QB);   // (kb, 2 qb128) and the next tile
+          tma_load_2d(sd, &tmDS, &full[st], 0, tile * KV_ROWS);
+#pragma unroll
+          for (int a = 0; a < HD / 64; ++a)
+            tma_load_2d(sd + Gm::DS2 + a * KVA, &tmQKV128, &full[st], kcol + 64 * a, base + kb * KV_ROWS);
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    constexpr uint32_t ID_DQ = umma_idesc_bf16(128, HD, 1) | (1u << 15);   // A (dS) and B (K) MN-major
+    int gb = 0, it = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      const int q0 = p.items[item].y;
+      const int buf = it & 1;
+      wait_bar(&acc_free[buf], ((it >> 1) & 1) ^ 1);
+      tc_fence_after();
+      for (int kb = 0; kb <= q0 / KV_ROWS; ++kb, ++gb) {
+        const int st = gb % DSQ_STAGES;
+        wait_bar(&full[st], (gb / DSQ_STAGES) & 1);
+        tc_fence_after();
+        __syncwarp();
+        if (elect_one()) {
+          const uint32_t sd = smem_u32(sStage + st * Gm::STAGE), sk = sd + Gm::DS2;
+#pragma unroll
+          for (int kk = 0; kk < KV_ROWS / 16; ++kk)   // 16 keys = 2048 B of both the dS^T pair and the K block
+            tc_mma_bf16(tmem + buf * HD, umma_desc_sw128(sd + kk * 2048, 16384, 1024),
+                        umma_desc_sw128(sk + kk * 2048, 16384, 1024), ID_DQ, (kb > 0 || kk > 0) ? 1u : 0u);
+          tc_commit(&empty[st]);
+        }
+        __syncwarp();
+      }
+      if (elect_one()) tc_commit(&acc_full[buf]);
+      __syncwarp();
+    }
+  } else {
+    const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
+    const int r = w4 * 32 + lane;   // query row = TMEM lane
+    const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
+    bool tma_pending = false;
+    int it = 0;
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+      int base, L, q0, h, seq;
+      geo(item, base, L, q0, h, seq);
+      const int sh = p.pos_shift ? p.pos_shift[seq] : 0;
+      const int buf = it & 1;
+      const int nv = min(Q_ROWS, L - q0);
+      const bool rope = p.rope_cs != nullptr && r < nv;
+      RopeCS<HD> csq;
+      rope_cs_load<HD>(csq, p.rope_cs, max(0, q0 + r - sh), g, rope);   // in flight during the wait below
+      wait_bar(&acc_full[buf], (it >> 1) & 1);
+      tc_fence_after();
+      if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's TMA store has read the staging
+      tma_pending = false;
+      ew_sync();
+      acc_row_to_bf16<HD>(tmem + buf * HD + lane_off, sStg, r, g, csq, rope);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free[buf]);
+      if (nv == Q_ROWS) {
+        fence_proxy_async();
+        ew_sync();
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sStg, base + q0, h * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+      } else {
+        ew_sync();
+        bf16* dq = p.dqkv + (size_t)(base + q0) * p.ld_dqkv + h * HD;
+        stage16_store<HD>(sStg, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
+        ew_sync();
+      }
+    }
+    if (t == 0) bulk_wait0();
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<2 * HD>(tmem);
+  }
+}
+
 }  // namespace
 
 #ifdef MENOS_BWS_PROF
@@ -1123,6 +1315,7 @@ static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv
   if (!tma_map_2d(&mDO64, a.dO, a.T, a.H * HD, a.ld_do, 64, 64)) return -2;
   if (!tma_map_2d(&mDO128, a.dO, a.T, a.H * HD, a.ld_do, 64, 128)) return -2;
   BwParams p;
+  memset(&p, 0, sizeof p);
   p.cu_seqlens = a.cu_seqlens; p.lse = a.lse; p.D = a.D; p.dqkv = a.dqkv;
   p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.pos_shift = a.pos_shift; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv;
   p.scale = a.scale;
@@ -1135,7 +1328,7 @@ static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv
   p.items = items_kv; p.n_items = n_items_kv;
   if (n_items_kv > 0)
     attn_bwd_dkdv_ws_kernel<HD><<<min(n_items_kv, num_sms), NTHREADS, DkdvGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO64,
-                                                                                                mOut, p);
+                                                                                                mOut, mQKV128, p);
   ++g_launch_count;
   p.items = items_q; p.n_items = n_items_q;
   if (n_items_q > 0)
@@ -1143,6 +1336,97 @@ static int launch_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv
                                                                                             mOut, p);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+// dS-stored variant: dK/dV (storing dS^T tiles) then dQ from the tiles
+template <int HD>
+static int launch_bwd_ws_ds(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                            bf16* ds, long long ds_tiles, const int* ds_base, int num_sms, cudaStream_t st) {
+  CUtensorMap mQKV128, mQKV64, mDO64, mOut, mDS;
+  if (!tma_map_2d(&mQKV128, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 128)) return -2;
+  if (!tma_map_2d(&mOut, a.dqkv, a.T, (a.H + 2 * a.Hkv) * HD, a.ld_dqkv, 64, 128)) return -2;
+  if (!tma_map_2d(&mQKV64, a.qkv, a.T, a.ld_qkv, a.ld_qkv, 64, 64)) return -2;
+  if (!tma_map_2d(&mDO64, a.dO, a.T, a.H * HD, a.ld_do, 64, 64)) return -2;
+  if (!tma_map_2d(&mDS, ds, (uint64_t)ds_tiles * KV_ROWS, QB, QB, 64, KV_ROWS)) return -2;      // dK/dV: store
+  CUtensorMap mDS2;
+  if (!tma_map_2d(&mDS2, ds, (uint64_t)ds_tiles * KV_ROWS, QB, QB, 64, 2 * KV_ROWS)) return -2;  // dQ: tile pairs
+  BwParams p;
+  memset(&p, 0, sizeof p);
+  p.cu_seqlens = a.cu_seqlens; p.lse = a.lse; p.D = a.D; p.dqkv = a.dqkv;
+  p.ld_dqkv = a.ld_dqkv; p.rope_cs = a.rope_cs; p.pos_shift = a.pos_shift; p.T = a.T; p.H = a.H; p.Hkv = a.Hkv;
+  p.scale = a.scale; p.ds = ds; p.ds_base = ds_base;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(attn_bwd_dkdv_ws_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, DkdvGeo<HD>::SMEM);
+    cudaFuncSetAttribute(attn_bwd_dq_ds_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize, DqDsGeo<HD>::SMEM);
+    attr = true;
+  }
+  p.items = items_kv; p.n_items = n_items_kv;
+  if (n_items_kv > 0) {
+    attn_bwd_dkdv_ws_kernel<HD><<<min(n_items_kv, num_sms), NTHREADS, DkdvGeo<HD>::SMEM, st>>>(mQKV128, mQKV64, mDO64,
+                                                                                                mOut, mDS, p);
+    ++g_launch_count;
+  }
+  p.items = items_q; p.n_items = n_items_q;
+  if (n_items_q > 0) {
+    attn_bwd_dq_ds_kernel<HD><<<min(n_items_q, num_sms), NTHREADS, DqDsGeo<HD>::SMEM, st>>>(mDS2, mQKV128, mOut, p);
+    ++g_launch_count;
+  }
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int attn_bwd_ws_ds(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                   bf16* ds, long long ds_tiles, const int* ds_base, int num_sms, cudaStream_t st) {
+  if (!MENOS_BWS_ALT) return -1;   // the dS^T stores live in the alternating-group elementwise path
+  if (n_items_kv <= 0 && n_items_q <= 0) return 0;
+  if (a.hd == 128) return launch_bwd_ws_ds<128>(a, items_kv, n_items_kv, items_q, n_items_q, ds, ds_tiles, ds_base, num_sms, st);
+  if (a.hd == 64) return launch_bwd_ws_ds<64>(a, items_kv, n_items_kv, items_q, n_items_q, ds, ds_tiles, ds_base, num_sms, st);
+  return -1;
+}
+int attn_ds_tiles(int L) { return ds_tiles_of(L); }
+
+long long attn_ds_total_tiles(const int* seq_len, int n_seqs, int H) {
+  long long t = 0;
+  for (int i = 0; i < n_seqs; ++i) t += (long long)H * ds_tiles_of(seq_len[i]);
+  return t;
+}
+
+bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out) {
+  const int rep = H / Hkv;
+  out.base.assign((size_t)n_seqs * Hkv, 0);
+  out.items_kv.clear(); out.items_q.clear(); out.chunks.clear();
+  std::vector<int2> units;   // (seq, kv head) of the open chunk
+  long long cur = 0;
+  auto flush = [&]() {
+    if (units.empty()) return;
+    const int kv0 = (int)out.items_kv.size(), q0 = (int)out.items_q.size();
+    for (const int2& u : units) {
+      const int L = seq_len[u.x];
+      for (int k = 0; k < L; k += 128) out.items_kv.push_back(make_int4(u.x, k, u.y, 0));
+      for (int h = u.y * rep; h < (u.y + 1) * rep; ++h)
+        for (int q = ((L - 1) / 128) * 128; q >= 0; q -= 128) out.items_q.push_back(make_int4(u.x, q, h, 0));
+    }
+    // dK/dV: LPT for the persistent grid's static round-robin (largest = most query blocks after the key block)
+    std::stable_sort(out.items_kv.begin() + kv0, out.items_kv.end(), [&](const int4& a, const int4& b) {
+      return seq_len[a.x] - a.y > seq_len[b.x] - b.y;
+    });
+    // dQ items stay grouped by (sequence, head), last query block first: neighbouring CTAs read the same K blocks
+    // at the same time (one L2 fill instead of one per query block)
+    out.chunks.push_back(make_int4(kv0, (int)out.items_kv.size() - kv0, q0, (int)out.items_q.size() - q0));
+    units.clear();
+    cur = 0;
+  };
+  for (int i = 0; i < n_seqs; ++i)
+    for (int hk = 0; hk < Hkv; ++hk) {
+      const long long ut = (long long)rep * ds_tiles_of(seq_len[i]);
+      if (ut > cap_tiles) return false;
+      if (cur + ut > cap_tiles) flush();
+      out.base[(size_t)i * Hkv + hk] = (int)cur;
+      cur += ut;
+      units.push_back(make_int2(i, hk));
+    }
+  flush();
+  return true;
 }
 
 int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,

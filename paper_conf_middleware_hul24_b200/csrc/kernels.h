@@ -89,9 +89,17 @@ struct LoraDUBProblem {
   float scale;
 };
 int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st);
-int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st);
+int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, int nt, cudaStream_t st);
 void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out);
 void lora_tokred_tiles(const LoraTokRedProblem* probs, int n, int mt, int nt, std::vector<int4>& out);
+// shrink on tcgen05: U[t0 + m, col + n] = bf16(scale * sum_k X[t0 + m, k] Acat[col + n, k]), m < T, n < w
+// (w <= 128, w % 8 == 0 and col % 8 == 0); X [x_rows, K] (ld ldx) and Acat [a_rows, K] (ld lda) are whole buffers
+// (one TMA map each), problems index into them; tiles = (problem, 128-token tile start) from lora_shrink_tiles
+struct LoraShrinkProblem { int t0, T, col, w; float scale; };
+void lora_shrink_tiles(const LoraShrinkProblem* probs, int n, std::vector<int2>& out);
+int lora_shrink_tc_run(const bf16* X, int x_rows, int ldx, const bf16* Acat, int a_rows, int lda, int K,
+                       const LoraShrinkProblem* d_probs, const int2* d_tiles, int n_tiles, int max_w, bf16* U, int ldu,
+                       cudaStream_t st);
 // dU/dB slab width (dY columns per CTA) used for n_slabs
 constexpr int LORA_DUB_MT = 128;
 // grid: (max n_slabs * ceil(max rank / 16), n_probs); CTAs past a problem's slabs exit
@@ -154,6 +162,23 @@ void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out
 // head, -) per 128-key block, items_q = (seq, q0, head, -) per 128-query block
 int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
                 int num_sms, cudaStream_t st);
+// same, with S / P / dP computed once per (key, query) pair: the dK/dV kernel also stores bf16 dS^T tiles
+// ([128 keys][64 queries], `ds`, ds_tiles of them) and a second kernel computes dQ = dS K from them.
+// ds_base[seq * Hkv + kv head] = first tile of that (sequence, kv head) unit; a unit holds, per head of its group,
+// attn_ds_tiles(L) tiles numbered key block by key block (64-query blocks 2 kb .. ceil(L/64) - 1 of key block kb).
+// The items must cover exactly the units whose tiles fit in `ds` (the caller chunks larger batches).
+int attn_bwd_ws_ds(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
+                   bf16* ds, long long ds_tiles, const int* ds_base, int num_sms, cudaStream_t st);
+int attn_ds_tiles(int L);
+long long attn_ds_total_tiles(const int* seq_len, int n_seqs, int H);
+// Host plan of the dS-stored backward over sequences [0, n_seqs): units (sequence, kv head) packed in order into
+// chunks of at most cap_tiles tiles; base[seq * Hkv + kv head] = the unit's first tile within its chunk; per chunk c
+// the work lists items_kv[chunks[c].x, + .y) and items_q[chunks[c].z, + .w) (LPT-ordered).  false: a single unit
+// is larger than cap_tiles (the caller takes the recompute path).
+struct AttnDsPlan { std::vector<int> base; std::vector<int4> items_kv, items_q, chunks; };
+bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out);
+// tiles the dS-stored backward may use at most (the buffer a chunk fills): 16 KB each
+extern long long g_attn_ds_cap_tiles;
 // one-pass persistent tcgen05 backward for head_dim 128 (attention_bwd_fused.cu): items = (seq, -, kv head, -), one
 // per (sequence, kv head), longest sequence first (attn_seq_items)
 int attn_bwd_fused(const AttnArgs& a, const int4* items_seq, int n_items, int num_sms, cudaStream_t st);

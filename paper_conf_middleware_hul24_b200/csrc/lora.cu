@@ -35,11 +35,11 @@ __device__ __forceinline__ int tsw(int row, int chunk) {
 // ROWS_BM tokens per CTA, one warp per 16 of them.  64 (default) vs 32 measured at cfg1 shapes
 // (profiles/r1n_lora_rows_bm.txt): 32-token blocks double the CTAs but each CTA still re-stages the whole
 // [N, K] adapter operand from L2, so the shrink is no faster and the per-target dU is 38% slower.
-// Stages: as many 128-wide K tiles as ~196 KB of shared memory holds (one CTA per SM): the shrink has one CTA per
-// 64 tokens (128 CTAs at cfg1), so the bytes each SM keeps in flight set its HBM rate (4 stages: 1.9 TB/s, r2bb)
+// 4 stages: 8 (one CTA per SM) measured no faster at cfg1 (35 us per layer either way: the 128 CTAs are bound by
+// their per-warp issue chain, not by bytes in flight) and 1.5x slower at cfg3 (r2bc, profiles/r2bc_lora.txt)
 constexpr int ROWS_BM = MENOS_LORA_ROWS_BM, ROWS_BK = 128, ROWS_NTH = ROWS_BM / 16 * 32;
 template <int NT>
-__host__ __device__ constexpr int rows_stages() { return NT <= 32 ? 8 : NT <= 64 ? 6 : 4; }
+__host__ __device__ constexpr int rows_stages() { return 4; }
 template <int NT>
 constexpr int rows_smem_bytes() { return rows_stages<NT>() * (ROWS_BM + NT) * ROWS_BK * 2; }
 
@@ -343,10 +343,15 @@ __global__ void __launch_bounds__(128) lora_dub_kernel(const LoraDUBProblem* __r
 #pragma unroll
         for (int j = 0; j < NJ; ++j) mma_bf16_16816(accb[i][j], a[i], b[2 * j], b[2 * j + 1]);
     }
-    // dU share: warp w takes the stage's tokens 16w..16w+15, reduction over the slab's MT columns (two independent
-    // accumulator chains when NJ = 1, summed at the end in a fixed order)
+    // dU share: warp w takes the stage's tokens 16w..16w+15, reduction over the slab's MT columns in two independent
+    // accumulator chains (even / odd 16-column steps) summed at the end -- the same order for every NJ, so a
+    // client's dU does not depend on the ranks of the clients sharing its batch
     {
-      float accu[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+      float acc2[NJ][2][4];
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) acc2[j][c][0] = acc2[j][c][1] = acc2[j][c][2] = acc2[j][c][3] = 0.f;
 #pragma unroll
       for (int kk = 0; kk < MT; kk += 16) {
         uint32_t a[4], b[4];
@@ -358,17 +363,14 @@ __global__ void __launch_bounds__(128) lora_dub_kernel(const LoraDUBProblem* __r
           const int row = kk + (mat & 1) * 8 + rr, col = (mat >> 1) * 8;
           ldsm_x4_t(smem_u32(Bs + tsw<NT>(row, col >> 3)), b[0], b[1], b[2], b[3]);
         }
-        if (NJ == 2) {
-          mma_bf16_16816(accu[0], a, b[0], b[1]);
-          mma_bf16_16816(accu[1], a, b[2], b[3]);
-        } else {
-          mma_bf16_16816(accu[(kk >> 4) & 1], a, b[0], b[1]);
-        }
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) mma_bf16_16816(acc2[j][(kk >> 4) & 1], a, b[2 * j], b[2 * j + 1]);
       }
-      if (NJ == 1)
+      float accu[NJ][4];
 #pragma unroll
-        for (int e = 0; e < 4; ++e) accu[0][e] += accu[1][e];
+      for (int j = 0; j < NJ; ++j)
 #pragma unroll
+        for (int e = 0; e < 4; ++e) accu[j][e] = acc2[j][0][e] + acc2[j][1][e];
       for (int j = 0; j < NJ; ++j)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
@@ -407,9 +409,112 @@ __global__ void __launch_bounds__(256) lora_du_reduce_kernel(const LoraDUBProble
   if (n < P.rank) {
     const float* w = P.W + (size_t)tok * P.rank + n;
     const size_t step = (size_t)P.T * P.rank;
+#pragma unroll 8
     for (int i = 0; i < P.n_slabs; ++i) s += w[i * step];
   }
   P.dU[(size_t)tok * P.lddu + n] = __float2bfloat16_rn(s * P.scale);
+}
+
+// ============================================================================ shrink on tcgen05
+// U[t0 + m, col + n] = bf16(scale * sum_k X[t0 + m, k] Acat[col + n, k])  (m < T, n < w): a [128 x K] . [K x N]
+// skinny GEMM per 128-token tile of one client.  TMA streams X and the client's Acat rows (both K-major, 128-byte
+// swizzle) through a ring of ~200 KB, one elected thread issues tcgen05.mma into a [128 x N] TMEM accumulator, four
+// warps scale, convert and store.  Pure streaming of X: on mma.sync the same contraction ran at ~2 TB/s (r2bc).
+constexpr int SHK_BK = 64;
+template <int N> struct ShkGeo {
+  static constexpr int A_BYTES = 128 * SHK_BK * 2, B_BYTES = N * SHK_BK * 2, STAGE = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (200 * 1024) / STAGE;
+  static constexpr int SMEM = STAGES * STAGE + 1024;
+  static constexpr int TCOLS = N < 32 ? 32 : N;
+};
+
+template <int N>
+__global__ void __launch_bounds__(192, 1)
+lora_shrink_tc_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmA,
+                      const LoraShrinkProblem* __restrict__ probs, const int2* __restrict__ tiles, int K, bf16* U,
+                      int ldu) {
+  using G = ShkGeo<N>;
+  constexpr int S = G::STAGES;
+  extern __shared__ uint8_t shk_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(shk_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full[S], empty[S], acc_full;
+  __shared__ uint32_t tmem_sh;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int2 tl = tiles[blockIdx.x];
+  const LoraShrinkProblem P = probs[tl.x];
+  const int m0 = tl.y, nk = (K + SHK_BK - 1) / SHK_BK;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmX); tma_prefetch(&tmA);
+    for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    mbar_init(&acc_full, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<G::TCOLS>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;
+  if (warp == 0) {
+    if (elect_one()) {
+      for (int kb = 0; kb < nk; ++kb) {
+        const int st = kb % S;
+        mbar_wait(&empty[st], ((kb / S) & 1) ^ 1);
+        mbar_expect_tx(&full[st], G::STAGE);
+        uint8_t* sa = smem + st * G::STAGE;
+        tma_load_2d(sa, &tmX, &full[st], kb * SHK_BK, P.t0 + m0);
+        tma_load_2d(sa + G::A_BYTES, &tmA, &full[st], kb * SHK_BK, P.col);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    constexpr uint32_t ID = umma_idesc_bf16(128, N, 0);
+    for (int kb = 0; kb < nk; ++kb) {
+      const int st = kb % S;
+      mbar_wait(&full[st], (kb / S) & 1);
+      tc_fence_after();
+      __syncwarp();
+      if (elect_one()) {
+        const uint32_t sa = smem_u32(smem + st * G::STAGE), sb = sa + G::A_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < SHK_BK / 16; ++kk)
+          tc_mma_bf16(tmem, umma_desc_sw128(sa + kk * 32, 16, 1024), umma_desc_sw128(sb + kk * 32, 16, 1024), ID,
+                      (kb > 0 || kk > 0) ? 1u : 0u);
+        tc_commit(&empty[st]);
+        if (kb == nk - 1) tc_commit(&acc_full);
+      }
+      __syncwarp();
+    }
+  } else {
+    const int q = warp & 3, row = q * 32 + lane;   // TMEM lane quadrant of this warp
+    mbar_wait(&acc_full, 0);
+    tc_fence_after();
+    const bool ok = m0 + row < P.T;
+    bf16* dst = U + (size_t)(P.t0 + m0 + row) * ldu + P.col;
+#pragma unroll
+    for (int c0 = 0; c0 < N; c0 += 32) {
+      uint32_t r[32];
+      tmem_ld32_nw(tmem + c0 + ((uint32_t)(q * 32) << 16), r);
+      tmem_wait_ld();
+      if (ok) {
+#pragma unroll
+        for (int j = 0; j < 32; j += 8)
+          if (c0 + j < P.w) {
+            uint4 v;
+            v.x = pack_bf16x2(__uint_as_float(r[j]) * P.scale, __uint_as_float(r[j + 1]) * P.scale);
+            v.y = pack_bf16x2(__uint_as_float(r[j + 2]) * P.scale, __uint_as_float(r[j + 3]) * P.scale);
+            v.z = pack_bf16x2(__uint_as_float(r[j + 4]) * P.scale, __uint_as_float(r[j + 5]) * P.scale);
+            v.w = pack_bf16x2(__uint_as_float(r[j + 6]) * P.scale, __uint_as_float(r[j + 7]) * P.scale);
+            *reinterpret_cast<uint4*>(dst + c0 + j) = v;
+          }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<G::TCOLS>(tmem);
+  }
 }
 
 }  // namespace
@@ -441,7 +546,7 @@ int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_til
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }
 
-int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, cudaStream_t st) {
+int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, int nt, cudaStream_t st) {
   if (n_tiles <= 0) return 0;
   static bool attr = false;
   if (!attr) {
@@ -453,12 +558,17 @@ int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n
                          tokred_smem_bytes<32, 128>());
     cudaFuncSetAttribute(lora_tokred_kernel<64, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          tokred_smem_bytes<64, 128>());
+
     attr = true;
   }
-  if (mt == 128) lora_tokred_kernel<128, 16><<<n_tiles, 128, tokred_smem_bytes<128, 16>(), st>>>(d_probs, d_tiles);
-  else if (mt == 16) lora_tokred_kernel<16, 128><<<n_tiles, 128, tokred_smem_bytes<16, 128>(), st>>>(d_probs, d_tiles);
-  else if (mt == 32) lora_tokred_kernel<32, 128><<<n_tiles, 128, tokred_smem_bytes<32, 128>(), st>>>(d_probs, d_tiles);
-  else if (mt == 64) lora_tokred_kernel<64, 128><<<n_tiles, 128, tokred_smem_bytes<64, 128>(), st>>>(d_probs, d_tiles);
+#define TOKRED_CASE(MT_, NT_) \
+  else if (mt == MT_ && nt == NT_) lora_tokred_kernel<MT_, NT_><<<n_tiles, 128, tokred_smem_bytes<MT_, NT_>(), st>>>(d_probs, d_tiles);
+  if (false) {}
+  TOKRED_CASE(128, 16)
+  TOKRED_CASE(16, 128)
+  TOKRED_CASE(32, 128)
+  TOKRED_CASE(64, 128)
+#undef TOKRED_CASE
   else return -1;
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
@@ -489,4 +599,44 @@ int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }
 
+}  // namespace menos
+
+namespace menos {
+bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
+                uint32_t br);
+
+void lora_shrink_tiles(const LoraShrinkProblem* probs, int n, std::vector<int2>& out) {
+  for (int i = 0; i < n; ++i)
+    for (int m = 0; m < probs[i].T; m += 128) out.push_back(make_int2(i, m));
+}
+
+template <int N>
+static int shrink_launch(const CUtensorMap& mX, const CUtensorMap& mA, const LoraShrinkProblem* d_probs,
+                         const int2* d_tiles, int n_tiles, int K, bf16* U, int ldu, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_shrink_tc_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, ShkGeo<N>::SMEM);
+    attr = true;
+  }
+  lora_shrink_tc_kernel<N><<<n_tiles, 192, ShkGeo<N>::SMEM, st>>>(mX, mA, d_probs, d_tiles, K, U, ldu);
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int lora_shrink_tc_run(const bf16* X, int x_rows, int ldx, const bf16* Acat, int a_rows, int lda, int K,
+                       const LoraShrinkProblem* d_probs, const int2* d_tiles, int n_tiles, int max_w, bf16* U, int ldu,
+                       cudaStream_t st) {
+  if (n_tiles <= 0) return 0;
+  const int N = max_w <= 16 ? 16 : max_w <= 32 ? 32 : max_w <= 64 ? 64 : max_w <= 128 ? 128 : -1;
+  if (N < 0 || ldx % 8 || lda % 8 || ldu % 8) return -1;   // TMA: 16-byte row strides; any K (OOB columns read 0)
+  CUtensorMap mX, mA;
+  if (!tma_map_2d(&mX, X, x_rows, K, ldx, SHK_BK, 128)) return -2;
+  if (!tma_map_2d(&mA, Acat, a_rows, K, lda, SHK_BK, N)) return -2;
+  switch (N) {
+    case 16: return shrink_launch<16>(mX, mA, d_probs, d_tiles, n_tiles, K, U, ldu, st);
+    case 32: return shrink_launch<32>(mX, mA, d_probs, d_tiles, n_tiles, K, U, ldu, st);
+    case 64: return shrink_launch<64>(mX, mA, d_probs, d_tiles, n_tiles, K, U, ldu, st);
+    default: return shrink_launch<128>(mX, mA, d_probs, d_tiles, n_tiles, K, U, ldu, st);
+  }
+}
 }  // namespace menos

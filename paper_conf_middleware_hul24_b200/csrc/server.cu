@@ -62,6 +62,7 @@ void set_last_error(const char* fmt, ...) {
   } while (0)
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+constexpr size_t kDsTileBytes = 128 * 64 * 2;   // one bf16 dS^T tile [128 keys][64 queries]
 
 // =====================================================================================================
 // per-kernel-class CUDA-event profiler (bench.py's live roofline; off by default)
@@ -279,6 +280,7 @@ struct LayerSave {
 struct SGList {
   int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0;
   int max_rank = 0; long long max_elems = 0;   // fused dU+dB lists: widest rank, largest T * rs
+  int tile_n = 0;                              // token-reduction lists: tile width
 };
 
 struct menos_batch {
@@ -301,6 +303,12 @@ struct menos_batch {
     double pairs = 0;
     size_t o_items = 0, o_items_kv = 0, o_items_q = 0, o_items_seq = 0;
     int4 *items = nullptr, *items_kv = nullptr, *items_q = nullptr, *items_seq = nullptr;
+    // dS-stored backward plan over this view's sequences (attn_ds_plan): per chunk (kv off, n, q off, n)
+    bool ds_ok = false;
+    std::vector<int4> ds_chunks;
+    size_t o_ds_kv = 0, o_ds_q = 0, o_ds_base = 0;
+    int4 *ds_kv = nullptr, *ds_q = nullptr;
+    int* ds_base = nullptr;
   };
   std::vector<AttnView> views;
   // device metadata
@@ -311,6 +319,16 @@ struct menos_batch {
   LoraRowsProblem* d_rprobs = nullptr; int2* d_rtiles = nullptr;
   LoraTokRedProblem* d_tprobs = nullptr; int4* d_ttiles = nullptr;
   LoraDUBProblem* d_dprobs = nullptr;
+  // forward LoRA shrink on tcgen05, per layer and group: whole-buffer operands + (client, 128-column chunk) problems
+  struct ShkList {
+    const bf16* X = nullptr; int x_rows = 0, ldx = 0; const bf16* A = nullptr; int a_rows = 0, lda = 0, K = 0;
+    bf16* U = nullptr; int ldu = 0;
+    int probs_off = 0, tiles_off = 0, n_tiles = 0, max_w = 0; double flops = 0;
+  };
+  std::vector<ShkList> sg_shk;   // [layer * NG + g]
+  LoraShrinkProblem* d_sprobs = nullptr; int2* d_stiles = nullptr;
+  // dS-stored attention backward: chunk buffer tiles (0 = the recompute path for this batch)
+  long long ds_tiles = 0;
   // per layer, per group: fwd shrink, bwd fused dU + dB (one pass over dY per target), bwd dA (one pass over X per
   // client and group)
   std::vector<SGList> sg_fwd, sg_dub, sg_da;  // [layer * NG + g]
@@ -937,8 +955,22 @@ extern "C" int menos_client_memory(menos_server* s, int32_t id, int n_tokens, si
 }
 
 static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], bool save_a, bool save, int Text);
-static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text);
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text, long long ds_tiles);
+static long long ds_tiles_bound(const menos_server* s, long long T);
 static size_t meta_bytes_bound(int T, int Ls, int n_clients);
+
+// The dS-stored attention backward (testing mode bit 6 with bit 3, the default) runs for head_dim 128 / 64 batches
+// without prefix-tuning clients
+static bool ds_path_on(const menos_server* s) {
+  return (g_attn_tc & 72) == 72 && !(g_attn_tc & 32) && (s->D.hd == 128 || s->D.hd == 64);
+}
+// H * sum over sequences of attn_ds_tiles(L) <= H * T * (1 + max_seq_len / 16384) for any split of T tokens into
+// sequences of at most max_seq_len (attn_ds_tiles(L) <= L + L^2 / 16384), capped by the chunk budget
+static long long ds_tiles_bound(const menos_server* s, long long T) {
+  if (!ds_path_on(s) || T <= 0) return 0;
+  const double per = 1.0 + s->opts.max_seq_len / 16384.0;
+  return std::min(g_attn_ds_cap_tiles, (long long)std::ceil((double)s->D.H * (double)T * per));
+}
 
 extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t* ids, const int32_t* n_tokens,
                                   int flags, size_t* fwd_bytes, size_t* bwd_bytes) {
@@ -972,8 +1004,12 @@ extern "C" int menos_batch_memory(menos_server* s, int n_clients, const int32_t*
   // forward: scratch (+ the NOGRAD layer set) + slab (+ meta); backward of a NOGRAD batch re-forwards with SAVE
   if (Text > (1ll << 30)) FAIL(MENOS_EINVAL, "too many tokens");
   const int Tx = (int)Text;
-  const size_t fwd = scratch_bytes_of(D, (int)T, R, nograd, Tx) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, !nograd, Tx) + meta;
-  const size_t bwd = scratch_bytes_of(D, (int)T, R, nograd, Tx) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, true, Tx) +
+  // dS-stored attention backward (no prefix clients): a bound on the chunk buffer without the sequence lengths
+  bool pfx = false;
+  for (int i = 0; i < n_clients; ++i) pfx = pfx || s->clients[ids[i]].n_prefix > 0;
+  const long long dst = pfx ? 0 : ds_tiles_bound(s, T);
+  const size_t fwd = scratch_bytes_of(D, (int)T, R, nograd, Tx, dst) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, !nograd, Tx) + meta;
+  const size_t bwd = scratch_bytes_of(D, (int)T, R, nograd, Tx, dst) + slab_bytes_of(D, s->n_layers, (int)T, R, save_a, true, Tx) +
                      (nograd ? slab_bytes_of(D, s->n_layers, (int)T, R, save_a, false, Tx) : 0) + 2 * meta;
   if (fwd_bytes) *fwd_bytes = fwd;
   if (bwd_bytes) *bwd_bytes = bwd;
@@ -1135,6 +1171,7 @@ struct Scratch {
   float *D_x, *dqacc_x;
   float* Dsum;
   float* wsp;                        // fused dU + dB: per-slab fp32 dU partials (one group at a time)
+  bf16* ds;                          // dS-stored attention backward: bf16 dS^T tiles of one chunk (or nullptr)
   bf16* dU[NG];
 };
 
@@ -1170,6 +1207,8 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
     b->Text += b->ext_len[i];
     b->pairs_ext += 0.5 * (double)b->ext_len[i] * (b->ext_len[i] + 1);
   }
+  b->ds_tiles = (ds_path_on(s) && !b->has_pfx)
+                    ? std::min(g_attn_ds_cap_tiles, attn_ds_total_tiles(b->seq_len.data(), n_seqs, D.H)) : 0;
   if (b->has_pfx) {
     if (D.sp) FAIL(MENOS_EINVAL, "prefix tuning is not supported with tensor parallelism");
     for (int c : b->bclients)
@@ -1205,6 +1244,7 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   (void)D;
   // small-GEMM problem lists are filled later (need layer buffers); reserve host vectors here
   b->sg_fwd.resize((size_t)s->n_layers * NG);
+  b->sg_shk.assign((size_t)s->n_layers * NG, menos_batch::ShkList());
   b->sg_dub.resize((size_t)s->n_layers * NG);
   b->sg_da.resize((size_t)s->n_layers * NG);
 
@@ -1244,7 +1284,7 @@ static size_t wsp_bytes_of(const Dims& D, int T, const int R_used[NG]) {
   return w * (size_t)T;
 }
 
-static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text) {
+static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool nograd_set, int Text, long long ds_tiles) {
   size_t need = 0;
   auto A = [&](size_t n) { need += align_up(n, 256); };
   const Rows Rw = rows_of(D, T);
@@ -1266,6 +1306,7 @@ static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool 
     A((size_t)T * D.gu_cols * 2); A((size_t)D.H * std::max(T, Text) * 4); A((size_t)Rw.Tloc * 8); A(dp);
     for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   }
+  A((size_t)ds_tiles * kDsTileBytes);   // dS-stored attention backward: the chunk buffer, last
   return need;
 }
 // generous bound of a batch's metadata block (segment tables, positions, tile maps, LoRA problem lists)
@@ -1297,6 +1338,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->views.clear();
   b->view_of.assign(Ls, -1);
   std::vector<std::vector<int4>> v_items, v_items_kv, v_items_q, v_items_seq;
+  std::vector<AttnDsPlan> v_ds;
   for (int l = 0; l < Ls; ++l) {
     const int ns = b->nseq_l[l];
     if (ns == 0) continue;
@@ -1317,6 +1359,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     v.n_items = (int)v_items.back().size();
     v.n_items_kv = (int)v_items_kv.back().size();
     v.n_items_seq = (int)v_items_seq.back().size();
+    v_ds.emplace_back();
+    if (b->ds_tiles > 0) {
+      v.ds_ok = attn_ds_plan(b->seq_len.data(), ns, D.H, D.Hkv, b->ds_tiles, v_ds.back());
+      if (v.ds_ok) v.ds_chunks = v_ds.back().chunks;
+    }
     b->views.push_back(v);
     b->view_of[l] = (int)b->views.size() - 1;
   }
@@ -1354,6 +1401,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->views[v].o_items_kv = put(v_items_kv[v].data(), v_items_kv[v].size() * sizeof(int4));
     b->views[v].o_items_q = put(v_items_q[v].data(), v_items_q[v].size() * sizeof(int4));
     b->views[v].o_items_seq = put(v_items_seq[v].data(), v_items_seq[v].size() * sizeof(int4));
+    if (b->views[v].ds_ok) {
+      b->views[v].o_ds_kv = put(v_ds[v].items_kv.data(), v_ds[v].items_kv.size() * sizeof(int4));
+      b->views[v].o_ds_q = put(v_ds[v].items_q.data(), v_ds[v].items_q.size() * sizeof(int4));
+      b->views[v].o_ds_base = put(v_ds[v].base.data(), v_ds[v].base.size() * sizeof(int));
+    }
   }
   // prefix tuning: the extended batch's segment tables, row maps and attention work lists (one view)
   size_t o_xcu = 0, o_xblk = 0, o_xblk128 = 0, o_xsrc = 0, o_xtok = 0, o_tokx = 0, o_seqx = 0, o_pc = 0, o_seqsh = 0;
@@ -1441,6 +1493,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   std::vector<LoraTokRedProblem> tprobs;
   std::vector<int4> ttiles;
   std::vector<LoraDUBProblem> dprobs;
+  std::vector<LoraShrinkProblem> sprobs;
+  std::vector<int2> stiles;
   auto add_rows = [&](SGList& L, const std::vector<LoraRowsProblem>& ps) {
     L.probs_off = (int)rprobs.size(); L.n_probs = (int)ps.size(); L.tiles_off = (int)rtiles.size();
     std::vector<int2> tl;
@@ -1457,7 +1511,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     lora_tokred_tiles(ps.data(), (int)ps.size(), mt, nt, tl);
     for (auto& x : tl) x.x += L.probs_off;
     for (const auto& pp : ps) L.flops += 2.0 * pp.M * pp.N * pp.T;
-    L.n_tiles = (int)tl.size(); L.max_n = mt;
+    L.n_tiles = (int)tl.size(); L.max_n = mt; L.tile_n = nt;
     tprobs.insert(tprobs.end(), ps.begin(), ps.end());
     ttiles.insert(ttiles.end(), tl.begin(), tl.end());
   };
@@ -1479,6 +1533,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         case GD: X = S.a; ldx = D.fpad; dY = dyl; ldy = D.d; break;
       }
       std::vector<LoraRowsProblem> f;
+      std::vector<LoraShrinkProblem> shk;
       std::vector<LoraDUBProblem> dub;
       std::vector<LoraTokRedProblem> da;
       size_t woff = 0;   // fp32 offset of the next problem's dU partials in sc.wsp (the group's lists run in turn)
@@ -1497,6 +1552,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           p.C = U + (size_t)t0 * R + col; p.ldc = R;
           p.M = Tc; p.N = w; p.K = D.K_g[g]; p.scale = c.s;
           f.push_back(p);
+          shk.push_back(LoraShrinkProblem{t0, Tc, col, w, c.s});
         }
         // per target, ONE pass over its dY columns: dB = dY_t^T (s U_t) and dU_t = s dY_t B_t (per-slab partials,
         // then a fixed-order slab sum); targets own contiguous (gate/up: 128-interleaved) row ranges of Bcat
@@ -1535,6 +1591,19 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       const size_t li = (size_t)l * NG + g;
       add_rows(b->sg_fwd[li], f);
       {
+        menos_batch::ShkList& H = b->sg_shk[li];
+        H.X = X; H.x_rows = T; H.ldx = ldx; H.A = s->Acat[g][l]; H.a_rows = s->cols[g].cap; H.lda = D.ldK_g[g];
+        H.K = D.K_g[g]; H.U = U; H.ldu = R;
+        H.probs_off = (int)sprobs.size(); H.tiles_off = (int)stiles.size();
+        std::vector<int2> tl;
+        lora_shrink_tiles(shk.data(), (int)shk.size(), tl);
+        for (auto& x : tl) x.x += H.probs_off;
+        for (const auto& q : shk) { H.max_w = std::max(H.max_w, q.w); H.flops += 2.0 * q.T * q.w * H.K; }
+        H.n_tiles = (int)tl.size();
+        sprobs.insert(sprobs.end(), shk.begin(), shk.end());
+        stiles.insert(stiles.end(), tl.begin(), tl.end());
+      }
+      {
         SGList& Ld = b->sg_dub[li];
         Ld.probs_off = (int)dprobs.size(); Ld.n_probs = (int)dub.size();
         for (const auto& q : dub) {
@@ -1546,6 +1615,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         dprobs.insert(dprobs.end(), dub.begin(), dub.end());
       }
       const int da_mt = da_w <= 16 ? 16 : da_w <= 32 ? 32 : 64;
+      // 128-column tiles: 64-column ones (twice the CTAs at cfg1) measured slower, 33.6 vs 28.6 us per layer (r2bf)
       add_tokred(b->sg_da[li], da, da_mt, 128);
     }
   }
@@ -1554,6 +1624,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_tp = put(tprobs.data(), tprobs.size() * sizeof(LoraTokRedProblem));
   const size_t o_tt = put(ttiles.data(), ttiles.size() * sizeof(int4));
   const size_t o_dp = put(dprobs.data(), dprobs.size() * sizeof(LoraDUBProblem));
+  const size_t o_sp = put(sprobs.data(), sprobs.size() * sizeof(LoraShrinkProblem));
+  const size_t o_st = put(stiles.data(), stiles.size() * sizeof(int2));
   uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
   if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
   b->meta = meta;
@@ -1575,6 +1647,9 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     v.items_kv = (int4*)(meta + v.o_items_kv);
     v.items_q = (int4*)(meta + v.o_items_q);
     v.items_seq = (int4*)(meta + v.o_items_seq);
+    if (v.ds_ok) {
+      v.ds_kv = (int4*)(meta + v.o_ds_kv); v.ds_q = (int4*)(meta + v.o_ds_q); v.ds_base = (int*)(meta + v.o_ds_base);
+    }
   }
   for (int g = 0; g < NG; ++g) b->d_mtile[g] = (int2*)(meta + o_mt) + (size_t)g * b->n_mt;
   b->d_ntile_qkv = meta + o_nt;
@@ -1586,6 +1661,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->d_tprobs = (LoraTokRedProblem*)(meta + o_tp);
   b->d_ttiles = (int4*)(meta + o_tt);
   b->d_dprobs = (LoraDUBProblem*)(meta + o_dp);
+  b->d_sprobs = (LoraShrinkProblem*)(meta + o_sp);
+  b->d_stiles = (int2*)(meta + o_st);
   b->h_dprobs = std::move(dprobs);
   return MENOS_OK;
 }
@@ -1593,9 +1670,10 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
 // scratch (per server, grown to the largest batch; used only inside one call)
 // nograd_set: also reserve the NOGRAD forward's layer buffers (only a MENOS_FWD_NOGRAD forward needs them; the
 // backward's re-forward writes into the batch's SAVE slab), so SAVE batches use exactly scratch_bytes_per_token
-static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set, int Text) {
+static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc, bool nograd_set, int Text,
+                       long long ds_tiles) {
   const Dims& D = s->D;
-  const size_t need = scratch_bytes_of(D, T, R_used, nograd_set, Text);
+  const size_t need = scratch_bytes_of(D, T, R_used, nograd_set, Text, ds_tiles);
   const Rows Rw = rows_of(D, T);
   const size_t df = (size_t)Rw.Tloc * D.d * 4, db = (size_t)Rw.Tloc * D.d * 2, dp = (size_t)Rw.Tpad * D.d * 2;
   if (need != s->scratch_bytes) {   // shrink-to-fit too: a stale large block must not outlive the call that needed it
@@ -1622,6 +1700,7 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   sc.Dsum = (float*)take((size_t)D.H * T * 4);
   sc.wsp = (float*)take(wsp_bytes_of(D, T, R_used));
   for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
+  sc.ds = ds_tiles > 0 ? (bf16*)(s->scratch + need - align_up((size_t)ds_tiles * kDsTileBytes, 256)) : nullptr;
   return MENOS_OK;
 }
 
@@ -1643,6 +1722,21 @@ static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scr
 // =====================================================================================================
 // per-layer schedules
 // =====================================================================================================
+// forward shrink U = s X A^T of one group's clients (tcgen05; MENOS_LORA_SHRINK_MMA=1: the mma.sync rows kernel)
+static int run_shrink(menos_batch* b, size_t li, cudaStream_t st) {
+  static const bool mma = [] { const char* e = getenv("MENOS_LORA_SHRINK_MMA"); return e && atoi(e) == 1; }();
+  const menos_batch::ShkList& H = b->sg_shk[li];
+  if (H.n_tiles == 0) return 0;
+  if (mma || H.max_w > 128) {
+    const SGList& L = b->sg_fwd[li];
+    if (L.n_tiles == 0) return 0;
+    ProfScope ps(PC_LORA, L.flops, 0, st);
+    return lora_rows_run(b->d_rprobs, b->d_rtiles + L.tiles_off, L.n_tiles, L.max_n, st);
+  }
+  ProfScope ps(PC_LORA, H.flops, 0, st);
+  return lora_shrink_tc_run(H.X, H.x_rows, H.ldx, H.A, H.a_rows, H.lda, H.K, b->d_sprobs, b->d_stiles + H.tiles_off,
+                            H.n_tiles, H.max_w, H.U, H.ldu, st);
+}
 static int run_rows(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
@@ -1659,7 +1753,7 @@ static int run_dub(menos_batch* b, const SGList& L, cudaStream_t st) {
 static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
-  return lora_tokred_run(b->d_tprobs, b->d_ttiles + L.tiles_off, L.n_tiles, L.max_n, st);
+  return lora_tokred_run(b->d_tprobs, b->d_ttiles + L.tiles_off, L.n_tiles, L.max_n, L.tile_n, st);
 }
 
 // tensor-parallel all-reduce (sum, in place, stream-ordered) through the caller's callback (menos_tp_cfg)
@@ -1709,7 +1803,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
   // A2: QKV GEMM (+ segmented LoRA q/k/v expand, + RoPE epilogue)
   if (b->g_active[GQKV]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GQKV], 0, (size_t)T * b->R_used[GQKV] * 2, st));
-    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GQKV], st));
+    if (use_lists) K_TRY(run_shrink(b, (size_t)l * NG + GQKV, st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1749,7 +1843,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
   // A4: O GEMM (+ LoRA o) + residual
   if (b->g_active[GO]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GO], 0, (size_t)T * b->R_used[GO] * 2, st));
-    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GO], st));
+    if (use_lists) K_TRY(run_shrink(b, (size_t)l * NG + GO, st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1779,7 +1873,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
   // A6: gate/up GEMM (+ LoRA gate/up) + SwiGLU epilogue
   if (b->g_active[GGU]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GGU], 0, (size_t)T * b->R_used[GGU] * 2, st));
-    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GGU], st));
+    if (use_lists) K_TRY(run_shrink(b, (size_t)l * NG + GGU, st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1795,7 +1889,7 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
   // A7: down GEMM (+ LoRA down) + residual
   if (b->g_active[GD]) {
     CUDA_TRY(cudaMemsetAsync(S.U[GD], 0, (size_t)T * b->R_used[GD] * 2, st));
-    if (use_lists) K_TRY(run_rows(b, b->sg_fwd[(size_t)l * NG + GD], st));
+    if (use_lists) K_TRY(run_shrink(b, (size_t)l * NG + GD, st));
   }
   {
     GemmArgs a = gemm_base(s);
@@ -1927,7 +2021,11 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     a.dq_acc = xp ? sc.dqacc_x : sc.xout;
     {
       ProfScope ps(PC_ATTN_BWD, 8.0 * D.hd * D.H * AV.pairs, 0, st);
-      if (D.hd == 128 && (g_attn_tc & 32))
+      if (!xp && AV.ds_ok && sc.ds) {   // S, P, dP once per pair: dK/dV (+ dS^T tiles), then dQ from the tiles
+        for (const int4& c : AV.ds_chunks)
+          K_TRY(attn_bwd_ws_ds(a, AV.ds_kv + c.x, c.y, AV.ds_q + c.z, c.w, sc.ds, b->ds_tiles, AV.ds_base,
+                               s->num_sms, st));
+      } else if (D.hd == 128 && (g_attn_tc & 32))
         K_TRY(attn_bwd_fused(a, AV.items_seq, AV.n_items_seq, s->num_sms, st));
       else if ((D.hd == 128 || D.hd == 64) && (g_attn_tc & 8))
         K_TRY(attn_bwd_ws(a, AV.items_kv, AV.n_items_kv, AV.items_q, AV.n_items, s->num_sms, st));
@@ -2007,7 +2105,7 @@ extern "C" int menos_forward(menos_server* s, int n_seqs, const int32_t* seq_cli
   const Dims& D = s->D;
   const int T = b->T;
   Scratch sc;
-  rc = get_scratch(s, T, b->R_used, sc, b->nograd, b->Text);
+  rc = get_scratch(s, T, b->R_used, sc, b->nograd, b->Text, b->ds_tiles);
   if (rc) return rc;
   LayerSave ng{};
   if (b->nograd) nograd_layer(s, T, b->R_used, sc, ng, b->Text);
@@ -2112,7 +2210,7 @@ extern "C" int menos_backward(menos_server* s, menos_batch* b, const void* g_c, 
   const int T = b->T;
   const Rows R = rows_of(D, T);
   Scratch sc;
-  int rc = get_scratch(s, T, b->R_used, sc, false, b->Text);
+  int rc = get_scratch(s, T, b->R_used, sc, false, b->Text, b->ds_tiles);
   if (rc) return rc;
   if (b->nograd) {
     // Alg.1 L10: re-forward with gradient preparation from the cached x_c; the SAVE slab is

@@ -1,4 +1,5 @@
 // Kernel-level test entry points (include/menos_testing.h): same kernels as the server path.
+#include <algorithm>
 #include <cmath>
 #include <cstring>
 #include <string>
@@ -126,9 +127,30 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
       cudaMalloc(&d_acc, (size_t)T * H * hd * sizeof(float));
       a.dq_acc = d_acc;
     }
-    rc = fused_bwd ? attn_bwd_fused(a, d_items_seq, (int)items_seq.size(), sms, 0)
-         : ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
-                  : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+    // bit 6: the dS-stored backward, chunked under g_attn_ds_cap_tiles exactly as the server runs it
+    AttnDsPlan plan;
+    const bool ds_bwd = ws_bwd && !fused_bwd && (g_attn_tc & 64) &&
+                        attn_ds_plan(seq_len, n_seqs, H, Hkv, g_attn_ds_cap_tiles, plan);
+    if (ds_bwd) {
+      const long long cap = std::min(g_attn_ds_cap_tiles, attn_ds_total_tiles(seq_len, n_seqs, H));
+      bf16* d_ds; int* d_base; int4 *d_ikv, *d_iq;
+      cudaMalloc(&d_ds, (size_t)std::max(1LL, cap) * 128 * 64 * 2);
+      cudaMalloc(&d_base, std::max<size_t>(1, plan.base.size()) * 4);
+      cudaMalloc(&d_ikv, std::max<size_t>(1, plan.items_kv.size()) * sizeof(int4));
+      cudaMalloc(&d_iq, std::max<size_t>(1, plan.items_q.size()) * sizeof(int4));
+      cudaMemcpy(d_base, plan.base.data(), plan.base.size() * 4, cudaMemcpyHostToDevice);
+      cudaMemcpy(d_ikv, plan.items_kv.data(), plan.items_kv.size() * sizeof(int4), cudaMemcpyHostToDevice);
+      cudaMemcpy(d_iq, plan.items_q.data(), plan.items_q.size() * sizeof(int4), cudaMemcpyHostToDevice);
+      rc = 0;
+      for (const int4& c : plan.chunks)
+        if (!rc) rc = attn_bwd_ws_ds(a, d_ikv + c.x, c.y, d_iq + c.z, c.w, d_ds, cap, d_base, sms, 0);
+      cudaDeviceSynchronize();
+      cudaFree(d_ds); cudaFree(d_base); cudaFree(d_ikv); cudaFree(d_iq);
+    } else {
+      rc = fused_bwd ? attn_bwd_fused(a, d_items_seq, (int)items_seq.size(), sms, 0)
+           : ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
+                    : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+    }
     cudaDeviceSynchronize();
     cudaFree(d_items_kv); cudaFree(d_acc); cudaFree(d_items_seq);
   }
@@ -182,7 +204,7 @@ extern "C" int menos_test_lora_tokred(const void* P, const void* Q, float* C, in
   cudaMalloc(&dt, tiles.size() * sizeof(int4) + 16);
   cudaMemcpy(dp, &p, sizeof p, cudaMemcpyHostToDevice);
   cudaMemcpy(dt, tiles.data(), tiles.size() * sizeof(int4), cudaMemcpyHostToDevice);
-  int rc = lora_tokred_run(dp, dt, (int)tiles.size(), mt, 0);
+  int rc = lora_tokred_run(dp, dt, (int)tiles.size(), mt, mt == 128 ? 16 : 128, 0);
   cudaError_t e = cudaDeviceSynchronize();
   cudaFree(dp); cudaFree(dt);
   if (rc) return fail("lora tokred rejected");
@@ -229,17 +251,27 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
 // Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward (2-pass, serialized), 2 = tcgen05 backward
 // (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1),
 // 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; overrides 2).
-// Default 14: the persistent tcgen05 forward and backward (LPT work order, bit 4 selects (sequence, head) order).
-namespace menos { int g_attn_tc = 14; int g_attn_order = 1; }
+// 64 = with 8: the dK/dV kernel stores dS^T and dQ is computed from it (S, P, dP once per pair; chunked under
+// g_attn_ds_cap_tiles, 16 KB tiles).
+// Default 78: the persistent tcgen05 forward and the dS-stored persistent backward (LPT work order, bit 4 selects
+// (sequence, head) order).
+namespace menos { int g_attn_tc = 78; int g_attn_order = 1; long long g_attn_ds_cap_tiles = 32768; }
 extern "C" int menos_test_abf_prof(unsigned long long* out16) {
   if (!out16) return fail("null output");
   return menos::attn_bwd_fused_prof(out16);
 }
 
 extern "C" int menos_test_set_attn_tc(int mode) {
-  if (mode < 0 || mode > 63) { fail("attention mode must be in [0, 63]"); return MENOS_EINVAL; }
+  if (mode < 0 || mode > 127) { fail("attention mode must be in [0, 127]"); return MENOS_EINVAL; }
   menos::g_attn_order = (mode & 16) ? 0 : 1;   // bit 4: (sequence, head)-grouped work order instead of LPT
-  mode &= 47;                                  // bit 5: one-pass fused backward
+  mode &= 111;                                 // bit 5: one-pass fused backward; bit 6: dS-stored backward
   menos::g_attn_tc = mode;
+  return MENOS_OK;
+}
+
+// dS-stored backward: tile budget of one chunk (16 KB tiles; default 32768 = 512 MB); small values force chunking
+extern "C" int menos_test_set_ds_cap(long long tiles) {
+  if (tiles < 1) { fail("ds cap must be >= 1 tile"); return MENOS_EINVAL; }
+  menos::g_attn_ds_cap_tiles = tiles;
   return MENOS_OK;
 }

@@ -244,7 +244,8 @@ def test_gemm_swiglu_fwd_and_bwd_epilogues():
     assert maxrel(got_u, du) < 1.5e-2
 
 
-DEFAULT_ATTN_MODE = 14   # testing.cu g_attn_tc default: persistent tcgen05 forward + two-kernel persistent backward
+DEFAULT_ATTN_MODE = 78   # testing.cu g_attn_tc default: persistent tcgen05 forward + dS-stored persistent backward
+DEFAULT_DS_CAP = 32768   # testing.cu g_attn_ds_cap_tiles default (512 MB of 16 KB dS^T tiles)
 
 
 @pytest.fixture(autouse=True)
@@ -254,6 +255,7 @@ def _restore_attention_mode():
     yield
     from paper_conf_middleware_hul24_b200.menos import check
     check(lib().menos_test_set_attn_tc(DEFAULT_ATTN_MODE), testing=True)
+    check(lib().menos_test_set_ds_cap(DEFAULT_DS_CAP), testing=True)
 
 
 @pytest.mark.parametrize("hd,H,Hkv,lens,tc", [(128, 4, 2, [1, 17, 64, 129, 300], 46), (128, 8, 1, [130, 7, 256], 46),
@@ -269,9 +271,27 @@ def _restore_attention_mode():
                                              (128, 4, 2, [1, 17, 64, 129, 300], 2), (128, 8, 1, [130, 7, 256], 3),
                                              (128, 2, 2, [512, 1024, 255], 3), (128, 2, 2, [512, 1024, 255], 0),
                                              (16, 4, 4, [16, 16, 3], 3), (64, 8, 1, [200, 65], 3),
-                                             (128, 4, 4, [1, 17, 64, 129, 300], -14), (64, 4, 4, [200, 65], -3)])
+                                             (128, 4, 4, [1, 17, 64, 129, 300], -14), (64, 4, 4, [200, 65], -3),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 78), (128, 8, 1, [130, 7, 256], 78),
+                                             (128, 2, 2, [512, 1024, 255], 78), (128, 3, 1, [2048, 1, 700], 78),
+                                             (128, 8, 8, [512] * 16 + [77], 78), (128, 4, 4, [1, 17, 64, 129, 300], -78),
+                                             (64, 8, 1, [200, 65, 1], 78), (64, 4, 4, [200, 65, 1000, 3], -78)])
 def test_attention_fwd_bwd(hd, H, Hkv, lens, tc):
     """tc < 0: kernel variant |tc| with no RoPE (theta 0: the OPT path, NEXT-4)."""
+    _attention_case(hd, H, Hkv, lens, tc)
+
+
+@pytest.mark.parametrize("hd,cap", [(128, 80), (64, 80), (128, 9)])
+def test_attention_ds_chunked(hd, cap):
+    """dS-stored backward with a chunk budget far below the batch's tiles: (sequence, kv head) units are packed into
+    several chunks (two launches each) that reuse one buffer; a unit larger than the budget (cap 9 with the 700-token
+    sequence) falls back to the recompute path for the whole call."""
+    from paper_conf_middleware_hul24_b200.menos import check
+    check(lib().menos_test_set_ds_cap(cap), testing=True)
+    _attention_case(hd, 4, 2, [300, 129, 17, 700, 64, 1], 78)
+
+
+def _attention_case(hd, H, Hkv, lens, tc):
     rope = tc >= 0
     tc = abs(tc)
     from paper_conf_middleware_hul24_b200.menos import check
