@@ -62,9 +62,9 @@ MENOS_API int menos_test_set_gemm_cta_group(int cta_group);
 MENOS_API int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A, const void* B, void* out, int epi,
                                    const void* aux, int iters, float* ms_out);
 
-/* Attention kernels for head_dim 128, bitmask: bit 0 = tcgen05 forward (else mma.sync),
-   bit 1 = tcgen05 backward (else mma.sync), bit 2 = persistent warp-specialized tcgen05 forward (overrides
-   bit 0), bit 3 = persistent warp-specialized tcgen05 backward (overrides bit 1), bit 4 = (sequence, head)-grouped
+/* Attention kernels for head_dim 128 / 64, bitmask: bits 0, 1 = ignored (round-1 non-persistent tcgen05 kernels,
+   removed), bit 2 = persistent warp-specialized tcgen05 forward (else mma.sync), bit 3 = persistent
+   warp-specialized tcgen05 backward (else mma.sync), bit 4 = (sequence, head)-grouped
    work order instead of LPT, bit 5 = one-pass fused tcgen05 backward (overrides bits 3 and 1), bit 6 (with bit 3)
    = dS-stored backward: the dK/dV kernel also stores bf16 dS^T tiles and dQ = dS K is computed from them, so S, P and
    dP are evaluated once per (key, query) pair.  Default mode 78 (persistent forward + dS-stored

@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OUT_DIR = os.path.join(HERE, "_lib")
 LIB = os.path.join(OUT_DIR, "libmenos.so")
-SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_tc.cu", "attention_fwd_ws.cu", "attention_bwd_tc.cu", "attention_bwd_ws.cu", "attention_bwd_fused.cu", "lora.cu", "prefix.cu", "elementwise.cu", "server.cu", "testing.cu", "sched.cpp", "comm.cpp"]
+SOURCES = ["gemm_tcgen05.cu", "attention.cu", "attention_fwd_ws.cu", "attention_bwd_ws.cu", "attention_bwd_fused.cu", "lora.cu", "prefix.cu", "elementwise.cu", "server.cu", "testing.cu", "sched.cpp", "comm.cpp"]
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"),

@@ -666,6 +666,20 @@ bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols,
   return get_map(out, ptr, rows, cols, ld, bc, br);
 }
 
+// row-major [rows, cols] bf16, no swizzle (small boxes staged linearly, e.g. a [128][16] LoRA U tile); not cached
+bool tma_map_2d_plain(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
+                      uint32_t br) {
+  PFN_encodeTiled_t enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {ld * 2};
+  cuuint32_t box[2] = {bc, br};
+  cuuint32_t es[2] = {1, 1};
+  return enc(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 int gemm_run(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0 || a.K <= 0) return 0;
   if (a.N % 32 != 0 || (a.lda % 8) || (a.ldb % 8) || (a.ldo % 8)) return -1;

@@ -76,7 +76,12 @@ struct LoraTokRedProblem {
   float scale;
   float* C1; float* C2;
   int m_seg, m_valid;
+  int t0, pcol0;   // tcgen05 dA: the client's first row and its dU slot column in the whole buffers
 };
+// dA on tcgen05 (lists of per-(client, group) problems with M = slot width <= 64): dA_seg[m % m_seg][k] =
+// sum_t dU[t0 + t, pcol0 + m] X[t0 + t, k]; X [rows, ldx] and dU [rows, lddu] are whole buffers
+int lora_da_tc_run(const LoraTokRedProblem* d_probs, int n_probs, int max_n, int max_w, const bf16* X, int rows,
+                   int ldx, const bf16* dU, int lddu, cudaStream_t st);
 // fused dU + dB of one (client, target) in ONE pass over its dY columns:
 //   dB[m, n]  = sum_t dY[t, map(m)] U[t, n]                                  (fp32 [Nt, rank], overwrite)
 //   W[s][t,n] = sum_{m in slab s} dY[t, map(m)] B[map(m), n]                 (fp32 partials, [n_slabs][T][rank])
@@ -87,6 +92,7 @@ struct LoraDUBProblem {
   float* dB; float* W; bf16* dU;
   int Nt, rank, rs, T, ldy, ldu, ldb, lddu, p_blk, p_blk_stride, n_slabs;
   float scale;
+  int t0, ycol0, ucol0;   // tcgen05 variant: the problem's first row and its dY / U columns in the whole buffers
 };
 int lora_rows_run(const LoraRowsProblem* d_probs, const int2* d_tiles, int n_tiles, int max_n, cudaStream_t st);
 int lora_tokred_run(const LoraTokRedProblem* d_probs, const int4* d_tiles, int n_tiles, int mt, int nt, cudaStream_t st);
@@ -104,6 +110,10 @@ int lora_shrink_tc_run(const bf16* X, int x_rows, int ldx, const bf16* Acat, int
 constexpr int LORA_DUB_MT = 128;
 // grid: (max n_slabs * ceil(max rank / 16), n_probs); CTAs past a problem's slabs exit
 int lora_dub_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, int max_rank, cudaStream_t st);
+// tcgen05 variant (rank <= 16): the same contract; dY [y_rows, ldy] and U [y_rows, ldu] are the whole buffers the
+// problems index with (t0, ycol0) / (t0, ucol0); 128-token stages by TMA, dB and the per-stage dU share on tcgen05
+int lora_dub_tc_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, const bf16* dY, int y_rows, int ldy,
+                    const bf16* U, int ldu, cudaStream_t st);
 // grid: (ceil(max T * rs / 256), n_probs)
 int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max_elems, cudaStream_t st);
 
@@ -152,8 +162,6 @@ struct AttnArgs {
   const int* pos_shift;          // [n_seqs] or nullptr
 };
 int attn_fwd(const AttnArgs& a, cudaStream_t st);
-// tcgen05 forward for head_dim 128 (attention_tc.cu); qblocks128 = (seq, local start) per 128-row q block
-int attn_fwd_tc(const AttnArgs& a, const int2* qblocks128, int n_qblocks128, cudaStream_t st);
 // persistent warp-specialized tcgen05 forward for head_dim 128 (attention_fwd_ws.cu); items = (seq, q0, head, -)
 int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st);
 // order: 0 = (sequence, head) groups (L2 locality), 1 = largest forward / dQ work first, 2 = largest dK/dV first
@@ -184,14 +192,13 @@ extern long long g_attn_ds_cap_tiles;
 int attn_bwd_fused(const AttnArgs& a, const int4* items_seq, int n_items, int num_sms, cudaStream_t st);
 void attn_seq_items(const int* seq_len, int n_seqs, int Hkv, std::vector<int4>& out);
 int attn_bwd_fused_prof(unsigned long long* out16);   // tuning: per-phase cycles (-DMENOS_ABF_PROF builds)
-// head_dim 128 variant bitmask: 1 = tcgen05 forward (2-pass), 2 = tcgen05 backward, 4 = persistent
-// warp-specialized tcgen05 forward (takes precedence over 1), 8 = persistent warp-specialized tcgen05 backward
-// (takes precedence over 2), 32 = one-pass fused tcgen05 backward (takes precedence over 8 and 2)
+// head_dim 128 / 64 variant bitmask: 4 = persistent warp-specialized tcgen05 forward, 8 = persistent
+// warp-specialized tcgen05 backward, 64 (with 8) = the dS-stored backward, 32 = one-pass fused tcgen05 backward
+// (head_dim 128; takes precedence over 8); without 4 / 8 the mma.sync kernels (attention.cu)
 extern int g_attn_tc;
 extern int g_attn_order;   // persistent attention work order: 1 = LPT (default), 0 = (sequence, head) grouped
 int attn_bwd(const AttnArgs& a, cudaStream_t st);
-// tcgen05 backward for head_dim 128 (attention_bwd_tc.cu); blocks128 = (seq, local start) per 128-row block
-int attn_bwd_tc(const AttnArgs& a, const int2* blocks128, int n_blocks128, cudaStream_t st);
+
 
 // ---------------------------------------------------------------- prefix tuning (prefix.cu; NEXT-3, R28)
 struct PrefixClient {        // one prefix-tuning client of a batch

@@ -402,6 +402,24 @@ __global__ void __launch_bounds__(128) lora_dub_kernel(const LoraDUBProblem* __r
 // dU[t, n] = bf16(scale * sum over slabs, in slab order, of W[s][t, n]); zero in the slot's padding columns
 __global__ void __launch_bounds__(256) lora_du_reduce_kernel(const LoraDUBProblem* __restrict__ probs) {
   const LoraDUBProblem P = probs[blockIdx.y];
+  if ((P.rank & 3) == 0 && (P.rs & 3) == 0 && (P.lddu & 3) == 0 && (reinterpret_cast<uintptr_t>(P.W) & 15) == 0) {
+    const long long e4 = (long long)blockIdx.x * 256 + threadIdx.x;
+    if (e4 * 4 >= (long long)P.T * P.rs) return;
+    const int tok = (int)(e4 * 4 / P.rs), n = (int)(e4 * 4 % P.rs);
+    float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (n < P.rank) {
+      const float4* w = reinterpret_cast<const float4*>(P.W + (size_t)tok * P.rank + n);
+      const size_t step = (size_t)P.T * P.rank / 4;
+#pragma unroll 8
+      for (int i = 0; i < P.n_slabs; ++i) {
+        const float4 v = w[i * step];
+        a.x += v.x; a.y += v.y; a.z += v.z; a.w += v.w;
+      }
+    }
+    uint2 o = make_uint2(pack_bf16x2(a.x * P.scale, a.y * P.scale), pack_bf16x2(a.z * P.scale, a.w * P.scale));
+    *reinterpret_cast<uint2*>(P.dU + (size_t)tok * P.lddu + n) = o;
+    return;
+  }
   const long long e = (long long)blockIdx.x * 256 + threadIdx.x;
   if (e >= (long long)P.T * P.rs) return;
   const int tok = (int)(e / P.rs), n = (int)(e % P.rs);
@@ -517,6 +535,310 @@ lora_shrink_tc_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_cons
   }
 }
 
+// ============================================================================ fused dU + dB on tcgen05
+// Same contract as lora_dub_kernel for rank <= 16, with the contractions on the 5th-gen tensor cores: CTA = (problem,
+// 128-column slab), 128-token stages.  One staged dY tile [128 tokens][128 columns] (two TMA boxes, 128-byte
+// swizzle) is BOTH the MN-major A operand of dB[slab] += dY^T U (M = 128 columns, K = tokens) and the K-major A
+// operand of this slab's dU share W = dY B_slab (M = 128 tokens, K = columns); the two small B operands (U^T of the
+// stage, B_slab^T once) are transposed by the epilogue warps into K-major swizzled tiles.  dB accumulates in TMEM
+// over all stages; each stage's dU share lands in one of two TMEM buffers and is written out as fp32 partial rows
+// while the next stage runs.  Rows past the client's tokens and columns past the target's are zeroed in the
+// transposed operands, so they contribute nothing.
+constexpr int DUBT_BK = 128, DUBT_ST = 2;
+constexpr int DUBT_Y = 128 * 128 * 2;            // dY stage: two [128 rows][64 cols] atoms
+constexpr int DUBT_U = 128 * 16 * 2;             // U stage, linear [128][16]
+constexpr int DUBT_T = 16 * 128 * 2;             // transposed [16][128] K-major tile (two [16][64] atoms)
+constexpr int DUBT_STAGE = DUBT_Y + DUBT_U + DUBT_T;
+constexpr int DUBT_SMEM = DUBT_ST * DUBT_STAGE + DUBT_T + 1024;
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+// the first `rank` (<= 16) of 16 fp32 values -> dst; 16-byte stores when rank % 4 == 0 and dst is aligned
+__device__ __forceinline__ void store_row16(float* dst, const uint32_t (&r)[16], int rank) {
+  if ((rank & 3) == 0 && (reinterpret_cast<uintptr_t>(dst) & 15) == 0) {
+#pragma unroll
+    for (int n = 0; n < 16; n += 4)
+      if (n < rank) *reinterpret_cast<uint4*>(dst + n) = make_uint4(r[n], r[n + 1], r[n + 2], r[n + 3]);
+  } else {
+#pragma unroll
+    for (int n = 0; n < 16; ++n)
+      if (n < rank) dst[n] = __uint_as_float(r[n]);
+  }
+}
+// element (row n < 16, k < 128) of a K-major [16][128] bf16 tile in two 128-byte-swizzled [16][64] atoms
+__device__ __forceinline__ uint32_t kt_off(int n, int k) {
+  return (uint32_t)((k >> 6) * 2048 + n * 128 + ((((k & 63) >> 3) ^ (n & 7)) << 4) + (k & 7) * 2);
+}
+
+__global__ void __launch_bounds__(192, 2)
+lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmU,
+                   const LoraDUBProblem* __restrict__ probs) {
+  extern __shared__ uint8_t dubt_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(dubt_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* const sBT = smem + DUBT_ST * DUBT_STAGE;
+  __shared__ __align__(8) uint64_t full[DUBT_ST], empty[DUBT_ST], ut_full[DUBT_ST], bt_ready, du_full[2], du_free[2],
+      db_full;
+  __shared__ uint32_t tmem_sh;
+  const LoraDUBProblem P = probs[blockIdx.y];
+  const int slab = blockIdx.x;
+  if (slab >= P.n_slabs) return;
+  const int m0 = slab * 128, nst = (P.T + DUBT_BK - 1) / DUBT_BK;
+  const int pcol0 = (m0 / P.p_blk) * P.p_blk_stride + m0 % P.p_blk;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmY); tma_prefetch(&tmU);
+    for (int i = 0; i < DUBT_ST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); mbar_init(&ut_full[i], 4); }
+    mbar_init(&bt_ready, 4);
+    for (int i = 0; i < 2; ++i) { mbar_init(&du_full[i], 1); mbar_init(&du_free[i], 4); }
+    mbar_init(&db_full, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<64>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;   // dB at column 0, dU buffers at 16 / 32
+  if (warp == 0) {
+    if (elect_one()) {
+      for (int s = 0; s < nst; ++s) {
+        const int st = s % DUBT_ST;
+        mbar_wait(&empty[st], ((s / DUBT_ST) & 1) ^ 1);
+        mbar_expect_tx(&full[st], DUBT_Y + DUBT_U);
+        uint8_t* sy = smem + st * DUBT_STAGE;
+        const int row = P.t0 + s * DUBT_BK;
+        tma_load_2d(sy, &tmY, &full[st], P.ycol0 + pcol0, row);
+        tma_load_2d(sy + 16384, &tmY, &full[st], P.ycol0 + pcol0 + 64, row);
+        tma_load_2d(sy + DUBT_Y, &tmU, &full[st], P.ucol0, row);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    constexpr uint32_t ID_DB = umma_idesc_bf16(128, 16, 0) | (1u << 15);   // A (dY^T) MN-major, B (U^T) K-major
+    constexpr uint32_t ID_DU = umma_idesc_bf16(128, 16, 0);                // A (dY) K-major, B (B_slab^T) K-major
+    mbar_wait(&bt_ready, 0);
+    for (int s = 0; s < nst; ++s) {
+      const int st = s % DUBT_ST, b = s & 1;
+      mbar_wait(&full[st], (s / DUBT_ST) & 1);
+      mbar_wait(&ut_full[st], (s / DUBT_ST) & 1);
+      mbar_wait(&du_free[b], ((s >> 1) & 1) ^ 1);
+      tc_fence_after();
+      __syncwarp();
+      if (elect_one()) {
+        const uint32_t sy = smem_u32(smem + st * DUBT_STAGE), sut = sy + DUBT_Y + DUBT_U, sbt = smem_u32(sBT);
+#pragma unroll
+        for (int kk = 0; kk < DUBT_BK / 16; ++kk)   // dB: K = 16 tokens = 16 rows of both dY atoms, of U^T
+          tc_mma_bf16(tmem, umma_desc_sw128(sy + kk * 2048, 16384, 1024),
+                      umma_desc_sw128(sut + (kk >> 2) * 2048 + (kk & 3) * 32, 16, 1024), ID_DB,
+                      (s > 0 || kk > 0) ? 1u : 0u);
+#pragma unroll
+        for (int kk = 0; kk < 128 / 16; ++kk)       // dU share: K = 16 slab columns
+          tc_mma_bf16(tmem + 16 + 16 * b, umma_desc_sw128(sy + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
+                      umma_desc_sw128(sbt + (kk >> 2) * 2048 + (kk & 3) * 32, 16, 1024), ID_DU, kk > 0 ? 1u : 0u);
+        tc_commit(&empty[st]);
+        tc_commit(&du_full[b]);
+        if (s == nst - 1) tc_commit(&db_full);
+      }
+      __syncwarp();
+    }
+  } else {
+    const int q = warp & 3, row = q * 32 + lane;   // TMEM lane quadrant; row = token (dU) / slab column (dB)
+    const uint32_t loff = (uint32_t)(q * 32) << 16;
+    {   // B_slab^T [16][128]: row n = rank column n, k = slab column; zero past the target's columns / the rank
+      const bool ok = m0 + row < P.Nt;
+      const uint4* src = reinterpret_cast<const uint4*>(P.B + (size_t)(pcol0 + row) * P.ldb);
+      uint4 v0 = ok ? src[0] : make_uint4(0, 0, 0, 0), v1 = ok ? src[1] : make_uint4(0, 0, 0, 0);
+      const bf16* e0 = reinterpret_cast<const bf16*>(&v0);
+      const bf16* e1 = reinterpret_cast<const bf16*>(&v1);
+      const bf16 z = __float2bfloat16_rn(0.f);
+#pragma unroll
+      for (int n = 0; n < 16; ++n)
+        *reinterpret_cast<bf16*>(sBT + kt_off(n, row)) = n < P.rank ? (n < 8 ? e0[n] : e1[n - 8]) : z;
+      fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bt_ready);
+    }
+    float* const Wb = P.W + (size_t)slab * P.T * P.rank;
+    auto du_out = [&](int s) {   // stage s's dU share -> fp32 partial rows
+      const int b = s & 1;
+      mbar_wait(&du_full[b], (s >> 1) & 1);
+      tc_fence_after();
+      uint32_t r[16];
+      tmem_ld16(tmem + 16 + 16 * b + loff, r);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&du_free[b]);
+      const int tok = s * DUBT_BK + row;
+      if (tok < P.T) store_row16(Wb + (size_t)tok * P.rank, r, P.rank);
+    };
+    for (int s = 0; s < nst; ++s) {
+      const int st = s % DUBT_ST;
+      mbar_wait(&full[st], (s / DUBT_ST) & 1);
+      {   // U^T [16][128 tokens] of this stage, zero past the client's tokens and the rank
+        const uint8_t* su = smem + st * DUBT_STAGE + DUBT_Y;
+        uint8_t* sut = smem + st * DUBT_STAGE + DUBT_Y + DUBT_U;
+        const bool ok = s * DUBT_BK + row < P.T;
+        uint4 v0 = ok ? reinterpret_cast<const uint4*>(su + row * 32)[0] : make_uint4(0, 0, 0, 0);
+        uint4 v1 = ok ? reinterpret_cast<const uint4*>(su + row * 32)[1] : make_uint4(0, 0, 0, 0);
+        const bf16* e0 = reinterpret_cast<const bf16*>(&v0);
+        const bf16* e1 = reinterpret_cast<const bf16*>(&v1);
+        const bf16 z = __float2bfloat16_rn(0.f);
+#pragma unroll
+        for (int n = 0; n < 16; ++n)
+          *reinterpret_cast<bf16*>(sut + kt_off(n, row)) = n < P.rank ? (n < 8 ? e0[n] : e1[n - 8]) : z;
+        fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&ut_full[st]);
+      }
+      if (s > 0) du_out(s - 1);
+    }
+    if (nst > 0) du_out(nst - 1);
+    mbar_wait(&db_full, 0);
+    tc_fence_after();
+    uint32_t r[16];
+    tmem_ld16(tmem + loff, r);
+    if (m0 + row < P.Nt) store_row16(P.dB + (size_t)(m0 + row) * P.rank, r, P.rank);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<64>(tmem);
+  }
+}
+
+// ============================================================================ dA on tcgen05
+// dA^T[k, m] = sum_t X[t, k] dU[t, m] for one client's group: CTA = (problem, 128 columns of X), 128-token stages.
+// The staged X tile [128 tokens][128 columns] (two TMA boxes, 128-byte swizzle) is the MN-major A operand (M = 128
+// columns, K = tokens); the stage's dU columns [128 tokens][NW] are transposed by the epilogue warps into a K-major
+// [NW][128] operand (rows past the client's tokens / slot width zeroed).  The [128 x NW] accumulator stays in TMEM
+// over all stages; one thread per column k writes it to every target's dA rows.
+constexpr int DAT_BK = 128;
+template <int NW> struct DatGeo {
+  static constexpr int X = 128 * 128 * 2, U = 128 * NW * 2, UT = NW * 128 * 2, STAGE = X + U + UT;
+  static constexpr int ST = (200 * 1024) / STAGE < 4 ? (200 * 1024) / STAGE : 4;   // ring of ~200 KB, <= 4 stages
+  static constexpr int SMEM = ST * STAGE + 1024;
+  static constexpr int TCOLS = NW < 32 ? 32 : NW;
+};
+
+template <int NW>
+__global__ void __launch_bounds__(192, 1)
+lora_da_tc_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmU,
+                  const LoraTokRedProblem* __restrict__ probs) {
+  using G = DatGeo<NW>;
+  constexpr int DAT_ST = G::ST;
+  extern __shared__ uint8_t dat_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(dat_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full[DAT_ST], empty[DAT_ST], ut_full[DAT_ST], acc_full;
+  __shared__ uint32_t tmem_sh;
+  const LoraTokRedProblem P = probs[blockIdx.y];
+  const int k0 = blockIdx.x * 128;
+  if (k0 >= P.N) return;
+  const int nst = (P.T + DAT_BK - 1) / DAT_BK;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    tma_prefetch(&tmX); tma_prefetch(&tmU);
+    for (int i = 0; i < DAT_ST; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); mbar_init(&ut_full[i], 4); }
+    mbar_init(&acc_full, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<G::TCOLS>(&tmem_sh);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_sh;
+  if (warp == 0) {
+    if (elect_one()) {
+      for (int s = 0; s < nst; ++s) {
+        const int st = s % DAT_ST;
+        mbar_wait(&empty[st], ((s / DAT_ST) & 1) ^ 1);
+        mbar_expect_tx(&full[st], G::X + G::U);
+        uint8_t* sx = smem + st * G::STAGE;
+        const int row = P.t0 + s * DAT_BK;
+        tma_load_2d(sx, &tmX, &full[st], k0, row);
+        tma_load_2d(sx + 16384, &tmX, &full[st], k0 + 64, row);
+        tma_load_2d(sx + G::X, &tmU, &full[st], P.pcol0, row);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    constexpr uint32_t ID = umma_idesc_bf16(128, NW, 0) | (1u << 15);   // A (X^T) MN-major, B (dU^T) K-major
+    for (int s = 0; s < nst; ++s) {
+      const int st = s % DAT_ST;
+      mbar_wait(&full[st], (s / DAT_ST) & 1);
+      mbar_wait(&ut_full[st], (s / DAT_ST) & 1);
+      tc_fence_after();
+      __syncwarp();
+      if (elect_one()) {
+        const uint32_t sx = smem_u32(smem + st * G::STAGE), sut = sx + G::X + G::U;
+#pragma unroll
+        for (int kk = 0; kk < DAT_BK / 16; ++kk)
+          tc_mma_bf16(tmem, umma_desc_sw128(sx + kk * 2048, 16384, 1024),
+                      umma_desc_sw128(sut + (kk >> 2) * (NW * 128) + (kk & 3) * 32, 16, 1024), ID,
+                      (s > 0 || kk > 0) ? 1u : 0u);
+        tc_commit(&empty[st]);
+        if (s == nst - 1) tc_commit(&acc_full);
+      }
+      __syncwarp();
+    }
+  } else {
+    const int q = warp & 3, row = q * 32 + lane;
+    for (int s = 0; s < nst; ++s) {
+      const int st = s % DAT_ST;
+      mbar_wait(&full[st], (s / DAT_ST) & 1);
+      const uint8_t* su = smem + st * G::STAGE + G::X;
+      uint8_t* sut = smem + st * G::STAGE + G::X + G::U;
+      const bool ok = s * DAT_BK + row < P.T;
+      const bf16 z = __float2bfloat16_rn(0.f);
+#pragma unroll
+      for (int c = 0; c < NW / 8; ++c) {
+        uint4 v = ok ? reinterpret_cast<const uint4*>(su + row * (NW * 2))[c] : make_uint4(0, 0, 0, 0);
+        const bf16* e = reinterpret_cast<const bf16*>(&v);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int n = c * 8 + i;   // dU^T row n, K = token `row`: atom (row >> 6) of [NW][64]
+          *reinterpret_cast<bf16*>(sut + (row >> 6) * (NW * 128) + n * 128 + ((((row & 63) >> 3) ^ (n & 7)) << 4) +
+                                   (row & 7) * 2) = n < P.M ? e[i] : z;
+        }
+      }
+      fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&ut_full[st]);
+    }
+    mbar_wait(&acc_full, 0);
+    tc_fence_after();
+    const int k = k0 + row;
+#pragma unroll
+    for (int c0 = 0; c0 < NW; c0 += 16) {
+      uint32_t r[16];
+      tmem_ld16(tmem + c0 + ((uint32_t)(q * 32) << 16), r);
+      if (k < P.N) {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int m = c0 + i;
+          if (m >= P.M) continue;
+          const int seg = P.m_seg > 0 ? m / P.m_seg : 0, mr = P.m_seg > 0 ? m % P.m_seg : m;
+          if (P.m_valid > 0 && mr >= P.m_valid) continue;
+          float* C = seg == 0 ? P.C : seg == 1 ? P.C1 : P.C2;
+          C[(size_t)mr * P.ldc + k] = __uint_as_float(r[i]) * P.scale;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<G::TCOLS>(tmem);
+  }
+}
+
 }  // namespace
 
 void lora_rows_tiles(const LoraRowsProblem* probs, int n, std::vector<int2>& out) {
@@ -604,6 +926,51 @@ int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max
 namespace menos {
 bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
                 uint32_t br);
+bool tma_map_2d_plain(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
+                      uint32_t br);
+
+template <int NW>
+static int da_tc_launch(const CUtensorMap& mX, const CUtensorMap& mU, const LoraTokRedProblem* d_probs, int n_probs,
+                        int max_n, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_da_tc_kernel<NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, DatGeo<NW>::SMEM);
+    attr = true;
+  }
+  lora_da_tc_kernel<NW><<<dim3((max_n + 127) / 128, n_probs), 192, DatGeo<NW>::SMEM, st>>>(mX, mU, d_probs);
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
+
+int lora_da_tc_run(const LoraTokRedProblem* d_probs, int n_probs, int max_n, int max_w, const bf16* X, int rows,
+                   int ldx, const bf16* dU, int lddu, cudaStream_t st) {
+  if (n_probs <= 0 || max_n <= 0) return 0;
+  const int NW = max_w <= 16 ? 16 : max_w <= 32 ? 32 : max_w <= 64 ? 64 : -1;
+  if (NW < 0 || ldx % 8 || lddu % 8) return -1;
+  CUtensorMap mX, mU;
+  if (!tma_map_2d(&mX, X, rows, max_n, ldx, 64, 128)) return -2;
+  if (!tma_map_2d_plain(&mU, dU, rows, lddu, lddu, NW, 128)) return -2;
+  if (NW == 16) return da_tc_launch<16>(mX, mU, d_probs, n_probs, max_n, st);
+  if (NW == 32) return da_tc_launch<32>(mX, mU, d_probs, n_probs, max_n, st);
+  return da_tc_launch<64>(mX, mU, d_probs, n_probs, max_n, st);
+}
+
+int lora_dub_tc_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, const bf16* dY, int y_rows, int ldy,
+                    const bf16* U, int ldu, cudaStream_t st) {
+  if (n_probs <= 0 || max_slabs <= 0) return 0;
+  if (ldy % 8 || ldu % 8) return -1;
+  CUtensorMap mY, mU;
+  if (!tma_map_2d(&mY, dY, y_rows, ldy, ldy, 64, 128)) return -2;
+  if (!tma_map_2d_plain(&mU, U, y_rows, ldu, ldu, 16, 128)) return -2;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lora_dub_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, DUBT_SMEM);
+    attr = true;
+  }
+  lora_dub_tc_kernel<<<dim3(max_slabs, n_probs), 192, DUBT_SMEM, st>>>(mY, mU, d_probs);
+  ++g_launch_count;
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
+}
 
 void lora_shrink_tiles(const LoraShrinkProblem* probs, int n, std::vector<int2>& out) {
   for (int i = 0; i < n; ++i)

@@ -281,6 +281,7 @@ struct SGList {
   int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0;
   int max_rank = 0; long long max_elems = 0;   // fused dU+dB lists: widest rank, largest T * rs
   int tile_n = 0;                              // token-reduction lists: tile width
+  int n_small = 0;                             // fused dU+dB lists: problems [0, n_small) have rank <= 16
 };
 
 struct menos_batch {
@@ -326,6 +327,17 @@ struct menos_batch {
     int probs_off = 0, tiles_off = 0, n_tiles = 0, max_w = 0; double flops = 0;
   };
   std::vector<ShkList> sg_shk;   // [layer * NG + g]
+  // whole-buffer operands of the tcgen05 dU + dB kernel, per layer and group (dY lives in the per-call scratch)
+  struct DubBufs { const bf16* Y = nullptr; int ldy = 0; const bf16* U = nullptr; int ldu = 0, rows = 0; };
+  std::vector<DubBufs> dub_bufs;
+  // dA on tcgen05 (clients whose group slot is <= 64 wide), per layer and group
+  struct DaTc {
+    int probs_off = 0, n = 0, max_w = 0, max_n = 0; double flops = 0;
+    const bf16* X = nullptr; int rows = 0, ldx = 0; const bf16* dU = nullptr; int lddu = 0;
+  };
+  std::vector<DaTc> da_tc;
+  LoraTokRedProblem* d_daprobs = nullptr;
+  std::vector<LoraTokRedProblem> h_daprobs;
   LoraShrinkProblem* d_sprobs = nullptr; int2* d_stiles = nullptr;
   // dS-stored attention backward: chunk buffer tiles (0 = the recompute path for this batch)
   long long ds_tiles = 0;
@@ -1245,6 +1257,8 @@ static int build_batch(menos_server* s, int n_seqs, const int32_t* seq_client, c
   // small-GEMM problem lists are filled later (need layer buffers); reserve host vectors here
   b->sg_fwd.resize((size_t)s->n_layers * NG);
   b->sg_shk.assign((size_t)s->n_layers * NG, menos_batch::ShkList());
+  b->dub_bufs.assign((size_t)s->n_layers * NG, menos_batch::DubBufs());
+  b->da_tc.assign((size_t)s->n_layers * NG, menos_batch::DaTc());
   b->sg_dub.resize((size_t)s->n_layers * NG);
   b->sg_da.resize((size_t)s->n_layers * NG);
 
@@ -1494,6 +1508,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   std::vector<int4> ttiles;
   std::vector<LoraDUBProblem> dprobs;
   std::vector<LoraShrinkProblem> sprobs;
+  std::vector<LoraTokRedProblem> daprobs;
   std::vector<int2> stiles;
   auto add_rows = [&](SGList& L, const std::vector<LoraRowsProblem>& ps) {
     L.probs_off = (int)rprobs.size(); L.n_probs = (int)ps.size(); L.tiles_off = (int)rtiles.size();
@@ -1571,6 +1586,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           q.dU = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.lddu = R;
           q.Nt = D.N_t[t]; q.rank = c.rank; q.rs = c.rs; q.T = Tc; q.scale = c.s;
           q.n_slabs = (q.Nt + LORA_DUB_MT - 1) / LORA_DUB_MT;
+          q.t0 = t0; q.ycol0 = D.rb_base[t]; q.ucol0 = c.col_off[g] + c.sub[t];
           if (q.p_blk % LORA_DUB_MT) FAIL(MENOS_EINVAL, "LoRA row block %d not a multiple of %d", q.p_blk, LORA_DUB_MT);
           woff += (size_t)q.n_slabs * Tc * c.rank;
           dub.push_back(q);
@@ -1585,6 +1601,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         pa.Q = X + (size_t)t0 * ldx; pa.ldq = ldx;
         pa.M = c.width[g]; pa.T = Tc; pa.scale = 1.f;
         pa.m_seg = c.rs; pa.m_valid = c.rank;
+        pa.t0 = t0; pa.pcol0 = c.col_off[g];
         da.push_back(pa);
         da_w = std::max(da_w, c.width[g]);
       }
@@ -1592,6 +1609,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       add_rows(b->sg_fwd[li], f);
       {
         menos_batch::ShkList& H = b->sg_shk[li];
+        H = menos_batch::ShkList();
         H.X = X; H.x_rows = T; H.ldx = ldx; H.A = s->Acat[g][l]; H.a_rows = s->cols[g].cap; H.lda = D.ldK_g[g];
         H.K = D.K_g[g]; H.U = U; H.ldu = R;
         H.probs_off = (int)sprobs.size(); H.tiles_off = (int)stiles.size();
@@ -1603,8 +1621,14 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         sprobs.insert(sprobs.end(), shk.begin(), shk.end());
         stiles.insert(stiles.end(), tl.begin(), tl.end());
       }
+      b->dub_bufs[li] = menos_batch::DubBufs{dY, ldy, U, R, T};
+      // rank <= 16 first (tcgen05 kernel), larger ranks after (mma.sync kernel): the kernel a client's problem
+      // takes depends on its own rank only, never on who shares the batch
+      std::stable_partition(dub.begin(), dub.end(), [](const LoraDUBProblem& q) { return q.rank <= 16; });
       {
         SGList& Ld = b->sg_dub[li];
+        Ld = SGList();
+        for (const auto& q : dub) Ld.n_small += q.rank <= 16;
         Ld.probs_off = (int)dprobs.size(); Ld.n_probs = (int)dub.size();
         for (const auto& q : dub) {
           Ld.flops += 4.0 * q.Nt * q.rank * q.T;
@@ -1615,8 +1639,28 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
         dprobs.insert(dprobs.end(), dub.begin(), dub.end());
       }
       const int da_mt = da_w <= 16 ? 16 : da_w <= 32 ? 32 : 64;
-      // 128-column tiles: 64-column ones (twice the CTAs at cfg1) measured slower, 33.6 vs 28.6 us per layer (r2bf)
-      add_tokred(b->sg_da[li], da, da_mt, 128);
+      // slots <= 32 wide: tcgen05 (per client: the kernel never depends on who shares the batch); wider: mma.sync
+      // with 128-column tiles (64-column ones, twice the CTAs at cfg1, measured slower: 33.6 vs 28.6 us, r2bf)
+      {
+        static const bool da_mma = [] { const char* e = getenv("MENOS_LORA_DA_MMA"); return e && atoi(e) == 1; }();
+        std::vector<LoraTokRedProblem> da_big;
+        menos_batch::DaTc& Dt = b->da_tc[li];
+        Dt = menos_batch::DaTc();   // lists are rebuilt when a NOGRAD batch re-forwards
+        Dt.probs_off = (int)daprobs.size(); Dt.X = X; Dt.rows = T; Dt.ldx = ldx; Dt.dU = sc.dU[g]; Dt.lddu = R;
+        for (const auto& pa : da) {
+          if (!da_mma && pa.M <= 32) {   // wider slots: the per-stage transpose of 48-64 dU columns makes the
+                                           // tcgen05 kernel slower than the token reduction (r2bh: 150 vs 119 us)
+            daprobs.push_back(pa); ++Dt.n;
+            Dt.max_w = std::max(Dt.max_w, pa.M); Dt.max_n = std::max(Dt.max_n, pa.N);
+            Dt.flops += 2.0 * pa.M * pa.N * pa.T;
+          } else {
+            da_big.push_back(pa);
+          }
+        }
+        int big_w = 0;
+        for (const auto& pa : da_big) big_w = std::max(big_w, pa.M);
+        add_tokred(b->sg_da[li], da_big, big_w <= 16 ? 16 : big_w <= 32 ? 32 : 64, 128);
+      }
     }
   }
   const size_t o_rp = put(rprobs.data(), rprobs.size() * sizeof(LoraRowsProblem));
@@ -1625,6 +1669,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   const size_t o_tt = put(ttiles.data(), ttiles.size() * sizeof(int4));
   const size_t o_dp = put(dprobs.data(), dprobs.size() * sizeof(LoraDUBProblem));
   const size_t o_sp = put(sprobs.data(), sprobs.size() * sizeof(LoraShrinkProblem));
+  const size_t o_dap = put(daprobs.data(), daprobs.size() * sizeof(LoraTokRedProblem));
   const size_t o_st = put(stiles.data(), stiles.size() * sizeof(int2));
   uint8_t* meta = (uint8_t*)s->arena.alloc(blob.size());
   if (!meta) { s->arena.release(slab); b->slab = nullptr; FAIL(MENOS_ENOMEM, "arena: batch metadata"); }
@@ -1662,6 +1707,8 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
   b->d_ttiles = (int4*)(meta + o_tt);
   b->d_dprobs = (LoraDUBProblem*)(meta + o_dp);
   b->d_sprobs = (LoraShrinkProblem*)(meta + o_sp);
+  b->d_daprobs = (LoraTokRedProblem*)(meta + o_dap);
+  b->h_daprobs = std::move(daprobs);
   b->d_stiles = (int2*)(meta + o_st);
   b->h_dprobs = std::move(dprobs);
   return MENOS_OK;
@@ -1743,17 +1790,36 @@ static int run_rows(menos_batch* b, const SGList& L, cudaStream_t st) {
   return lora_rows_run(b->d_rprobs, b->d_rtiles + L.tiles_off, L.n_tiles, L.max_n, st);
 }
 // fused dU + dB (one pass over each target's dY), then the fixed-order slab sum into the bf16 dU slot columns
-static int run_dub(menos_batch* b, const SGList& L, cudaStream_t st) {
+// (tcgen05 for rank <= 16; MENOS_LORA_DUB_MMA=1 or larger ranks: the mma.sync kernel)
+static int run_dub(menos_batch* b, size_t li, cudaStream_t st) {
+  static const bool mma = [] { const char* e = getenv("MENOS_LORA_DUB_MMA"); return e && atoi(e) == 1; }();
+  const SGList& L = b->sg_dub[li];
   if (L.n_probs == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
-  int rc = lora_dub_run(b->d_dprobs + L.probs_off, L.n_probs, L.max_n, L.max_rank, st);
+  const menos_batch::DubBufs& Bf = b->dub_bufs[li];
+  const int n_tc = mma ? 0 : L.n_small;
+  int rc = lora_dub_tc_run(b->d_dprobs + L.probs_off, n_tc, L.max_n, Bf.Y, Bf.rows, Bf.ldy, Bf.U, Bf.ldu, st);
+  if (!rc && L.n_probs > n_tc)
+    rc = lora_dub_run(b->d_dprobs + L.probs_off + n_tc, L.n_probs - n_tc, L.max_n, L.max_rank, st);
   if (rc) return rc;
   return lora_du_reduce_run(b->d_dprobs + L.probs_off, L.n_probs, L.max_elems, st);
 }
+// dA of every client's group: tcgen05 for slots <= 32 wide, the mma.sync token reduction for wider ones
+static int run_da(menos_batch* b, size_t li, cudaStream_t st);
 static int run_tokred(menos_batch* b, const SGList& L, cudaStream_t st) {
   if (L.n_tiles == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
   return lora_tokred_run(b->d_tprobs, b->d_ttiles + L.tiles_off, L.n_tiles, L.max_n, L.tile_n, st);
+}
+static int run_da(menos_batch* b, size_t li, cudaStream_t st) {
+  const menos_batch::DaTc& Dt = b->da_tc[li];
+  if (Dt.n > 0) {
+    ProfScope ps(PC_LORA, Dt.flops, 0, st);
+    int rc = lora_da_tc_run(b->d_daprobs + Dt.probs_off, Dt.n, Dt.max_n, Dt.max_w, Dt.X, Dt.rows, Dt.ldx, Dt.dU,
+                            Dt.lddu, st);
+    if (rc) return rc;
+  }
+  return run_tokred(b, b->sg_da[li], st);
 }
 
 // tensor-parallel all-reduce (sum, in place, stream-ordered) through the caller's callback (menos_tp_cfg)
@@ -1835,7 +1901,6 @@ static int layer_forward(menos_server* s, menos_batch* b, int l, const float* x,
     {
       ProfScope ps(PC_ATTN_FWD, 4.0 * D.hd * D.H * AV.pairs, 0, st);
       if ((D.hd == 128 || D.hd == 64) && (g_attn_tc & 4)) K_TRY(attn_fwd_ws(a, AV.items, AV.n_items, s->num_sms, st));
-      else if (D.hd == 128 && (g_attn_tc & 1)) K_TRY(attn_fwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
       else K_TRY(attn_fwd(a, st));
     }
     if (xp) K_TRY(rows_map(sc.O_x, D.Nq, b->d_tok_ext, T, D.Nq, S.O, D.Nq, st));   // drop the prefix rows' outputs
@@ -1930,7 +1995,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     dy = sc.gath;
   }
   // A8: down dX (+ LoRA down) with SwiGLU backward epilogue -> dgu
-  if (b->g_active[GD]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GD], st));
+  if (b->g_active[GD]) K_TRY(run_dub(b, (size_t)l * NG + GD, st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.fpad; a.K = D.d; a.b_mn_major = 1;
@@ -1943,9 +2008,9 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     if (opt) { a.epi = EPI_RELU_BWD; a.ldo = D.fpad; a.ldaux = D.fpad; }   // dz = da * (relu(z) > 0)
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GD]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GD], st));
+  if (b->g_active[GD]) K_TRY(run_da(b, (size_t)l * NG + GD, st));
   // A9: gate/up dX (+ LoRA) -> dhn; RMSNorm2 backward + residual -> dh
-  if (b->g_active[GGU]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GGU], st));
+  if (b->g_active[GGU]) K_TRY(run_dub(b, (size_t)l * NG + GGU, st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = D.gu_cols; a.b_mn_major = 1;
@@ -1958,7 +2023,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: gate|up-dX partials
   }
-  if (b->g_active[GGU]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GGU], st));
+  if (b->g_active[GGU]) K_TRY(run_da(b, (size_t)l * NG + GGU, st));
   {
     ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
     const bf16* dhn = D.sp ? sc.rsout : sc.dhn;
@@ -1974,7 +2039,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
   }
   // A10: O dX (+ LoRA o) -> dO (and, for head_dim % 32 == 0, the attention backward's row sums D)
   const bool fuse_dsum = D.hd % 32 == 0 && 128 % D.hd == 0;
-  if (b->g_active[GO]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GO], st));
+  if (b->g_active[GO]) K_TRY(run_dub(b, (size_t)l * NG + GO, st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.Nq; a.K = D.d; a.b_mn_major = 1;
@@ -1989,7 +2054,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     }
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
   }
-  if (b->g_active[GO]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GO], st));
+  if (b->g_active[GO]) K_TRY(run_da(b, (size_t)l * NG + GO, st));
   // A11: attention backward (+ RoPE backward) -> dqkv
   if (!fuse_dsum) {
     ProfScope ps(PC_ATTN_PREP, 0, (double)T * (4.0 * D.Nq + 4 * D.H), st);
@@ -2029,7 +2094,6 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
         K_TRY(attn_bwd_fused(a, AV.items_seq, AV.n_items_seq, s->num_sms, st));
       else if ((D.hd == 128 || D.hd == 64) && (g_attn_tc & 8))
         K_TRY(attn_bwd_ws(a, AV.items_kv, AV.n_items_kv, AV.items_q, AV.n_items, s->num_sms, st));
-      else if (D.hd == 128 && (g_attn_tc & 2)) K_TRY(attn_bwd_tc(a, xp ? b->d_blocks128_ext : b->d_blocks128, AV.n_blocks128, st));
       else K_TRY(attn_bwd(a, st));
     }
     if (xp) {
@@ -2040,7 +2104,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     }
   }
   // A12: QKV dX (+ LoRA q/k/v) -> dxn; RMSNorm1 backward + residual -> dx
-  if (b->g_active[GQKV]) K_TRY(run_dub(b, b->sg_dub[(size_t)l * NG + GQKV], st));
+  if (b->g_active[GQKV]) K_TRY(run_dub(b, (size_t)l * NG + GQKV, st));
   {
     GemmArgs a = gemm_base(s);
     a.M = T; a.N = D.d; a.K = D.Nqkv; a.b_mn_major = 1;
@@ -2053,7 +2117,7 @@ static int layer_backward(menos_server* s, menos_batch* b, int l, const float* d
     { ProfScope ps(PC_GEMM, 2.0 * a.M * a.N * a.K, 0, st); K_TRY(gemm_run(a, st)); }
     if (D.sp) { int rc = sp_scatter(s, R, sc.dhn, sc.rsout, st); if (rc) return rc; }   // A16: qkv-dX partials
   }
-  if (b->g_active[GQKV]) K_TRY(run_tokred(b, b->sg_da[(size_t)l * NG + GQKV], st));
+  if (b->g_active[GQKV]) K_TRY(run_da(b, (size_t)l * NG + GQKV, st));
   {
     ProfScope ps(PC_NORM, 0, (double)R.Tloc * (16.0 * D.d + 4), st);
     const bf16* dxn = D.sp ? sc.rsout : sc.dhn;
@@ -2189,6 +2253,8 @@ static int relocate_scratch_refs(menos_server* s, menos_batch* b, cudaStream_t s
   for (auto& p : b->h_rprobs) { mv(p.A); mv(p.B); mv(p.C); }
   for (auto& p : b->h_tprobs) { mv(p.P); mv(p.Q); mv(p.C); mv(p.C1); mv(p.C2); }
   for (auto& p : b->h_dprobs) { mv(p.dY); mv(p.U); mv(p.B); mv(p.dB); mv(p.W); mv(p.dU); }
+  for (auto& d : b->dub_bufs) { mv(d.Y); mv(d.U); }
+  for (auto& d : b->da_tc) { mv(d.X); mv(d.dU); }
   int rc = 0;
   if (!b->h_rprobs.empty()) rc = upload(s, b->d_rprobs, b->h_rprobs.data(), b->h_rprobs.size() * sizeof(LoraRowsProblem), st);
   if (!rc && !b->h_tprobs.empty())

@@ -94,7 +94,6 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   int2* d_b128;
   cudaMalloc(&d_b128, std::max<size_t>(1, b128.size()) * sizeof(int2));
   cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
-  const bool tc_fwd = hd == 128 && (g_attn_tc & 1), tc_bwd = hd == 128 && (g_attn_tc & 2);
   const bool ws_fwd = (hd == 128 || hd == 64) && (g_attn_tc & 4);
   std::vector<int4> items;
   attn_ws_items(seq_len, n_seqs, H, items, g_attn_order ? 1 : 0);
@@ -105,7 +104,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   rc = ws_fwd ? attn_fwd_ws(a, d_items, (int)items.size(), sms, 0)
-              : tc_fwd ? attn_fwd_tc(a, d_b128, (int)b128.size(), 0) : attn_fwd(a, 0);
+              : attn_fwd(a, 0);
   if (rc == 0 && dO) {
     attn_bwd_prep((const bf16*)dO, (const bf16*)O, d_D, T, H, hd, 0);
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv;
@@ -149,7 +148,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
     } else {
       rc = fused_bwd ? attn_bwd_fused(a, d_items_seq, (int)items_seq.size(), sms, 0)
            : ws_bwd ? attn_bwd_ws(a, d_items_kv, (int)items_kv.size(), d_items, (int)items.size(), sms, 0)
-                    : tc_bwd ? attn_bwd_tc(a, d_b128, (int)b128.size(), 0) : attn_bwd(a, 0);
+                    : attn_bwd(a, 0);
     }
     cudaDeviceSynchronize();
     cudaFree(d_items_kv); cudaFree(d_acc); cudaFree(d_items_seq);
@@ -248,9 +247,9 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
   return MENOS_OK;
 }
 
-// Attention variant for head_dim 128, bitmask: 1 = tcgen05 forward (2-pass, serialized), 2 = tcgen05 backward
-// (dK/dV + dQ kernels), 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; overrides 1),
-// 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; overrides 2).
+// Attention variant for head_dim 128 / 64, bitmask (bits 0, 1: round-1 non-persistent tcgen05 kernels, removed in
+// round 2; ignored): 4 = persistent warp-specialized tcgen05 forward (attention_fwd_ws.cu; else mma.sync),
+// 8 = persistent warp-specialized tcgen05 backward (attention_bwd_ws.cu; else mma.sync).
 // 64 = with 8: the dK/dV kernel stores dS^T and dQ is computed from it (S, P, dP once per pair; chunked under
 // g_attn_ds_cap_tiles, 16 KB tiles).
 // Default 78: the persistent tcgen05 forward and the dS-stored persistent backward (LPT work order, bit 4 selects

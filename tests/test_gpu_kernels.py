@@ -265,13 +265,11 @@ def _restore_attention_mode():
                                              (64, 8, 1, [200, 65, 1], 14), (64, 4, 4, [200, 65, 1000, 3], -14),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 14), (128, 8, 1, [130, 7, 256], 14),
                                              (128, 2, 2, [512, 1024, 255], 14), (128, 3, 1, [2048, 1, 700], 14),
-                                             (128, 4, 2, [1, 17, 64, 129, 300], 6), (128, 8, 1, [130, 7, 256], 6),
-                                             (128, 2, 2, [512, 1024, 255], 6), (128, 3, 1, [2048, 1, 700], 6),
-                                             (128, 4, 2, [1, 17, 64, 129, 300], 3), (128, 4, 2, [1, 17, 64, 129, 300], 0),
-                                             (128, 4, 2, [1, 17, 64, 129, 300], 2), (128, 8, 1, [130, 7, 256], 3),
-                                             (128, 2, 2, [512, 1024, 255], 3), (128, 2, 2, [512, 1024, 255], 0),
-                                             (16, 4, 4, [16, 16, 3], 3), (64, 8, 1, [200, 65], 3),
-                                             (128, 4, 4, [1, 17, 64, 129, 300], -14), (64, 4, 4, [200, 65], -3),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 4), (128, 8, 1, [130, 7, 256], 4),
+                                             (128, 4, 2, [1, 17, 64, 129, 300], 0),
+                                             (128, 2, 2, [512, 1024, 255], 0),
+                                             (16, 4, 4, [16, 16, 3], 0), (64, 8, 1, [200, 65], 0),
+                                             (128, 4, 4, [1, 17, 64, 129, 300], -14), (64, 4, 4, [200, 65], -16),
                                              (128, 4, 2, [1, 17, 64, 129, 300], 78), (128, 8, 1, [130, 7, 256], 78),
                                              (128, 2, 2, [512, 1024, 255], 78), (128, 3, 1, [2048, 1, 700], 78),
                                              (128, 8, 8, [512] * 16 + [77], 78), (128, 4, 4, [1, 17, 64, 129, 300], -78),

@@ -68,12 +68,15 @@ def test_zero_b_equals_base_bitwise():
 def test_batched_equals_alone_bitwise():
     """Invariant (c): a client's outputs and grads do not depend on who shares the batch."""
     m = MODELS["tiny"]
+    # slot widths differ per group (the tcgen05 shrink's MMA N follows the widest client of the batch) and one rank
+    # is above 16 (its dU + dB problems take the mma.sync kernel, the others the tcgen05 one)
     cl = [ClientCfg(4, 8.0, ("q", "v"), [50, 30]), ClientCfg(16, 32.0, ("q", "v", "o"), [100]),
-          ClientCfg(8, 16.0, ("q", "v", "down"), [7, 70])]
+          ClientCfg(8, 16.0, ("q", "v", "down"), [7, 70]), ClientCfg(16, 32.0, TARGETS, [45]),
+          ClientCfg(24, 48.0, ("q", "k", "v", "gate"), [33])]
     w = Workload("bva", m, cl)
     inputs = make_inputs(w, seed=7)
     weights, adapters, io = inputs
-    srv = new_server(w, weights)
+    srv = new_server(w, weights, max_rank=32)
     ids = register(srv, w, adapters)
     full = run_gpu_step(w, inputs=inputs, srv=srv, ids=ids)
     for i in range(len(cl)):
@@ -262,3 +265,32 @@ def test_interleaved_save_batches_bitwise():
         for t in ("q", "v", "down"):
             assert np.array_equal(srv.get_adapter(ids[0], l, t, "dA"), ref_a["grads"][0][l][t][0])
     srv.close()
+
+
+def test_attention_ds_chunking_end_to_end():
+    """The dS-stored attention backward through the server: parity vs the oracle on a head_dim-128 GQA model with
+    ragged sequences; a chunk budget far below the batch's dS^T tiles (several (sequence, kv head) chunks, one
+    buffer) gives bitwise the same step; the recompute path (mode 14) also meets the bars."""
+    from paper_conf_middleware_hul24_b200.menos import check, lib
+    from workloads.synth import ModelCfg
+    m = ModelCfg("hd128", 512, 4, 2, 1024, 2, model_layers=3)
+    cl = [ClientCfg(8, 16.0, ("q", "v"), [300, 129]), ClientCfg(16, 32.0, TARGETS, [700, 17, 1]),
+          ClientCfg(4, 8.0, ("k", "o", "down"), [64])]
+    w = Workload("hd128_ds", m, cl)
+    inputs = make_inputs(w, seed=41)
+    ora = run_oracle_step(w, inputs=inputs)
+    try:
+        full = run_gpu_step(w, inputs=inputs)
+        assert_report(compare_step(full, ora))
+        check(lib().menos_test_set_ds_cap(80), testing=True)    # 700-token unit = 2 x 36 tiles; several chunks
+        chunked = run_gpu_step(w, inputs=inputs)
+        for i in range(len(cl)):
+            assert np.array_equal(full["x_s"][i], chunked["x_s"][i]) and np.array_equal(full["g_s"][i], chunked["g_s"][i])
+            for l, d in enumerate(full["grads"][i]):
+                for t, (dA, dB) in d.items():
+                    assert np.array_equal(chunked["grads"][i][l][t][0], dA) and np.array_equal(chunked["grads"][i][l][t][1], dB)
+        check(lib().menos_test_set_attn_tc(14), testing=True)   # recompute path
+        assert_report(compare_step(run_gpu_step(w, inputs=inputs), ora))
+    finally:
+        check(lib().menos_test_set_ds_cap(32768), testing=True)
+        check(lib().menos_test_set_attn_tc(78), testing=True)
