@@ -76,6 +76,14 @@ MENOS_API int menos_test_set_attn_tc(int mode);
    Small values force chunking (tests).  MENOS_EINVAL if tiles < 1. */
 MENOS_API int menos_test_set_ds_cap(long long tiles);
 
+/* Host-only (no GPU): the dS-stored backward's plan for n_seqs sequences -- tiles[i] = dS^T tiles of sequence i per
+   head, base[seq * Hkv + kv head] = the unit's first tile in its chunk, chunks[4c..4c+3] = (kv item offset, count,
+   q item offset, count) for c < min(*n_chunks, max_chunks); *n_chunks = -1 when a unit alone exceeds `cap` (the
+   recompute path).  Any output pointer but n_chunks may be NULL. */
+MENOS_API int menos_test_ds_plan(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int32_t* tiles,
+                                 int32_t* base, int32_t* chunks, int max_chunks, int32_t* n_chunks,
+                                 int32_t* n_items_kv, int32_t* n_items_q);
+
 /* Tuning aid: per-phase clock64 totals of the one-pass attention backward's role threads (16 counters, cleared by the
  * read) when libmenos.so was built with -DMENOS_ABF_PROF (MENOS_NVCC_DEFS); zeros otherwise. */
 MENOS_API int menos_test_abf_prof(unsigned long long* out16);

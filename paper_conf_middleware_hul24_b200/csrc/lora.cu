@@ -720,18 +720,20 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
 // [NW][128] operand (rows past the client's tokens / slot width zeroed).  The [128 x NW] accumulator stays in TMEM
 // over all stages; one thread per column k writes it to every target's dA rows.
 constexpr int DAT_BK = 128;
-template <int NW> struct DatGeo {
+// STG stages: 4 (one CTA per SM, ~200 KB in flight) when the grid is small (cfg1: 128 CTAs; 25.0 -> 19.7 us per
+// layer), 2 (two CTAs per SM) when it is large (cfg3: 4 stages measured 217 -> 246 us), r2bh / r2bi
+template <int NW, int STG> struct DatGeo {
   static constexpr int X = 128 * 128 * 2, U = 128 * NW * 2, UT = NW * 128 * 2, STAGE = X + U + UT;
-  static constexpr int ST = (200 * 1024) / STAGE < 4 ? (200 * 1024) / STAGE : 4;   // ring of ~200 KB, <= 4 stages
+  static constexpr int ST = STG;
   static constexpr int SMEM = ST * STAGE + 1024;
   static constexpr int TCOLS = NW < 32 ? 32 : NW;
 };
 
-template <int NW>
+template <int NW, int STG>
 __global__ void __launch_bounds__(192, 1)
 lora_da_tc_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmU,
                   const LoraTokRedProblem* __restrict__ probs) {
-  using G = DatGeo<NW>;
+  using G = DatGeo<NW, STG>;
   constexpr int DAT_ST = G::ST;
   extern __shared__ uint8_t dat_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(dat_raw) + 1023) & ~uintptr_t(1023));
@@ -929,15 +931,16 @@ bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols,
 bool tma_map_2d_plain(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
                       uint32_t br);
 
-template <int NW>
+template <int NW, int STG>
 static int da_tc_launch(const CUtensorMap& mX, const CUtensorMap& mU, const LoraTokRedProblem* d_probs, int n_probs,
                         int max_n, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(lora_da_tc_kernel<NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, DatGeo<NW>::SMEM);
+    cudaFuncSetAttribute(lora_da_tc_kernel<NW, STG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         DatGeo<NW, STG>::SMEM);
     attr = true;
   }
-  lora_da_tc_kernel<NW><<<dim3((max_n + 127) / 128, n_probs), 192, DatGeo<NW>::SMEM, st>>>(mX, mU, d_probs);
+  lora_da_tc_kernel<NW, STG><<<dim3((max_n + 127) / 128, n_probs), 192, DatGeo<NW, STG>::SMEM, st>>>(mX, mU, d_probs);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }
@@ -950,9 +953,16 @@ int lora_da_tc_run(const LoraTokRedProblem* d_probs, int n_probs, int max_n, int
   CUtensorMap mX, mU;
   if (!tma_map_2d(&mX, X, rows, max_n, ldx, 64, 128)) return -2;
   if (!tma_map_2d_plain(&mU, dU, rows, lddu, lddu, NW, 128)) return -2;
-  if (NW == 16) return da_tc_launch<16>(mX, mU, d_probs, n_probs, max_n, st);
-  if (NW == 32) return da_tc_launch<32>(mX, mU, d_probs, n_probs, max_n, st);
-  return da_tc_launch<64>(mX, mU, d_probs, n_probs, max_n, st);
+  int sms = 148, dev = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const bool deep = (long long)((max_n + 127) / 128) * n_probs < 2LL * sms;
+  if (NW == 16) return deep ? da_tc_launch<16, 4>(mX, mU, d_probs, n_probs, max_n, st)
+                            : da_tc_launch<16, 2>(mX, mU, d_probs, n_probs, max_n, st);
+  if (NW == 32) return deep ? da_tc_launch<32, 4>(mX, mU, d_probs, n_probs, max_n, st)
+                            : da_tc_launch<32, 2>(mX, mU, d_probs, n_probs, max_n, st);
+  return deep ? da_tc_launch<64, 3>(mX, mU, d_probs, n_probs, max_n, st)
+              : da_tc_launch<64, 2>(mX, mU, d_probs, n_probs, max_n, st);
 }
 
 int lora_dub_tc_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, const bf16* dY, int y_rows, int ldy,

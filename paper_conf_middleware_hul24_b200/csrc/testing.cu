@@ -274,3 +274,25 @@ extern "C" int menos_test_set_ds_cap(long long tiles) {
   menos::g_attn_ds_cap_tiles = tiles;
   return MENOS_OK;
 }
+
+// Host plan of the dS-stored attention backward (no GPU needed): per-sequence tile counts, unit bases and chunks.
+// tiles[i] = attn_ds_tiles(seq_len[i]); base[seq * Hkv + hk]; chunks[c] = (kv item offset, count, q offset, count).
+extern "C" int menos_test_ds_plan(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int32_t* tiles,
+                                  int32_t* base, int32_t* chunks, int max_chunks, int32_t* n_chunks,
+                                  int32_t* n_items_kv, int32_t* n_items_q) {
+  if (n_seqs < 0 || !seq_len || H <= 0 || Hkv <= 0 || H % Hkv || !n_chunks) return fail("bad arguments");
+  for (int i = 0; i < n_seqs; ++i) if (tiles) tiles[i] = menos::attn_ds_tiles(seq_len[i]);
+  menos::AttnDsPlan plan;
+  std::vector<int> lens(seq_len, seq_len + n_seqs);
+  if (!menos::attn_ds_plan(lens.data(), n_seqs, H, Hkv, cap, plan)) { *n_chunks = -1; return MENOS_OK; }
+  *n_chunks = (int)plan.chunks.size();
+  if (n_items_kv) *n_items_kv = (int)plan.items_kv.size();
+  if (n_items_q) *n_items_q = (int)plan.items_q.size();
+  if (base) for (size_t i = 0; i < plan.base.size(); ++i) base[i] = plan.base[i];
+  if (chunks)
+    for (int c = 0; c < (int)plan.chunks.size() && c < max_chunks; ++c) {
+      chunks[4 * c] = plan.chunks[c].x; chunks[4 * c + 1] = plan.chunks[c].y;
+      chunks[4 * c + 2] = plan.chunks[c].z; chunks[4 * c + 3] = plan.chunks[c].w;
+    }
+  return MENOS_OK;
+}
