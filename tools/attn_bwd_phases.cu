@@ -1,6 +1,7 @@
 // Per-phase clock accounting of the persistent dK/dV backward kernel at the cfg1 shape (tuning aid).
 // Build (on the GPU box): MENOS_NVCC_DEFS=-DMENOS_BWS_PROF python -m paper_conf_middleware_hul24_b200.build -f, then
 //   nvcc -std=c++17 -gencode arch=compute_100a,code=sm_100a tools/attn_bwd_phases.cu -I<pkg>/csrc <pkg>/_lib/*.o -lcuda -ldl
+// Run: ./a.out [ds]   (ds: the dS-stored backward; else the recompute path)
 #include <cstdio>
 #include <vector>
 #include <cmath>
@@ -8,7 +9,8 @@
 #include "../paper_conf_middleware_hul24_b200/csrc/kernels.h"
 namespace menos { int attn_bws_prof_read(unsigned long long* out); extern int g_attn_order; }
 using namespace menos;
-int main() {
+int main(int argc, char** argv) {
+  const bool ds_path = argc > 1 && argv[1][0] == 'd';   // "ds": the dS-stored backward (default path since r2)
   const int nseq = 16, S = 512, H = 32, Hkv = 32, hd = 128, T = nseq * S, N = (H + 2 * Hkv) * hd;
   std::vector<int> cu(nseq + 1), lens(nseq, S);
   for (int i = 0; i <= nseq; ++i) cu[i] = i * S;
@@ -29,11 +31,24 @@ int main() {
   a.qkv = qkv; a.ld_qkv = N; a.cu_seqlens = dcu; a.T = T; a.H = H; a.Hkv = Hkv; a.hd = hd; a.scale = 1.f / sqrtf(hd);
   a.dO = dO; a.ld_do = H * hd; a.D = D; a.lse = lse; a.dqkv = dqkv; a.ld_dqkv = N; a.rope_cs = cs;
   unsigned long long pr[16];
-  for (int r = 0; r < 3; ++r) attn_bwd_ws(a, ikv, (int)a1.size(), iq, (int)a2.size(), 148, 0);
+  AttnDsPlan plan;
+  attn_ds_plan(lens.data(), nseq, H, Hkv, 32768, plan);
+  bf16* ds; int* dbase; int4 *pkv, *pq;
+  const long long cap = attn_ds_total_tiles(lens.data(), nseq, H);
+  cudaMalloc(&ds, (size_t)cap * 16384); cudaMalloc(&dbase, plan.base.size() * 4);
+  cudaMalloc(&pkv, plan.items_kv.size() * 16); cudaMalloc(&pq, plan.items_q.size() * 16);
+  cudaMemcpy(dbase, plan.base.data(), plan.base.size() * 4, cudaMemcpyHostToDevice);
+  cudaMemcpy(pkv, plan.items_kv.data(), plan.items_kv.size() * 16, cudaMemcpyHostToDevice);
+  cudaMemcpy(pq, plan.items_q.data(), plan.items_q.size() * 16, cudaMemcpyHostToDevice);
+  auto run = [&]() {
+    if (ds_path) attn_bwd_ws_ds(a, pkv, (int)plan.items_kv.size(), pq, (int)plan.items_q.size(), ds, cap, dbase, 148, 0);
+    else attn_bwd_ws(a, ikv, (int)a1.size(), iq, (int)a2.size(), 148, 0);
+  };
+  for (int r = 0; r < 3; ++r) run();
   attn_bws_prof_read(pr);
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   cudaEventRecord(e0);
-  for (int r = 0; r < 10; ++r) attn_bwd_ws(a, ikv, (int)a1.size(), iq, (int)a2.size(), 148, 0);
+  for (int r = 0; r < 10; ++r) run();
   cudaEventRecord(e1); cudaEventSynchronize(e1);
   float ms; cudaEventElapsedTime(&ms, e0, e1);
   attn_bws_prof_read(pr);
