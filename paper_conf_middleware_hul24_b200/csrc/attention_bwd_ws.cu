@@ -100,6 +100,11 @@ __device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
                  : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   }
 }
+// 1-D bulk copy global -> shared (16-byte aligned source and destination, size % 16 == 0), completion on `bar`
+__device__ __forceinline__ void bulk_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void ew_sync() { asm volatile("bar.sync 1, %0;" ::"n"(32 * EW_WARPS) : "memory"); }
 
 // CPT consecutive TMEM columns (32x32b.x16 / .x32), no wait
@@ -282,6 +287,7 @@ __device__ __forceinline__ void pds_math(const uint32_t (&su)[CPT], const uint32
 
 // ======================================================================================= dK / dV
 constexpr int KV_ROWS = 128, QB = 64;
+constexpr uint32_t LD_BYTES = (QB + 4) * 4;    // a block's lse (or D) row from the aligned start: 272 B
 constexpr int PT_TILE = KV_ROWS * QB * 2;      // 16 KB (1 atom [128][64])
 constexpr int KVA = KV_ROWS * 128, QBA = QB * 128;   // one SW128 atom (64 columns) of a K / V tile, of a Q / dO tile
 template <int HD> struct DkdvGeo {
@@ -308,8 +314,10 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
   __shared__ __align__(8) uint64_t acc_full, acc_free;
   __shared__ uint32_t tmem_sh;
 #if MENOS_BWS_ALT
-  // lse (log2 domain) | D (pre-scaled) of a block's 64 queries, per warp group a ring of 2 filled by cp.async one
-  // group block (two blocks) ahead
+  // raw lse | D of each Q / dO stage's 64 queries, brought by the TMA warp with the stage (two 272-byte bulk copies
+  // from the 16-byte-aligned start at or below the first query; `off` = the first query's index inside), and the
+  // group's scaled copy (lse in the log2 domain, D pre-scaled), a ring of 2 blocks
+  __shared__ __align__(16) float s_ldr[STAGES][2][QB + 4];
   __shared__ __align__(16) float s_ld[2][2][2 * QB];
 #else
   // lse (log2 domain) | D (pre-scaled) of a block's 64 queries, ring of 3 blocks filled by cp.async two blocks ahead
@@ -373,7 +381,16 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
           const int st = gb % STAGES;
           const int h = hk * rep + j / nqb, q0 = k0 + (j % nqb) * QB;
           wait_bar(&empty[st], ((gb / STAGES) & 1) ^ 1);
+#if MENOS_BWS_ALT
+          mbar_expect_tx(&full[st], 2 * QB_TILE + 2 * LD_BYTES);
+          {
+            const size_t i0 = ((size_t)h * p.T + G.base + q0) & ~(size_t)3;   // 16-byte aligned start
+            bulk_load_1d(&s_ldr[st][0][0], p.lse + i0, LD_BYTES, &full[st]);
+            bulk_load_1d(&s_ldr[st][1][0], p.D + i0, LD_BYTES, &full[st]);
+          }
+#else
           mbar_expect_tx(&full[st], 2 * QB_TILE);
+#endif
           uint8_t* q = sQ0 + st * QB_TILE;
           uint8_t* o = sO0 + st * QB_TILE;
 #pragma unroll
@@ -478,18 +495,6 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
     auto gsync = [&]() {   // the group's four warps
       if (gr == 0) asm volatile("bar.sync 2, 128;" ::: "memory"); else asm volatile("bar.sync 3, 128;" ::: "memory");
     };
-    // lse (tt < 64) / D (64 <= tt < 128) of query tt & 63 of block jj of G -> s_ld[gr][slot][tt] by cp.async (0 outside)
-    auto issue = [&](int slot, const Geo& G, int jj) {
-      const float* src = p.lse;
-      int sz = 0;
-      if (jj < G.n) {
-        const int nqb = (G.L - G.blk0 + QB - 1) / QB;
-        const int h = G.head * rep + jj / nqb, qpos = G.blk0 + (jj % nqb) * QB + (tt & (QB - 1));
-        if (qpos < G.L) { src = (tt < QB ? p.lse : p.D) + (size_t)h * p.T + G.base + qpos; sz = 4; }
-      }
-      cp_async4(smem_u32(&s_ld[gr][slot][tt]), src, sz);
-    };
-    bool have_cur = false;      // this block's copy was issued one group block ago
     bool tma_pending = false;   // this thread (t == 0) has TMA stores reading the staging buffer
     int it = 0, gb = 0, kb = 0;
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
@@ -506,21 +511,17 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         // (sP0: idle between item epilogues; group gr stages in its half)
         uint8_t* const ds_stg = sP0 + gr * PT_TILE + r * 128;
         const bool ds_lead = p.ds != nullptr && w4 == 0 && lane == 0;
-        if (!have_cur) { issue(sl, G, j); cp_async_commit(); }
-        cp_async_wait<0>();
-        s_ld[gr][sl][tt] *= tt < QB ? LOG2E_W : p.scale;   // lse to the log2 domain, D pre-scaled
+        {   // this block's lse / D arrived with its Q / dO stage (the MMA warp already waited for it): scale one each
+          const int st = gb % STAGES, h = G.head * rep + j / nqb;
+          wait_bar(&full[st], (gb / STAGES) & 1);
+          const int off = (int)(((size_t)h * p.T + base + q0) & 3);
+          const float v = s_ldr[st][tt >= QB][off + (tt & (QB - 1))];
+          s_ld[gr][sl][tt] = v * (tt < QB ? LOG2E_W : p.scale);   // lse to the log2 domain, D pre-scaled
+        }
         if (p.ds && w4 == 0 && lane == 0) bulk_wait_read0();   // the group's staging tile is free again
         BP(9);
         gsync();
         BP(1);
-        {   // the group's next block (gb + 2): its copy now, when its item is known (else at its turn)
-          const Geo N = j + 2 >= G.n ? decode(ip) : G;
-          have_cur = true;
-          if (j + 2 < G.n) issue(sl ^ 1, G, j + 2);
-          else if (j + 2 - G.n < N.n) issue(sl ^ 1, N, j + 2 - G.n);
-          else have_cur = false;
-          cp_async_commit();
-        }
         BP(0);
         wait_bar(&s_full[gr], (gb >> 1) & 1);
         BP(2);

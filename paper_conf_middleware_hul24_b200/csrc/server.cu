@@ -63,6 +63,8 @@ void set_last_error(const char* fmt, ...) {
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 constexpr size_t kDsTileBytes = 128 * 64 * 2;   // one bf16 dS^T tile [128 keys][64 queries]
+// lse / D rows are read by 272-byte bulk copies from a 16-byte-aligned start (attention backward): 512 B of slack
+constexpr size_t kLsePad = 512;
 
 // =====================================================================================================
 // per-kernel-class CUDA-event profiler (bench.py's live roofline; off by default)
@@ -1276,7 +1278,7 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
   size_t per_layer = 0;
   auto A = [&](size_t n) { per_layer += align_up(n, 256); };
   A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // x (fp32), xn, rstd1
-  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * std::max(T, Text) * 4);   // qkv, O, lse
+  A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2); A((size_t)D.H * std::max(T, Text) * 4 + kLsePad);   // qkv, O, lse
   A((size_t)R.Tloc * D.d * 4); A((size_t)R.Tpad * D.d * 2); A((size_t)R.Tloc * 4);   // h (fp32), hn, rstd2
   A((size_t)T * D.gu_cols * 2);                                             // gu
   if (save_a) A((size_t)T * D.fpad * 2);
@@ -1308,16 +1310,16 @@ static size_t scratch_bytes_of(const Dims& D, int T, const int R_used[NG], bool 
   if (D.sp) { A(dp); A(db); }                                                 // gathered dy / dh, reduce-scatter out
   if (Text > T) {   // prefix-tuning extension: qkv, O, dO, dqkv, D (fp32), the one-pass backward's dQ sums (fp32)
     A((size_t)Text * D.Nqkv * 2); A((size_t)Text * D.Nq * 2); A((size_t)Text * D.Nq * 2);
-    A((size_t)Text * D.Nqkv * 2); A((size_t)D.H * Text * 4); A((size_t)Text * D.Nq * 4);
+    A((size_t)Text * D.Nqkv * 2); A((size_t)D.H * Text * 4 + kLsePad); A((size_t)Text * D.Nq * 4);
   }
   A((size_t)T * D.Nq * 2); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.gu_cols * 2); A((size_t)T * D.fpad * 2);
-  A((size_t)D.H * T * 4);                                                     // Dsum
+  A((size_t)D.H * T * 4 + kLsePad);                                           // Dsum
   A(wsp_bytes_of(D, T, R_used));                                              // dU partials
   for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   // NOGRAD forward layer set (x ping-pong = xout/dxf; intermediates reuse the grad buffers where free)
   if (nograd_set) {
     A(dp); A(df); A((size_t)T * D.Nqkv * 2); A((size_t)T * D.Nq * 2);
-    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * std::max(T, Text) * 4); A((size_t)Rw.Tloc * 8); A(dp);
+    A((size_t)T * D.gu_cols * 2); A((size_t)D.H * std::max(T, Text) * 4 + kLsePad); A((size_t)Rw.Tloc * 8); A(dp);
     for (int g = 0; g < NG; ++g) A((size_t)T * R_used[g] * 2);
   }
   A((size_t)ds_tiles * kDsTileBytes);   // dS-stored attention backward: the chunk buffer, last
@@ -1490,7 +1492,7 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       S.x = (float*)take((size_t)Rw.Tloc * D.d * 4); S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
       S.rstd1 = (float*)take((size_t)Rw.Tloc * 4);
       S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
-      S.lse = (float*)take((size_t)D.H * std::max(T, b->Text) * 4);
+      S.lse = (float*)take((size_t)D.H * std::max(T, b->Text) * 4 + kLsePad);
       S.h = (float*)take((size_t)Rw.Tloc * D.d * 4); S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
       S.rstd2 = (float*)take((size_t)Rw.Tloc * 4);
       S.gu = (bf16*)take((size_t)T * D.gu_cols * 2);
@@ -1740,11 +1742,11 @@ static int get_scratch(menos_server* s, int T, const int R_used[NG], Scratch& sc
   if (Text > T) {
     sc.qkv_x = (bf16*)take((size_t)Text * D.Nqkv * 2); sc.O_x = (bf16*)take((size_t)Text * D.Nq * 2);
     sc.dO_x = (bf16*)take((size_t)Text * D.Nq * 2); sc.dqkv_x = (bf16*)take((size_t)Text * D.Nqkv * 2);
-    sc.D_x = (float*)take((size_t)D.H * Text * 4); sc.dqacc_x = (float*)take((size_t)Text * D.Nq * 4);
+    sc.D_x = (float*)take((size_t)D.H * Text * 4 + kLsePad); sc.dqacc_x = (float*)take((size_t)Text * D.Nq * 4);
   }
   sc.dO = (bf16*)take((size_t)T * D.Nq * 2); sc.dqkv = (bf16*)take((size_t)T * D.Nqkv * 2);
   sc.dgu = (bf16*)take((size_t)T * D.gu_cols * 2); sc.a = (bf16*)take((size_t)T * D.fpad * 2);
-  sc.Dsum = (float*)take((size_t)D.H * T * 4);
+  sc.Dsum = (float*)take((size_t)D.H * T * 4 + kLsePad);
   sc.wsp = (float*)take(wsp_bytes_of(D, T, R_used));
   for (int g = 0; g < NG; ++g) sc.dU[g] = (bf16*)take((size_t)T * R_used[g] * 2);
   sc.ds = ds_tiles > 0 ? (bf16*)(s->scratch + need - align_up((size_t)ds_tiles * kDsTileBytes, 256)) : nullptr;
@@ -1759,7 +1761,7 @@ static void nograd_layer(menos_server* s, int T, const int R_used[NG], const Scr
   auto take = [&](size_t n) { uint8_t* r = p; p += align_up(n, 256); return r; };
   S.xn = (bf16*)take((size_t)Rw.Tpad * D.d * 2); S.h = (float*)take((size_t)Rw.Tloc * D.d * 4);
   S.qkv = (bf16*)take((size_t)T * D.Nqkv * 2); S.O = (bf16*)take((size_t)T * D.Nq * 2);
-  S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * std::max(T, Text) * 4);
+  S.gu = (bf16*)take((size_t)T * D.gu_cols * 2); S.lse = (float*)take((size_t)D.H * std::max(T, Text) * 4 + kLsePad);
   S.rstd1 = (float*)take((size_t)Rw.Tloc * 8); S.rstd2 = S.rstd1 + Rw.Tloc;
   S.hn = (bf16*)take((size_t)Rw.Tpad * D.d * 2);
   S.a = D.arch == MENOS_ARCH_OPT ? S.gu : sc.a;   // OPT: the down projection's input is relu(fc1), kept in gu
