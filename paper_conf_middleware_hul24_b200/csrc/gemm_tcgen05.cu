@@ -65,6 +65,7 @@ struct KParams {
   const int* pos;
   int head_dim, rope_cols;
   int group_m;             // rasterisation group (m-tiles per group)
+  int gu_pf;               // SwiGLU bwd: L2 prefetch distance (chunks) of the saved g|u beyond the register prefetch
 };
 
 #ifndef MENOS_GEMM_EPI_PREFETCH
@@ -536,6 +537,16 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 #pragma unroll
           for (int i = 0; i < 4; ++i) { g0[i] = gq[i]; u0[i] = uq[i]; }
           if (rok && c + 1 < cl) ld_gu(c + 1, gq, uq);
+          if (p.gu_pf > 0 && rok && c + 1 + p.gu_pf < cl) {
+            // L2 prefetch of a later chunk's g and u (this warp's 32 rows x 32 columns: two contiguous 2 KB runs in
+            // warp-tile order), so that chunk's register loads hit L2 instead of waiting for HBM
+            const int pc = c + 1 + p.gu_pf, pcol = n0 + pc * 32, pg = (pcol >> 7) * 256 + (pcol & 127);
+            const int r0 = row & ~31, nr = min(32, p.M - r0);
+            if (lane * 32 < nr * 32) {
+              prefetch_l2(p.aux + gu_tile_off(r0, pg, p.M, 2 * p.N) + lane * 32);
+              prefetch_l2(p.aux + gu_tile_off(r0, pg + 128, p.M, 2 * p.N) + lane * 32);
+            }
+          }
           float da[32];
           tmem_ld32(tb + c * 32, da);
           if (rok) {
@@ -716,6 +727,9 @@ int gemm_run(const GemmArgs& a, cudaStream_t st) {
   p.rope_cs = a.rope_cs; p.pos = a.pos; p.head_dim = a.head_dim; p.rope_cols = a.rope_cols;
   static const int group_env = [] { const char* e = getenv("MENOS_GEMM_GROUP_M"); return e ? atoi(e) : 0; }();
   p.group_m = group_env > 0 ? group_env : GROUP_M;
+  // off by default: 1-3 chunks ahead measured no faster (down-dX 0.601 / 0.604 / 0.605 / 0.604 ms, r2bn)
+  static const int gu_pf_env = [] { const char* e = getenv("MENOS_GEMM_GU_PF"); return e ? atoi(e) : 0; }();
+  p.gu_pf = gu_pf_env;
   const int tiles = ((a.M + BM * CG - 1) / (BM * CG)) * ((a.N + BN - 1) / BN);
   int sms = a.num_sms > 0 ? a.num_sms : 148;
   int clusters = sms / CG;
