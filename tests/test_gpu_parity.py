@@ -217,6 +217,35 @@ def test_batch_memory_is_exact_bound(flags):
     assert err is not None and err.code == -2
 
 
+def test_batch_memory_bounds_the_ds_stored_backward():
+    """head_dim 128: the demand menos_batch_memory reports includes the dS^T chunk buffer's bound (the sequence
+    lengths are not part of the query): an arena of exactly that many bytes runs the SAVE and the NOGRAD step, and the
+    observed peak stays below it."""
+    from workloads.synth import ModelCfg
+    m = ModelCfg("hd128", 512, 4, 2, 1024, 2, model_layers=3)
+    cl = [ClientCfg(8, 16.0, ("q", "v"), [300, 1, 129]), ClientCfg(16, 32.0, TARGETS, [700])]
+    w = Workload("bm128", m, cl)
+    inputs = make_inputs(w, seed=23)
+    weights, adapters, io = inputs
+    x = torch.from_numpy(np.concatenate([a for a, _ in io])).to(torch.bfloat16).cuda()
+    for flags in (0, 1):
+        srv = new_server(w, weights, arena_bytes=1 << 30)
+        ids = register(srv, w, adapters)
+        need = max(srv.batch_memory(ids, [c.n_tokens for c in cl], flags))
+        srv.close()
+        srv = new_server(w, weights, arena_bytes=need)
+        ids = register(srv, w, adapters)
+        sc, sl = [], []
+        for i, c in enumerate(cl):
+            sc += [ids[i]] * len(c.seq_lens)
+            sl += list(c.seq_lens)
+        b = srv.forward(sc, sl, x, torch.empty_like(x), flags=flags)
+        srv.backward(b, x, torch.empty_like(x))
+        torch.cuda.synchronize()
+        assert srv.stats()["arena_peak"] <= need
+        srv.close()
+
+
 def test_host_buffers_e2e_path():
     """x_c / g_c given as (pinned) host buffers: same results as device buffers."""
     w = workload("cfg0_tiny")
