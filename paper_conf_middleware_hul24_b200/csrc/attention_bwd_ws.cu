@@ -1392,27 +1392,32 @@ long long attn_ds_total_tiles(const int* seq_len, int n_seqs, int H) {
   return t;
 }
 
-bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out) {
+bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out, int grid) {
   const int rep = H / Hkv;
   out.base.assign((size_t)n_seqs * Hkv, 0);
   out.items_kv.clear(); out.items_q.clear(); out.chunks.clear();
   std::vector<int2> units;   // (seq, kv head) of the open chunk
   long long cur = 0;
+  int grp = 0;               // (sequence, head) groups of dQ items so far (rotation of their query-block order)
   auto flush = [&]() {
     if (units.empty()) return;
     const int kv0 = (int)out.items_kv.size(), q0 = (int)out.items_q.size();
     for (const int2& u : units) {
       const int L = seq_len[u.x];
       for (int k = 0; k < L; k += 128) out.items_kv.push_back(make_int4(u.x, k, u.y, 0));
-      for (int h = u.y * rep; h < (u.y + 1) * rep; ++h)
-        for (int q = ((L - 1) / 128) * 128; q >= 0; q -= 128) out.items_q.push_back(make_int4(u.x, q, h, 0));
+      const int nq = (L + 127) / 128;
+      for (int h = u.y * rep; h < (u.y + 1) * rep; ++h, ++grp)
+        for (int j = 0; j < nq; ++j) out.items_q.push_back(make_int4(u.x, (nq - 1 - (j + grp) % nq) * 128, h, 0));
     }
     // dK/dV: LPT for the persistent grid's static round-robin (largest = most query blocks after the key block)
     std::stable_sort(out.items_kv.begin() + kv0, out.items_kv.end(), [&](const int4& a, const int4& b) {
       return seq_len[a.x] - a.y > seq_len[b.x] - b.y;
     });
-    // dQ items stay grouped by (sequence, head), last query block first: neighbouring CTAs read the same K blocks
-    // at the same time (one L2 fill instead of one per query block)
+    attn_snake_waves(out.items_kv, kv0, grid);
+    // dQ items stay grouped by (sequence, head) so neighbouring CTAs read the same K blocks at the same time (one
+    // L2 fill instead of one per query block); inside a group the query blocks are ROTATED by the group's index, so
+    // the static round-robin (stride = grid, a multiple of 4 when the grid is 148) does not hand one CTA the same
+    // query-block position -- the same cost -- in every group (r2bn: 1.6x load imbalance at cfg1)
     out.chunks.push_back(make_int4(kv0, (int)out.items_kv.size() - kv0, q0, (int)out.items_q.size() - q0));
     units.clear();
     cur = 0;

@@ -165,7 +165,10 @@ int attn_fwd(const AttnArgs& a, cudaStream_t st);
 // persistent warp-specialized tcgen05 forward for head_dim 128 (attention_fwd_ws.cu); items = (seq, q0, head, -)
 int attn_fwd_ws(const AttnArgs& a, const int4* items, int n_items, int num_sms, cudaStream_t st);
 // order: 0 = (sequence, head) groups (L2 locality), 1 = largest forward / dQ work first, 2 = largest dK/dV first
-void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order = 0);
+// grid > 0 (with order 1 / 2): the LPT list is laid out in boustrophedon waves of `grid` items (every second wave
+// reversed), so the persistent kernels' static round-robin (item i -> CTA i % grid) balances the per-CTA work
+void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order = 0, int grid = 0);
+void attn_snake_waves(std::vector<int4>& v, size_t first, int grid);
 // persistent warp-specialized tcgen05 backward for head_dim 128 (attention_bwd_ws.cu): items_kv = (seq, k0, kv
 // head, -) per 128-key block, items_q = (seq, q0, head, -) per 128-query block
 int attn_bwd_ws(const AttnArgs& a, const int4* items_kv, int n_items_kv, const int4* items_q, int n_items_q,
@@ -184,7 +187,8 @@ long long attn_ds_total_tiles(const int* seq_len, int n_seqs, int H);
 // the work lists items_kv[chunks[c].x, + .y) and items_q[chunks[c].z, + .w) (LPT-ordered).  false: a single unit
 // is larger than cap_tiles (the caller takes the recompute path).
 struct AttnDsPlan { std::vector<int> base; std::vector<int4> items_kv, items_q, chunks; };
-bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out);
+bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_tiles, AttnDsPlan& out,
+                  int grid = 0);
 // tiles the dS-stored backward may use at most (the buffer a chunk fills): 16 KB each
 extern long long g_attn_ds_cap_tiles;
 // one-pass persistent tcgen05 backward for head_dim 128 (attention_bwd_fused.cu): items = (seq, -, kv head, -), one

@@ -1367,17 +1367,17 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       v.pairs += 0.5 * (double)b->seq_len[i] * (b->seq_len[i] + 1);
     }
     v_items.emplace_back(); v_items_kv.emplace_back(); v_items_q.emplace_back();
-    attn_ws_items(b->seq_len.data(), ns, D.H, v_items.back(), g_attn_order ? 1 : 0);
-    attn_ws_items(b->seq_len.data(), ns, D.Hkv, v_items_kv.back(), g_attn_order ? 2 : 0);
+    attn_ws_items(b->seq_len.data(), ns, D.H, v_items.back(), g_attn_order ? 1 : 0, s->num_sms);
+    attn_ws_items(b->seq_len.data(), ns, D.Hkv, v_items_kv.back(), g_attn_order ? 2 : 0, s->num_sms);
     v_items_seq.emplace_back();
     attn_seq_items(b->seq_len.data(), ns, D.Hkv, v_items_seq.back());
-    attn_ws_items(b->seq_len.data(), ns, D.H, v_items_q.back(), g_attn_order ? 1 : 0);
+    attn_ws_items(b->seq_len.data(), ns, D.H, v_items_q.back(), g_attn_order ? 1 : 0, s->num_sms);
     v.n_items = (int)v_items.back().size();
     v.n_items_kv = (int)v_items_kv.back().size();
     v.n_items_seq = (int)v_items_seq.back().size();
     v_ds.emplace_back();
     if (b->ds_tiles > 0) {
-      v.ds_ok = attn_ds_plan(b->seq_len.data(), ns, D.H, D.Hkv, b->ds_tiles, v_ds.back());
+      v.ds_ok = attn_ds_plan(b->seq_len.data(), ns, D.H, D.Hkv, b->ds_tiles, v_ds.back(), s->num_sms);
       if (v.ds_ok) v.ds_chunks = v_ds.back().chunks;
     }
     b->views.push_back(v);
@@ -1460,9 +1460,9 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
     b->pc_rows = 0;
     for (auto& pc : pcs) b->pc_rows += pc.n;
     std::vector<int4> xi, xikv, xiq, xiseq;
-    attn_ws_items(xl.data(), b->n_seqs, D.H, xi, g_attn_order ? 1 : 0);
-    attn_ws_items(xl.data(), b->n_seqs, D.Hkv, xikv, g_attn_order ? 2 : 0);
-    attn_ws_items(xl.data(), b->n_seqs, D.H, xiq, g_attn_order ? 1 : 0);
+    attn_ws_items(xl.data(), b->n_seqs, D.H, xi, g_attn_order ? 1 : 0, s->num_sms);
+    attn_ws_items(xl.data(), b->n_seqs, D.Hkv, xikv, g_attn_order ? 2 : 0, s->num_sms);
+    attn_ws_items(xl.data(), b->n_seqs, D.H, xiq, g_attn_order ? 1 : 0, s->num_sms);
     attn_seq_items(xl.data(), b->n_seqs, D.Hkv, xiseq);
     menos_batch::AttnView& xv = b->xview;
     xv.n_seqs = b->n_seqs; xv.n_blocks = (int)xb64.size(); xv.n_blocks128 = (int)xb128.size(); xv.pairs = b->pairs_ext;

@@ -62,6 +62,13 @@ extern "C" int menos_test_gemm(int M, int N, int K, int b_mn, const void* A, int
   return MENOS_OK;
 }
 
+static int sms_of_device() {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return sms;
+}
+
 extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, int Hkv, int hd, const void* qkv,
                                     void* O, float* lse, const void* dO, void* dqkv, float theta) {
   std::vector<int> cu(1, 0);
@@ -96,7 +103,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
   cudaMemcpy(d_b128, b128.data(), b128.size() * sizeof(int2), cudaMemcpyHostToDevice);
   const bool ws_fwd = (hd == 128 || hd == 64) && (g_attn_tc & 4);
   std::vector<int4> items;
-  attn_ws_items(seq_len, n_seqs, H, items, g_attn_order ? 1 : 0);
+  attn_ws_items(seq_len, n_seqs, H, items, g_attn_order ? 1 : 0, sms_of_device());
   int4* d_items;
   cudaMalloc(&d_items, std::max<size_t>(1, items.size()) * sizeof(int4));
   cudaMemcpy(d_items, items.data(), items.size() * sizeof(int4), cudaMemcpyHostToDevice);
@@ -110,7 +117,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
     a.dO = (const bf16*)dO; a.ld_do = H * hd; a.D = d_D; a.dqkv = (bf16*)dqkv; a.ld_dqkv = Nqkv;
     a.rope_cs = theta > 0.f ? d_cs : nullptr;   // theta <= 0: no RoPE backward (OPT)
     std::vector<int4> items_kv;
-    attn_ws_items(seq_len, n_seqs, Hkv, items_kv, g_attn_order ? 2 : 0);
+    attn_ws_items(seq_len, n_seqs, Hkv, items_kv, g_attn_order ? 2 : 0, sms_of_device());
     int4* d_items_kv;
     cudaMalloc(&d_items_kv, std::max<size_t>(1, items_kv.size()) * sizeof(int4));
     cudaMemcpy(d_items_kv, items_kv.data(), items_kv.size() * sizeof(int4), cudaMemcpyHostToDevice);
@@ -129,7 +136,7 @@ extern "C" int menos_test_attention(int n_seqs, const int32_t* seq_len, int H, i
     // bit 6: the dS-stored backward, chunked under g_attn_ds_cap_tiles exactly as the server runs it
     AttnDsPlan plan;
     const bool ds_bwd = ws_bwd && !fused_bwd && (g_attn_tc & 64) &&
-                        attn_ds_plan(seq_len, n_seqs, H, Hkv, g_attn_ds_cap_tiles, plan);
+                        attn_ds_plan(seq_len, n_seqs, H, Hkv, g_attn_ds_cap_tiles, plan, sms_of_device());
     if (ds_bwd) {
       const long long cap = std::min(g_attn_ds_cap_tiles, attn_ds_total_tiles(seq_len, n_seqs, H));
       bf16* d_ds; int* d_base; int4 *d_ikv, *d_iq;
