@@ -34,6 +34,13 @@ template <int HD> struct FwdGeo {
 constexpr float LOG2E = 1.4426950408889634f;
 constexpr float RESCALE_THRESHOLD = 8.0f;            // log2 units
 constexpr int NTHREADS = 256;
+// MENOS_FWS_TMEM_P (default 1): the softmax threads write P as packed bf16 into the TMEM columns of the S tile they
+// have just read and the PV MMA takes it as the A operand from TMEM ("ts" tcgen05.mma), as in the backward: no
+// shared-memory P tile, no proxy fence.  The S buffer is only reissued after the PV that reads its P (the MMA warp
+// issues PV(j) before S(j + 2), and the tensor pipe runs a thread's MMAs in order).  0: P through shared memory.
+#ifndef MENOS_FWS_TMEM_P
+#define MENOS_FWS_TMEM_P 1
+#endif
 
 // -DMENOS_WS_PROF: per-phase clock64 accounting of one softmax thread and the MMA lane (tuning aid only)
 #ifdef MENOS_WS_PROF
@@ -188,9 +195,14 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           const uint32_t pa = smem_u32(sP + b * P_BYTES), vb = smem_u32(sV + s * K_BYTES);
 #pragma unroll
           for (int kk = 0; kk < BKV / 16; ++kk) {
-            const uint64_t ad = umma_desc_sw128(pa + kk * 32, 16, 1024);
             const uint64_t bd = umma_desc_sw128(vb + kk * 2048, KA_BYTES, 1024);
+#if MENOS_FWS_TMEM_P
+            (void)pa;   // A = P packed in S[b]'s first 32 columns: 8 columns (16 keys) per K step
+            tc_mma_bf16_ts(tO, tS0 + b * 64 + kk * 8, bd, IDESC_PV, (j > 0 || kk > 0) ? 1u : 0u);
+#else
+            const uint64_t ad = umma_desc_sw128(pa + kk * 32, 16, 1024);
             tc_mma_bf16(tO, ad, bd, IDESC_PV, (j > 0 || kk > 0) ? 1u : 0u);
+#endif
           }
           tc_commit(&pv_done[b]);
           tc_commit(&v_empty[s]);
@@ -293,11 +305,16 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           }
         }
         WSP(2);
+#if !MENOS_FWS_TMEM_P
         // P[b] was last read by the PV of block sc-2
         if (sc >= 2) wait_spin(&pv_done[b], ((sc - 2) >> 1) & 1);
+#endif
         WSP(4);
         uint8_t* prow = sP + b * P_BYTES + row * 128;
         float sum = 0.f;
+#if MENOS_FWS_TMEM_P
+        uint32_t pw[32];
+#endif
 #pragma unroll
         for (int c8 = 0; c8 < 8; ++c8) {
           float e[8];
@@ -310,11 +327,27 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
           }
           const uint4 u = make_uint4(pack_bf16x2(e[0], e[1]), pack_bf16x2(e[2], e[3]), pack_bf16x2(e[4], e[5]),
                                      pack_bf16x2(e[6], e[7]));
+#if MENOS_FWS_TMEM_P
+          pw[4 * c8] = u.x; pw[4 * c8 + 1] = u.y; pw[4 * c8 + 2] = u.z; pw[4 * c8 + 3] = u.w;
+#else
           *reinterpret_cast<uint4*>(prow + ((c8 ^ (row & 7)) << 4)) = u;
+#endif
         }
         l += sum;
         WSP(5);
+#if MENOS_FWS_TMEM_P
+        {
+          uint32_t lo[16], hi[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) { lo[i] = pw[i]; hi[i] = pw[16 + i]; }
+          tmem_st16_nw(tS0 + b * 64 + lane_off, lo);
+          tmem_st16_nw(tS0 + b * 64 + 16 + lane_off, hi);
+          tmem_wait_st();
+        }
+        (void)prow;
+#else
         fence_proxy_async();                        // generic smem writes -> async proxy (tensor core)
+#endif
         tc_fence_before();
         mbar_arrive(&p_full[b]);
         WSP(6);
@@ -379,7 +412,18 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
 bool tma_map_2d(CUtensorMap* out, const void* ptr, uint64_t rows, uint64_t cols, uint64_t ld, uint32_t bc,
                 uint32_t br);
 
-void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order) {
+void attn_snake_waves(std::vector<int4>& v, size_t first, int grid) {
+  if (grid <= 1) return;
+  const size_t n = v.size() - first, G = (size_t)grid;
+  if (n <= G) return;   // one wave: the launch grid is n, nothing to balance
+  for (size_t w = 1; w * G < n; w += 2) {
+    const size_t a = first + w * G, b = first + std::min(n, (w + 1) * G);
+    if (b - a == G) std::reverse(v.begin() + a, v.begin() + b);   // a partial last wave stays as it is (the kernels
+                                                                   // take no placeholder items)
+  }
+}
+
+void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out, int order, int grid) {
   // (sequence, head) groups, q blocks of a group adjacent and largest first: the group's K/V stays in L2
   const size_t first = out.size();
   for (int i = 0; i < n_seqs; ++i)
@@ -394,6 +438,7 @@ void attn_ws_items(const int* seq_len, int n_seqs, int H, std::vector<int4>& out
     return order == 1 ? std::min(L, it.y + BQ) : L - it.y;
   };
   std::stable_sort(out.begin() + first, out.end(), [&](const int4& a, const int4& b) { return cost(a) > cost(b); });
+  attn_snake_waves(out, first, grid);
 }
 
 // (sequence, kv head) items of the one-pass backward, LPT: longest sequence first (stable)
