@@ -50,6 +50,12 @@ constexpr float LOG2E_W = 1.4426950408889634f;
 #if MENOS_BWS_ALT
 static_assert(MENOS_BWS_TMEM_P && EW_WARPS == 8, "MENOS_BWS_ALT needs the TMEM operand path and 8 elementwise warps");
 #endif
+// MENOS_BWS_DV_DIRECT (tuning variant, default 0; ALT path): the dK/dV epilogue sends dK out by TMA store and writes
+// dV straight from registers instead of staging it after the dK store's read -- measured slower (cfg1 214 -> 230 us,
+// cfg3 2.34 -> 2.46 ms per layer, r2bs): 16-byte stores of 32 rows per warp instruction cost more than the wait
+#ifndef MENOS_BWS_DV_DIRECT
+#define MENOS_BWS_DV_DIRECT 0
+#endif
 // TMEM column (relative to the tile) of K-chunk kk (16 queries / keys) of a packed operand: thread group g wrote its
 // CPT columns' values into the first CPT / 2 of the CPT columns it had read (columns [CPT g, CPT g + CPT / 2))
 __device__ __forceinline__ uint32_t packed_col(int kk) {
@@ -596,6 +602,23 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
       BP(7);
       if (full) fence_proxy_async();
       ew_sync();
+#if MENOS_BWS_DV_DIRECT
+      if (full) {   // dK leaves by TMA store; dV straight from registers (no second staging round, no wait between)
+        if (t == 0) {
+          stage_tma_store<HD>(&tmOut, sP0, base + k0, (p.H + G.head) * HD);
+          bulk_commit();
+        }
+        tma_pending = true;
+        constexpr int EC = HD / (2 * NGRP);
+        bf16* vrow = dst + (size_t)r * p.ld_dqkv + (p.H + p.Hkv + G.head) * HD + EC * gr;
+#pragma unroll
+        for (int c = 0; c < EC / 8; ++c) {
+          *reinterpret_cast<uint4*>(vrow + 8 * c) = vpk.x[c];
+          *reinterpret_cast<uint4*>(vrow + HD / 2 + 8 * c) = vpk.y[c];
+        }
+      } else
+#endif
+      {
       if (full) {
         if (t == 0) {
           stage_tma_store<HD>(&tmOut, sP0, base + k0, (p.H + G.head) * HD);
@@ -620,7 +643,8 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         stage16_store<HD>(sP0, 1, w8, lane, nv, dst + (p.H + p.Hkv + G.head) * HD, dst, p.ld_dqkv);
         ew_sync();
       }
-      if (p.ds) {   // the next item's dS^T staging reuses sP0: the dV store must have read it
+      }
+      if (p.ds) {   // the next item's dS^T staging reuses sP0: the dK / dV store must have read it
         if (t == 0 && tma_pending) { bulk_wait_read0(); tma_pending = false; }
         ew_sync();
       }
