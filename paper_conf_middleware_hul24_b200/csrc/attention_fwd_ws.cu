@@ -110,28 +110,35 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
   // TMEM columns: S[0] 0..63, S[1] 64..127, O[0] 128..128+HD, O[1] 256..256+HD
   const uint32_t tS0 = tmem, tO0 = tmem + 128;
 
-  // work-item geometry; every role loads the NEXT item's geometry at the top of the current one (two dependent
-  // global loads whose latency then hides behind the current item)
-  struct Geo { int base, L, q0, h, nkv; };
-  auto load_geo = [&](int item) {
-    Geo g{0, 0, 0, 0, 0};
-    if (item < p.n_items) {
-      const int4 it = p.items[item];
-      g.base = p.cu_seqlens[it.x]; g.L = p.cu_seqlens[it.x + 1] - g.base; g.q0 = it.y; g.h = it.z;
-      g.nkv = (min(g.L, g.q0 + BQ) + BKV - 1) / BKV;
-    }
+  // work-item geometry, two items deep so that no role stalls on a dependent load at an item boundary: at the top
+  // of item i the items entry of i + 2G is loaded and the cu_seqlens entries of i + G (whose items entry arrived an
+  // item earlier) are fetched; i + G's values are consumed one item later
+  struct GeoPipe { int4 far, nxt; int c0, c1; };
+  auto fetch = [&](GeoPipe& g) {
+    g.c0 = 0; g.c1 = 0;
+    if (g.nxt.x >= 0) { g.c0 = p.cu_seqlens[g.nxt.x]; g.c1 = p.cu_seqlens[g.nxt.x + 1]; }
+  };
+  auto entry = [&](int item) { return item < p.n_items ? p.items[item] : make_int4(-1, 0, 0, 0); };
+  auto pipe_init = [&]() {
+    GeoPipe g;
+    g.nxt = entry(blockIdx.x);
+    fetch(g);
+    g.far = entry(blockIdx.x + gridDim.x);
     return g;
   };
-  auto item_geom = [&](Geo& nxt, int item, int& base, int& L, int& q0, int& h, int& nkv) {
-    base = nxt.base; L = nxt.L; q0 = nxt.q0; h = nxt.h; nkv = nxt.nkv;
-    nxt = load_geo(item + gridDim.x);
+  auto item_geom = [&](GeoPipe& g, int item, int& base, int& L, int& q0, int& h, int& nkv) {
+    base = g.c0; L = g.c1 - g.c0; q0 = g.nxt.y; h = g.nxt.z;
+    nkv = g.nxt.x >= 0 ? (min(L, q0 + BQ) + BKV - 1) / BKV : 0;
+    g.nxt = g.far;
+    fetch(g);
+    g.far = entry(item + 2 * gridDim.x);
   };
 
   if (warp == 0 || warp == 2) {
     // ============================================================ TMA producers (warp 0: Q, K; warp 2: V)
     if (elect_one()) {
       int it = 0, kc = 0;
-      Geo nxt = load_geo(blockIdx.x);
+      GeoPipe nxt = pipe_init();
       for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
         int base, L, q0, h, nkv;
         item_geom(nxt, item, base, L, q0, h, nkv);
@@ -170,7 +177,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
     // ============================================================ MMA issuer
     constexpr uint32_t IDESC_S = umma_idesc_bf16(BQ, BKV, 0);
     constexpr uint32_t IDESC_PV = umma_idesc_bf16(BQ, HD, 1);
-    Geo nxt = load_geo(blockIdx.x);
+    GeoPipe nxt = pipe_init();
     WSP_DECL
     int it = 0, kvc = 0, sc = 0;   // kvc: global 64-key block counter (K and V rings), sc: S / P buffer counter
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
@@ -244,7 +251,7 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
     const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
     const float sl2 = p.scale * LOG2E;
     int it = 0, sc = 0;
-    Geo nxt = load_geo(blockIdx.x);
+    GeoPipe nxt = pipe_init();
     WSP_DECL
     for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
       int base, L, q0, h, nkv;
