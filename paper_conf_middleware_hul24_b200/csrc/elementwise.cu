@@ -246,6 +246,36 @@ __global__ void adamw_kernel(const AdamSeg* __restrict__ segs, const int4* __res
   const int4 w = work[blockIdx.x];
   const AdamSeg sg = segs[w.x];
   const AdamHyper hp = hyp[sg.client];
+  // 4 elements per thread with 16-byte loads / stores when the block, its row length and the bf16 copy allow it
+  // (the same fp32 operations per element as the scalar loop below: results are bitwise identical)
+  const bool vec = (sg.p_off & 3) == 0 && (sg.cols & 3) == 0 && (w.y & 3) == 0 && (w.z & 3) == 0 &&
+                   (sg.dst_ld & 3) == 0 && (reinterpret_cast<uintptr_t>(sg.dst) & 7) == 0;
+  if (vec) {
+    for (int e = w.y + 4 * threadIdx.x; e < w.y + w.z; e += 4 * blockDim.x) {
+      const long long i = sg.p_off + e;
+      float4 p = *reinterpret_cast<const float4*>(hp.p + i);
+      if (hp.do_update) {
+        const float4 g = *reinterpret_cast<const float4*>(hp.g + i);
+        float4 m = *reinterpret_cast<const float4*>(hp.m + i), v = *reinterpret_cast<const float4*>(hp.v + i);
+        float* pp = &p.x; const float* gg = &g.x; float* mm = &m.x; float* vv = &v.x;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          pp[k] = pp[k] * hp.decay;
+          mm[k] = hp.beta1 * mm[k] + hp.omb1 * gg[k];
+          vv[k] = hp.beta2 * vv[k] + hp.omb2 * (gg[k] * gg[k]);
+          const float denom = sqrtf(vv[k]) / hp.bc2_sqrt + hp.eps;
+          pp[k] = pp[k] - hp.step_size * (mm[k] / denom);
+        }
+        *reinterpret_cast<float4*>(hp.p + i) = p; *reinterpret_cast<float4*>(hp.m + i) = m;
+        *reinterpret_cast<float4*>(hp.v + i) = v; *reinterpret_cast<float4*>(hp.g + i) = make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+      const int rr = e / sg.cols, cc = e % sg.cols;   // the 4 elements share a row (cols % 4 == 0)
+      const size_t drow = !sg.is_b ? (size_t)rr
+                                   : (size_t)(sg.row_base + (rr / sg.row_blk) * sg.row_blk_stride + rr % sg.row_blk);
+      *reinterpret_cast<uint2*>(sg.dst + drow * sg.dst_ld + cc) = make_uint2(pack_bf16x2(p.x, p.y), pack_bf16x2(p.z, p.w));
+    }
+    return;
+  }
   for (int e = w.y + threadIdx.x; e < w.y + w.z; e += blockDim.x) {
     const long long i = sg.p_off + e;
     float p = hp.p[i];
