@@ -1,5 +1,6 @@
 // Kernel-level test entry points (include/menos_testing.h): same kernels as the server path.
 #include <algorithm>
+#include <cstdlib>
 #include <cmath>
 #include <cstring>
 #include <string>
@@ -261,7 +262,11 @@ extern "C" int menos_test_gemm_time(int M, int N, int K, int b_mn, const void* A
 // g_attn_ds_cap_tiles, 16 KB tiles).
 // Default 78: the persistent tcgen05 forward and the dS-stored persistent backward (LPT work order, bit 4 selects
 // (sequence, head) order).
-namespace menos { int g_attn_tc = 78; int g_attn_order = 1; long long g_attn_ds_cap_tiles = 32768; }
+namespace menos {
+int g_attn_tc = 78; int g_attn_order = 1;
+// MENOS_DS_CAP_TILES: tuning override of the dS-stored backward's chunk budget (16 KB tiles; default 32768 = 512 MB)
+long long g_attn_ds_cap_tiles = [] { const char* e = getenv("MENOS_DS_CAP_TILES"); return e ? atoll(e) : 32768LL; }();
+}
 extern "C" int menos_test_abf_prof(unsigned long long* out16) {
   if (!out16) return fail("null output");
   return menos::attn_bwd_fused_prof(out16);
