@@ -431,12 +431,12 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         if (elect_one()) {
           const uint32_t ob = smem_u32(sO0 + sp * QB_TILE), qb = smem_u32(sQ0 + sp * QB_TILE);
 #if MENOS_BWS_TMEM_P
+          const uint64_t od0 = umma_desc_sw128(ob, 8192, 1024), qd0 = umma_desc_sw128(qb, 8192, 1024);
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk) {   // A = P^T / dS^T packed in the S^T / dP^T tiles of buffer bp
-            const uint32_t acc = (jp > 0 || kk > 0) ? 1u : 0u;
-            tc_mma_bf16_ts(tdV, tmem + 64 * bp + packed_col(kk), umma_desc_sw128(ob + kk * 2048, 8192, 1024), ID_ACC, acc);
-            tc_mma_bf16_ts(tdK, tmem + 128 + 64 * bp + packed_col(kk), umma_desc_sw128(qb + kk * 2048, 8192, 1024), ID_ACC,
-                           acc);
+            const uint32_t acc = (jp > 0 || kk > 0) ? 1u : 0u;   // B: base descriptor + constant K-step offset
+            tc_mma_bf16_ts(tdV, tmem + 64 * bp + packed_col(kk), od0 + (uint64_t)((kk * 2048) >> 4), ID_ACC, acc);
+            tc_mma_bf16_ts(tdK, tmem + 128 + 64 * bp + packed_col(kk), qd0 + (uint64_t)((kk * 2048) >> 4), ID_ACC, acc);
           }
           tc_commit(&empty[sp]);     // Q/dO stage free
 #else
@@ -466,13 +466,16 @@ attn_bwd_dkdv_ws_kernel(const __grid_constant__ CUtensorMap tmQKV128, const __gr
         tc_fence_after();
         __syncwarp();
         if (elect_one()) {
-          const uint32_t k = smem_u32(sK), v = smem_u32(sV);
-          const uint32_t q = smem_u32(sQ0 + st * QB_TILE), o = smem_u32(sO0 + st * QB_TILE);
+          // one base descriptor per operand, K steps as constant 16-byte-unit offsets (no carry: smem < 256 KB)
+          const uint64_t kd0 = umma_desc_sw128(smem_u32(sK), 16, 1024), vd0 = umma_desc_sw128(smem_u32(sV), 16, 1024);
+          const uint64_t qd0 = umma_desc_sw128(smem_u32(sQ0 + st * QB_TILE), 16, 1024);
+          const uint64_t od0 = umma_desc_sw128(smem_u32(sO0 + st * QB_TILE), 16, 1024);
 #pragma unroll
           for (int kk = 0; kk < HD / 16; ++kk) {
-            const uint32_t offa = (kk >> 2) * KVA + (kk & 3) * 32, offb = (kk >> 2) * QBA + (kk & 3) * 32;
-            tc_mma_bf16(tmem + 64 * b, umma_desc_sw128(k + offa, 16, 1024), umma_desc_sw128(q + offb, 16, 1024), ID_S, kk > 0);
-            tc_mma_bf16(tmem + 128 + 64 * b, umma_desc_sw128(v + offa, 16, 1024), umma_desc_sw128(o + offb, 16, 1024), ID_S, kk > 0);
+            const uint64_t offa = (uint64_t)(((kk >> 2) * KVA + (kk & 3) * 32) >> 4);
+            const uint64_t offb = (uint64_t)(((kk >> 2) * QBA + (kk & 3) * 32) >> 4);
+            tc_mma_bf16(tmem + 64 * b, kd0 + offa, qd0 + offb, ID_S, kk > 0);
+            tc_mma_bf16(tmem + 128 + 64 * b, vd0 + offa, od0 + offb, ID_S, kk > 0);
           }
           tc_commit(&s_full[b]);
           if (j == G.n - 1) tc_commit(&kv_empty);   // K / V free once the item's last S^T / dP^T completes
@@ -1257,10 +1260,11 @@ attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_con
         __syncwarp();
         if (elect_one()) {
           const uint32_t sd = smem_u32(sStage + st * Gm::STAGE), sk = sd + Gm::DS2;
+          const uint64_t dd0 = umma_desc_sw128(sd, 16384, 1024), kd0 = umma_desc_sw128(sk, 16384, 1024);
 #pragma unroll
           for (int kk = 0; kk < KV_ROWS / 16; ++kk)   // 16 keys = 2048 B of both the dS^T pair and the K block
-            tc_mma_bf16(tmem + buf * HD, umma_desc_sw128(sd + kk * 2048, 16384, 1024),
-                        umma_desc_sw128(sk + kk * 2048, 16384, 1024), ID_DQ, (kb > 0 || kk > 0) ? 1u : 0u);
+            tc_mma_bf16(tmem + buf * HD, dd0 + (uint64_t)((kk * 2048) >> 4), kd0 + (uint64_t)((kk * 2048) >> 4), ID_DQ,
+                        (kb > 0 || kk > 0) ? 1u : 0u);
           tc_commit(&empty[st]);
         }
         __syncwarp();

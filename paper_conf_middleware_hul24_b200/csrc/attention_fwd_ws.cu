@@ -200,9 +200,10 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
         tc_fence_after();
         if (elect_one()) {
           const uint32_t pa = smem_u32(sP + b * P_BYTES), vb = smem_u32(sV + s * K_BYTES);
+          const uint64_t vd0 = umma_desc_sw128(vb, KA_BYTES, 1024);
 #pragma unroll
           for (int kk = 0; kk < BKV / 16; ++kk) {
-            const uint64_t bd = umma_desc_sw128(vb + kk * 2048, KA_BYTES, 1024);
+            const uint64_t bd = vd0 + (uint64_t)((kk * 2048) >> 4);
 #if MENOS_FWS_TMEM_P
             (void)pa;   // A = P packed in S[b]'s first 32 columns: 8 columns (16 keys) per K step
             tc_mma_bf16_ts(tO, tS0 + b * 64 + kk * 8, bd, IDESC_PV, (j > 0 || kk > 0) ? 1u : 0u);
@@ -225,11 +226,14 @@ attn_fwd_ws_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constan
         WSP(11);
         tc_fence_after();
         if (elect_one()) {
-          const uint32_t ka = smem_u32(sK + s * K_BYTES);
+          // descriptors: one base per operand, the K steps as constant 16-byte-unit offsets (the start-address field
+          // cannot carry: shared memory is < 256 KB)
+          const uint64_t ad0 = umma_desc_sw128(qa, 16, 1024);
+          const uint64_t bd0 = umma_desc_sw128(smem_u32(sK + s * K_BYTES), 16, 1024);
 #pragma unroll
           for (int kk = 0; kk < HD / 16; ++kk) {
-            const uint64_t ad = umma_desc_sw128(qa + (kk >> 2) * QA_BYTES + (kk & 3) * 32, 16, 1024);
-            const uint64_t bd = umma_desc_sw128(ka + (kk >> 2) * KA_BYTES + (kk & 3) * 32, 16, 1024);
+            const uint64_t ad = ad0 + (uint64_t)(((kk >> 2) * QA_BYTES + (kk & 3) * 32) >> 4);
+            const uint64_t bd = bd0 + (uint64_t)(((kk >> 2) * KA_BYTES + (kk & 3) * 32) >> 4);
             tc_mma_bf16(tS0 + b * 64, ad, bd, IDESC_S, kk > 0 ? 1u : 0u);
           }
           tc_commit(&s_full[b]);
