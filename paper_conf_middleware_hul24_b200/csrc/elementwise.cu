@@ -327,6 +327,13 @@ __global__ void bf16_to_f32_kernel(const bf16* __restrict__ s, float* __restrict
 // WPR warps per row (1 for d <= 1024, 2 above: d = 2048 at one warp per row held 215 registers in the backward,
 // one CTA per SM); the row sums go warp_sum -> shared slots of the row's warps (fixed order), the same helper in
 // fwd and bwd so the backward's recomputed mu / rstd equal the forward's bit for bit.
+// the row's WPR warps synchronise on their own named barrier (1 + the row's index in the CTA), not the whole CTA:
+// the rows of a CTA do not wait for each other (same summation order as before: results unchanged)
+template <int WPR>
+__device__ __forceinline__ void ln_row_bar() {
+  const int id = 1 + (int)(threadIdx.x >> 5) / WPR;
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "n"(32 * WPR) : "memory");
+}
 template <int WPR>
 __device__ __forceinline__ float ln_row_sum(float v, float* red) {
   v = warp_sum(v);
@@ -335,12 +342,28 @@ __device__ __forceinline__ float ln_row_sum(float v, float* red) {
   } else {
     const int w = threadIdx.x >> 5, base = (w / WPR) * WPR;
     if ((threadIdx.x & 31) == 0) red[w] = v;
-    __syncthreads();
+    ln_row_bar<WPR>();
     float s = red[base];
 #pragma unroll
     for (int k = 1; k < WPR; ++k) s += red[base + k];
-    __syncthreads();   // red is reused by the next reduction
+    ln_row_bar<WPR>();   // red is reused by the next reduction
     return s;
+  }
+}
+// two row sums in one exchange (the backward's mean(gh) and mean(gh * xh)); each in the order ln_row_sum uses
+template <int WPR>
+__device__ __forceinline__ void ln_row_sum2(float& a, float& b, float2* red2) {
+  a = warp_sum(a);
+  b = warp_sum(b);
+  if constexpr (WPR > 1) {
+    const int w = threadIdx.x >> 5, base = (w / WPR) * WPR;
+    if ((threadIdx.x & 31) == 0) red2[w] = make_float2(a, b);
+    ln_row_bar<WPR>();
+    float2 s = red2[base];
+#pragma unroll
+    for (int k = 1; k < WPR; ++k) { s.x += red2[base + k].x; s.y += red2[base + k].y; }
+    ln_row_bar<WPR>();
+    a = s.x; b = s.y;
   }
 }
 
@@ -401,6 +424,7 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(const TDY* __restric
                                                             const float* __restrict__ resid, float* __restrict__ dx,
                                                             bf16* __restrict__ dxb, int T, int d, float eps) {
   __shared__ float red[8];
+  __shared__ float2 red2[8];
   const int row = blockIdx.x * (8 / WPR) + threadIdx.x / (32 * WPR), tr = threadIdx.x % (32 * WPR);
   const bool ok = row < T;
   const size_t ro = (size_t)(ok ? row : 0) * d;
@@ -433,7 +457,8 @@ __global__ void __launch_bounds__(256) layernorm_bwd_kernel(const TDY* __restric
     if ((c * 32 * WPR + tr) * 8 < d)
 #pragma unroll
       for (int k = 0; k < 8; ++k) { sg += gh[c][k]; sgx += gh[c][k] * (v[c][k] - mu) * r; }
-  const float mg = ln_row_sum<WPR>(sg, red) / (float)d, mgx = ln_row_sum<WPR>(sgx, red) / (float)d;
+  ln_row_sum2<WPR>(sg, sgx, red2);
+  const float mg = sg / (float)d, mgx = sgx / (float)d;
   if (!ok) return;
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
