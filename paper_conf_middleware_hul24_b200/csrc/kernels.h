@@ -112,8 +112,9 @@ constexpr int LORA_DUB_MT = 128;
 int lora_dub_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, int max_rank, cudaStream_t st);
 // tcgen05 variant (rank <= 16): the same contract; dY [y_rows, ldy] and U [y_rows, ldu] are the whole buffers the
 // problems index with (t0, ycol0) / (t0, ucol0); 128-token stages by TMA, dB and the per-stage dU share on tcgen05
+// mts: dY columns per CTA (128, or 256: half the partials; the problems' n_slabs must use the same width)
 int lora_dub_tc_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, const bf16* dY, int y_rows, int ldy,
-                    const bf16* U, int ldu, cudaStream_t st);
+                    const bf16* U, int ldu, int mts, cudaStream_t st);
 // grid: (ceil(max T * rs / 256), n_probs)
 int lora_du_reduce_run(const LoraDUBProblem* d_probs, int n_probs, long long max_elems, cudaStream_t st);
 

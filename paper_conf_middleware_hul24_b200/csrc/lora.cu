@@ -544,12 +544,17 @@ lora_shrink_tc_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_cons
 // over all stages; each stage's dU share lands in one of two TMEM buffers and is written out as fp32 partial rows
 // while the next stage runs.  Rows past the client's tokens and columns past the target's are zeroed in the
 // transposed operands, so they contribute nothing.
+// MTS = dY columns per CTA (slab): 128, or 256 for large grids (half the fp32 dU partials to write and sum; two
+// M = 128 dB accumulators)
 constexpr int DUBT_BK = 128, DUBT_ST = 2;
-constexpr int DUBT_Y = 128 * 128 * 2;            // dY stage: two [128 rows][64 cols] atoms
 constexpr int DUBT_U = 128 * 16 * 2;             // U stage, linear [128][16]
-constexpr int DUBT_T = 16 * 128 * 2;             // transposed [16][128] K-major tile (two [16][64] atoms)
-constexpr int DUBT_STAGE = DUBT_Y + DUBT_U + DUBT_T;
-constexpr int DUBT_SMEM = DUBT_ST * DUBT_STAGE + DUBT_T + 1024;
+constexpr int DUBT_UT = 16 * 128 * 2;            // U^T: [16][128 tokens] K-major (two [16][64] atoms)
+template <int MTS> struct DubtGeo {
+  static constexpr int Y = 128 * MTS * 2;        // dY stage: MTS / 64 atoms of [128 rows][64 cols]
+  static constexpr int BT = 16 * MTS * 2;        // B_slab^T: [16][MTS] K-major (MTS / 64 atoms of [16][64])
+  static constexpr int STAGE = Y + DUBT_U + DUBT_UT;
+  static constexpr int SMEM = DUBT_ST * STAGE + BT + 1024;
+};
 
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
@@ -577,9 +582,13 @@ __device__ __forceinline__ uint32_t kt_off(int n, int k) {
   return (uint32_t)((k >> 6) * 2048 + n * 128 + ((((k & 63) >> 3) ^ (n & 7)) << 4) + (k & 7) * 2);
 }
 
-__global__ void __launch_bounds__(192, 2)
+template <int MTS>
+__global__ void __launch_bounds__(192, MTS == 128 ? 2 : 1)
 lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmU,
                    const LoraDUBProblem* __restrict__ probs) {
+  using Gd = DubtGeo<MTS>;
+  constexpr int NH = MTS / 128;                  // dB accumulators (M = 128 each)
+  constexpr int DUBT_Y = Gd::Y, DUBT_STAGE = Gd::STAGE;
   extern __shared__ uint8_t dubt_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(dubt_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* const sBT = smem + DUBT_ST * DUBT_STAGE;
@@ -589,8 +598,9 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
   const LoraDUBProblem P = probs[blockIdx.y];
   const int slab = blockIdx.x;
   if (slab >= P.n_slabs) return;
-  const int m0 = slab * 128, nst = (P.T + DUBT_BK - 1) / DUBT_BK;
-  const int pcol0 = (m0 / P.p_blk) * P.p_blk_stride + m0 % P.p_blk;
+  const int m0 = slab * MTS, nst = (P.T + DUBT_BK - 1) / DUBT_BK;
+  auto pcol = [&](int m) { return (m / P.p_blk) * P.p_blk_stride + m % P.p_blk; };   // per 64-column atom
+  const int pcol0 = pcol(m0);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     tma_prefetch(&tmY); tma_prefetch(&tmU);
@@ -604,7 +614,7 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = tmem_sh;   // dB at column 0, dU buffers at 16 / 32
+  const uint32_t tmem = tmem_sh;   // dB halves at columns 0 (/ 16), dU buffers after them
   if (warp == 0) {
     if (elect_one()) {
       for (int s = 0; s < nst; ++s) {
@@ -613,8 +623,8 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
         mbar_expect_tx(&full[st], DUBT_Y + DUBT_U);
         uint8_t* sy = smem + st * DUBT_STAGE;
         const int row = P.t0 + s * DUBT_BK;
-        tma_load_2d(sy, &tmY, &full[st], P.ycol0 + pcol0, row);
-        tma_load_2d(sy + 16384, &tmY, &full[st], P.ycol0 + pcol0 + 64, row);
+#pragma unroll
+        for (int a = 0; a < MTS / 64; ++a) tma_load_2d(sy + a * 16384, &tmY, &full[st], P.ycol0 + pcol(m0 + 64 * a), row);
         tma_load_2d(sy + DUBT_Y, &tmU, &full[st], P.ucol0, row);
       }
     }
@@ -633,13 +643,15 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
       if (elect_one()) {
         const uint32_t sy = smem_u32(smem + st * DUBT_STAGE), sut = sy + DUBT_Y + DUBT_U, sbt = smem_u32(sBT);
 #pragma unroll
-        for (int kk = 0; kk < DUBT_BK / 16; ++kk)   // dB: K = 16 tokens = 16 rows of both dY atoms, of U^T
-          tc_mma_bf16(tmem, umma_desc_sw128(sy + kk * 2048, 16384, 1024),
-                      umma_desc_sw128(sut + (kk >> 2) * 2048 + (kk & 3) * 32, 16, 1024), ID_DB,
-                      (s > 0 || kk > 0) ? 1u : 0u);
+        for (int h = 0; h < NH; ++h)                 // dB half h: slab columns 128 h .. 128 h + 127 (atoms 2h, 2h+1)
 #pragma unroll
-        for (int kk = 0; kk < 128 / 16; ++kk)       // dU share: K = 16 slab columns
-          tc_mma_bf16(tmem + 16 + 16 * b, umma_desc_sw128(sy + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
+          for (int kk = 0; kk < DUBT_BK / 16; ++kk)   // K = 16 tokens = 16 rows of the dY atoms, of U^T
+            tc_mma_bf16(tmem + 16 * h, umma_desc_sw128(sy + h * 32768 + kk * 2048, 16384, 1024),
+                        umma_desc_sw128(sut + (kk >> 2) * 2048 + (kk & 3) * 32, 16, 1024), ID_DB,
+                        (s > 0 || kk > 0) ? 1u : 0u);
+#pragma unroll
+        for (int kk = 0; kk < MTS / 16; ++kk)       // dU share: K = 16 slab columns
+          tc_mma_bf16(tmem + 16 * NH + 16 * b, umma_desc_sw128(sy + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
                       umma_desc_sw128(sbt + (kk >> 2) * 2048 + (kk & 3) * 32, 16, 1024), ID_DU, kk > 0 ? 1u : 0u);
         tc_commit(&empty[st]);
         tc_commit(&du_full[b]);
@@ -650,16 +662,21 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
   } else {
     const int q = warp & 3, row = q * 32 + lane;   // TMEM lane quadrant; row = token (dU) / slab column (dB)
     const uint32_t loff = (uint32_t)(q * 32) << 16;
-    {   // B_slab^T [16][128]: row n = rank column n, k = slab column; zero past the target's columns / the rank
-      const bool ok = m0 + row < P.Nt;
-      const uint4* src = reinterpret_cast<const uint4*>(P.B + (size_t)(pcol0 + row) * P.ldb);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {   // B_slab^T [16][MTS]: row n = rank column n, k = slab column; zero past the
+                                     // target's columns / the rank
+      const int k = 128 * h + row;
+      const bool ok = m0 + k < P.Nt;
+      const uint4* src = reinterpret_cast<const uint4*>(P.B + (size_t)(ok ? pcol(m0 + k) : 0) * P.ldb);
       uint4 v0 = ok ? src[0] : make_uint4(0, 0, 0, 0), v1 = ok ? src[1] : make_uint4(0, 0, 0, 0);
       const bf16* e0 = reinterpret_cast<const bf16*>(&v0);
       const bf16* e1 = reinterpret_cast<const bf16*>(&v1);
       const bf16 z = __float2bfloat16_rn(0.f);
 #pragma unroll
       for (int n = 0; n < 16; ++n)
-        *reinterpret_cast<bf16*>(sBT + kt_off(n, row)) = n < P.rank ? (n < 8 ? e0[n] : e1[n - 8]) : z;
+        *reinterpret_cast<bf16*>(sBT + kt_off(n, k)) = n < P.rank ? (n < 8 ? e0[n] : e1[n - 8]) : z;
+    }
+    {
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(&bt_ready);
@@ -670,7 +687,7 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
       mbar_wait(&du_full[b], (s >> 1) & 1);
       tc_fence_after();
       uint32_t r[16];
-      tmem_ld16(tmem + 16 + 16 * b + loff, r);
+      tmem_ld16(tmem + 16 * NH + 16 * b + loff, r);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&du_free[b]);
@@ -701,9 +718,13 @@ lora_dub_tc_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constan
     if (nst > 0) du_out(nst - 1);
     mbar_wait(&db_full, 0);
     tc_fence_after();
-    uint32_t r[16];
-    tmem_ld16(tmem + loff, r);
-    if (m0 + row < P.Nt) store_row16(P.dB + (size_t)(m0 + row) * P.rank, r, P.rank);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      uint32_t r[16];
+      tmem_ld16(tmem + 16 * h + loff, r);
+      const int m = m0 + 128 * h + row;
+      if (m < P.Nt) store_row16(P.dB + (size_t)m * P.rank, r, P.rank);
+    }
   }
   tc_fence_before();
   __syncthreads();
@@ -966,18 +987,20 @@ int lora_da_tc_run(const LoraTokRedProblem* d_probs, int n_probs, int max_n, int
 }
 
 int lora_dub_tc_run(const LoraDUBProblem* d_probs, int n_probs, int max_slabs, const bf16* dY, int y_rows, int ldy,
-                    const bf16* U, int ldu, cudaStream_t st) {
+                    const bf16* U, int ldu, int mts, cudaStream_t st) {
   if (n_probs <= 0 || max_slabs <= 0) return 0;
-  if (ldy % 8 || ldu % 8) return -1;
+  if (ldy % 8 || ldu % 8 || (mts != 128 && mts != 256)) return -1;
   CUtensorMap mY, mU;
   if (!tma_map_2d(&mY, dY, y_rows, ldy, ldy, 64, 128)) return -2;
   if (!tma_map_2d_plain(&mU, U, y_rows, ldu, ldu, 16, 128)) return -2;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(lora_dub_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, DUBT_SMEM);
+    cudaFuncSetAttribute(lora_dub_tc_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, DubtGeo<128>::SMEM);
+    cudaFuncSetAttribute(lora_dub_tc_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, DubtGeo<256>::SMEM);
     attr = true;
   }
-  lora_dub_tc_kernel<<<dim3(max_slabs, n_probs), 192, DUBT_SMEM, st>>>(mY, mU, d_probs);
+  if (mts == 256) lora_dub_tc_kernel<256><<<dim3(max_slabs, n_probs), 192, DubtGeo<256>::SMEM, st>>>(mY, mU, d_probs);
+  else lora_dub_tc_kernel<128><<<dim3(max_slabs, n_probs), 192, DubtGeo<128>::SMEM, st>>>(mY, mU, d_probs);
   ++g_launch_count;
   return cudaPeekAtLastError() == cudaSuccess ? 0 : -3;
 }

@@ -283,7 +283,8 @@ struct SGList {
   int probs_off = 0, n_probs = 0, tiles_off = 0, n_tiles = 0, max_n = 0; double flops = 0;
   int max_rank = 0; long long max_elems = 0;   // fused dU+dB lists: widest rank, largest T * rs
   int tile_n = 0;                              // token-reduction lists: tile width
-  int n_small = 0;                             // fused dU+dB lists: problems [0, n_small) have rank <= 16
+  int n_small = 0;                             // fused dU+dB lists: problems [0, n_small) have rank <= 16 (tcgen05),
+  int n_wide = 0;                              // of which [0, n_wide) use 256-column slabs
 };
 
 struct menos_batch {
@@ -1286,6 +1287,18 @@ static size_t slab_bytes_of(const Dims& D, int Ls, int T, const int R_used[NG], 
   return per_layer * Ls;
 }
 // arena bytes of the per-call scratch block (see get_scratch)
+// slab width of a fused dU + dB problem (see finalize_batch); MENOS_LORA_DUB_MT=128 forces 128 (A/B), and
+// MENOS_LORA_DUB_MMA=1 puts every problem on the mma.sync kernel (128)
+static bool dub_env_mma() {
+  static const bool v = [] { const char* e = getenv("MENOS_LORA_DUB_MMA"); return e && atoi(e) == 1; }();
+  return v;
+}
+static int dub_mts(const LoraDUBProblem& q) {
+  static const int force = [] { const char* e = getenv("MENOS_LORA_DUB_MT"); return e ? atoi(e) : 0; }();
+  if (dub_env_mma() || q.rank > 16 || force == 128) return 128;
+  return q.Nt >= 8192 ? 256 : 128;
+}
+
 // fused dU + dB partials of one group's problems: sum over clients and targets of ceil(N_t/128) * T_c * rank * 4 B,
 // bounded per token by (max over the group's targets of ceil(N_t/128)) * (slot span R_used[g]) * 4 B
 static size_t wsp_bytes_of(const Dims& D, int T, const int R_used[NG]) {
@@ -1584,10 +1597,12 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
           q.B = s->Bcat[g][l] + (size_t)D.rb_base[t] * s->cols[g].cap + c.col_off[g] + c.sub[t];
           q.ldb = s->cols[g].cap;
           q.dB = c.G() + c.offB[l * NT + t];
-          q.W = sc.wsp + woff;
           q.dU = sc.dU[g] + (size_t)t0 * R + c.col_off[g] + c.sub[t]; q.lddu = R;
           q.Nt = D.N_t[t]; q.rank = c.rank; q.rs = c.rs; q.T = Tc; q.scale = c.s;
-          q.n_slabs = (q.Nt + LORA_DUB_MT - 1) / LORA_DUB_MT;
+          // slab width from the target's own shape and rank (never from the batch: bitwise batched == alone):
+          // 256 columns for the wide targets (N_t >= 8192: half the fp32 dU partials), 128 otherwise / on mma.sync
+          q.n_slabs = (q.Nt + dub_mts(q) - 1) / dub_mts(q);
+          q.W = sc.wsp + woff;
           q.t0 = t0; q.ycol0 = D.rb_base[t]; q.ucol0 = c.col_off[g] + c.sub[t];
           if (q.p_blk % LORA_DUB_MT) FAIL(MENOS_EINVAL, "LoRA row block %d not a multiple of %d", q.p_blk, LORA_DUB_MT);
           woff += (size_t)q.n_slabs * Tc * c.rank;
@@ -1627,10 +1642,11 @@ static int finalize_batch(menos_server* s, menos_batch* b, Scratch& sc, const La
       // rank <= 16 first (tcgen05 kernel), larger ranks after (mma.sync kernel): the kernel a client's problem
       // takes depends on its own rank only, never on who shares the batch
       std::stable_partition(dub.begin(), dub.end(), [](const LoraDUBProblem& q) { return q.rank <= 16; });
+      std::stable_partition(dub.begin(), dub.end(), [](const LoraDUBProblem& q) { return dub_mts(q) == 256; });
       {
         SGList& Ld = b->sg_dub[li];
         Ld = SGList();
-        for (const auto& q : dub) Ld.n_small += q.rank <= 16;
+        for (const auto& q : dub) { Ld.n_small += q.rank <= 16 && !dub_env_mma(); Ld.n_wide += dub_mts(q) == 256; }
         Ld.probs_off = (int)dprobs.size(); Ld.n_probs = (int)dub.size();
         for (const auto& q : dub) {
           Ld.flops += 4.0 * q.Nt * q.rank * q.T;
@@ -1794,15 +1810,17 @@ static int run_rows(menos_batch* b, const SGList& L, cudaStream_t st) {
 // fused dU + dB (one pass over each target's dY), then the fixed-order slab sum into the bf16 dU slot columns
 // (tcgen05 for rank <= 16; MENOS_LORA_DUB_MMA=1 or larger ranks: the mma.sync kernel)
 static int run_dub(menos_batch* b, size_t li, cudaStream_t st) {
-  static const bool mma = [] { const char* e = getenv("MENOS_LORA_DUB_MMA"); return e && atoi(e) == 1; }();
   const SGList& L = b->sg_dub[li];
   if (L.n_probs == 0) return 0;
   ProfScope ps(PC_LORA, L.flops, 0, st);
   const menos_batch::DubBufs& Bf = b->dub_bufs[li];
-  const int n_tc = mma ? 0 : L.n_small;
-  int rc = lora_dub_tc_run(b->d_dprobs + L.probs_off, n_tc, L.max_n, Bf.Y, Bf.rows, Bf.ldy, Bf.U, Bf.ldu, st);
-  if (!rc && L.n_probs > n_tc)
-    rc = lora_dub_run(b->d_dprobs + L.probs_off + n_tc, L.n_probs - n_tc, L.max_n, L.max_rank, st);
+  // [0, n_wide): tcgen05 with 256-column slabs; [n_wide, n_small): tcgen05, 128; the rest: mma.sync, 128
+  int rc = lora_dub_tc_run(b->d_dprobs + L.probs_off, L.n_wide, L.max_n, Bf.Y, Bf.rows, Bf.ldy, Bf.U, Bf.ldu, 256, st);
+  if (!rc)
+    rc = lora_dub_tc_run(b->d_dprobs + L.probs_off + L.n_wide, L.n_small - L.n_wide, L.max_n, Bf.Y, Bf.rows, Bf.ldy, Bf.U,
+                         Bf.ldu, 128, st);
+  if (!rc && L.n_probs > L.n_small)
+    rc = lora_dub_run(b->d_dprobs + L.probs_off + L.n_small, L.n_probs - L.n_small, L.max_n, L.max_rank, st);
   if (rc) return rc;
   return lora_du_reduce_run(b->d_dprobs + L.probs_off, L.n_probs, L.max_elems, st);
 }
