@@ -384,14 +384,18 @@ def run_gpu(args):
         if world > 1:
             dist.barrier()
 
+    host_ms = [0.0]
+
     def timed(fn, K):
         barrier()
         torch.cuda.synchronize(device)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
+        h0 = time.perf_counter()
         for _ in range(K):
             fn()
         e1.record(stream)
+        host_ms[0] = (time.perf_counter() - h0) * 1e3   # host time to enqueue the K steps (diagnostic)
         torch.cuda.synchronize(device)
         barrier()
         ms = e0.elapsed_time(e1)
@@ -406,10 +410,12 @@ def run_gpu(args):
     torch.cuda.synchronize(device)
 
     clocks = ClockSampler(device.index)
-    clocks.start()
-    time.sleep(0.3)
+    if os.environ.get("MENOS_BENCH_CLOCKS", "1") != "0":   # =0: diagnostic runs without the nvidia-smi sampler
+        clocks.start()
+        time.sleep(0.3)
     l0 = M.launch_count()
     ms = timed(lambda: step(x_c, x_s, g_c, g_s), args.steps)
+    host_enqueue_ms = host_ms[0] / args.steps
     launches = M.launch_count() - l0
     clk = clocks.stop()
     ms_per_step = ms / args.steps
@@ -532,7 +538,8 @@ def run_gpu(args):
                              f"streamed per step vs 126 MB L2"},
             "roofline": roofline, "step_tflops": step_tflops,
             "step_frac_of_peak": step_tflops / (peak * n_dev) if peak else None,
-            "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm}
+            "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm,
+            "host_enqueue_ms_per_step": host_enqueue_ms}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
             line["cpu_baseline"] = oracle_sample(512)
