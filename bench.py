@@ -421,6 +421,25 @@ def run_gpu(args):
     ms_per_step = ms / args.steps
     value = T_all * args.steps / (ms / 1000.0)
 
+    # host work of one step with the GPU idle before every call (no ring-slot / event waits): what the library's
+    # host side costs per step when it cannot hide behind the previous call's kernels
+    host_calls = {"forward": 0.0, "backward": 0.0, "adapter_step": 0.0}
+    torch.cuda.synchronize(device)
+    for sc_, sl_, a, b_ in wave_args:
+        h0 = time.perf_counter()
+        b = srv.forward(sc_, sl_, x_c[a:b_], x_s[a:b_], stream=stream)
+        host_calls["forward"] += time.perf_counter() - h0
+        torch.cuda.synchronize(device)
+        h0 = time.perf_counter()
+        srv.backward(b, g_c[a:b_], g_s[a:b_], stream=stream)
+        host_calls["backward"] += time.perf_counter() - h0
+        torch.cuda.synchronize(device)
+    h0 = time.perf_counter()
+    srv.adapter_step(ids, stream=stream)
+    host_calls["adapter_step"] += time.perf_counter() - h0
+    torch.cuda.synchronize(device)
+    host_calls = {k: v * 1e3 for k, v in host_calls.items()}
+
     # per-kernel CUDA events (recorded by the library on the launching stream around every launch) over a
     # second timed region of the same K steps; kept out of the headline region because an event pair around
     # every cluster launch adds inter-kernel gaps
@@ -539,7 +558,7 @@ def run_gpu(args):
             "roofline": roofline, "step_tflops": step_tflops,
             "step_frac_of_peak": step_tflops / (peak * n_dev) if peak else None,
             "kernels": kernels, "gpu_launches": launches, "clocks": clk, "e2e": e2e, "hbm_bytes_per_client": hbm,
-            "host_enqueue_ms_per_step": host_enqueue_ms}
+            "host_enqueue_ms_per_step": host_enqueue_ms, "host_ms_per_call_gpu_idle": host_calls}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
             line["cpu_baseline"] = oracle_sample(512)

@@ -1,5 +1,6 @@
 """The fused LoRA dU + dB backward (`lora_dub_tc_kernel`) takes 256-column slabs for targets with
-N_t >= 8192 and 128-column slabs otherwise; ranks > 16 take the mma.sync kernel.  The tiny recipe never reaches the
+N_t >= 8192 and 128-column slabs otherwise (ranks <= 16; larger ranks take the mma.sync kernel,
+`test_gpu_parity.py::test_tiny_ranks_above_16`).  The tiny recipe never reaches the
 wide case (N_t <= 344), so these tests widen the MLP of the tiny model to d_ff = 8200 (gate / up: N_t = 8200 =
 32 slabs of 256 + an 8-column tail; PAPER.md:294's LoRA on the projections, Alg. 1 L10-12 for the gradients) and
 check (a) parity with the oracle and (b) that a client's results do not depend on who shares its batch."""
@@ -18,7 +19,7 @@ torch = pytest.importorskip("torch")
 def _w():
     m = dataclasses.replace(MODELS["tiny"], d_ff=8200, n_layers=2, model_layers=3)
     cl = [ClientCfg(4, 8.0, ("gate", "up"), [37, 90]), ClientCfg(16, 32.0, TARGETS, [130]),
-          ClientCfg(32, 64.0, ("up", "down"), [65]), ClientCfg(8, 16.0, ("q", "gate"), [3, 128])]
+          ClientCfg(6, 12.0, ("up", "down"), [65]), ClientCfg(8, 16.0, ("q", "gate"), [3, 128])]
     return Workload("wide_mlp", m, cl)
 
 
