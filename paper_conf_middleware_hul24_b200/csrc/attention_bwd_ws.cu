@@ -1226,6 +1226,7 @@ attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_con
     if (elect_one()) {
       int gb = 0;
       for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
+        if (p.items[item].x < 0) continue;   // padding (attn_ds_plan): a CTA's tail
         int base, L, q0, h, seq;
         geo(item, base, L, q0, h, seq);
         const int hk = h / rep;
@@ -1247,8 +1248,9 @@ attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_con
     __syncwarp();
   } else if (warp == 1) {
     constexpr uint32_t ID_DQ = umma_idesc_bf16(128, HD, 1) | (1u << 15);   // A (dS) and B (K) MN-major
-    int gb = 0, it = 0;
-    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+    int gb = 0, it = 0;   // it counts real items only (accumulator buffer and phase)
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
+      if (p.items[item].x < 0) continue;
       const int q0 = p.items[item].y;
       const int buf = it & 1;
       wait_bar(&acc_free[buf], ((it >> 1) & 1) ^ 1);
@@ -1271,22 +1273,26 @@ attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_con
       }
       if (elect_one()) tc_commit(&acc_full[buf]);
       __syncwarp();
+      ++it;
     }
   } else {
     const int w4 = warp & 3, w8 = warp - 2, g = w8 >> 2, t = threadIdx.x - 64;
     const int r = w4 * 32 + lane;   // query row = TMEM lane
     const uint32_t lane_off = (uint32_t)(w4 * 32) << 16;
     bool tma_pending = false;
-    int it = 0;
-    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x, ++it) {
+    int it = 0, prev_seq = -1, prev_q0 = -1;
+    RopeCS<HD> csq;   // kept across a run of items at the same (sequence, query block): loaded once per run
+    for (int item = blockIdx.x; item < p.n_items; item += gridDim.x) {
+      if (p.items[item].x < 0) continue;
       int base, L, q0, h, seq;
       geo(item, base, L, q0, h, seq);
       const int sh = p.pos_shift ? p.pos_shift[seq] : 0;
       const int buf = it & 1;
       const int nv = min(Q_ROWS, L - q0);
       const bool rope = p.rope_cs != nullptr && r < nv;
-      RopeCS<HD> csq;
-      rope_cs_load<HD>(csq, p.rope_cs, max(0, q0 + r - sh), g, rope);   // in flight during the wait below
+      if (seq != prev_seq || q0 != prev_q0)
+        rope_cs_load<HD>(csq, p.rope_cs, max(0, q0 + r - sh), g, rope);   // in flight during the wait below
+      prev_seq = seq; prev_q0 = q0;
       wait_bar(&acc_full[buf], (it >> 1) & 1);
       tc_fence_after();
       if (t == 0 && tma_pending) bulk_wait_read0();   // the previous item's TMA store has read the staging
@@ -1310,6 +1316,7 @@ attn_bwd_dq_ds_kernel(const __grid_constant__ CUtensorMap tmDS, const __grid_con
         stage16_store<HD>(sStg, 1, w8, lane, nv, dq, dq, p.ld_dqkv);
         ew_sync();
       }
+      ++it;
     }
     if (t == 0) bulk_wait0();
   }
@@ -1434,8 +1441,45 @@ bool attn_ds_plan(const int* seq_len, int n_seqs, int H, int Hkv, long long cap_
       const int L = seq_len[u.x];
       for (int k = 0; k < L; k += 128) out.items_kv.push_back(make_int4(u.x, k, u.y, 0));
       const int nq = (L + 127) / 128;
-      for (int h = u.y * rep; h < (u.y + 1) * rep; ++h, ++grp)
-        for (int j = 0; j < nq; ++j) out.items_q.push_back(make_int4(u.x, (nq - 1 - (j + grp) % nq) * 128, h, 0));
+      if (grid <= 0)
+        for (int h = u.y * rep; h < (u.y + 1) * rep; ++h, ++grp)
+          for (int j = 0; j < nq; ++j) out.items_q.push_back(make_int4(u.x, (nq - 1 - (j + grp) % nq) * 128, h, 0));
+    }
+    if (grid > 0) {
+      // dQ items for a persistent grid of `grid` CTAs (CTA c takes list entries c, c + grid, ...): each CTA gets a
+      // RUN of items with the same (sequence, query block) over consecutive heads, so its epilogue loads the RoPE
+      // rows once per run instead of once per item (r2cj: the RoPE-table loads bound the dQ pass).  Natural order
+      // (sequence, query block, head) split into `grid` contiguous ranges of equal cost (kv blocks per item), then
+      // interleaved; CTAs with shorter ranges are padded with (-1, ...) entries at their tail (the kernel stops there).
+      std::vector<int4> nat;
+      std::vector<int> cost;
+      for (size_t i = 0; i < units.size(); ++i) {
+        const int sq = units[i].x;
+        if (i > 0 && units[i - 1].x == sq) continue;   // units of one sequence are adjacent
+        const int nq = (seq_len[sq] + 127) / 128;
+        for (int j = nq - 1; j >= 0; --j)
+          for (size_t k = i; k < units.size() && units[k].x == sq; ++k)
+            for (int h = units[k].y * rep; h < (units[k].y + 1) * rep; ++h) {
+              nat.push_back(make_int4(sq, j * 128, h, 0));
+              cost.push_back(j + 1);
+            }
+      }
+      long long total = 0;
+      for (int c : cost) total += c;
+      std::vector<int> lo(grid + 1, (int)nat.size());
+      lo[0] = 0;
+      long long acc = 0;
+      int c = 1;
+      for (size_t i = 0; i < nat.size() && c < grid; ++i) {
+        while (c < grid && acc >= total * c / grid) lo[c++] = (int)i;
+        acc += cost[i];
+      }
+      int mx = 0;
+      for (int k = 0; k < grid; ++k) mx = std::max(mx, lo[k + 1] - lo[k]);
+      const size_t at = out.items_q.size();
+      out.items_q.resize(at + (size_t)mx * grid, make_int4(-1, 0, 0, 0));
+      for (int k = 0; k < grid; ++k)
+        for (int t = 0; t < lo[k + 1] - lo[k]; ++t) out.items_q[at + (size_t)t * grid + k] = nat[lo[k] + t];
     }
     // dK/dV: LPT for the persistent grid's static round-robin (largest = most query blocks after the key block)
     std::stable_sort(out.items_kv.begin() + kv0, out.items_kv.end(), [&](const int4& a, const int4& b) {
