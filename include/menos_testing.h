@@ -80,6 +80,15 @@ MENOS_API int menos_test_set_ds_cap(long long tiles);
    head, base[seq * Hkv + kv head] = the unit's first tile in its chunk, chunks[4c..4c+3] = (kv item offset, count,
    q item offset, count) for c < min(*n_chunks, max_chunks); *n_chunks = -1 when a unit alone exceeds `cap` (the
    recompute path).  Any output pointer but n_chunks may be NULL. */
+/* Host-only (no GPU): the dS-stored backward's dQ item list for a persistent grid of `grid` CTAs (CTA c takes entries
+   c, c + grid, ...): items[4i..4i+3] = (sequence, first query row, head, 0), sequence -1 = padding at a CTA's tail;
+   each CTA's items form runs of one (sequence, query block) over consecutive heads (the epilogue loads the RoPE rows
+   once per run).  *n_items = list length (copied up to max_items), chunks as menos_test_ds_plan (*n_chunks = -1:
+   no plan).  items / chunks may be NULL. */
+MENOS_API int menos_test_ds_plan_q(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int grid,
+                                   int32_t* items, int max_items, int32_t* n_items, int32_t* chunks, int max_chunks,
+                                   int32_t* n_chunks);
+
 MENOS_API int menos_test_ds_plan(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int32_t* tiles,
                                  int32_t* base, int32_t* chunks, int max_chunks, int32_t* n_chunks,
                                  int32_t* n_items_kv, int32_t* n_items_q);

@@ -287,6 +287,29 @@ extern "C" int menos_test_set_ds_cap(long long tiles) {
   return MENOS_OK;
 }
 
+// Host-only: the dS-stored backward's dQ item list for a persistent grid of `grid` CTAs (attn_ds_plan with grid > 0):
+// items[4 i .. 4 i + 3] = (sequence, q0, head, 0), or sequence -1 for padding; chunks as menos_test_ds_plan.
+extern "C" int menos_test_ds_plan_q(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int grid,
+                                    int32_t* items, int max_items, int32_t* n_items, int32_t* chunks, int max_chunks,
+                                    int32_t* n_chunks) {
+  if (n_seqs < 0 || !seq_len || H <= 0 || Hkv <= 0 || H % Hkv || grid <= 0 || !n_items || !n_chunks)
+    return fail("bad arguments");
+  menos::AttnDsPlan plan;
+  std::vector<int> lens(seq_len, seq_len + n_seqs);
+  if (!menos::attn_ds_plan(lens.data(), n_seqs, H, Hkv, cap, plan, grid)) { *n_chunks = -1; return MENOS_OK; }
+  *n_items = (int)plan.items_q.size();
+  *n_chunks = (int)plan.chunks.size();
+  for (int i = 0; i < (int)plan.items_q.size() && i < max_items && items; ++i) {
+    items[4 * i] = plan.items_q[i].x; items[4 * i + 1] = plan.items_q[i].y;
+    items[4 * i + 2] = plan.items_q[i].z; items[4 * i + 3] = plan.items_q[i].w;
+  }
+  for (int c = 0; c < (int)plan.chunks.size() && c < max_chunks && chunks; ++c) {
+    chunks[4 * c] = plan.chunks[c].x; chunks[4 * c + 1] = plan.chunks[c].y;
+    chunks[4 * c + 2] = plan.chunks[c].z; chunks[4 * c + 3] = plan.chunks[c].w;
+  }
+  return MENOS_OK;
+}
+
 // Host plan of the dS-stored attention backward (no GPU needed): per-sequence tile counts, unit bases and chunks.
 // tiles[i] = attn_ds_tiles(seq_len[i]); base[seq * Hkv + hk]; chunks[c] = (kv item offset, count, q offset, count).
 extern "C" int menos_test_ds_plan(int n_seqs, const int32_t* seq_len, int H, int Hkv, long long cap, int32_t* tiles,

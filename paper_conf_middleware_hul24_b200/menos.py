@@ -113,6 +113,7 @@ SIGNATURES = {
     "menos_test_set_attn_tc": (_I, [_I]),
     "menos_test_set_ds_cap": (_I, [C.c_longlong]),
     "menos_test_ds_plan": (_I, [_I, _PI32, _I, _I, C.c_longlong, _PI32, _PI32, _PI32, _I, _PI32, _PI32, _PI32]),
+    "menos_test_ds_plan_q": (_I, [_I, _PI32, _I, _I, C.c_longlong, _I, _PI32, _I, _PI32, _PI32, _I, _PI32]),
     "menos_test_abf_prof": (_I, [C.POINTER(C.c_ulonglong)]),
     "menos_testing_last_error": (C.c_char_p, []),
     "menos_sched_create": (_I, [_S, _I, C.POINTER(_P)]),

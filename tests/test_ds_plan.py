@@ -85,3 +85,53 @@ def test_plan_invariants(lib, seed):
             assert nc == 1
     # a unit larger than the budget: no plan (the recompute path)
     assert plan(lib, lens, H, Hkv, max(unit) - 1)[3] == -1
+
+
+def plan_q(lib, lens, H, Hkv, cap, grid):
+    n = len(lens)
+    arr = (C.c_int32 * n)(*lens)
+    n_items, nc = C.c_int32(), C.c_int32()
+    assert lib.menos_test_ds_plan_q(n, arr, H, Hkv, cap, grid, None, 0, C.byref(n_items), None, 0, C.byref(nc)) == 0
+    items = (C.c_int32 * (4 * max(1, n_items.value)))()
+    chunks = (C.c_int32 * (4 * max(1, nc.value)))()
+    assert lib.menos_test_ds_plan_q(n, arr, H, Hkv, cap, grid, items, n_items.value, C.byref(n_items), chunks,
+                                    nc.value, C.byref(nc)) == 0
+    it = np.array(items[:4 * n_items.value], dtype=np.int64).reshape(-1, 4)
+    return it, [tuple(chunks[4 * c:4 * c + 4]) for c in range(nc.value)]
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_dq_runs_plan(lib, seed):
+    """The dQ list for a persistent grid (r2ck): per chunk, every (sequence, query block, head) exactly once; CTA c
+    (entries c, c + grid, ...) holds its real items before its padding; the items of a CTA come in runs of one
+    (sequence, query block); the CTAs' costs (kv blocks per item = query block + 1) differ by at most one item's."""
+    rng = np.random.default_rng(seed)
+    H, Hkv = [(32, 32), (8, 2), (6, 1)][seed]
+    rep = H // Hkv
+    lens = [int(x) for x in rng.integers(1, 1100, size=int(rng.integers(1, 20)))]
+    grid = [148, 7, 64][seed]
+    unit = [rep * brute_tiles(L) for L in lens for _ in range(Hkv)]
+    for cap in (max(unit) + 3, 10 ** 9):
+        items, chunks = plan_q(lib, lens, H, Hkv, cap, grid)
+        seen = set()
+        for (_, _, q_off, q_n) in chunks:
+            assert q_n % grid == 0
+            ch = items[q_off:q_off + q_n]
+            real = [tuple(x[:3]) for x in ch if x[0] >= 0]
+            assert len(real) == len(set(real))
+            seen |= set(real)
+            costs = []
+            for c in range(grid):
+                col = ch[c::grid]
+                flags = col[:, 0] >= 0
+                k = int(flags.sum())
+                assert flags[:k].all() and not flags[k:].any()      # padding only at the tail
+                col = col[:k]
+                runs = 1 + int(np.sum((col[1:, 0] != col[:-1, 0]) | (col[1:, 1] != col[:-1, 1]))) if k else 0
+                fams = len({(int(a), int(b)) for a, b in col[:, :2]})
+                assert runs == fams                                  # one run per (sequence, query block)
+                costs.append(int(np.sum(col[:, 1] // 128 + 1)) if k else 0)
+            mx = max(int(x[1]) // 128 + 1 for x in ch if x[0] >= 0)
+            assert max(costs) - min(costs) <= 2 * mx
+        want = {(s, q, h) for s, L in enumerate(lens) for q in range(0, L, 128) for h in range(H)}
+        assert seen == want
